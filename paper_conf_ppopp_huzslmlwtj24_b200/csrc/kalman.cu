@@ -1,0 +1,614 @@
+// Blocked FEKF Kalman update (Algorithm 1 lines 8-13; RLEKF blocks P:L123).
+//
+// Storage: every block P_i (n_i x n_i, fp64) is padded to a multiple of T = 64 and stored as its
+// upper-triangle tiles (diagonal tiles full), each tile 64x64 row-major and contiguous (32 KiB).
+// Symmetrisation (Alg. 1 line 11) is therefore exact by construction.
+//
+// One update streams the local P exactly once (kf_pass_kernel):
+//   P_IJ <- (P_IJ - A' u'_I u'_J^T) / lambda'      (pending rank-1 of the previous update, line 10)
+//   u_I  += P_IJ g_J ;  u_J += P_IJ^T g_I          (Pg, cached for A, K and the next pass: P:L283)
+// Tiles are moved HBM <-> SMEM with 1-D TMA bulk copies (cp.async.bulk + mbarrier), a producer warp
+// keeps up to STAGES tiles in flight, 8 consumer warps update in SMEM and a bulk store writes back.
+// Partial u's go to a workspace slot per (item row) / (tile column) and are summed in a fixed order
+// (kf_reduce_u) — no floating-point atomics, bit-reproducible.
+// Then A = 1/(c + g^T u) with c = L*lambda (reading Z1) or lambda, w += sqrt(bs)*ABE*A*u, and the
+// update (A, u, lambda) becomes the pending correction of the next pass.
+#include <algorithm>
+#include <cmath>
+#include <numeric>
+
+#include "kalman.cuh"
+
+namespace fekf {
+
+// ------------------------------------------------------------------------------------------------
+// host planner
+// ------------------------------------------------------------------------------------------------
+void KfPlan::build(const std::vector<int>& blocks, int world_, int rank_, int seg_tiles) {
+  n = blocks;
+  L = (int)n.size();
+  world = world_;
+  rank = rank_;
+  nt.resize(L);
+  off.resize(L + 1);
+  tc_off.resize(L + 1);
+  off[0] = 0;
+  tc_off[0] = 0;
+  for (int i = 0; i < L; ++i) {
+    nt[i] = (n[i] + KT - 1) / KT;
+    off[i + 1] = off[i] + n[i];
+    tc_off[i + 1] = tc_off[i] + nt[i];
+  }
+  N = off[L];
+  n_tc = tc_off[L];
+  Npad = n_tc * KT;
+  tc_blk.resize(n_tc);
+  tc_c.resize(n_tc);
+  for (int i = 0; i < L; ++i)
+    for (int c = 0; c < nt[i]; ++c) {
+      tc_blk[tc_off[i] + c] = i;
+      tc_c[tc_off[i] + c] = c;
+    }
+  // all items (tile-row segments) in canonical order
+  struct It { int blk, I, J0, nJ; };
+  std::vector<It> all;
+  for (int i = 0; i < L; ++i)
+    for (int I = 0; I < nt[i]; ++I)
+      for (int J0 = I; J0 < nt[i]; J0 += seg_tiles) all.push_back({i, I, J0, std::min(seg_tiles, nt[i] - J0)});
+  total_tiles = 0;
+  for (auto& it : all) total_tiles += it.nJ;
+  // LPT over ranks by tile count (largest first, ties -> canonical order, lowest rank)
+  std::vector<int> order(all.size());
+  std::iota(order.begin(), order.end(), 0);
+  std::stable_sort(order.begin(), order.end(), [&](int a, int b) { return all[a].nJ > all[b].nJ; });
+  std::vector<int64_t> load(world, 0);
+  owner.assign(all.size(), 0);
+  for (int k : order) {
+    int r = (int)(std::min_element(load.begin(), load.end()) - load.begin());
+    owner[k] = r;
+    load[r] += all[k].nJ;
+  }
+  // this rank's items, largest first (dynamic scheduling on the device picks them in this order)
+  items.clear();
+  int64_t tile_off = 0;
+  for (int k : order) {
+    if (owner[k] != rank) continue;
+    ItemD d;
+    d.blk = all[k].blk; d.I = all[k].I; d.J0 = all[k].J0; d.nJ = all[k].nJ;
+    d.tile_off = tile_off;
+    d.vbase = (long long)tc_off[d.blk] * KT;
+    tile_off += d.nJ;
+    items.push_back(d);
+  }
+  tiles_local = tile_off;
+  const int64_t n_items = (int64_t)items.size();
+  for (int64_t k = 0; k < n_items; ++k) {
+    items[k].row_slot = (int)k;
+    items[k].col_slot0 = (long long)(n_items + items[k].tile_off);
+  }
+  ws_slots = n_items + tiles_local;
+  // per-tile owner in canonical packed order (for fekf_plan_shard)
+  tile_owner.clear();
+  tile_owner.reserve(total_tiles);
+  for (size_t k = 0; k < all.size(); ++k)
+    for (int t = 0; t < all[k].nJ; ++t) tile_owner.push_back(owner[k]);
+  // CSR of workspace slots per tile column: row partials of strip c (by J0), then column partials
+  // of tiles (I < c, c) (by I).  Fixed order => deterministic sums.
+  std::vector<std::vector<std::pair<long long, long long>>> rows(n_tc), cols(n_tc);
+  for (int64_t k = 0; k < n_items; ++k) {
+    const ItemD& d = items[k];
+    rows[tc_off[d.blk] + d.I].push_back({d.J0, d.row_slot});
+    for (int t = 0; t < d.nJ; ++t) {
+      int J = d.J0 + t;
+      if (J == d.I) continue;
+      cols[tc_off[d.blk] + J].push_back({d.I, d.col_slot0 + t});
+    }
+  }
+  csr_ptr.assign(n_tc + 1, 0);
+  csr_idx.clear();
+  for (int64_t tc = 0; tc < n_tc; ++tc) {
+    std::sort(rows[tc].begin(), rows[tc].end());
+    std::sort(cols[tc].begin(), cols[tc].end());
+    for (auto& e : rows[tc]) csr_idx.push_back(e.second);
+    for (auto& e : cols[tc]) csr_idx.push_back(e.second);
+    csr_ptr[tc + 1] = (long long)csr_idx.size();
+  }
+}
+
+// ------------------------------------------------------------------------------------------------
+// PTX helpers (mbarrier + 1-D TMA bulk copies)
+// ------------------------------------------------------------------------------------------------
+__device__ __forceinline__ uint32_t smem_u32(const void* p) {
+  return (uint32_t)__cvta_generic_to_shared(p);
+}
+__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count));
+}
+__device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive_tx(uint64_t* bar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes)
+               : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+  uint32_t addr = smem_u32(bar);
+  asm volatile(
+      "{\n"
+      ".reg .pred p;\n"
+      "WAIT_%=:\n"
+      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
+      "@!p bra WAIT_%=;\n"
+      "}\n" ::"r"(addr),
+      "r"(parity)
+      : "memory");
+}
+__device__ __forceinline__ void tma_load_1d(void* dst_smem, const void* src_gmem, uint32_t bytes, uint64_t* bar) {
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+          smem_u32(dst_smem)),
+      "l"(src_gmem), "r"(bytes), "r"(smem_u32(bar))
+      : "memory");
+}
+__device__ __forceinline__ void tma_store_1d(void* dst_gmem, const void* src_smem, uint32_t bytes) {
+  asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(dst_gmem),
+               "r"(smem_u32(src_smem)), "r"(bytes)
+               : "memory");
+}
+__device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.commit_group;" ::: "memory"); }
+template <int N>
+__device__ __forceinline__ void bulk_wait_read() {
+  asm volatile("cp.async.bulk.wait_group.read %0;" ::"n"(N) : "memory");
+}
+__device__ __forceinline__ void bulk_wait_all() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
+__device__ __forceinline__ void fence_proxy_async() {
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+}
+__device__ __forceinline__ void fence_mbar_init() {
+  asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+}
+__device__ __forceinline__ void consumer_bar() { asm volatile("bar.sync 1, 256;" ::: "memory"); }
+
+// ------------------------------------------------------------------------------------------------
+// the P pass
+// ------------------------------------------------------------------------------------------------
+constexpr int STAGES = 6;
+constexpr int TILE_ELEMS = KT * KT;
+constexpr uint32_t TILE_BYTES = TILE_ELEMS * sizeof(double);
+constexpr int PASS_THREADS = 288;  // 8 consumer warps + 1 producer warp
+constexpr size_t PASS_SMEM = STAGES * TILE_BYTES + 2 * 8 * KT * sizeof(double) +
+                             2 * STAGES * sizeof(uint64_t) + STAGES * sizeof(int4);
+
+__global__ void __launch_bounds__(PASS_THREADS, 1)
+kf_pass_kernel(double* __restrict__ P, const ItemD* __restrict__ items, int n_items, int* counter,
+               const double* __restrict__ gpad, const double* __restrict__ upend, const KfState* st,
+               double* __restrict__ ws) {
+  extern __shared__ __align__(128) unsigned char smem[];
+  double* tiles = reinterpret_cast<double*>(smem);
+  double* colred = tiles + STAGES * TILE_ELEMS;
+  uint64_t* full = reinterpret_cast<uint64_t*>(colred + 2 * 8 * KT);
+  uint64_t* empty = full + STAGES;
+  int4* meta = reinterpret_cast<int4*>(empty + STAGES);
+  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+
+  if (tid == 0) {
+    for (int s = 0; s < STAGES; ++s) {
+      mbar_init(&full[s], 1);
+      mbar_init(&empty[s], 1);
+    }
+    fence_mbar_init();
+  }
+  __syncthreads();
+
+  if (warp == 8) {
+    // ------------------------------ producer ------------------------------
+    if (lane == 0) {
+      int s = 0;
+      uint32_t ph = 0;
+      while (true) {
+        const int itx = atomicAdd(counter, 1);
+        if (itx >= n_items) break;
+        const ItemD it = items[itx];
+        for (int t = 0; t < it.nJ; ++t) {
+          mbar_wait(&empty[s], ph ^ 1);
+          meta[s] = make_int4(itx, it.J0 + t, (t == 0 ? 1 : 0) | (t == it.nJ - 1 ? 2 : 0), 0);
+          mbar_arrive_tx(&full[s], TILE_BYTES);
+          tma_load_1d(tiles + (size_t)s * TILE_ELEMS, P + (size_t)(it.tile_off + t) * TILE_ELEMS, TILE_BYTES,
+                      &full[s]);
+          if (++s == STAGES) { s = 0; ph ^= 1; }
+        }
+      }
+      mbar_wait(&empty[s], ph ^ 1);
+      meta[s] = make_int4(-1, 0, 0, 0);
+      mbar_arrive(&full[s]);
+    }
+    return;
+  }
+
+  // ------------------------------ consumers ------------------------------
+  const int pend = st->pend;
+  const double Ap = st->A_pend;
+  const double il = st->invlam_pend;
+  const int c0 = 2 * lane;
+  double gI[8], uI[8], racc[8];
+#pragma unroll
+  for (int k = 0; k < 8; ++k) { gI[k] = 0.0; uI[k] = 0.0; racc[k] = 0.0; }
+  int s = 0, prev_s = -1;
+  uint32_t ph = 0;
+  uint32_t tcount = 0;
+  while (true) {
+    mbar_wait(&full[s], ph);
+    const int4 mt = meta[s];
+    if (mt.x < 0) break;
+    const ItemD it = items[mt.x];
+    const int J = mt.y;
+    const bool first = mt.z & 1, last = mt.z & 2, diag = (J == it.I);
+    if (first) {
+#pragma unroll
+      for (int k = 0; k < 8; ++k) {
+        const long long v = it.vbase + (long long)it.I * KT + warp + 8 * k;
+        gI[k] = __ldg(gpad + v);
+        uI[k] = __ldg(upend + v);
+        racc[k] = 0.0;
+      }
+    }
+    const long long vj = it.vbase + (long long)J * KT + c0;
+    const double2 gJ = __ldg(reinterpret_cast<const double2*>(gpad + vj));
+    const double2 uJ = __ldg(reinterpret_cast<const double2*>(upend + vj));
+    double* t = tiles + (size_t)s * TILE_ELEMS;
+    double ca0 = 0.0, ca1 = 0.0;
+#pragma unroll
+    for (int k = 0; k < 8; ++k) {
+      const int r = warp + 8 * k;
+      double2 v = *reinterpret_cast<double2*>(t + r * KT + c0);
+      if (pend) {
+        v.x = __dmul_rn(__dsub_rn(v.x, __dmul_rn(Ap, __dmul_rn(uI[k], uJ.x))), il);
+        v.y = __dmul_rn(__dsub_rn(v.y, __dmul_rn(Ap, __dmul_rn(uI[k], uJ.y))), il);
+        *reinterpret_cast<double2*>(t + r * KT + c0) = v;
+      }
+      racc[k] = fma(v.x, gJ.x, fma(v.y, gJ.y, racc[k]));
+      ca0 = fma(v.x, gI[k], ca0);
+      ca1 = fma(v.y, gI[k], ca1);
+    }
+    double* cr = colred + (tcount & 1) * (8 * KT);
+    if (!diag) {
+      cr[warp * KT + c0] = ca0;
+      cr[warp * KT + c0 + 1] = ca1;
+    }
+    consumer_bar();
+    if (tid == 0) {
+      if (pend) {
+        fence_proxy_async();
+        tma_store_1d(P + (size_t)(it.tile_off + (J - it.J0)) * TILE_ELEMS, t, TILE_BYTES);
+        bulk_commit();
+        if (prev_s >= 0) {
+          bulk_wait_read<1>();
+          mbar_arrive(&empty[prev_s]);
+        }
+        prev_s = s;
+      } else {
+        mbar_arrive(&empty[s]);  // read-only pass: the stage is free once every consumer passed the barrier
+      }
+    }
+    if (!diag && tid < KT) {
+      double a = 0.0;
+#pragma unroll
+      for (int w = 0; w < 8; ++w) a += cr[w * KT + tid];
+      ws[(size_t)(it.col_slot0 + (J - it.J0)) * KT + tid] = a;
+    }
+    if (last) {
+#pragma unroll
+      for (int k = 0; k < 8; ++k) {
+        double v = racc[k];
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+        if (lane == 0) ws[(size_t)it.row_slot * KT + warp + 8 * k] = v;
+      }
+    }
+    if (++s == STAGES) { s = 0; ph ^= 1; }
+    ++tcount;
+  }
+  if (tid == 0) {
+    if (prev_s >= 0) {
+      bulk_wait_read<0>();
+      mbar_arrive(&empty[prev_s]);
+    }
+    bulk_wait_all();
+  }
+}
+
+// ------------------------------------------------------------------------------------------------
+// small kernels
+// ------------------------------------------------------------------------------------------------
+// g (flat, n_i per block) -> padded vector (n_t*T per block, zero pad)
+__global__ void kf_pad_kernel(const double* __restrict__ g, double* __restrict__ gpad, const int* tc_blk,
+                              const int* tc_c, const long long* off, const int* nblk, long long npad) {
+  long long p = (long long)blockIdx.x * blockDim.x + threadIdx.x;
+  if (p >= npad) return;
+  const long long tc = p / KT;
+  const int b = tc_blk[tc];
+  const int loc = tc_c[tc] * KT + (int)(p % KT);
+  gpad[p] = loc < nblk[b] ? g[off[b] + loc] : 0.0;
+}
+
+// u[tc*T + t] = sum over the CSR entries of tile column tc (fixed order)
+__global__ void kf_reduce_u_kernel(const double* __restrict__ ws, const long long* __restrict__ ptr,
+                                   const long long* __restrict__ idx, long long n_tc, double* __restrict__ u) {
+  const long long tc = (long long)blockIdx.x * (blockDim.x / KT) + threadIdx.x / KT;
+  const int t = threadIdx.x % KT;
+  if (tc >= n_tc) return;
+  double a = 0.0;
+  for (long long e = ptr[tc]; e < ptr[tc + 1]; ++e) a += ws[(size_t)idx[e] * KT + t];
+  u[tc * KT + t] = a;
+}
+
+// dotp[tc] = sum_t gpad * u over tile column tc
+__global__ void kf_dot_kernel(const double* __restrict__ gpad, const double* __restrict__ u, long long n_tc,
+                              double* __restrict__ dotp) {
+  const long long tc = (long long)blockIdx.x * (blockDim.x / 32) + threadIdx.x / 32;
+  const int lane = threadIdx.x & 31;
+  if (tc >= n_tc) return;
+  double a = gpad[tc * KT + lane] * u[tc * KT + lane] + gpad[tc * KT + 32 + lane] * u[tc * KT + 32 + lane];
+  for (int o = 16; o > 0; o >>= 1) a += __shfl_xor_sync(0xffffffffu, a, o);
+  if (lane == 0) dotp[tc] = a;
+}
+
+// A = 1/(c + g^T u), K = A u, coef = sqrt(bs) ABE A, pending <- (A, 1/lambda), lambda update (Eq. 3)
+__global__ void kf_finish_kernel(const double* __restrict__ dotp, long long n_tc, KfState* st,
+                                 const double* abe, double sqrt_bs) {
+  __shared__ double red[1024];
+  double a = 0.0;
+  for (long long i = threadIdx.x; i < n_tc; i += blockDim.x) a += dotp[i];
+  red[threadIdx.x] = a;
+  __syncthreads();
+  for (int s = blockDim.x / 2; s > 0; s >>= 1) {
+    if ((int)threadIdx.x < s) red[threadIdx.x] += red[threadIdx.x + s];
+    __syncthreads();
+  }
+  if (threadIdx.x == 0) {
+    const double lam = st->lambda;
+    const double c = st->c_mult * lam;                  // c = L*lambda (Z1) or lambda
+    const double A = 1.0 / (c + red[0]);                // Alg. 1 line 8
+    const double e = abe ? *abe : 0.0;
+    st->A_last = A;
+    st->A_pend = A;
+    st->invlam_pend = 1.0 / lam;                        // line 10 uses the pre-increment lambda
+    st->pend = 1;
+    st->coef = sqrt_bs * e * A;                         // line 13 / Eq. 2: w += sqrt(bs) ABE K, K = A u
+    st->lambda = lam * st->nu + 1.0 - st->nu;           // line 12 (Eq. 3)
+    st->t += 1;
+    if (!isfinite(A) || !isfinite(e)) st->flags |= 2;
+  }
+}
+
+__global__ void kf_w_update_kernel(double* __restrict__ w, const double* __restrict__ u, const KfState* st,
+                                   const int* tc_blk, const int* tc_c, const long long* off, const int* nblk,
+                                   long long npad) {
+  long long p = (long long)blockIdx.x * blockDim.x + threadIdx.x;
+  if (p >= npad) return;
+  const long long tc = p / KT;
+  const int b = tc_blk[tc];
+  const int loc = tc_c[tc] * KT + (int)(p % KT);
+  if (loc < nblk[b]) w[off[b] + loc] += st->coef * u[p];
+}
+
+// apply the pending correction to stored tiles (flush) — one CTA per item
+__global__ void kf_apply_pending_kernel(double* __restrict__ P, const ItemD* __restrict__ items,
+                                        const double* __restrict__ upend, KfState* st) {
+  if (!st->pend) return;
+  const ItemD it = items[blockIdx.x];
+  const double Ap = st->A_pend, il = st->invlam_pend;
+  for (int t = 0; t < it.nJ; ++t) {
+    double* tile = P + (size_t)(it.tile_off + t) * TILE_ELEMS;
+    const int J = it.J0 + t;
+    for (int e = threadIdx.x; e < TILE_ELEMS; e += blockDim.x) {
+      const int r = e / KT, c = e % KT;
+      const double ur = upend[it.vbase + (long long)it.I * KT + r];
+      const double uc = upend[it.vbase + (long long)J * KT + c];
+      tile[e] = __dmul_rn(__dsub_rn(tile[e], __dmul_rn(Ap, __dmul_rn(ur, uc))), il);
+    }
+  }
+}
+__global__ void kf_clear_pending_kernel(KfState* st) { st->pend = 0; }
+
+// P = I on the valid part of every block, 0 on the padding
+__global__ void kf_init_kernel(double* __restrict__ P, const ItemD* __restrict__ items, const int* nblk) {
+  const ItemD it = items[blockIdx.x];
+  const int n = nblk[it.blk];
+  for (int t = 0; t < it.nJ; ++t) {
+    double* tile = P + (size_t)(it.tile_off + t) * TILE_ELEMS;
+    const int J = it.J0 + t;
+    for (int e = threadIdx.x; e < TILE_ELEMS; e += blockDim.x) {
+      const int r = e / KT, c = e % KT;
+      const int gr = it.I * KT + r, gc = J * KT + c;
+      tile[e] = (gr == gc && gr < n) ? 1.0 : 0.0;
+    }
+  }
+}
+
+// dense <-> packed for one block (tests / checkpoints)
+__global__ void kf_get_block_kernel(const double* __restrict__ P, const ItemD* __restrict__ items, int blk, int n,
+                                    const double* __restrict__ upend, const KfState* st, double* __restrict__ dst) {
+  const ItemD it = items[blockIdx.x];
+  if (it.blk != blk) return;
+  const int pend = st->pend;
+  const double Ap = st->A_pend, il = st->invlam_pend;
+  for (int t = 0; t < it.nJ; ++t) {
+    const double* tile = P + (size_t)(it.tile_off + t) * TILE_ELEMS;
+    const int J = it.J0 + t;
+    for (int e = threadIdx.x; e < TILE_ELEMS; e += blockDim.x) {
+      const int r = e / KT, c = e % KT;
+      const int gr = it.I * KT + r, gc = J * KT + c;
+      if (gr >= n || gc >= n) continue;
+      double v = tile[e];
+      if (pend) {
+        const double ur = upend[it.vbase + gr], uc = upend[it.vbase + gc];
+        v = __dmul_rn(__dsub_rn(v, __dmul_rn(Ap, __dmul_rn(ur, uc))), il);
+      }
+      dst[(size_t)gr * n + gc] = v;
+      if (J != it.I) dst[(size_t)gc * n + gr] = v;
+    }
+  }
+}
+__global__ void kf_set_block_kernel(double* __restrict__ P, const ItemD* __restrict__ items, int blk, int n,
+                                    const double* __restrict__ src) {
+  const ItemD it = items[blockIdx.x];
+  if (it.blk != blk) return;
+  for (int t = 0; t < it.nJ; ++t) {
+    double* tile = P + (size_t)(it.tile_off + t) * TILE_ELEMS;
+    const int J = it.J0 + t;
+    for (int e = threadIdx.x; e < TILE_ELEMS; e += blockDim.x) {
+      const int r = e / KT, c = e % KT;
+      const int gr = it.I * KT + r, gc = J * KT + c;
+      tile[e] = (gr < n && gc < n) ? src[(size_t)gr * n + gc] : 0.0;
+    }
+  }
+}
+
+// ------------------------------------------------------------------------------------------------
+// host side of fekf_kf
+// ------------------------------------------------------------------------------------------------
+static int num_sms() {
+  static int sms = 0;
+  if (!sms) {
+    int dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    if (sms <= 0) sms = 148;
+  }
+  return sms;
+}
+
+fekf_status Kf::create(const std::vector<int>& blocks, const fekf_opt_cfg& o, fekf_comm* c) {
+  opt = o;
+  comm = c;
+  int world = 1, rank = 0;
+  if (comm) { world = comm_world(comm); rank = comm_rank(comm); }
+  plan.build(blocks, world, rank, SEG_TILES);
+  const KfPlan& p = plan;
+  FEKF_TRY(dalloc(P, (size_t)p.tiles_local * TILE_BYTES + 16));
+  FEKF_TRY(dalloc(items_d, std::max<size_t>(1, p.items.size()) * sizeof(ItemD)));
+  FEKF_TRY(dalloc(ws, (size_t)std::max<int64_t>(1, p.ws_slots) * KT * sizeof(double)));
+  FEKF_TRY(dalloc(gpad, p.Npad * sizeof(double)));
+  FEKF_TRY(dalloc(unew, p.Npad * sizeof(double)));
+  FEKF_TRY(dalloc(upend, p.Npad * sizeof(double)));
+  FEKF_TRY(dalloc(dotp, p.n_tc * sizeof(double)));
+  FEKF_TRY(dalloc(csr_ptr, (p.n_tc + 1) * sizeof(long long)));
+  FEKF_TRY(dalloc(csr_idx, std::max<size_t>(1, p.csr_idx.size()) * sizeof(long long)));
+  FEKF_TRY(dalloc(tc_blk, p.n_tc * sizeof(int)));
+  FEKF_TRY(dalloc(tc_c, p.n_tc * sizeof(int)));
+  FEKF_TRY(dalloc(off_d, (p.L + 1) * sizeof(long long)));
+  FEKF_TRY(dalloc(n_d, p.L * sizeof(int)));
+  FEKF_TRY(dalloc(state, sizeof(KfState)));
+  FEKF_TRY(dalloc(counter, sizeof(int)));
+  if (!p.items.empty())
+    FEKF_CHECK_CUDA(cudaMemcpy(items_d.p, p.items.data(), p.items.size() * sizeof(ItemD), cudaMemcpyHostToDevice));
+  FEKF_CHECK_CUDA(cudaMemcpy(csr_ptr.p, p.csr_ptr.data(), (p.n_tc + 1) * sizeof(long long), cudaMemcpyHostToDevice));
+  if (!p.csr_idx.empty())
+    FEKF_CHECK_CUDA(cudaMemcpy(csr_idx.p, p.csr_idx.data(), p.csr_idx.size() * sizeof(long long), cudaMemcpyHostToDevice));
+  FEKF_CHECK_CUDA(cudaMemcpy(tc_blk.p, p.tc_blk.data(), p.n_tc * sizeof(int), cudaMemcpyHostToDevice));
+  FEKF_CHECK_CUDA(cudaMemcpy(tc_c.p, p.tc_c.data(), p.n_tc * sizeof(int), cudaMemcpyHostToDevice));
+  FEKF_CHECK_CUDA(cudaMemcpy(off_d.p, p.off.data(), (p.L + 1) * sizeof(long long), cudaMemcpyHostToDevice));
+  FEKF_CHECK_CUDA(cudaMemcpy(n_d.p, p.n.data(), p.L * sizeof(int), cudaMemcpyHostToDevice));
+  KfState s{};
+  s.lambda = o.lambda0;
+  s.nu = o.nu;
+  s.c_mult = o.noise_mode == 0 ? (double)p.L : 1.0;
+  FEKF_CHECK_CUDA(cudaMemcpy(state.p, &s, sizeof(KfState), cudaMemcpyHostToDevice));
+  FEKF_CHECK_CUDA(cudaMemset(upend.p, 0, p.Npad * sizeof(double)));
+  FEKF_CHECK_CUDA(cudaMemset(unew.p, 0, p.Npad * sizeof(double)));
+  FEKF_CHECK_CUDA(cudaFuncSetAttribute(kf_pass_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)PASS_SMEM));
+  if (!p.items.empty()) {
+    kf_init_kernel<<<(unsigned)p.items.size(), 256>>>(P.as<double>(), items_d.as<ItemD>(), n_d.as<int>());
+    FEKF_LAUNCH_CHECK();
+  }
+  FEKF_CHECK_CUDA(cudaDeviceSynchronize());
+  return FEKF_OK;
+}
+
+Kf::~Kf() {
+  for (DBuf* b : {&P, &items_d, &ws, &gpad, &unew, &upend, &dotp, &csr_ptr, &csr_idx, &tc_blk, &tc_c, &off_d, &n_d,
+                  &state, &counter})
+    dfree(*b);
+}
+
+fekf_status Kf::pass(const double* g, cudaStream_t s) {
+  const KfPlan& p = plan;
+  const int tb = 256;
+  kf_pad_kernel<<<cdiv(p.Npad, tb), tb, 0, s>>>(g, gpad.as<double>(), tc_blk.as<int>(), tc_c.as<int>(),
+                                                 off_d.as<long long>(), n_d.as<int>(), p.Npad);
+  FEKF_LAUNCH_CHECK();
+  count_launch();
+  if (!p.items.empty()) {
+    FEKF_CHECK_CUDA(cudaMemsetAsync(counter.p, 0, sizeof(int), s));
+    const int grid = std::min<int>((int)p.items.size(), num_sms());
+    kf_pass_kernel<<<grid, PASS_THREADS, PASS_SMEM, s>>>(P.as<double>(), items_d.as<ItemD>(), (int)p.items.size(),
+                                                          counter.as<int>(), gpad.as<double>(), upend.as<double>(),
+                                                          state.as<KfState>(), ws.as<double>());
+    FEKF_LAUNCH_CHECK();
+    count_launch();
+  }
+  kf_reduce_u_kernel<<<cdiv(p.n_tc, 4), 256, 0, s>>>(ws.as<double>(), csr_ptr.as<long long>(),
+                                                      csr_idx.as<long long>(), p.n_tc, unew.as<double>());
+  FEKF_LAUNCH_CHECK();
+  count_launch();
+  return FEKF_OK;
+}
+
+fekf_status Kf::update(const double* g, const double* abe, double sqrt_bs, double* w, cudaStream_t s) {
+  const KfPlan& p = plan;
+  FEKF_TRY(pass(g, s));
+  if (comm && comm_world(comm) > 1) FEKF_TRY(comm_allreduce(comm, unew.as<double>(), p.Npad, s));
+  kf_dot_kernel<<<cdiv(p.n_tc, 8), 256, 0, s>>>(gpad.as<double>(), unew.as<double>(), p.n_tc, dotp.as<double>());
+  FEKF_LAUNCH_CHECK();
+  kf_finish_kernel<<<1, 1024, 0, s>>>(dotp.as<double>(), p.n_tc, state.as<KfState>(), abe, sqrt_bs);
+  FEKF_LAUNCH_CHECK();
+  kf_w_update_kernel<<<cdiv(p.Npad, 256), 256, 0, s>>>(w, unew.as<double>(), state.as<KfState>(), tc_blk.as<int>(),
+                                                        tc_c.as<int>(), off_d.as<long long>(), n_d.as<int>(), p.Npad);
+  FEKF_LAUNCH_CHECK();
+  FEKF_CHECK_CUDA(cudaMemcpyAsync(upend.p, unew.p, p.Npad * sizeof(double), cudaMemcpyDeviceToDevice, s));
+  count_launch(3);
+  return FEKF_OK;
+}
+
+fekf_status Kf::flush(cudaStream_t s) {
+  if (!plan.items.empty()) {
+    kf_apply_pending_kernel<<<(unsigned)plan.items.size(), 256, 0, s>>>(P.as<double>(), items_d.as<ItemD>(),
+                                                                         upend.as<double>(), state.as<KfState>());
+    FEKF_LAUNCH_CHECK();
+  }
+  kf_clear_pending_kernel<<<1, 1, 0, s>>>(state.as<KfState>());
+  FEKF_LAUNCH_CHECK();
+  return FEKF_OK;
+}
+
+fekf_status Kf::get_block(int b, double* dst, cudaStream_t s) {
+  if (b < 0 || b >= plan.L) { set_error("get_block: bad block"); return FEKF_EINVAL; }
+  if (plan.items.empty()) return FEKF_OK;
+  kf_get_block_kernel<<<(unsigned)plan.items.size(), 256, 0, s>>>(P.as<double>(), items_d.as<ItemD>(), b, plan.n[b],
+                                                                   upend.as<double>(), state.as<KfState>(), dst);
+  FEKF_LAUNCH_CHECK();
+  return FEKF_OK;
+}
+
+fekf_status Kf::set_block(int b, const double* src, cudaStream_t s) {
+  if (b < 0 || b >= plan.L) { set_error("set_block: bad block"); return FEKF_EINVAL; }
+  FEKF_TRY(flush(s));
+  if (plan.items.empty()) return FEKF_OK;
+  kf_set_block_kernel<<<(unsigned)plan.items.size(), 256, 0, s>>>(P.as<double>(), items_d.as<ItemD>(), b, plan.n[b],
+                                                                   src);
+  FEKF_LAUNCH_CHECK();
+  return FEKF_OK;
+}
+
+fekf_status Kf::get_state(double* lambda, double* A_last, int* flags) {
+  KfState s;
+  FEKF_CHECK_CUDA(cudaDeviceSynchronize());
+  FEKF_CHECK_CUDA(cudaMemcpy(&s, state.p, sizeof(KfState), cudaMemcpyDeviceToHost));
+  if (lambda) *lambda = s.lambda;
+  if (A_last) *A_last = s.A_last;
+  if (flags) *flags = s.flags;
+  return FEKF_OK;
+}
+
+}  // namespace fekf

@@ -1,0 +1,70 @@
+// Blocked Kalman filter state (see kalman.cu for the algorithm and its citations).
+#pragma once
+#include <vector>
+
+#include "common.cuh"
+
+namespace fekf {
+
+constexpr int KT = FEKF_TILE;    // tile edge (64 fp64 = 32 KiB per tile)
+constexpr int SEG_TILES = 32;    // max tiles per work item (tile-row segment)
+
+// One P-pass work item: tiles (I, J0..J0+nJ-1) of block `blk`, stored contiguously at tile_off.
+struct ItemD {
+  int blk, I, J0, nJ;
+  long long tile_off;   // in tiles, into this rank's P buffer
+  long long vbase;      // offset of the block in the padded vectors
+  long long col_slot0;  // workspace slot of the first tile's column partial
+  int row_slot;         // workspace slot of the item's row partial
+  int pad_;
+};
+
+// Device-resident optimizer scalars.
+struct KfState {
+  double lambda, nu;
+  double A_pend, invlam_pend;  // pending rank-1 correction (applied by the next pass)
+  double A_last, coef;         // last A and sqrt(bs)*ABE*A
+  double c_mult;               // L (noise_mode 0) or 1
+  long long t;
+  int pend, flags;
+};
+
+struct KfPlan {
+  int L = 0, world = 1, rank = 0;
+  std::vector<int> n, nt;
+  std::vector<long long> off, tc_off;
+  long long N = 0, n_tc = 0, Npad = 0;
+  std::vector<int> tc_blk, tc_c;
+  std::vector<ItemD> items;           // this rank's items (largest first)
+  long long tiles_local = 0, total_tiles = 0, ws_slots = 0;
+  std::vector<int> owner;             // owner rank of every canonical item
+  std::vector<int> tile_owner;        // owner rank of every tile, canonical packed order
+  std::vector<long long> csr_ptr, csr_idx;
+  void build(const std::vector<int>& blocks, int world, int rank, int seg_tiles);
+};
+
+// communicator helpers (comm.cu)
+int comm_world(fekf_comm* c);
+int comm_rank(fekf_comm* c);
+fekf_status comm_allreduce(fekf_comm* c, double* buf, long long n, cudaStream_t s);
+
+struct Kf {
+  fekf_opt_cfg opt{};
+  fekf_comm* comm = nullptr;
+  KfPlan plan;
+  DBuf P, items_d, ws, gpad, unew, upend, dotp, csr_ptr, csr_idx, tc_blk, tc_c, off_d, n_d, state, counter;
+  fekf_status create(const std::vector<int>& blocks, const fekf_opt_cfg& o, fekf_comm* c);
+  ~Kf();
+  fekf_status pass(const double* g, cudaStream_t s);
+  fekf_status update(const double* g, const double* abe, double sqrt_bs, double* w, cudaStream_t s);
+  fekf_status flush(cudaStream_t s);
+  fekf_status get_block(int b, double* dst, cudaStream_t s);
+  fekf_status set_block(int b, const double* src, cudaStream_t s);
+  fekf_status get_state(double* lambda, double* A_last, int* flags);
+};
+
+}  // namespace fekf
+
+struct fekf_kf {
+  fekf::Kf kf;
+};

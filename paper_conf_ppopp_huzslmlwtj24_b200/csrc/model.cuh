@@ -1,0 +1,87 @@
+// DeePMD se_a model context: parameter layout, work buffers and the kernel launchers of the
+// forward / backward / Jacobian passes.  See nets.cu for the math and citations.
+#pragma once
+#include <memory>
+#include <vector>
+
+#include "kalman.cuh"
+
+namespace fekf {
+
+struct Layer {
+  int din, dout;
+  long long W, b, dt;  // offsets into the flat parameter vector (dt = -1: none)
+  int skip;            // 0 none, 1 identity (d_l == d_{l-1}), 2 concat [h, h] (d_l == 2 d_{l-1})
+};
+
+struct PairNet {       // embedding net of the type pair (ti, tj)
+  int ti, tj;
+  long long R;         // rows = B * n_ti * sel_tj (padded slots included; they carry R~ = 0)
+  std::vector<Layer> L;
+  DBuf hin;            // [2R]       s (primal rows) and s-dot (tangent rows)
+  std::vector<DBuf> Y, H, Hb, Zb;   // per layer [2R x d_l]
+  DBuf sbar;           // [R] adjoint of s (forces)
+};
+
+struct FitNet {        // fitting net of type t
+  int t;
+  long long F;         // rows = B * n_t
+  std::vector<Layer> L;
+  long long Wout, bout;
+  DBuf D, Db;          // [2F x M*M2]
+  std::vector<DBuf> Y, H, Hb, Zb;
+  DBuf eout, ebar;     // [2F]
+};
+
+struct Ctx {
+  fekf_model_cfg m{};
+  fekf_opt_cfg o{};
+  int Na = 0, B = 0, Bg = 0, nt = 0, Nm = 0, M = 0, M2 = 0;
+  int sec[FEKF_MAX_TYPES + 1]{};
+  std::vector<int> types, tindex;                 // type of atom, index within its type
+  std::vector<std::vector<int>> atoms_of;         // atoms of each type
+  long long Np = 0;
+  std::vector<int> blocks;
+  std::vector<PairNet> pairs;                     // nt*nt, index ti*nt + tj
+  std::vector<FitNet> fits;                       // nt
+  fekf_comm* comm = nullptr;
+  std::unique_ptr<::fekf_kf> kfo;                 // owns the Kalman filter
+  Kf* kf = nullptr;
+  // device
+  DBuf types_d, tindex_d, atoms_d, atoms_off_d, sel_d, sec_d, err_d;
+  DBuf w, gbuf;                                   // [Np], [Np + 1] (g || error sum, the allreduce payload)
+  DBuf nl_j, nl_s, overflow, em, jac, rij, rdot, vdir;
+  DBuf X, Xb;                                     // [2 * B*Na*4*M] (primal | tangent)
+  DBuf eatom, etot, force, virial;
+  DBuf splitk_ws, colsum_ws;
+  DBuf abe, metrics_tmp, abs_sum;
+  size_t splitk_elems = 0, colsum_elems = 0;
+  int64_t last_launches = 0;
+
+  fekf_status init(const fekf_model_cfg& m, const fekf_opt_cfg& o, int natoms, const int32_t* types_host, int B,
+                   int Bg, fekf_comm* comm);
+  ~Ctx();
+};
+
+// geom.cu
+fekf_status launch_nlist(Ctx& c, const double* coord, const double* box, int nb, int* nl_j, int* nl_s, int* overflow,
+                         cudaStream_t s);
+fekf_status launch_envmat(Ctx& c, const double* coord, const double* box, const int* nl_j, const int* nl_s, int nb,
+                          double* em, double* jac, double* rij, cudaStream_t s);
+
+// nets.cu
+enum Mode { MODE_ENERGY_GRAD = 0, MODE_FORCE = 1, MODE_FORCE_JAC = 2 };
+fekf_status model_forward(Ctx& c, int nb, bool tangent, cudaStream_t s);
+fekf_status model_backward(Ctx& c, int nb, Mode mode, double* g, cudaStream_t s);
+fekf_status energy_outputs(Ctx& c, int nb, cudaStream_t s);
+fekf_status energy_error(Ctx& c, int nb, const double* e_label, double* abs_sum, cudaStream_t s);
+fekf_status force_error(Ctx& c, int nb, const double* f_label, const int* atom_idx, int n_sel, double* abs_sum,
+                        cudaStream_t s);
+fekf_status tangent_env(Ctx& c, int nb, cudaStream_t s);
+fekf_status seed_force(Ctx& c, int nb, cudaStream_t s);
+
+}  // namespace fekf
+
+struct fekf_ctx {
+  fekf::Ctx c;
+};

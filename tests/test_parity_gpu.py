@@ -1,0 +1,176 @@
+"""GPU parity: the CUDA path (through the C ABI) against the fp64 CPU oracle on the same seeded inputs.
+
+Tolerances (north_star): neighbour lists / indices bit-exact; descriptor, energy, force rel 1e-12;
+weights and P after 10 EKF steps rel 1e-9.  "rel" is normwise: max|gpu - ref| / max|ref| per tensor
+(reading Z19).  Jacobians: rel 1e-11.
+"""
+import numpy as np
+import pytest
+import torch
+
+import oracle as O
+from fixtures import get_config, make_dataset, init_weights, force_groups
+
+pytestmark = pytest.mark.gpu
+
+fk = pytest.importorskip("paper_conf_ppopp_huzslmlwtj24_b200")
+
+
+def rel(a, b):
+    a = np.asarray(a, dtype=np.float64)
+    b = np.asarray(b, dtype=np.float64)
+    den = np.abs(b).max()
+    return float(np.abs(a - b).max() / (den if den > 0 else 1.0))
+
+
+def cu(x, dtype=torch.float64):
+    return torch.as_tensor(np.ascontiguousarray(x)).to(dtype).cuda()
+
+
+@pytest.fixture(scope="module", autouse=True)
+def _gpu():
+    if not torch.cuda.is_available():
+        pytest.skip("no GPU")
+    fk.lib()
+
+
+def _setup(name, nb, sel=None, seed=3):
+    wl = get_config(name)
+    m = wl.model
+    if sel is not None:
+        m = type(m)(**{**m.__dict__, "sel": sel})
+    ds = make_dataset(name, nb)
+    w = init_weights(m, seed, float(ds["energy"].mean() / len(ds["types"])))
+    ctx = fk.Context(m, wl.opt, types=ds["types"], local_batch=nb, global_batch=nb)
+    ctx.set_params(cu(w))
+    return wl, m, ds, w, ctx
+
+
+CASES = [("t2_tiny", 3), ("c1_cu32", 4), ("paper_cu108", 2), ("c2_water64", 2)]
+
+
+@pytest.mark.parametrize("name,nb", CASES)
+def test_nlist_bit_exact(name, nb):
+    wl, m, ds, w, ctx = _setup(name, nb)
+    nj, ns, ov = ctx.build_nlist(cu(ds["coord"]), cu(ds["box"]))
+    rj, rs, rov = O.build_nlist(ds["coord"], ds["box"], ds["types"], m.rcut, m.sel)
+    assert np.array_equal(nj.cpu().numpy(), rj)
+    assert np.array_equal(ns.cpu().numpy(), rs)
+    assert np.array_equal(ov.cpu().numpy(), rov)
+
+
+def test_nlist_overflow_bit_exact():
+    wl, m, ds, w, ctx = _setup("t2_tiny", 3, sel=[5, 9])
+    nj, ns, ov = ctx.build_nlist(cu(ds["coord"]), cu(ds["box"]))
+    rj, rs, rov = O.build_nlist(ds["coord"], ds["box"], ds["types"], m.rcut, [5, 9])
+    assert rov.sum() > 0
+    assert np.array_equal(nj.cpu().numpy(), rj) and np.array_equal(ns.cpu().numpy(), rs)
+    assert np.array_equal(ov.cpu().numpy(), rov)
+
+
+@pytest.mark.parametrize("name,nb", CASES)
+def test_env_mat(name, nb):
+    wl, m, ds, w, ctx = _setup(name, nb)
+    rj, rs, _ = O.build_nlist(ds["coord"], ds["box"], ds["types"], m.rcut, m.sel)
+    em, jac, rij = ctx.env_mat(cu(ds["coord"]), cu(ds["box"]), cu(rj, torch.int32), cu(rs, torch.int32))
+    d, R, mask = O.env_mat(torch.as_tensor(ds["coord"]), ds["box"], rj, rs, m.rcut, m.rcut_smth)
+    assert rel(rij.cpu(), d) < 1e-14
+    assert rel(em.cpu(), R) < 1e-12
+    # J = dR~/dd by autograd on the oracle's R~(d)
+    dl = d.detach().clone().requires_grad_(True)
+    rows = O.env_rows(dl, mask, m.rcut, m.rcut_smth)
+    J = torch.stack([torch.autograd.grad(rows[..., k].sum(), dl, retain_graph=True)[0] for k in range(4)], dim=-2)
+    assert rel(jac.cpu(), J) < 1e-12
+
+
+@pytest.mark.parametrize("name,nb", CASES)
+def test_forward_energy_force_virial(name, nb):
+    wl, m, ds, w, ctx = _setup(name, nb)
+    ea, e, f, v = ctx.forward(cu(ds["coord"]), cu(ds["box"]))
+    rj, rs, _ = O.build_nlist(ds["coord"], ds["box"], ds["types"], m.rcut, m.sel)
+    Ea, E, F, V = O.energy_force_virial(w, ds["coord"], ds["box"], ds["types"], rj, rs, m)
+    assert rel(ea.cpu(), Ea) < 1e-12
+    assert rel(e.cpu(), E) < 1e-12
+    assert rel(f.cpu(), F) < 1e-12
+    assert rel(v.cpu().reshape(-1, 3, 3), V) < 1e-12
+
+
+@pytest.mark.parametrize("name,nb", CASES[:3])
+def test_energy_jacobian(name, nb):
+    wl, m, ds, w, ctx = _setup(name, nb)
+    g, s = ctx.energy_jacobian(cu(ds["coord"]), cu(ds["box"]), cu(ds["energy"]))
+    rj, rs, _ = O.build_nlist(ds["coord"], ds["box"], ds["types"], m.rcut, m.sel)
+    gr, sr, _ = O.energy_grad(w, ds["coord"], ds["box"], ds["types"], rj, rs, ds["energy"], m)
+    assert rel(g.cpu(), gr) < 1e-11
+    assert abs(float(s.cpu()[0]) - sr) <= 1e-13 * max(1.0, abs(sr))
+
+
+@pytest.mark.parametrize("name,nb", CASES[:3])
+def test_force_jacobian(name, nb):
+    wl, m, ds, w, ctx = _setup(name, nb)
+    atoms = force_groups(len(ds["types"]), 0, 5)[0]
+    g, s = ctx.force_jacobian(cu(ds["coord"]), cu(ds["box"]), cu(ds["force"]), cu(atoms, torch.int32))
+    rj, rs, _ = O.build_nlist(ds["coord"], ds["box"], ds["types"], m.rcut, m.sel)
+    gr, sr, _ = O.force_grad(w, ds["coord"], ds["box"], ds["types"], rj, rs, ds["force"], atoms, m)
+    assert rel(g.cpu(), gr) < 1e-11
+    assert abs(float(s.cpu()[0]) - sr) <= 1e-12 * max(1.0, abs(sr))
+
+
+def _rand_spd(rng, n):
+    a = rng.standard_normal((n, n))
+    return a @ a.T / n + np.eye(n)
+
+
+@pytest.mark.parametrize("blocks", [[5, 70, 130], [64], [1, 200, 127, 65]])
+@pytest.mark.parametrize("noise_mode", [0, 1])
+def test_kalman_updates(blocks, noise_mode):
+    rng = np.random.default_rng(7)
+    opt = dict(lambda0=0.98, nu=0.9987, block_size=1024, noise_mode=noise_mode)
+    kf = fk.KalmanFilter(blocks, opt)
+    N = sum(blocks)
+    st = O.FEKF(np.zeros(N), blocks, lam=0.98, nu=0.9987, noise_mode=noise_mode)
+    st.P = [_rand_spd(rng, n) for n in blocks]
+    for b, P in enumerate(st.P):
+        kf.set_block(b, cu(P))
+    w = torch.zeros(N, dtype=torch.float64, device="cuda")
+    for it in range(10):
+        g = rng.standard_normal(N)
+        abe = float(rng.uniform(0.01, 1.0))
+        kf.update(cu(g), cu([abe]), 3.0, w)
+        st.update(g, abe, 9)
+    torch.cuda.synchronize()
+    assert rel(w.cpu(), st.w) < 1e-12
+    for b in range(len(blocks)):
+        assert rel(kf.get_block(b).cpu(), st.P[b]) < 1e-12
+    assert abs(kf.state()["lambda"] - st.lam) < 1e-15
+    kf.flush()
+    for b in range(len(blocks)):
+        assert rel(kf.get_block(b).cpu(), st.P[b]) < 1e-12
+
+
+@pytest.mark.parametrize("name,steps", [("c1_cu32", 10), ("t2_tiny", 4)])
+def test_train_steps(name, steps):
+    wl = get_config(name)
+    m, opt = wl.model, wl.opt
+    ds = make_dataset(name, wl.batch * 2)
+    na = len(ds["types"])
+    w0 = init_weights(m, 3, float(ds["energy"].mean() / na))
+    B = wl.batch
+    ctx = fk.Context(m, opt, types=ds["types"], local_batch=B, global_batch=B)
+    ctx.set_params(cu(w0))
+    st = O.FEKF.create(w0, m, opt)
+    for step in range(steps):
+        sl = slice((step % 2) * B, (step % 2) * B + B)
+        groups = force_groups(na, step, 17, opt.force_groups, opt.atoms_per_group)
+        met = ctx.train_step(cu(ds["coord"][sl]), cu(ds["box"][sl]), cu(ds["energy"][sl]), cu(ds["force"][sl]),
+                             cu(groups, torch.int32))
+        ref = O.train_step(st, ds["coord"][sl], ds["box"][sl], ds["types"], ds["energy"][sl], ds["force"][sl],
+                           groups, m, opt)
+        mt = met.cpu().numpy()
+        assert abs(mt[0] - ref["abe_e"]) <= 1e-9 * abs(ref["abe_e"])
+        np.testing.assert_allclose(mt[1:5], ref["abe_f"], rtol=1e-9)
+        assert abs(mt[6] - ref["lambda"]) < 1e-14
+        assert mt[7] == 0
+    assert rel(ctx.get_params().cpu(), st.w) < 1e-9
+    for b, n in enumerate(st.blocks):
+        assert rel(ctx.kf.get_block(b).cpu(), st.P[b]) < 1e-9
