@@ -1,0 +1,328 @@
+#!/usr/bin/env python
+"""EKF training throughput of the B200-native FEKF DeePMD step (BASELINE.json metric).
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--config c2_water64] [--impl fekf|reference]
+
+One step = one minibatch of the paper's schedule: 1 energy update + 4 force updates, each a
+forward, a Jacobian, the early reduction (NCCL all-reduce over ranks) and the blocked Kalman update.
+Workload at N=1: BASELINE.json configs[1] (water-64, 192 atoms, se_a 6.0/0.5, sel [46,92], embedding
+(25,50,100), M^<=16, fitting (240,240,240), 32 images per GPU, N_b = 10240 -> 1 027 082 parameters,
+110 P blocks, 39 GiB of packed fp64 P).  Weak scaling: 32 images per GPU, global batch 32*N, P sharded.
+Prints ONE JSON line on rank 0.
+"""
+import argparse
+import json
+import math
+import os
+import statistics
+import subprocess
+import sys
+import tempfile
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+from fixtures import get_config, make_dataset, init_weights, force_groups  # noqa: E402
+
+METRIC = "EKF train images/sec"
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--config", default="c2_water64")
+    ap.add_argument("--impl", default="fekf", choices=["fekf", "reference"])
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    return ap.parse_args()
+
+
+def dist_env():
+    return int(os.environ.get("RANK", 0)), int(os.environ.get("WORLD_SIZE", 1)), int(os.environ.get("LOCAL_RANK", 0))
+
+
+def load_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        with open(p) as f:
+            d = json.load(f)
+        return float(d["hbm_gbs"]), "measured"
+    return 6650.0, "fallback (B200_PROFILING.md)"
+
+
+# ---------------------------------------------------------------------------------------------
+# clocks sampled during the timed region (B200_PROFILING.md clocks line)
+# ---------------------------------------------------------------------------------------------
+class Clocks:
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,clocks_event_reasons.hw_slowdown,"
+         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+         "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index):
+        self.index = index
+        self.f = tempfile.NamedTemporaryFile("w+", suffix=".csv", delete=False)
+        try:
+            self.p = subprocess.Popen(["nvidia-smi", "-i", str(index), f"--query-gpu={self.Q}", "--format=csv,noheader,nounits",
+                                       "-lms", "200"], stdout=self.f, stderr=subprocess.DEVNULL)
+        except Exception:
+            self.p = None
+
+    def stop(self):
+        if self.p is None:
+            return None
+        self.p.terminate()
+        try:
+            self.p.wait(5)
+        except Exception:
+            self.p.kill()
+        self.f.flush()
+        rows = []
+        with open(self.f.name) as f:
+            for line in f:
+                parts = [x.strip() for x in line.split(",")]
+                if len(parts) >= 9:
+                    rows.append(parts)
+        os.unlink(self.f.name)
+        if not rows:
+            return None
+        sm = [float(r[1]) for r in rows if r[1].replace(".", "").isdigit()]
+        mx = [float(r[2]) for r in rows if r[2].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[k] for r in rows for k in range(4) if r[5 + k].lower().startswith("active")})
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": reasons, "samples": len(rows)}
+
+
+# ---------------------------------------------------------------------------------------------
+# oracle timings (cpu_baseline leg and --impl reference): the oracle as it stands, host cores
+# ---------------------------------------------------------------------------------------------
+def oracle_sample(name, n_img=1, kf_blocks=1, seed=99):
+    """Bounded sample of one minibatch step: the oracle's nets (1 energy + 4 force gradients) on
+    `n_img` images and its Kalman update on `kf_blocks` blocks; extrapolated to a full step of the
+    workload (nets scale with images, Kalman with sum n_i^2 over all blocks, 5 updates per step)."""
+    import torch
+    import oracle as O
+    wl = get_config(name)
+    m, opt = wl.model, wl.opt
+    ds = make_dataset(name, n_img, seed=seed)
+    na = len(ds["types"])
+    w = init_weights(m, 3, float(ds["energy"].mean() / na))
+    sizes = [int(np.prod(s)) for _, s in O.param_tensors(m)]
+    blocks = O.block_split(sizes, opt.block_size)
+    groups = force_groups(na, 0, 5)
+    t0 = time.perf_counter()
+    nl = O.build_nlist(ds["coord"], ds["box"], ds["types"], m.rcut, m.sel)
+    O.energy_grad(w, ds["coord"], ds["box"], ds["types"], nl[0], nl[1], ds["energy"], m)
+    for a in groups:
+        O.force_grad(w, ds["coord"], ds["box"], ds["types"], nl[0], nl[1], ds["force"], a, m)
+    t_nets = time.perf_counter() - t0
+    big = sorted(blocks)[::-1][:kf_blocks]
+    st = O.FEKF(np.zeros(sum(big)), big, lam=opt.lambda0, nu=opt.nu)
+    st.P = [np.eye(n) for n in big]
+    rng = np.random.default_rng(1)
+    t0 = time.perf_counter()
+    st.update(rng.standard_normal(sum(big)), 0.1, wl.batch)
+    t_kf = time.perf_counter() - t0
+    frac = sum(n * n for n in big) / sum(n * n for n in blocks)
+    step_s = t_nets * wl.batch / n_img + 5 * t_kf / frac
+    return {"step_s": step_s, "t_nets": t_nets, "t_kf": t_kf, "cores": torch.get_num_threads(),
+            "sample": f"oracle nets (1 E + 4 F gradients) on {n_img} image(s) + oracle Kalman update on "
+                      f"{kf_blocks} of {len(blocks)} P blocks ({big[0]}^2), extrapolated to {wl.batch} images and "
+                      f"5 updates over all blocks"}
+
+
+def run_reference(args, rank, world):
+    if rank != 0:
+        return
+    wl = get_config(args.config)
+    vals = []
+    info = None
+    for k in range(args.warmup + args.steps):
+        info = oracle_sample(args.config, n_img=1, kf_blocks=1, seed=1000 + k)
+        if k >= args.warmup:
+            vals.append(wl.batch / info["step_s"])
+    v = statistics.median(vals)
+    out = {"impl": "reference", "metric": METRIC, "value": v, "unit": "images/s", "n_gpus": args.gpus,
+           "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1000.0 * wl.batch / v, "higher_is_better": True,
+           "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic (seeded LJ-labelled lattices)",
+           "config": {"workload": args.config, "images_per_step": wl.batch},
+           "cpu_baseline": {"value": v, "unit": "images/s", "cores": info["cores"], "kind": "oracle",
+                            "sample": info["sample"]},
+           "e2e": {"value": v, "unit": "images/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(out), flush=True)
+
+
+# ---------------------------------------------------------------------------------------------
+# the CUDA path
+# ---------------------------------------------------------------------------------------------
+def run_fekf(args, rank, world, local):
+    import torch
+    import torch.distributed as dist
+    import paper_conf_ppopp_huzslmlwtj24_b200 as fk
+
+    torch.cuda.set_device(local)
+    wl = get_config(args.config)
+    m, opt = wl.model, wl.opt
+    B = wl.batch
+    Bg = B * world
+    ds = make_dataset(args.config, 2 * B, seed=wl.seed + 1000 * rank)
+    na = len(ds["types"])
+    w0 = init_weights(m, 3, float(make_dataset(args.config, 4, seed=wl.seed)["energy"].mean() / na))
+    comm = fk.Comm.from_process_group() if world > 1 else None
+    ctx = fk.Context(m, opt, types=ds["types"], local_batch=B, global_batch=Bg, comm=comm)
+    ctx.set_params(torch.as_tensor(w0).cuda())
+    nsteps = args.warmup + args.steps
+    dev = lambda x, dt=torch.float64: torch.as_tensor(np.ascontiguousarray(x)).to(dt).cuda()
+    coord = [dev(ds["coord"][h * B:(h + 1) * B]) for h in range(2)]
+    box = [dev(ds["box"][h * B:(h + 1) * B]) for h in range(2)]
+    elab = [dev(ds["energy"][h * B:(h + 1) * B]) for h in range(2)]
+    flab = [dev(ds["force"][h * B:(h + 1) * B]) for h in range(2)]
+    gidx = np.stack([force_groups(na, s, wl.seed, opt.force_groups, opt.atoms_per_group) for s in range(nsteps)])
+    fidx = dev(gidx, torch.int32)
+    metrics = torch.zeros(8, dtype=torch.float64, device="cuda")
+
+    def barrier():
+        if world > 1:
+            dist.barrier()
+
+    def step(s):
+        h = s % 2
+        ctx.train_step(coord[h], box[h], elab[h], flab[h], fidx[s], metrics)
+
+    for s in range(args.warmup):
+        step(s)
+    torch.cuda.synchronize()
+    barrier()
+    clocks = Clocks(local)
+    ctx.kf.timing(True)
+    stream = torch.cuda.current_stream()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    barrier()
+    torch.cuda.synchronize()
+    e0.record(stream)
+    for s in range(args.warmup, nsteps):
+        step(s)
+    e1.record(stream)
+    torch.cuda.synchronize()
+    barrier()
+    pass_ms, pass_n = ctx.kf.timing(False)
+    clk = clocks.stop()
+    ms = e0.elapsed_time(e1)
+    launches = ctx.last_launch_count() * args.steps
+    met = metrics.cpu().numpy()
+    if world > 1:
+        t = torch.tensor([ms, pass_ms / max(pass_n, 1)], dtype=torch.float64, device="cuda")
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        ms = float(t[0])
+    value = Bg * args.steps / (ms / 1000.0)
+
+    # ---- end to end through the public API with host buffers (pinned), copies inside the timed region
+    e2e = None
+    if not args.no_e2e:
+        pin = lambda x, dt=torch.float64: torch.as_tensor(np.ascontiguousarray(x)).to(dt).pin_memory()
+        hc = [pin(ds["coord"][h * B:(h + 1) * B]) for h in range(2)]
+        hb = [pin(ds["box"][h * B:(h + 1) * B]) for h in range(2)]
+        he = [pin(ds["energy"][h * B:(h + 1) * B]) for h in range(2)]
+        hf = [pin(ds["force"][h * B:(h + 1) * B]) for h in range(2)]
+        hi = pin(gidx, torch.int32)
+        dc, db, de, df = (torch.empty_like(coord[0]), torch.empty_like(box[0]), torch.empty_like(elab[0]),
+                          torch.empty_like(flab[0]))
+        di = torch.empty_like(fidx[0])
+        hm = torch.empty(8, dtype=torch.float64).pin_memory()
+        h2d = (hc[0].numel() + hb[0].numel() + he[0].numel() + hf[0].numel()) * 8 + hi[0].numel() * 4
+        d2h = 8 * 8
+        barrier()
+        torch.cuda.synchronize()
+        t0 = torch.cuda.Event(enable_timing=True)
+        t1 = torch.cuda.Event(enable_timing=True)
+        t0.record(stream)
+        for s in range(args.warmup, nsteps):
+            h = s % 2
+            dc.copy_(hc[h], non_blocking=True)
+            db.copy_(hb[h], non_blocking=True)
+            de.copy_(he[h], non_blocking=True)
+            df.copy_(hf[h], non_blocking=True)
+            di.copy_(hi[s], non_blocking=True)
+            ctx.train_step(dc, db, de, df, di, metrics)
+            hm.copy_(metrics, non_blocking=True)
+            stream.synchronize()
+        t1.record(stream)
+        torch.cuda.synchronize()
+        barrier()
+        ems = t0.elapsed_time(t1)
+        if world > 1:
+            t = torch.tensor([ems], dtype=torch.float64, device="cuda")
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            ems = float(t[0])
+        e2e = {"value": Bg * args.steps / (ems / 1000.0), "unit": "images/s", "h2d_bytes_per_step": h2d,
+               "d2h_bytes_per_step": d2h}
+
+    # ---- roofline of the dominant kernel (the P pass), measured live in the timed region
+    info = ctx.kf.info()
+    blocks = ctx.kf.blocks
+    nt = [(n + 63) // 64 for n in blocks]
+    total_tiles = sum(x * (x + 1) // 2 for x in nt)
+    alg_bytes = 8.0 * sum(n * (n + 1) for n in blocks) * info["tiles_local"] / total_tiles  # read + write, this rank
+    avg_pass_s = (pass_ms / max(pass_n, 1)) / 1000.0
+    peak, peak_kind = load_peaks()
+    achieved = alg_bytes / avg_pass_s / 1e9 if avg_pass_s > 0 else None
+    traffic = None
+    prof = os.path.join(ROOT, "profiles", "kf_pass_traffic.json")
+    if os.path.exists(prof):
+        try:
+            with open(prof) as f:
+                pj = json.load(f)
+            if pj.get("workload") == args.config:
+                traffic = pj.get("dram_bytes_per_launch")
+        except Exception:
+            pass
+    roof = {"kernel": "kf_pass_kernel", "bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+            "frac": (achieved / peak) if achieved else None, "traffic": traffic,
+            "peak_source": peak_kind, "alg_bytes_per_launch": alg_bytes, "avg_launch_ms": avg_pass_s * 1000.0,
+            "launches_timed": pass_n, "share_of_step": (pass_ms / max(ms, 1e-9))}
+
+    out = {"metric": METRIC, "value": value, "unit": "images/s", "n_gpus": world, "steps": args.steps,
+           "warmup": args.warmup, "ms_per_step": ms / args.steps, "higher_is_better": True, "scaling": "weak",
+           "vs_baseline": None, "dtype": "f64", "data": "synthetic (seeded perturbed water-64 lattices, LJ labels)",
+           "config": {"workload": args.config, "images_per_gpu": B, "global_batch": Bg, "n_atoms": na,
+                      "n_params": ctx.n_params, "p_blocks": len(blocks), "p_bytes_per_gpu": info["p_bytes_local"],
+                      "parallelism": f"dp{world}" + (" + P sharded" if world > 1 else ""),
+                      "l2": "inputs larger than L2: P (39 GiB packed fp64) is streamed 5x per step"},
+           "roofline": roof, "e2e": e2e, "gpu_launches": int(launches), "clocks": clk,
+           "last_metrics": {"abe_e": met[0], "abe_f": list(met[1:5]), "A_last": met[5], "lambda": met[6],
+                            "flags": met[7]}}
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        cb = oracle_sample(args.config, n_img=2, kf_blocks=2)
+        out["cpu_baseline"] = {"value": wl.batch / cb["step_s"], "unit": "images/s", "cores": cb["cores"],
+                               "kind": "oracle", "sample": cb["sample"]}
+    if rank == 0:
+        print(json.dumps(out), flush=True)
+    ctx.close()
+    if comm:
+        comm.close()
+
+
+def main():
+    args = parse()
+    rank, world, local = dist_env()
+    if args.impl == "reference":
+        run_reference(args, rank, world)
+        return
+    if world > 1:
+        import torch
+        import torch.distributed as dist
+        torch.cuda.set_device(local)
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    run_fekf(args, rank, world, local)
+    if world > 1:
+        import torch.distributed as dist
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

@@ -424,6 +424,10 @@ fekf_status fekf_kf_pass(fekf_kf* k, const double* g, cudaStream_t s) {
   if (!k || !g) { set_error("kf_pass: null"); return FEKF_EINVAL; }
   return k->kf.pass(g, s);
 }
+fekf_status fekf_kf_timing(fekf_kf* k, int mode, double* total_ms, int64_t* launches) {
+  if (!k || (mode != 0 && mode != 1)) { set_error("kf_timing: bad args"); return FEKF_EINVAL; }
+  return k->kf.timing_ctl(mode, total_ms, launches);
+}
 
 // ---- context ----
 fekf_status fekf_create(const fekf_model_cfg* m, const fekf_opt_cfg* opt, int natoms, const int32_t* types_host,

@@ -526,7 +526,27 @@ fekf_status Kf::create(const std::vector<int>& blocks, const fekf_opt_cfg& o, fe
   return FEKF_OK;
 }
 
+fekf_status Kf::timing_ctl(int mode, double* total_ms, int64_t* launches) {
+  if (mode == 1) {
+    timing = true;
+    ev_used = 0;
+    return FEKF_OK;
+  }
+  timing = false;
+  double tot = 0.0;
+  for (size_t k = 0; k + 1 < ev_used; k += 2) {
+    FEKF_CHECK_CUDA(cudaEventSynchronize(ev[k + 1]));
+    float ms = 0.f;
+    FEKF_CHECK_CUDA(cudaEventElapsedTime(&ms, ev[k], ev[k + 1]));
+    tot += ms;
+  }
+  if (total_ms) *total_ms = tot;
+  if (launches) *launches = (int64_t)(ev_used / 2);
+  return FEKF_OK;
+}
+
 Kf::~Kf() {
+  for (cudaEvent_t e : ev) cudaEventDestroy(e);
   for (DBuf* b : {&P, &items_d, &ws, &gpad, &unew, &upend, &dotp, &csr_ptr, &csr_idx, &tc_blk, &tc_c, &off_d, &n_d,
                   &state, &counter})
     dfree(*b);
@@ -542,11 +562,23 @@ fekf_status Kf::pass(const double* g, cudaStream_t s) {
   if (!p.items.empty()) {
     FEKF_CHECK_CUDA(cudaMemsetAsync(counter.p, 0, sizeof(int), s));
     const int grid = std::min<int>((int)p.items.size(), num_sms());
+    if (timing) {
+      while (ev.size() < ev_used + 2) {
+        cudaEvent_t e;
+        FEKF_CHECK_CUDA(cudaEventCreate(&e));
+        ev.push_back(e);
+      }
+      FEKF_CHECK_CUDA(cudaEventRecord(ev[ev_used], s));
+    }
     kf_pass_kernel<<<grid, PASS_THREADS, PASS_SMEM, s>>>(P.as<double>(), items_d.as<ItemD>(), (int)p.items.size(),
                                                           counter.as<int>(), gpad.as<double>(), upend.as<double>(),
                                                           state.as<KfState>(), ws.as<double>());
     FEKF_LAUNCH_CHECK();
     count_launch();
+    if (timing) {
+      FEKF_CHECK_CUDA(cudaEventRecord(ev[ev_used + 1], s));
+      ev_used += 2;
+    }
   }
   kf_reduce_u_kernel<<<cdiv(p.n_tc, 4), 256, 0, s>>>(ws.as<double>(), csr_ptr.as<long long>(),
                                                       csr_idx.as<long long>(), p.n_tc, unew.as<double>());

@@ -53,6 +53,10 @@ struct Kf {
   fekf_comm* comm = nullptr;
   KfPlan plan;
   DBuf P, items_d, ws, gpad, unew, upend, dotp, csr_ptr, csr_idx, tc_blk, tc_c, off_d, n_d, state, counter;
+  bool timing = false;
+  std::vector<cudaEvent_t> ev;   // [start, stop] per timed pass launch
+  size_t ev_used = 0;
+  fekf_status timing_ctl(int mode, double* total_ms, int64_t* launches);
   fekf_status create(const std::vector<int>& blocks, const fekf_opt_cfg& o, fekf_comm* c);
   ~Kf();
   fekf_status pass(const double* g, cudaStream_t s);

@@ -62,6 +62,7 @@ def lib():
         "fekf_kf_get_state": ([vp, C.POINTER(dbl), C.POINTER(dbl), C.POINTER(i32)], i32),
         "fekf_kf_info": ([vp, C.POINTER(i64), C.POINTER(i64), C.POINTER(i64), C.POINTER(i64)], i32),
         "fekf_kf_pass": ([vp, vp, vp], i32),
+        "fekf_kf_timing": ([vp, i32, C.POINTER(dbl), C.POINTER(i64)], i32),
         "fekf_create": ([C.POINTER(ModelCfg), C.POINTER(OptCfg), i32, vp, i32, i32, vp, C.POINTER(vp)], i32),
         "fekf_destroy": ([vp], i32), "fekf_param_count": ([vp, C.POINTER(i64)], i32),
         "fekf_get_kf": ([vp, C.POINTER(vp)], i32), "fekf_set_params": ([vp, vp, vp], i32),
@@ -87,7 +88,7 @@ EXPORTED = [
     "fekf_last_error", "fekf_version", "fekf_plan_layout", "fekf_plan_shard", "fekf_get_unique_id",
     "fekf_comm_init", "fekf_comm_destroy", "fekf_comm_allreduce_sum", "fekf_kf_create", "fekf_kf_destroy",
     "fekf_kf_update", "fekf_kf_flush", "fekf_kf_get_block", "fekf_kf_set_block", "fekf_kf_get_state",
-    "fekf_kf_info", "fekf_kf_pass", "fekf_create", "fekf_destroy", "fekf_param_count", "fekf_get_kf",
+    "fekf_kf_info", "fekf_kf_pass", "fekf_kf_timing", "fekf_create", "fekf_destroy", "fekf_param_count", "fekf_get_kf",
     "fekf_set_params", "fekf_get_params", "fekf_build_nlist", "fekf_env_mat", "fekf_forward",
     "fekf_energy_jacobian", "fekf_force_jacobian", "fekf_kalman_update", "fekf_train_step",
     "fekf_last_launch_count",
@@ -259,6 +260,12 @@ class KalmanFilter:
         a, b, c, d = C.c_int64(), C.c_int64(), C.c_int64(), C.c_int64()
         _check(lib().fekf_kf_info(self.h, C.byref(a), C.byref(b), C.byref(c), C.byref(d)))
         return {"p_bytes_local": a.value, "tiles_local": b.value, "n_pad": c.value, "items_local": d.value}
+
+    def timing(self, enable):
+        """enable=True: start recording P-pass kernel times; False: stop, return (total_ms, launches)."""
+        ms, n = C.c_double(), C.c_int64()
+        _check(lib().fekf_kf_timing(self.h, 1 if enable else 0, C.byref(ms), C.byref(n)))
+        return ms.value, n.value
 
     def close(self):
         if self._own and self.h:
