@@ -216,6 +216,7 @@ fekf_status Ctx::init(const fekf_model_cfg& mm, const fekf_opt_cfg& oo, int nato
   FEKF_TRY(dalloc(etot, sizeof(double) * B));
   FEKF_TRY(dalloc(force, sizeof(double) * B * Na * 3));
   FEKF_TRY(dalloc(virial, sizeof(double) * B * 9));
+  FEKF_TRY(dalloc(vatom, sizeof(double) * B * Na * 9));
   FEKF_TRY(dalloc(abe, sizeof(double) * 2));
   FEKF_TRY(dalloc(abs_sum, sizeof(double) * 2));
   FEKF_TRY(dalloc(metrics_tmp, sizeof(double) * 64));
@@ -238,14 +239,22 @@ fekf_status Ctx::init(const fekf_model_cfg& mm, const fekf_opt_cfg& oo, int nato
       P.L = emb[ti * nt + tj];
       pairs.push_back(std::move(P));
     }
+  FEKF_TRY(dalloc(rowcnt, sizeof(int) * 2 * pairs.size()));
+  FEKF_CHECK_CUDA(cudaMemset(rowcnt.p, 0, sizeof(int) * 2 * pairs.size()));
   for (auto& P : pairs) {
-    const long long R2 = 2 * std::max<long long>(P.R, 1);
-    FEKF_TRY(dalloc(P.hin, sizeof(double) * R2));
-    FEKF_TRY(dalloc(P.sbar, sizeof(double) * R2 / 2));
-    P.Y.resize(P.L.size()); P.H.resize(P.L.size()); P.Hb.resize(P.L.size()); P.Zb.resize(P.L.size());
-    for (size_t l = 0; l < P.L.size(); ++l) {
-      const size_t n = sizeof(double) * R2 * P.L[l].dout;
-      FEKF_TRY(dalloc(P.Y[l], n)); FEKF_TRY(dalloc(P.H[l], n)); FEKF_TRY(dalloc(P.Hb[l], n)); FEKF_TRY(dalloc(P.Zb[l], n));
+    const long long R1 = std::max<long long>(P.R, 1);
+    FEKF_TRY(dalloc(P.row_idx, sizeof(int) * R1));
+    FEKF_TRY(dalloc(P.row_start, sizeof(int) * (B * atoms_of[P.ti].size() + 1)));
+    FEKF_TRY(dalloc(P.tidx, sizeof(int) * R1));
+    FEKF_TRY(dalloc(P.tpos, sizeof(int) * R1));
+    FEKF_TRY(dalloc(P.hin, sizeof(double) * R1));
+    FEKF_TRY(dalloc(P.hin_t, sizeof(double) * R1));
+    FEKF_TRY(dalloc(P.sbar, sizeof(double) * R1));
+    const size_t nl = P.L.size();
+    for (auto* v : {&P.Y, &P.H, &P.Hb, &P.Zb, &P.Yt, &P.Ht, &P.Hbt, &P.Zbt}) v->resize(nl);
+    for (size_t l = 0; l < nl; ++l) {
+      const size_t n = sizeof(double) * R1 * P.L[l].dout;
+      for (auto* v : {&P.Y, &P.H, &P.Hb, &P.Zb, &P.Yt, &P.Ht, &P.Hbt, &P.Zbt}) FEKF_TRY(dalloc((*v)[l], n));
     }
   }
   fits.clear();
@@ -287,12 +296,12 @@ Ctx::~Ctx() {
   kfo.reset();
   kf = nullptr;
   for (DBuf* b : {&types_d, &tindex_d, &atoms_d, &atoms_off_d, &sel_d, &sec_d, &err_d, &w, &gbuf, &nl_j, &nl_s,
-                  &overflow, &em, &jac, &rij, &rdot, &vdir, &X, &Xb, &eatom, &etot, &force, &virial, &splitk_ws,
-                  &colsum_ws, &abe, &metrics_tmp, &abs_sum})
+                  &overflow, &em, &jac, &rij, &rdot, &vdir, &X, &Xb, &eatom, &etot, &force, &virial, &vatom, &splitk_ws,
+                  &colsum_ws, &abe, &metrics_tmp, &abs_sum, &rowcnt})
     dfree(*b);
   for (auto& P : pairs) {
-    dfree(P.hin); dfree(P.sbar);
-    for (auto* v : {&P.Y, &P.H, &P.Hb, &P.Zb}) for (auto& b : *v) dfree(b);
+    for (DBuf* b : {&P.row_idx, &P.row_start, &P.tidx, &P.tpos, &P.hin, &P.hin_t, &P.sbar}) dfree(*b);
+    for (auto* v : {&P.Y, &P.H, &P.Hb, &P.Zb, &P.Yt, &P.Ht, &P.Hbt, &P.Zbt}) for (auto& b : *v) dfree(b);
   }
   for (auto& F : fits) {
     dfree(F.D); dfree(F.Db); dfree(F.eout); dfree(F.ebar);
@@ -319,6 +328,7 @@ static fekf_status geometry(Ctx& c, const double* coord, const double* box, int 
   FEKF_TRY(launch_nlist(c, coord, box, nb, c.nl_j.as<int>(), c.nl_s.as<int>(), c.overflow.as<int>(), s));
   FEKF_TRY(launch_envmat(c, coord, box, c.nl_j.as<int>(), c.nl_s.as<int>(), nb, c.em.as<double>(), c.jac.as<double>(),
                          c.rij.as<double>(), s));
+  FEKF_TRY(build_rows(c, nb, s));
   return FEKF_OK;
 }
 

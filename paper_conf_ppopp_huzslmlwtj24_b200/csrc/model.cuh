@@ -16,10 +16,14 @@ struct Layer {
 
 struct PairNet {       // embedding net of the type pair (ti, tj)
   int ti, tj;
-  long long R;         // rows = B * n_ti * sel_tj (padded slots included; they carry R~ = 0)
+  long long R;         // max rows = B * n_ti * sel_tj; the live count (valid slots only) is on the device
   std::vector<Layer> L;
-  DBuf hin;            // [2R]       s (primal rows) and s-dot (tangent rows)
-  std::vector<DBuf> Y, H, Hb, Zb;   // per layer [2R x d_l]
+  DBuf row_idx;        // [R]  global slot index (b*Na + i)*Nm + slot of every compacted row
+  DBuf row_start;      // [B*n_ti + 1] first row of atom (b, k)
+  DBuf tidx, tpos;     // [R]  tangent row -> primal row, primal row -> tangent row or -1
+  DBuf hin, hin_t;     // [R]  s (primal rows), s-dot (active tangent rows)
+  std::vector<DBuf> Y, H, Hb, Zb;       // primal   [R x d_l]
+  std::vector<DBuf> Yt, Ht, Hbt, Zbt;   // tangent  [R x d_l] (only the first T rows are live)
   DBuf sbar;           // [R] adjoint of s (forces)
 };
 
@@ -52,8 +56,9 @@ struct Ctx {
   DBuf w, gbuf;                                   // [Np], [Np + 1] (g || error sum, the allreduce payload)
   DBuf nl_j, nl_s, overflow, em, jac, rij, rdot, vdir;
   DBuf X, Xb;                                     // [2 * B*Na*4*M] (primal | tangent)
-  DBuf eatom, etot, force, virial;
+  DBuf eatom, etot, force, virial, vatom;
   DBuf splitk_ws, colsum_ws;
+  DBuf rowcnt;                                    // [2 * npairs] live primal / tangent rows per pair
   DBuf abe, metrics_tmp, abs_sum;
   size_t splitk_elems = 0, colsum_elems = 0;
   int64_t last_launches = 0;
@@ -78,6 +83,7 @@ fekf_status energy_error(Ctx& c, int nb, const double* e_label, double* abs_sum,
 fekf_status force_error(Ctx& c, int nb, const double* f_label, const int* atom_idx, int n_sel, double* abs_sum,
                         cudaStream_t s);
 fekf_status tangent_env(Ctx& c, int nb, cudaStream_t s);
+fekf_status build_rows(Ctx& c, int nb, cudaStream_t s);
 fekf_status seed_force(Ctx& c, int nb, cudaStream_t s);
 
 }  // namespace fekf

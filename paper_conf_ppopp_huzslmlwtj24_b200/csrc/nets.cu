@@ -5,157 +5,26 @@
 //   fitting    E_i = F3 o F2 o F1 o F0(D)    P:L95-101, residual timestep dt: reading Z14
 //   forces     F = -dE/dx via dE/dX by Eq. 4 and the R~ chain rule (Opt1)
 //   force-Jacobian: d/dw of Edot = <dE/dx, v> (forward-mode tangent along v, then reverse over the
-//     primal+tangent graph): every activation carries a tangent row stacked under its primal row
-//     ([primal rows | tangent rows]), so each weight-gradient is ONE GEMM over 2R rows.
+//     primal+tangent graph).  Each weight gradient is one split-K GEMM over primal + tangent rows.
 //
-// Row layouts (padded slots kept: their R~ rows are 0 so they add exact zeros):
-//   pair net (ti,tj): row r = (b*n_ti + k)*sel_tj + s  <->  atom atoms_of[ti][k], slot sec[tj]+s
-//   fitting net t:    row r = b*n_t + k
+// Row layouts:
+//   embedding net (ti,tj): COMPACTED rows, valid slots only (a prefix of each type section of the
+//     sorted neighbour list), ordered (b, k, s); row_start[b*n_ti + k] gives atom (b, atoms_of[ti][k]).
+//     Tangent rows (force-Jacobian) are the ACTIVE rows only (i or j among the selected atoms, where
+//     R~-dot = J (v_j - v_i) can be non-zero), kept in primal order: tidx[t] -> r, tpos[r] -> t | -1.
+//     Row counts live on the device (graph-friendly); launches are sized for the maxima.
+//   fitting net t: row r = b*n_t + k, stacked [primal rows | tangent rows] (every atom is active).
 #include <algorithm>
 
-#include "model.cuh"
+#include "gemm.cuh"
 
 namespace fekf {
 
 // =================================================================================================
-// fp64 GEMM  C = op(A) op(B)   (64x64x16 tiles, 256 threads, 4x4 register micro-tiles, smem double
-// buffering).  TA: A stored [K x M]; TB: B stored [N x K].  Optional "ones" row: op(A) row aug_m is
-// (k < aug_k ? 1 : 0) so [W-grad ; b-grad] = [H | 1]^T Zbar comes out of one GEMM.
+// weight gradients: [W-grad ; b-grad] (din+1 x dout) = [H | 1]^T Zbar + [Hdot | 0]^T Zdotbar
+// (the bias does not enter the tangent).  Two row segments (primal, tangent), split-K partials summed
+// in a fixed order -> written to g at the W offset (W then b are contiguous in the layout).
 // =================================================================================================
-constexpr int GB_M = 64, GB_N = 64, GB_K = 16;
-
-struct EpiStore {
-  double* C; int ldc;
-  __device__ void operator()(int r, int c, double v) const { C[(size_t)r * ldc + c] = v; }
-};
-struct EpiPartial {
-  double* ws; int M, N;
-  __device__ void operator()(int r, int c, double v) const { ws[((size_t)blockIdx.z * M + r) * N + c] = v; }
-};
-// forward layer: y = tanh(z + b) (primal) or ydot = (1 - y^2) zdot (tangent); h = skip(h_prev) + dt*y
-struct EpiFwd {
-  double* Y; double* H; int ld;
-  const double* bias; const double* dt;
-  const double* Hp; int ldp; int skip; int dprev;
-  const double* Yprim;  // non-null: tangent rows (Y/H point to the tangent half, Yprim to the primal)
-  __device__ void operator()(int r, int c, double v) const {
-    double sk = 0.0;
-    if (skip == 1) sk = Hp[(size_t)r * ldp + c];
-    else if (skip == 2) sk = Hp[(size_t)r * ldp + (c % dprev)];
-    double y;
-    if (Yprim == nullptr) {
-      y = tanh(v + bias[c]);
-    } else {
-      const double yp = Yprim[(size_t)r * ld + c];
-      y = (1.0 - yp * yp) * v;
-    }
-    Y[(size_t)r * ld + c] = y;
-    H[(size_t)r * ld + c] = sk + (dt ? dt[c] * y : y);
-  }
-};
-// data gradient: hbar_prev = Zbar W^T + skip^T(hbar)
-struct EpiDgrad {
-  double* out; int ldo; const double* Hb; int ld; int skip; int dprev;
-  __device__ void operator()(int r, int c, double v) const {
-    double s = 0.0;
-    if (skip == 1) s = Hb[(size_t)r * ld + c];
-    else if (skip == 2) s = Hb[(size_t)r * ld + c] + Hb[(size_t)r * ld + c + dprev];
-    out[(size_t)r * ldo + c] = v + s;
-  }
-};
-
-template <bool TA, bool TB, class Epi>
-__global__ void __launch_bounds__(256)
-dgemm_kernel(int M, int N, int K, const double* __restrict__ A, int lda, const double* __restrict__ B, int ldb,
-             int aug_m, int aug_k, int kps, Epi epi) {
-  __shared__ __align__(16) double As[2][GB_K][GB_M + 2];
-  __shared__ __align__(16) double Bs[2][GB_K][GB_N + 2];
-  const int tid = threadIdx.x;
-  const int m0 = blockIdx.x * GB_M, n0 = blockIdx.y * GB_N;
-  const int kbeg = blockIdx.z * kps;
-  const int kend = min(K, kbeg + kps);
-  const int tm = tid >> 4, tn = tid & 15;
-  double acc[4][4];
-#pragma unroll
-  for (int i = 0; i < 4; ++i)
-#pragma unroll
-    for (int j = 0; j < 4; ++j) acc[i][j] = 0.0;
-  double ra[4], rb[4];
-  auto load = [&](int k0) {
-#pragma unroll
-    for (int q = 0; q < 4; ++q) {
-      const int idx = tid + 256 * q;
-      int r, kk;
-      if (!TA) { r = idx >> 4; kk = idx & 15; } else { kk = idx >> 6; r = idx & 63; }
-      const int m = m0 + r, k = k0 + kk;
-      double v = 0.0;
-      if (m < M && k < kend) {
-        if (m == aug_m) v = (k < aug_k) ? 1.0 : 0.0;
-        else v = TA ? A[(size_t)k * lda + m] : A[(size_t)m * lda + k];
-      }
-      ra[q] = v;
-      int c;
-      if (!TB) { kk = idx >> 6; c = idx & 63; } else { c = idx >> 4; kk = idx & 15; }
-      const int n = n0 + c, k2 = k0 + kk;
-      double u = 0.0;
-      if (n < N && k2 < kend) u = TB ? B[(size_t)n * ldb + k2] : B[(size_t)k2 * ldb + n];
-      rb[q] = u;
-    }
-  };
-  auto store = [&](int buf) {
-#pragma unroll
-    for (int q = 0; q < 4; ++q) {
-      const int idx = tid + 256 * q;
-      if (!TA) As[buf][idx & 15][idx >> 4] = ra[q]; else As[buf][idx >> 6][idx & 63] = ra[q];
-      if (!TB) Bs[buf][idx >> 6][idx & 63] = rb[q]; else Bs[buf][idx & 15][idx >> 4] = rb[q];
-    }
-  };
-  const int nk = kend > kbeg ? (kend - kbeg + GB_K - 1) / GB_K : 0;
-  if (nk > 0) {
-    load(kbeg);
-    store(0);
-    __syncthreads();
-    for (int t = 0; t < nk; ++t) {
-      if (t + 1 < nk) load(kbeg + (t + 1) * GB_K);
-      const int buf = t & 1;
-#pragma unroll
-      for (int kk = 0; kk < GB_K; ++kk) {
-        const double2 a01 = *reinterpret_cast<const double2*>(&As[buf][kk][tm * 4]);
-        const double2 a23 = *reinterpret_cast<const double2*>(&As[buf][kk][tm * 4 + 2]);
-        const double2 b01 = *reinterpret_cast<const double2*>(&Bs[buf][kk][tn * 4]);
-        const double2 b23 = *reinterpret_cast<const double2*>(&Bs[buf][kk][tn * 4 + 2]);
-        const double a[4] = {a01.x, a01.y, a23.x, a23.y};
-        const double b[4] = {b01.x, b01.y, b23.x, b23.y};
-#pragma unroll
-        for (int i = 0; i < 4; ++i)
-#pragma unroll
-          for (int j = 0; j < 4; ++j) acc[i][j] = fma(a[i], b[j], acc[i][j]);
-      }
-      if (t + 1 < nk) store((t + 1) & 1);
-      __syncthreads();
-    }
-  }
-#pragma unroll
-  for (int i = 0; i < 4; ++i)
-#pragma unroll
-    for (int j = 0; j < 4; ++j) {
-      const int r = m0 + tm * 4 + i, c = n0 + tn * 4 + j;
-      if (r < M && c < N) epi(r, c, acc[i][j]);
-    }
-}
-
-template <bool TA, bool TB, class Epi>
-static fekf_status gemm(long long M, int N, int K, const double* A, int lda, const double* B, int ldb, Epi epi,
-                        cudaStream_t s, int aug_m = -1, int aug_k = 0, int splits = 1, int kps = 0) {
-  if (M <= 0 || N <= 0) return FEKF_OK;
-  if (kps <= 0) kps = K;
-  dim3 grid((unsigned)cdiv(M, GB_M), (unsigned)cdiv(N, GB_N), (unsigned)splits);
-  dgemm_kernel<TA, TB, Epi><<<grid, 256, 0, s>>>((int)M, N, K, A, lda, B, ldb, aug_m, aug_k, kps, epi);
-  FEKF_LAUNCH_CHECK();
-  count_launch();
-  return FEKF_OK;
-}
-
 __global__ void splitk_reduce_kernel(const double* __restrict__ ws, int splits, int M, int N, double* __restrict__ out) {
   const long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x;
   if (i >= (long long)M * N) return;
@@ -164,24 +33,30 @@ __global__ void splitk_reduce_kernel(const double* __restrict__ ws, int splits, 
   out[i] = a;
 }
 
-// [W-grad ; b-grad] (din+1 x dout) = [Hprev | 1]^T Zbar over `rows` rows; the ones column covers
-// the first `rows_primal` rows (the bias does not enter the tangent).  Written to g at the W offset
-// (W then b are contiguous in the layout).  Split-K partials are summed in a fixed order.
-static fekf_status wgrad(Ctx& c, int din, int dout, long long rows, long long rows_primal, const double* Hprev,
-                         const double* Zb, double* gout, cudaStream_t s) {
+struct Seg {
+  const double* H; const double* Zb; long long kmax; const int* kdev; int ones;
+};
+
+static fekf_status wgrad(Ctx& c, int din, int dout, Seg s0, Seg s1, double* gout, cudaStream_t s) {
   const int M = din + 1, N = dout;
   const long long tiles = (long long)cdiv(M, GB_M) * cdiv(N, GB_N);
-  long long splits = std::max<long long>(1, std::min<long long>(cdiv(rows, 256), cdiv(4 * 148, tiles)));
-  splits = std::min<long long>(splits, (long long)(c.splitk_elems / ((size_t)M * N)));
-  splits = std::max<long long>(1, splits);
-  int kps = (int)(cdiv(cdiv(rows, splits), GB_K) * GB_K);
-  splits = cdiv(rows, kps);
-  if (splits <= 1) {
-    return gemm<true, false>(M, N, (int)rows, Hprev, din, Zb, dout, EpiStore{gout, dout}, s, din, (int)rows_primal);
-  }
-  FEKF_TRY(gemm<true, false>(M, N, (int)rows, Hprev, din, Zb, dout, EpiPartial{c.splitk_ws.as<double>(), M, N}, s,
-                             din, (int)rows_primal, (int)splits, kps));
-  splitk_reduce_kernel<<<cdiv((long long)M * N, 256), 256, 0, s>>>(c.splitk_ws.as<double>(), (int)splits, M, N, gout);
+  const long long kmax = std::max(s0.kmax, s1.kmax);
+  const long long budget = std::max<long long>(1, (long long)(c.splitk_elems / ((size_t)M * N)));
+  long long want = std::max<long long>(1, cdiv(4 * 148, tiles));
+  int kps = (int)std::max<long long>(GB_K, cdiv(cdiv(kmax, want), GB_K) * GB_K);
+  auto nsplit = [&](const Seg& g) { return g.kmax > 0 ? (long long)cdiv(g.kmax, kps) : 0LL; };
+  while (nsplit(s0) + nsplit(s1) > budget) kps *= 2;
+  const long long S0 = nsplit(s0), S1 = nsplit(s1);
+  if (S0 + S1 == 0) return FEKF_OK;
+  if (S0 == 1 && S1 == 0)
+    return gemm<true, false>(M, N, (int)s0.kmax, s0.H, din, s0.Zb, dout, EpiStore{gout, dout}, s, nullptr, s0.kdev,
+                             din, s0.ones ? (int)s0.kmax : 0);
+  double* ws = c.splitk_ws.as<double>();
+  if (S0) FEKF_TRY(gemm<true, false>(M, N, (int)s0.kmax, s0.H, din, s0.Zb, dout, EpiPartial{ws, M, N, 0}, s, nullptr,
+                                     s0.kdev, din, s0.ones ? (int)s0.kmax : 0, (int)S0, kps));
+  if (S1) FEKF_TRY(gemm<true, false>(M, N, (int)s1.kmax, s1.H, din, s1.Zb, dout, EpiPartial{ws, M, N, (int)S0}, s,
+                                     nullptr, s1.kdev, din, s1.ones ? (int)s1.kmax : 0, (int)S1, kps));
+  splitk_reduce_kernel<<<cdiv((long long)M * N, 256), 256, 0, s>>>(ws, (int)(S0 + S1), M, N, gout);
   FEKF_LAUNCH_CHECK();
   count_launch();
   return FEKF_OK;
@@ -190,8 +65,8 @@ static fekf_status wgrad(Ctx& c, int din, int dout, long long rows, long long ro
 // =================================================================================================
 // elementwise / small kernels
 // =================================================================================================
-// zbar = (1 - y^2) ybar - 2 y ydot ydotbar  (primal rows), zdotbar = (1 - y^2) ydotbar  (tangent rows);
-// ybar = dt * hbar (residual layers with a timestep vector) else hbar.
+// fitting (stacked rows): zbar = (1 - y^2) ybar - 2 y ydot ydotbar, zdotbar = (1 - y^2) ydotbar;
+// ybar = dt * hbar on residual layers with a timestep vector, else hbar.
 __global__ void act_bwd_kernel(long long R, int d, const double* __restrict__ Y, const double* __restrict__ Hb,
                                const double* __restrict__ dt, int dual, double* __restrict__ Zb) {
   const long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x;
@@ -211,6 +86,31 @@ __global__ void act_bwd_kernel(long long R, int d, const double* __restrict__ Y,
   } else {
     Zb[i] = t * yb;
   }
+}
+
+// embedding (compacted rows; tangent rows via tpos)
+__global__ void emb_act_bwd_kernel(int Rmax, const int* __restrict__ Rdev, int d, const double* __restrict__ Y,
+                                   const double* __restrict__ Hb, const int* __restrict__ tpos,
+                                   const double* __restrict__ Yt, const double* __restrict__ Hbt, int dual,
+                                   double* __restrict__ Zb, double* __restrict__ Zbt) {
+  const long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x;
+  const long long R = min(Rmax, *Rdev);
+  if (i >= R * d) return;
+  const long long r = i / d;
+  const int c = (int)(i % d);
+  const double y = Y[i];
+  const double t = 1.0 - y * y;
+  double z = t * Hb[i];
+  if (dual) {
+    const int tr = tpos[r];
+    if (tr >= 0) {
+      const size_t j = (size_t)tr * d + c;
+      const double ydb = Hbt[j];
+      z -= 2.0 * y * Yt[j] * ydb;
+      Zbt[j] = t * ydb;
+    }
+  }
+  Zb[i] = z;
 }
 
 // dt-grad: out[c] = sum_r A[r][c] B[r][c] (two fixed-order stages)
@@ -244,6 +144,8 @@ static fekf_status colsum_prod(Ctx& c, const double* A, const double* B, long lo
   return FEKF_OK;
 }
 
+constexpr int NP = FEKF_MAX_TYPES * FEKF_MAX_TYPES;
+
 struct Geo {
   int Na, Nm, nt, M, M2, nb;
   int sec[FEKF_MAX_TYPES + 1];
@@ -255,9 +157,12 @@ struct Geo {
   const int* atoms_off;  // [nt+1]
 };
 struct PairPtrs {
-  const double* G[FEKF_MAX_TYPES * FEKF_MAX_TYPES];
-  double* Gb[FEKF_MAX_TYPES * FEKF_MAX_TYPES];
-  long long R[FEKF_MAX_TYPES * FEKF_MAX_TYPES];
+  const double* G[NP];       // primal H_last (G)
+  const double* Gt[NP];      // tangent H_last (Gdot)
+  const int* row_start[NP];
+  const int* row_idx[NP];
+  const int* tpos[NP];
+  const double* sbar[NP];
 };
 struct FitPtrs {
   double* D[FEKF_MAX_TYPES];
@@ -282,19 +187,97 @@ static long long pair_rows(Ctx& c, int p, int nb) {
   return (long long)nb * c.atoms_of[c.pairs[p].ti].size() * c.m.sel[c.pairs[p].tj];
 }
 static long long fit_rows(Ctx& c, int t, int nb) { return (long long)nb * c.atoms_of[t].size(); }
+static const int* rcount(Ctx& c, int p) { return c.rowcnt.as<int>() + p; }
+static const int* tcount(Ctx& c, int p) { return c.rowcnt.as<int>() + c.pairs.size() + p; }
 
-// embedding input s (primal rows) or s-dot (tangent rows) gathered from R~ / R~-dot column 0
-__global__ void emb_input_kernel(Geo g, int ti, int tj, long long R, const double* __restrict__ src, double* __restrict__ out) {
-  const long long r = (long long)blockIdx.x * blockDim.x + threadIdx.x;
-  if (r >= R) return;
+// ---------------------------------------------------------------------------------------------
+// compaction (one CTA per pair; fixed-order scans -> deterministic row order)
+// ---------------------------------------------------------------------------------------------
+__device__ __forceinline__ int section_count(const int* __restrict__ nl_j, size_t base, int sel) {
+  int c = 0;
+  while (c < sel && nl_j[base + c] >= 0) ++c;
+  return c;
+}
+
+__global__ void __launch_bounds__(1024)
+rows_kernel(Geo g, int ti, int tj, const int* __restrict__ nl_j, int* __restrict__ row_start,
+            int* __restrict__ row_idx, int* __restrict__ cnt) {
+  __shared__ int part[1025];
+  const int E = g.nb * g.ncnt[ti];
   const int sel = g.sel[tj];
-  const long long bk = r / sel;
-  const int s = (int)(r % sel);
-  const int b = (int)(bk / g.ncnt[ti]);
-  const int k = (int)(bk % g.ncnt[ti]);
-  const int i = g.atoms[g.atoms_off[ti] + k];
-  const size_t idx = ((size_t)b * g.Na + i) * g.Nm + g.sec[tj] + s;
-  out[r] = src[idx * 4];
+  const int per = (E + blockDim.x - 1) / blockDim.x;
+  const int e0 = min(E, (int)threadIdx.x * per), e1 = min(E, e0 + per);
+  auto base_of = [&](int e) {
+    const int b = e / g.ncnt[ti], k = e % g.ncnt[ti];
+    const int i = g.atoms[g.atoms_off[ti] + k];
+    return ((size_t)b * g.Na + i) * g.Nm + g.sec[tj];
+  };
+  int local = 0;
+  for (int e = e0; e < e1; ++e) local += section_count(nl_j, base_of(e), sel);
+  part[threadIdx.x] = local;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    int run = 0;
+    for (int t = 0; t < (int)blockDim.x; ++t) { const int v = part[t]; part[t] = run; run += v; }
+    part[blockDim.x] = run;
+  }
+  __syncthreads();
+  int r = part[threadIdx.x];
+  for (int e = e0; e < e1; ++e) {
+    const size_t base = base_of(e);
+    const int c = section_count(nl_j, base, sel);
+    row_start[e] = r;
+    for (int s = 0; s < c; ++s) row_idx[r + s] = (int)(base + s);
+    r += c;
+  }
+  if (threadIdx.x == 0) {
+    row_start[E] = part[blockDim.x];
+    *cnt = part[blockDim.x];
+  }
+}
+
+// active tangent rows: v_i != 0 or v_j != 0 (R~-dot = J (v_j - v_i) vanishes otherwise)
+__global__ void __launch_bounds__(1024)
+trows_kernel(int Na, int Nm, int Rmax, const int* __restrict__ Rdev, const int* __restrict__ row_idx,
+             const int* __restrict__ nl_j, const double* __restrict__ v, int* __restrict__ tidx,
+             int* __restrict__ tpos, int* __restrict__ cnt) {
+  __shared__ int part[1025];
+  const int R = min(Rmax, *Rdev);
+  const int per = (R + blockDim.x - 1) / blockDim.x;
+  const int r0 = min(R, (int)threadIdx.x * per), r1 = min(R, r0 + per);
+  auto active = [&](int r) {
+    const int idx = row_idx[r];
+    const int atom = idx / Nm;
+    const int b = atom / Na;
+    const int j = nl_j[idx];
+    const double* vi = v + (size_t)atom * 3;
+    const double* vj = v + ((size_t)b * Na + j) * 3;
+    return vi[0] != 0.0 || vi[1] != 0.0 || vi[2] != 0.0 || vj[0] != 0.0 || vj[1] != 0.0 || vj[2] != 0.0;
+  };
+  int local = 0;
+  for (int r = r0; r < r1; ++r) local += active(r) ? 1 : 0;
+  part[threadIdx.x] = local;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    int run = 0;
+    for (int t = 0; t < (int)blockDim.x; ++t) { const int x = part[t]; part[t] = run; run += x; }
+    part[blockDim.x] = run;
+  }
+  __syncthreads();
+  int t = part[threadIdx.x];
+  for (int r = r0; r < r1; ++r) {
+    if (active(r)) { tidx[t] = r; tpos[r] = t; ++t; } else { tpos[r] = -1; }
+  }
+  if (threadIdx.x == 0) *cnt = part[blockDim.x];
+}
+
+// embedding input s (primal rows) or s-dot (tangent rows) = column 0 of R~ / R~-dot
+__global__ void emb_input_kernel(int Rmax, const int* __restrict__ Rdev, const int* __restrict__ row_idx,
+                                 const int* __restrict__ tidx, const double* __restrict__ src, double* __restrict__ out) {
+  const int r = blockIdx.x * blockDim.x + threadIdx.x;
+  if (r >= min(Rmax, *Rdev)) return;
+  const int pr = tidx ? tidx[r] : r;
+  out[r] = src[(size_t)row_idx[pr] * 4];
 }
 
 // X = R~^T G / N_m (4 x M) per atom and D = X^T X^< (Fig. 6); tangent: Xdot = (Rdot^T G + R~^T Gdot)/N_m,
@@ -309,26 +292,28 @@ __global__ void desc_fwd_kernel(Geo g, PairPtrs pp, FitPtrs fp, const double* __
   const int atom = blockIdx.x;
   const int b = atom / g.Na, i = atom % g.Na;
   const int ti = g.types[i], k = g.tindex[i];
+  const int e = b * g.ncnt[ti] + k;
   for (int m = threadIdx.x; m < M; m += blockDim.x) {
     double a0 = 0, a1 = 0, a2 = 0, a3 = 0, d0 = 0, d1 = 0, d2 = 0, d3 = 0;
     for (int tj = 0; tj < g.nt; ++tj) {
       const int p = ti * g.nt + tj;
-      const int sel = g.sel[tj];
-      const long long base = ((long long)b * g.ncnt[ti] + k) * sel;
+      const int r0 = pp.row_start[p][e], r1 = pp.row_start[p][e + 1];
       const double* G = pp.G[p];
-      const long long R = pp.R[p];
-      for (int s = 0; s < sel; ++s) {
-        const size_t idx = ((size_t)b * g.Na + i) * g.Nm + g.sec[tj] + s;
-        const double* e = em + idx * 4;
-        const double gv = G[(size_t)(base + s) * M + m];
-        a0 = fma(e[0], gv, a0); a1 = fma(e[1], gv, a1); a2 = fma(e[2], gv, a2); a3 = fma(e[3], gv, a3);
-        if (tangent) {
+      for (int r = r0; r < r1; ++r) {
+        const size_t idx = (size_t)atom * g.Nm + g.sec[tj] + (r - r0);
+        const double* er = em + idx * 4;
+        const double gv = G[(size_t)r * M + m];
+        if (!tangent) {
+          a0 = fma(er[0], gv, a0); a1 = fma(er[1], gv, a1); a2 = fma(er[2], gv, a2); a3 = fma(er[3], gv, a3);
+        } else {
+          const int t = pp.tpos[p][r];
+          if (t < 0) continue;
           const double* ed = rdot + idx * 4;
-          const double gd = G[(size_t)(R + base + s) * M + m];
-          d0 = fma(ed[0], gv, fma(e[0], gd, d0));
-          d1 = fma(ed[1], gv, fma(e[1], gd, d1));
-          d2 = fma(ed[2], gv, fma(e[2], gd, d2));
-          d3 = fma(ed[3], gv, fma(e[3], gd, d3));
+          const double gd = pp.Gt[p][(size_t)t * M + m];
+          d0 = fma(ed[0], gv, fma(er[0], gd, d0));
+          d1 = fma(ed[1], gv, fma(er[1], gd, d1));
+          d2 = fma(ed[2], gv, fma(er[2], gd, d2));
+          d3 = fma(ed[3], gv, fma(er[3], gd, d3));
         }
       }
     }
@@ -345,15 +330,14 @@ __global__ void desc_fwd_kernel(Geo g, PairPtrs pp, FitPtrs fp, const double* __
   }
   __syncthreads();
   if (tangent) {
-    // primal X of this atom (computed by the primal pass)
     const double* xo = X + (size_t)atom * 4 * M;
-    for (int e = threadIdx.x; e < 4 * M; e += blockDim.x) xs[e] = xo[e];
+    for (int q = threadIdx.x; q < 4 * M; q += blockDim.x) xs[q] = xo[q];
     __syncthreads();
   }
   const long long row = (long long)b * g.ncnt[ti] + k;
   double* D = fp.D[ti] + (size_t)(tangent ? fp.F[ti] + row : row) * M * M2;
-  for (int e = threadIdx.x; e < M * M2; e += blockDim.x) {
-    const int m = e / M2, n = e % M2;
+  for (int q = threadIdx.x; q < M * M2; q += blockDim.x) {
+    const int m = q / M2, n = q % M2;
     double v;
     if (!tangent) {
       v = xs[m] * xs[n] + xs[M + m] * xs[M + n] + xs[2 * M + m] * xs[2 * M + n] + xs[3 * M + m] * xs[3 * M + n];
@@ -362,7 +346,7 @@ __global__ void desc_fwd_kernel(Geo g, PairPtrs pp, FitPtrs fp, const double* __
 #pragma unroll
       for (int kk = 0; kk < 4; ++kk) v += xds[kk * M + m] * xs[kk * M + n] + xs[kk * M + m] * xds[kk * M + n];
     }
-    D[e] = v;
+    D[q] = v;
   }
 }
 
@@ -411,88 +395,123 @@ __global__ void desc_bwd_kernel(Geo g, FitPtrs fp, const double* __restrict__ X,
 
 // adjoint of G (and Gdot) per embedding row from the atom's Xbar (and Xdotbar):
 //   Gbar = (R~ Xbar + Rdot Xdotbar)/N_m ; Gdotbar = R~ Xdotbar / N_m
-__global__ void emb_seed_kernel(Geo g, int ti, int tj, long long R, const double* __restrict__ em,
-                                const double* __restrict__ rdot, const double* __restrict__ Xb,
-                                const double* __restrict__ Xdb, int dual, double* __restrict__ Hb) {
+// fused with the last layer's activation adjoint (G = skip + y, no timestep):
+//   zbar = (1 - y^2) Gbar - 2 y ydot Gdotbar ; zdotbar = (1 - y^2) Gdotbar
+__global__ void emb_seed_kernel(int Rmax, const int* __restrict__ Rdev, int M, int Nm,
+                                const int* __restrict__ row_idx, const int* __restrict__ tpos,
+                                const double* __restrict__ em, const double* __restrict__ rdot,
+                                const double* __restrict__ Xb, const double* __restrict__ Xdb, int dual,
+                                const double* __restrict__ Y, const double* __restrict__ Yt, double* __restrict__ Hb,
+                                double* __restrict__ Zb, double* __restrict__ Hbt, double* __restrict__ Zbt) {
   const long long e = (long long)blockIdx.x * blockDim.x + threadIdx.x;
-  const int M = g.M;
+  const long long R = min(Rmax, *Rdev);
   if (e >= R * M) return;
   const long long r = e / M;
   const int m = (int)(e % M);
-  const int sel = g.sel[tj];
-  const long long bk = r / sel;
-  const int s = (int)(r % sel);
-  const int b = (int)(bk / g.ncnt[ti]);
-  const int k = (int)(bk % g.ncnt[ti]);
-  const int i = g.atoms[g.atoms_off[ti] + k];
-  const size_t idx = ((size_t)b * g.Na + i) * g.Nm + g.sec[tj] + s;
-  const size_t atom = (size_t)b * g.Na + i;
+  const size_t idx = (size_t)row_idx[r];
+  const size_t atom = idx / Nm;
   const double* xb = Xb + atom * 4 * M;
   const double* rr = em + idx * 4;
   double a = rr[0] * xb[m] + rr[1] * xb[M + m] + rr[2] * xb[2 * M + m] + rr[3] * xb[3 * M + m];
-  const double inv = 1.0 / g.Nm;
-  if (dual) {
+  const double inv = 1.0 / Nm;
+  const size_t o = (size_t)r * M + m;
+  const double y = Y[o];
+  const double t = 1.0 - y * y;
+  const int tr = dual ? tpos[r] : -1;
+  if (tr >= 0) {
     const double* xdb = Xdb + atom * 4 * M;
     const double* rd = rdot + idx * 4;
     a += rd[0] * xdb[m] + rd[1] * xdb[M + m] + rd[2] * xdb[2 * M + m] + rd[3] * xdb[3 * M + m];
-    const double ad = rr[0] * xdb[m] + rr[1] * xdb[M + m] + rr[2] * xdb[2 * M + m] + rr[3] * xdb[3 * M + m];
-    Hb[(size_t)(R + r) * M + m] = ad * inv;
+    const double ad = (rr[0] * xdb[m] + rr[1] * xdb[M + m] + rr[2] * xdb[2 * M + m] + rr[3] * xdb[3 * M + m]) * inv;
+    const size_t od = (size_t)tr * M + m;
+    Hbt[od] = ad;
+    Zbt[od] = t * ad;
+    a *= inv;
+    Hb[o] = a;
+    Zb[o] = t * a - 2.0 * y * Yt[od] * ad;
+  } else {
+    a *= inv;
+    Hb[o] = a;
+    Zb[o] = t * a;
   }
-  Hb[(size_t)r * M + m] = a * inv;
 }
 
 // prod_force / prod_virial: dE/dR~_row = G Xbar^T / N_m + sbar e_0 ; f = dE/dd = (dE/dR~) J ;
-// F_i += f, F_j -= f (F = -dE/dx), W -= d (x) f.  One warp per row.
-__global__ void prod_force_kernel(Geo g, int ti, int tj, long long R, const double* __restrict__ G,
-                                  const double* __restrict__ Xb, const double* __restrict__ sbar,
-                                  const double* __restrict__ jac, const double* __restrict__ rij,
-                                  const int* __restrict__ nl_j, double* __restrict__ force, double* __restrict__ virial) {
-  const long long r = ((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-  const int lane = threadIdx.x & 31;
-  if (r >= R) return;
+// F_i += f, F_j -= f (F = -dE/dx), W -= d (x) f.  One CTA (4 warps) per centre atom: the
+// atom's own force and virial are reduced in the CTA (fixed order), only F_j needs atomics.
+__global__ void __launch_bounds__(128)
+prod_force_kernel(Geo g, PairPtrs pp, const double* __restrict__ Xb, const double* __restrict__ jac,
+                  const double* __restrict__ rij, const int* __restrict__ nl_j, double* __restrict__ force,
+                  double* __restrict__ vatom) {
+  __shared__ double red[4][12];
+  const int atom = blockIdx.x;
+  const int b = atom / g.Na, i = atom % g.Na;
+  const int ti = g.types[i], k = g.tindex[i];
+  const int e = b * g.ncnt[ti] + k;
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int M = g.M;
-  const int sel = g.sel[tj];
-  const long long bk = r / sel;
-  const int s = (int)(r % sel);
-  const int b = (int)(bk / g.ncnt[ti]);
-  const int k = (int)(bk % g.ncnt[ti]);
-  const int i = g.atoms[g.atoms_off[ti] + k];
-  const size_t idx = ((size_t)b * g.Na + i) * g.Nm + g.sec[tj] + s;
-  const int j = nl_j[idx];
-  if (j < 0) return;
-  const double* xb = Xb + ((size_t)b * g.Na + i) * 4 * M;
-  const double* gr = G + (size_t)r * M;
-  double a0 = 0, a1 = 0, a2 = 0, a3 = 0;
-  for (int m = lane; m < M; m += 32) {
-    const double gv = gr[m];
-    a0 = fma(gv, xb[m], a0); a1 = fma(gv, xb[M + m], a1); a2 = fma(gv, xb[2 * M + m], a2); a3 = fma(gv, xb[3 * M + m], a3);
-  }
-  for (int o = 16; o > 0; o >>= 1) {
-    a0 += __shfl_xor_sync(0xffffffffu, a0, o);
-    a1 += __shfl_xor_sync(0xffffffffu, a1, o);
-    a2 += __shfl_xor_sync(0xffffffffu, a2, o);
-    a3 += __shfl_xor_sync(0xffffffffu, a3, o);
-  }
-  if (lane != 0) return;
+  const double* xb = Xb + (size_t)atom * 4 * M;
   const double inv = 1.0 / g.Nm;
-  const double rb[4] = {a0 * inv + sbar[r], a1 * inv, a2 * inv, a3 * inv};
-  const double* J = jac + idx * 12;
-  const double* d = rij + idx * 3;
-  double f[3];
+  double fi[3] = {0, 0, 0}, vir[9] = {0, 0, 0, 0, 0, 0, 0, 0, 0};
+  for (int slot = warp; slot < g.Nm; slot += 4) {
+    const size_t idx = (size_t)atom * g.Nm + slot;
+    const int j = nl_j[idx];
+    if (j < 0) continue;
+    int tj = 0;
+    while (slot >= g.sec[tj + 1]) ++tj;
+    const int p = ti * g.nt + tj;
+    const long long r = pp.row_start[p][e] + (slot - g.sec[tj]);
+    const double* gr = pp.G[p] + (size_t)r * M;
+    double a0 = 0, a1 = 0, a2 = 0, a3 = 0;
+    for (int m = lane; m < M; m += 32) {
+      const double gv = gr[m];
+      a0 = fma(gv, xb[m], a0); a1 = fma(gv, xb[M + m], a1); a2 = fma(gv, xb[2 * M + m], a2); a3 = fma(gv, xb[3 * M + m], a3);
+    }
+    for (int o = 16; o > 0; o >>= 1) {
+      a0 += __shfl_xor_sync(0xffffffffu, a0, o);
+      a1 += __shfl_xor_sync(0xffffffffu, a1, o);
+      a2 += __shfl_xor_sync(0xffffffffu, a2, o);
+      a3 += __shfl_xor_sync(0xffffffffu, a3, o);
+    }
+    if (lane == 0) {
+      const double rb[4] = {a0 * inv + pp.sbar[p][r], a1 * inv, a2 * inv, a3 * inv};
+      const double* J = jac + idx * 12;
+      const double* d = rij + idx * 3;
+      double f[3];
 #pragma unroll
-  for (int be = 0; be < 3; ++be) f[be] = rb[0] * J[be] + rb[1] * J[3 + be] + rb[2] * J[6 + be] + rb[3] * J[9 + be];
-  double* Fi = force + ((size_t)b * g.Na + i) * 3;
-  double* Fj = force + ((size_t)b * g.Na + j) * 3;
+      for (int be = 0; be < 3; ++be) f[be] = rb[0] * J[be] + rb[1] * J[3 + be] + rb[2] * J[6 + be] + rb[3] * J[9 + be];
+      double* Fj = force + ((size_t)b * g.Na + j) * 3;
 #pragma unroll
-  for (int be = 0; be < 3; ++be) {
-    atomicAdd(Fi + be, f[be]);
-    atomicAdd(Fj + be, -f[be]);
+      for (int be = 0; be < 3; ++be) {
+        fi[be] += f[be];
+        atomicAdd(Fj + be, -f[be]);
+      }
+#pragma unroll
+      for (int a = 0; a < 3; ++a)
+#pragma unroll
+        for (int be = 0; be < 3; ++be) vir[3 * a + be] -= d[a] * f[be];
+    }
   }
-  double* V = virial + (size_t)b * 9;
+  if (lane == 0) {
 #pragma unroll
-  for (int a = 0; a < 3; ++a)
+    for (int q = 0; q < 3; ++q) red[warp][q] = fi[q];
 #pragma unroll
-    for (int be = 0; be < 3; ++be) atomicAdd(V + 3 * a + be, -d[a] * f[be]);
+    for (int q = 0; q < 9; ++q) red[warp][3 + q] = vir[q];
+  }
+  __syncthreads();
+  if (threadIdx.x < 12) {
+    const double v = red[0][threadIdx.x] + red[1][threadIdx.x] + red[2][threadIdx.x] + red[3][threadIdx.x];
+    if (threadIdx.x < 3) atomicAdd(force + (size_t)atom * 3 + threadIdx.x, v);
+    else vatom[(size_t)atom * 9 + threadIdx.x - 3] = v;
+  }
+}
+// per-image virial = sum of the atoms' contributions in atom order (deterministic)
+__global__ void virial_reduce_kernel(const double* __restrict__ vatom, int Na, double* __restrict__ virial) {
+  const int b = blockIdx.x, q = threadIdx.x;
+  if (q >= 9) return;
+  double a = 0.0;
+  for (int i = 0; i < Na; ++i) a += vatom[((size_t)b * Na + i) * 9 + q];
+  virial[(size_t)b * 9 + q] = a;
 }
 
 // E_i = h_F W_out + b_out (primal rows), Edot_i = hdot_F W_out (tangent rows); one warp per row
@@ -564,9 +583,9 @@ __global__ void force_error_kernel(Geo g, const double* __restrict__ force, cons
         const int at = atom_idx[q];
         for (int al = 0; al < 3; ++al) {
           const size_t o = ((size_t)b * g.Na + at) * 3 + al;
-          const double fp = force[o], fl = label[o];
-          a += fabs(fl - fp);
-          v[o] += (fp >= fl ? -1.0 : 1.0);
+          const double fpred = force[o], fl = label[o];
+          a += fabs(fl - fpred);
+          v[o] += (fpred >= fl ? -1.0 : 1.0);
         }
       }
     *abs_sum = a;
@@ -595,15 +614,24 @@ __global__ void tangent_env_kernel(const double* __restrict__ jac, const int* __
   for (int k = 0; k < 4; ++k) o[k] = J[3 * k] * dd[0] + J[3 * k + 1] * dd[1] + J[3 * k + 2] * dd[2];
 }
 
+__global__ void fill_kernel(double* p, long long n, double v) {
+  const long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i < n) p[i] = v;
+}
+
 // =================================================================================================
 // host orchestration
 // =================================================================================================
-static PairPtrs make_pp(Ctx& c, int nb) {
+static PairPtrs make_pp(Ctx& c) {
   PairPtrs pp{};
   for (size_t p = 0; p < c.pairs.size(); ++p) {
-    pp.G[p] = c.pairs[p].H.back().as<double>();
-    pp.Gb[p] = c.pairs[p].Hb.back().as<double>();
-    pp.R[p] = pair_rows(c, (int)p, nb);
+    PairNet& P = c.pairs[p];
+    pp.G[p] = P.H.back().as<double>();
+    pp.Gt[p] = P.Ht.back().as<double>();
+    pp.row_start[p] = P.row_start.as<int>();
+    pp.row_idx[p] = P.row_idx.as<int>();
+    pp.tpos[p] = P.tpos.as<int>();
+    pp.sbar[p] = P.sbar.as<double>();
   }
   return pp;
 }
@@ -619,45 +647,81 @@ static FitPtrs make_fp(Ctx& c, int nb) {
   return fp;
 }
 
-static fekf_status layer_fwd(const Layer& L, const double* w, long long R, const double* Ain, const double* Hprev,
-                             double* Y, double* H, bool tangent, cudaStream_t s) {
-  // tangent: rows [R, 2R) of every stacked buffer; the primal half provides y for (1 - y^2)
-  const double* A = tangent ? Ain + (size_t)R * L.din : Ain;
+fekf_status build_rows(Ctx& c, int nb, cudaStream_t s) {
+  Geo g = make_geo(c, nb);
+  for (size_t p = 0; p < c.pairs.size(); ++p) {
+    PairNet& P = c.pairs[p];
+    rows_kernel<<<1, 1024, 0, s>>>(g, P.ti, P.tj, c.nl_j.as<int>(), P.row_start.as<int>(), P.row_idx.as<int>(),
+                                   c.rowcnt.as<int>() + p);
+    FEKF_LAUNCH_CHECK();
+    count_launch();
+  }
+  return FEKF_OK;
+}
+
+static fekf_status build_trows(Ctx& c, int nb, cudaStream_t s) {
+  for (size_t p = 0; p < c.pairs.size(); ++p) {
+    PairNet& P = c.pairs[p];
+    const long long Rmax = pair_rows(c, (int)p, nb);
+    if (Rmax == 0) continue;
+    trows_kernel<<<1, 1024, 0, s>>>(c.Na, c.Nm, (int)Rmax, rcount(c, (int)p), P.row_idx.as<int>(), c.nl_j.as<int>(),
+                                    c.vdir.as<double>(), P.tidx.as<int>(), P.tpos.as<int>(),
+                                    c.rowcnt.as<int>() + c.pairs.size() + p);
+    FEKF_LAUNCH_CHECK();
+    count_launch();
+  }
+  return FEKF_OK;
+}
+
+// one layer of the forward: primal rows (tanh(z + b)) or tangent rows ((1 - y^2) zdot)
+static fekf_status layer_fwd(const Layer& L, const double* w, long long Rmax, const int* Rdev, const double* A,
+                             const double* Hprev, double* Y, double* H, const double* Yprim, const int* rowmap,
+                             cudaStream_t s) {
   EpiFwd e;
-  e.Y = tangent ? Y + (size_t)R * L.dout : Y;
-  e.H = tangent ? H + (size_t)R * L.dout : H;
+  e.Y = Y;
+  e.H = H;
   e.ld = L.dout;
   e.bias = w + L.b;
   e.dt = L.dt >= 0 ? w + L.dt : nullptr;
-  e.Hp = Hprev ? (tangent ? Hprev + (size_t)R * L.din : Hprev) : nullptr;
+  e.Hp = Hprev;
   e.ldp = L.din;
   e.skip = Hprev ? L.skip : 0;
   e.dprev = L.din;
-  e.Yprim = tangent ? Y : nullptr;
-  return gemm<false, false>(R, L.dout, L.din, A, L.din, w + L.W, L.dout, e, s);
+  e.Yprim = Yprim;
+  e.rowmap = rowmap;
+  return gemm<false, false>(Rmax, L.dout, L.din, A, L.din, w + L.W, L.dout, e, s, Rdev);
 }
 
 fekf_status model_forward(Ctx& c, int nb, bool tangent, cudaStream_t s) {
   const double* w = c.w.as<double>();
   Geo g = make_geo(c, nb);
-  // embedding nets
+  if (tangent) FEKF_TRY(build_trows(c, nb, s));
+  // embedding nets (compacted rows)
   for (size_t p = 0; p < c.pairs.size(); ++p) {
     PairNet& P = c.pairs[p];
-    const long long R = pair_rows(c, (int)p, nb);
-    if (R == 0) continue;
-    double* hin = P.hin.as<double>();
-    emb_input_kernel<<<cdiv(R, 256), 256, 0, s>>>(g, P.ti, P.tj, R, tangent ? c.rdot.as<double>() : c.em.as<double>(),
-                                                   tangent ? hin + R : hin);
+    const long long Rmax = pair_rows(c, (int)p, nb);
+    if (Rmax == 0) continue;
+    const int* cnt = tangent ? tcount(c, (int)p) : rcount(c, (int)p);
+    double* hin = tangent ? P.hin_t.as<double>() : P.hin.as<double>();
+    emb_input_kernel<<<cdiv(Rmax, 256), 256, 0, s>>>((int)Rmax, cnt, P.row_idx.as<int>(),
+                                                     tangent ? P.tidx.as<int>() : nullptr,
+                                                     tangent ? c.rdot.as<double>() : c.em.as<double>(), hin);
     FEKF_LAUNCH_CHECK();
     count_launch();
     for (size_t l = 0; l < P.L.size(); ++l) {
-      const double* Ain = l == 0 ? hin : P.H[l - 1].as<double>();
-      const double* Hprev = l == 0 ? nullptr : P.H[l - 1].as<double>();
-      FEKF_TRY(layer_fwd(P.L[l], w, R, Ain, Hprev, P.Y[l].as<double>(), P.H[l].as<double>(), tangent, s));
+      if (!tangent) {
+        const double* A = l == 0 ? hin : P.H[l - 1].as<double>();
+        FEKF_TRY(layer_fwd(P.L[l], w, Rmax, cnt, A, l == 0 ? nullptr : P.H[l - 1].as<double>(), P.Y[l].as<double>(),
+                           P.H[l].as<double>(), nullptr, nullptr, s));
+      } else {
+        const double* A = l == 0 ? hin : P.Ht[l - 1].as<double>();
+        FEKF_TRY(layer_fwd(P.L[l], w, Rmax, cnt, A, l == 0 ? nullptr : P.Ht[l - 1].as<double>(), P.Yt[l].as<double>(),
+                           P.Ht[l].as<double>(), P.Y[l].as<double>(), P.tidx.as<int>(), s));
+      }
     }
   }
   // descriptor
-  PairPtrs pp = make_pp(c, nb);
+  PairPtrs pp = make_pp(c);
   FitPtrs fp = make_fp(c, nb);
   const size_t smem = 8 * c.M * sizeof(double);
   const size_t Xoff = (size_t)c.B * c.Na * 4 * c.M;
@@ -665,15 +729,18 @@ fekf_status model_forward(Ctx& c, int nb, bool tangent, cudaStream_t s) {
                                                c.X.as<double>(), c.X.as<double>() + Xoff);
   FEKF_LAUNCH_CHECK();
   count_launch();
-  // fitting nets
+  // fitting nets (stacked rows: the tangent half starts at row F)
   for (int t = 0; t < c.nt; ++t) {
     FitNet& Fn = c.fits[t];
     const long long F = fit_rows(c, t, nb);
     if (F == 0) continue;
     for (size_t l = 0; l < Fn.L.size(); ++l) {
+      const Layer& L = Fn.L[l];
       const double* Ain = l == 0 ? Fn.D.as<double>() : Fn.H[l - 1].as<double>();
       const double* Hprev = l == 0 ? nullptr : Fn.H[l - 1].as<double>();
-      FEKF_TRY(layer_fwd(Fn.L[l], w, F, Ain, Hprev, Fn.Y[l].as<double>(), Fn.H[l].as<double>(), tangent, s));
+      const size_t oi = tangent ? (size_t)F * L.din : 0, oo = tangent ? (size_t)F * L.dout : 0;
+      FEKF_TRY(layer_fwd(L, w, F, nullptr, Ain + oi, Hprev ? Hprev + oi : nullptr, Fn.Y[l].as<double>() + oo,
+                         Fn.H[l].as<double>() + oo, tangent ? Fn.Y[l].as<double>() : nullptr, nullptr, s));
     }
     const int h = Fn.L.back().dout;
     const double* Hl = Fn.H.back().as<double>();
@@ -703,11 +770,6 @@ fekf_status energy_error(Ctx& c, int nb, const double* e_label, double* abs_sum,
   FEKF_LAUNCH_CHECK();
   count_launch();
   return FEKF_OK;
-}
-
-__global__ void fill_kernel(double* p, long long n, double v) {
-  const long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x;
-  if (i < n) p[i] = v;
 }
 
 fekf_status seed_force(Ctx& c, int nb, cudaStream_t s) {
@@ -752,9 +814,9 @@ fekf_status model_backward(Ctx& c, int nb, Mode mode, double* gout, cudaStream_t
   const bool dual = mode == MODE_FORCE_JAC;
   const bool want_w = mode != MODE_FORCE;
   Geo g = make_geo(c, nb);
-  PairPtrs pp = make_pp(c, nb);
+  PairPtrs pp = make_pp(c);
   FitPtrs fp = make_fp(c, nb);
-  // ---- fitting nets ----
+  // ---- fitting nets (stacked rows) ----
   for (int t = 0; t < c.nt; ++t) {
     FitNet& Fn = c.fits[t];
     const long long F = fit_rows(c, t, nb);
@@ -764,7 +826,13 @@ fekf_status model_backward(Ctx& c, int nb, Mode mode, double* gout, cudaStream_t
     fit_out_bwd_kernel<<<cdiv(nF * h, 256), 256, 0, s>>>(nF, h, Fn.ebar.as<double>(), w + Fn.Wout, Fn.Hb.back().as<double>());
     FEKF_LAUNCH_CHECK();
     count_launch();
-    if (want_w) FEKF_TRY(wgrad(c, h, 1, nF, F, Fn.H.back().as<double>(), Fn.ebar.as<double>(), gout + Fn.Wout, s));
+    if (want_w) {
+      const double* Hl = Fn.H.back().as<double>();
+      const double* eb = Fn.ebar.as<double>();
+      FEKF_TRY(wgrad(c, h, 1, Seg{Hl, eb, F, nullptr, 1},
+                     Seg{dual ? Hl + (size_t)F * h : nullptr, dual ? eb + F : nullptr, dual ? F : 0, nullptr, 0},
+                     gout + Fn.Wout, s));
+    }
     for (int l = (int)Fn.L.size() - 1; l >= 0; --l) {
       const Layer& L = Fn.L[l];
       const double* dt = L.dt >= 0 ? w + L.dt : nullptr;
@@ -774,7 +842,11 @@ fekf_status model_backward(Ctx& c, int nb, Mode mode, double* gout, cudaStream_t
       count_launch();
       const double* Hprev = l == 0 ? Fn.D.as<double>() : Fn.H[l - 1].as<double>();
       if (want_w) {
-        FEKF_TRY(wgrad(c, L.din, L.dout, nF, F, Hprev, Fn.Zb[l].as<double>(), gout + L.W, s));
+        // stacked rows; the ones column covers the primal half only (bias not in the tangent)
+        FEKF_TRY(wgrad(c, L.din, L.dout, Seg{Hprev, Fn.Zb[l].as<double>(), F, nullptr, 1},
+                       Seg{dual ? Hprev + (size_t)F * L.din : nullptr, dual ? Fn.Zb[l].as<double>() + (size_t)F * L.dout : nullptr,
+                           dual ? F : 0, nullptr, 0},
+                       gout + L.W, s));
         if (L.dt >= 0) FEKF_TRY(colsum_prod(c, Fn.Y[l].as<double>(), Fn.Hb[l].as<double>(), nF, L.dout, gout + L.dt, s));
       }
       double* out = l == 0 ? Fn.Db.as<double>() : Fn.Hb[l - 1].as<double>();
@@ -789,44 +861,57 @@ fekf_status model_backward(Ctx& c, int nb, Mode mode, double* gout, cudaStream_t
                                                c.Xb.as<double>(), c.Xb.as<double>() + Xoff);
   FEKF_LAUNCH_CHECK();
   count_launch();
-  if (mode == MODE_FORCE) {
-    FEKF_CHECK_CUDA(cudaMemsetAsync(c.force.p, 0, sizeof(double) * nb * c.Na * 3, s));
-    FEKF_CHECK_CUDA(cudaMemsetAsync(c.virial.p, 0, sizeof(double) * nb * 9, s));
-  }
-  // ---- embedding nets ----
+  // ---- embedding nets (compacted rows; tangent rows separately) ----
   for (size_t p = 0; p < c.pairs.size(); ++p) {
     PairNet& P = c.pairs[p];
-    const long long R = pair_rows(c, (int)p, nb);
-    if (R == 0) continue;
-    const long long nR = dual ? 2 * R : R;
-    emb_seed_kernel<<<cdiv(R * c.M, 256), 256, 0, s>>>(g, P.ti, P.tj, R, c.em.as<double>(), c.rdot.as<double>(),
-                                                       c.Xb.as<double>(), c.Xb.as<double>() + Xoff, dual ? 1 : 0,
-                                                       P.Hb.back().as<double>());
+    const long long Rmax = pair_rows(c, (int)p, nb);
+    if (Rmax == 0) continue;
+    const int* rc = rcount(c, (int)p);
+    const int* tc = tcount(c, (int)p);
+    const int nl = (int)P.L.size();
+    emb_seed_kernel<<<cdiv(Rmax * c.M, 256), 256, 0, s>>>(
+        (int)Rmax, rc, c.M, c.Nm, P.row_idx.as<int>(), P.tpos.as<int>(), c.em.as<double>(), c.rdot.as<double>(),
+        c.Xb.as<double>(), c.Xb.as<double>() + Xoff, dual ? 1 : 0, P.Y.back().as<double>(), P.Yt.back().as<double>(),
+        P.Hb.back().as<double>(), P.Zb.back().as<double>(), P.Hbt.back().as<double>(), P.Zbt.back().as<double>());
     FEKF_LAUNCH_CHECK();
     count_launch();
-    for (int l = (int)P.L.size() - 1; l >= 0; --l) {
+    for (int l = nl - 1; l >= 0; --l) {
       const Layer& L = P.L[l];
-      act_bwd_kernel<<<cdiv(R * L.dout, 256), 256, 0, s>>>(R, L.dout, P.Y[l].as<double>(), P.Hb[l].as<double>(), nullptr,
-                                                            dual ? 1 : 0, P.Zb[l].as<double>());
-      FEKF_LAUNCH_CHECK();
-      count_launch();
-      const double* Hprev = l == 0 ? P.hin.as<double>() : P.H[l - 1].as<double>();
-      if (want_w) FEKF_TRY(wgrad(c, L.din, L.dout, nR, R, Hprev, P.Zb[l].as<double>(), gout + L.W, s));
+      if (l + 1 < nl) {  // the last layer's activation adjoint is fused into emb_seed
+        emb_act_bwd_kernel<<<cdiv(Rmax * L.dout, 256), 256, 0, s>>>(
+            (int)Rmax, rc, L.dout, P.Y[l].as<double>(), P.Hb[l].as<double>(), P.tpos.as<int>(), P.Yt[l].as<double>(),
+            P.Hbt[l].as<double>(), dual ? 1 : 0, P.Zb[l].as<double>(), P.Zbt[l].as<double>());
+        FEKF_LAUNCH_CHECK();
+        count_launch();
+      }
+      if (want_w) {
+        const double* Hp = l == 0 ? P.hin.as<double>() : P.H[l - 1].as<double>();
+        const double* Hpt = l == 0 ? P.hin_t.as<double>() : P.Ht[l - 1].as<double>();
+        FEKF_TRY(wgrad(c, L.din, L.dout, Seg{Hp, P.Zb[l].as<double>(), Rmax, rc, 1},
+                       Seg{dual ? Hpt : nullptr, dual ? P.Zbt[l].as<double>() : nullptr, dual ? Rmax : 0, tc, 0},
+                       gout + L.W, s));
+      }
       if (l > 0) {
         EpiDgrad e{P.Hb[l - 1].as<double>(), L.din, P.Hb[l].as<double>(), L.dout, L.skip, L.din};
-        FEKF_TRY(gemm<false, true>(nR, L.din, L.dout, P.Zb[l].as<double>(), L.dout, w + L.W, L.dout, e, s));
+        FEKF_TRY(gemm<false, true>(Rmax, L.din, L.dout, P.Zb[l].as<double>(), L.dout, w + L.W, L.dout, e, s, rc));
+        if (dual) {
+          EpiDgrad et{P.Hbt[l - 1].as<double>(), L.din, P.Hbt[l].as<double>(), L.dout, L.skip, L.din};
+          FEKF_TRY(gemm<false, true>(Rmax, L.din, L.dout, P.Zbt[l].as<double>(), L.dout, w + L.W, L.dout, et, s, tc));
+        }
       } else if (mode == MODE_FORCE) {
-        FEKF_TRY(gemm<false, true>(R, 1, L.dout, P.Zb[0].as<double>(), L.dout, w + L.W, L.dout,
-                                   EpiStore{P.sbar.as<double>(), 1}, s));
+        FEKF_TRY(gemm<false, true>(Rmax, 1, L.dout, P.Zb[0].as<double>(), L.dout, w + L.W, L.dout,
+                                   EpiStore{P.sbar.as<double>(), 1}, s, rc));
       }
     }
-    if (mode == MODE_FORCE) {
-      prod_force_kernel<<<cdiv(R * 32, 256), 256, 0, s>>>(g, P.ti, P.tj, R, P.H.back().as<double>(), c.Xb.as<double>(),
-                                                          P.sbar.as<double>(), c.jac.as<double>(), c.rij.as<double>(),
-                                                          c.nl_j.as<int>(), c.force.as<double>(), c.virial.as<double>());
-      FEKF_LAUNCH_CHECK();
-      count_launch();
-    }
+  }
+  if (mode == MODE_FORCE) {
+    FEKF_CHECK_CUDA(cudaMemsetAsync(c.force.p, 0, sizeof(double) * nb * c.Na * 3, s));
+    prod_force_kernel<<<nb * c.Na, 128, 0, s>>>(g, pp, c.Xb.as<double>(), c.jac.as<double>(), c.rij.as<double>(),
+                                                c.nl_j.as<int>(), c.force.as<double>(), c.vatom.as<double>());
+    FEKF_LAUNCH_CHECK();
+    virial_reduce_kernel<<<nb, 32, 0, s>>>(c.vatom.as<double>(), c.Na, c.virial.as<double>());
+    FEKF_LAUNCH_CHECK();
+    count_launch(2);
   }
   return FEKF_OK;
 }
