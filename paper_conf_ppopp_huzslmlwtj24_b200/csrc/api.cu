@@ -240,6 +240,8 @@ fekf_status Ctx::init(const fekf_model_cfg& mm, const fekf_opt_cfg& oo, int nato
       pairs.push_back(std::move(P));
     }
   FEKF_TRY(dalloc(rowcnt, sizeof(int) * 2 * pairs.size()));
+  for (auto& P : pairs) max_chunks = std::max(max_chunks, cdiv(std::max<long long>(P.R, 1), 1024));
+  FEKF_TRY(dalloc(chunks, sizeof(int) * pairs.size() * max_chunks));
   FEKF_CHECK_CUDA(cudaMemset(rowcnt.p, 0, sizeof(int) * 2 * pairs.size()));
   for (auto& P : pairs) {
     const long long R1 = std::max<long long>(P.R, 1);
@@ -297,7 +299,7 @@ Ctx::~Ctx() {
   kf = nullptr;
   for (DBuf* b : {&types_d, &tindex_d, &atoms_d, &atoms_off_d, &sel_d, &sec_d, &err_d, &w, &gbuf, &nl_j, &nl_s,
                   &overflow, &em, &jac, &rij, &rdot, &vdir, &X, &Xb, &eatom, &etot, &force, &virial, &vatom, &splitk_ws,
-                  &colsum_ws, &abe, &metrics_tmp, &abs_sum, &rowcnt})
+                  &colsum_ws, &abe, &metrics_tmp, &abs_sum, &rowcnt, &chunks})
     dfree(*b);
   for (auto& P : pairs) {
     for (DBuf* b : {&P.row_idx, &P.row_start, &P.tidx, &P.tpos, &P.hin, &P.hin_t, &P.sbar}) dfree(*b);

@@ -2,13 +2,15 @@
 // stays off tcgen05).  C = op(A) op(B) with a fused epilogue.
 //   TA: A stored [K x M] (weight gradients, K = rows); TB: B stored [N x K] (data gradients, W^T).
 //   Optional "ones" row aug_m of op(A): (k < aug_k ? 1 : 0), so [W-grad ; b-grad] = [H | 1]^T Zbar.
-//   Mdev / Kdev: device-resident row counts (compacted rows); CTAs past them exit / contribute 0.
+//   Mdev / Kdev: device-resident row counts (compacted rows); CTAs past them exit.
+// Tiles BM x BN x 16 (BM, BN in {32, 64, 128}), 256 threads, (BM/16) x (BN/16) register micro-tiles,
+// SMEM double buffering with register staging; the tile shape is picked per call from (M, N).
 #pragma once
 #include "model.cuh"
 
 namespace fekf {
 
-constexpr int GB_M = 64, GB_N = 64, GB_K = 16;
+constexpr int GB_K = 16;
 
 struct EpiStore {
   double* C; int ldc;
@@ -54,13 +56,16 @@ struct EpiDgrad {
   }
 };
 
-template <bool TA, bool TB, class Epi>
+template <int BM, int BN, bool TA, bool TB, class Epi>
 __global__ void __launch_bounds__(256)
 dgemm_kernel(int M, int N, int K, const int* __restrict__ Mdev, const int* __restrict__ Kdev,
              const double* __restrict__ A, int lda, const double* __restrict__ B, int ldb, int aug_m, int aug_k,
              int kps, Epi epi) {
-  __shared__ __align__(16) double As[2][GB_K][GB_M + 2];
-  __shared__ __align__(16) double Bs[2][GB_K][GB_N + 2];
+  constexpr int TM = BM / 16, TN = BN / 16;
+  constexpr int AE = BM * GB_K / 256, BE = BN * GB_K / 256;
+  extern __shared__ __align__(16) double gsm[];
+  auto As = reinterpret_cast<double (*)[GB_K][BM + 2]>(gsm);
+  auto Bs = reinterpret_cast<double (*)[GB_K][BN + 2]>(gsm + 2 * GB_K * (BM + 2));
   if (Mdev) M = min(M, *Mdev);
   if (Kdev) {
     const int kd = *Kdev;
@@ -68,44 +73,52 @@ dgemm_kernel(int M, int N, int K, const int* __restrict__ Mdev, const int* __res
     aug_k = min(aug_k, kd);
   }
   const int tid = threadIdx.x;
-  const int m0 = blockIdx.x * GB_M, n0 = blockIdx.y * GB_N;
-  if (m0 >= M) return;
+  const int m0 = blockIdx.x * BM, n0 = blockIdx.y * BN;
   const int kbeg = blockIdx.z * kps;
+  if (m0 >= M || (blockIdx.z > 0 && kbeg >= K)) return;  // empty split: the reduction skips it
   const int kend = min(K, kbeg + kps);
   const int tm = tid >> 4, tn = tid & 15;
-  double acc[4][4];
+  double acc[TM][TN];
 #pragma unroll
-  for (int i = 0; i < 4; ++i)
+  for (int i = 0; i < TM; ++i)
 #pragma unroll
-    for (int j = 0; j < 4; ++j) acc[i][j] = 0.0;
-  double ra[4], rb[4];
+    for (int j = 0; j < TN; ++j) acc[i][j] = 0.0;
+  double ra[AE], rb[BE];
   auto load = [&](int k0) {
 #pragma unroll
-    for (int q = 0; q < 4; ++q) {
+    for (int q = 0; q < AE; ++q) {
       const int idx = tid + 256 * q;
       int r, kk;
-      if (!TA) { r = idx >> 4; kk = idx & 15; } else { kk = idx >> 6; r = idx & 63; }
+      if (!TA) { r = idx / GB_K; kk = idx % GB_K; } else { kk = idx / BM; r = idx % BM; }
       const int m = m0 + r, k = k0 + kk;
       double v = 0.0;
       if (m < M && k < kend) {
         if (m == aug_m) v = (k < aug_k) ? 1.0 : 0.0;
-        else v = TA ? A[(size_t)k * lda + m] : A[(size_t)m * lda + k];
+        else v = TA ? __ldg(A + (size_t)k * lda + m) : __ldg(A + (size_t)m * lda + k);
       }
       ra[q] = v;
-      int c;
-      if (!TB) { kk = idx >> 6; c = idx & 63; } else { c = idx >> 4; kk = idx & 15; }
-      const int n = n0 + c, k2 = k0 + kk;
+    }
+#pragma unroll
+    for (int q = 0; q < BE; ++q) {
+      const int idx = tid + 256 * q;
+      int c, kk;
+      if (!TB) { kk = idx / BN; c = idx % BN; } else { c = idx / GB_K; kk = idx % GB_K; }
+      const int n = n0 + c, k = k0 + kk;
       double u = 0.0;
-      if (n < N && k2 < kend) u = TB ? B[(size_t)n * ldb + k2] : B[(size_t)k2 * ldb + n];
+      if (n < N && k < kend) u = TB ? __ldg(B + (size_t)n * ldb + k) : __ldg(B + (size_t)k * ldb + n);
       rb[q] = u;
     }
   };
   auto store = [&](int buf) {
 #pragma unroll
-    for (int q = 0; q < 4; ++q) {
+    for (int q = 0; q < AE; ++q) {
       const int idx = tid + 256 * q;
-      if (!TA) As[buf][idx & 15][idx >> 4] = ra[q]; else As[buf][idx >> 6][idx & 63] = ra[q];
-      if (!TB) Bs[buf][idx >> 6][idx & 63] = rb[q]; else Bs[buf][idx & 15][idx >> 4] = rb[q];
+      if (!TA) As[buf][idx % GB_K][idx / GB_K] = ra[q]; else As[buf][idx / BM][idx % BM] = ra[q];
+    }
+#pragma unroll
+    for (int q = 0; q < BE; ++q) {
+      const int idx = tid + 256 * q;
+      if (!TB) Bs[buf][idx / BN][idx % BN] = rb[q]; else Bs[buf][idx % GB_K][idx / GB_K] = rb[q];
     }
   };
   const int nk = kend > kbeg ? (kend - kbeg + GB_K - 1) / GB_K : 0;
@@ -118,41 +131,68 @@ dgemm_kernel(int M, int N, int K, const int* __restrict__ Mdev, const int* __res
       const int buf = t & 1;
 #pragma unroll
       for (int kk = 0; kk < GB_K; ++kk) {
-        const double2 a01 = *reinterpret_cast<const double2*>(&As[buf][kk][tm * 4]);
-        const double2 a23 = *reinterpret_cast<const double2*>(&As[buf][kk][tm * 4 + 2]);
-        const double2 b01 = *reinterpret_cast<const double2*>(&Bs[buf][kk][tn * 4]);
-        const double2 b23 = *reinterpret_cast<const double2*>(&Bs[buf][kk][tn * 4 + 2]);
-        const double a[4] = {a01.x, a01.y, a23.x, a23.y};
-        const double b[4] = {b01.x, b01.y, b23.x, b23.y};
+        double a[TM], b[TN];
 #pragma unroll
-        for (int i = 0; i < 4; ++i)
+        for (int i = 0; i < TM; i += 2) {
+          const double2 v = *reinterpret_cast<const double2*>(&As[buf][kk][tm * TM + i]);
+          a[i] = v.x; a[i + 1] = v.y;
+        }
 #pragma unroll
-          for (int j = 0; j < 4; ++j) acc[i][j] = fma(a[i], b[j], acc[i][j]);
+        for (int j = 0; j < TN; j += 2) {
+          const double2 v = *reinterpret_cast<const double2*>(&Bs[buf][kk][tn * TN + j]);
+          b[j] = v.x; b[j + 1] = v.y;
+        }
+#pragma unroll
+        for (int i = 0; i < TM; ++i)
+#pragma unroll
+          for (int j = 0; j < TN; ++j) acc[i][j] = fma(a[i], b[j], acc[i][j]);
       }
       if (t + 1 < nk) store((t + 1) & 1);
       __syncthreads();
     }
   }
 #pragma unroll
-  for (int i = 0; i < 4; ++i)
+  for (int i = 0; i < TM; ++i)
 #pragma unroll
-    for (int j = 0; j < 4; ++j) {
-      const int r = m0 + tm * 4 + i, c = n0 + tn * 4 + j;
+    for (int j = 0; j < TN; ++j) {
+      const int r = m0 + tm * TM + i, c = n0 + tn * TN + j;
       if (r < M && c < N) epi(r, c, acc[i][j]);
     }
 }
 
+template <int BM, int BN, bool TA, bool TB, class Epi>
+static fekf_status gemm_t(long long M, int N, int K, const double* A, int lda, const double* B, int ldb, Epi epi,
+                          cudaStream_t s, const int* Mdev, const int* Kdev, int aug_m, int aug_k, int splits, int kps) {
+  constexpr size_t smem = sizeof(double) * 2 * GB_K * ((BM + 2) + (BN + 2));
+  static bool attr = false;
+  if (!attr) {
+    FEKF_CHECK_CUDA(cudaFuncSetAttribute(dgemm_kernel<BM, BN, TA, TB, Epi>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                         (int)smem));
+    attr = true;
+  }
+  dim3 grid((unsigned)cdiv(M, BM), (unsigned)cdiv(N, BN), (unsigned)splits);
+  dgemm_kernel<BM, BN, TA, TB, Epi><<<grid, 256, smem, s>>>((int)M, N, K, Mdev, Kdev, A, lda, B, ldb, aug_m, aug_k, kps, epi);
+  FEKF_LAUNCH_CHECK();
+  count_launch();
+  return FEKF_OK;
+}
+
+// Tile choice: BN = 32 for N <= 32 (embedding widths 25/32), 128 for N >= 200 (fitting 240,
+// fitting W0 data-gradient 1600), else 64; BM = 128 when there are many rows, 64 otherwise.
 template <bool TA, bool TB, class Epi>
 static fekf_status gemm(long long M, int N, int K, const double* A, int lda, const double* B, int ldb, Epi epi,
                         cudaStream_t s, const int* Mdev = nullptr, const int* Kdev = nullptr, int aug_m = -1,
                         int aug_k = 0, int splits = 1, int kps = 0) {
   if (M <= 0 || N <= 0) return FEKF_OK;
   if (kps <= 0) kps = K;
-  dim3 grid((unsigned)cdiv(M, GB_M), (unsigned)cdiv(N, GB_N), (unsigned)splits);
-  dgemm_kernel<TA, TB, Epi><<<grid, 256, 0, s>>>((int)M, N, K, Mdev, Kdev, A, lda, B, ldb, aug_m, aug_k, kps, epi);
-  FEKF_LAUNCH_CHECK();
-  count_launch();
-  return FEKF_OK;
+  const bool tallM = M >= 4096;
+  if (N <= 32)
+    return tallM ? gemm_t<128, 32, TA, TB>(M, N, K, A, lda, B, ldb, epi, s, Mdev, Kdev, aug_m, aug_k, splits, kps)
+                 : gemm_t<64, 32, TA, TB>(M, N, K, A, lda, B, ldb, epi, s, Mdev, Kdev, aug_m, aug_k, splits, kps);
+  if (N >= 200 && tallM)
+    return gemm_t<64, 128, TA, TB>(M, N, K, A, lda, B, ldb, epi, s, Mdev, Kdev, aug_m, aug_k, splits, kps);
+  return tallM ? gemm_t<128, 64, TA, TB>(M, N, K, A, lda, B, ldb, epi, s, Mdev, Kdev, aug_m, aug_k, splits, kps)
+               : gemm_t<64, 64, TA, TB>(M, N, K, A, lda, B, ldb, epi, s, Mdev, Kdev, aug_m, aug_k, splits, kps);
 }
 
 }  // namespace fekf

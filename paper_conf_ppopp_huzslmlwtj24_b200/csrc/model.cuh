@@ -59,6 +59,8 @@ struct Ctx {
   DBuf eatom, etot, force, virial, vatom;
   DBuf splitk_ws, colsum_ws;
   DBuf rowcnt;                                    // [2 * npairs] live primal / tangent rows per pair
+  DBuf chunks;                                    // [npairs * max_chunks] tangent-row scan workspace
+  int max_chunks = 1;
   DBuf abe, metrics_tmp, abs_sum;
   size_t splitk_elems = 0, colsum_elems = 0;
   int64_t last_launches = 0;

@@ -25,12 +25,32 @@ namespace fekf {
 // (the bias does not enter the tangent).  Two row segments (primal, tangent), split-K partials summed
 // in a fixed order -> written to g at the W offset (W then b are contiguous in the layout).
 // =================================================================================================
-__global__ void splitk_reduce_kernel(const double* __restrict__ ws, int splits, int M, int N, double* __restrict__ out) {
-  const long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x;
-  if (i >= (long long)M * N) return;
+// Sum the live split-K partials in a fixed order: splits [0, S0eff) of segment 0 and
+// [S0max, S0max + S1eff) of segment 1, where S*eff follow the device row counts (empty splits never
+// wrote).  32 outputs x 8 split-lanes per CTA, fixed 8-way combine -> deterministic.
+__global__ void splitk_reduce_kernel(const double* __restrict__ ws, int S0max, int S1max, int kps,
+                                     const int* __restrict__ K0dev, const int* __restrict__ K1dev, int M, int N,
+                                     double* __restrict__ out) {
+  __shared__ double red[8][32];
+  const int lane = threadIdx.x & 31, zl = threadIdx.x >> 5;
+  const long long i = (long long)blockIdx.x * 32 + lane;
+  const long long MN = (long long)M * N;
+  int S0 = S0max, S1 = S1max;
+  if (K0dev) S0 = min(S0max, max(1, (*K0dev + kps - 1) / kps));
+  if (K1dev && S1max > 0) S1 = min(S1max, max(1, (*K1dev + kps - 1) / kps));
   double a = 0.0;
-  for (int z = 0; z < splits; ++z) a += ws[(size_t)z * M * N + i];
-  out[i] = a;
+  if (i < MN) {
+    for (int z = zl; z < S0; z += 8) a += ws[(size_t)z * MN + i];
+    for (int z = zl; z < S1; z += 8) a += ws[(size_t)(S0max + z) * MN + i];
+  }
+  red[zl][lane] = a;
+  __syncthreads();
+  if (zl == 0 && i < MN) {
+    double t = red[0][lane];
+#pragma unroll
+    for (int q = 1; q < 8; ++q) t += red[q][lane];
+    out[i] = t;
+  }
 }
 
 struct Seg {
@@ -39,11 +59,11 @@ struct Seg {
 
 static fekf_status wgrad(Ctx& c, int din, int dout, Seg s0, Seg s1, double* gout, cudaStream_t s) {
   const int M = din + 1, N = dout;
-  const long long tiles = (long long)cdiv(M, GB_M) * cdiv(N, GB_N);
+  const long long tiles = (long long)cdiv(M, 64) * cdiv(N, 64);
   const long long kmax = std::max(s0.kmax, s1.kmax);
   const long long budget = std::max<long long>(1, (long long)(c.splitk_elems / ((size_t)M * N)));
-  long long want = std::max<long long>(1, cdiv(4 * 148, tiles));
-  int kps = (int)std::max<long long>(GB_K, cdiv(cdiv(kmax, want), GB_K) * GB_K);
+  long long want = std::max<long long>(1, cdiv(2 * 148, tiles));
+  int kps = (int)std::max<long long>(4 * GB_K, cdiv(cdiv(kmax, want), GB_K) * GB_K);
   auto nsplit = [&](const Seg& g) { return g.kmax > 0 ? (long long)cdiv(g.kmax, kps) : 0LL; };
   while (nsplit(s0) + nsplit(s1) > budget) kps *= 2;
   const long long S0 = nsplit(s0), S1 = nsplit(s1);
@@ -56,7 +76,8 @@ static fekf_status wgrad(Ctx& c, int din, int dout, Seg s0, Seg s1, double* gout
                                      s0.kdev, din, s0.ones ? (int)s0.kmax : 0, (int)S0, kps));
   if (S1) FEKF_TRY(gemm<true, false>(M, N, (int)s1.kmax, s1.H, din, s1.Zb, dout, EpiPartial{ws, M, N, (int)S0}, s,
                                      nullptr, s1.kdev, din, s1.ones ? (int)s1.kmax : 0, (int)S1, kps));
-  splitk_reduce_kernel<<<cdiv((long long)M * N, 256), 256, 0, s>>>(ws, (int)(S0 + S1), M, N, gout);
+  splitk_reduce_kernel<<<cdiv((long long)M * N, 32), 256, 0, s>>>(ws, (int)S0, (int)S1, kps, s0.kdev, s1.kdev, M, N,
+                                                                  gout);
   FEKF_LAUNCH_CHECK();
   count_launch();
   return FEKF_OK;
@@ -236,39 +257,61 @@ rows_kernel(Geo g, int ti, int tj, const int* __restrict__ nl_j, int* __restrict
   }
 }
 
-// active tangent rows: v_i != 0 or v_j != 0 (R~-dot = J (v_j - v_i) vanishes otherwise)
-__global__ void __launch_bounds__(1024)
-trows_kernel(int Na, int Nm, int Rmax, const int* __restrict__ Rdev, const int* __restrict__ row_idx,
-             const int* __restrict__ nl_j, const double* __restrict__ v, int* __restrict__ tidx,
-             int* __restrict__ tpos, int* __restrict__ cnt) {
-  __shared__ int part[1025];
+// active tangent rows: v_i != 0 or v_j != 0 (R~-dot = J (v_j - v_i) vanishes otherwise).
+// Three passes (chunk counts, chunk scan, scatter), chunks of 1024 rows, order = primal order.
+constexpr int TCHUNK = 1024;
+__device__ __forceinline__ bool row_active(int r, int Na, int Nm, const int* __restrict__ row_idx,
+                                           const int* __restrict__ nl_j, const double* __restrict__ v) {
+  const int idx = row_idx[r];
+  const int atom = idx / Nm;
+  const int b = atom / Na;
+  const int j = nl_j[idx];
+  const double* vi = v + (size_t)atom * 3;
+  const double* vj = v + ((size_t)b * Na + j) * 3;
+  return vi[0] != 0.0 || vi[1] != 0.0 || vi[2] != 0.0 || vj[0] != 0.0 || vj[1] != 0.0 || vj[2] != 0.0;
+}
+__global__ void __launch_bounds__(TCHUNK)
+tcount_kernel(int Na, int Nm, int Rmax, const int* __restrict__ Rdev, const int* __restrict__ row_idx,
+              const int* __restrict__ nl_j, const double* __restrict__ v, int* __restrict__ chunk_cnt) {
   const int R = min(Rmax, *Rdev);
-  const int per = (R + blockDim.x - 1) / blockDim.x;
-  const int r0 = min(R, (int)threadIdx.x * per), r1 = min(R, r0 + per);
-  auto active = [&](int r) {
-    const int idx = row_idx[r];
-    const int atom = idx / Nm;
-    const int b = atom / Na;
-    const int j = nl_j[idx];
-    const double* vi = v + (size_t)atom * 3;
-    const double* vj = v + ((size_t)b * Na + j) * 3;
-    return vi[0] != 0.0 || vi[1] != 0.0 || vi[2] != 0.0 || vj[0] != 0.0 || vj[1] != 0.0 || vj[2] != 0.0;
-  };
-  int local = 0;
-  for (int r = r0; r < r1; ++r) local += active(r) ? 1 : 0;
-  part[threadIdx.x] = local;
+  const int r = blockIdx.x * TCHUNK + threadIdx.x;
+  const bool a = r < R && row_active(r, Na, Nm, row_idx, nl_j, v);
+  const int n = __syncthreads_count(a);
+  if (threadIdx.x == 0) chunk_cnt[blockIdx.x] = n;
+}
+__global__ void tscan_kernel(int* __restrict__ chunk_cnt, int nchunk, int* __restrict__ cnt) {
+  if (threadIdx.x == 0) {
+    int run = 0;
+    for (int k = 0; k < nchunk; ++k) { const int x = chunk_cnt[k]; chunk_cnt[k] = run; run += x; }
+    *cnt = run;
+  }
+}
+__global__ void __launch_bounds__(TCHUNK)
+tscatter_kernel(int Na, int Nm, int Rmax, const int* __restrict__ Rdev, const int* __restrict__ row_idx,
+                const int* __restrict__ nl_j, const double* __restrict__ v, const int* __restrict__ chunk_off,
+                int* __restrict__ tidx, int* __restrict__ tpos) {
+  __shared__ int wsum[TCHUNK / 32];
+  const int R = min(Rmax, *Rdev);
+  const int r = blockIdx.x * TCHUNK + threadIdx.x;
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const bool a = r < R && row_active(r, Na, Nm, row_idx, nl_j, v);
+  const unsigned bal = __ballot_sync(0xffffffffu, a);
+  if (lane == 0) wsum[warp] = __popc(bal);
   __syncthreads();
   if (threadIdx.x == 0) {
     int run = 0;
-    for (int t = 0; t < (int)blockDim.x; ++t) { const int x = part[t]; part[t] = run; run += x; }
-    part[blockDim.x] = run;
+    for (int w = 0; w < TCHUNK / 32; ++w) { const int x = wsum[w]; wsum[w] = run; run += x; }
   }
   __syncthreads();
-  int t = part[threadIdx.x];
-  for (int r = r0; r < r1; ++r) {
-    if (active(r)) { tidx[t] = r; tpos[r] = t; ++t; } else { tpos[r] = -1; }
+  if (r < R) {
+    if (a) {
+      const int t = chunk_off[blockIdx.x] + wsum[warp] + __popc(bal & ((1u << lane) - 1u));
+      tidx[t] = r;
+      tpos[r] = t;
+    } else {
+      tpos[r] = -1;
+    }
   }
-  if (threadIdx.x == 0) *cnt = part[blockDim.x];
 }
 
 // embedding input s (primal rows) or s-dot (tangent rows) = column 0 of R~ / R~-dot
@@ -278,6 +321,28 @@ __global__ void emb_input_kernel(int Rmax, const int* __restrict__ Rdev, const i
   if (r >= min(Rmax, *Rdev)) return;
   const int pr = tidx ? tidx[r] : r;
   out[r] = src[(size_t)row_idx[pr] * 4];
+}
+
+// embedding layer 0 (input width 1): y = tanh(s W0 + b0), h = y;  tangent: ydot = (1 - y^2) sdot W0
+__global__ void emb_l0_kernel(int Rmax, const int* __restrict__ Rdev, int d, const double* __restrict__ s,
+                              const double* __restrict__ W, const double* __restrict__ bias,
+                              const double* __restrict__ Yprim, const int* __restrict__ rowmap, double* __restrict__ Y,
+                              double* __restrict__ H) {
+  const long long e = (long long)blockIdx.x * blockDim.x + threadIdx.x;
+  const long long R = min(Rmax, *Rdev);
+  if (e >= R * d) return;
+  const long long r = e / d;
+  const int c = (int)(e % d);
+  const double z = s[r] * W[c];
+  double y;
+  if (Yprim == nullptr) {
+    y = tanh(z + bias[c]);
+  } else {
+    const double yp = Yprim[(size_t)rowmap[r] * d + c];
+    y = (1.0 - yp * yp) * z;
+  }
+  Y[e] = y;
+  H[e] = y;
 }
 
 // X = R~^T G / N_m (4 x M) per atom and D = X^T X^< (Fig. 6); tangent: Xdot = (Rdot^T G + R~^T Gdot)/N_m,
@@ -664,11 +729,18 @@ static fekf_status build_trows(Ctx& c, int nb, cudaStream_t s) {
     PairNet& P = c.pairs[p];
     const long long Rmax = pair_rows(c, (int)p, nb);
     if (Rmax == 0) continue;
-    trows_kernel<<<1, 1024, 0, s>>>(c.Na, c.Nm, (int)Rmax, rcount(c, (int)p), P.row_idx.as<int>(), c.nl_j.as<int>(),
-                                    c.vdir.as<double>(), P.tidx.as<int>(), P.tpos.as<int>(),
-                                    c.rowcnt.as<int>() + c.pairs.size() + p);
+    const int nchunk = cdiv(Rmax, TCHUNK);
+    int* ck = c.chunks.as<int>() + p * c.max_chunks;
+    tcount_kernel<<<nchunk, TCHUNK, 0, s>>>(c.Na, c.Nm, (int)Rmax, rcount(c, (int)p), P.row_idx.as<int>(),
+                                            c.nl_j.as<int>(), c.vdir.as<double>(), ck);
     FEKF_LAUNCH_CHECK();
-    count_launch();
+    tscan_kernel<<<1, 32, 0, s>>>(ck, nchunk, c.rowcnt.as<int>() + c.pairs.size() + p);
+    FEKF_LAUNCH_CHECK();
+    tscatter_kernel<<<nchunk, TCHUNK, 0, s>>>(c.Na, c.Nm, (int)Rmax, rcount(c, (int)p), P.row_idx.as<int>(),
+                                              c.nl_j.as<int>(), c.vdir.as<double>(), ck, P.tidx.as<int>(),
+                                              P.tpos.as<int>());
+    FEKF_LAUNCH_CHECK();
+    count_launch(3);
   }
   return FEKF_OK;
 }
@@ -709,6 +781,16 @@ fekf_status model_forward(Ctx& c, int nb, bool tangent, cudaStream_t s) {
     FEKF_LAUNCH_CHECK();
     count_launch();
     for (size_t l = 0; l < P.L.size(); ++l) {
+      if (l == 0 && P.L[0].din == 1) {
+        const Layer& L = P.L[0];
+        emb_l0_kernel<<<cdiv(Rmax * L.dout, 256), 256, 0, s>>>(
+            (int)Rmax, cnt, L.dout, hin, w + L.W, w + L.b, tangent ? P.Y[0].as<double>() : nullptr,
+            tangent ? P.tidx.as<int>() : nullptr, tangent ? P.Yt[0].as<double>() : P.Y[0].as<double>(),
+            tangent ? P.Ht[0].as<double>() : P.H[0].as<double>());
+        FEKF_LAUNCH_CHECK();
+        count_launch();
+        continue;
+      }
       if (!tangent) {
         const double* A = l == 0 ? hin : P.H[l - 1].as<double>();
         FEKF_TRY(layer_fwd(P.L[l], w, Rmax, cnt, A, l == 0 ? nullptr : P.H[l - 1].as<double>(), P.Y[l].as<double>(),
