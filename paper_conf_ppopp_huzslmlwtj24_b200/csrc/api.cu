@@ -434,7 +434,7 @@ fekf_status fekf_kf_info(const fekf_kf* k, int64_t* pb, int64_t* tl, int64_t* np
 }
 fekf_status fekf_kf_pass(fekf_kf* k, const double* g, cudaStream_t s) {
   if (!k || !g) { set_error("kf_pass: null"); return FEKF_EINVAL; }
-  return k->kf.pass(g, s);
+  return k->kf.pass(g, false, s);
 }
 fekf_status fekf_kf_timing(fekf_kf* k, int mode, double* total_ms, int64_t* launches) {
   if (!k || (mode != 0 && mode != 1)) { set_error("kf_timing: bad args"); return FEKF_EINVAL; }

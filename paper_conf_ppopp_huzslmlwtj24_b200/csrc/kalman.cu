@@ -4,15 +4,18 @@
 // upper-triangle tiles (diagonal tiles full), each tile 64x64 row-major and contiguous (32 KiB).
 // Symmetrisation (Alg. 1 line 11) is therefore exact by construction.
 //
-// One update streams the local P exactly once (kf_pass_kernel):
-//   P_IJ <- (P_IJ - A' u'_I u'_J^T) / lambda'      (pending rank-1 of the previous update, line 10)
-//   u_I  += P_IJ g_J ;  u_J += P_IJ^T g_I          (Pg, cached for A, K and the next pass: P:L283)
-// Tiles are moved HBM <-> SMEM with 1-D TMA bulk copies (cp.async.bulk + mbarrier), a producer warp
-// keeps up to STAGES tiles in flight, 8 consumer warps update in SMEM and a bulk store writes back.
+// Deferred corrections (a generalisation of the paper's Pg caching): the stored "base"
+// B and the covariance are related by P_t = sigma (B - sum_k beta_k u_k u_k^T), k over at most `defer`
+// deferred rank-1 terms (u_k = P_k g_k, beta_k = A_k / sigma_k).  One update streams the local P once:
+//   - read-only pass while fewer than `defer` corrections are pending:  u_B = B g, then
+//     u_t = P_t g = sigma (u_B - sum_k beta_k (u_k . g) u_k) in vector form;
+//   - read-write pass otherwise: B <- sigma (B - sum_k beta_k u_k u_k^T) tile by tile in SMEM, written
+//     back, and u_B = B_new g in the same pass.
+// With defer = 5 a minibatch (5 updates) costs 1 read-write + 4 read-only passes instead of 5
+// read-write passes.  Tiles move HBM <-> SMEM with 1-D TMA bulk copies (cp.async.bulk + mbarrier), a
+// producer warp keeps STAGES tiles in flight, 8 consumer warps work in SMEM, a bulk store writes back.
 // Partial u's go to a workspace slot per (item row) / (tile column) and are summed in a fixed order
 // (kf_reduce_u) — no floating-point atomics, bit-reproducible.
-// Then A = 1/(c + g^T u) with c = L*lambda (reading Z1) or lambda, w += sqrt(bs)*ABE*A*u, and the
-// update (A, u, lambda) becomes the pending correction of the next pass.
 #include <algorithm>
 #include <cmath>
 #include <numeric>
@@ -172,24 +175,30 @@ __device__ __forceinline__ void consumer_bar() { asm volatile("bar.sync 1, 256;"
 // ------------------------------------------------------------------------------------------------
 // the P pass
 // ------------------------------------------------------------------------------------------------
-constexpr int STAGES = 6;
+constexpr int STAGES = 5;
 constexpr int TILE_ELEMS = KT * KT;
 constexpr uint32_t TILE_BYTES = TILE_ELEMS * sizeof(double);
+constexpr int VEC_ELEMS = 2 * KMAX * KT;   // per stage: u_k[I-rows] and u_k[J-cols] for k < K
+constexpr int STAGE_ELEMS = TILE_ELEMS + VEC_ELEMS;
 constexpr int PASS_THREADS = 288;  // 8 consumer warps + 1 producer warp
-constexpr size_t PASS_SMEM = STAGES * TILE_BYTES + 2 * 8 * KT * sizeof(double) +
+constexpr size_t PASS_SMEM = (size_t)STAGES * STAGE_ELEMS * sizeof(double) + 2 * 8 * KT * sizeof(double) +
                              2 * STAGES * sizeof(uint64_t) + STAGES * sizeof(int4);
 
+// rw = 0: read-only pass, u_B = B g.  rw = 1: B <- sigma (B - sum_{k<K} beta_k u_k u_k^T) written back,
+// then u_B = B_new g.  Tile-row segments are pulled from an atomic counter by a producer warp that
+// streams each 32 KiB tile (and, for rw, the 2K 512-byte vector segments it needs) with TMA bulk copies.
 __global__ void __launch_bounds__(PASS_THREADS, 1)
 kf_pass_kernel(double* __restrict__ P, const ItemD* __restrict__ items, int n_items, int* counter,
-               const double* __restrict__ gpad, const double* __restrict__ upend, const KfState* st,
-               double* __restrict__ ws) {
+               const double* __restrict__ gpad, const double* __restrict__ ulist, long long npad, int rw, int K,
+               const KfState* st, double* __restrict__ ws) {
   extern __shared__ __align__(128) unsigned char smem[];
-  double* tiles = reinterpret_cast<double*>(smem);
-  double* colred = tiles + STAGES * TILE_ELEMS;
+  double* stages = reinterpret_cast<double*>(smem);
+  double* colred = stages + STAGES * STAGE_ELEMS;
   uint64_t* full = reinterpret_cast<uint64_t*>(colred + 2 * 8 * KT);
   uint64_t* empty = full + STAGES;
   int4* meta = reinterpret_cast<int4*>(empty + STAGES);
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+  if (!rw) K = 0;
 
   if (tid == 0) {
     for (int s = 0; s < STAGES; ++s) {
@@ -205,6 +214,7 @@ kf_pass_kernel(double* __restrict__ P, const ItemD* __restrict__ items, int n_it
     if (lane == 0) {
       int s = 0;
       uint32_t ph = 0;
+      const uint32_t bytes = TILE_BYTES + 2u * (uint32_t)K * KT * sizeof(double);
       while (true) {
         const int itx = atomicAdd(counter, 1);
         if (itx >= n_items) break;
@@ -212,9 +222,15 @@ kf_pass_kernel(double* __restrict__ P, const ItemD* __restrict__ items, int n_it
         for (int t = 0; t < it.nJ; ++t) {
           mbar_wait(&empty[s], ph ^ 1);
           meta[s] = make_int4(itx, it.J0 + t, (t == 0 ? 1 : 0) | (t == it.nJ - 1 ? 2 : 0), 0);
-          mbar_arrive_tx(&full[s], TILE_BYTES);
-          tma_load_1d(tiles + (size_t)s * TILE_ELEMS, P + (size_t)(it.tile_off + t) * TILE_ELEMS, TILE_BYTES,
-                      &full[s]);
+          double* st_s = stages + (size_t)s * STAGE_ELEMS;
+          mbar_arrive_tx(&full[s], bytes);
+          tma_load_1d(st_s, P + (size_t)(it.tile_off + t) * TILE_ELEMS, TILE_BYTES, &full[s]);
+          for (int k = 0; k < K; ++k) {
+            const double* uk = ulist + (size_t)k * npad + it.vbase;
+            tma_load_1d(st_s + TILE_ELEMS + k * KT, uk + (size_t)it.I * KT, KT * sizeof(double), &full[s]);
+            tma_load_1d(st_s + TILE_ELEMS + (KMAX + k) * KT, uk + (size_t)(it.J0 + t) * KT, KT * sizeof(double),
+                        &full[s]);
+          }
           if (++s == STAGES) { s = 0; ph ^= 1; }
         }
       }
@@ -226,13 +242,14 @@ kf_pass_kernel(double* __restrict__ P, const ItemD* __restrict__ items, int n_it
   }
 
   // ------------------------------ consumers ------------------------------
-  const int pend = st->pend;
-  const double Ap = st->A_pend;
-  const double il = st->invlam_pend;
-  const int c0 = 2 * lane;
-  double gI[8], uI[8], racc[8];
+  double beta[KMAX];
 #pragma unroll
-  for (int k = 0; k < 8; ++k) { gI[k] = 0.0; uI[k] = 0.0; racc[k] = 0.0; }
+  for (int k = 0; k < KMAX; ++k) beta[k] = k < K ? st->beta[k] : 0.0;
+  const double sig = st->sigma;
+  const int c0 = 2 * lane;
+  double gI[8], racc[8];
+#pragma unroll
+  for (int k = 0; k < 8; ++k) { gI[k] = 0.0; racc[k] = 0.0; }
   int s = 0, prev_s = -1;
   uint32_t ph = 0;
   uint32_t tcount = 0;
@@ -246,29 +263,37 @@ kf_pass_kernel(double* __restrict__ P, const ItemD* __restrict__ items, int n_it
     if (first) {
 #pragma unroll
       for (int k = 0; k < 8; ++k) {
-        const long long v = it.vbase + (long long)it.I * KT + warp + 8 * k;
-        gI[k] = __ldg(gpad + v);
-        uI[k] = __ldg(upend + v);
+        gI[k] = __ldg(gpad + it.vbase + (long long)it.I * KT + warp + 8 * k);
         racc[k] = 0.0;
       }
     }
-    const long long vj = it.vbase + (long long)J * KT + c0;
-    const double2 gJ = __ldg(reinterpret_cast<const double2*>(gpad + vj));
-    const double2 uJ = __ldg(reinterpret_cast<const double2*>(upend + vj));
-    double* t = tiles + (size_t)s * TILE_ELEMS;
+    const double2 gJ = __ldg(reinterpret_cast<const double2*>(gpad + it.vbase + (long long)J * KT + c0));
+    double* t = stages + (size_t)s * STAGE_ELEMS;
+    const double* vI = t + TILE_ELEMS;
+    const double* vJ = t + TILE_ELEMS + KMAX * KT;
     double ca0 = 0.0, ca1 = 0.0;
 #pragma unroll
-    for (int k = 0; k < 8; ++k) {
-      const int r = warp + 8 * k;
+    for (int q = 0; q < 8; ++q) {
+      const int r = warp + 8 * q;
       double2 v = *reinterpret_cast<double2*>(t + r * KT + c0);
-      if (pend) {
-        v.x = __dmul_rn(__dsub_rn(v.x, __dmul_rn(Ap, __dmul_rn(uI[k], uJ.x))), il);
-        v.y = __dmul_rn(__dsub_rn(v.y, __dmul_rn(Ap, __dmul_rn(uI[k], uJ.y))), il);
+      if (rw) {
+        double cx = 0.0, cy = 0.0;
+#pragma unroll
+        for (int k = 0; k < KMAX; ++k) {
+          if (k < K) {
+            const double bu = beta[k] * vI[k * KT + r];
+            const double2 uj = *reinterpret_cast<const double2*>(vJ + k * KT + c0);
+            cx = fma(bu, uj.x, cx);
+            cy = fma(bu, uj.y, cy);
+          }
+        }
+        v.x = sig * (v.x - cx);
+        v.y = sig * (v.y - cy);
         *reinterpret_cast<double2*>(t + r * KT + c0) = v;
       }
-      racc[k] = fma(v.x, gJ.x, fma(v.y, gJ.y, racc[k]));
-      ca0 = fma(v.x, gI[k], ca0);
-      ca1 = fma(v.y, gI[k], ca1);
+      racc[q] = fma(v.x, gJ.x, fma(v.y, gJ.y, racc[q]));
+      ca0 = fma(v.x, gI[q], ca0);
+      ca1 = fma(v.y, gI[q], ca1);
     }
     double* cr = colred + (tcount & 1) * (8 * KT);
     if (!diag) {
@@ -277,7 +302,7 @@ kf_pass_kernel(double* __restrict__ P, const ItemD* __restrict__ items, int n_it
     }
     consumer_bar();
     if (tid == 0) {
-      if (pend) {
+      if (rw) {
         fence_proxy_async();
         tma_store_1d(P + (size_t)(it.tile_off + (J - it.J0)) * TILE_ELEMS, t, TILE_BYTES);
         bulk_commit();
@@ -287,7 +312,7 @@ kf_pass_kernel(double* __restrict__ P, const ItemD* __restrict__ items, int n_it
         }
         prev_s = s;
       } else {
-        mbar_arrive(&empty[s]);  // read-only pass: the stage is free once every consumer passed the barrier
+        mbar_arrive(&empty[s]);  // read-only: the stage is free once every consumer passed the barrier
       }
     }
     if (!diag && tid < KT) {
@@ -298,11 +323,11 @@ kf_pass_kernel(double* __restrict__ P, const ItemD* __restrict__ items, int n_it
     }
     if (last) {
 #pragma unroll
-      for (int k = 0; k < 8; ++k) {
-        double v = racc[k];
+      for (int q = 0; q < 8; ++q) {
+        double v = racc[q];
 #pragma unroll
         for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
-        if (lane == 0) ws[(size_t)it.row_slot * KT + warp + 8 * k] = v;
+        if (lane == 0) ws[(size_t)it.row_slot * KT + warp + 8 * q] = v;
       }
     }
     if (++s == STAGES) { s = 0; ph ^= 1; }
@@ -331,7 +356,7 @@ __global__ void kf_pad_kernel(const double* __restrict__ g, double* __restrict__
   gpad[p] = loc < nblk[b] ? g[off[b] + loc] : 0.0;
 }
 
-// u[tc*T + t] = sum over the CSR entries of tile column tc (fixed order)
+// u_B[tc*T + t] = sum over the CSR entries of tile column tc (fixed order)
 __global__ void kf_reduce_u_kernel(const double* __restrict__ ws, const long long* __restrict__ ptr,
                                    const long long* __restrict__ idx, long long n_tc, double* __restrict__ u) {
   const long long tc = (long long)blockIdx.x * (blockDim.x / KT) + threadIdx.x / KT;
@@ -342,74 +367,110 @@ __global__ void kf_reduce_u_kernel(const double* __restrict__ ws, const long lon
   u[tc * KT + t] = a;
 }
 
-// dotp[tc] = sum_t gpad * u over tile column tc
-__global__ void kf_dot_kernel(const double* __restrict__ gpad, const double* __restrict__ u, long long n_tc,
+// per tile column: dotp[0][tc] = g . u_B, dotp[1+k][tc] = g . u_k (k < K deferred vectors)
+__global__ void kf_dot_kernel(const double* __restrict__ gpad, const double* __restrict__ ub,
+                              const double* __restrict__ ulist, long long npad, int K, long long n_tc,
                               double* __restrict__ dotp) {
   const long long tc = (long long)blockIdx.x * (blockDim.x / 32) + threadIdx.x / 32;
   const int lane = threadIdx.x & 31;
   if (tc >= n_tc) return;
-  double a = gpad[tc * KT + lane] * u[tc * KT + lane] + gpad[tc * KT + 32 + lane] * u[tc * KT + 32 + lane];
-  for (int o = 16; o > 0; o >>= 1) a += __shfl_xor_sync(0xffffffffu, a, o);
-  if (lane == 0) dotp[tc] = a;
+  const double g0 = gpad[tc * KT + lane], g1 = gpad[tc * KT + 32 + lane];
+  for (int k = -1; k < K; ++k) {
+    const double* u = k < 0 ? ub : ulist + (size_t)k * npad;
+    double a = g0 * u[tc * KT + lane] + g1 * u[tc * KT + 32 + lane];
+    for (int o = 16; o > 0; o >>= 1) a += __shfl_xor_sync(0xffffffffu, a, o);
+    if (lane == 0) dotp[(size_t)(k + 1) * n_tc + tc] = a;
+  }
 }
 
-// A = 1/(c + g^T u), K = A u, coef = sqrt(bs) ABE A, pending <- (A, 1/lambda), lambda update (Eq. 3)
-__global__ void kf_finish_kernel(const double* __restrict__ dotp, long long n_tc, KfState* st,
+// With P_t = sigma (B - sum_k beta_k u_k u_k^T):  u_t = P_t g = sigma (u_B - sum_k beta_k (u_k . g) u_k),
+// A = 1/(c + g^T u_t) (Alg. 1 line 8, c = L*lambda or lambda), K = A u_t (line 9),
+// P_{t+1} = (P_t - A u_t u_t^T)/lambda (line 10)  =>  append beta = A/sigma, sigma <- sigma/lambda;
+// lambda <- nu lambda + 1 - nu (line 12, Eq. 3); w += sqrt(bs) ABE K (line 13, Eq. 2).
+// rw: the pass just rewrote B = P_t, so sigma = 1 and the deferred list is empty.
+__global__ void kf_finish_kernel(const double* __restrict__ dotp, long long n_tc, int K, int rw, KfState* st,
                                  const double* abe, double sqrt_bs) {
-  __shared__ double red[1024];
-  double a = 0.0;
-  for (long long i = threadIdx.x; i < n_tc; i += blockDim.x) a += dotp[i];
-  red[threadIdx.x] = a;
-  __syncthreads();
-  for (int s = blockDim.x / 2; s > 0; s >>= 1) {
-    if ((int)threadIdx.x < s) red[threadIdx.x] += red[threadIdx.x + s];
-    __syncthreads();
+  __shared__ double red[1 + KMAX][128];
+  __shared__ double tot[1 + KMAX];
+  for (int k = 0; k <= K; ++k) {
+    double a = 0.0;
+    for (long long i = threadIdx.x; i < n_tc; i += blockDim.x) a += dotp[(size_t)k * n_tc + i];
+    red[k][threadIdx.x] = a;
   }
+  __syncthreads();
+  if (threadIdx.x <= (unsigned)K) {
+    double a = 0.0;
+    for (int i = 0; i < (int)blockDim.x; ++i) a += red[threadIdx.x][i];
+    tot[threadIdx.x] = a;
+  }
+  __syncthreads();
   if (threadIdx.x == 0) {
     const double lam = st->lambda;
-    const double c = st->c_mult * lam;                  // c = L*lambda (Z1) or lambda
-    const double A = 1.0 / (c + red[0]);                // Alg. 1 line 8
+    const double sig = rw ? 1.0 : st->sigma;
+    double gtu = tot[0];
+    for (int k = 0; k < K; ++k) {
+      const double d = tot[1 + k];
+      st->cu[k] = sig * st->beta[k] * d;
+      gtu -= st->beta[k] * d * d;
+    }
+    gtu *= sig;
+    const double A = 1.0 / (st->c_mult * lam + gtu);
     const double e = abe ? *abe : 0.0;
+    const int slot = rw ? 0 : st->npend;
+    st->sig_cur = sig;
     st->A_last = A;
-    st->A_pend = A;
-    st->invlam_pend = 1.0 / lam;                        // line 10 uses the pre-increment lambda
-    st->pend = 1;
-    st->coef = sqrt_bs * e * A;                         // line 13 / Eq. 2: w += sqrt(bs) ABE K, K = A u
-    st->lambda = lam * st->nu + 1.0 - st->nu;           // line 12 (Eq. 3)
+    st->coef_w = sqrt_bs * e * A;
+    st->slot = slot;
+    st->beta[slot] = A / sig;
+    st->npend = slot + 1;
+    st->sigma = sig / lam;
+    st->lambda = lam * st->nu + 1.0 - st->nu;
     st->t += 1;
     if (!isfinite(A) || !isfinite(e)) st->flags |= 2;
   }
 }
 
-__global__ void kf_w_update_kernel(double* __restrict__ w, const double* __restrict__ u, const KfState* st,
-                                   const int* tc_blk, const int* tc_c, const long long* off, const int* nblk,
-                                   long long npad) {
-  long long p = (long long)blockIdx.x * blockDim.x + threadIdx.x;
+// u_t = sigma (u_B - sum_k cu_k u_k) -> deferred slot; w += sqrt(bs) ABE A u_t
+__global__ void kf_vec_kernel(const double* __restrict__ ub, double* __restrict__ ulist, long long npad, int K,
+                              const KfState* st, double* __restrict__ w, const int* tc_blk, const int* tc_c,
+                              const long long* off, const int* nblk) {
+  const long long p = (long long)blockIdx.x * blockDim.x + threadIdx.x;
   if (p >= npad) return;
+  double v = ub[p];
+  for (int k = 0; k < K; ++k) v -= st->cu[k] * ulist[(size_t)k * npad + p];
+  v *= st->sig_cur;
+  ulist[(size_t)st->slot * npad + p] = v;
   const long long tc = p / KT;
   const int b = tc_blk[tc];
   const int loc = tc_c[tc] * KT + (int)(p % KT);
-  if (loc < nblk[b]) w[off[b] + loc] += st->coef * u[p];
+  if (loc < nblk[b]) w[off[b] + loc] += st->coef_w * v;
 }
 
-// apply the pending correction to stored tiles (flush) — one CTA per item
+__device__ __forceinline__ double deferred_value(double b, const KfState* st, const double* ulist, long long npad,
+                                                 long long pr, long long pc) {
+  double c = 0.0;
+  for (int k = 0; k < st->npend; ++k) c += st->beta[k] * ulist[(size_t)k * npad + pr] * ulist[(size_t)k * npad + pc];
+  return st->sigma * (b - c);
+}
+
+// rewrite B = P_t (flush) — one CTA per item
 __global__ void kf_apply_pending_kernel(double* __restrict__ P, const ItemD* __restrict__ items,
-                                        const double* __restrict__ upend, KfState* st) {
-  if (!st->pend) return;
+                                        const double* __restrict__ ulist, long long npad, const KfState* st) {
   const ItemD it = items[blockIdx.x];
-  const double Ap = st->A_pend, il = st->invlam_pend;
   for (int t = 0; t < it.nJ; ++t) {
     double* tile = P + (size_t)(it.tile_off + t) * TILE_ELEMS;
     const int J = it.J0 + t;
     for (int e = threadIdx.x; e < TILE_ELEMS; e += blockDim.x) {
       const int r = e / KT, c = e % KT;
-      const double ur = upend[it.vbase + (long long)it.I * KT + r];
-      const double uc = upend[it.vbase + (long long)J * KT + c];
-      tile[e] = __dmul_rn(__dsub_rn(tile[e], __dmul_rn(Ap, __dmul_rn(ur, uc))), il);
+      tile[e] = deferred_value(tile[e], st, ulist, npad, it.vbase + (long long)it.I * KT + r,
+                               it.vbase + (long long)J * KT + c);
     }
   }
 }
-__global__ void kf_clear_pending_kernel(KfState* st) { st->pend = 0; }
+__global__ void kf_clear_pending_kernel(KfState* st) {
+  st->npend = 0;
+  st->sigma = 1.0;
+}
 
 // P = I on the valid part of every block, 0 on the padding
 __global__ void kf_init_kernel(double* __restrict__ P, const ItemD* __restrict__ items, const int* nblk) {
@@ -426,13 +487,12 @@ __global__ void kf_init_kernel(double* __restrict__ P, const ItemD* __restrict__
   }
 }
 
-// dense <-> packed for one block (tests / checkpoints)
+// dense <-> packed for one block (tests / checkpoints); get applies the deferred corrections on the fly
 __global__ void kf_get_block_kernel(const double* __restrict__ P, const ItemD* __restrict__ items, int blk, int n,
-                                    const double* __restrict__ upend, const KfState* st, double* __restrict__ dst) {
+                                    const double* __restrict__ ulist, long long npad, const KfState* st,
+                                    double* __restrict__ dst) {
   const ItemD it = items[blockIdx.x];
   if (it.blk != blk) return;
-  const int pend = st->pend;
-  const double Ap = st->A_pend, il = st->invlam_pend;
   for (int t = 0; t < it.nJ; ++t) {
     const double* tile = P + (size_t)(it.tile_off + t) * TILE_ELEMS;
     const int J = it.J0 + t;
@@ -440,11 +500,7 @@ __global__ void kf_get_block_kernel(const double* __restrict__ P, const ItemD* _
       const int r = e / KT, c = e % KT;
       const int gr = it.I * KT + r, gc = J * KT + c;
       if (gr >= n || gc >= n) continue;
-      double v = tile[e];
-      if (pend) {
-        const double ur = upend[it.vbase + gr], uc = upend[it.vbase + gc];
-        v = __dmul_rn(__dsub_rn(v, __dmul_rn(Ap, __dmul_rn(ur, uc))), il);
-      }
+      const double v = deferred_value(tile[e], st, ulist, npad, it.vbase + gr, it.vbase + gc);
       dst[(size_t)gr * n + gc] = v;
       if (J != it.I) dst[(size_t)gc * n + gr] = v;
     }
@@ -482,6 +538,7 @@ static int num_sms() {
 fekf_status Kf::create(const std::vector<int>& blocks, const fekf_opt_cfg& o, fekf_comm* c) {
   opt = o;
   comm = c;
+  defer = std::max(1, std::min(KMAX, o.p_defer > 0 ? o.p_defer : 1));
   int world = 1, rank = 0;
   if (comm) { world = comm_world(comm); rank = comm_rank(comm); }
   plan.build(blocks, world, rank, SEG_TILES);
@@ -490,9 +547,9 @@ fekf_status Kf::create(const std::vector<int>& blocks, const fekf_opt_cfg& o, fe
   FEKF_TRY(dalloc(items_d, std::max<size_t>(1, p.items.size()) * sizeof(ItemD)));
   FEKF_TRY(dalloc(ws, (size_t)std::max<int64_t>(1, p.ws_slots) * KT * sizeof(double)));
   FEKF_TRY(dalloc(gpad, p.Npad * sizeof(double)));
-  FEKF_TRY(dalloc(unew, p.Npad * sizeof(double)));
-  FEKF_TRY(dalloc(upend, p.Npad * sizeof(double)));
-  FEKF_TRY(dalloc(dotp, p.n_tc * sizeof(double)));
+  FEKF_TRY(dalloc(ub, p.Npad * sizeof(double)));
+  FEKF_TRY(dalloc(ulist, (size_t)KMAX * p.Npad * sizeof(double)));
+  FEKF_TRY(dalloc(dotp, (size_t)(1 + KMAX) * p.n_tc * sizeof(double)));
   FEKF_TRY(dalloc(csr_ptr, (p.n_tc + 1) * sizeof(long long)));
   FEKF_TRY(dalloc(csr_idx, std::max<size_t>(1, p.csr_idx.size()) * sizeof(long long)));
   FEKF_TRY(dalloc(tc_blk, p.n_tc * sizeof(int)));
@@ -513,16 +570,17 @@ fekf_status Kf::create(const std::vector<int>& blocks, const fekf_opt_cfg& o, fe
   KfState s{};
   s.lambda = o.lambda0;
   s.nu = o.nu;
+  s.sigma = 1.0;
   s.c_mult = o.noise_mode == 0 ? (double)p.L : 1.0;
   FEKF_CHECK_CUDA(cudaMemcpy(state.p, &s, sizeof(KfState), cudaMemcpyHostToDevice));
-  FEKF_CHECK_CUDA(cudaMemset(upend.p, 0, p.Npad * sizeof(double)));
-  FEKF_CHECK_CUDA(cudaMemset(unew.p, 0, p.Npad * sizeof(double)));
+  FEKF_CHECK_CUDA(cudaMemset(ulist.p, 0, (size_t)KMAX * p.Npad * sizeof(double)));
   FEKF_CHECK_CUDA(cudaFuncSetAttribute(kf_pass_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)PASS_SMEM));
   if (!p.items.empty()) {
     kf_init_kernel<<<(unsigned)p.items.size(), 256>>>(P.as<double>(), items_d.as<ItemD>(), n_d.as<int>());
     FEKF_LAUNCH_CHECK();
   }
   FEKF_CHECK_CUDA(cudaDeviceSynchronize());
+  npend = 0;
   return FEKF_OK;
 }
 
@@ -547,12 +605,12 @@ fekf_status Kf::timing_ctl(int mode, double* total_ms, int64_t* launches) {
 
 Kf::~Kf() {
   for (cudaEvent_t e : ev) cudaEventDestroy(e);
-  for (DBuf* b : {&P, &items_d, &ws, &gpad, &unew, &upend, &dotp, &csr_ptr, &csr_idx, &tc_blk, &tc_c, &off_d, &n_d,
+  for (DBuf* b : {&P, &items_d, &ws, &gpad, &ub, &ulist, &dotp, &csr_ptr, &csr_idx, &tc_blk, &tc_c, &off_d, &n_d,
                   &state, &counter})
     dfree(*b);
 }
 
-fekf_status Kf::pass(const double* g, cudaStream_t s) {
+fekf_status Kf::pass(const double* g, bool rw, cudaStream_t s) {
   const KfPlan& p = plan;
   const int tb = 256;
   kf_pad_kernel<<<cdiv(p.Npad, tb), tb, 0, s>>>(g, gpad.as<double>(), tc_blk.as<int>(), tc_c.as<int>(),
@@ -571,46 +629,56 @@ fekf_status Kf::pass(const double* g, cudaStream_t s) {
       FEKF_CHECK_CUDA(cudaEventRecord(ev[ev_used], s));
     }
     kf_pass_kernel<<<grid, PASS_THREADS, PASS_SMEM, s>>>(P.as<double>(), items_d.as<ItemD>(), (int)p.items.size(),
-                                                          counter.as<int>(), gpad.as<double>(), upend.as<double>(),
-                                                          state.as<KfState>(), ws.as<double>());
+                                                          counter.as<int>(), gpad.as<double>(), ulist.as<double>(),
+                                                          p.Npad, rw ? 1 : 0, rw ? npend : 0, state.as<KfState>(),
+                                                          ws.as<double>());
     FEKF_LAUNCH_CHECK();
     count_launch();
+    if (rw) ++rw_passes; else ++r_passes;
     if (timing) {
       FEKF_CHECK_CUDA(cudaEventRecord(ev[ev_used + 1], s));
       ev_used += 2;
     }
   }
   kf_reduce_u_kernel<<<cdiv(p.n_tc, 4), 256, 0, s>>>(ws.as<double>(), csr_ptr.as<long long>(),
-                                                      csr_idx.as<long long>(), p.n_tc, unew.as<double>());
+                                                      csr_idx.as<long long>(), p.n_tc, ub.as<double>());
   FEKF_LAUNCH_CHECK();
   count_launch();
   return FEKF_OK;
 }
 
+// One update (Alg. 1 lines 8-13).  The stored P is rewritten only when `defer` corrections are
+// pending; otherwise the pass is read-only and the corrections are applied to u in vector form.
 fekf_status Kf::update(const double* g, const double* abe, double sqrt_bs, double* w, cudaStream_t s) {
   const KfPlan& p = plan;
-  FEKF_TRY(pass(g, s));
-  if (comm && comm_world(comm) > 1) FEKF_TRY(comm_allreduce(comm, unew.as<double>(), p.Npad, s));
-  kf_dot_kernel<<<cdiv(p.n_tc, 8), 256, 0, s>>>(gpad.as<double>(), unew.as<double>(), p.n_tc, dotp.as<double>());
+  const bool rw = npend >= defer;
+  FEKF_TRY(pass(g, rw, s));
+  if (comm && comm_world(comm) > 1) FEKF_TRY(comm_allreduce(comm, ub.as<double>(), p.Npad, s));
+  const int K = rw ? 0 : npend;
+  kf_dot_kernel<<<cdiv(p.n_tc, 8), 256, 0, s>>>(gpad.as<double>(), ub.as<double>(), ulist.as<double>(), p.Npad, K,
+                                                p.n_tc, dotp.as<double>());
   FEKF_LAUNCH_CHECK();
-  kf_finish_kernel<<<1, 1024, 0, s>>>(dotp.as<double>(), p.n_tc, state.as<KfState>(), abe, sqrt_bs);
+  kf_finish_kernel<<<1, 128, 0, s>>>(dotp.as<double>(), p.n_tc, K, rw ? 1 : 0, state.as<KfState>(), abe, sqrt_bs);
   FEKF_LAUNCH_CHECK();
-  kf_w_update_kernel<<<cdiv(p.Npad, 256), 256, 0, s>>>(w, unew.as<double>(), state.as<KfState>(), tc_blk.as<int>(),
-                                                        tc_c.as<int>(), off_d.as<long long>(), n_d.as<int>(), p.Npad);
+  kf_vec_kernel<<<cdiv(p.Npad, 256), 256, 0, s>>>(ub.as<double>(), ulist.as<double>(), p.Npad, K, state.as<KfState>(),
+                                                   w, tc_blk.as<int>(), tc_c.as<int>(), off_d.as<long long>(),
+                                                   n_d.as<int>());
   FEKF_LAUNCH_CHECK();
-  FEKF_CHECK_CUDA(cudaMemcpyAsync(upend.p, unew.p, p.Npad * sizeof(double), cudaMemcpyDeviceToDevice, s));
   count_launch(3);
+  npend = (rw ? 0 : npend) + 1;
   return FEKF_OK;
 }
 
 fekf_status Kf::flush(cudaStream_t s) {
-  if (!plan.items.empty()) {
+  if (!plan.items.empty() && npend > 0) {
     kf_apply_pending_kernel<<<(unsigned)plan.items.size(), 256, 0, s>>>(P.as<double>(), items_d.as<ItemD>(),
-                                                                         upend.as<double>(), state.as<KfState>());
+                                                                         ulist.as<double>(), plan.Npad,
+                                                                         state.as<KfState>());
     FEKF_LAUNCH_CHECK();
   }
   kf_clear_pending_kernel<<<1, 1, 0, s>>>(state.as<KfState>());
   FEKF_LAUNCH_CHECK();
+  npend = 0;
   return FEKF_OK;
 }
 
@@ -618,7 +686,8 @@ fekf_status Kf::get_block(int b, double* dst, cudaStream_t s) {
   if (b < 0 || b >= plan.L) { set_error("get_block: bad block"); return FEKF_EINVAL; }
   if (plan.items.empty()) return FEKF_OK;
   kf_get_block_kernel<<<(unsigned)plan.items.size(), 256, 0, s>>>(P.as<double>(), items_d.as<ItemD>(), b, plan.n[b],
-                                                                   upend.as<double>(), state.as<KfState>(), dst);
+                                                                   ulist.as<double>(), plan.Npad, state.as<KfState>(),
+                                                                   dst);
   FEKF_LAUNCH_CHECK();
   return FEKF_OK;
 }

@@ -8,6 +8,7 @@ namespace fekf {
 
 constexpr int KT = FEKF_TILE;    // tile edge (64 fp64 = 32 KiB per tile)
 constexpr int SEG_TILES = 32;    // max tiles per work item (tile-row segment)
+constexpr int KMAX = 8;          // max deferred rank-1 corrections held before P is rewritten
 
 // One P-pass work item: tiles (I, J0..J0+nJ-1) of block `blk`, stored contiguously at tile_off.
 struct ItemD {
@@ -19,14 +20,16 @@ struct ItemD {
   int pad_;
 };
 
-// Device-resident optimizer scalars.
+// Device-resident optimizer scalars.  The stored P (the "base" B) and the current covariance are
+// related by P_t = sigma (B - sum_k beta_k u_k u_k^T) over the npend deferred corrections.
 struct KfState {
-  double lambda, nu;
-  double A_pend, invlam_pend;  // pending rank-1 correction (applied by the next pass)
-  double A_last, coef;         // last A and sqrt(bs)*ABE*A
-  double c_mult;               // L (noise_mode 0) or 1
+  double lambda, nu, sigma, c_mult;
+  double A_last, coef_w;       // last A and sqrt(bs) * ABE * A
+  double sig_cur;              // sigma used to form the current u
+  double beta[KMAX];           // deferred coefficients
+  double cu[KMAX];             // sigma * beta_k * (u_k . g) of the current update
   long long t;
-  int pend, flags;
+  int npend, flags, slot, pad_;
 };
 
 struct KfPlan {
@@ -52,14 +55,17 @@ struct Kf {
   fekf_opt_cfg opt{};
   fekf_comm* comm = nullptr;
   KfPlan plan;
-  DBuf P, items_d, ws, gpad, unew, upend, dotp, csr_ptr, csr_idx, tc_blk, tc_c, off_d, n_d, state, counter;
+  int defer = 1;                 // corrections deferred before P is rewritten (1 = rewrite every update)
+  int npend = 0;                 // host mirror of the device npend
+  DBuf P, items_d, ws, gpad, ub, ulist, dotp, csr_ptr, csr_idx, tc_blk, tc_c, off_d, n_d, state, counter;
   bool timing = false;
   std::vector<cudaEvent_t> ev;   // [start, stop] per timed pass launch
   size_t ev_used = 0;
+  long long rw_passes = 0, r_passes = 0;
   fekf_status timing_ctl(int mode, double* total_ms, int64_t* launches);
   fekf_status create(const std::vector<int>& blocks, const fekf_opt_cfg& o, fekf_comm* c);
   ~Kf();
-  fekf_status pass(const double* g, cudaStream_t s);
+  fekf_status pass(const double* g, bool rw, cudaStream_t s);
   fekf_status update(const double* g, const double* abe, double sqrt_bs, double* w, cudaStream_t s);
   fekf_status flush(cudaStream_t s);
   fekf_status get_block(int b, double* dst, cudaStream_t s);

@@ -35,7 +35,8 @@ class ModelCfg(C.Structure):
 
 class OptCfg(C.Structure):
     _fields_ = [("lambda0", C.c_double), ("nu", C.c_double), ("block_size", C.c_int), ("noise_mode", C.c_int),
-                ("grad_reduce", C.c_int), ("force_groups", C.c_int), ("atoms_per_group", C.c_int)]
+                ("grad_reduce", C.c_int), ("force_groups", C.c_int), ("atoms_per_group", C.c_int),
+                ("p_defer", C.c_int)]
 
 
 _lib = None
@@ -154,6 +155,7 @@ def opt_cfg(o=None) -> OptCfg:
     c.grad_reduce = int(_get(o, "grad_reduce", 0)) if o is not None else 0
     c.force_groups = int(_get(o, "force_groups", 4)) if o is not None else 4
     c.atoms_per_group = int(_get(o, "atoms_per_group", 6)) if o is not None else 6
+    c.p_defer = int(_get(o, "p_defer", 5)) if o is not None else 5
     return c
 
 

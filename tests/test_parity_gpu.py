@@ -122,10 +122,10 @@ def _rand_spd(rng, n):
 
 
 @pytest.mark.parametrize("blocks", [[5, 70, 130], [64], [1, 200, 127, 65]])
-@pytest.mark.parametrize("noise_mode", [0, 1])
-def test_kalman_updates(blocks, noise_mode):
+@pytest.mark.parametrize("noise_mode,p_defer", [(0, 5), (1, 1), (0, 3), (1, 8)])
+def test_kalman_updates(blocks, noise_mode, p_defer):
     rng = np.random.default_rng(7)
-    opt = dict(lambda0=0.98, nu=0.9987, block_size=1024, noise_mode=noise_mode)
+    opt = dict(lambda0=0.98, nu=0.9987, block_size=1024, noise_mode=noise_mode, p_defer=p_defer)
     kf = fk.KalmanFilter(blocks, opt)
     N = sum(blocks)
     st = O.FEKF(np.zeros(N), blocks, lam=0.98, nu=0.9987, noise_mode=noise_mode)
