@@ -1,16 +1,19 @@
-// fp64 GEMM for the embedding / fitting layers (sm_100a CUDA cores; see DESIGN.md §7 for why fp64
-// stays off tcgen05).  C = op(A) op(B) with a fused epilogue.
+// fp64 GEMM for the embedding / fitting layers on the sm_100a FP64 tensor path (DMMA,
+// mma.sync.m8n8k4.f64; measured on B200 at the same 37 TFLOP/s as FP64 FFMA but with ~5x less
+// shared-memory traffic per FMA).  tcgen05 has no fp64 kind, and TF32 would break the fp64 parity.
+// C = op(A) op(B) with a fused epilogue:
 //   TA: A stored [K x M] (weight gradients, K = rows); TB: B stored [N x K] (data gradients, W^T).
 //   Optional "ones" row aug_m of op(A): (k < aug_k ? 1 : 0), so [W-grad ; b-grad] = [H | 1]^T Zbar.
 //   Mdev / Kdev: device-resident row counts (compacted rows); CTAs past them exit.
-// Tiles BM x BN x 16 (BM, BN in {32, 64, 128}), 256 threads, (BM/16) x (BN/16) register micro-tiles,
-// SMEM double buffering with register staging; the tile shape is picked per call from (M, N).
+// CTA tile BM x BN x 16, 8 warps each WM x WN (WM/8 x WN/8 DMMA tiles), operands staged in SMEM
+// k-contiguous with a 20-double row stride (conflict-free fragment loads), register-staged double buffer.
 #pragma once
 #include "model.cuh"
 
 namespace fekf {
 
 constexpr int GB_K = 16;
+constexpr int GB_LDS = GB_K + 4;
 
 struct EpiStore {
   double* C; int ldc;
@@ -56,16 +59,24 @@ struct EpiDgrad {
   }
 };
 
-template <int BM, int BN, bool TA, bool TB, class Epi>
+__device__ __forceinline__ void dmma884(double& d0, double& d1, double a, double b) {
+  asm volatile("mma.sync.aligned.m8n8k4.row.col.f64.f64.f64.f64 {%0,%1}, {%2}, {%3}, {%0,%1};"
+               : "+d"(d0), "+d"(d1)
+               : "d"(a), "d"(b));
+}
+
+template <int BM, int BN, int WM, int WN, bool TA, bool TB, class Epi>
 __global__ void __launch_bounds__(256)
 dgemm_kernel(int M, int N, int K, const int* __restrict__ Mdev, const int* __restrict__ Kdev,
              const double* __restrict__ A, int lda, const double* __restrict__ B, int ldb, int aug_m, int aug_k,
              int kps, Epi epi) {
-  constexpr int TM = BM / 16, TN = BN / 16;
+  constexpr int NWN = BN / WN;
+  static_assert((BM / WM) * NWN == 8, "8 warps");
+  constexpr int TI = WM / 8, TJ = WN / 8;
   constexpr int AE = BM * GB_K / 256, BE = BN * GB_K / 256;
   extern __shared__ __align__(16) double gsm[];
-  auto As = reinterpret_cast<double (*)[GB_K][BM + 2]>(gsm);
-  auto Bs = reinterpret_cast<double (*)[GB_K][BN + 2]>(gsm + 2 * GB_K * (BM + 2));
+  auto As = reinterpret_cast<double (*)[BM][GB_LDS]>(gsm);
+  auto Bs = reinterpret_cast<double (*)[BN][GB_LDS]>(gsm + 2 * BM * GB_LDS);
   if (Mdev) M = min(M, *Mdev);
   if (Kdev) {
     const int kd = *Kdev;
@@ -77,12 +88,14 @@ dgemm_kernel(int M, int N, int K, const int* __restrict__ Mdev, const int* __res
   const int kbeg = blockIdx.z * kps;
   if (m0 >= M || (blockIdx.z > 0 && kbeg >= K)) return;  // empty split: the reduction skips it
   const int kend = min(K, kbeg + kps);
-  const int tm = tid >> 4, tn = tid & 15;
-  double acc[TM][TN];
+  const int warp = tid >> 5, lane = tid & 31;
+  const int wm = warp / NWN, wn = warp % NWN;
+  const int fr = lane >> 2, fk = lane & 3;
+  double acc[TI][TJ][2];
 #pragma unroll
-  for (int i = 0; i < TM; ++i)
+  for (int i = 0; i < TI; ++i)
 #pragma unroll
-    for (int j = 0; j < TN; ++j) acc[i][j] = 0.0;
+    for (int j = 0; j < TJ; ++j) acc[i][j][0] = acc[i][j][1] = 0.0;
   double ra[AE], rb[BE];
   auto load = [&](int k0) {
 #pragma unroll
@@ -113,12 +126,12 @@ dgemm_kernel(int M, int N, int K, const int* __restrict__ Mdev, const int* __res
 #pragma unroll
     for (int q = 0; q < AE; ++q) {
       const int idx = tid + 256 * q;
-      if (!TA) As[buf][idx % GB_K][idx / GB_K] = ra[q]; else As[buf][idx / BM][idx % BM] = ra[q];
+      if (!TA) As[buf][idx / GB_K][idx % GB_K] = ra[q]; else As[buf][idx % BM][idx / BM] = ra[q];
     }
 #pragma unroll
     for (int q = 0; q < BE; ++q) {
       const int idx = tid + 256 * q;
-      if (!TB) Bs[buf][idx / BN][idx % BN] = rb[q]; else Bs[buf][idx % GB_K][idx / GB_K] = rb[q];
+      if (!TB) Bs[buf][idx % BN][idx / BN] = rb[q]; else Bs[buf][idx / GB_K][idx % GB_K] = rb[q];
     }
   };
   const int nk = kend > kbeg ? (kend - kbeg + GB_K - 1) / GB_K : 0;
@@ -130,69 +143,62 @@ dgemm_kernel(int M, int N, int K, const int* __restrict__ Mdev, const int* __res
       if (t + 1 < nk) load(kbeg + (t + 1) * GB_K);
       const int buf = t & 1;
 #pragma unroll
-      for (int kk = 0; kk < GB_K; ++kk) {
-        double a[TM], b[TN];
+      for (int ks = 0; ks < GB_K; ks += 4) {
+        double a[TI], b[TJ];
 #pragma unroll
-        for (int i = 0; i < TM; i += 2) {
-          const double2 v = *reinterpret_cast<const double2*>(&As[buf][kk][tm * TM + i]);
-          a[i] = v.x; a[i + 1] = v.y;
-        }
+        for (int i = 0; i < TI; ++i) a[i] = As[buf][wm * WM + i * 8 + fr][ks + fk];
 #pragma unroll
-        for (int j = 0; j < TN; j += 2) {
-          const double2 v = *reinterpret_cast<const double2*>(&Bs[buf][kk][tn * TN + j]);
-          b[j] = v.x; b[j + 1] = v.y;
-        }
+        for (int j = 0; j < TJ; ++j) b[j] = Bs[buf][wn * WN + j * 8 + fr][ks + fk];
 #pragma unroll
-        for (int i = 0; i < TM; ++i)
+        for (int i = 0; i < TI; ++i)
 #pragma unroll
-          for (int j = 0; j < TN; ++j) acc[i][j] = fma(a[i], b[j], acc[i][j]);
+          for (int j = 0; j < TJ; ++j) dmma884(acc[i][j][0], acc[i][j][1], a[i], b[j]);
       }
       if (t + 1 < nk) store((t + 1) & 1);
       __syncthreads();
     }
   }
 #pragma unroll
-  for (int i = 0; i < TM; ++i)
+  for (int i = 0; i < TI; ++i)
 #pragma unroll
-    for (int j = 0; j < TN; ++j) {
-      const int r = m0 + tm * TM + i, c = n0 + tn * TN + j;
-      if (r < M && c < N) epi(r, c, acc[i][j]);
-    }
+    for (int j = 0; j < TJ; ++j)
+#pragma unroll
+      for (int h = 0; h < 2; ++h) {
+        const int r = m0 + wm * WM + i * 8 + fr, c = n0 + wn * WN + j * 8 + 2 * fk + h;
+        if (r < M && c < N) epi(r, c, acc[i][j][h]);
+      }
 }
 
-template <int BM, int BN, bool TA, bool TB, class Epi>
+template <int BM, int BN, int WM, int WN, bool TA, bool TB, class Epi>
 static fekf_status gemm_t(long long M, int N, int K, const double* A, int lda, const double* B, int ldb, Epi epi,
                           cudaStream_t s, const int* Mdev, const int* Kdev, int aug_m, int aug_k, int splits, int kps) {
-  constexpr size_t smem = sizeof(double) * 2 * GB_K * ((BM + 2) + (BN + 2));
+  constexpr size_t smem = sizeof(double) * 2 * GB_LDS * (BM + BN);
   static bool attr = false;
   if (!attr) {
-    FEKF_CHECK_CUDA(cudaFuncSetAttribute(dgemm_kernel<BM, BN, TA, TB, Epi>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                         (int)smem));
+    FEKF_CHECK_CUDA(cudaFuncSetAttribute(dgemm_kernel<BM, BN, WM, WN, TA, TB, Epi>,
+                                         cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
     attr = true;
   }
   dim3 grid((unsigned)cdiv(M, BM), (unsigned)cdiv(N, BN), (unsigned)splits);
-  dgemm_kernel<BM, BN, TA, TB, Epi><<<grid, 256, smem, s>>>((int)M, N, K, Mdev, Kdev, A, lda, B, ldb, aug_m, aug_k, kps, epi);
+  dgemm_kernel<BM, BN, WM, WN, TA, TB, Epi><<<grid, 256, smem, s>>>((int)M, N, K, Mdev, Kdev, A, lda, B, ldb, aug_m,
+                                                                     aug_k, kps, epi);
   FEKF_LAUNCH_CHECK();
   count_launch();
   return FEKF_OK;
 }
 
-// Tile choice: BN = 32 for N <= 32 (embedding widths 25/32), 128 for N >= 200 (fitting 240,
-// fitting W0 data-gradient 1600), else 64; BM = 128 when there are many rows, 64 otherwise.
+// Tile choice from (M, N): N <= 32 -> 128x32 (embedding widths 25/32); few rows -> 64x64 (more CTAs
+// for the fitting nets' 2048..8192 rows); otherwise 128x64.
 template <bool TA, bool TB, class Epi>
 static fekf_status gemm(long long M, int N, int K, const double* A, int lda, const double* B, int ldb, Epi epi,
                         cudaStream_t s, const int* Mdev = nullptr, const int* Kdev = nullptr, int aug_m = -1,
                         int aug_k = 0, int splits = 1, int kps = 0) {
   if (M <= 0 || N <= 0) return FEKF_OK;
   if (kps <= 0) kps = K;
-  const bool tallM = M >= 4096;
-  if (N <= 32)
-    return tallM ? gemm_t<128, 32, TA, TB>(M, N, K, A, lda, B, ldb, epi, s, Mdev, Kdev, aug_m, aug_k, splits, kps)
-                 : gemm_t<64, 32, TA, TB>(M, N, K, A, lda, B, ldb, epi, s, Mdev, Kdev, aug_m, aug_k, splits, kps);
-  if (N >= 200 && tallM)
-    return gemm_t<64, 128, TA, TB>(M, N, K, A, lda, B, ldb, epi, s, Mdev, Kdev, aug_m, aug_k, splits, kps);
-  return tallM ? gemm_t<128, 64, TA, TB>(M, N, K, A, lda, B, ldb, epi, s, Mdev, Kdev, aug_m, aug_k, splits, kps)
-               : gemm_t<64, 64, TA, TB>(M, N, K, A, lda, B, ldb, epi, s, Mdev, Kdev, aug_m, aug_k, splits, kps);
+  if (N <= 32) return gemm_t<128, 32, 32, 16, TA, TB>(M, N, K, A, lda, B, ldb, epi, s, Mdev, Kdev, aug_m, aug_k, splits, kps);
+  if (M < 16384 || N <= 64)
+    return gemm_t<64, 64, 32, 16, TA, TB>(M, N, K, A, lda, B, ldb, epi, s, Mdev, Kdev, aug_m, aug_k, splits, kps);
+  return gemm_t<128, 64, 32, 32, TA, TB>(M, N, K, A, lda, B, ldb, epi, s, Mdev, Kdev, aug_m, aug_k, splits, kps);
 }
 
 }  // namespace fekf

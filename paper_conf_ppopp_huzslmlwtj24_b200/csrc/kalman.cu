@@ -410,7 +410,7 @@ __global__ void kf_finish_kernel(const double* __restrict__ dotp, long long n_tc
     double gtu = tot[0];
     for (int k = 0; k < K; ++k) {
       const double d = tot[1 + k];
-      st->cu[k] = sig * st->beta[k] * d;
+      st->cu[k] = st->beta[k] * d;
       gtu -= st->beta[k] * d * d;
     }
     gtu *= sig;
@@ -584,10 +584,11 @@ fekf_status Kf::create(const std::vector<int>& blocks, const fekf_opt_cfg& o, fe
   return FEKF_OK;
 }
 
-fekf_status Kf::timing_ctl(int mode, double* total_ms, int64_t* launches) {
+fekf_status Kf::timing_ctl(int mode, double* total_ms, int64_t* launches, int64_t* rw_launches) {
   if (mode == 1) {
     timing = true;
     ev_used = 0;
+    ev_rw.clear();
     return FEKF_OK;
   }
   timing = false;
@@ -600,6 +601,11 @@ fekf_status Kf::timing_ctl(int mode, double* total_ms, int64_t* launches) {
   }
   if (total_ms) *total_ms = tot;
   if (launches) *launches = (int64_t)(ev_used / 2);
+  if (rw_launches) {
+    int64_t n = 0;
+    for (char c : ev_rw) n += c;
+    *rw_launches = n;
+  }
   return FEKF_OK;
 }
 
@@ -638,6 +644,7 @@ fekf_status Kf::pass(const double* g, bool rw, cudaStream_t s) {
     if (timing) {
       FEKF_CHECK_CUDA(cudaEventRecord(ev[ev_used + 1], s));
       ev_used += 2;
+      ev_rw.push_back(rw ? 1 : 0);
     }
   }
   kf_reduce_u_kernel<<<cdiv(p.n_tc, 4), 256, 0, s>>>(ws.as<double>(), csr_ptr.as<long long>(),

@@ -27,7 +27,7 @@ struct KfState {
   double A_last, coef_w;       // last A and sqrt(bs) * ABE * A
   double sig_cur;              // sigma used to form the current u
   double beta[KMAX];           // deferred coefficients
-  double cu[KMAX];             // sigma * beta_k * (u_k . g) of the current update
+  double cu[KMAX];             // beta_k * (u_k . g) of the current update
   long long t;
   int npend, flags, slot, pad_;
 };
@@ -61,8 +61,9 @@ struct Kf {
   bool timing = false;
   std::vector<cudaEvent_t> ev;   // [start, stop] per timed pass launch
   size_t ev_used = 0;
+  std::vector<char> ev_rw;       // 1 = read-write pass
   long long rw_passes = 0, r_passes = 0;
-  fekf_status timing_ctl(int mode, double* total_ms, int64_t* launches);
+  fekf_status timing_ctl(int mode, double* total_ms, int64_t* launches, int64_t* rw_launches);
   fekf_status create(const std::vector<int>& blocks, const fekf_opt_cfg& o, fekf_comm* c);
   ~Kf();
   fekf_status pass(const double* g, bool rw, cudaStream_t s);

@@ -63,7 +63,7 @@ def lib():
         "fekf_kf_get_state": ([vp, C.POINTER(dbl), C.POINTER(dbl), C.POINTER(i32)], i32),
         "fekf_kf_info": ([vp, C.POINTER(i64), C.POINTER(i64), C.POINTER(i64), C.POINTER(i64)], i32),
         "fekf_kf_pass": ([vp, vp, vp], i32),
-        "fekf_kf_timing": ([vp, i32, C.POINTER(dbl), C.POINTER(i64)], i32),
+        "fekf_kf_timing": ([vp, i32, C.POINTER(dbl), C.POINTER(i64), C.POINTER(i64)], i32),
         "fekf_create": ([C.POINTER(ModelCfg), C.POINTER(OptCfg), i32, vp, i32, i32, vp, C.POINTER(vp)], i32),
         "fekf_destroy": ([vp], i32), "fekf_param_count": ([vp, C.POINTER(i64)], i32),
         "fekf_get_kf": ([vp, C.POINTER(vp)], i32), "fekf_set_params": ([vp, vp, vp], i32),
@@ -264,10 +264,10 @@ class KalmanFilter:
         return {"p_bytes_local": a.value, "tiles_local": b.value, "n_pad": c.value, "items_local": d.value}
 
     def timing(self, enable):
-        """enable=True: start recording P-pass kernel times; False: stop, return (total_ms, launches)."""
-        ms, n = C.c_double(), C.c_int64()
-        _check(lib().fekf_kf_timing(self.h, 1 if enable else 0, C.byref(ms), C.byref(n)))
-        return ms.value, n.value
+        """enable=True: start recording P-pass kernel times; False: stop, return (total_ms, launches, rw_launches)."""
+        ms, n, rw = C.c_double(), C.c_int64(), C.c_int64()
+        _check(lib().fekf_kf_timing(self.h, 1 if enable else 0, C.byref(ms), C.byref(n), C.byref(rw)))
+        return ms.value, n.value, rw.value
 
     def close(self):
         if self._own and self.h:
