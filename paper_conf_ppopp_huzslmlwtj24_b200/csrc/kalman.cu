@@ -383,36 +383,45 @@ __global__ void kf_dot_kernel(const double* __restrict__ gpad, const double* __r
   }
 }
 
-// With P_t = sigma (B - sum_k beta_k u_k u_k^T):  u_t = P_t g = sigma (u_B - sum_k beta_k (u_k . g) u_k),
+// Per block i (P is block-diagonal; the deferred terms live inside each block):
+//   P_t,i = sigma (B_i - sum_k beta_k u_k,i u_k,i^T)  =>  u_t,i = sigma (u_B,i - sum_k beta_k d_k,i u_k,i),
+//   d_k,i = u_k,i . g_i, and g^T u_t = sigma sum_i (g_i . u_B,i - sum_k beta_k d_k,i^2).
+// kf_block_dot_kernel: dblk[k][i] = sum of the tile-column partials of block i (fixed order).
+__global__ void kf_block_dot_kernel(const double* __restrict__ dotp, long long n_tc, int K, int L,
+                                    const long long* __restrict__ tcoff, double* __restrict__ dblk) {
+  const int e = blockIdx.x * blockDim.x + threadIdx.x;
+  if (e >= (K + 1) * L) return;
+  const int k = e / L, i = e % L;
+  double a = 0.0;
+  for (long long tc = tcoff[i]; tc < tcoff[i + 1]; ++tc) a += dotp[(size_t)k * n_tc + tc];
+  dblk[e] = a;
+}
+
 // A = 1/(c + g^T u_t) (Alg. 1 line 8, c = L*lambda or lambda), K = A u_t (line 9),
-// P_{t+1} = (P_t - A u_t u_t^T)/lambda (line 10)  =>  append beta = A/sigma, sigma <- sigma/lambda;
+// P_{t+1} = (P_t - A u_t u_t^T)/lambda blockwise (line 10)  =>  append beta = A/sigma, sigma <- sigma/lambda;
 // lambda <- nu lambda + 1 - nu (line 12, Eq. 3); w += sqrt(bs) ABE K (line 13, Eq. 2).
 // rw: the pass just rewrote B = P_t, so sigma = 1 and the deferred list is empty.
-__global__ void kf_finish_kernel(const double* __restrict__ dotp, long long n_tc, int K, int rw, KfState* st,
-                                 const double* abe, double sqrt_bs) {
-  __shared__ double red[1 + KMAX][128];
-  __shared__ double tot[1 + KMAX];
-  for (int k = 0; k <= K; ++k) {
-    double a = 0.0;
-    for (long long i = threadIdx.x; i < n_tc; i += blockDim.x) a += dotp[(size_t)k * n_tc + i];
-    red[k][threadIdx.x] = a;
+__global__ void kf_finish_kernel(const double* __restrict__ dblk, int L, int K, int rw, KfState* st,
+                                 double* __restrict__ cub, const double* abe, double sqrt_bs) {
+  __shared__ double red[256];
+  double a = 0.0;
+  for (int i = threadIdx.x; i < L; i += blockDim.x) {
+    double v = dblk[i];
+    for (int k = 0; k < K; ++k) {
+      const double d = dblk[(size_t)(k + 1) * L + i];
+      const double bd = st->beta[k] * d;
+      cub[(size_t)k * L + i] = bd;
+      v -= bd * d;
+    }
+    a += v;
   }
-  __syncthreads();
-  if (threadIdx.x <= (unsigned)K) {
-    double a = 0.0;
-    for (int i = 0; i < (int)blockDim.x; ++i) a += red[threadIdx.x][i];
-    tot[threadIdx.x] = a;
-  }
+  red[threadIdx.x] = a;
   __syncthreads();
   if (threadIdx.x == 0) {
     const double lam = st->lambda;
     const double sig = rw ? 1.0 : st->sigma;
-    double gtu = tot[0];
-    for (int k = 0; k < K; ++k) {
-      const double d = tot[1 + k];
-      st->cu[k] = st->beta[k] * d;
-      gtu -= st->beta[k] * d * d;
-    }
+    double gtu = 0.0;
+    for (int t = 0; t < (int)blockDim.x; ++t) gtu += red[t];
     gtu *= sig;
     const double A = 1.0 / (st->c_mult * lam + gtu);
     const double e = abe ? *abe : 0.0;
@@ -430,18 +439,18 @@ __global__ void kf_finish_kernel(const double* __restrict__ dotp, long long n_tc
   }
 }
 
-// u_t = sigma (u_B - sum_k cu_k u_k) -> deferred slot; w += sqrt(bs) ABE A u_t
-__global__ void kf_vec_kernel(const double* __restrict__ ub, double* __restrict__ ulist, long long npad, int K,
-                              const KfState* st, double* __restrict__ w, const int* tc_blk, const int* tc_c,
-                              const long long* off, const int* nblk) {
+// u_t = sigma (u_B - sum_k beta_k d_k,i u_k) -> deferred slot; w += sqrt(bs) ABE A u_t
+__global__ void kf_vec_kernel(const double* __restrict__ ub, double* __restrict__ ulist, long long npad, int K, int L,
+                              const double* __restrict__ cub, const KfState* st, double* __restrict__ w,
+                              const int* tc_blk, const int* tc_c, const long long* off, const int* nblk) {
   const long long p = (long long)blockIdx.x * blockDim.x + threadIdx.x;
   if (p >= npad) return;
-  double v = ub[p];
-  for (int k = 0; k < K; ++k) v -= st->cu[k] * ulist[(size_t)k * npad + p];
-  v *= st->sig_cur;
-  ulist[(size_t)st->slot * npad + p] = v;
   const long long tc = p / KT;
   const int b = tc_blk[tc];
+  double v = ub[p];
+  for (int k = 0; k < K; ++k) v -= cub[(size_t)k * L + b] * ulist[(size_t)k * npad + p];
+  v *= st->sig_cur;
+  ulist[(size_t)st->slot * npad + p] = v;
   const int loc = tc_c[tc] * KT + (int)(p % KT);
   if (loc < nblk[b]) w[off[b] + loc] += st->coef_w * v;
 }
@@ -558,6 +567,10 @@ fekf_status Kf::create(const std::vector<int>& blocks, const fekf_opt_cfg& o, fe
   FEKF_TRY(dalloc(n_d, p.L * sizeof(int)));
   FEKF_TRY(dalloc(state, sizeof(KfState)));
   FEKF_TRY(dalloc(counter, sizeof(int)));
+  FEKF_TRY(dalloc(tcoff_d, (p.L + 1) * sizeof(long long)));
+  FEKF_TRY(dalloc(dblk, (size_t)(1 + KMAX) * p.L * sizeof(double)));
+  FEKF_TRY(dalloc(cub, (size_t)KMAX * p.L * sizeof(double)));
+  FEKF_CHECK_CUDA(cudaMemcpy(tcoff_d.p, p.tc_off.data(), (p.L + 1) * sizeof(long long), cudaMemcpyHostToDevice));
   if (!p.items.empty())
     FEKF_CHECK_CUDA(cudaMemcpy(items_d.p, p.items.data(), p.items.size() * sizeof(ItemD), cudaMemcpyHostToDevice));
   FEKF_CHECK_CUDA(cudaMemcpy(csr_ptr.p, p.csr_ptr.data(), (p.n_tc + 1) * sizeof(long long), cudaMemcpyHostToDevice));
@@ -612,7 +625,7 @@ fekf_status Kf::timing_ctl(int mode, double* total_ms, int64_t* launches, int64_
 Kf::~Kf() {
   for (cudaEvent_t e : ev) cudaEventDestroy(e);
   for (DBuf* b : {&P, &items_d, &ws, &gpad, &ub, &ulist, &dotp, &csr_ptr, &csr_idx, &tc_blk, &tc_c, &off_d, &n_d,
-                  &state, &counter})
+                  &state, &counter, &tcoff_d, &dblk, &cub})
     dfree(*b);
 }
 
@@ -665,13 +678,17 @@ fekf_status Kf::update(const double* g, const double* abe, double sqrt_bs, doubl
   kf_dot_kernel<<<cdiv(p.n_tc, 8), 256, 0, s>>>(gpad.as<double>(), ub.as<double>(), ulist.as<double>(), p.Npad, K,
                                                 p.n_tc, dotp.as<double>());
   FEKF_LAUNCH_CHECK();
-  kf_finish_kernel<<<1, 128, 0, s>>>(dotp.as<double>(), p.n_tc, K, rw ? 1 : 0, state.as<KfState>(), abe, sqrt_bs);
+  kf_block_dot_kernel<<<cdiv((K + 1) * p.L, 128), 128, 0, s>>>(dotp.as<double>(), p.n_tc, K, p.L,
+                                                                 tcoff_d.as<long long>(), dblk.as<double>());
   FEKF_LAUNCH_CHECK();
-  kf_vec_kernel<<<cdiv(p.Npad, 256), 256, 0, s>>>(ub.as<double>(), ulist.as<double>(), p.Npad, K, state.as<KfState>(),
-                                                   w, tc_blk.as<int>(), tc_c.as<int>(), off_d.as<long long>(),
-                                                   n_d.as<int>());
+  kf_finish_kernel<<<1, 256, 0, s>>>(dblk.as<double>(), p.L, K, rw ? 1 : 0, state.as<KfState>(), cub.as<double>(), abe,
+                                     sqrt_bs);
   FEKF_LAUNCH_CHECK();
-  count_launch(3);
+  kf_vec_kernel<<<cdiv(p.Npad, 256), 256, 0, s>>>(ub.as<double>(), ulist.as<double>(), p.Npad, K, p.L, cub.as<double>(),
+                                                   state.as<KfState>(), w, tc_blk.as<int>(), tc_c.as<int>(),
+                                                   off_d.as<long long>(), n_d.as<int>());
+  FEKF_LAUNCH_CHECK();
+  count_launch(4);
   npend = (rw ? 0 : npend) + 1;
   return FEKF_OK;
 }

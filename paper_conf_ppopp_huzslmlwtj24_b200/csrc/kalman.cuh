@@ -27,7 +27,6 @@ struct KfState {
   double A_last, coef_w;       // last A and sqrt(bs) * ABE * A
   double sig_cur;              // sigma used to form the current u
   double beta[KMAX];           // deferred coefficients
-  double cu[KMAX];             // beta_k * (u_k . g) of the current update
   long long t;
   int npend, flags, slot, pad_;
 };
@@ -58,6 +57,7 @@ struct Kf {
   int defer = 1;                 // corrections deferred before P is rewritten (1 = rewrite every update)
   int npend = 0;                 // host mirror of the device npend
   DBuf P, items_d, ws, gpad, ub, ulist, dotp, csr_ptr, csr_idx, tc_blk, tc_c, off_d, n_d, state, counter;
+  DBuf tcoff_d, dblk, cub;       // block -> tile-column offsets, per-block dots, per-block coefficients
   bool timing = false;
   std::vector<cudaEvent_t> ev;   // [start, stop] per timed pass launch
   size_t ev_used = 0;

@@ -95,7 +95,7 @@ def test_forward_energy_force_virial(name, nb):
     assert rel(v.cpu().reshape(-1, 3, 3), V) < 1e-12
 
 
-@pytest.mark.parametrize("name,nb", CASES[:3])
+@pytest.mark.parametrize("name,nb", CASES)
 def test_energy_jacobian(name, nb):
     wl, m, ds, w, ctx = _setup(name, nb)
     g, s = ctx.energy_jacobian(cu(ds["coord"]), cu(ds["box"]), cu(ds["energy"]))
@@ -105,7 +105,7 @@ def test_energy_jacobian(name, nb):
     assert abs(float(s.cpu()[0]) - sr) <= 1e-13 * max(1.0, abs(sr))
 
 
-@pytest.mark.parametrize("name,nb", CASES[:3])
+@pytest.mark.parametrize("name,nb", CASES)
 def test_force_jacobian(name, nb):
     wl, m, ds, w, ctx = _setup(name, nb)
     atoms = force_groups(len(ds["types"]), 0, 5)[0]
@@ -146,6 +146,38 @@ def test_kalman_updates(blocks, noise_mode, p_defer):
     kf.flush()
     for b in range(len(blocks)):
         assert rel(kf.get_block(b).cpu(), st.P[b]) < 1e-12
+
+
+def test_kalman_full_size_sampled_blocks():
+    """Bench-size Kalman filter (water-64: 110 blocks, 39 GiB packed P, default p_defer): one update
+    checked on sampled blocks against the update recomputed in numpy from the GPU's previous P
+    (P_new = (P - A u u^T)/lambda with u = P g per block; w increment sqrt(bs) ABE A u)."""
+    wl = get_config("c2_water64")
+    _, blocks = fk.plan_layout(wl.model, wl.opt.block_size)
+    assert len(blocks) == 110
+    kf = fk.KalmanFilter(blocks, dict(block_size=wl.opt.block_size))
+    N = sum(blocks)
+    off = np.concatenate([[0], np.cumsum(blocks)])
+    gen = torch.Generator(device="cuda").manual_seed(3)
+    w = torch.zeros(N, dtype=torch.float64, device="cuda")
+    abe = torch.full((1,), 0.05, dtype=torch.float64, device="cuda")
+    for _ in range(7):   # crosses one read-write pass (p_defer = 5)
+        kf.update(torch.randn(N, dtype=torch.float64, device="cuda", generator=gen), abe, 4.0, w)
+    sample = [0, 37, 109]
+    before = {b: kf.get_block(b).cpu().numpy() for b in sample}
+    lam = kf.state()["lambda"]
+    w0 = w.cpu().numpy()
+    g = torch.randn(N, dtype=torch.float64, device="cuda", generator=gen)
+    kf.update(g, abe, 4.0, w)
+    A = kf.state()["A"]
+    assert np.isfinite(A) and A > 0
+    gn, w1 = g.cpu().numpy(), w.cpu().numpy()
+    for b in sample:
+        sl = slice(off[b], off[b + 1])
+        u = before[b] @ gn[sl]
+        ref = (before[b] - A * np.outer(u, u)) / lam
+        assert rel(kf.get_block(b).cpu(), ref) < 1e-11
+        assert rel(w1[sl] - w0[sl], 4.0 * 0.05 * A * u) < 1e-11
 
 
 @pytest.mark.parametrize("name,steps", [("c1_cu32", 10), ("t2_tiny", 4)])
