@@ -74,9 +74,20 @@ dgemm_kernel(int M, int N, int K, const int* __restrict__ Mdev, const int* __res
   static_assert((BM / WM) * NWN == 8, "8 warps");
   constexpr int TI = WM / 8, TJ = WN / 8;
   constexpr int AE = BM * GB_K / 256, BE = BN * GB_K / 256;
+  // SMEM layout follows the operand's global layout so every store is contiguous: k-contiguous
+  // [mn][GB_LDS] (A row-major / B given as [N x K]) or mn-contiguous [k][MN + 4] (A given as [K x M] /
+  // B row-major [K x N]).  Both strides make the 8x4 DMMA fragment loads bank-conflict free.
+  constexpr int ASZ = TA ? GB_K * (BM + 4) : BM * GB_LDS;
+  constexpr int BSZ = TB ? BN * GB_LDS : GB_K * (BN + 4);
   extern __shared__ __align__(16) double gsm[];
-  auto As = reinterpret_cast<double (*)[BM][GB_LDS]>(gsm);
-  auto Bs = reinterpret_cast<double (*)[BN][GB_LDS]>(gsm + 2 * BM * GB_LDS);
+  double* As0 = gsm;
+  double* Bs0 = gsm + 2 * ASZ;
+  auto a_at = [&](int buf, int m, int k) -> double& {
+    return TA ? As0[buf * ASZ + k * (BM + 4) + m] : As0[buf * ASZ + m * GB_LDS + k];
+  };
+  auto b_at = [&](int buf, int n, int k) -> double& {
+    return TB ? Bs0[buf * BSZ + n * GB_LDS + k] : Bs0[buf * BSZ + k * (BN + 4) + n];
+  };
   if (Mdev) M = min(M, *Mdev);
   if (Kdev) {
     const int kd = *Kdev;
@@ -126,12 +137,12 @@ dgemm_kernel(int M, int N, int K, const int* __restrict__ Mdev, const int* __res
 #pragma unroll
     for (int q = 0; q < AE; ++q) {
       const int idx = tid + 256 * q;
-      if (!TA) As[buf][idx / GB_K][idx % GB_K] = ra[q]; else As[buf][idx % BM][idx / BM] = ra[q];
+      if (!TA) a_at(buf, idx / GB_K, idx % GB_K) = ra[q]; else a_at(buf, idx % BM, idx / BM) = ra[q];
     }
 #pragma unroll
     for (int q = 0; q < BE; ++q) {
       const int idx = tid + 256 * q;
-      if (!TB) Bs[buf][idx % BN][idx / BN] = rb[q]; else Bs[buf][idx / GB_K][idx % GB_K] = rb[q];
+      if (!TB) b_at(buf, idx % BN, idx / BN) = rb[q]; else b_at(buf, idx / GB_K, idx % GB_K) = rb[q];
     }
   };
   const int nk = kend > kbeg ? (kend - kbeg + GB_K - 1) / GB_K : 0;
@@ -146,9 +157,9 @@ dgemm_kernel(int M, int N, int K, const int* __restrict__ Mdev, const int* __res
       for (int ks = 0; ks < GB_K; ks += 4) {
         double a[TI], b[TJ];
 #pragma unroll
-        for (int i = 0; i < TI; ++i) a[i] = As[buf][wm * WM + i * 8 + fr][ks + fk];
+        for (int i = 0; i < TI; ++i) a[i] = a_at(buf, wm * WM + i * 8 + fr, ks + fk);
 #pragma unroll
-        for (int j = 0; j < TJ; ++j) b[j] = Bs[buf][wn * WN + j * 8 + fr][ks + fk];
+        for (int j = 0; j < TJ; ++j) b[j] = b_at(buf, wn * WN + j * 8 + fr, ks + fk);
 #pragma unroll
         for (int i = 0; i < TI; ++i)
 #pragma unroll
@@ -172,7 +183,9 @@ dgemm_kernel(int M, int N, int K, const int* __restrict__ Mdev, const int* __res
 template <int BM, int BN, int WM, int WN, bool TA, bool TB, class Epi>
 static fekf_status gemm_t(long long M, int N, int K, const double* A, int lda, const double* B, int ldb, Epi epi,
                           cudaStream_t s, const int* Mdev, const int* Kdev, int aug_m, int aug_k, int splits, int kps) {
-  constexpr size_t smem = sizeof(double) * 2 * GB_LDS * (BM + BN);
+  constexpr size_t asz = TA ? GB_K * (BM + 4) : BM * GB_LDS;
+  constexpr size_t bsz = TB ? BN * GB_LDS : GB_K * (BN + 4);
+  constexpr size_t smem = sizeof(double) * 2 * (asz + bsz);
   static bool attr = false;
   if (!attr) {
     FEKF_CHECK_CUDA(cudaFuncSetAttribute(dgemm_kernel<BM, BN, WM, WN, TA, TB, Epi>,
