@@ -175,33 +175,34 @@ __device__ __forceinline__ void consumer_bar() { asm volatile("bar.sync 1, 256;"
 // ------------------------------------------------------------------------------------------------
 // the P pass
 // ------------------------------------------------------------------------------------------------
-constexpr int STAGES = 5;
+constexpr int MAX_STAGES = 8;
 constexpr int TILE_ELEMS = KT * KT;
 constexpr uint32_t TILE_BYTES = TILE_ELEMS * sizeof(double);
-constexpr int VEC_ELEMS = 2 * KMAX * KT;   // per stage: u_k[I-rows] and u_k[J-cols] for k < K
-constexpr int STAGE_ELEMS = TILE_ELEMS + VEC_ELEMS;
 constexpr int PASS_THREADS = 288;  // 8 consumer warps + 1 producer warp
-constexpr size_t PASS_SMEM = (size_t)STAGES * STAGE_ELEMS * sizeof(double) + 2 * 8 * KT * sizeof(double) +
-                             2 * STAGES * sizeof(uint64_t) + STAGES * sizeof(int4);
+constexpr size_t PASS_SMEM = 227 * 1024;
+// [full[8] | empty[8] | meta[8]] (256 B), column-reduction buffers (8 KiB), then the stage ring; a stage
+// is one tile plus, for a read-write pass, the 2K vector segments (u_k rows I, u_k columns J) it needs.
+constexpr size_t PASS_HDR = 2 * MAX_STAGES * sizeof(uint64_t) + MAX_STAGES * sizeof(int4) + 2 * 8 * KT * sizeof(double);
 
 // rw = 0: read-only pass, u_B = B g.  rw = 1: B <- sigma (B - sum_{k<K} beta_k u_k u_k^T) written back,
 // then u_B = B_new g.  Tile-row segments are pulled from an atomic counter by a producer warp that
-// streams each 32 KiB tile (and, for rw, the 2K 512-byte vector segments it needs) with TMA bulk copies.
+// streams each 32 KiB tile (and, for rw, the 2K 512-byte vector segments it needs) with TMA bulk copies
+// into a ring of `nst` stages (6 for read-only passes, 5 when 5 corrections ride along).
 __global__ void __launch_bounds__(PASS_THREADS, 1)
 kf_pass_kernel(double* __restrict__ P, const ItemD* __restrict__ items, int n_items, int* counter,
                const double* __restrict__ gpad, const double* __restrict__ ulist, long long npad, int rw, int K,
-               const KfState* st, double* __restrict__ ws) {
+               int nst, int stage_elems, const KfState* st, double* __restrict__ ws) {
   extern __shared__ __align__(128) unsigned char smem[];
-  double* stages = reinterpret_cast<double*>(smem);
-  double* colred = stages + STAGES * STAGE_ELEMS;
-  uint64_t* full = reinterpret_cast<uint64_t*>(colred + 2 * 8 * KT);
-  uint64_t* empty = full + STAGES;
-  int4* meta = reinterpret_cast<int4*>(empty + STAGES);
+  uint64_t* full = reinterpret_cast<uint64_t*>(smem);
+  uint64_t* empty = full + MAX_STAGES;
+  int4* meta = reinterpret_cast<int4*>(empty + MAX_STAGES);
+  double* colred = reinterpret_cast<double*>(meta + MAX_STAGES);
+  double* stages = colred + 2 * 8 * KT;
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   if (!rw) K = 0;
 
   if (tid == 0) {
-    for (int s = 0; s < STAGES; ++s) {
+    for (int s = 0; s < nst; ++s) {
       mbar_init(&full[s], 1);
       mbar_init(&empty[s], 1);
     }
@@ -222,16 +223,16 @@ kf_pass_kernel(double* __restrict__ P, const ItemD* __restrict__ items, int n_it
         for (int t = 0; t < it.nJ; ++t) {
           mbar_wait(&empty[s], ph ^ 1);
           meta[s] = make_int4(itx, it.J0 + t, (t == 0 ? 1 : 0) | (t == it.nJ - 1 ? 2 : 0), 0);
-          double* st_s = stages + (size_t)s * STAGE_ELEMS;
+          double* st_s = stages + (size_t)s * stage_elems;
           mbar_arrive_tx(&full[s], bytes);
           tma_load_1d(st_s, P + (size_t)(it.tile_off + t) * TILE_ELEMS, TILE_BYTES, &full[s]);
           for (int k = 0; k < K; ++k) {
             const double* uk = ulist + (size_t)k * npad + it.vbase;
             tma_load_1d(st_s + TILE_ELEMS + k * KT, uk + (size_t)it.I * KT, KT * sizeof(double), &full[s]);
-            tma_load_1d(st_s + TILE_ELEMS + (KMAX + k) * KT, uk + (size_t)(it.J0 + t) * KT, KT * sizeof(double),
+            tma_load_1d(st_s + TILE_ELEMS + (K + k) * KT, uk + (size_t)(it.J0 + t) * KT, KT * sizeof(double),
                         &full[s]);
           }
-          if (++s == STAGES) { s = 0; ph ^= 1; }
+          if (++s == nst) { s = 0; ph ^= 1; }
         }
       }
       mbar_wait(&empty[s], ph ^ 1);
@@ -268,9 +269,9 @@ kf_pass_kernel(double* __restrict__ P, const ItemD* __restrict__ items, int n_it
       }
     }
     const double2 gJ = __ldg(reinterpret_cast<const double2*>(gpad + it.vbase + (long long)J * KT + c0));
-    double* t = stages + (size_t)s * STAGE_ELEMS;
+    double* t = stages + (size_t)s * stage_elems;
     const double* vI = t + TILE_ELEMS;
-    const double* vJ = t + TILE_ELEMS + KMAX * KT;
+    const double* vJ = t + TILE_ELEMS + K * KT;
     double ca0 = 0.0, ca1 = 0.0;
 #pragma unroll
     for (int q = 0; q < 8; ++q) {
@@ -330,7 +331,7 @@ kf_pass_kernel(double* __restrict__ P, const ItemD* __restrict__ items, int n_it
         if (lane == 0) ws[(size_t)it.row_slot * KT + warp + 8 * q] = v;
       }
     }
-    if (++s == STAGES) { s = 0; ph ^= 1; }
+    if (++s == nst) { s = 0; ph ^= 1; }
     ++tcount;
   }
   if (tid == 0) {
@@ -647,10 +648,13 @@ fekf_status Kf::pass(const double* g, bool rw, cudaStream_t s) {
       }
       FEKF_CHECK_CUDA(cudaEventRecord(ev[ev_used], s));
     }
+    const int K = rw ? npend : 0;
+    const int stage_elems = TILE_ELEMS + 2 * K * KT;
+    const int nst = (int)std::min<size_t>(MAX_STAGES, (PASS_SMEM - PASS_HDR) / (stage_elems * sizeof(double)));
     kf_pass_kernel<<<grid, PASS_THREADS, PASS_SMEM, s>>>(P.as<double>(), items_d.as<ItemD>(), (int)p.items.size(),
                                                           counter.as<int>(), gpad.as<double>(), ulist.as<double>(),
-                                                          p.Npad, rw ? 1 : 0, rw ? npend : 0, state.as<KfState>(),
-                                                          ws.as<double>());
+                                                          p.Npad, rw ? 1 : 0, K, nst, stage_elems,
+                                                          state.as<KfState>(), ws.as<double>());
     FEKF_LAUNCH_CHECK();
     count_launch();
     if (rw) ++rw_passes; else ++r_passes;
