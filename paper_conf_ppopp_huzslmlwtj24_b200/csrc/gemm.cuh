@@ -59,6 +59,35 @@ struct EpiDgrad {
   }
 };
 
+// data gradient fused with the previous layer's activation adjoint (embedding, no timestep):
+//   hbar_prev = Zbar W^T + skip^T(hbar);  zbar_prev = (1 - y^2) hbar_prev [- 2 y ydot hdotbar_prev]
+// primal launch: the tangent rows of the same layer are done first (tpos / Yt / Hbt);
+// tangent launch: y of the primal row rowmap[r].
+struct EpiDgradAct {
+  double* out; int ldo; const double* Hb; int ld; int skip; int dprev;
+  const double* Y; double* Zb;
+  const int* tpos; const double* Yt; const double* Hbt;
+  const int* rowmap;
+  __device__ void operator()(int r, int c, double v) const {
+    double s = 0.0;
+    if (skip == 1) s = Hb[(size_t)r * ld + c];
+    else if (skip == 2) s = Hb[(size_t)r * ld + c] + Hb[(size_t)r * ld + c + dprev];
+    const double hb = v + s;
+    const size_t o = (size_t)r * ldo + c;
+    out[o] = hb;
+    const double y = Y[(rowmap ? (size_t)rowmap[r] : (size_t)r) * ldo + c];
+    double z = (1.0 - y * y) * hb;
+    if (tpos) {
+      const int tr = tpos[r];
+      if (tr >= 0) {
+        const size_t ot = (size_t)tr * ldo + c;
+        z -= 2.0 * y * Yt[ot] * Hbt[ot];
+      }
+    }
+    Zb[o] = z;
+  }
+};
+
 __device__ __forceinline__ void dmma884(double& d0, double& d1, double a, double b) {
   asm volatile("mma.sync.aligned.m8n8k4.row.col.f64.f64.f64.f64 {%0,%1}, {%2}, {%3}, {%0,%1};"
                : "+d"(d0), "+d"(d1)

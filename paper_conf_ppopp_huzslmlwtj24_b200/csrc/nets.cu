@@ -501,6 +501,66 @@ __global__ void emb_seed_kernel(int Rmax, const int* __restrict__ Rdev, int M, i
   }
 }
 
+// Same as emb_seed_kernel, one CTA per centre atom for all its rows of every pair: the atom's Xbar
+// (and Xdotbar) are staged once in SMEM instead of being re-read for every (row, m).
+struct SeedPtrs {
+  const double* Y[NP];
+  const double* Yt[NP];
+  double* Hb[NP];
+  double* Zb[NP];
+  double* Hbt[NP];
+  double* Zbt[NP];
+};
+__global__ void __launch_bounds__(128)
+emb_seed_atom_kernel(Geo g, PairPtrs pp, SeedPtrs sp, const double* __restrict__ em, const double* __restrict__ rdot,
+                     const double* __restrict__ Xb, const double* __restrict__ Xdb, int dual) {
+  extern __shared__ double sm[];
+  const int M = g.M;
+  double* xb = sm;
+  double* xdb = sm + 4 * M;
+  const int atom = blockIdx.x;
+  const int b = atom / g.Na, i = atom % g.Na;
+  const int ti = g.types[i], k = g.tindex[i];
+  const int e = b * g.ncnt[ti] + k;
+  for (int q = threadIdx.x; q < 4 * M; q += blockDim.x) {
+    xb[q] = Xb[(size_t)atom * 4 * M + q];
+    if (dual) xdb[q] = Xdb[(size_t)atom * 4 * M + q];
+  }
+  __syncthreads();
+  const double inv = 1.0 / g.Nm;
+  for (int tj = 0; tj < g.nt; ++tj) {
+    const int p = ti * g.nt + tj;
+    const int r0 = pp.row_start[p][e], r1 = pp.row_start[p][e + 1];
+    const int n = (r1 - r0) * M;
+    for (int q = threadIdx.x; q < n; q += blockDim.x) {
+      const int s = q / M, m = q % M;
+      const int r = r0 + s;
+      const size_t idx = (size_t)atom * g.Nm + g.sec[tj] + s;
+      const double* rr = em + idx * 4;
+      double a = rr[0] * xb[m] + rr[1] * xb[M + m] + rr[2] * xb[2 * M + m] + rr[3] * xb[3 * M + m];
+      const size_t o = (size_t)r * M + m;
+      const double y = sp.Y[p][o];
+      const double t = 1.0 - y * y;
+      const int tr = dual ? pp.tpos[p][r] : -1;
+      if (tr >= 0) {
+        const double* rd = rdot + idx * 4;
+        a += rd[0] * xdb[m] + rd[1] * xdb[M + m] + rd[2] * xdb[2 * M + m] + rd[3] * xdb[3 * M + m];
+        const double ad = (rr[0] * xdb[m] + rr[1] * xdb[M + m] + rr[2] * xdb[2 * M + m] + rr[3] * xdb[3 * M + m]) * inv;
+        const size_t od = (size_t)tr * M + m;
+        sp.Hbt[p][od] = ad;
+        sp.Zbt[p][od] = t * ad;
+        a *= inv;
+        sp.Hb[p][o] = a;
+        sp.Zb[p][o] = t * a - 2.0 * y * sp.Yt[p][od] * ad;
+      } else {
+        a *= inv;
+        sp.Hb[p][o] = a;
+        sp.Zb[p][o] = t * a;
+      }
+    }
+  }
+}
+
 // prod_force / prod_virial: dE/dR~_row = G Xbar^T / N_m + sbar e_0 ; f = dE/dd = (dE/dR~) J ;
 // F_i += f, F_j -= f (F = -dE/dx), W -= d (x) f.  One CTA (4 warps) per centre atom: the
 // atom's own force and virial are reduced in the CTA (fixed order), only F_j needs atomics.
@@ -944,6 +1004,22 @@ fekf_status model_backward(Ctx& c, int nb, Mode mode, double* gout, cudaStream_t
   FEKF_LAUNCH_CHECK();
   count_launch();
   // ---- embedding nets (compacted rows; tangent rows separately) ----
+  {
+    SeedPtrs sp{};
+    for (size_t p = 0; p < c.pairs.size(); ++p) {
+      PairNet& P = c.pairs[p];
+      sp.Y[p] = P.Y.back().as<double>();
+      sp.Yt[p] = P.Yt.back().as<double>();
+      sp.Hb[p] = P.Hb.back().as<double>();
+      sp.Zb[p] = P.Zb.back().as<double>();
+      sp.Hbt[p] = P.Hbt.back().as<double>();
+      sp.Zbt[p] = P.Zbt.back().as<double>();
+    }
+    emb_seed_atom_kernel<<<nb * c.Na, 128, 8 * c.M * sizeof(double), s>>>(
+        g, pp, sp, c.em.as<double>(), c.rdot.as<double>(), c.Xb.as<double>(), c.Xb.as<double>() + Xoff, dual ? 1 : 0);
+    FEKF_LAUNCH_CHECK();
+    count_launch();
+  }
   for (size_t p = 0; p < c.pairs.size(); ++p) {
     PairNet& P = c.pairs[p];
     const long long Rmax = pair_rows(c, (int)p, nb);
@@ -951,21 +1027,10 @@ fekf_status model_backward(Ctx& c, int nb, Mode mode, double* gout, cudaStream_t
     const int* rc = rcount(c, (int)p);
     const int* tc = tcount(c, (int)p);
     const int nl = (int)P.L.size();
-    emb_seed_kernel<<<cdiv(Rmax * c.M, 256), 256, 0, s>>>(
-        (int)Rmax, rc, c.M, c.Nm, P.row_idx.as<int>(), P.tpos.as<int>(), c.em.as<double>(), c.rdot.as<double>(),
-        c.Xb.as<double>(), c.Xb.as<double>() + Xoff, dual ? 1 : 0, P.Y.back().as<double>(), P.Yt.back().as<double>(),
-        P.Hb.back().as<double>(), P.Zb.back().as<double>(), P.Hbt.back().as<double>(), P.Zbt.back().as<double>());
-    FEKF_LAUNCH_CHECK();
-    count_launch();
+    // Zbar of the last layer comes from emb_seed; every other layer's Zbar from the fused epilogue of
+    // the data-gradient GEMM one layer up (tangent rows first: the primal zbar needs their hdotbar)
     for (int l = nl - 1; l >= 0; --l) {
       const Layer& L = P.L[l];
-      if (l + 1 < nl) {  // the last layer's activation adjoint is fused into emb_seed
-        emb_act_bwd_kernel<<<cdiv(Rmax * L.dout, 256), 256, 0, s>>>(
-            (int)Rmax, rc, L.dout, P.Y[l].as<double>(), P.Hb[l].as<double>(), P.tpos.as<int>(), P.Yt[l].as<double>(),
-            P.Hbt[l].as<double>(), dual ? 1 : 0, P.Zb[l].as<double>(), P.Zbt[l].as<double>());
-        FEKF_LAUNCH_CHECK();
-        count_launch();
-      }
       if (want_w) {
         const double* Hp = l == 0 ? P.hin.as<double>() : P.H[l - 1].as<double>();
         const double* Hpt = l == 0 ? P.hin_t.as<double>() : P.Ht[l - 1].as<double>();
@@ -974,12 +1039,16 @@ fekf_status model_backward(Ctx& c, int nb, Mode mode, double* gout, cudaStream_t
                        gout + L.W, s));
       }
       if (l > 0) {
-        EpiDgrad e{P.Hb[l - 1].as<double>(), L.din, P.Hb[l].as<double>(), L.dout, L.skip, L.din};
-        FEKF_TRY(gemm<false, true>(Rmax, L.din, L.dout, P.Zb[l].as<double>(), L.dout, w + L.W, L.dout, e, s, rc));
         if (dual) {
-          EpiDgrad et{P.Hbt[l - 1].as<double>(), L.din, P.Hbt[l].as<double>(), L.dout, L.skip, L.din};
+          EpiDgradAct et{P.Hbt[l - 1].as<double>(), L.din, P.Hbt[l].as<double>(), L.dout, L.skip, L.din,
+                         P.Y[l - 1].as<double>(), P.Zbt[l - 1].as<double>(), nullptr, nullptr, nullptr,
+                         P.tidx.as<int>()};
           FEKF_TRY(gemm<false, true>(Rmax, L.din, L.dout, P.Zbt[l].as<double>(), L.dout, w + L.W, L.dout, et, s, tc));
         }
+        EpiDgradAct e{P.Hb[l - 1].as<double>(), L.din, P.Hb[l].as<double>(), L.dout, L.skip, L.din,
+                      P.Y[l - 1].as<double>(), P.Zb[l - 1].as<double>(), dual ? P.tpos.as<int>() : nullptr,
+                      P.Yt[l - 1].as<double>(), P.Hbt[l - 1].as<double>(), nullptr};
+        FEKF_TRY(gemm<false, true>(Rmax, L.din, L.dout, P.Zb[l].as<double>(), L.dout, w + L.W, L.dout, e, s, rc));
       } else if (mode == MODE_FORCE) {
         FEKF_TRY(gemm<false, true>(Rmax, 1, L.dout, P.Zb[0].as<double>(), L.dout, w + L.W, L.dout,
                                    EpiStore{P.sbar.as<double>(), 1}, s, rc));
