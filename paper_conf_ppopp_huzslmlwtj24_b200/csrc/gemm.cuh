@@ -238,6 +238,8 @@ static fekf_status gemm(long long M, int N, int K, const double* A, int lda, con
   if (M <= 0 || N <= 0) return FEKF_OK;
   if (kps <= 0) kps = K;
   if (N <= 32) return gemm_t<128, 32, 32, 16, TA, TB>(M, N, K, A, lda, B, ldb, epi, s, Mdev, Kdev, aug_m, aug_k, splits, kps);
+  if (M <= 8192 && !TA)  // fitting nets: few rows, keep >= 2 CTAs per SM busy
+    return gemm_t<32, 64, 8, 32, TA, TB>(M, N, K, A, lda, B, ldb, epi, s, Mdev, Kdev, aug_m, aug_k, splits, kps);
   if (M < 16384 || N <= 64)
     return gemm_t<64, 64, 32, 16, TA, TB>(M, N, K, A, lda, B, ldb, epi, s, Mdev, Kdev, aug_m, aug_k, splits, kps);
   return gemm_t<128, 64, 32, 32, TA, TB>(M, N, K, A, lda, B, ldb, epi, s, Mdev, Kdev, aug_m, aug_k, splits, kps);
