@@ -6,7 +6,7 @@
 //   Optional "ones" row aug_m of op(A): (k < aug_k ? 1 : 0), so [W-grad ; b-grad] = [H | 1]^T Zbar.
 //   Mdev / Kdev: device-resident row counts (compacted rows); CTAs past them exit.
 // CTA tile BM x BN x 16, 8 warps each WM x WN (WM/8 x WN/8 DMMA tiles), operands staged in SMEM
-// k-contiguous with a 20-double row stride (conflict-free fragment loads), register-staged double buffer.
+// k-contiguous with a 20-double row stride (conflict-free fragment loads), 3-stage cp.async ring.
 #pragma once
 #include "model.cuh"
 
@@ -94,6 +94,19 @@ __device__ __forceinline__ void dmma884(double& d0, double& d1, double a, double
                : "d"(a), "d"(b));
 }
 
+__device__ __forceinline__ void cp_async8(double* dst, const double* src, bool valid) {
+  const unsigned d = (unsigned)__cvta_generic_to_shared(dst);
+  const int n = valid ? 8 : 0;  // src-size 0: zero-fill
+  asm volatile("cp.async.ca.shared.global [%0], [%1], 8, %2;" ::"r"(d), "l"(src), "r"(n) : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+template <int N>
+__device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory"); }
+
+constexpr int GB_STAGES = 3;
+
+// Mainloop: GB_STAGES-deep cp.async ring (global -> SMEM without register staging), one
+// __syncthreads per BK slice, warp tiles of (WM/8) x (WN/8) DMMA 8x8 tiles.
 template <int BM, int BN, int WM, int WN, bool TA, bool TB, class Epi>
 __global__ void __launch_bounds__(256)
 dgemm_kernel(int M, int N, int K, const int* __restrict__ Mdev, const int* __restrict__ Kdev,
@@ -103,14 +116,15 @@ dgemm_kernel(int M, int N, int K, const int* __restrict__ Mdev, const int* __res
   static_assert((BM / WM) * NWN == 8, "8 warps");
   constexpr int TI = WM / 8, TJ = WN / 8;
   constexpr int AE = BM * GB_K / 256, BE = BN * GB_K / 256;
-  // SMEM layout follows the operand's global layout so every store is contiguous: k-contiguous
-  // [mn][GB_LDS] (A row-major / B given as [N x K]) or mn-contiguous [k][MN + 4] (A given as [K x M] /
-  // B row-major [K x N]).  Both strides make the 8x4 DMMA fragment loads bank-conflict free.
+  // SMEM layout follows the operand's global layout so consecutive threads copy consecutive
+  // addresses: k-contiguous [mn][GB_LDS] (A row-major / B given as [N x K]) or mn-contiguous
+  // [k][MN + 4] (A given as [K x M] / B row-major [K x N]).  Both strides make the 8x4 DMMA fragment
+  // loads bank-conflict free.
   constexpr int ASZ = TA ? GB_K * (BM + 4) : BM * GB_LDS;
   constexpr int BSZ = TB ? BN * GB_LDS : GB_K * (BN + 4);
   extern __shared__ __align__(16) double gsm[];
   double* As0 = gsm;
-  double* Bs0 = gsm + 2 * ASZ;
+  double* Bs0 = gsm + GB_STAGES * ASZ;
   auto a_at = [&](int buf, int m, int k) -> double& {
     return TA ? As0[buf * ASZ + k * (BM + 4) + m] : As0[buf * ASZ + m * GB_LDS + k];
   };
@@ -136,20 +150,21 @@ dgemm_kernel(int M, int N, int K, const int* __restrict__ Mdev, const int* __res
   for (int i = 0; i < TI; ++i)
 #pragma unroll
     for (int j = 0; j < TJ; ++j) acc[i][j][0] = acc[i][j][1] = 0.0;
-  double ra[AE], rb[BE];
-  auto load = [&](int k0) {
+  auto issue = [&](int buf, int k0) {
 #pragma unroll
     for (int q = 0; q < AE; ++q) {
       const int idx = tid + 256 * q;
       int r, kk;
       if (!TA) { r = idx / GB_K; kk = idx % GB_K; } else { kk = idx / BM; r = idx % BM; }
       const int m = m0 + r, k = k0 + kk;
-      double v = 0.0;
-      if (m < M && k < kend) {
-        if (m == aug_m) v = (k < aug_k) ? 1.0 : 0.0;
-        else v = TA ? __ldg(A + (size_t)k * lda + m) : __ldg(A + (size_t)m * lda + k);
+      double* dst = &a_at(buf, r, kk);
+      if (m == aug_m) {
+        *dst = (k < aug_k) ? 1.0 : 0.0;
+      } else {
+        const bool ok = m < M && k < kend;
+        const double* src = ok ? (TA ? A + (size_t)k * lda + m : A + (size_t)m * lda + k) : A;
+        cp_async8(dst, src, ok);
       }
-      ra[q] = v;
     }
 #pragma unroll
     for (int q = 0; q < BE; ++q) {
@@ -157,47 +172,38 @@ dgemm_kernel(int M, int N, int K, const int* __restrict__ Mdev, const int* __res
       int c, kk;
       if (!TB) { kk = idx / BN; c = idx % BN; } else { c = idx / GB_K; kk = idx % GB_K; }
       const int n = n0 + c, k = k0 + kk;
-      double u = 0.0;
-      if (n < N && k < kend) u = TB ? __ldg(B + (size_t)n * ldb + k) : __ldg(B + (size_t)k * ldb + n);
-      rb[q] = u;
-    }
-  };
-  auto store = [&](int buf) {
-#pragma unroll
-    for (int q = 0; q < AE; ++q) {
-      const int idx = tid + 256 * q;
-      if (!TA) a_at(buf, idx / GB_K, idx % GB_K) = ra[q]; else a_at(buf, idx % BM, idx / BM) = ra[q];
-    }
-#pragma unroll
-    for (int q = 0; q < BE; ++q) {
-      const int idx = tid + 256 * q;
-      if (!TB) b_at(buf, idx % BN, idx / BN) = rb[q]; else b_at(buf, idx / GB_K, idx % GB_K) = rb[q];
+      const bool ok = n < N && k < kend;
+      const double* src = ok ? (TB ? B + (size_t)n * ldb + k : B + (size_t)k * ldb + n) : B;
+      cp_async8(&b_at(buf, c, kk), src, ok);
     }
   };
   const int nk = kend > kbeg ? (kend - kbeg + GB_K - 1) / GB_K : 0;
-  if (nk > 0) {
-    load(kbeg);
-    store(0);
-    __syncthreads();
-    for (int t = 0; t < nk; ++t) {
-      if (t + 1 < nk) load(kbeg + (t + 1) * GB_K);
-      const int buf = t & 1;
 #pragma unroll
-      for (int ks = 0; ks < GB_K; ks += 4) {
-        double a[TI], b[TJ];
+  for (int st = 0; st < GB_STAGES - 1; ++st) {
+    if (st < nk) issue(st, kbeg + st * GB_K);
+    cp_async_commit();
+  }
+  for (int t = 0; t < nk; ++t) {
+    cp_async_wait<GB_STAGES - 2>();
+    __syncthreads();  // slice t visible to all; slice t-1's buffer free for reuse
+    const int tn = t + GB_STAGES - 1;
+    if (tn < nk) issue(tn % GB_STAGES, kbeg + tn * GB_K);
+    cp_async_commit();
+    const int buf = t % GB_STAGES;
 #pragma unroll
-        for (int i = 0; i < TI; ++i) a[i] = a_at(buf, wm * WM + i * 8 + fr, ks + fk);
+    for (int ks = 0; ks < GB_K; ks += 4) {
+      double a[TI], b[TJ];
 #pragma unroll
-        for (int j = 0; j < TJ; ++j) b[j] = b_at(buf, wn * WN + j * 8 + fr, ks + fk);
+      for (int i = 0; i < TI; ++i) a[i] = a_at(buf, wm * WM + i * 8 + fr, ks + fk);
 #pragma unroll
-        for (int i = 0; i < TI; ++i)
+      for (int j = 0; j < TJ; ++j) b[j] = b_at(buf, wn * WN + j * 8 + fr, ks + fk);
 #pragma unroll
-          for (int j = 0; j < TJ; ++j) dmma884(acc[i][j][0], acc[i][j][1], a[i], b[j]);
-      }
-      if (t + 1 < nk) store((t + 1) & 1);
-      __syncthreads();
+      for (int i = 0; i < TI; ++i)
+#pragma unroll
+        for (int j = 0; j < TJ; ++j) dmma884(acc[i][j][0], acc[i][j][1], a[i], b[j]);
     }
   }
+  cp_async_wait<0>();
 #pragma unroll
   for (int i = 0; i < TI; ++i)
 #pragma unroll
@@ -214,7 +220,7 @@ static fekf_status gemm_t(long long M, int N, int K, const double* A, int lda, c
                           cudaStream_t s, const int* Mdev, const int* Kdev, int aug_m, int aug_k, int splits, int kps) {
   constexpr size_t asz = TA ? GB_K * (BM + 4) : BM * GB_LDS;
   constexpr size_t bsz = TB ? BN * GB_LDS : GB_K * (BN + 4);
-  constexpr size_t smem = sizeof(double) * 2 * (asz + bsz);
+  constexpr size_t smem = sizeof(double) * GB_STAGES * (asz + bsz);
   static bool attr = false;
   if (!attr) {
     FEKF_CHECK_CUDA(cudaFuncSetAttribute(dgemm_kernel<BM, BN, WM, WN, TA, TB, Epi>,

@@ -273,6 +273,11 @@ kf_pass_kernel(double* __restrict__ P, const ItemD* __restrict__ items, int n_it
     const double* vI = t + TILE_ELEMS;
     const double* vJ = t + TILE_ELEMS + K * KT;
     double ca0 = 0.0, ca1 = 0.0;
+    // this lane's two columns of every deferred u_k (J segment): loaded once per tile, not per row
+    double2 uj[KMAX];
+#pragma unroll
+    for (int k = 0; k < KMAX; ++k)
+      uj[k] = k < K ? *reinterpret_cast<const double2*>(vJ + k * KT + c0) : make_double2(0.0, 0.0);
 #pragma unroll
     for (int q = 0; q < 8; ++q) {
       const int r = warp + 8 * q;
@@ -283,9 +288,8 @@ kf_pass_kernel(double* __restrict__ P, const ItemD* __restrict__ items, int n_it
         for (int k = 0; k < KMAX; ++k) {
           if (k < K) {
             const double bu = beta[k] * vI[k * KT + r];
-            const double2 uj = *reinterpret_cast<const double2*>(vJ + k * KT + c0);
-            cx = fma(bu, uj.x, cx);
-            cy = fma(bu, uj.y, cy);
+            cx = fma(bu, uj[k].x, cx);
+            cy = fma(bu, uj[k].y, cy);
           }
         }
         v.x = sig * (v.x - cx);

@@ -17,6 +17,7 @@
 #include <algorithm>
 
 #include "gemm.cuh"
+#include "emb.cuh"
 
 namespace fekf {
 
@@ -829,10 +830,15 @@ fekf_status model_forward(Ctx& c, int nb, bool tangent, cudaStream_t s) {
   Geo g = make_geo(c, nb);
   if (tangent) FEKF_TRY(build_trows(c, nb, s));
   // embedding nets (compacted rows)
+  const bool fused = emb_fused_ok(c);
   for (size_t p = 0; p < c.pairs.size(); ++p) {
     PairNet& P = c.pairs[p];
     const long long Rmax = pair_rows(c, (int)p, nb);
     if (Rmax == 0) continue;
+    if (fused) {
+      FEKF_TRY(emb_forward(c, (int)p, Rmax, tangent, s));
+      continue;
+    }
     const int* cnt = tangent ? tcount(c, (int)p) : rcount(c, (int)p);
     double* hin = tangent ? P.hin_t.as<double>() : P.hin.as<double>();
     emb_input_kernel<<<cdiv(Rmax, 256), 256, 0, s>>>((int)Rmax, cnt, P.row_idx.as<int>(),
@@ -1004,6 +1010,13 @@ fekf_status model_backward(Ctx& c, int nb, Mode mode, double* gout, cudaStream_t
   FEKF_LAUNCH_CHECK();
   count_launch();
   // ---- embedding nets (compacted rows; tangent rows separately) ----
+  if (emb_bwd_fused_ok(c)) {
+    for (size_t p = 0; p < c.pairs.size(); ++p) {
+      const long long Rmax = pair_rows(c, (int)p, nb);
+      if (Rmax == 0) continue;
+      FEKF_TRY(emb_backward(c, (int)p, Rmax, (int)mode, gout, s));
+    }
+  } else {
   {
     SeedPtrs sp{};
     for (size_t p = 0; p < c.pairs.size(); ++p) {
@@ -1054,6 +1067,7 @@ fekf_status model_backward(Ctx& c, int nb, Mode mode, double* gout, cudaStream_t
                                    EpiStore{P.sbar.as<double>(), 1}, s, rc));
       }
     }
+  }
   }
   if (mode == MODE_FORCE) {
     FEKF_CHECK_CUDA(cudaMemsetAsync(c.force.p, 0, sizeof(double) * nb * c.Na * 3, s));
