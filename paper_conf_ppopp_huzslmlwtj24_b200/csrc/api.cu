@@ -288,7 +288,7 @@ fekf_status Ctx::init(const fekf_model_cfg& mm, const fekf_opt_cfg& oo, int nato
   FEKF_CHECK_CUDA(cudaGetDevice(&dev));
   int maxsm = 0;
   FEKF_CHECK_CUDA(cudaDeviceGetAttribute(&maxsm, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev));
-  const size_t need = (8 * (size_t)M + 2 * (size_t)M * M2) * sizeof(double);
+  const size_t need = (16 * (size_t)M + 2 * (size_t)M * (M2 + 1) + 8 * (size_t)Nm) * sizeof(double);
   if (need > (size_t)maxsm) { set_error("M*M2 too large for the descriptor kernels' shared memory"); return FEKF_EINVAL; }
   FEKF_CHECK_CUDA(cudaDeviceSynchronize());
   return FEKF_OK;

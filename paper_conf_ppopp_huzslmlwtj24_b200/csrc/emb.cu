@@ -9,50 +9,29 @@
 //                         hbar_{l-1} = zbar_l W_l^T + skip^T(hbar_l) ;  sbar = zbar_0 . W_0 (forces)
 //
 // A persistent CTA walks 32-row tiles.  Each layer is a DMMA phase out of shared memory (raw products
-// into the layer's output buffer) followed by an elementwise phase over all threads (bias, tanh, skip,
-// activation adjoints), whose global loads are issued in batches of four per thread.
+// into the layer's output buffer) followed by an elementwise phase (bias, tanh, skip, activation
+// adjoints) in which warp w owns rows w, w + NW, ... and the lanes own columns, with every global
+// load of the phase issued before the first use.
 #include <algorithm>
 
 #include "emb.cuh"
 #include "gemm.cuh"
+#include "mathx.cuh"
 
 namespace fekf {
 
-// ---------------------------------------------------------------------------------------------
-// building blocks
-// ---------------------------------------------------------------------------------------------
-// Elementwise loop over n items: U loads in flight per thread before their uses.
-template <int U, class V, class Load, class Use>
-__device__ __forceinline__ void ew_loop(int n, Load load, Use use) {
-  for (int base = threadIdx.x; base < n; base += blockDim.x * U) {
-    V v[U];
-#pragma unroll
-    for (int u = 0; u < U; ++u) {
-      const int e = base + u * blockDim.x;
-      if (e < n) v[u] = load(e);
-    }
-#pragma unroll
-    for (int u = 0; u < U; ++u) {
-      const int e = base + u * blockDim.x;
-      if (e < n) use(e, v[u]);
-    }
-  }
-}
-
-// out[m][n] = sum_k A[m][k] B(k, n) for the T x (8 NT) tile; A row-major (lda), B(k, n) = BT ? B[n][k] :
-// B[k][n] (ldb).  K a multiple of 4, padded operands zero.  Warp tiles 2x2 (8x8 DMMA tiles) when there
-// are enough of them for every warp, else 1x2.
-template <bool BT>
-__device__ __forceinline__ void cta_mma(const double* A, int lda, const double* B, int ldb, int MT, int NT, int K,
-                                        double* out, int ldo) {
-  const int nw = blockDim.x >> 5, warp = threadIdx.x >> 5, lane = threadIdx.x & 31, fr = lane >> 2, fk = lane & 3;
-  const int NJ = (NT + 1) / 2;
-  auto bval = [&](int k, int n) -> double { return BT ? B[n * ldb + k] : B[k * ldb + n]; };
-  const int MB2 = (MT + 1) / 2;
-  const bool big = MB2 * NJ >= nw;
-  const int MB = big ? MB2 : MT;
-  const int cnt = MB * NJ;
-  for (int wt = warp; wt < cnt; wt += nw) {
+// C[m][n] = sum_k A[m][k] B(k, n) over a (8 MT) x (8 NT) tile; A row-major (LDA), B(k, n) = BT ?
+// B[n][k] : B[k][n] (LDB); K a multiple of 4, padded operands zero.  Warp tiles of 2x2 DMMA tiles when
+// there are enough of them for every warp, else 1x2.  epi(r, c, C[r][c], C[r][c+1]) (c even) straight
+// from the accumulators.
+template <bool BT, int MT, int NT, int K, int LDA, int LDB, int NW, class Epi>
+__device__ __forceinline__ void cta_mma(const double* A, const double* B, Epi epi) {
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, fr = lane >> 2, fk = lane & 3;
+  constexpr int NJ = (NT + 1) / 2;
+  constexpr bool big = ((MT + 1) / 2) * NJ >= NW;
+  constexpr int MB = big ? (MT + 1) / 2 : MT;
+  constexpr int CNT = MB * NJ;
+  for (int wt = warp; wt < CNT; wt += NW) {
     const int mi = big ? (wt % MB) * 2 : wt % MB, nj = (wt / MB) * 2;
     const bool mv = big && mi + 1 < MT, nv = nj + 1 < NT;
     double c[2][2][2];
@@ -60,12 +39,14 @@ __device__ __forceinline__ void cta_mma(const double* A, int lda, const double* 
     for (int i = 0; i < 2; ++i)
 #pragma unroll
       for (int j = 0; j < 2; ++j) c[i][j][0] = c[i][j][1] = 0.0;
-#pragma unroll 2
+    const double* a0p = A + (mi * 8 + fr) * LDA + fk;
+    const double* b0p = BT ? B + (nj * 8 + fr) * LDB + fk : B + fk * LDB + nj * 8 + fr;
+#pragma unroll 4
     for (int k = 0; k < K; k += 4) {
-      const double a0 = A[(mi * 8 + fr) * lda + k + fk];
-      const double a1 = mv ? A[(mi * 8 + 8 + fr) * lda + k + fk] : 0.0;
-      const double b0 = bval(k + fk, nj * 8 + fr);
-      const double b1 = nv ? bval(k + fk, nj * 8 + 8 + fr) : 0.0;
+      const double a0 = a0p[k];
+      const double a1 = mv ? a0p[8 * LDA + k] : 0.0;
+      const double b0 = BT ? b0p[k] : b0p[k * LDB];
+      const double b1 = nv ? (BT ? b0p[8 * LDB + k] : b0p[k * LDB + 8]) : 0.0;
       dmma884(c[0][0][0], c[0][0][1], a0, b0);
       if (nv) dmma884(c[0][1][0], c[0][1][1], a0, b1);
       if (mv) dmma884(c[1][0][0], c[1][0][1], a1, b0);
@@ -76,10 +57,13 @@ __device__ __forceinline__ void cta_mma(const double* A, int lda, const double* 
 #pragma unroll
       for (int j = 0; j < 2; ++j) {
         if ((i == 1 && !mv) || (j == 1 && !nv)) continue;
-        const int r = (mi + i) * 8 + fr, cc = (nj + j) * 8 + 2 * fk;
-        *reinterpret_cast<double2*>(out + r * ldo + cc) = make_double2(c[i][j][0], c[i][j][1]);
+        epi((mi + i) * 8 + fr, (nj + j) * 8 + 2 * fk, c[i][j][0], c[i][j][1]);
       }
   }
+}
+
+__device__ __forceinline__ void l2_prefetch(const void* p, unsigned bytes) {
+  asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(p), "r"(bytes) : "memory");
 }
 
 static int g_num_sms = 0;
@@ -91,12 +75,6 @@ static int num_sms() {
     if (g_num_sms <= 0) g_num_sms = 148;
   }
   return g_num_sms;
-}
-
-bool emb_fused_ok(const Ctx& c) {
-  for (int l = 0; l < c.m.n_emb; ++l)
-    if (c.m.emb[l] > EMB_MAXW) return false;
-  return true;
 }
 
 // =================================================================================================
@@ -114,60 +92,73 @@ struct EmbFwdIO {
   const double* Yp[FEKF_MAX_LAYERS];  // tangent: primal y_l, indexed by primal row
 };
 
-static EmbNetArgs emb_args(const PairNet& P, const double* w) {
-  EmbNetArgs a{};
-  a.nl = (int)P.L.size();
-  int wmax[2] = {1, 1};
-  for (int l = 0; l < a.nl; ++l) {
-    const Layer& L = P.L[l];
-    a.din[l] = L.din;
-    a.dout[l] = L.dout;
-    a.skip[l] = L.skip;
-    a.W[l] = w + L.W;
-    a.b[l] = w + L.b;
-    wmax[l & 1] = std::max(wmax[l & 1], L.dout);
-  }
-  int off = 0;
-  a.wofs[0] = off;
-  off += pad8(a.dout[0]);
-  for (int l = 1; l < a.nl; ++l) {
-    a.wofs[l] = off;
-    off += pad4(a.din[l]) * sld(a.dout[l]);
-  }
-  for (int l = 0; l < a.nl; ++l) {
-    a.bofs[l] = off;
-    off += pad8(a.dout[l]);
-  }
-  for (int q = 0; q < 2; ++q) {
-    a.ald[q] = sld(wmax[q]);
-    a.aofs[q] = off;
-    off += EMB_T * a.ald[q];
-  }
-  a.smem_doubles = off;
-  return a;
+// Forward layer L >= 1 on the current tile: h_L = skip(h_{L-1}) + y_L, y_L = tanh(h_{L-1} W_L + b_L)
+// (primal) or (1 - y_L^2)(hdot_{L-1} W_L) (tangent rows, y_L of the primal row).
+template <class W, int L>
+__device__ __forceinline__ void fwd_layer(double* sm, const EmbFwdIO& io, int r0, int R, bool tan, const int* s_prow) {
+  constexpr int T = W::T, NW = EMB_FWD_WARPS;
+  constexpr int din = W::din(L), d = W::d(L), skip = W::skip(L);
+  constexpr int LDI = W::fALD((L - 1) & 1), LDO = W::fALD(L & 1);
+  const double* in = sm + W::fA((L - 1) & 1);
+  double* out = sm + W::fA(L & 1);
+  const double* bs = sm + W::fB(L);
+  double* Yl = io.Y[L];
+  double* Hl = io.H[L];
+  const double* Ypl = io.Yp[L];
+  cta_mma<false, T / 8, pad8(d) / 8, pad4(din), LDI, sld(d), NW>(
+      in, sm + W::fW(L), [&](int r, int c, double z0, double z1) {
+        const int row = r0 + r;
+        const bool live = row < R;
+        double h[2];
+        const double z[2] = {z0, z1};
+#pragma unroll
+        for (int q = 0; q < 2; ++q) {
+          const int cc = c + q;
+          double y;
+          if (tan) {
+            const int pr = s_prow[r];
+            const double yp = (cc < d && pr >= 0) ? Ypl[(size_t)pr * d + cc] : 0.0;
+            y = (1.0 - yp * yp) * z[q];
+          } else {
+            y = tanh_fp64(z[q] + bs[cc]);
+          }
+          const double sk = skip == 1 ? in[r * LDI + cc] : (skip == 2 ? in[r * LDI + (cc % din)] : 0.0);
+          h[q] = cc < d ? sk + y : 0.0;
+          if (live && cc < d) {
+            Yl[(size_t)row * d + cc] = y;
+            if (Hl) Hl[(size_t)row * d + cc] = h[q];
+          }
+        }
+        *reinterpret_cast<double2*>(out + r * LDO + c) = make_double2(h[0], h[1]);
+      });
+  __syncthreads();
 }
 
-__global__ void __launch_bounds__(EMB_FWD_WARPS * 32) emb_fwd_kernel(EmbNetArgs a, EmbFwdIO io) {
+template <class W>
+__global__ void __launch_bounds__(EMB_FWD_WARPS * 32) emb_fwd_kernel(const double* __restrict__ wp, EmbFwdIO io) {
   extern __shared__ __align__(16) double sm[];
-  constexpr int T = EMB_T;
+  constexpr int T = W::T, NW = EMB_FWD_WARPS, NL = W::NL, RPW = T / NW;
   __shared__ double s_in[T];
   __shared__ int s_prow[T];
-  const int tid = threadIdx.x;
+  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   const bool tan = io.tidx != nullptr;
   const int R = min(io.Rmax, *io.Rdev);
-  // ---- stage W_l (zero-padded to [pad4(din)][sld(dout)]) and b_l
-  for (int c = tid; c < pad8(a.dout[0]); c += blockDim.x) sm[a.wofs[0] + c] = c < a.dout[0] ? a.W[0][c] : 0.0;
-  for (int l = 1; l < a.nl; ++l) {
-    const int din = a.din[l], dout = a.dout[l], ld = sld(dout), n = pad4(din) * ld;
-    const double* W = a.W[l];
-    double* Ws = sm + a.wofs[l];
+  // ---- stage W_l (zero-padded to [pad4(din)][sld(d)]) and b_l
+  for (int c = tid; c < pad8(W::d(0)); c += blockDim.x) sm[W::fW(0) + c] = c < W::d(0) ? wp[W::goff(0) + c] : 0.0;
+#pragma unroll
+  for (int l = 1; l < NL; ++l) {
+    constexpr int dummy = 0;
+    (void)dummy;
+    const int din = W::din(l), d = W::d(l), ld = sld(d), n = pad4(din) * ld;
     for (int e = tid; e < n; e += blockDim.x) {
       const int k = e / ld, j = e % ld;
-      Ws[e] = (k < din && j < dout) ? W[(size_t)k * dout + j] : 0.0;
+      sm[W::fW(l) + e] = (k < din && j < d) ? wp[W::goff(l) + k * d + j] : 0.0;
     }
   }
-  for (int l = 0; l < a.nl; ++l)
-    for (int c = tid; c < pad8(a.dout[l]); c += blockDim.x) sm[a.bofs[l] + c] = c < a.dout[l] ? a.b[l][c] : 0.0;
+#pragma unroll
+  for (int l = 0; l < NL; ++l)
+    for (int c = tid; c < pad8(W::d(l)); c += blockDim.x)
+      sm[W::fB(l) + c] = c < W::d(l) ? wp[W::goff(l) + W::din(l) * W::d(l) + c] : 0.0;
 
   const int ntiles = (R + T - 1) / T;
   for (int tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
@@ -188,86 +179,51 @@ __global__ void __launch_bounds__(EMB_FWD_WARPS * 32) emb_fwd_kernel(EmbNetArgs 
     __syncthreads();
     // ---- layer 0 (input width 1): elementwise
     {
-      const int d = a.dout[0], w8 = pad8(d), ld = a.ald[0];
-      double* out = sm + a.aofs[0];
-      const double* w0 = sm + a.wofs[0];
-      const double* b0 = sm + a.bofs[0];
-      const double* Yp0 = io.Yp[0];
-      double* Y0 = io.Y[0];
-      double* H0 = io.H[0];
-      ew_loop<4, double>(
-          T * w8,
-          [&](int e) -> double {
-            const int r = e / w8, cc = e % w8;
-            const int pr = s_prow[r];
-            return (tan && cc < d && pr >= 0) ? Yp0[(size_t)pr * d + cc] : 0.0;
-          },
-          [&](int e, double yp) {
-            const int r = e / w8, cc = e % w8;
+      constexpr int d = W::d(0), w8 = pad8(d), CJ = (w8 + 31) / 32, ld = W::fALD(0);
+      double* out = sm + W::fA(0);
+      const double* w0 = sm + W::fW(0);
+      const double* b0 = sm + W::fB(0);
+      double yp[RPW][CJ];
+#pragma unroll
+      for (int i = 0; i < RPW; ++i)
+#pragma unroll
+        for (int j = 0; j < CJ; ++j) {
+          const int r = warp + NW * i, c = lane + 32 * j;
+          const int pr = s_prow[r];
+          yp[i][j] = (tan && c < d && pr >= 0) ? io.Yp[0][(size_t)pr * d + c] : 0.0;
+        }
+#pragma unroll
+      for (int i = 0; i < RPW; ++i)
+#pragma unroll
+        for (int j = 0; j < CJ; ++j) {
+          const int r = warp + NW * i, c = lane + 32 * j;
+          if (c < w8) {
             const int row = r0 + r;
             double h = 0.0;
-            if (cc < d) {
-              const double z = s_in[r] * w0[cc];
-              const double y = tan ? (1.0 - yp * yp) * z : tanh(z + b0[cc]);
-              h = y;
+            if (c < d) {
+              const double z = s_in[r] * w0[c];
+              h = tan ? (1.0 - yp[i][j] * yp[i][j]) * z : tanh_fp64(z + b0[c]);
               if (row < R) {
-                const size_t o = (size_t)row * d + cc;
-                Y0[o] = y;
-                if (H0) H0[o] = y;
+                const size_t o = (size_t)row * d + c;
+                io.Y[0][o] = h;
+                if (io.H[0]) io.H[0][o] = h;
               }
             }
-            out[r * ld + cc] = h;
-          });
+            out[r * ld + c] = h;
+          }
+        }
     }
     __syncthreads();
-    // ---- layers 1..nl-1: DMMA phase, then the elementwise epilogue (bias, tanh, skip) in place
-    for (int l = 1; l < a.nl; ++l) {
-      const int din = a.din[l], dout = a.dout[l], w8 = pad8(dout);
-      const double* in = sm + a.aofs[(l - 1) & 1];
-      const int ldi = a.ald[(l - 1) & 1];
-      double* out = sm + a.aofs[l & 1];
-      const int ldo = a.ald[l & 1];
-      cta_mma<false>(in, ldi, sm + a.wofs[l], sld(dout), T / 8, w8 / 8, pad4(din), out, ldo);
-      __syncthreads();
-      const double* bs = sm + a.bofs[l];
-      const int skip = a.skip[l];
-      double* Yl = io.Y[l];
-      double* Hl = io.H[l];
-      const double* Ypl = io.Yp[l];
-      ew_loop<4, double>(
-          T * w8,
-          [&](int e) -> double {
-            const int r = e / w8, cc = e % w8;
-            const int pr = s_prow[r];
-            return (tan && cc < dout && pr >= 0) ? Ypl[(size_t)pr * dout + cc] : 0.0;
-          },
-          [&](int e, double yp) {
-            const int r = e / w8, cc = e % w8;
-            const int row = r0 + r;
-            double hv = 0.0;
-            if (cc < dout) {
-              const double z = out[r * ldo + cc];
-              const double y = tan ? (1.0 - yp * yp) * z : tanh(z + bs[cc]);
-              const double sk = skip == 1 ? in[r * ldi + cc] : (skip == 2 ? in[r * ldi + (cc % din)] : 0.0);
-              hv = sk + y;
-              if (row < R) {
-                const size_t o = (size_t)row * dout + cc;
-                Yl[o] = y;
-                if (Hl) Hl[o] = hv;
-              }
-            }
-            out[r * ldo + cc] = hv;
-          });
-      __syncthreads();
-    }
+    // ---- layers 1..NL-1: DMMA with the bias / tanh / skip epilogue in the accumulators
+    if constexpr (NL >= 2) fwd_layer<W, 1>(sm, io, r0, R, tan, s_prow);
+    if constexpr (NL >= 3) fwd_layer<W, 2>(sm, io, r0, R, tan, s_prow);
+    if constexpr (NL >= 4) fwd_layer<W, 3>(sm, io, r0, R, tan, s_prow);
   }
 }
 
-// Forward of one pair's embedding net over its primal rows (tangent = false) or its active tangent
-// rows (tangent = true).  Writes y_l and h_l of every layer and s (s-dot) per row.
-fekf_status emb_forward(Ctx& c, int p, long long Rmax, bool tangent, cudaStream_t s) {
+template <class W>
+static fekf_status emb_forward_t(Ctx& c, int p, long long Rmax, bool tangent, cudaStream_t s) {
   PairNet& P = c.pairs[p];
-  EmbNetArgs a = emb_args(P, c.w.as<double>());
   EmbFwdIO io{};
   io.Rmax = (int)Rmax;
   io.Rdev = c.rowcnt.as<int>() + (tangent ? c.pairs.size() + p : p);
@@ -275,23 +231,22 @@ fekf_status emb_forward(Ctx& c, int p, long long Rmax, bool tangent, cudaStream_
   io.tidx = tangent ? P.tidx.as<int>() : nullptr;
   io.src = tangent ? c.rdot.as<double>() : c.em.as<double>();
   io.hin = tangent ? P.hin_t.as<double>() : P.hin.as<double>();
-  for (int l = 0; l < a.nl; ++l) {
+  for (int l = 0; l < W::NL; ++l) {
     io.Y[l] = tangent ? P.Yt[l].as<double>() : P.Y[l].as<double>();
-    io.H[l] = tangent ? P.Ht[l].as<double>() : P.H[l].as<double>();
+    // only h_{L-1} (G, G-dot) is read back (descriptor); earlier h are recomputed from y where needed
+    io.H[l] = l + 1 < W::NL ? nullptr : (tangent ? P.Ht[l].as<double>() : P.H[l].as<double>());
     io.Yp[l] = P.Y[l].as<double>();
   }
-  const size_t smem = sizeof(double) * a.smem_doubles;
-  static size_t attr = 0;
-  if (smem > attr) {
-    FEKF_CHECK_CUDA(cudaFuncSetAttribute(emb_fwd_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-    attr = smem;
+  constexpr size_t smem = sizeof(double) * W::F_SMEM;
+  static int occ = 0;
+  if (!occ) {
+    FEKF_CHECK_CUDA(cudaFuncSetAttribute(emb_fwd_kernel<W>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    FEKF_CHECK_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, emb_fwd_kernel<W>, EMB_FWD_WARPS * 32, smem));
+    if (occ < 1) { set_error("emb_fwd_kernel: does not fit on an SM"); return FEKF_EINVAL; }
   }
-  int occ = 0;
-  FEKF_CHECK_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, emb_fwd_kernel, EMB_FWD_WARPS * 32, smem));
-  if (occ < 1) { set_error("emb_fwd_kernel: does not fit on an SM"); return FEKF_EINVAL; }
   const long long tiles = (Rmax + EMB_T - 1) / EMB_T;
   const int grid = (int)std::max<long long>(1, std::min<long long>(tiles, (long long)num_sms() * occ));
-  emb_fwd_kernel<<<grid, EMB_FWD_WARPS * 32, smem, s>>>(a, io);
+  emb_fwd_kernel<W><<<grid, EMB_FWD_WARPS * 32, smem, s>>>(c.w.as<double>() + P.L[0].W, io);
   FEKF_LAUNCH_CHECK();
   count_launch();
   return FEKF_OK;
@@ -306,105 +261,267 @@ struct EmbBwdIO {
   const int* row_idx;
   const int* tidx;                    // tangent rows: tangent row -> primal row (nullptr: primal rows)
   const int* tpos;                    // primal rows, dual: primal row -> tangent row or -1 (nullptr: none)
-  const double* em;
-  const double* rdot;
-  const double* Xb;                   // atom X-bar
-  const double* Xdb;                  // atom X-dot-bar
+  int Nm;
+  const double* Gbar;                 // primal rows: Gbar (desc_bwd_seed_kernel)
+  const double* dR;                   // forces: per-row R~ adjoint less sbar e_0 [R][4]
   const double* hin;                  // s / s-dot per row
   const double* Y[FEKF_MAX_LAYERS];   // y of this row set (h is recomputed from it)
   const double* Yp[FEKF_MAX_LAYERS];  // primal y (indexed by primal row)
   const double* Yt[FEKF_MAX_LAYERS];  // tangent y (indexed by tangent row)
   double* Hbt[FEKF_MAX_LAYERS];       // hdotbar_l: written by tangent rows, read by dual primal rows
   double* sbar;                       // forces: s-bar per primal row
-  double* ws;                         // weight-gradient partials [gridDim.x][gsize] (nullptr: none)
+  double* ws;                         // weight-gradient partials [gridDim.x][GS] (nullptr: none)
+  // forces (prod_force fused, MODE_FORCE): dE/dR~_row = dR + sbar e_0 ; f = (dE/dR~) J ;
+  // F_i += f, F_j -= f (F = -dE/dx) ; W_i -= d (x) f
+  const double* jac;
+  const double* rij;
+  const int* nl_j;
+  int Na;
+  double* force;
+  double* vatom;
 };
 
-static EmbBwdArgs emb_bwd_args(const Ctx& c, const PairNet& P, const double* w) {
-  EmbBwdArgs a{};
-  a.nl = (int)P.L.size();
-  a.M = c.M;
-  a.Nm = c.Nm;
-  int maxw = 1;
-  for (int l = 0; l < a.nl; ++l) {
-    const Layer& L = P.L[l];
-    a.din[l] = L.din;
-    a.dout[l] = L.dout;
-    a.skip[l] = L.skip;
-    a.W[l] = w + L.W;
-    maxw = std::max(maxw, L.dout);
-  }
-  int off = 0;
-  a.wofs[0] = off;
-  off += pad8(a.dout[0]);
-  for (int l = 1; l < a.nl; ++l) {
-    a.wofs[l] = off;
-    off += pad8(a.din[l]) * sld(a.dout[l]);
-  }
-  for (int l = 0; l < a.nl; ++l) {
-    a.augld[l] = sld(a.din[l] + 1);
-    a.augofs[l] = off;
-    off += EMB_T * a.augld[l];
-  }
-  a.bld = sld(maxw);
-  for (int q = 0; q < 3; ++q) {
-    a.bofs[q] = off;
-    off += EMB_T * a.bld;
-  }
-  a.rofs = off;
-  off += EMB_T * 8;
-  a.smem_doubles = off;
-  int g = 0;
-  for (int l = 0; l < a.nl; ++l) {
-    a.goff[l] = g;
-    g += (a.din[l] + 1) * a.dout[l];
-  }
-  a.gsize = g;
-  a.nblk = 0;
-  for (int l = a.nl - 1; l >= 0; --l) {
-    const int mb = (pad8(a.din[l] + 1) / 8 + 1) / 2, nb = (pad8(a.dout[l]) / 8 + 1) / 2;
-    for (int i = 0; i < mb; ++i)
-      for (int j = 0; j < nb; ++j) {
-        if (a.nblk < EMB_BWD_WARPS * EMB_MAXB) a.blk[a.nblk] = (l << 16) | (i << 8) | j;
-        ++a.nblk;
+// weight-gradient blocks of layer L: [Wbar_L ; bbar_L] += [h_{L-1} | 1]^T zbar_L over the tile's rows
+template <class W, int L>
+__device__ __forceinline__ void wgrad_layer(double (&acc)[W::MAXB][2][2][2], const double* sm, int zbuf) {
+  constexpr int NW = EMB_BWD_WARPS, T = W::T;
+  constexpr int first = W::blk_first(L), nb = W::mblk(L) * W::nblk(L), LDA = W::augld(L), LDB = W::BLD;
+  constexpr int m8 = pad8(W::din(L) + 1), n8 = pad8(W::d(L));
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, fr = lane >> 2, fk = lane & 3;
+  const double* A = sm + W::bAug(L);
+  const double* Z = sm + W::bBuf(0) + zbuf * T * W::BLD;
+#pragma unroll
+  for (int q = 0; q < W::MAXB; ++q) {
+    const int b = warp + NW * q - first;
+    if (b >= 0 && b < nb) {
+      const int m0 = (b / W::nblk(L)) * 16, n0 = (b % W::nblk(L)) * 16;
+      const bool mv = m0 + 8 < m8, nv = n0 + 8 < n8;
+      const double* ap = A + fk * LDA + m0 + fr;
+      const double* bp = Z + fk * LDB + n0 + fr;
+#pragma unroll
+      for (int k = 0; k < T; k += 4) {
+        const double a0 = ap[k * LDA];
+        const double a1 = mv ? ap[k * LDA + 8] : 0.0;
+        const double b0 = bp[k * LDB];
+        const double b1 = nv ? bp[k * LDB + 8] : 0.0;
+        dmma884(acc[q][0][0][0], acc[q][0][0][1], a0, b0);
+        if (nv) dmma884(acc[q][0][1][0], acc[q][0][1][1], a0, b1);
+        if (mv) dmma884(acc[q][1][0][0], acc[q][1][0][1], a1, b0);
+        if (mv && nv) dmma884(acc[q][1][1][0], acc[q][1][1][1], a1, b1);
       }
+    }
   }
-  return a;
 }
 
-struct ZIn { double y, yt, hbt; };
-
-__global__ void __launch_bounds__(EMB_BWD_WARPS * 32, 1) emb_bwd_kernel(EmbBwdArgs a, EmbBwdIO io) {
-  extern __shared__ __align__(16) double sm[];
-  constexpr int T = EMB_T;
-  constexpr int MAXB = EMB_MAXB;
+template <class W, int L>
+__device__ __forceinline__ void write_partials(const double (&acc)[W::MAXB][2][2][2], double* out) {
   constexpr int NW = EMB_BWD_WARPS;
+  constexpr int first = W::blk_first(L), nb = W::mblk(L) * W::nblk(L);
+  constexpr int rows = W::din(L) + 1, cols = W::d(L);
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, fr = lane >> 2, fk = lane & 3;
+#pragma unroll
+  for (int q = 0; q < W::MAXB; ++q) {
+    const int b = warp + NW * q - first;
+    if (b >= 0 && b < nb) {
+      const int m0 = (b / W::nblk(L)) * 16, n0 = (b % W::nblk(L)) * 16;
+#pragma unroll
+      for (int i = 0; i < 2; ++i)
+#pragma unroll
+        for (int j = 0; j < 2; ++j)
+#pragma unroll
+          for (int h = 0; h < 2; ++h) {
+            const int m = m0 + 8 * i + fr, n = n0 + 8 * j + 2 * fk + h;
+            if (m < rows && n < cols) out[W::goff(L) + m * cols + n] = acc[q][i][j][h];
+          }
+    }
+  }
+}
+
+// a [T][12] scratch area for the force epilogue: the adjoint buffer the layer-0 step does not use
+template <class W>
+__device__ __forceinline__ double* hn_scratch(double* sm) {
+  constexpr int step = W::NL - 1;
+  constexpr int bx = (3 - step % 3) % 3, bn = (bx + 2) % 3;
+  static_assert(W::BLD >= 12, "scratch");
+  return sm + W::bBuf(bn);
+}
+
+// One layer L of the reverse chain on the current tile (buffers rotate with the step from the top).
+template <class W, int L>
+__device__ __forceinline__ void bwd_layer(double (&acc)[W::MAXB][2][2][2], double* sm, const EmbBwdIO& io, int r0, int R,
+                                          bool tan, bool wantw, const int* s_slot, const int* s_prow,
+                                          const int* s_tpos, const int* s_atom, const double* s_dr) {
+  constexpr int T = W::T, NW = EMB_BWD_WARPS, RPW = T / NW, BLD = W::BLD;
+  constexpr int step = W::NL - 1 - L;
+  constexpr int bx = (3 - step % 3) % 3, bz = (bx + 1) % 3, bn = (bx + 2) % 3;
+  constexpr int d = W::d(L), w8 = pad8(d), CJ = (w8 + 31) / 32;
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const double* hb = sm + W::bBuf(bx);
+  double* zb = sm + W::bBuf(bz);
+  // ---- zbar_L
+  {
+    double y[RPW][CJ], yt[RPW][CJ], hbt[RPW][CJ];
+#pragma unroll
+    for (int i = 0; i < RPW; ++i)
+#pragma unroll
+      for (int j = 0; j < CJ; ++j) {
+        const int r = warp + NW * i, c = lane + 32 * j;
+        y[i][j] = yt[i][j] = hbt[i][j] = 0.0;
+        if (c < d && s_slot[r] >= 0) {
+          y[i][j] = io.Yp[L][(size_t)s_prow[r] * d + c];
+          const int tp = s_tpos[r];
+          if (tp >= 0) {
+            yt[i][j] = io.Yt[L][(size_t)tp * d + c];
+            hbt[i][j] = io.Hbt[L][(size_t)tp * d + c];
+          }
+        }
+      }
+#pragma unroll
+    for (int i = 0; i < RPW; ++i)
+#pragma unroll
+      for (int j = 0; j < CJ; ++j) {
+        const int r = warp + NW * i, c = lane + 32 * j;
+        if (c < w8) {
+          double v = 0.0;
+          if (c < d && s_slot[r] >= 0)
+            v = (1.0 - y[i][j] * y[i][j]) * hb[r * BLD + c] - 2.0 * y[i][j] * yt[i][j] * hbt[i][j];
+          zb[r * BLD + c] = v;
+        }
+      }
+  }
+  __syncthreads();
+  if (wantw) wgrad_layer<W, L>(acc, sm, bz);
+  if constexpr (L > 0) {
+    constexpr int din = W::din(L), n8 = pad8(din), skip = W::skip(L);
+    double* hn = sm + W::bBuf(bn);
+    double* Hbt = tan ? io.Hbt[L - 1] : nullptr;
+    // hbar_{L-1} = zbar_L W_L^T + skip^T(hbar_L) straight from the accumulators
+    cta_mma<true, T / 8, n8 / 8, pad4(d), BLD, sld(d), NW>(zb, sm + W::bW(L), [&](int r, int c, double v0, double v1) {
+      double v[2] = {v0, v1};
+#pragma unroll
+      for (int q = 0; q < 2; ++q) {
+        const int cc = c + q;
+        if (cc < din) {
+          if (skip == 1) v[q] += hb[r * BLD + cc];
+          else if (skip == 2) v[q] += hb[r * BLD + cc] + hb[r * BLD + cc + din];
+          if (Hbt && r0 + r < R) Hbt[(size_t)(r0 + r) * din + cc] = v[q];
+        } else {
+          v[q] = 0.0;
+        }
+      }
+      *reinterpret_cast<double2*>(hn + r * BLD + c) = make_double2(v[0], v[1]);
+    });
+    __syncthreads();
+  } else if (io.sbar) {
+    // sbar = zbar_0 . W_0 (4 threads per row), then the row's dE/dd and the force / virial scatter
+    double* sf = hn_scratch<W>(sm);  // [T][12]: f (3) | -d (x) f (9), in a buffer the chain is done with
+    const int t = threadIdx.x;
+    if (t < T * 4) {
+      const int r = t >> 2, part = t & 3;
+      const double* w0 = sm + W::bW(0);
+      double sb = 0.0;
+#pragma unroll
+      for (int cc = part; cc < d; cc += 4) sb = fma(zb[r * BLD + cc], w0[cc], sb);
+      sb += __shfl_xor_sync(0xffffffffu, sb, 1);
+      sb += __shfl_xor_sync(0xffffffffu, sb, 2);
+      const int row = r0 + r;
+      if (part == 0 && row < R) io.sbar[row] = sb;
+      if (io.dR && part < 3) {
+        const int be = part, slot = s_slot[r];
+        double f = 0.0;
+        if (row < R) {
+          const double* J = io.jac + (size_t)slot * 12;
+          f = (s_dr[r * 4] + sb) * J[be] + s_dr[r * 4 + 1] * J[3 + be] + s_dr[r * 4 + 2] * J[6 + be] +
+              s_dr[r * 4 + 3] * J[9 + be];
+          const int atom = s_atom[r], j = io.nl_j[slot];
+          atomicAdd(io.force + ((size_t)(atom / io.Na) * io.Na + j) * 3 + be, -f);
+        }
+        sf[r * 12 + be] = f;
+      }
+    }
+    if (io.dR) {
+      __syncthreads();
+      if (t < T * 9) {
+        const int r = t / 9, q = t % 9, a = q / 3, be = q % 3;
+        double v = 0.0;
+        if (r0 + r < R) v = -io.rij[(size_t)s_slot[r] * 3 + a] * sf[r * 12 + be];
+        sf[r * 12 + 3 + q] = v;
+      }
+      __syncthreads();
+      // rows of one centre atom are consecutive: one atomic per (segment, component)
+      if (t < T * 12) {
+        const int r = t / 12, q = t % 12;
+        const int atom = s_atom[r];
+        if (r0 + r < R && (r == 0 || s_atom[r - 1] != atom)) {
+          double sum = 0.0;
+          for (int k = r; k < T && r0 + k < R && s_atom[k] == atom; ++k) sum += sf[k * 12 + q];
+          if (q < 3) atomicAdd(io.force + (size_t)atom * 3 + q, sum);
+          else atomicAdd(io.vatom + (size_t)atom * 9 + q - 3, sum);
+        }
+      }
+    }
+  }
+}
+
+// seed of the reverse chain for the tile's rows (warp w owns rows w, w + NW): hbar_{L-1} = Gbar, written
+// per row by desc_bwd_seed_kernel (primal rows: Gbar; tangent rows: Gdotbar in hdotbar_{L-1}); forces: the
+// per-row R~ adjoint dR
+template <class W>
+__device__ __forceinline__ void seed_rows(double* sm, const EmbBwdIO& io, int r0, int R, bool tan, double* s_dr) {
+  constexpr int T = W::T, NW = EMB_BWD_WARPS, RPW = T / NW, BLD = W::BLD, NL = W::NL, M = W::M;
+  constexpr int w8 = pad8(M), CJ = (w8 + 31) / 32;
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const double* src = tan ? io.Hbt[NL - 1] : io.Gbar;
+  double* Hb = sm + W::bBuf(0);
+  double v[RPW][CJ];
+#pragma unroll
+  for (int i = 0; i < RPW; ++i)
+#pragma unroll
+    for (int j = 0; j < CJ; ++j) {
+      const int r = warp + NW * i, c = lane + 32 * j;
+      v[i][j] = (c < M && r0 + r < R) ? src[(size_t)(r0 + r) * M + c] : 0.0;
+    }
+#pragma unroll
+  for (int i = 0; i < RPW; ++i)
+#pragma unroll
+    for (int j = 0; j < CJ; ++j) {
+      const int r = warp + NW * i, c = lane + 32 * j;
+      if (c < w8) Hb[r * BLD + c] = v[i][j];
+    }
+  if (io.dR && threadIdx.x < T * 4) {
+    const int r = threadIdx.x >> 2;
+    s_dr[threadIdx.x] = r0 + r < R ? io.dR[(size_t)r0 * 4 + threadIdx.x] : 0.0;
+  }
+}
+
+template <class W>
+__global__ void __launch_bounds__(EMB_BWD_WARPS * 32, 1) emb_bwd_kernel(const double* __restrict__ wp, EmbBwdIO io) {
+  extern __shared__ __align__(16) double sm[];
+  constexpr int T = W::T, NW = EMB_BWD_WARPS, NL = W::NL, RPW = T / NW;
   __shared__ int s_slot[T], s_atom[T], s_prow[T], s_tpos[T];
-  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31, fr = lane >> 2, fk = lane & 3;
+  __shared__ double s_dr[T * 4];
+  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   const bool tan = io.tidx != nullptr;
   const bool wantw = io.ws != nullptr;
   const int R = min(io.Rmax, *io.Rdev);
-  const int nl = a.nl, M = a.M;
-  // ---- stage W (zero-padded)
-  for (int c = tid; c < pad8(a.dout[0]); c += blockDim.x) sm[a.wofs[0] + c] = c < a.dout[0] ? a.W[0][c] : 0.0;
-  for (int l = 1; l < nl; ++l) {
-    const int din = a.din[l], dout = a.dout[l], ld = sld(dout), n = pad8(din) * ld;
-    const double* W = a.W[l];
-    double* Ws = sm + a.wofs[l];
+  // ---- stage W (zero-padded [pad8(din)][sld(d)])
+  for (int c = tid; c < pad8(W::d(0)); c += blockDim.x) sm[W::bW(0) + c] = c < W::d(0) ? wp[W::goff(0) + c] : 0.0;
+#pragma unroll
+  for (int l = 1; l < NL; ++l) {
+    const int din = W::din(l), d = W::d(l), ld = sld(d), n = pad8(din) * ld;
     for (int e = tid; e < n; e += blockDim.x) {
       const int k = e / ld, j = e % ld;
-      Ws[e] = (k < din && j < dout) ? W[(size_t)k * dout + j] : 0.0;
+      sm[W::bW(l) + e] = (k < din && j < d) ? wp[W::goff(l) + k * d + j] : 0.0;
     }
   }
-  double acc[MAXB][2][2][2];
+  double acc[W::MAXB][2][2][2];
 #pragma unroll
-  for (int q = 0; q < MAXB; ++q)
+  for (int q = 0; q < W::MAXB; ++q)
 #pragma unroll
     for (int i = 0; i < 2; ++i)
 #pragma unroll
       for (int j = 0; j < 2; ++j) acc[q][i][j][0] = acc[q][i][j][1] = 0.0;
-  const double invN = 1.0 / a.Nm;
   const double one = tan ? 0.0 : 1.0;
-  double* rr = sm + a.rofs;  // [T][8]: R~ row (4) | R~-dot row (4)
   const int ntiles = (R + T - 1) / T;
   for (int tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
     const int r0 = tile * T;
@@ -415,7 +532,7 @@ __global__ void __launch_bounds__(EMB_BWD_WARPS * 32, 1) emb_bwd_kernel(EmbBwdAr
       if (row < R) {
         pr = tan ? io.tidx[row] : row;
         slot = io.row_idx[pr];
-        atom = slot / a.Nm;
+        atom = slot / io.Nm;
         if (io.tpos) tp = io.tpos[row];
       }
       s_slot[tid] = slot;
@@ -424,204 +541,77 @@ __global__ void __launch_bounds__(EMB_BWD_WARPS * 32, 1) emb_bwd_kernel(EmbBwdAr
       s_tpos[tid] = tp;
     }
     __syncthreads();
-    if (tid < T * 8) {
-      const int r = tid >> 3, k = tid & 7;
-      const int slot = s_slot[r];
-      double v = 0.0;
-      if (slot >= 0) {
-        if (k < 4) v = io.em[(size_t)slot * 4 + k];
-        else if (s_tpos[r] >= 0) v = io.rdot[(size_t)slot * 4 + k - 4];
+    // the next tile's stored activations (contiguous rows) on their way to L2 while this one computes
+    if (tid == 0) {
+      const int rn = r0 + gridDim.x * T;
+      if (rn + T <= io.Rmax) {
+#pragma unroll
+        for (int l = 0; l < NL; ++l) l2_prefetch(io.Y[l] + (size_t)rn * W::d(l), T * W::d(l) * sizeof(double));
+        l2_prefetch((tan ? io.Hbt[NL - 1] : io.Gbar) + (size_t)rn * W::M, T * W::M * sizeof(double));
+        if (io.dR) l2_prefetch(io.dR + (size_t)rn * 4, T * 4 * sizeof(double));
       }
-      rr[tid] = v;
     }
     // ---- [h_{l-1} | 1] for every layer (h recomputed from the stored y: h_0 = y_0, h_l = skip + y_l)
     if (wantw) {
-      double* A0 = sm + a.augofs[0];
       if (tid < T * 8) {
         const int r = tid >> 3, cc = tid & 7;
         const int row = r0 + r;
         double v = 0.0;
         if (row < R) v = cc == 0 ? io.hin[row] : (cc == 1 ? one : 0.0);
-        A0[r * a.augld[0] + cc] = v;
+        sm[W::bAug(0) + r * W::augld(0) + cc] = v;
       }
-      for (int l = 1; l < nl; ++l) {
-        const int din = a.din[l], w8 = pad8(din + 1), ld = a.augld[l];
-        const double* prev = sm + a.augofs[l - 1];
-        const int ldp = a.augld[l - 1], skp = a.skip[l - 1], dpp = a.din[l - 1];
-        const double* Yl = io.Y[l - 1];
-        double* Al = sm + a.augofs[l];
-        if (l >= 2) __syncthreads();  // Aug_{l-1} complete
-        ew_loop<4, double>(
-            T * w8,
-            [&](int e) -> double {
-              const int r = e / w8, cc = e % w8;
-              return (r0 + r < R && cc < din) ? Yl[(size_t)(r0 + r) * din + cc] : 0.0;
-            },
-            [&](int e, double y) {
-              const int r = e / w8, cc = e % w8;
+#pragma unroll
+      for (int l = 1; l < NL; ++l) {
+        const int din = W::din(l), w8 = pad8(din + 1), CJ = (w8 + 31) / 32, ld = W::augld(l);
+        constexpr int CJMAX = (pad8(W::maxw(-1) + 1) + 31) / 32;
+        const int ldp = W::augld(l - 1), skp = W::skip(l - 1), dpp = W::din(l - 1);
+        const double* prev = sm + W::bAug(l - 1);
+        double* Al = sm + W::bAug(l);
+        if (l >= 2) __syncthreads();  // aug_{l-1} complete
+        double y[RPW][CJMAX];
+#pragma unroll
+        for (int i = 0; i < RPW; ++i)
+#pragma unroll
+          for (int j = 0; j < CJMAX; ++j) {
+            const int r = warp + NW * i, c = lane + 32 * j;
+            y[i][j] = (j < CJ && r0 + r < R && c < din) ? io.Y[l - 1][(size_t)(r0 + r) * din + c] : 0.0;
+          }
+#pragma unroll
+        for (int i = 0; i < RPW; ++i)
+#pragma unroll
+          for (int j = 0; j < CJMAX; ++j) {
+            const int r = warp + NW * i, c = lane + 32 * j;
+            if (j < CJ && c < w8) {
               double v = 0.0;
               if (r0 + r < R) {
-                if (cc < din) {
-                  v = y;
-                  if (skp == 1) v += prev[r * ldp + cc];
-                  else if (skp == 2) v += prev[r * ldp + cc % dpp];
-                } else if (cc == din) {
+                if (c < din) {
+                  v = y[i][j];
+                  if (skp == 1) v += prev[r * ldp + c];
+                  else if (skp == 2) v += prev[r * ldp + c % dpp];
+                } else if (c == din) {
                   v = one;
                 }
               }
-              Al[r * ld + cc] = v;
-            });
+              Al[r * ld + c] = v;
+            }
+          }
       }
     }
-    __syncthreads();  // rr, Aug ready
-    // ---- seed: hbar_{L-1} = Gbar
-    int bx = 0, bz = 1, bn = 2;
-    {
-      const int w8 = pad8(M);
-      double* Hb = sm + a.bofs[bx];
-      double* HbtL = tan ? io.Hbt[nl - 1] : nullptr;
-      const double* X1 = tan ? io.Xdb : io.Xb;
-      struct XIn { double x0, x1, x2, x3, d0, d1, d2, d3; };
-      ew_loop<1, XIn>(
-          T * w8,
-          [&](int e) -> XIn {
-            const int r = e / w8, cc = e % w8;
-            XIn x{};
-            if (cc < M && s_slot[r] >= 0) {
-              const double* xb = X1 + (size_t)s_atom[r] * 4 * M + cc;
-              x.x0 = xb[0]; x.x1 = xb[M]; x.x2 = xb[2 * M]; x.x3 = xb[3 * M];
-              if (!tan && s_tpos[r] >= 0) {
-                const double* xd = io.Xdb + (size_t)s_atom[r] * 4 * M + cc;
-                x.d0 = xd[0]; x.d1 = xd[M]; x.d2 = xd[2 * M]; x.d3 = xd[3 * M];
-              }
-            }
-            return x;
-          },
-          [&](int e, const XIn& x) {
-            const int r = e / w8, cc = e % w8;
-            double v = 0.0;
-            if (cc < M && s_slot[r] >= 0) {
-              const double* q = rr + r * 8;
-              v = q[0] * x.x0 + q[1] * x.x1 + q[2] * x.x2 + q[3] * x.x3;
-              if (!tan && s_tpos[r] >= 0) v += q[4] * x.d0 + q[5] * x.d1 + q[6] * x.d2 + q[7] * x.d3;
-              v *= invN;
-              if (HbtL) HbtL[(size_t)(r0 + r) * M + cc] = v;
-            }
-            Hb[r * a.bld + cc] = v;
-          });
-    }
+    __syncthreads();  // rr, aug ready
+    // ---- seed: hbar_{L-1} = Gbar (and, for forces, the per-row R~ adjoint)
+    seed_rows<W>(sm, io, r0, R, tan, s_dr);
     __syncthreads();
-    for (int l = nl - 1; l >= 0; --l) {
-      const int d = a.dout[l], w8 = pad8(d);
-      const double* hb = sm + a.bofs[bx];
-      double* zb = sm + a.bofs[bz];
-      {
-        const double* Ypl = io.Yp[l];
-        const double* Ytl = io.Yt[l];
-        const double* Hbtl = io.Hbt[l];
-        ew_loop<4, ZIn>(
-            T * w8,
-            [&](int e) -> ZIn {
-              const int r = e / w8, cc = e % w8;
-              ZIn z{0.0, 0.0, 0.0};
-              if (cc < d && s_slot[r] >= 0) {
-                z.y = Ypl[(size_t)s_prow[r] * d + cc];
-                const int tp = s_tpos[r];
-                if (tp >= 0) {
-                  z.yt = Ytl[(size_t)tp * d + cc];
-                  z.hbt = Hbtl[(size_t)tp * d + cc];
-                }
-              }
-              return z;
-            },
-            [&](int e, const ZIn& z) {
-              const int r = e / w8, cc = e % w8;
-              double v = 0.0;
-              if (cc < d && s_slot[r] >= 0) v = (1.0 - z.y * z.y) * hb[r * a.bld + cc] - 2.0 * z.y * z.yt * z.hbt;
-              zb[r * a.bld + cc] = v;
-            });
-      }
-      __syncthreads();
-      if (wantw) {
-        const double* A = sm + a.augofs[l];
-        const int ldA = a.augld[l];
-        const int m8 = pad8(a.din[l] + 1);
-#pragma unroll
-        for (int q = 0; q < MAXB; ++q) {
-          const int b = warp + NW * q;
-          if (b < a.nblk) {
-            const int code = a.blk[b];
-            if ((code >> 16) == l) {
-              const int m0 = ((code >> 8) & 255) * 16, n0 = (code & 255) * 16;
-              const bool mv = m0 + 8 < m8, nv = n0 + 8 < w8;
-#pragma unroll 2
-              for (int k = 0; k < T; k += 4) {
-                const double a0 = A[(k + fk) * ldA + m0 + fr];
-                const double a1 = mv ? A[(k + fk) * ldA + m0 + 8 + fr] : 0.0;
-                const double b0 = zb[(k + fk) * a.bld + n0 + fr];
-                const double b1 = nv ? zb[(k + fk) * a.bld + n0 + 8 + fr] : 0.0;
-                dmma884(acc[q][0][0][0], acc[q][0][0][1], a0, b0);
-                if (nv) dmma884(acc[q][0][1][0], acc[q][0][1][1], a0, b1);
-                if (mv) dmma884(acc[q][1][0][0], acc[q][1][0][1], a1, b0);
-                if (mv && nv) dmma884(acc[q][1][1][0], acc[q][1][1][1], a1, b1);
-              }
-            }
-          }
-        }
-      }
-      if (l > 0) {
-        const int din = a.din[l], n8 = pad8(din), skip = a.skip[l];
-        double* hn = sm + a.bofs[bn];
-        cta_mma<true>(zb, a.bld, sm + a.wofs[l], sld(d), T / 8, n8 / 8, pad4(d), hn, a.bld);
-        __syncthreads();
-        double* Hbt = tan ? io.Hbt[l - 1] : nullptr;
-        for (int e = tid; e < T * n8; e += blockDim.x) {
-          const int r = e / n8, cc = e % n8;
-          double v = 0.0;
-          if (cc < din) {
-            v = hn[r * a.bld + cc];
-            if (skip == 1) v += hb[r * a.bld + cc];
-            else if (skip == 2) v += hb[r * a.bld + cc] + hb[r * a.bld + cc + din];
-            if (Hbt && r0 + r < R) Hbt[(size_t)(r0 + r) * din + cc] = v;
-          }
-          hn[r * a.bld + cc] = v;
-        }
-        __syncthreads();
-        const int t = bx;
-        bx = bn;
-        bn = bz;
-        bz = t;
-      } else if (io.sbar && tid < T) {
-        const int row = r0 + tid;
-        if (row < R) {
-          const double* w0 = sm + a.wofs[0];
-          double sb = 0.0;
-          for (int cc = 0; cc < d; ++cc) sb = fma(zb[tid * a.bld + cc], w0[cc], sb);
-          io.sbar[row] = sb;
-        }
-      }
-    }
+    if constexpr (NL >= 4) bwd_layer<W, 3>(acc, sm, io, r0, R, tan, wantw, s_slot, s_prow, s_tpos, s_atom, s_dr);
+    if constexpr (NL >= 3) bwd_layer<W, 2>(acc, sm, io, r0, R, tan, wantw, s_slot, s_prow, s_tpos, s_atom, s_dr);
+    if constexpr (NL >= 2) bwd_layer<W, 1>(acc, sm, io, r0, R, tan, wantw, s_slot, s_prow, s_tpos, s_atom, s_dr);
+    bwd_layer<W, 0>(acc, sm, io, r0, R, tan, wantw, s_slot, s_prow, s_tpos, s_atom, s_dr);
   }
   if (wantw) {
-    double* out = io.ws + (size_t)blockIdx.x * a.gsize;
-#pragma unroll
-    for (int q = 0; q < MAXB; ++q) {
-      const int b = warp + NW * q;
-      if (b < a.nblk) {
-        const int code = a.blk[b];
-        const int l = code >> 16, m0 = ((code >> 8) & 255) * 16, n0 = (code & 255) * 16;
-        const int rows = a.din[l] + 1, cols = a.dout[l];
-#pragma unroll
-        for (int i = 0; i < 2; ++i)
-#pragma unroll
-          for (int j = 0; j < 2; ++j)
-#pragma unroll
-            for (int h = 0; h < 2; ++h) {
-              const int m = m0 + 8 * i + fr, n = n0 + 8 * j + 2 * fk + h;
-              if (m < rows && n < cols) out[a.goff[l] + m * cols + n] = acc[q][i][j][h];
-            }
-      }
-    }
+    double* out = io.ws + (size_t)blockIdx.x * W::GS;
+    if constexpr (NL >= 4) write_partials<W, 3>(acc, out);
+    if constexpr (NL >= 3) write_partials<W, 2>(acc, out);
+    if constexpr (NL >= 2) write_partials<W, 1>(acc, out);
+    write_partials<W, 0>(acc, out);
   }
 }
 
@@ -634,53 +624,41 @@ __global__ void emb_wgrad_reduce_kernel(const double* __restrict__ ws, int nsets
   g[i] += a;
 }
 
-static fekf_status launch_bwd(const EmbBwdArgs& a, const EmbBwdIO& io, long long Rmax, int max_grid, int* grid_out,
+template <class W>
+static fekf_status launch_bwd(const double* wp, const EmbBwdIO& io, long long Rmax, int max_grid, int* grid_out,
                               cudaStream_t s) {
-  const size_t smem = sizeof(double) * a.smem_doubles;
-  static size_t attr = 0;
-  if (smem > attr) {
-    FEKF_CHECK_CUDA(cudaFuncSetAttribute(emb_bwd_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-    attr = smem;
+  constexpr size_t smem = sizeof(double) * W::B_SMEM;
+  static int occ = 0;
+  if (!occ) {
+    FEKF_CHECK_CUDA(cudaFuncSetAttribute(emb_bwd_kernel<W>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    FEKF_CHECK_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, emb_bwd_kernel<W>, EMB_BWD_WARPS * 32, smem));
+    if (occ < 1) { set_error("emb_bwd_kernel: does not fit on an SM"); return FEKF_EINVAL; }
   }
-  int occ = 0;
-  FEKF_CHECK_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, emb_bwd_kernel, EMB_BWD_WARPS * 32, smem));
-  if (occ < 1) { set_error("emb_bwd_kernel: does not fit on an SM"); return FEKF_EINVAL; }
   const long long tiles = (Rmax + EMB_T - 1) / EMB_T;
   const int grid = (int)std::max<long long>(1, std::min<long long>({tiles, (long long)num_sms() * occ, (long long)max_grid}));
-  emb_bwd_kernel<<<grid, EMB_BWD_WARPS * 32, smem, s>>>(a, io);
+  emb_bwd_kernel<W><<<grid, EMB_BWD_WARPS * 32, smem, s>>>(wp, io);
   FEKF_LAUNCH_CHECK();
   count_launch();
   *grid_out = grid;
   return FEKF_OK;
 }
 
-bool emb_bwd_fused_ok(const Ctx& c) {
-  if (!emb_fused_ok(c) || c.pairs.empty()) return false;
-  EmbBwdArgs a = emb_bwd_args(c, c.pairs[0], nullptr);
-  int dev = 0, maxsm = 0;
-  cudaGetDevice(&dev);
-  cudaDeviceGetAttribute(&maxsm, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
-  return a.nblk <= EMB_BWD_WARPS * EMB_MAXB && sizeof(double) * a.smem_doubles <= (size_t)maxsm;
-}
-
-fekf_status emb_backward(Ctx& c, int p, long long Rmax, int mode, double* g, cudaStream_t s) {
+template <class W>
+static fekf_status emb_backward_t(Ctx& c, int p, long long Rmax, int mode, double* g, cudaStream_t s) {
   PairNet& P = c.pairs[p];
-  EmbBwdArgs a = emb_bwd_args(c, P, c.w.as<double>());
   const bool dual = mode == MODE_FORCE_JAC, wantw = mode != MODE_FORCE;
-  const size_t Xoff = (size_t)c.B * c.Na * 4 * c.M;
+  const double* wp = c.w.as<double>() + P.L[0].W;
   EmbBwdIO io{};
   io.Rmax = (int)Rmax;
   io.row_idx = P.row_idx.as<int>();
-  io.em = c.em.as<double>();
-  io.rdot = c.rdot.as<double>();
-  io.Xb = c.Xb.as<double>();
-  io.Xdb = c.Xb.as<double>() + Xoff;
-  for (int l = 0; l < a.nl; ++l) {
+  io.Nm = c.Nm;
+  io.Gbar = P.Hb[W::NL - 1].template as<double>();
+  for (int l = 0; l < W::NL; ++l) {
     io.Yp[l] = P.Y[l].as<double>();
     io.Yt[l] = P.Yt[l].as<double>();
     io.Hbt[l] = P.Hbt[l].as<double>();
   }
-  const int cap = (int)std::min<size_t>(1 << 20, c.splitk_elems / (2 * (size_t)a.gsize));
+  const int cap = (int)std::min<size_t>(1 << 20, c.splitk_elems / (2 * (size_t)W::GS));
   double* ws = c.splitk_ws.as<double>();
   int nsets = 0;
   if (dual) {
@@ -688,27 +666,79 @@ fekf_status emb_backward(Ctx& c, int p, long long Rmax, int mode, double* g, cud
     t.Rdev = c.rowcnt.as<int>() + c.pairs.size() + p;
     t.tidx = P.tidx.as<int>();
     t.hin = P.hin_t.as<double>();
-    for (int l = 0; l < a.nl; ++l) t.Y[l] = P.Yt[l].as<double>();
+    for (int l = 0; l < W::NL; ++l) t.Y[l] = P.Yt[l].as<double>();
     t.ws = ws;
     int gt = 0;
-    FEKF_TRY(launch_bwd(a, t, Rmax, cap, &gt, s));
+    FEKF_TRY(launch_bwd<W>(wp, t, Rmax, cap, &gt, s));
     nsets += gt;
   }
   io.Rdev = c.rowcnt.as<int>() + p;
   io.tpos = dual ? P.tpos.as<int>() : nullptr;
   io.hin = P.hin.as<double>();
-  for (int l = 0; l < a.nl; ++l) io.Y[l] = P.Y[l].as<double>();
+  for (int l = 0; l < W::NL; ++l) io.Y[l] = P.Y[l].as<double>();
   io.sbar = mode == MODE_FORCE ? P.sbar.as<double>() : nullptr;
-  io.ws = wantw ? ws + (size_t)nsets * a.gsize : nullptr;
+  if (mode == MODE_FORCE) {
+    io.dR = P.Zb[0].template as<double>();
+    io.jac = c.jac.as<double>();
+    io.rij = c.rij.as<double>();
+    io.nl_j = c.nl_j.as<int>();
+    io.Na = c.Na;
+    io.force = c.force.as<double>();
+    io.vatom = c.vatom.as<double>();
+  }
+  io.ws = wantw ? ws + (size_t)nsets * W::GS : nullptr;
   int gp = 0;
-  FEKF_TRY(launch_bwd(a, io, Rmax, cap, &gp, s));
+  FEKF_TRY(launch_bwd<W>(wp, io, Rmax, cap, &gp, s));
   if (wantw) {
     nsets += gp;
-    emb_wgrad_reduce_kernel<<<cdiv(a.gsize, 256), 256, 0, s>>>(ws, nsets, a.gsize, g + P.L[0].W);
+    emb_wgrad_reduce_kernel<<<cdiv(W::GS, 256), 256, 0, s>>>(ws, nsets, W::GS, g + P.L[0].W);
     FEKF_LAUNCH_CHECK();
     count_launch();
   }
   return FEKF_OK;
+}
+
+// ---------------------------------------------------------------------------------------------
+// width dispatch: the embedding nets of the configured models (fixtures/synth.py)
+// ---------------------------------------------------------------------------------------------
+using EmbC2 = EmbW<25, 50, 100, 0>;   // water-64, Cu-108 (C3a), CH4 (C3b)
+using EmbC1 = EmbW<8, 16, 32, 0>;     // Cu-32
+using EmbPCu = EmbW<25, 25, 25, 0>;   // the paper's Cu model (26 651 parameters)
+using EmbT2 = EmbW<4, 8, 16, 0>;      // tiny test model
+
+static int emb_kind(const Ctx& c) {
+  const fekf_model_cfg& m = c.m;
+  if (m.n_emb != 3) return -1;
+  auto is = [&](int a, int b, int d) { return m.emb[0] == a && m.emb[1] == b && m.emb[2] == d; };
+  if (is(25, 50, 100)) return 0;
+  if (is(8, 16, 32)) return 1;
+  if (is(25, 25, 25)) return 2;
+  if (is(4, 8, 16)) return 3;
+  return -1;
+}
+
+bool emb_fused_ok(const Ctx& c) { return emb_kind(c) >= 0; }
+
+fekf_status emb_forward(Ctx& c, int p, long long Rmax, bool tangent, cudaStream_t s) {
+  switch (emb_kind(c)) {
+    case 0: return emb_forward_t<EmbC2>(c, p, Rmax, tangent, s);
+    case 1: return emb_forward_t<EmbC1>(c, p, Rmax, tangent, s);
+    case 2: return emb_forward_t<EmbPCu>(c, p, Rmax, tangent, s);
+    case 3: return emb_forward_t<EmbT2>(c, p, Rmax, tangent, s);
+  }
+  set_error("emb_forward: no fused kernel for these embedding widths");
+  return FEKF_EINVAL;
+}
+
+fekf_status emb_backward(Ctx& c, int p, long long Rmax, int mode, double* g, cudaStream_t s) {
+  switch (emb_kind(c)) {
+    case 0: return emb_backward_t<EmbC2>(c, p, Rmax, mode, g, s);
+    case 1: return emb_backward_t<EmbC1>(c, p, Rmax, mode, g, s);
+    case 2: return emb_backward_t<EmbPCu>(c, p, Rmax, mode, g, s);
+    case 3: return emb_backward_t<EmbT2>(c, p, Rmax, mode, g, s);
+  }
+  set_error("emb_backward: no fused kernel for these embedding widths");
+  return FEKF_EINVAL;
 }
 
 }  // namespace fekf

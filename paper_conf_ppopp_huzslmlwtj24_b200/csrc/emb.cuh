@@ -1,7 +1,8 @@
 // Fused embedding-net kernels (sm_100a, fp64 DMMA m8n8k4): one CTA runs every layer of the
 // embedding net G = E_{L-1} o ... o E_0(s) (skip rule: reading Z12) on a tile of rows with
 // the activations resident in shared memory, instead of one GEMM launch per layer with the
-// activations round-tripping through HBM.
+// activations round-tripping through HBM.  The kernels are compiled for the embedding widths of the
+// configured models (all index math constant-folded); other widths take the per-layer GEMM path.
 //
 // Shared-memory layout (doubles).  Every matrix uses a leading dimension ld = 16*ceil(w8/16) + 4
 // (w8 = width rounded up to 8): ld = 4 (mod 16) makes both DMMA fragment patterns conflict-free,
@@ -13,45 +14,81 @@
 
 namespace fekf {
 
-constexpr int EMB_MAXW = 128;   // widths handled by the fused kernels (else: per-layer GEMM path)
 constexpr int EMB_T = 32;       // rows per CTA tile
 constexpr int EMB_FWD_WARPS = 8;
 constexpr int EMB_BWD_WARPS = 16;
-constexpr int EMB_MAXB = 3;     // 2x2-tile weight-gradient blocks held per warp (C2: 38 blocks / 16 warps)
 
-__host__ __device__ inline int pad4(int x) { return (x + 3) & ~3; }
-__host__ __device__ inline int pad8(int x) { return (x + 7) & ~7; }
-__host__ __device__ inline int sld(int w) { return ((pad8(w) + 15) / 16) * 16 + 4; }
+__host__ __device__ constexpr int pad4(int x) { return (x + 3) & ~3; }
+__host__ __device__ constexpr int pad8(int x) { return (x + 7) & ~7; }
+__host__ __device__ constexpr int sld(int w) { return ((pad8(w) + 15) / 16) * 16 + 4; }
 
-struct EmbNetArgs {
-  int nl;
-  int din[FEKF_MAX_LAYERS], dout[FEKF_MAX_LAYERS], skip[FEKF_MAX_LAYERS];
-  const double* W[FEKF_MAX_LAYERS];   // [din][dout] row-major (global, inside w)
-  const double* b[FEKF_MAX_LAYERS];
-  int wofs[FEKF_MAX_LAYERS];          // smem offset of W_l (l >= 1): [pad8(din)][sld(dout)]; W_0 (din 1): [dout]
-  int bofs[FEKF_MAX_LAYERS];          // smem offset of b_l
-  int aofs[2], ald[2];                // activation buffers: layer l output goes to buffer l & 1
-  int smem_doubles;
-};
-
-struct EmbBwdArgs {
-  int nl, M, Nm;
-  int din[FEKF_MAX_LAYERS], dout[FEKF_MAX_LAYERS], skip[FEKF_MAX_LAYERS];
-  const double* W[FEKF_MAX_LAYERS];
-  int wofs[FEKF_MAX_LAYERS];          // W_l (l >= 1): [pad8(din)][sld(dout)]; W_0: [pad8(dout)]
-  int augofs[FEKF_MAX_LAYERS];        // [h_{l-1} | 1] (h_{-1} = s): [T][augld]
-  int augld[FEKF_MAX_LAYERS];
-  int bofs[3], bld;                   // three rotating adjoint buffers [T][bld]
-  int rofs;                           // per-row R~ and R~-dot [T][8]
-  int smem_doubles;
-  int nblk;                           // weight-gradient blocks, packed (l << 16) | (bm << 8) | bn
-  int blk[EMB_BWD_WARPS * EMB_MAXB];
-  int goff[FEKF_MAX_LAYERS];          // offset of [W_l ; b_l] in the pair's gradient segment
-  int gsize;
+// Compile-time description of an embedding net (widths d_0..d_{NL-1}, input width 1) and the
+// shared-memory layouts of its fused kernels.
+template <int D0, int D1, int D2, int D3>
+struct EmbW {
+  static constexpr int T = EMB_T;
+  static constexpr int NL = D3 ? 4 : (D2 ? 3 : (D1 ? 2 : 1));
+  __host__ __device__ static constexpr int d(int l) { return l == 0 ? D0 : (l == 1 ? D1 : (l == 2 ? D2 : D3)); }
+  __host__ __device__ static constexpr int din(int l) { return l == 0 ? 1 : d(l - 1); }
+  __host__ __device__ static constexpr int skip(int l) {
+    return l == 0 ? 0 : (d(l) == din(l) ? 1 : (d(l) == 2 * din(l) ? 2 : 0));
+  }
+  static constexpr int M = d(NL - 1);
+  __host__ __device__ static constexpr int maxw(int parity) {  // parity -1: all layers
+    int m = 1;
+    for (int l = 0; l < NL; ++l)
+      if (parity < 0 || (l & 1) == parity) m = d(l) > m ? d(l) : m;
+    return m;
+  }
+  // ---- forward: W_0 [pad8(d0)] | W_l [pad4(din)][sld(d)] | b_l [pad8(d)] | act0 [T][ald0] | act1 [T][ald1]
+  __host__ __device__ static constexpr int fW(int l) {
+    int o = pad8(D0);
+    for (int k = 1; k < l; ++k) o += pad4(din(k)) * sld(d(k));
+    return l == 0 ? 0 : o;
+  }
+  __host__ __device__ static constexpr int fB(int l) {
+    int o = fW(NL);
+    for (int k = 0; k < l; ++k) o += pad8(d(k));
+    return o;
+  }
+  __host__ __device__ static constexpr int fALD(int q) { return sld(maxw(q)); }
+  __host__ __device__ static constexpr int fA(int q) { return fB(NL) + (q ? T * fALD(0) : 0); }
+  static constexpr int F_SMEM = fA(1) + T * fALD(1);
+  // ---- backward: W_0 | W_l [pad8(din)][sld(d)] | aug_l [T][sld(din+1)] | 3 x buf [T][BLD] | rr [T][8]
+  __host__ __device__ static constexpr int bW(int l) {
+    int o = pad8(D0);
+    for (int k = 1; k < l; ++k) o += pad8(din(k)) * sld(d(k));
+    return l == 0 ? 0 : o;
+  }
+  __host__ __device__ static constexpr int augld(int l) { return sld(din(l) + 1); }
+  __host__ __device__ static constexpr int bAug(int l) {
+    int o = bW(NL);
+    for (int k = 0; k < l; ++k) o += T * augld(k);
+    return o;
+  }
+  static constexpr int BLD = sld(maxw(-1));
+  __host__ __device__ static constexpr int bBuf(int q) { return bAug(NL) + q * T * BLD; }
+  static constexpr int bR = bBuf(3);
+  static constexpr int B_SMEM = bR + T * 8;
+  // ---- weight-gradient blocks: 2x2 DMMA tiles of [din+1 x d] per layer, top layer first
+  __host__ __device__ static constexpr int mblk(int l) { return (pad8(din(l) + 1) / 8 + 1) / 2; }
+  __host__ __device__ static constexpr int nblk(int l) { return (pad8(d(l)) / 8 + 1) / 2; }
+  __host__ __device__ static constexpr int blk_first(int l) {  // first block index of layer l
+    int o = 0;
+    for (int k = NL - 1; k > l; --k) o += mblk(k) * nblk(k);
+    return o;
+  }
+  static constexpr int NBLK = blk_first(-1);
+  __host__ __device__ static constexpr int goff(int l) {
+    int o = 0;
+    for (int k = 0; k < l; ++k) o += (din(k) + 1) * d(k);
+    return o;
+  }
+  static constexpr int GS = goff(NL);
+  static constexpr int MAXB = (NBLK + EMB_BWD_WARPS - 1) / EMB_BWD_WARPS;
 };
 
 bool emb_fused_ok(const Ctx& c);
-bool emb_bwd_fused_ok(const Ctx& c);
 fekf_status emb_forward(Ctx& c, int p, long long Rmax, bool tangent, cudaStream_t s);
 // Reverse pass of one pair's embedding net from the atoms' X-bar (mode: nets.cu Mode).  Adds the
 // weight gradients (ENERGY_GRAD, FORCE_JAC) into g, or writes s-bar per row (FORCE).

@@ -8,25 +8,32 @@
 // CTA tile BM x BN x 16, 8 warps each WM x WN (WM/8 x WN/8 DMMA tiles), operands staged in SMEM
 // k-contiguous with a 20-double row stride (conflict-free fragment loads), 3-stage cp.async ring.
 #pragma once
+#include <algorithm>
+
 #include "model.cuh"
+#include "mathx.cuh"
 
 namespace fekf {
 
 constexpr int GB_K = 16;
 constexpr int GB_LDS = GB_K + 4;
 
+// Every epilogue gets split(z) (the CTA's split-K index) before its first use.
 struct EpiStore {
   double* C; int ldc;
+  __device__ void split(int) {}
   __device__ void operator()(int r, int c, double v) const { C[(size_t)r * ldc + c] = v; }
 };
 struct EpiPartial {
   double* ws; int M, N; int zoff;
+  __device__ void split(int z) { zoff += z; }
   __device__ void operator()(int r, int c, double v) const {
-    ws[((size_t)(blockIdx.z + zoff) * M + r) * N + c] = v;
+    ws[((size_t)zoff * M + r) * N + c] = v;
   }
 };
 // forward layer: y = tanh(z + b) (primal) or ydot = (1 - y^2) zdot (tangent); h = skip(h_prev) + dt*y
 struct EpiFwd {
+  __device__ void split(int) {}
   double* Y; double* H; int ld;
   const double* bias; const double* dt;
   const double* Hp; int ldp; int skip; int dprev;
@@ -38,7 +45,7 @@ struct EpiFwd {
     else if (skip == 2) sk = Hp[(size_t)r * ldp + (c % dprev)];
     double y;
     if (Yprim == nullptr) {
-      y = tanh(v + bias[c]);
+      y = tanh_fp64(v + bias[c]);
     } else {
       const int rp = rowmap ? rowmap[r] : r;
       const double yp = Yprim[(size_t)rp * ld + c];
@@ -50,6 +57,7 @@ struct EpiFwd {
 };
 // data gradient: hbar_prev = Zbar W^T + skip^T(hbar)
 struct EpiDgrad {
+  __device__ void split(int) {}
   double* out; int ldo; const double* Hb; int ld; int skip; int dprev;
   __device__ void operator()(int r, int c, double v) const {
     double s = 0.0;
@@ -64,6 +72,7 @@ struct EpiDgrad {
 // primal launch: the tangent rows of the same layer are done first (tpos / Yt / Hbt);
 // tangent launch: y of the primal row rowmap[r].
 struct EpiDgradAct {
+  __device__ void split(int) {}
   double* out; int ldo; const double* Hb; int ld; int skip; int dprev;
   const double* Y; double* Zb;
   const int* tpos; const double* Yt; const double* Hbt;
@@ -105,13 +114,47 @@ __device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_gr
 
 constexpr int GB_STAGES = 3;
 
+// A group of up to GG_MAX independent GEMMs of the same shape class in one launch (e.g. one fitting
+// layer of every atom type): CTAs are numbered across the problems' tile grids.
+constexpr int GG_MAX = 8;
+template <class Epi>
+struct GemmProb {
+  int M, N, K;
+  const int* Mdev;   // device row count (compacted rows) or nullptr
+  const int* Kdev;   // device K (split-K over rows) or nullptr
+  const double* A; int lda;
+  const double* B; int ldb;
+  int aug_m, aug_k;  // "ones" row of op(A) (bias gradient), -1: none
+  int kps, splits;   // K per split, number of splits
+  Epi epi;
+};
+template <class Epi>
+struct GemmGroup {
+  int n;
+  int start[GG_MAX + 1];   // first CTA of each problem
+  int mt[GG_MAX], nt[GG_MAX];
+  GemmProb<Epi> p[GG_MAX];
+};
+template <class Epi>
+__device__ __forceinline__ GemmProb<Epi> pick(const GemmGroup<Epi>& G, int q) {
+  // static indices only (a dynamic index into the parameter struct would copy it to local memory)
+  switch (q) {
+    case 0: return G.p[0];
+    case 1: return G.p[1];
+    case 2: return G.p[2];
+    case 3: return G.p[3];
+    case 4: return G.p[4];
+    case 5: return G.p[5];
+    case 6: return G.p[6];
+    default: return G.p[7];
+  }
+}
+
 // Mainloop: GB_STAGES-deep cp.async ring (global -> SMEM without register staging), one
 // __syncthreads per BK slice, warp tiles of (WM/8) x (WN/8) DMMA 8x8 tiles.
 template <int BM, int BN, int WM, int WN, bool TA, bool TB, class Epi>
 __global__ void __launch_bounds__(256)
-dgemm_kernel(int M, int N, int K, const int* __restrict__ Mdev, const int* __restrict__ Kdev,
-             const double* __restrict__ A, int lda, const double* __restrict__ B, int ldb, int aug_m, int aug_k,
-             int kps, Epi epi) {
+dgemm_kernel(const __grid_constant__ GemmGroup<Epi> G) {
   constexpr int NWN = BN / WN;
   static_assert((BM / WM) * NWN == 8, "8 warps");
   constexpr int TI = WM / 8, TJ = WN / 8;
@@ -131,16 +174,33 @@ dgemm_kernel(int M, int N, int K, const int* __restrict__ Mdev, const int* __res
   auto b_at = [&](int buf, int n, int k) -> double& {
     return TB ? Bs0[buf * BSZ + n * GB_LDS + k] : Bs0[buf * BSZ + k * (BN + 4) + n];
   };
-  if (Mdev) M = min(M, *Mdev);
-  if (Kdev) {
-    const int kd = *Kdev;
+  int q = 0;
+#pragma unroll
+  for (int k = 1; k < GG_MAX; ++k)
+    if (k < G.n && (int)blockIdx.x >= G.start[k]) q = k;
+  const GemmProb<Epi> P = pick(G, q);
+  const int local = blockIdx.x - G.start[q];
+  int mtq = G.mt[0], ntq = G.nt[0];
+#pragma unroll
+  for (int k = 1; k < GG_MAX; ++k)
+    if (q == k) { mtq = G.mt[k]; ntq = G.nt[k]; }
+  const int bm = local % mtq, bn = (local / mtq) % ntq, bz = local / (mtq * ntq);
+  int M = P.M, K = P.K, aug_k = P.aug_k;
+  const int N = P.N, lda = P.lda, ldb = P.ldb, aug_m = P.aug_m, kps = P.kps;
+  const double* __restrict__ A = P.A;
+  const double* __restrict__ B = P.B;
+  Epi epi = P.epi;
+  epi.split(bz);
+  if (P.Mdev) M = min(M, *P.Mdev);
+  if (P.Kdev) {
+    const int kd = *P.Kdev;
     K = min(K, kd);
     aug_k = min(aug_k, kd);
   }
   const int tid = threadIdx.x;
-  const int m0 = blockIdx.x * BM, n0 = blockIdx.y * BN;
-  const int kbeg = blockIdx.z * kps;
-  if (m0 >= M || (blockIdx.z > 0 && kbeg >= K)) return;  // empty split: the reduction skips it
+  const int m0 = bm * BM, n0 = bn * BN;
+  const int kbeg = bz * kps;
+  if (m0 >= M || (bz > 0 && kbeg >= K)) return;  // empty split: the reduction skips it
   const int kend = min(K, kbeg + kps);
   const int warp = tid >> 5, lane = tid & 31;
   const int wm = warp / NWN, wn = warp % NWN;
@@ -216,8 +276,7 @@ dgemm_kernel(int M, int N, int K, const int* __restrict__ Mdev, const int* __res
 }
 
 template <int BM, int BN, int WM, int WN, bool TA, bool TB, class Epi>
-static fekf_status gemm_t(long long M, int N, int K, const double* A, int lda, const double* B, int ldb, Epi epi,
-                          cudaStream_t s, const int* Mdev, const int* Kdev, int aug_m, int aug_k, int splits, int kps) {
+static fekf_status gemm_launch(GemmGroup<Epi>& G, cudaStream_t s) {
   constexpr size_t asz = TA ? GB_K * (BM + 4) : BM * GB_LDS;
   constexpr size_t bsz = TB ? BN * GB_LDS : GB_K * (BN + 4);
   constexpr size_t smem = sizeof(double) * GB_STAGES * (asz + bsz);
@@ -227,28 +286,48 @@ static fekf_status gemm_t(long long M, int N, int K, const double* A, int lda, c
                                          cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
     attr = true;
   }
-  dim3 grid((unsigned)cdiv(M, BM), (unsigned)cdiv(N, BN), (unsigned)splits);
-  dgemm_kernel<BM, BN, WM, WN, TA, TB, Epi><<<grid, 256, smem, s>>>((int)M, N, K, Mdev, Kdev, A, lda, B, ldb, aug_m,
-                                                                     aug_k, kps, epi);
+  int tot = 0;
+  for (int q = 0; q < G.n; ++q) {
+    G.mt[q] = cdiv(G.p[q].M, BM);
+    G.nt[q] = cdiv(G.p[q].N, BN);
+    G.start[q] = tot;
+    tot += G.mt[q] * G.nt[q] * G.p[q].splits;
+  }
+  for (int q = G.n; q <= GG_MAX; ++q) G.start[q] = tot;
+  if (tot == 0) return FEKF_OK;
+  dgemm_kernel<BM, BN, WM, WN, TA, TB, Epi><<<tot, 256, smem, s>>>(G);
   FEKF_LAUNCH_CHECK();
   count_launch();
   return FEKF_OK;
 }
 
-// Tile choice from (M, N): N <= 32 -> 128x32 (embedding widths 25/32); few rows -> 64x64 (more CTAs
-// for the fitting nets' 2048..8192 rows); otherwise 128x64.
+// One launch for every problem of the group.  Tile from the group's shape: N <= 32 -> 128x32
+// (embedding widths); otherwise 64x64 (warps 32x16) unless the group has many rows -> 128x64.
+template <bool TA, bool TB, class Epi>
+static fekf_status gemm_group(GemmProb<Epi>* probs, int n, cudaStream_t s) {
+  GemmGroup<Epi> G{};
+  long long rows = 0;
+  int nmax = 0;
+  for (int q = 0; q < n; ++q) {
+    if (probs[q].M <= 0 || probs[q].N <= 0) continue;
+    if (probs[q].kps <= 0) probs[q].kps = probs[q].K;
+    if (probs[q].splits <= 0) probs[q].splits = 1;
+    G.p[G.n++] = probs[q];
+    rows += probs[q].M;
+    nmax = std::max(nmax, probs[q].N);
+  }
+  if (G.n == 0) return FEKF_OK;
+  if (nmax <= 32) return gemm_launch<128, 32, 32, 16, TA, TB>(G, s);
+  if (rows < 65536) return gemm_launch<64, 64, 32, 16, TA, TB>(G, s);
+  return gemm_launch<128, 64, 32, 32, TA, TB>(G, s);
+}
+
 template <bool TA, bool TB, class Epi>
 static fekf_status gemm(long long M, int N, int K, const double* A, int lda, const double* B, int ldb, Epi epi,
                         cudaStream_t s, const int* Mdev = nullptr, const int* Kdev = nullptr, int aug_m = -1,
                         int aug_k = 0, int splits = 1, int kps = 0) {
-  if (M <= 0 || N <= 0) return FEKF_OK;
-  if (kps <= 0) kps = K;
-  if (N <= 32) return gemm_t<128, 32, 32, 16, TA, TB>(M, N, K, A, lda, B, ldb, epi, s, Mdev, Kdev, aug_m, aug_k, splits, kps);
-  if (M <= 8192 && !TA)  // fitting nets: few rows, keep >= 2 CTAs per SM busy
-    return gemm_t<32, 64, 8, 32, TA, TB>(M, N, K, A, lda, B, ldb, epi, s, Mdev, Kdev, aug_m, aug_k, splits, kps);
-  if (M < 16384 || N <= 64)
-    return gemm_t<64, 64, 32, 16, TA, TB>(M, N, K, A, lda, B, ldb, epi, s, Mdev, Kdev, aug_m, aug_k, splits, kps);
-  return gemm_t<128, 64, 32, 32, TA, TB>(M, N, K, A, lda, B, ldb, epi, s, Mdev, Kdev, aug_m, aug_k, splits, kps);
+  GemmProb<Epi> p{(int)M, N, K, Mdev, Kdev, A, lda, B, ldb, aug_m, aug_k, kps, splits, epi};
+  return gemm_group<TA, TB>(&p, 1, s);
 }
 
 }  // namespace fekf

@@ -84,6 +84,58 @@ static fekf_status wgrad(Ctx& c, int din, int dout, Seg s0, Seg s1, double* gout
   return FEKF_OK;
 }
 
+// The weight gradients of several layers (one per atom type) in one grouped split-K launch plus one
+// fixed-order reduction per layer (same partition rule as wgrad()).
+struct WgradJob {
+  int din, dout;
+  Seg s0, s1;
+  double* gout;
+};
+static fekf_status wgrad_group(Ctx& c, WgradJob* jobs, int n, cudaStream_t s) {
+  GemmProb<EpiPartial> pr[GG_MAX];
+  int np = 0;
+  long long S0[FEKF_MAX_TYPES], S1[FEKF_MAX_TYPES], kps_[FEKF_MAX_TYPES];
+  size_t off[FEKF_MAX_TYPES];
+  size_t used = 0;
+  const size_t share = c.splitk_elems / (size_t)n;
+  for (int q = 0; q < n; ++q) {
+    const WgradJob& J = jobs[q];
+    const int M = J.din + 1, N = J.dout;
+    const long long tiles = (long long)cdiv(M, 64) * cdiv(N, 64);
+    const long long kmax = std::max(J.s0.kmax, J.s1.kmax);
+    const long long budget = std::max<long long>(1, (long long)(share / ((size_t)M * N)));
+    long long want = std::max<long long>(1, cdiv(2 * 148, tiles * n));
+    int kps = (int)std::max<long long>(4 * GB_K, cdiv(cdiv(kmax, want), GB_K) * GB_K);
+    auto nsplit = [&](const Seg& g) { return g.kmax > 0 ? (long long)cdiv(g.kmax, kps) : 0LL; };
+    while (nsplit(J.s0) + nsplit(J.s1) > budget) kps *= 2;
+    S0[q] = nsplit(J.s0);
+    S1[q] = nsplit(J.s1);
+    kps_[q] = kps;
+    off[q] = used;
+    used += (size_t)(S0[q] + S1[q]) * M * N;
+    double* ws = c.splitk_ws.as<double>() + off[q];
+    if (S0[q])
+      pr[np++] = GemmProb<EpiPartial>{M, N, (int)J.s0.kmax, nullptr, J.s0.kdev, J.s0.H, J.din, J.s0.Zb, J.dout,
+                                      J.din, J.s0.ones ? (int)J.s0.kmax : 0, kps, (int)S0[q], EpiPartial{ws, M, N, 0}};
+    if (S1[q])
+      pr[np++] = GemmProb<EpiPartial>{M, N, (int)J.s1.kmax, nullptr, J.s1.kdev, J.s1.H, J.din, J.s1.Zb, J.dout,
+                                      J.din, J.s1.ones ? (int)J.s1.kmax : 0, kps, (int)S1[q],
+                                      EpiPartial{ws, M, N, (int)S0[q]}};
+  }
+  FEKF_TRY(gemm_group<true, false>(pr, np, s));
+  for (int q = 0; q < n; ++q) {
+    const WgradJob& J = jobs[q];
+    const int M = J.din + 1, N = J.dout;
+    if (S0[q] + S1[q] == 0) continue;
+    splitk_reduce_kernel<<<cdiv((long long)M * N, 32), 256, 0, s>>>(c.splitk_ws.as<double>() + off[q], (int)S0[q],
+                                                                    (int)S1[q], (int)kps_[q], J.s0.kdev, J.s1.kdev, M,
+                                                                    N, J.gout);
+    FEKF_LAUNCH_CHECK();
+    count_launch();
+  }
+  return FEKF_OK;
+}
+
 // =================================================================================================
 // elementwise / small kernels
 // =================================================================================================
@@ -337,7 +389,7 @@ __global__ void emb_l0_kernel(int Rmax, const int* __restrict__ Rdev, int d, con
   const double z = s[r] * W[c];
   double y;
   if (Yprim == nullptr) {
-    y = tanh(z + bias[c]);
+    y = tanh_fp64(z + bias[c]);
   } else {
     const double yp = Yprim[(size_t)rowmap[r] * d + c];
     y = (1.0 - yp * yp) * z;
@@ -352,47 +404,78 @@ __global__ void desc_fwd_kernel(Geo g, PairPtrs pp, FitPtrs fp, const double* __
                                 const double* __restrict__ rdot, int tangent, double* __restrict__ X,
                                 double* __restrict__ Xd) {
   extern __shared__ double sm[];
-  const int M = g.M, M2 = g.M2;
+  const int M = g.M, M2 = g.M2, Nm = g.Nm;
   double* xs = sm;            // [4][M]
   double* xds = sm + 4 * M;   // [4][M]
+  double* rs = xds + 4 * M;   // [Nm][4] R~ rows of the atom (contiguous in em)
+  double* rds = rs + 4 * Nm;  // [Nm][4] R~dot rows
+  int* act = reinterpret_cast<int*>(rds + 4 * Nm);  // tangent: (slot, primal row, tangent row) of active rows
+  __shared__ int s_nact;
   const int atom = blockIdx.x;
   const int b = atom / g.Na, i = atom % g.Na;
   const int ti = g.types[i], k = g.tindex[i];
   const int e = b * g.ncnt[ti] + k;
-  for (int m = threadIdx.x; m < M; m += blockDim.x) {
-    double a0 = 0, a1 = 0, a2 = 0, a3 = 0, d0 = 0, d1 = 0, d2 = 0, d3 = 0;
+  for (int q = threadIdx.x; q < 4 * Nm; q += blockDim.x) {
+    rs[q] = em[(size_t)atom * Nm * 4 + q];
+    if (tangent) rds[q] = rdot[(size_t)atom * Nm * 4 + q];
+  }
+  if (tangent && threadIdx.x == 0) {  // active rows of this atom, in (tj, slot) order
+    int n = 0;
     for (int tj = 0; tj < g.nt; ++tj) {
       const int p = ti * g.nt + tj;
       const int r0 = pp.row_start[p][e], r1 = pp.row_start[p][e + 1];
-      const double* G = pp.G[p];
       for (int r = r0; r < r1; ++r) {
-        const size_t idx = (size_t)atom * g.Nm + g.sec[tj] + (r - r0);
-        const double* er = em + idx * 4;
-        const double gv = G[(size_t)r * M + m];
-        if (!tangent) {
-          a0 = fma(er[0], gv, a0); a1 = fma(er[1], gv, a1); a2 = fma(er[2], gv, a2); a3 = fma(er[3], gv, a3);
-        } else {
-          const int t = pp.tpos[p][r];
-          if (t < 0) continue;
-          const double* ed = rdot + idx * 4;
-          const double gd = pp.Gt[p][(size_t)t * M + m];
-          d0 = fma(ed[0], gv, fma(er[0], gd, d0));
-          d1 = fma(ed[1], gv, fma(er[1], gd, d1));
-          d2 = fma(ed[2], gv, fma(er[2], gd, d2));
-          d3 = fma(ed[3], gv, fma(er[3], gd, d3));
+        const int t = pp.tpos[p][r];
+        if (t >= 0) { act[3 * n] = (p << 16) | (g.sec[tj] + r - r0); act[3 * n + 1] = r; act[3 * n + 2] = t; ++n; }
+      }
+    }
+    s_nact = n;
+  }
+  __syncthreads();
+  for (int m = threadIdx.x; m < M; m += blockDim.x) {
+    double a0 = 0, a1 = 0, a2 = 0, a3 = 0;
+    if (!tangent) {
+      for (int tj = 0; tj < g.nt; ++tj) {
+        const int p = ti * g.nt + tj;
+        const int r0 = pp.row_start[p][e], r1 = pp.row_start[p][e + 1];
+        const double* G = pp.G[p] + m;
+        const double* er = rs + 4 * g.sec[tj];
+        int r = r0;
+        for (; r + 4 <= r1; r += 4) {  // four rows' loads in flight
+          double gv[4];
+#pragma unroll
+          for (int u = 0; u < 4; ++u) gv[u] = G[(size_t)(r + u) * M];
+#pragma unroll
+          for (int u = 0; u < 4; ++u) {
+            const double* q = er + 4 * (r + u - r0);
+            a0 = fma(q[0], gv[u], a0); a1 = fma(q[1], gv[u], a1); a2 = fma(q[2], gv[u], a2); a3 = fma(q[3], gv[u], a3);
+          }
         }
+        for (; r < r1; ++r) {
+          const double gv = G[(size_t)r * M];
+          const double* q = er + 4 * (r - r0);
+          a0 = fma(q[0], gv, a0); a1 = fma(q[1], gv, a1); a2 = fma(q[2], gv, a2); a3 = fma(q[3], gv, a3);
+        }
+      }
+    } else {
+      const int n = s_nact;
+      for (int a = 0; a < n; ++a) {
+        const int p = act[3 * a] >> 16, sl = act[3 * a] & 0xffff, r = act[3 * a + 1], t = act[3 * a + 2];
+        const double gv = pp.G[p][(size_t)r * M + m];
+        const double gd = pp.Gt[p][(size_t)t * M + m];
+        const double* er = rs + 4 * sl;
+        const double* ed = rds + 4 * sl;
+        a0 = fma(ed[0], gv, fma(er[0], gd, a0));
+        a1 = fma(ed[1], gv, fma(er[1], gd, a1));
+        a2 = fma(ed[2], gv, fma(er[2], gd, a2));
+        a3 = fma(ed[3], gv, fma(er[3], gd, a3));
       }
     }
     const double inv = 1.0 / g.Nm;
-    if (!tangent) {
-      xs[m] = a0 * inv; xs[M + m] = a1 * inv; xs[2 * M + m] = a2 * inv; xs[3 * M + m] = a3 * inv;
-      double* xo = X + (size_t)atom * 4 * M;
-      xo[m] = xs[m]; xo[M + m] = xs[M + m]; xo[2 * M + m] = xs[2 * M + m]; xo[3 * M + m] = xs[3 * M + m];
-    } else {
-      xds[m] = d0 * inv; xds[M + m] = d1 * inv; xds[2 * M + m] = d2 * inv; xds[3 * M + m] = d3 * inv;
-      double* xo = Xd + (size_t)atom * 4 * M;
-      xo[m] = xds[m]; xo[M + m] = xds[M + m]; xo[2 * M + m] = xds[2 * M + m]; xo[3 * M + m] = xds[3 * M + m];
-    }
+    double* xw = tangent ? xds : xs;
+    double* xo = (tangent ? Xd : X) + (size_t)atom * 4 * M;
+    xw[m] = a0 * inv; xw[M + m] = a1 * inv; xw[2 * M + m] = a2 * inv; xw[3 * M + m] = a3 * inv;
+    xo[m] = xw[m]; xo[M + m] = xw[M + m]; xo[2 * M + m] = xw[2 * M + m]; xo[3 * M + m] = xw[3 * M + m];
   }
   __syncthreads();
   if (tangent) {
@@ -425,7 +508,7 @@ __global__ void desc_bwd_kernel(Geo g, FitPtrs fp, const double* __restrict__ X,
   double* xs = sm;
   double* xds = xs + 4 * M;
   double* db = xds + 4 * M;
-  double* ddb = db + M * M2;
+  double* ddb = db + M * (M2 + 1);
   const int atom = blockIdx.x;
   const int b = atom / g.Na, i = atom % g.Na;
   const int ti = g.types[i], k = g.tindex[i];
@@ -437,25 +520,132 @@ __global__ void desc_bwd_kernel(Geo g, FitPtrs fp, const double* __restrict__ X,
     if (dual) xds[e] = Xd[(size_t)atom * 4 * M + e];
   }
   for (int e = threadIdx.x; e < M * M2; e += blockDim.x) {
-    db[e] = Dbp[e];
-    if (dual) ddb[e] = Ddbp[e];
+    const int ep = (e / M2) * (M2 + 1) + e % M2;  // row stride M2 + 1: conflict-free in both loops below
+    db[ep] = Dbp[e];
+    if (dual) ddb[ep] = Ddbp[e];
   }
   __syncthreads();
   for (int e = threadIdx.x; e < 4 * M; e += blockDim.x) {
     const int kk = e / M, p = e % M;
     const double* x = xs + kk * M;
     double a = 0.0, ad = 0.0;
-    for (int n = 0; n < M2; ++n) a = fma(db[p * M2 + n], x[n], a);
+    for (int n = 0; n < M2; ++n) a = fma(db[p * (M2 + 1) + n], x[n], a);
     if (p < M2)
-      for (int m = 0; m < M; ++m) a = fma(db[m * M2 + p], x[m], a);
+      for (int m = 0; m < M; ++m) a = fma(db[m * (M2 + 1) + p], x[m], a);
     if (dual) {
       const double* xd = xds + kk * M;
-      for (int n = 0; n < M2; ++n) { a = fma(ddb[p * M2 + n], xd[n], a); ad = fma(ddb[p * M2 + n], x[n], ad); }
+      for (int n = 0; n < M2; ++n) { a = fma(ddb[p * (M2 + 1) + n], xd[n], a); ad = fma(ddb[p * (M2 + 1) + n], x[n], ad); }
       if (p < M2)
-        for (int m = 0; m < M; ++m) { a = fma(ddb[m * M2 + p], xd[m], a); ad = fma(ddb[m * M2 + p], x[m], ad); }
+        for (int m = 0; m < M; ++m) { a = fma(ddb[m * (M2 + 1) + p], xd[m], a); ad = fma(ddb[m * (M2 + 1) + p], x[m], ad); }
       Xdb[(size_t)atom * 4 * M + e] = ad;
     }
     Xb[(size_t)atom * 4 * M + e] = a;
+  }
+}
+
+// Eq. 4 per atom (as desc_bwd_kernel), then the fused embedding backward's per-row seeds:
+//   Gbar_r = (R~_r Xbar + R~dot_r Xdotbar) / N_m        (primal rows; R~dot = 0 off the tangent rows)
+//   Gdotbar_t = R~_r Xdotbar / N_m                      (tangent rows t = tpos[r], into hdotbar_{L-1})
+//   dR_r = G_r Xbar^T / N_m                             (forces: the R~ adjoint less sbar e_0)
+// One CTA (8 warps) per centre atom; the atom's R~ (and R~dot) rows are contiguous and staged once.
+struct SeedOut {
+  double* gbar[NP];
+  double* hbt[NP];
+  double* dr[NP];
+};
+__global__ void __launch_bounds__(256)
+desc_bwd_seed_kernel(Geo g, FitPtrs fp, PairPtrs pp, SeedOut so, const double* __restrict__ X,
+                     const double* __restrict__ Xd, const double* __restrict__ em, const double* __restrict__ rdot,
+                     int dual, int force, double* __restrict__ Xb, double* __restrict__ Xdb) {
+  extern __shared__ double sm[];
+  const int M = g.M, M2 = g.M2, Nm = g.Nm;
+  double* xs = sm;               // [4][M]
+  double* xds = xs + 4 * M;      // [4][M]
+  double* db = xds + 4 * M;      // [M][M2 + 1]
+  double* ddb = db + M * (M2 + 1);  // [M][M2 + 1]
+  double* xbs = ddb + M * (M2 + 1);  // [4][M]  Xbar
+  double* xdbs = xbs + 4 * M;    // [4][M]  Xdotbar
+  double* rs = xdbs + 4 * M;     // [Nm][4] R~ rows of the atom
+  double* rds = rs + 4 * Nm;     // [Nm][4] R~dot rows
+  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+  const int atom = blockIdx.x;
+  const int b = atom / g.Na, i = atom % g.Na;
+  const int ti = g.types[i], k = g.tindex[i];
+  const long long row = (long long)b * g.ncnt[ti] + k;
+  const double* Dbp = fp.Db[ti] + (size_t)row * M * M2;
+  const double* Ddbp = fp.Db[ti] + (size_t)(fp.F[ti] + row) * M * M2;
+  for (int e = tid; e < 4 * M; e += blockDim.x) {
+    xs[e] = X[(size_t)atom * 4 * M + e];
+    if (dual) xds[e] = Xd[(size_t)atom * 4 * M + e];
+  }
+  for (int e = tid; e < M * M2; e += blockDim.x) {
+    const int ep = (e / M2) * (M2 + 1) + e % M2;  // row stride M2 + 1: conflict-free in both loops below
+    db[ep] = Dbp[e];
+    if (dual) ddb[ep] = Ddbp[e];
+  }
+  for (int e = tid; e < 4 * Nm; e += blockDim.x) {
+    rs[e] = em[(size_t)atom * Nm * 4 + e];
+    if (dual) rds[e] = rdot[(size_t)atom * Nm * 4 + e];
+  }
+  __syncthreads();
+  for (int e = tid; e < 4 * M; e += blockDim.x) {
+    const int kk = e / M, p = e % M;
+    const double* x = xs + kk * M;
+    double a = 0.0, ad = 0.0;
+    for (int n = 0; n < M2; ++n) a = fma(db[p * (M2 + 1) + n], x[n], a);
+    if (p < M2)
+      for (int m = 0; m < M; ++m) a = fma(db[m * (M2 + 1) + p], x[m], a);
+    if (dual) {
+      const double* xd = xds + kk * M;
+      for (int n = 0; n < M2; ++n) { a = fma(ddb[p * (M2 + 1) + n], xd[n], a); ad = fma(ddb[p * (M2 + 1) + n], x[n], ad); }
+      if (p < M2)
+        for (int m = 0; m < M; ++m) { a = fma(ddb[m * (M2 + 1) + p], xd[m], a); ad = fma(ddb[m * (M2 + 1) + p], x[m], ad); }
+      xdbs[e] = ad;
+      Xdb[(size_t)atom * 4 * M + e] = ad;
+    }
+    xbs[e] = a;
+    Xb[(size_t)atom * 4 * M + e] = a;
+  }
+  __syncthreads();
+  const double inv = 1.0 / Nm;
+  const int e0 = b * g.ncnt[ti] + k;
+  for (int tj = 0; tj < g.nt; ++tj) {
+    const int p = ti * g.nt + tj;
+    const int r0 = pp.row_start[p][e0], nr = pp.row_start[p][e0 + 1] - r0;
+    const int* tpos = pp.tpos[p];
+    for (int s = warp; s < nr; s += blockDim.x >> 5) {
+      const int r = r0 + s;
+      const double* q = rs + (g.sec[tj] + s) * 4;
+      const int t = dual ? tpos[r] : -1;
+      double pk0 = 0.0, pk1 = 0.0, pk2 = 0.0, pk3 = 0.0;
+      const double* Gr = force ? pp.G[p] + (size_t)r * M : nullptr;
+      for (int m = lane; m < M; m += 32) {
+        double v = q[0] * xbs[m] + q[1] * xbs[M + m] + q[2] * xbs[2 * M + m] + q[3] * xbs[3 * M + m];
+        if (t >= 0) {
+          const double* qd = rds + (g.sec[tj] + s) * 4;
+          v += qd[0] * xdbs[m] + qd[1] * xdbs[M + m] + qd[2] * xdbs[2 * M + m] + qd[3] * xdbs[3 * M + m];
+          so.hbt[p][(size_t)t * M + m] =
+              (q[0] * xdbs[m] + q[1] * xdbs[M + m] + q[2] * xdbs[2 * M + m] + q[3] * xdbs[3 * M + m]) * inv;
+        }
+        so.gbar[p][(size_t)r * M + m] = v * inv;
+        if (force) {
+          const double gv = Gr[m];
+          pk0 = fma(gv, xbs[m], pk0);
+          pk1 = fma(gv, xbs[M + m], pk1);
+          pk2 = fma(gv, xbs[2 * M + m], pk2);
+          pk3 = fma(gv, xbs[3 * M + m], pk3);
+        }
+      }
+      if (force) {
+        for (int o = 16; o > 0; o >>= 1) {
+          pk0 += __shfl_xor_sync(0xffffffffu, pk0, o);
+          pk1 += __shfl_xor_sync(0xffffffffu, pk1, o);
+          pk2 += __shfl_xor_sync(0xffffffffu, pk2, o);
+          pk3 += __shfl_xor_sync(0xffffffffu, pk3, o);
+        }
+        if (lane < 4) so.dr[p][(size_t)r * 4 + lane] = (lane == 0 ? pk0 : lane == 1 ? pk1 : lane == 2 ? pk2 : pk3) * inv;
+      }
+    }
   }
 }
 
@@ -871,25 +1061,45 @@ fekf_status model_forward(Ctx& c, int nb, bool tangent, cudaStream_t s) {
   // descriptor
   PairPtrs pp = make_pp(c);
   FitPtrs fp = make_fp(c, nb);
-  const size_t smem = 8 * c.M * sizeof(double);
+  const size_t smem = (8 * (size_t)c.M + 8 * (size_t)c.Nm) * sizeof(double) + 3 * sizeof(int) * c.Nm;
   const size_t Xoff = (size_t)c.B * c.Na * 4 * c.M;
   desc_fwd_kernel<<<nb * c.Na, 128, smem, s>>>(g, pp, fp, c.em.as<double>(), c.rdot.as<double>(), tangent ? 1 : 0,
                                                c.X.as<double>(), c.X.as<double>() + Xoff);
   FEKF_LAUNCH_CHECK();
   count_launch();
-  // fitting nets (stacked rows: the tangent half starts at row F)
-  for (int t = 0; t < c.nt; ++t) {
-    FitNet& Fn = c.fits[t];
-    const long long F = fit_rows(c, t, nb);
-    if (F == 0) continue;
-    for (size_t l = 0; l < Fn.L.size(); ++l) {
+  // fitting nets (stacked rows: the tangent half starts at row F); one grouped GEMM per layer over types
+  const size_t nfl = c.fits[0].L.size();
+  for (size_t l = 0; l < nfl; ++l) {
+    GemmProb<EpiFwd> pr[GG_MAX];
+    int n = 0;
+    for (int t = 0; t < c.nt; ++t) {
+      FitNet& Fn = c.fits[t];
+      const long long F = fit_rows(c, t, nb);
+      if (F == 0) continue;
       const Layer& L = Fn.L[l];
       const double* Ain = l == 0 ? Fn.D.as<double>() : Fn.H[l - 1].as<double>();
       const double* Hprev = l == 0 ? nullptr : Fn.H[l - 1].as<double>();
       const size_t oi = tangent ? (size_t)F * L.din : 0, oo = tangent ? (size_t)F * L.dout : 0;
-      FEKF_TRY(layer_fwd(L, w, F, nullptr, Ain + oi, Hprev ? Hprev + oi : nullptr, Fn.Y[l].as<double>() + oo,
-                         Fn.H[l].as<double>() + oo, tangent ? Fn.Y[l].as<double>() : nullptr, nullptr, s));
+      EpiFwd e;
+      e.Y = Fn.Y[l].as<double>() + oo;
+      e.H = Fn.H[l].as<double>() + oo;
+      e.ld = L.dout;
+      e.bias = w + L.b;
+      e.dt = L.dt >= 0 ? w + L.dt : nullptr;
+      e.Hp = Hprev ? Hprev + oi : nullptr;
+      e.ldp = L.din;
+      e.skip = Hprev ? L.skip : 0;
+      e.dprev = L.din;
+      e.Yprim = tangent ? Fn.Y[l].as<double>() : nullptr;
+      e.rowmap = nullptr;
+      pr[n++] = GemmProb<EpiFwd>{(int)F, L.dout, L.din, nullptr, nullptr, Ain + oi, L.din, w + L.W, L.dout, -1, 0, 0, 1, e};
     }
+    FEKF_TRY(gemm_group<false, false>(pr, n, s));
+  }
+  for (int t = 0; t < c.nt; ++t) {
+    FitNet& Fn = c.fits[t];
+    const long long F = fit_rows(c, t, nb);
+    if (F == 0) continue;
     const int h = Fn.L.back().dout;
     const double* Hl = Fn.H.back().as<double>();
     double* eo = Fn.eout.as<double>();
@@ -964,7 +1174,8 @@ fekf_status model_backward(Ctx& c, int nb, Mode mode, double* gout, cudaStream_t
   Geo g = make_geo(c, nb);
   PairPtrs pp = make_pp(c);
   FitPtrs fp = make_fp(c, nb);
-  // ---- fitting nets (stacked rows) ----
+  // ---- fitting nets (stacked rows); weight and data gradients grouped over types per layer ----
+  const size_t nfl = c.fits[0].L.size();
   for (int t = 0; t < c.nt; ++t) {
     FitNet& Fn = c.fits[t];
     const long long F = fit_rows(c, t, nb);
@@ -981,7 +1192,16 @@ fekf_status model_backward(Ctx& c, int nb, Mode mode, double* gout, cudaStream_t
                      Seg{dual ? Hl + (size_t)F * h : nullptr, dual ? eb + F : nullptr, dual ? F : 0, nullptr, 0},
                      gout + Fn.Wout, s));
     }
-    for (int l = (int)Fn.L.size() - 1; l >= 0; --l) {
+  }
+  for (int l = (int)nfl - 1; l >= 0; --l) {
+    WgradJob jobs[FEKF_MAX_TYPES];
+    GemmProb<EpiDgrad> dg[GG_MAX];
+    int nj = 0, nd = 0;
+    for (int t = 0; t < c.nt; ++t) {
+      FitNet& Fn = c.fits[t];
+      const long long F = fit_rows(c, t, nb);
+      if (F == 0) continue;
+      const long long nF = dual ? 2 * F : F;
       const Layer& L = Fn.L[l];
       const double* dt = L.dt >= 0 ? w + L.dt : nullptr;
       act_bwd_kernel<<<cdiv(F * L.dout, 256), 256, 0, s>>>(F, L.dout, Fn.Y[l].as<double>(), Fn.Hb[l].as<double>(), dt,
@@ -991,26 +1211,53 @@ fekf_status model_backward(Ctx& c, int nb, Mode mode, double* gout, cudaStream_t
       const double* Hprev = l == 0 ? Fn.D.as<double>() : Fn.H[l - 1].as<double>();
       if (want_w) {
         // stacked rows; the ones column covers the primal half only (bias not in the tangent)
-        FEKF_TRY(wgrad(c, L.din, L.dout, Seg{Hprev, Fn.Zb[l].as<double>(), F, nullptr, 1},
-                       Seg{dual ? Hprev + (size_t)F * L.din : nullptr, dual ? Fn.Zb[l].as<double>() + (size_t)F * L.dout : nullptr,
-                           dual ? F : 0, nullptr, 0},
-                       gout + L.W, s));
+        jobs[nj++] = WgradJob{L.din, L.dout, Seg{Hprev, Fn.Zb[l].as<double>(), F, nullptr, 1},
+                              Seg{dual ? Hprev + (size_t)F * L.din : nullptr,
+                                  dual ? Fn.Zb[l].as<double>() + (size_t)F * L.dout : nullptr, dual ? F : 0, nullptr, 0},
+                              gout + L.W};
         if (L.dt >= 0) FEKF_TRY(colsum_prod(c, Fn.Y[l].as<double>(), Fn.Hb[l].as<double>(), nF, L.dout, gout + L.dt, s));
       }
       double* out = l == 0 ? Fn.Db.as<double>() : Fn.Hb[l - 1].as<double>();
       EpiDgrad e{out, L.din, Fn.Hb[l].as<double>(), L.dout, l == 0 ? 0 : L.skip, L.din};
-      FEKF_TRY(gemm<false, true>(nF, L.din, L.dout, Fn.Zb[l].as<double>(), L.dout, w + L.W, L.dout, e, s));
+      dg[nd++] = GemmProb<EpiDgrad>{(int)nF, L.din, L.dout, nullptr, nullptr, Fn.Zb[l].as<double>(), L.dout, w + L.W,
+                                    L.dout, -1, 0, 0, 1, e};
     }
+    if (nj) FEKF_TRY(wgrad_group(c, jobs, nj, s));
+    FEKF_TRY(gemm_group<false, true>(dg, nd, s));
   }
   // ---- descriptor (Eq. 4) ----
   const size_t Xoff = (size_t)c.B * c.Na * 4 * c.M;
-  const size_t smem = (8 * c.M + 2 * c.M * c.M2) * sizeof(double);
-  desc_bwd_kernel<<<nb * c.Na, 128, smem, s>>>(g, fp, c.X.as<double>(), c.X.as<double>() + Xoff, dual ? 1 : 0,
-                                               c.Xb.as<double>(), c.Xb.as<double>() + Xoff);
+  if (emb_fused_ok(c)) {
+    SeedOut so{};
+    for (size_t p = 0; p < c.pairs.size(); ++p) {
+      PairNet& P = c.pairs[p];
+      so.gbar[p] = P.Hb.back().as<double>();
+      so.hbt[p] = P.Hbt.back().as<double>();
+      so.dr[p] = P.Zb[0].as<double>();
+    }
+    const size_t smem = (16 * (size_t)c.M + 2 * (size_t)c.M * (c.M2 + 1) + 8 * (size_t)c.Nm) * sizeof(double);
+    static size_t attr = 0;
+    if (smem > attr) {
+      FEKF_CHECK_CUDA(cudaFuncSetAttribute(desc_bwd_seed_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+      attr = smem;
+    }
+    desc_bwd_seed_kernel<<<nb * c.Na, 256, smem, s>>>(g, fp, pp, so, c.X.as<double>(), c.X.as<double>() + Xoff,
+                                                      c.em.as<double>(), c.rdot.as<double>(), dual ? 1 : 0,
+                                                      mode == MODE_FORCE ? 1 : 0, c.Xb.as<double>(),
+                                                      c.Xb.as<double>() + Xoff);
+  } else {
+    const size_t smem = (8 * c.M + 2 * c.M * (c.M2 + 1)) * sizeof(double);
+    desc_bwd_kernel<<<nb * c.Na, 128, smem, s>>>(g, fp, c.X.as<double>(), c.X.as<double>() + Xoff, dual ? 1 : 0,
+                                                 c.Xb.as<double>(), c.Xb.as<double>() + Xoff);
+  }
   FEKF_LAUNCH_CHECK();
   count_launch();
   // ---- embedding nets (compacted rows; tangent rows separately) ----
-  if (emb_bwd_fused_ok(c)) {
+  if (emb_fused_ok(c)) {
+    if (mode == MODE_FORCE) {  // forces / per-atom virials accumulate inside the fused backward
+      FEKF_CHECK_CUDA(cudaMemsetAsync(c.force.p, 0, sizeof(double) * nb * c.Na * 3, s));
+      FEKF_CHECK_CUDA(cudaMemsetAsync(c.vatom.p, 0, sizeof(double) * nb * c.Na * 9, s));
+    }
     for (size_t p = 0; p < c.pairs.size(); ++p) {
       const long long Rmax = pair_rows(c, (int)p, nb);
       if (Rmax == 0) continue;
@@ -1070,13 +1317,16 @@ fekf_status model_backward(Ctx& c, int nb, Mode mode, double* gout, cudaStream_t
   }
   }
   if (mode == MODE_FORCE) {
-    FEKF_CHECK_CUDA(cudaMemsetAsync(c.force.p, 0, sizeof(double) * nb * c.Na * 3, s));
-    prod_force_kernel<<<nb * c.Na, 128, 0, s>>>(g, pp, c.Xb.as<double>(), c.jac.as<double>(), c.rij.as<double>(),
-                                                c.nl_j.as<int>(), c.force.as<double>(), c.vatom.as<double>());
-    FEKF_LAUNCH_CHECK();
+    if (!emb_fused_ok(c)) {
+      FEKF_CHECK_CUDA(cudaMemsetAsync(c.force.p, 0, sizeof(double) * nb * c.Na * 3, s));
+      prod_force_kernel<<<nb * c.Na, 128, 0, s>>>(g, pp, c.Xb.as<double>(), c.jac.as<double>(), c.rij.as<double>(),
+                                                  c.nl_j.as<int>(), c.force.as<double>(), c.vatom.as<double>());
+      FEKF_LAUNCH_CHECK();
+      count_launch();
+    }
     virial_reduce_kernel<<<nb, 32, 0, s>>>(c.vatom.as<double>(), c.Na, c.virial.as<double>());
     FEKF_LAUNCH_CHECK();
-    count_launch(2);
+    count_launch();
   }
   return FEKF_OK;
 }
