@@ -61,7 +61,7 @@ class OptConfig:
     grad_reduce: int = 0     # 0: sum over the global batch (Alg. 1 line 7); 1: mean (Eq. 1)
     force_groups: int = 4
     atoms_per_group: int = 6
-    p_defer: int = 5         # CUDA path only: deferred rank-1 corrections of P (same P up to rounding)
+    p_defer: int = 15        # CUDA path only: deferred rank-1 corrections of P (same P up to rounding)
 
 
 @dataclass

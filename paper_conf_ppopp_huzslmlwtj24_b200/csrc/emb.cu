@@ -24,8 +24,11 @@ namespace fekf {
 // B[n][k] : B[k][n] (LDB); K a multiple of 4, padded operands zero.  Warp tiles of 2x2 DMMA tiles when
 // there are enough of them for every warp, else 1x2.  epi(r, c, C[r][c], C[r][c+1]) (c even) straight
 // from the accumulators.
-template <bool BT, int MT, int NT, int K, int LDA, int LDB, int NW, class Epi>
-__device__ __forceinline__ void cta_mma(const double* A, const double* B, Epi epi) {
+struct XfId {
+  __device__ double operator()(int, int, double v) const { return v; }
+};
+template <bool BT, int MT, int NT, int K, int LDA, int LDB, int NW, class Epi, class Xf = XfId>
+__device__ __forceinline__ void cta_mma(const double* A, const double* B, Epi epi, Xf xf = Xf()) {
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, fr = lane >> 2, fk = lane & 3;
   constexpr int NJ = (NT + 1) / 2;
   constexpr bool big = ((MT + 1) / 2) * NJ >= NW;
@@ -52,6 +55,15 @@ __device__ __forceinline__ void cta_mma(const double* A, const double* B, Epi ep
       if (mv) dmma884(c[1][0][0], c[1][0][1], a1, b0);
       if (mv && nv) dmma884(c[1][1][0], c[1][1][1], a1, b1);
     }
+    // pure per-value transform of the whole warp tile first (independent chains interleave), then stores
+#pragma unroll
+    for (int i = 0; i < 2; ++i)
+#pragma unroll
+      for (int j = 0; j < 2; ++j)
+#pragma unroll
+        for (int h = 0; h < 2; ++h)
+          if ((i == 0 || mv) && (j == 0 || nv))
+            c[i][j][h] = xf((mi + i) * 8 + fr, (nj + j) * 8 + 2 * fk + h, c[i][j][h]);
 #pragma unroll
     for (int i = 0; i < 2; ++i)
 #pragma unroll
@@ -138,8 +150,8 @@ template <class W>
 __global__ void __launch_bounds__(EMB_FWD_WARPS * 32) emb_fwd_kernel(const double* __restrict__ wp, EmbFwdIO io) {
   extern __shared__ __align__(16) double sm[];
   constexpr int T = W::T, NW = EMB_FWD_WARPS, NL = W::NL, RPW = T / NW;
-  __shared__ double s_in[T];
-  __shared__ int s_prow[T];
+  __shared__ double s_in[2][T];
+  __shared__ int s_prow[2][T];
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   const bool tan = io.tidx != nullptr;
   const int R = min(io.Rmax, *io.Rdev);
@@ -160,23 +172,37 @@ __global__ void __launch_bounds__(EMB_FWD_WARPS * 32) emb_fwd_kernel(const doubl
     for (int c = tid; c < pad8(W::d(l)); c += blockDim.x)
       sm[W::fB(l) + c] = c < W::d(l) ? wp[W::goff(l) + W::din(l) * W::d(l) + c] : 0.0;
 
-  const int ntiles = (R + T - 1) / T;
-  for (int tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
-    const int r0 = tile * T;
-    __syncthreads();  // weights staged / previous tile's buffers consumed
+  // The next tile's input (row -> primal row -> slot -> s) is fetched by warp 0 in three dependent
+  // steps spread over the current tile's layers, so its latency hides behind the compute.
+  int nx_pr = -1, nx_slot = -1;
+  double nx_v = 0.0;
+  auto fetch_a = [&](int rn) {
+    nx_pr = -1;
+    if (tid < T && rn + tid < R) nx_pr = tan ? io.tidx[rn + tid] : rn + tid;
+  };
+  auto fetch_b = [&]() { nx_slot = (tid < T && nx_pr >= 0) ? io.row_idx[nx_pr] : -1; };
+  auto fetch_c = [&]() { nx_v = nx_slot >= 0 ? io.src[(size_t)nx_slot * 4] : 0.0; };
+  auto fetch_d = [&](int rn, int b) {
     if (tid < T) {
-      const int row = r0 + tid;
-      double v = 0.0;
-      int pr = -1;
-      if (row < R) {
-        pr = tan ? io.tidx[row] : row;
-        v = io.src[(size_t)io.row_idx[pr] * 4];
-        io.hin[row] = v;
-      }
-      s_in[tid] = v;
-      s_prow[tid] = pr;
+      s_in[b][tid] = nx_v;
+      s_prow[b][tid] = nx_pr;
+      if (rn + tid < R) io.hin[rn + tid] = nx_v;
     }
-    __syncthreads();
+  };
+  const int ntiles = (R + T - 1) / T;
+  int buf = 0;
+  if ((int)blockIdx.x < ntiles) {
+    fetch_a(blockIdx.x * T);
+    fetch_b();
+    fetch_c();
+    fetch_d(blockIdx.x * T, 0);
+  }
+  for (int tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
+    const int r0 = tile * T, rn = r0 + gridDim.x * T;
+    __syncthreads();  // weights staged / this tile's inputs in s_in[buf] / previous tile's buffers consumed
+    fetch_a(rn);
+    const double* s_inb = s_in[buf];
+    const int* s_prowb = s_prow[buf];
     // ---- layer 0 (input width 1): elementwise
     {
       constexpr int d = W::d(0), w8 = pad8(d), CJ = (w8 + 31) / 32, ld = W::fALD(0);
@@ -189,7 +215,7 @@ __global__ void __launch_bounds__(EMB_FWD_WARPS * 32) emb_fwd_kernel(const doubl
 #pragma unroll
         for (int j = 0; j < CJ; ++j) {
           const int r = warp + NW * i, c = lane + 32 * j;
-          const int pr = s_prow[r];
+          const int pr = s_prowb[r];
           yp[i][j] = (tan && c < d && pr >= 0) ? io.Yp[0][(size_t)pr * d + c] : 0.0;
         }
 #pragma unroll
@@ -201,7 +227,7 @@ __global__ void __launch_bounds__(EMB_FWD_WARPS * 32) emb_fwd_kernel(const doubl
             const int row = r0 + r;
             double h = 0.0;
             if (c < d) {
-              const double z = s_in[r] * w0[c];
+              const double z = s_inb[r] * w0[c];
               h = tan ? (1.0 - yp[i][j] * yp[i][j]) * z : tanh_fp64(z + b0[c]);
               if (row < R) {
                 const size_t o = (size_t)row * d + c;
@@ -214,10 +240,14 @@ __global__ void __launch_bounds__(EMB_FWD_WARPS * 32) emb_fwd_kernel(const doubl
         }
     }
     __syncthreads();
+    fetch_b();
     // ---- layers 1..NL-1: DMMA with the bias / tanh / skip epilogue in the accumulators
-    if constexpr (NL >= 2) fwd_layer<W, 1>(sm, io, r0, R, tan, s_prow);
-    if constexpr (NL >= 3) fwd_layer<W, 2>(sm, io, r0, R, tan, s_prow);
-    if constexpr (NL >= 4) fwd_layer<W, 3>(sm, io, r0, R, tan, s_prow);
+    if constexpr (NL >= 2) fwd_layer<W, 1>(sm, io, r0, R, tan, s_prowb);
+    fetch_c();
+    if constexpr (NL >= 3) fwd_layer<W, 2>(sm, io, r0, R, tan, s_prowb);
+    if constexpr (NL >= 4) fwd_layer<W, 3>(sm, io, r0, R, tan, s_prowb);
+    fetch_d(rn, buf ^ 1);
+    buf ^= 1;
   }
 }
 
@@ -358,9 +388,12 @@ __device__ __forceinline__ void bwd_layer(double (&acc)[W::MAXB][2][2][2], doubl
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const double* hb = sm + W::bBuf(bx);
   double* zb = sm + W::bBuf(bz);
-  // ---- zbar_L
-  {
+  // ---- zbar_L (the top layer's comes with the seed); primal y_L from shared memory (y_0 = aug_1,
+  // middle layers: their copies), tangent rows' y_L of the primal row and dual terms gathered
+  if constexpr (L < W::NL - 1) {
     double y[RPW][CJ], yt[RPW][CJ], hbt[RPW][CJ];
+    const double* ys = L == 0 ? sm + W::bAug(1) : sm + W::bYc(L);
+    constexpr int ldy = L == 0 ? W::augld(1) : sld(d);
 #pragma unroll
     for (int i = 0; i < RPW; ++i)
 #pragma unroll
@@ -368,7 +401,7 @@ __device__ __forceinline__ void bwd_layer(double (&acc)[W::MAXB][2][2][2], doubl
         const int r = warp + NW * i, c = lane + 32 * j;
         y[i][j] = yt[i][j] = hbt[i][j] = 0.0;
         if (c < d && s_slot[r] >= 0) {
-          y[i][j] = io.Yp[L][(size_t)s_prow[r] * d + c];
+          y[i][j] = tan ? io.Yp[L][(size_t)s_prow[r] * d + c] : ys[r * ldy + c];
           const int tp = s_tpos[r];
           if (tp >= 0) {
             yt[i][j] = io.Yt[L][(size_t)tp * d + c];
@@ -388,8 +421,8 @@ __device__ __forceinline__ void bwd_layer(double (&acc)[W::MAXB][2][2][2], doubl
           zb[r * BLD + c] = v;
         }
       }
+    __syncthreads();
   }
-  __syncthreads();
   if (wantw) wgrad_layer<W, L>(acc, sm, bz);
   if constexpr (L > 0) {
     constexpr int din = W::din(L), n8 = pad8(din), skip = W::skip(L);
@@ -463,30 +496,98 @@ __device__ __forceinline__ void bwd_layer(double (&acc)[W::MAXB][2][2][2], doubl
   }
 }
 
-// seed of the reverse chain for the tile's rows (warp w owns rows w, w + NW): hbar_{L-1} = Gbar, written
-// per row by desc_bwd_seed_kernel (primal rows: Gbar; tangent rows: Gdotbar in hdotbar_{L-1}); forces: the
-// per-row R~ adjoint dR
-template <class W>
-__device__ __forceinline__ void seed_rows(double* sm, const EmbBwdIO& io, int r0, int R, bool tan, double* s_dr) {
-  constexpr int T = W::T, NW = EMB_BWD_WARPS, RPW = T / NW, BLD = W::BLD, NL = W::NL, M = W::M;
-  constexpr int w8 = pad8(M), CJ = (w8 + 31) / 32;
+// h_L of a stored row from the stored y (h_0 = y_0, h_l = skip(h_{l-1}) + y_l), all loads independent
+template <class W, int L>
+__device__ __forceinline__ double hval(const EmbBwdIO& io, int row, int c) {
+  double v = io.Y[L][(size_t)row * W::d(L) + c];
+  if constexpr (L > 0) {
+    if constexpr (W::skip(L) == 1) v += hval<W, L - 1>(io, row, c);
+    else if constexpr (W::skip(L) == 2) v += hval<W, L - 1>(io, row, c % W::d(L - 1));
+  }
+  return v;
+}
+
+// aug_L = [h_{L-1} | one] for L = 1..NL-1 and the middle layers' y copies, one load phase per tile
+template <class W, int L>
+__device__ __forceinline__ void build_aug(double* sm, const EmbBwdIO& io, int r0, int R, double one) {
+  constexpr int T = W::T, NW = EMB_BWD_WARPS, RPW = T / NW;
+  constexpr int din = W::din(L), w8 = pad8(din + 1), CJ = (w8 + 31) / 32, ld = W::augld(L);
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const double* src = tan ? io.Hbt[NL - 1] : io.Gbar;
-  double* Hb = sm + W::bBuf(0);
   double v[RPW][CJ];
 #pragma unroll
   for (int i = 0; i < RPW; ++i)
 #pragma unroll
     for (int j = 0; j < CJ; ++j) {
       const int r = warp + NW * i, c = lane + 32 * j;
-      v[i][j] = (c < M && r0 + r < R) ? src[(size_t)(r0 + r) * M + c] : 0.0;
+      v[i][j] = (r0 + r < R && c < din) ? hval<W, L - 1>(io, r0 + r, c) : 0.0;
     }
 #pragma unroll
   for (int i = 0; i < RPW; ++i)
 #pragma unroll
     for (int j = 0; j < CJ; ++j) {
       const int r = warp + NW * i, c = lane + 32 * j;
-      if (c < w8) Hb[r * BLD + c] = v[i][j];
+      if (c < w8) sm[W::bAug(L) + r * ld + c] = (c == din && r0 + r < R) ? one : v[i][j];
+    }
+  if constexpr (L >= 1 && L <= W::NL - 2) {  // y_L copy (primal rows' zbar_L reads it from here)
+    constexpr int d = W::d(L), d8 = pad8(d), CJY = (d8 + 31) / 32, ldy = sld(d);
+    double y[RPW][CJY];
+#pragma unroll
+    for (int i = 0; i < RPW; ++i)
+#pragma unroll
+      for (int j = 0; j < CJY; ++j) {
+        const int r = warp + NW * i, c = lane + 32 * j;
+        y[i][j] = (r0 + r < R && c < d) ? io.Y[L][(size_t)(r0 + r) * d + c] : 0.0;
+      }
+#pragma unroll
+    for (int i = 0; i < RPW; ++i)
+#pragma unroll
+      for (int j = 0; j < CJY; ++j) {
+        const int r = warp + NW * i, c = lane + 32 * j;
+        if (c < d8) sm[W::bYc(L) + r * ldy + c] = y[i][j];
+      }
+  }
+  if constexpr (L + 1 < W::NL) build_aug<W, L + 1>(sm, io, r0, R, one);
+}
+
+// seed of the reverse chain for the tile's rows (warp w owns rows w, w + NW): hbar_{L-1} = Gbar, written
+// per row by desc_bwd_seed_kernel (primal rows: Gbar; tangent rows: Gdotbar in hdotbar_{L-1}); forces: the
+// per-row R~ adjoint dR
+template <class W>
+__device__ __forceinline__ void seed_rows(double* sm, const EmbBwdIO& io, int r0, int R, bool tan, double* s_dr,
+                                          const int* s_prow, const int* s_tpos) {
+  constexpr int T = W::T, NW = EMB_BWD_WARPS, RPW = T / NW, BLD = W::BLD, NL = W::NL, M = W::M;
+  constexpr int w8 = pad8(M), CJ = (w8 + 31) / 32;
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const double* src = tan ? io.Hbt[NL - 1] : io.Gbar;
+  double* Hb = sm + W::bBuf(0);
+  double* Zb = sm + W::bBuf(1);
+  double v[RPW][CJ], y[RPW][CJ], yt[RPW][CJ], hbt[RPW][CJ];
+#pragma unroll
+  for (int i = 0; i < RPW; ++i)
+#pragma unroll
+    for (int j = 0; j < CJ; ++j) {
+      const int r = warp + NW * i, c = lane + 32 * j;
+      v[i][j] = y[i][j] = yt[i][j] = hbt[i][j] = 0.0;
+      if (c < M && r0 + r < R) {
+        v[i][j] = src[(size_t)(r0 + r) * M + c];
+        y[i][j] = io.Yp[NL - 1][(size_t)s_prow[r] * M + c];
+        const int tp = s_tpos[r];
+        if (tp >= 0) {
+          yt[i][j] = io.Yt[NL - 1][(size_t)tp * M + c];
+          hbt[i][j] = io.Hbt[NL - 1][(size_t)tp * M + c];
+        }
+      }
+    }
+  // hbar_{L-1} = Gbar and, in the same pass, zbar_{L-1} = (1 - y^2) hbar [- 2 y ydot hdotbar]
+#pragma unroll
+  for (int i = 0; i < RPW; ++i)
+#pragma unroll
+    for (int j = 0; j < CJ; ++j) {
+      const int r = warp + NW * i, c = lane + 32 * j;
+      if (c < w8) {
+        Hb[r * BLD + c] = v[i][j];
+        Zb[r * BLD + c] = (1.0 - y[i][j] * y[i][j]) * v[i][j] - 2.0 * y[i][j] * yt[i][j] * hbt[i][j];
+      }
     }
   if (io.dR && threadIdx.x < T * 4) {
     const int r = threadIdx.x >> 2;
@@ -551,55 +652,17 @@ __global__ void __launch_bounds__(EMB_BWD_WARPS * 32, 1) emb_bwd_kernel(const do
         if (io.dR) l2_prefetch(io.dR + (size_t)rn * 4, T * 4 * sizeof(double));
       }
     }
-    // ---- [h_{l-1} | 1] for every layer (h recomputed from the stored y: h_0 = y_0, h_l = skip + y_l)
-    if (wantw) {
-      if (tid < T * 8) {
-        const int r = tid >> 3, cc = tid & 7;
-        const int row = r0 + r;
-        double v = 0.0;
-        if (row < R) v = cc == 0 ? io.hin[row] : (cc == 1 ? one : 0.0);
-        sm[W::bAug(0) + r * W::augld(0) + cc] = v;
-      }
-#pragma unroll
-      for (int l = 1; l < NL; ++l) {
-        const int din = W::din(l), w8 = pad8(din + 1), CJ = (w8 + 31) / 32, ld = W::augld(l);
-        constexpr int CJMAX = (pad8(W::maxw(-1) + 1) + 31) / 32;
-        const int ldp = W::augld(l - 1), skp = W::skip(l - 1), dpp = W::din(l - 1);
-        const double* prev = sm + W::bAug(l - 1);
-        double* Al = sm + W::bAug(l);
-        if (l >= 2) __syncthreads();  // aug_{l-1} complete
-        double y[RPW][CJMAX];
-#pragma unroll
-        for (int i = 0; i < RPW; ++i)
-#pragma unroll
-          for (int j = 0; j < CJMAX; ++j) {
-            const int r = warp + NW * i, c = lane + 32 * j;
-            y[i][j] = (j < CJ && r0 + r < R && c < din) ? io.Y[l - 1][(size_t)(r0 + r) * din + c] : 0.0;
-          }
-#pragma unroll
-        for (int i = 0; i < RPW; ++i)
-#pragma unroll
-          for (int j = 0; j < CJMAX; ++j) {
-            const int r = warp + NW * i, c = lane + 32 * j;
-            if (j < CJ && c < w8) {
-              double v = 0.0;
-              if (r0 + r < R) {
-                if (c < din) {
-                  v = y[i][j];
-                  if (skp == 1) v += prev[r * ldp + c];
-                  else if (skp == 2) v += prev[r * ldp + c % dpp];
-                } else if (c == din) {
-                  v = one;
-                }
-              }
-              Al[r * ld + c] = v;
-            }
-          }
-      }
+    // ---- [h_{l-1} | 1] for every layer (h recomputed from the stored y) and the middle layers' y
+    if (tid < T * 8) {
+      const int r = tid >> 3, cc = tid & 7;
+      const int row = r0 + r;
+      double v = 0.0;
+      if (row < R) v = cc == 0 ? io.hin[row] : (cc == 1 ? one : 0.0);
+      sm[W::bAug(0) + r * W::augld(0) + cc] = v;
     }
-    __syncthreads();  // rr, aug ready
-    // ---- seed: hbar_{L-1} = Gbar (and, for forces, the per-row R~ adjoint)
-    seed_rows<W>(sm, io, r0, R, tan, s_dr);
+    if constexpr (NL >= 2) build_aug<W, 1>(sm, io, r0, R, one);
+    // ---- seed: hbar_{L-1} = Gbar, zbar_{L-1} (and, for forces, the per-row R~ adjoint)
+    seed_rows<W>(sm, io, r0, R, tan, s_dr, s_prow, s_tpos);
     __syncthreads();
     if constexpr (NL >= 4) bwd_layer<W, 3>(acc, sm, io, r0, R, tan, wantw, s_slot, s_prow, s_tpos, s_atom, s_dr);
     if constexpr (NL >= 3) bwd_layer<W, 2>(acc, sm, io, r0, R, tan, wantw, s_slot, s_prow, s_tpos, s_atom, s_dr);

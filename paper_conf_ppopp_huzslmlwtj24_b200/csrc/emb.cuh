@@ -68,8 +68,13 @@ struct EmbW {
   }
   static constexpr int BLD = sld(maxw(-1));
   __host__ __device__ static constexpr int bBuf(int q) { return bAug(NL) + q * T * BLD; }
-  static constexpr int bR = bBuf(3);
-  static constexpr int B_SMEM = bR + T * 8;
+  // y_l of the middle layers 1..NL-2 (y_0 sits in aug_1, y_{NL-1} is consumed by the seed phase)
+  __host__ __device__ static constexpr int bYc(int l) {
+    int o = bBuf(3);
+    for (int k = 1; k < l; ++k) o += T * sld(d(k));
+    return o;
+  }
+  static constexpr int B_SMEM = bYc(NL > 2 ? NL - 1 : 1);
   // ---- weight-gradient blocks: 2x2 DMMA tiles of [din+1 x d] per layer, top layer first
   __host__ __device__ static constexpr int mblk(int l) { return (pad8(din(l) + 1) / 8 + 1) / 2; }
   __host__ __device__ static constexpr int nblk(int l) { return (pad8(d(l)) / 8 + 1) / 2; }

@@ -179,7 +179,7 @@ constexpr int MAX_STAGES = 8;
 constexpr int TILE_ELEMS = KT * KT;
 constexpr uint32_t TILE_BYTES = TILE_ELEMS * sizeof(double);
 constexpr int PASS_THREADS = 288;  // 8 consumer warps + 1 producer warp
-constexpr size_t PASS_SMEM = 227 * 1024;
+constexpr size_t PASS_SMEM = 227 * 1024 - 256;  // + 128 B of static shared memory (deferred coefficients)
 // [full[8] | empty[8] | meta[8]] (256 B), column-reduction buffers (8 KiB), then the stage ring; a stage
 // is one tile plus, for a read-write pass, the 2K vector segments (u_k rows I, u_k columns J) it needs.
 constexpr size_t PASS_HDR = 2 * MAX_STAGES * sizeof(uint64_t) + MAX_STAGES * sizeof(int4) + 2 * 8 * KT * sizeof(double);
@@ -243,9 +243,9 @@ kf_pass_kernel(double* __restrict__ P, const ItemD* __restrict__ items, int n_it
   }
 
   // ------------------------------ consumers ------------------------------
-  double beta[KMAX];
-#pragma unroll
-  for (int k = 0; k < KMAX; ++k) beta[k] = k < K ? st->beta[k] : 0.0;
+  __shared__ double s_beta[KMAX];
+  if (tid < KMAX) s_beta[tid] = tid < K ? st->beta[tid] : 0.0;
+  asm volatile("bar.sync 1, 256;" ::: "memory");  // consumer warps only
   const double sig = st->sigma;
   const int c0 = 2 * lane;
   double gI[8], racc[8];
@@ -273,32 +273,36 @@ kf_pass_kernel(double* __restrict__ P, const ItemD* __restrict__ items, int n_it
     const double* vI = t + TILE_ELEMS;
     const double* vJ = t + TILE_ELEMS + K * KT;
     double ca0 = 0.0, ca1 = 0.0;
-    // this lane's two columns of every deferred u_k (J segment): loaded once per tile, not per row
-    double2 uj[KMAX];
+    double2 v[8];
 #pragma unroll
-    for (int k = 0; k < KMAX; ++k)
-      uj[k] = k < K ? *reinterpret_cast<const double2*>(vJ + k * KT + c0) : make_double2(0.0, 0.0);
+    for (int q = 0; q < 8; ++q) v[q] = *reinterpret_cast<const double2*>(t + (warp + 8 * q) * KT + c0);
+    if (rw) {
+      // sum_k beta_k u_k[r] u_k[c] for this lane's rows r and columns c, k outermost (u_k[c] loaded once)
+      double2 cc[8];
+#pragma unroll
+      for (int q = 0; q < 8; ++q) cc[q] = make_double2(0.0, 0.0);
+      for (int k = 0; k < K; ++k) {
+        const double2 uj = *reinterpret_cast<const double2*>(vJ + k * KT + c0);
+        const double bk = s_beta[k];
+#pragma unroll
+        for (int q = 0; q < 8; ++q) {
+          const double bu = bk * vI[k * KT + warp + 8 * q];
+          cc[q].x = fma(bu, uj.x, cc[q].x);
+          cc[q].y = fma(bu, uj.y, cc[q].y);
+        }
+      }
+#pragma unroll
+      for (int q = 0; q < 8; ++q) {
+        v[q].x = sig * (v[q].x - cc[q].x);
+        v[q].y = sig * (v[q].y - cc[q].y);
+        *reinterpret_cast<double2*>(t + (warp + 8 * q) * KT + c0) = v[q];
+      }
+    }
 #pragma unroll
     for (int q = 0; q < 8; ++q) {
-      const int r = warp + 8 * q;
-      double2 v = *reinterpret_cast<double2*>(t + r * KT + c0);
-      if (rw) {
-        double cx = 0.0, cy = 0.0;
-#pragma unroll
-        for (int k = 0; k < KMAX; ++k) {
-          if (k < K) {
-            const double bu = beta[k] * vI[k * KT + r];
-            cx = fma(bu, uj[k].x, cx);
-            cy = fma(bu, uj[k].y, cy);
-          }
-        }
-        v.x = sig * (v.x - cx);
-        v.y = sig * (v.y - cy);
-        *reinterpret_cast<double2*>(t + r * KT + c0) = v;
-      }
-      racc[q] = fma(v.x, gJ.x, fma(v.y, gJ.y, racc[q]));
-      ca0 = fma(v.x, gI[q], ca0);
-      ca1 = fma(v.y, gI[q], ca1);
+      racc[q] = fma(v[q].x, gJ.x, fma(v[q].y, gJ.y, racc[q]));
+      ca0 = fma(v[q].x, gI[q], ca0);
+      ca1 = fma(v[q].y, gI[q], ca1);
     }
     double* cr = colred + (tcount & 1) * (8 * KT);
     if (!diag) {

@@ -8,7 +8,7 @@ namespace fekf {
 
 constexpr int KT = FEKF_TILE;    // tile edge (64 fp64 = 32 KiB per tile)
 constexpr int SEG_TILES = 32;    // max tiles per work item (tile-row segment)
-constexpr int KMAX = 8;          // max deferred rank-1 corrections held before P is rewritten
+constexpr int KMAX = 16;         // max deferred rank-1 corrections held before P is rewritten
 
 // One P-pass work item: tiles (I, J0..J0+nJ-1) of block `blk`, stored contiguously at tile_off.
 struct ItemD {

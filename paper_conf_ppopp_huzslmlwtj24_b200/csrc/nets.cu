@@ -267,46 +267,81 @@ static const int* tcount(Ctx& c, int p) { return c.rowcnt.as<int>() + c.pairs.si
 // ---------------------------------------------------------------------------------------------
 // compaction (one CTA per pair; fixed-order scans -> deterministic row order)
 // ---------------------------------------------------------------------------------------------
-__device__ __forceinline__ int section_count(const int* __restrict__ nl_j, size_t base, int sel) {
-  int c = 0;
-  while (c < sel && nl_j[base + c] >= 0) ++c;
-  return c;
-}
-
+// One CTA (32 warps) per pair: per-atom valid-slot counts by warp ballots (the sorted section is a
+// valid prefix), an exclusive scan in fixed order, then the compacted row -> slot map.
 __global__ void __launch_bounds__(1024)
 rows_kernel(Geo g, int ti, int tj, const int* __restrict__ nl_j, int* __restrict__ row_start,
             int* __restrict__ row_idx, int* __restrict__ cnt) {
-  __shared__ int part[1025];
+  __shared__ int wsum[32];
   const int E = g.nb * g.ncnt[ti];
   const int sel = g.sel[tj];
-  const int per = (E + blockDim.x - 1) / blockDim.x;
-  const int e0 = min(E, (int)threadIdx.x * per), e1 = min(E, e0 + per);
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   auto base_of = [&](int e) {
     const int b = e / g.ncnt[ti], k = e % g.ncnt[ti];
     const int i = g.atoms[g.atoms_off[ti] + k];
     return ((size_t)b * g.Na + i) * g.Nm + g.sec[tj];
   };
+  // counts -> row_start[e] (temporarily)
+  for (int e0 = warp; e0 < E; e0 += 32 * 4) {
+    int c4[4];
+#pragma unroll
+    for (int u = 0; u < 4; ++u) {
+      const int e = e0 + 32 * u;
+      int c = 0;
+      if (e < E) {
+        const size_t base = base_of(e);
+        for (int s0 = 0; s0 < sel; s0 += 32) {
+          const bool v = s0 + lane < sel && nl_j[base + s0 + lane] >= 0;
+          c += __popc(__ballot_sync(0xffffffffu, v));
+        }
+      }
+      c4[u] = c;
+    }
+    if (lane == 0)
+#pragma unroll
+      for (int u = 0; u < 4; ++u)
+        if (e0 + 32 * u < E) row_start[e0 + 32 * u] = c4[u];
+  }
+  __syncthreads();
+  // exclusive scan: contiguous chunk per thread, then a block scan of the chunk sums
+  const int per = (E + 1023) / 1024;
+  const int a0 = min(E, (int)threadIdx.x * per), a1 = min(E, a0 + per);
   int local = 0;
-  for (int e = e0; e < e1; ++e) local += section_count(nl_j, base_of(e), sel);
-  part[threadIdx.x] = local;
+  for (int e = a0; e < a1; ++e) local += row_start[e];
+  int x = local;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const int y = __shfl_up_sync(0xffffffffu, x, o);
+    if (lane >= o) x += y;
+  }
+  if (lane == 31) wsum[warp] = x;
   __syncthreads();
-  if (threadIdx.x == 0) {
-    int run = 0;
-    for (int t = 0; t < (int)blockDim.x; ++t) { const int v = part[t]; part[t] = run; run += v; }
-    part[blockDim.x] = run;
+  if (warp == 0) {
+    int w = wsum[lane];
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const int y = __shfl_up_sync(0xffffffffu, w, o);
+      if (lane >= o) w += y;
+    }
+    wsum[lane] = w;
   }
   __syncthreads();
-  int r = part[threadIdx.x];
-  for (int e = e0; e < e1; ++e) {
+  int run = x - local + (warp > 0 ? wsum[warp - 1] : 0);
+  for (int e = a0; e < a1; ++e) {
+    const int c = row_start[e];
+    row_start[e] = run;
+    run += c;
+  }
+  if (threadIdx.x == 1023) {
+    row_start[E] = wsum[31];
+    *cnt = wsum[31];
+  }
+  __syncthreads();
+  // row -> slot map
+  for (int e = warp; e < E; e += 32) {
+    const int r0 = row_start[e], n = row_start[e + 1] - r0;
     const size_t base = base_of(e);
-    const int c = section_count(nl_j, base, sel);
-    row_start[e] = r;
-    for (int s = 0; s < c; ++s) row_idx[r + s] = (int)(base + s);
-    r += c;
-  }
-  if (threadIdx.x == 0) {
-    row_start[E] = part[blockDim.x];
-    *cnt = part[blockDim.x];
+    for (int s0 = lane; s0 < n; s0 += 32) row_idx[r0 + s0] = (int)(base + s0);
   }
 }
 
@@ -619,21 +654,31 @@ desc_bwd_seed_kernel(Geo g, FitPtrs fp, PairPtrs pp, SeedOut so, const double* _
       const int t = dual ? tpos[r] : -1;
       double pk0 = 0.0, pk1 = 0.0, pk2 = 0.0, pk3 = 0.0;
       const double* Gr = force ? pp.G[p] + (size_t)r * M : nullptr;
-      for (int m = lane; m < M; m += 32) {
-        double v = q[0] * xbs[m] + q[1] * xbs[M + m] + q[2] * xbs[2 * M + m] + q[3] * xbs[3 * M + m];
-        if (t >= 0) {
-          const double* qd = rds + (g.sec[tj] + s) * 4;
-          v += qd[0] * xdbs[m] + qd[1] * xdbs[M + m] + qd[2] * xdbs[2 * M + m] + qd[3] * xdbs[3 * M + m];
-          so.hbt[p][(size_t)t * M + m] =
-              (q[0] * xdbs[m] + q[1] * xdbs[M + m] + q[2] * xdbs[2 * M + m] + q[3] * xdbs[3 * M + m]) * inv;
+      for (int m0 = 0; m0 < M; m0 += 128) {
+        double gv[4];
+#pragma unroll
+        for (int u = 0; u < 4; ++u) {  // this row's G loads all in flight before their use
+          const int m = m0 + lane + 32 * u;
+          gv[u] = (force && m < M) ? Gr[m] : 0.0;
         }
-        so.gbar[p][(size_t)r * M + m] = v * inv;
-        if (force) {
-          const double gv = Gr[m];
-          pk0 = fma(gv, xbs[m], pk0);
-          pk1 = fma(gv, xbs[M + m], pk1);
-          pk2 = fma(gv, xbs[2 * M + m], pk2);
-          pk3 = fma(gv, xbs[3 * M + m], pk3);
+#pragma unroll
+        for (int u = 0; u < 4; ++u) {
+          const int m = m0 + lane + 32 * u;
+          if (m >= M) continue;
+          double v = q[0] * xbs[m] + q[1] * xbs[M + m] + q[2] * xbs[2 * M + m] + q[3] * xbs[3 * M + m];
+          if (t >= 0) {
+            const double* qd = rds + (g.sec[tj] + s) * 4;
+            v += qd[0] * xdbs[m] + qd[1] * xdbs[M + m] + qd[2] * xdbs[2 * M + m] + qd[3] * xdbs[3 * M + m];
+            so.hbt[p][(size_t)t * M + m] =
+                (q[0] * xdbs[m] + q[1] * xdbs[M + m] + q[2] * xdbs[2 * M + m] + q[3] * xdbs[3 * M + m]) * inv;
+          }
+          so.gbar[p][(size_t)r * M + m] = v * inv;
+          if (force) {
+            pk0 = fma(gv[u], xbs[m], pk0);
+            pk1 = fma(gv[u], xbs[M + m], pk1);
+            pk2 = fma(gv[u], xbs[2 * M + m], pk2);
+            pk3 = fma(gv[u], xbs[3 * M + m], pk3);
+          }
         }
       }
       if (force) {
@@ -887,25 +932,32 @@ __global__ void energy_error_kernel(Geo g, FitPtrs fp, const double* __restrict_
 // force update errors on the selected atoms (Alg. 1 lines 3-6 applied to force components):
 // e = F_label - F_pred, flip when F_pred >= F_label; v[b][a] accumulates the signs (tangent direction);
 // seeds: Ebar = 0, Edotbar = -1/(N_a n_sel 3) because sum s F = -Edot.
-__global__ void force_error_kernel(Geo g, const double* __restrict__ force, const double* __restrict__ label,
-                                   const int* __restrict__ atom_idx, int n_sel, double seed, double* __restrict__ v,
-                                   FitPtrs fp, double* __restrict__ abs_sum) {
+__global__ void __launch_bounds__(1024) force_error_kernel(Geo g, const double* __restrict__ force,
+                                                           const double* __restrict__ label,
+                                                           const int* __restrict__ atom_idx, int n_sel, double seed,
+                                                           double* __restrict__ v, FitPtrs fp,
+                                                           double* __restrict__ abs_sum) {
+  __shared__ double red[1024];
   for (long long e = threadIdx.x; e < (long long)g.nb * g.Na * 3; e += blockDim.x) v[e] = 0.0;
   __syncthreads();
-  if (threadIdx.x == 0) {
-    double a = 0.0;
-    for (int b = 0; b < g.nb; ++b)
-      for (int q = 0; q < n_sel; ++q) {
-        const int at = atom_idx[q];
-        for (int al = 0; al < 3; ++al) {
-          const size_t o = ((size_t)b * g.Na + at) * 3 + al;
-          const double fpred = force[o], fl = label[o];
-          a += fabs(fl - fpred);
-          v[o] += (fpred >= fl ? -1.0 : 1.0);
-        }
-      }
-    *abs_sum = a;
+  // one thread per (image, selected atom, component); the signs are integers, so their atomic sums
+  // (duplicate atoms in the list) are exact and order-free; |e| is reduced in a fixed tree
+  double a = 0.0;
+  const int n = g.nb * n_sel * 3;
+  for (int e = threadIdx.x; e < n; e += blockDim.x) {
+    const int b = e / (n_sel * 3), q = (e / 3) % n_sel, al = e % 3;
+    const size_t o = ((size_t)b * g.Na + atom_idx[q]) * 3 + al;
+    const double fpred = force[o], fl = label[o];
+    a += fabs(fl - fpred);
+    atomicAdd(v + o, fpred >= fl ? -1.0 : 1.0);
   }
+  red[threadIdx.x] = a;
+  __syncthreads();
+  for (int w = blockDim.x / 2; w > 0; w >>= 1) {
+    if ((int)threadIdx.x < w) red[threadIdx.x] += red[threadIdx.x + w];
+    __syncthreads();
+  }
+  if (threadIdx.x == 0) *abs_sum = red[0];
   for (int t = 0; t < g.nt; ++t) {
     const long long F = (long long)g.nb * g.ncnt[t];
     for (long long r = threadIdx.x; r < 2 * F; r += blockDim.x) fp.ebar[t][r] = r < F ? 0.0 : seed;
@@ -1148,7 +1200,7 @@ fekf_status force_error(Ctx& c, int nb, const double* f_label, const int* atom_i
   FitPtrs fp = make_fp(c, nb);
   double seed = -1.0 / ((double)c.Na * n_sel * 3);
   if (c.o.grad_reduce == 1) seed /= c.Bg;
-  force_error_kernel<<<1, 256, 0, s>>>(g, c.force.as<double>(), f_label, atom_idx, n_sel, seed, c.vdir.as<double>(), fp,
+  force_error_kernel<<<1, 1024, 0, s>>>(g, c.force.as<double>(), f_label, atom_idx, n_sel, seed, c.vdir.as<double>(), fp,
                                        abs_sum);
   FEKF_LAUNCH_CHECK();
   count_launch();

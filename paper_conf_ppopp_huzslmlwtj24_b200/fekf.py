@@ -155,7 +155,7 @@ def opt_cfg(o=None) -> OptCfg:
     c.grad_reduce = int(_get(o, "grad_reduce", 0)) if o is not None else 0
     c.force_groups = int(_get(o, "force_groups", 4)) if o is not None else 4
     c.atoms_per_group = int(_get(o, "atoms_per_group", 6)) if o is not None else 6
-    c.p_defer = int(_get(o, "p_defer", 5)) if o is not None else 5
+    c.p_defer = int(_get(o, "p_defer", 15)) if o is not None else 15
     return c
 
 

@@ -122,7 +122,7 @@ def _rand_spd(rng, n):
 
 
 @pytest.mark.parametrize("blocks", [[5, 70, 130], [64], [1, 200, 127, 65]])
-@pytest.mark.parametrize("noise_mode,p_defer", [(0, 5), (1, 1), (0, 3), (1, 8)])
+@pytest.mark.parametrize("noise_mode,p_defer", [(0, 5), (1, 1), (0, 3), (1, 8), (0, 16)])
 def test_kalman_updates(blocks, noise_mode, p_defer):
     rng = np.random.default_rng(7)
     opt = dict(lambda0=0.98, nu=0.9987, block_size=1024, noise_mode=noise_mode, p_defer=p_defer)
@@ -133,7 +133,7 @@ def test_kalman_updates(blocks, noise_mode, p_defer):
     for b, P in enumerate(st.P):
         kf.set_block(b, cu(P))
     w = torch.zeros(N, dtype=torch.float64, device="cuda")
-    for it in range(10):
+    for it in range(max(10, p_defer + 4)):   # at least one read-write pass
         g = rng.standard_normal(N)
         abe = float(rng.uniform(0.01, 1.0))
         kf.update(cu(g), cu([abe]), 3.0, w)
@@ -161,7 +161,7 @@ def test_kalman_full_size_sampled_blocks():
     gen = torch.Generator(device="cuda").manual_seed(3)
     w = torch.zeros(N, dtype=torch.float64, device="cuda")
     abe = torch.full((1,), 0.05, dtype=torch.float64, device="cuda")
-    for _ in range(7):   # crosses one read-write pass (p_defer = 5)
+    for _ in range(wl.opt.p_defer + 2):   # crosses one read-write pass
         kf.update(torch.randn(N, dtype=torch.float64, device="cuda", generator=gen), abe, 4.0, w)
     sample = [0, 37, 109]
     before = {b: kf.get_block(b).cpu().numpy() for b in sample}
