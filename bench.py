@@ -39,6 +39,9 @@ def parse():
     ap.add_argument("--impl", default="fekf", choices=["fekf", "reference"])
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--precision", type=int, default=64, choices=[64, 32],
+                    help="storage precision of P (32 = the fp32 variant, reading Z22; nets stay fp64)")
+    ap.add_argument("--p-defer", type=int, default=None, help="override the deferred-correction depth")
     return ap.parse_args()
 
 
@@ -168,6 +171,10 @@ def run_fekf(args, rank, world, local):
     torch.cuda.set_device(local)
     wl = get_config(args.config)
     m, opt = wl.model, wl.opt
+    over = {"precision": args.precision}
+    if args.p_defer is not None:
+        over["p_defer"] = args.p_defer
+    opt = type(opt)(**{**opt.__dict__, **over})
     B = wl.batch
     Bg = B * world
     ds = make_dataset(args.config, 2 * B, seed=wl.seed + 1000 * rank)
@@ -269,7 +276,8 @@ def run_fekf(args, rank, world, local):
     total_tiles = sum(x * (x + 1) // 2 for x in nt)
     # algorithmic bytes of one stream over this rank's share of the symmetric blocks: 8 * n(n+1)/2 each;
     # a read-write pass (the one that rewrites P) moves it twice, a read-only pass once
-    stream = 4.0 * sum(n * (n + 1) for n in blocks) * info["tiles_local"] / total_tiles
+    esize = 8 if args.precision == 64 else 4
+    stream = esize / 2 * sum(n * (n + 1) for n in blocks) * info["tiles_local"] / total_tiles
     alg_total = stream * (2 * pass_rw + (pass_n - pass_rw))
     alg_bytes = alg_total / max(pass_n, 1)
     avg_pass_s = (pass_ms / max(pass_n, 1)) / 1000.0
@@ -277,12 +285,16 @@ def run_fekf(args, rank, world, local):
     achieved = alg_total / (pass_ms / 1000.0) / 1e9 if pass_ms > 0 else None
     traffic = None
     prof = os.path.join(ROOT, "profiles", "kf_pass_traffic.json")
-    if os.path.exists(prof):
+    if os.path.exists(prof) and pass_n > 0:
         try:
             with open(prof) as f:
                 pj = json.load(f)
-            if pj.get("workload") == args.config:
-                traffic = pj.get("dram_bytes_per_launch")
+            if pj.get("workload") == args.config and world == 1 and pj.get("precision", 64) == args.precision:
+                # DRAM bytes per launch from one ncu --set full capture, blended over the read-only and
+                # read-write launches of this run (a read-write pass moves twice the read-only bytes)
+                ro = pj["ro_dram_bytes_per_launch"] / pj["ro_alg_bytes_per_launch"]
+                rwr = pj["rw_traffic_over_alg"]
+                traffic = (stream * ro * (pass_n - pass_rw) + 2 * stream * rwr * pass_rw) / pass_n
         except Exception:
             pass
     roof = {"kernel": "kf_pass_kernel", "bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
@@ -292,11 +304,14 @@ def run_fekf(args, rank, world, local):
 
     out = {"metric": METRIC, "value": value, "unit": "images/s", "n_gpus": world, "steps": args.steps,
            "warmup": args.warmup, "ms_per_step": ms / args.steps, "higher_is_better": True, "scaling": "weak",
-           "vs_baseline": None, "dtype": "f64", "data": "synthetic (seeded perturbed water-64 lattices, LJ labels)",
+           "vs_baseline": None, "dtype": "f64" if args.precision == 64 else "f64 nets / f32 P",
+           "data": "synthetic (seeded perturbed water-64 lattices, LJ labels)",
            "config": {"workload": args.config, "images_per_gpu": B, "global_batch": Bg, "n_atoms": na,
                       "n_params": ctx.n_params, "p_blocks": len(blocks), "p_bytes_per_gpu": info["p_bytes_local"],
                       "parallelism": f"dp{world}" + (" + P sharded" if world > 1 else ""),
-                      "l2": "inputs larger than L2: P (39 GiB packed fp64) is streamed 5x per step"},
+                      "p_precision": args.precision, "p_defer": opt.p_defer,
+                      "l2": "inputs larger than L2: P (%.1f GiB packed) is streamed 5x per step"
+                            % (info["p_bytes_local"] / 2**30)},
            "roofline": roof, "e2e": e2e, "gpu_launches": int(launches), "clocks": clk,
            "last_metrics": {"abe_e": met[0], "abe_f": list(met[1:5]), "A_last": met[5], "lambda": met[6],
                             "flags": met[7]}}

@@ -290,11 +290,39 @@ fekf_status Ctx::init(const fekf_model_cfg& mm, const fekf_opt_cfg& oo, int nato
   FEKF_CHECK_CUDA(cudaDeviceGetAttribute(&maxsm, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev));
   const size_t need = (16 * (size_t)M + 2 * (size_t)M * (M2 + 1) + 8 * (size_t)Nm) * sizeof(double);
   if (need > (size_t)maxsm) { set_error("M*M2 too large for the descriptor kernels' shared memory"); return FEKF_EINVAL; }
+  // step-graph staging buffers and the capture stream
+  FEKF_TRY(dalloc(st_coord, sizeof(double) * B * Na * 3));
+  FEKF_TRY(dalloc(st_box, sizeof(double) * B * 9));
+  FEKF_TRY(dalloc(st_e, sizeof(double) * B));
+  FEKF_TRY(dalloc(st_f, sizeof(double) * B * Na * 3));
+  FEKF_TRY(dalloc(st_fidx, sizeof(int) * std::max(1, o.force_groups * o.atoms_per_group)));
+  FEKF_TRY(dalloc(st_met, sizeof(double) * 8));
+  FEKF_CHECK_CUDA(cudaStreamCreateWithFlags(&gstream, cudaStreamNonBlocking));
+  FEKF_CHECK_CUDA(cudaEventCreateWithFlags(&gev_in, cudaEventDisableTiming));
+  FEKF_CHECK_CUDA(cudaEventCreateWithFlags(&gev_out, cudaEventDisableTiming));
   FEKF_CHECK_CUDA(cudaDeviceSynchronize());
   return FEKF_OK;
 }
 
+void Ctx::drop_graphs() {
+  for (auto& kv : graphs) {
+    if (kv.second.exec) cudaGraphExecDestroy(kv.second.exec);
+    if (kf) {
+      kf->pend_graphs.erase(std::remove(kf->pend_graphs.begin(), kf->pend_graphs.end(), &kv.second.tm),
+                            kf->pend_graphs.end());
+    }
+    for (EvPair& e : kv.second.tm.ev) { cudaEventDestroy(e.a); cudaEventDestroy(e.b); }
+  }
+  graphs.clear();
+}
+
 Ctx::~Ctx() {
+  if (gstream) cudaStreamSynchronize(gstream);
+  drop_graphs();
+  if (gstream) cudaStreamDestroy(gstream);
+  if (gev_in) cudaEventDestroy(gev_in);
+  if (gev_out) cudaEventDestroy(gev_out);
+  for (DBuf* b : {&st_coord, &st_box, &st_e, &st_f, &st_fidx, &st_met}) dfree(*b);
   kfo.reset();
   kf = nullptr;
   for (DBuf* b : {&types_d, &tindex_d, &atoms_d, &atoms_off_d, &sel_d, &sec_d, &err_d, &w, &gbuf, &nl_j, &nl_s,
@@ -353,6 +381,82 @@ static fekf_status force_grad_pass(Ctx& c, int nb, const double* f_label, const 
   FEKF_TRY(model_forward(c, nb, true, s));
   FEKF_CHECK_CUDA(cudaMemsetAsync(g, 0, sizeof(double) * c.Np, s));
   FEKF_TRY(model_backward(c, nb, MODE_FORCE_JAC, g, s));
+  return FEKF_OK;
+}
+
+// One minibatch: geometry, 1 energy update, force_groups force updates, metrics.
+static fekf_status step_body(Ctx& c, const double* coord, const double* box, const double* e_label,
+                             const double* f_label, const int32_t* force_idx, double* metrics, cudaStream_t s) {
+  const int nb = c.B;
+  const double sqrt_bs = std::sqrt((double)c.Bg);
+  double* g = c.gbuf.as<double>();
+  double* esum = g + c.Np;
+  FEKF_CHECK_CUDA(cudaMemsetAsync(metrics, 0, sizeof(double) * 8, s));
+  FEKF_TRY(geometry(c, coord, box, nb, s));
+  // energy update (1 per minibatch)
+  FEKF_TRY(energy_grad_pass(c, nb, e_label, g, esum, s));
+  FEKF_TRY(comm_allreduce(c.comm, g, c.Np + 1, s));
+  abe_kernel<<<1, 1, 0, s>>>(esum, 1.0 / c.Bg, c.abe.as<double>(), metrics + 0);
+  FEKF_LAUNCH_CHECK();
+  count_launch();
+  FEKF_TRY(c.kf->update(g, c.abe.as<double>(), sqrt_bs, c.w.as<double>(), s));
+  // force updates
+  const int apg = c.o.atoms_per_group;
+  for (int k = 0; k < c.o.force_groups; ++k) {
+    FEKF_TRY(force_grad_pass(c, nb, f_label, force_idx + (size_t)k * apg, apg, g, esum, s));
+    FEKF_TRY(comm_allreduce(c.comm, g, c.Np + 1, s));
+    abe_kernel<<<1, 1, 0, s>>>(esum, 1.0 / ((double)c.Bg * apg * 3) / c.Na, c.abe.as<double>(),
+                               k < 4 ? metrics + 1 + k : nullptr);
+    FEKF_LAUNCH_CHECK();
+    count_launch();
+    FEKF_TRY(c.kf->update(g, c.abe.as<double>(), sqrt_bs, c.w.as<double>(), s));
+  }
+  metrics_kernel<<<1, 1, 0, s>>>(c.kf->state.as<KfState>(), c.err_d.as<int>(), c.overflow.as<int>(), nb, metrics);
+  FEKF_LAUNCH_CHECK();
+  count_launch();
+  return FEKF_OK;
+}
+
+// Capture the step for the current host state (pending-correction count) unless cached.
+static fekf_status step_graph(Ctx& c, StepGraph** out) {
+  Kf& k = *c.kf;
+  // every graph records a P-pass event pair (a negligible node) whether or not timing is on, so timing
+  // never forces a re-capture; two graphs per count alternate by step parity
+  const int key = k.npend * 2 + (int)(c.nsteps & 1);
+  StepGraph& G = c.graphs[key];
+  if (!G.exec) {
+    const int npend0 = k.npend;
+    const int64_t l0 = g_launches;
+    const long long rwp = k.rw_passes, rp = k.r_passes;
+    k.capturing = true;
+    k.rec = &G.tm.ev;
+    FEKF_CHECK_CUDA(cudaStreamBeginCapture(c.gstream, cudaStreamCaptureModeRelaxed));
+    fekf_status st = step_body(c, c.st_coord.as<double>(), c.st_box.as<double>(), c.st_e.as<double>(),
+                               c.st_f.as<double>(), c.st_fidx.as<int32_t>(), c.st_met.as<double>(), c.gstream);
+    cudaGraph_t graph = nullptr;
+    cudaError_t e = cudaStreamEndCapture(c.gstream, &graph);
+    k.capturing = false;
+    k.rec = nullptr;
+    G.npend_after = k.npend;
+    G.launches = g_launches - l0;
+    k.npend = npend0;
+    k.rw_passes = rwp;
+    k.r_passes = rp;
+    g_launches = l0;
+    if (st != FEKF_OK || e != cudaSuccess) {
+      if (graph) cudaGraphDestroy(graph);
+      c.graphs.erase(key);
+      if (st != FEKF_OK) return st;
+      FEKF_CHECK_CUDA(e);
+    }
+    e = cudaGraphInstantiate(&G.exec, graph, 0);
+    cudaGraphDestroy(graph);
+    if (e != cudaSuccess) {
+      c.graphs.erase(key);
+      FEKF_CHECK_CUDA(e);
+    }
+  }
+  *out = &G;
   return FEKF_OK;
 }
 
@@ -426,7 +530,7 @@ fekf_status fekf_kf_get_state(fekf_kf* k, double* lambda, double* A_last, int* f
 fekf_status fekf_kf_info(const fekf_kf* k, int64_t* pb, int64_t* tl, int64_t* npad, int64_t* items) {
   if (!k) return FEKF_EINVAL;
   const KfPlan& p = k->kf.plan;
-  if (pb) *pb = p.tiles_local * (int64_t)KT * KT * (int64_t)sizeof(double);
+  if (pb) *pb = p.tiles_local * (int64_t)KT * KT * (int64_t)k->kf.elem();
   if (tl) *tl = p.tiles_local;
   if (npad) *npad = p.Npad;
   if (items) *items = (int64_t)p.items.size();
@@ -553,35 +657,48 @@ fekf_status fekf_train_step(fekf_ctx* ctx, const double* coord, const double* bo
     return FEKF_EINVAL;
   }
   Ctx& c = ctx->c;
-  const int64_t l0 = g_launches;
-  const int nb = c.B;
-  const double sqrt_bs = std::sqrt((double)c.Bg);
-  double* g = c.gbuf.as<double>();
-  double* esum = g + c.Np;
-  FEKF_CHECK_CUDA(cudaMemsetAsync(metrics, 0, sizeof(double) * 8, s));
-  FEKF_TRY(geometry(c, coord, box, nb, s));
-  // energy update (1 per minibatch)
-  FEKF_TRY(energy_grad_pass(c, nb, e_label, g, esum, s));
-  FEKF_TRY(comm_allreduce(c.comm, g, c.Np + 1, s));
-  abe_kernel<<<1, 1, 0, s>>>(esum, 1.0 / c.Bg, c.abe.as<double>(), metrics + 0);
-  FEKF_LAUNCH_CHECK();
-  count_launch();
-  FEKF_TRY(c.kf->update(g, c.abe.as<double>(), sqrt_bs, c.w.as<double>(), s));
-  // force updates
-  const int apg = c.o.atoms_per_group;
-  for (int k = 0; k < c.o.force_groups; ++k) {
-    FEKF_TRY(force_grad_pass(c, nb, f_label, force_idx + (size_t)k * apg, apg, g, esum, s));
-    FEKF_TRY(comm_allreduce(c.comm, g, c.Np + 1, s));
-    abe_kernel<<<1, 1, 0, s>>>(esum, 1.0 / ((double)c.Bg * apg * 3) / c.Na, c.abe.as<double>(),
-                               k < 4 ? metrics + 1 + k : nullptr);
-    FEKF_LAUNCH_CHECK();
-    count_launch();
-    FEKF_TRY(c.kf->update(g, c.abe.as<double>(), sqrt_bs, c.w.as<double>(), s));
+  if (!c.use_graph) {
+    const int64_t l0 = g_launches;
+    FEKF_TRY(step_body(c, coord, box, e_label, f_label, force_idx, metrics, s));
+    c.last_launches = g_launches - l0;
+    ++c.nsteps;
+    return FEKF_OK;
   }
-  metrics_kernel<<<1, 1, 0, s>>>(c.kf->state.as<KfState>(), c.err_d.as<int>(), c.overflow.as<int>(), nb, metrics);
-  FEKF_LAUNCH_CHECK();
-  count_launch();
-  c.last_launches = g_launches - l0;
+  // stage the step's inputs into the captured buffers (stream order on s), then replay on gstream
+  const size_t na3 = sizeof(double) * (size_t)c.B * c.Na * 3;
+  FEKF_CHECK_CUDA(cudaMemcpyAsync(c.st_coord.p, coord, na3, cudaMemcpyDeviceToDevice, s));
+  FEKF_CHECK_CUDA(cudaMemcpyAsync(c.st_box.p, box, sizeof(double) * c.B * 9, cudaMemcpyDeviceToDevice, s));
+  FEKF_CHECK_CUDA(cudaMemcpyAsync(c.st_e.p, e_label, sizeof(double) * c.B, cudaMemcpyDeviceToDevice, s));
+  FEKF_CHECK_CUDA(cudaMemcpyAsync(c.st_f.p, f_label, na3, cudaMemcpyDeviceToDevice, s));
+  if (c.o.force_groups > 0)
+    FEKF_CHECK_CUDA(cudaMemcpyAsync(c.st_fidx.p, force_idx, sizeof(int32_t) * c.o.force_groups * c.o.atoms_per_group,
+                                    cudaMemcpyDeviceToDevice, s));
+  StepGraph* G = nullptr;
+  FEKF_TRY(step_graph(c, &G));
+  if (G->tm.pending) FEKF_TRY(c.kf->harvest_graph(&G->tm));
+  FEKF_CHECK_CUDA(cudaEventRecord(c.gev_in, s));
+  FEKF_CHECK_CUDA(cudaStreamWaitEvent(c.gstream, c.gev_in, 0));
+  FEKF_CHECK_CUDA(cudaGraphLaunch(G->exec, c.gstream));
+  FEKF_CHECK_CUDA(cudaEventRecord(c.gev_out, c.gstream));
+  FEKF_CHECK_CUDA(cudaStreamWaitEvent(s, c.gev_out, 0));
+  FEKF_CHECK_CUDA(cudaMemcpyAsync(metrics, c.st_met.p, sizeof(double) * 8, cudaMemcpyDeviceToDevice, s));
+  if (c.kf->timing && !G->tm.ev.empty()) {
+    G->tm.pending = true;
+    c.kf->pend_graphs.push_back(&G->tm);
+  }
+  c.kf->npend = G->npend_after;
+  g_launches += G->launches;
+  c.last_launches = G->launches;
+  ++c.nsteps;
+  return FEKF_OK;
+}
+
+fekf_status fekf_set_graph_mode(fekf_ctx* ctx, int enable) {
+  if (!ctx || (enable != 0 && enable != 1)) { set_error("set_graph_mode: bad args"); return FEKF_EINVAL; }
+  Ctx& c = ctx->c;
+  if (c.gstream) FEKF_CHECK_CUDA(cudaStreamSynchronize(c.gstream));
+  if (!enable) c.drop_graphs();
+  c.use_graph = enable != 0;
   return FEKF_OK;
 }
 

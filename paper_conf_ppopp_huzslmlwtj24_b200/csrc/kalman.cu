@@ -175,29 +175,45 @@ __device__ __forceinline__ void consumer_bar() { asm volatile("bar.sync 1, 256;"
 // ------------------------------------------------------------------------------------------------
 // the P pass
 // ------------------------------------------------------------------------------------------------
-constexpr int MAX_STAGES = 8;
+constexpr int MAX_STAGES = 12;
 constexpr int TILE_ELEMS = KT * KT;
-constexpr uint32_t TILE_BYTES = TILE_ELEMS * sizeof(double);
+
+// Storage element of P: fp64 (default) or fp32 (the fp32 variant, reading Z22).  A lane handles two
+// adjacent columns of a tile row; values are widened to fp64 for every product and correction.
+__device__ __forceinline__ double2 ld2(const double* p) { return *reinterpret_cast<const double2*>(p); }
+__device__ __forceinline__ double2 ld2(const float* p) {
+  const float2 v = *reinterpret_cast<const float2*>(p);
+  return make_double2((double)v.x, (double)v.y);
+}
+__device__ __forceinline__ void st2(double* p, double2 v) { *reinterpret_cast<double2*>(p) = v; }
+__device__ __forceinline__ void st2(float* p, double2 v) {
+  *reinterpret_cast<float2*>(p) = make_float2(__double2float_rn(v.x), __double2float_rn(v.y));
+}
 constexpr int PASS_THREADS = 288;  // 8 consumer warps + 1 producer warp
 constexpr size_t PASS_SMEM = 227 * 1024 - 256;  // + 128 B of static shared memory (deferred coefficients)
-// [full[8] | empty[8] | meta[8]] (256 B), column-reduction buffers (8 KiB), then the stage ring; a stage
-// is one tile plus, for a read-write pass, the 2K vector segments (u_k rows I, u_k columns J) it needs.
+// [full | empty | meta] barriers and stage metadata, column-reduction buffers (8 KiB), then the stage
+// ring; a stage is one tile plus, for a read-write pass, the 2K fp64 vector segments (u_k rows I, u_k
+// columns J) it needs.
 constexpr size_t PASS_HDR = 2 * MAX_STAGES * sizeof(uint64_t) + MAX_STAGES * sizeof(int4) + 2 * 8 * KT * sizeof(double);
 
 // rw = 0: read-only pass, u_B = B g.  rw = 1: B <- sigma (B - sum_{k<K} beta_k u_k u_k^T) written back,
 // then u_B = B_new g.  Tile-row segments are pulled from an atomic counter by a producer warp that
 // streams each 32 KiB tile (and, for rw, the 2K 512-byte vector segments it needs) with TMA bulk copies
-// into a ring of `nst` stages (6 for read-only passes, 5 when 5 corrections ride along).
+// into a ring of `nst` stages (fp64: 6 for read-only passes, fewer when corrections ride along; fp32
+// tiles are 16 KiB, so twice as many).  `stage_bytes` = tile bytes + (1 + 2K)*T*8: the tile, its g_J
+// segment and the 2K correction segments.
+template <typename PT>
 __global__ void __launch_bounds__(PASS_THREADS, 1)
-kf_pass_kernel(double* __restrict__ P, const ItemD* __restrict__ items, int n_items, int* counter,
+kf_pass_kernel(PT* __restrict__ P, const ItemD* __restrict__ items, int n_items, int* counter,
                const double* __restrict__ gpad, const double* __restrict__ ulist, long long npad, int rw, int K,
-               int nst, int stage_elems, const KfState* st, double* __restrict__ ws) {
+               int nst, int stage_bytes, const KfState* st, double* __restrict__ ws) {
+  constexpr uint32_t TILE_BYTES = TILE_ELEMS * sizeof(PT);
   extern __shared__ __align__(128) unsigned char smem[];
   uint64_t* full = reinterpret_cast<uint64_t*>(smem);
   uint64_t* empty = full + MAX_STAGES;
   int4* meta = reinterpret_cast<int4*>(empty + MAX_STAGES);
   double* colred = reinterpret_cast<double*>(meta + MAX_STAGES);
-  double* stages = colred + 2 * 8 * KT;
+  unsigned char* stages = reinterpret_cast<unsigned char*>(colred + 2 * 8 * KT);
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   if (!rw) K = 0;
 
@@ -215,7 +231,7 @@ kf_pass_kernel(double* __restrict__ P, const ItemD* __restrict__ items, int n_it
     if (lane == 0) {
       int s = 0;
       uint32_t ph = 0;
-      const uint32_t bytes = TILE_BYTES + 2u * (uint32_t)K * KT * sizeof(double);
+      const uint32_t bytes = TILE_BYTES + (1u + 2u * (uint32_t)K) * KT * sizeof(double);
       while (true) {
         const int itx = atomicAdd(counter, 1);
         if (itx >= n_items) break;
@@ -223,14 +239,17 @@ kf_pass_kernel(double* __restrict__ P, const ItemD* __restrict__ items, int n_it
         for (int t = 0; t < it.nJ; ++t) {
           mbar_wait(&empty[s], ph ^ 1);
           meta[s] = make_int4(itx, it.J0 + t, (t == 0 ? 1 : 0) | (t == it.nJ - 1 ? 2 : 0), 0);
-          double* st_s = stages + (size_t)s * stage_elems;
+          unsigned char* st_s = stages + (size_t)s * stage_bytes;
+          double* st_g = reinterpret_cast<double*>(st_s + TILE_BYTES);
+          double* st_v = st_g + KT;
           mbar_arrive_tx(&full[s], bytes);
           tma_load_1d(st_s, P + (size_t)(it.tile_off + t) * TILE_ELEMS, TILE_BYTES, &full[s]);
+          // g_J rides with its tile: no dependent global load on the consumers' per-tile path
+          tma_load_1d(st_g, gpad + it.vbase + (size_t)(it.J0 + t) * KT, KT * sizeof(double), &full[s]);
           for (int k = 0; k < K; ++k) {
             const double* uk = ulist + (size_t)k * npad + it.vbase;
-            tma_load_1d(st_s + TILE_ELEMS + k * KT, uk + (size_t)it.I * KT, KT * sizeof(double), &full[s]);
-            tma_load_1d(st_s + TILE_ELEMS + (K + k) * KT, uk + (size_t)(it.J0 + t) * KT, KT * sizeof(double),
-                        &full[s]);
+            tma_load_1d(st_v + k * KT, uk + (size_t)it.I * KT, KT * sizeof(double), &full[s]);
+            tma_load_1d(st_v + (K + k) * KT, uk + (size_t)(it.J0 + t) * KT, KT * sizeof(double), &full[s]);
           }
           if (++s == nst) { s = 0; ph ^= 1; }
         }
@@ -268,14 +287,15 @@ kf_pass_kernel(double* __restrict__ P, const ItemD* __restrict__ items, int n_it
         racc[k] = 0.0;
       }
     }
-    const double2 gJ = __ldg(reinterpret_cast<const double2*>(gpad + it.vbase + (long long)J * KT + c0));
-    double* t = stages + (size_t)s * stage_elems;
-    const double* vI = t + TILE_ELEMS;
-    const double* vJ = t + TILE_ELEMS + K * KT;
+    PT* t = reinterpret_cast<PT*>(stages + (size_t)s * stage_bytes);
+    const double* vg = reinterpret_cast<const double*>(t + TILE_ELEMS);
+    const double2 gJ = *reinterpret_cast<const double2*>(vg + c0);
+    const double* vI = vg + KT;
+    const double* vJ = vI + K * KT;
     double ca0 = 0.0, ca1 = 0.0;
     double2 v[8];
 #pragma unroll
-    for (int q = 0; q < 8; ++q) v[q] = *reinterpret_cast<const double2*>(t + (warp + 8 * q) * KT + c0);
+    for (int q = 0; q < 8; ++q) v[q] = ld2(t + (warp + 8 * q) * KT + c0);
     if (rw) {
       // sum_k beta_k u_k[r] u_k[c] for this lane's rows r and columns c, k outermost (u_k[c] loaded once)
       double2 cc[8];
@@ -295,7 +315,8 @@ kf_pass_kernel(double* __restrict__ P, const ItemD* __restrict__ items, int n_it
       for (int q = 0; q < 8; ++q) {
         v[q].x = sig * (v[q].x - cc[q].x);
         v[q].y = sig * (v[q].y - cc[q].y);
-        *reinterpret_cast<double2*>(t + (warp + 8 * q) * KT + c0) = v[q];
+        st2(t + (warp + 8 * q) * KT + c0, v[q]);
+        if constexpr (sizeof(PT) == 4) v[q] = ld2(t + (warp + 8 * q) * KT + c0);  // u_B = B_new g, B_new as stored
       }
     }
 #pragma unroll
@@ -472,16 +493,17 @@ __device__ __forceinline__ double deferred_value(double b, const KfState* st, co
 }
 
 // rewrite B = P_t (flush) — one CTA per item
-__global__ void kf_apply_pending_kernel(double* __restrict__ P, const ItemD* __restrict__ items,
+template <typename PT>
+__global__ void kf_apply_pending_kernel(PT* __restrict__ P, const ItemD* __restrict__ items,
                                         const double* __restrict__ ulist, long long npad, const KfState* st) {
   const ItemD it = items[blockIdx.x];
   for (int t = 0; t < it.nJ; ++t) {
-    double* tile = P + (size_t)(it.tile_off + t) * TILE_ELEMS;
+    PT* tile = P + (size_t)(it.tile_off + t) * TILE_ELEMS;
     const int J = it.J0 + t;
     for (int e = threadIdx.x; e < TILE_ELEMS; e += blockDim.x) {
       const int r = e / KT, c = e % KT;
-      tile[e] = deferred_value(tile[e], st, ulist, npad, it.vbase + (long long)it.I * KT + r,
-                               it.vbase + (long long)J * KT + c);
+      tile[e] = (PT)deferred_value((double)tile[e], st, ulist, npad, it.vbase + (long long)it.I * KT + r,
+                                   it.vbase + (long long)J * KT + c);
     }
   }
 }
@@ -491,50 +513,53 @@ __global__ void kf_clear_pending_kernel(KfState* st) {
 }
 
 // P = I on the valid part of every block, 0 on the padding
-__global__ void kf_init_kernel(double* __restrict__ P, const ItemD* __restrict__ items, const int* nblk) {
+template <typename PT>
+__global__ void kf_init_kernel(PT* __restrict__ P, const ItemD* __restrict__ items, const int* nblk) {
   const ItemD it = items[blockIdx.x];
   const int n = nblk[it.blk];
   for (int t = 0; t < it.nJ; ++t) {
-    double* tile = P + (size_t)(it.tile_off + t) * TILE_ELEMS;
+    PT* tile = P + (size_t)(it.tile_off + t) * TILE_ELEMS;
     const int J = it.J0 + t;
     for (int e = threadIdx.x; e < TILE_ELEMS; e += blockDim.x) {
       const int r = e / KT, c = e % KT;
       const int gr = it.I * KT + r, gc = J * KT + c;
-      tile[e] = (gr == gc && gr < n) ? 1.0 : 0.0;
+      tile[e] = (gr == gc && gr < n) ? (PT)1 : (PT)0;
     }
   }
 }
 
 // dense <-> packed for one block (tests / checkpoints); get applies the deferred corrections on the fly
-__global__ void kf_get_block_kernel(const double* __restrict__ P, const ItemD* __restrict__ items, int blk, int n,
+template <typename PT>
+__global__ void kf_get_block_kernel(const PT* __restrict__ P, const ItemD* __restrict__ items, int blk, int n,
                                     const double* __restrict__ ulist, long long npad, const KfState* st,
                                     double* __restrict__ dst) {
   const ItemD it = items[blockIdx.x];
   if (it.blk != blk) return;
   for (int t = 0; t < it.nJ; ++t) {
-    const double* tile = P + (size_t)(it.tile_off + t) * TILE_ELEMS;
+    const PT* tile = P + (size_t)(it.tile_off + t) * TILE_ELEMS;
     const int J = it.J0 + t;
     for (int e = threadIdx.x; e < TILE_ELEMS; e += blockDim.x) {
       const int r = e / KT, c = e % KT;
       const int gr = it.I * KT + r, gc = J * KT + c;
       if (gr >= n || gc >= n) continue;
-      const double v = deferred_value(tile[e], st, ulist, npad, it.vbase + gr, it.vbase + gc);
+      const double v = deferred_value((double)tile[e], st, ulist, npad, it.vbase + gr, it.vbase + gc);
       dst[(size_t)gr * n + gc] = v;
       if (J != it.I) dst[(size_t)gc * n + gr] = v;
     }
   }
 }
-__global__ void kf_set_block_kernel(double* __restrict__ P, const ItemD* __restrict__ items, int blk, int n,
+template <typename PT>
+__global__ void kf_set_block_kernel(PT* __restrict__ P, const ItemD* __restrict__ items, int blk, int n,
                                     const double* __restrict__ src) {
   const ItemD it = items[blockIdx.x];
   if (it.blk != blk) return;
   for (int t = 0; t < it.nJ; ++t) {
-    double* tile = P + (size_t)(it.tile_off + t) * TILE_ELEMS;
+    PT* tile = P + (size_t)(it.tile_off + t) * TILE_ELEMS;
     const int J = it.J0 + t;
     for (int e = threadIdx.x; e < TILE_ELEMS; e += blockDim.x) {
       const int r = e / KT, c = e % KT;
       const int gr = it.I * KT + r, gc = J * KT + c;
-      tile[e] = (gr < n && gc < n) ? src[(size_t)gr * n + gc] : 0.0;
+      tile[e] = (PT)((gr < n && gc < n) ? src[(size_t)gr * n + gc] : 0.0);
     }
   }
 }
@@ -557,11 +582,16 @@ fekf_status Kf::create(const std::vector<int>& blocks, const fekf_opt_cfg& o, fe
   opt = o;
   comm = c;
   defer = std::max(1, std::min(KMAX, o.p_defer > 0 ? o.p_defer : 1));
+  if (o.precision != 0 && o.precision != 32 && o.precision != 64) {
+    set_error("kf_create: precision must be 32 or 64");
+    return FEKF_EINVAL;
+  }
+  p32 = o.precision == 32;
   int world = 1, rank = 0;
   if (comm) { world = comm_world(comm); rank = comm_rank(comm); }
   plan.build(blocks, world, rank, SEG_TILES);
   const KfPlan& p = plan;
-  FEKF_TRY(dalloc(P, (size_t)p.tiles_local * TILE_BYTES + 16));
+  FEKF_TRY(dalloc(P, (size_t)p.tiles_local * TILE_ELEMS * elem() + 16));
   FEKF_TRY(dalloc(items_d, std::max<size_t>(1, p.items.size()) * sizeof(ItemD)));
   FEKF_TRY(dalloc(ws, (size_t)std::max<int64_t>(1, p.ws_slots) * KT * sizeof(double)));
   FEKF_TRY(dalloc(gpad, p.Npad * sizeof(double)));
@@ -596,9 +626,11 @@ fekf_status Kf::create(const std::vector<int>& blocks, const fekf_opt_cfg& o, fe
   s.c_mult = o.noise_mode == 0 ? (double)p.L : 1.0;
   FEKF_CHECK_CUDA(cudaMemcpy(state.p, &s, sizeof(KfState), cudaMemcpyHostToDevice));
   FEKF_CHECK_CUDA(cudaMemset(ulist.p, 0, (size_t)KMAX * p.Npad * sizeof(double)));
-  FEKF_CHECK_CUDA(cudaFuncSetAttribute(kf_pass_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)PASS_SMEM));
+  FEKF_CHECK_CUDA(cudaFuncSetAttribute(kf_pass_kernel<double>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)PASS_SMEM));
+  FEKF_CHECK_CUDA(cudaFuncSetAttribute(kf_pass_kernel<float>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)PASS_SMEM));
   if (!p.items.empty()) {
-    kf_init_kernel<<<(unsigned)p.items.size(), 256>>>(P.as<double>(), items_d.as<ItemD>(), n_d.as<int>());
+    if (p32) kf_init_kernel<<<(unsigned)p.items.size(), 256>>>(P.as<float>(), items_d.as<ItemD>(), n_d.as<int>());
+    else kf_init_kernel<<<(unsigned)p.items.size(), 256>>>(P.as<double>(), items_d.as<ItemD>(), n_d.as<int>());
     FEKF_LAUNCH_CHECK();
   }
   FEKF_CHECK_CUDA(cudaDeviceSynchronize());
@@ -606,33 +638,47 @@ fekf_status Kf::create(const std::vector<int>& blocks, const fekf_opt_cfg& o, fe
   return FEKF_OK;
 }
 
-fekf_status Kf::timing_ctl(int mode, double* total_ms, int64_t* launches, int64_t* rw_launches) {
-  if (mode == 1) {
-    timing = true;
-    ev_used = 0;
-    ev_rw.clear();
-    return FEKF_OK;
-  }
-  timing = false;
-  double tot = 0.0;
-  for (size_t k = 0; k + 1 < ev_used; k += 2) {
-    FEKF_CHECK_CUDA(cudaEventSynchronize(ev[k + 1]));
+fekf_status Kf::harvest(std::vector<EvPair>& pairs, size_t n) {
+  for (size_t k = 0; k < n; ++k) {
+    FEKF_CHECK_CUDA(cudaEventSynchronize(pairs[k].b));
     float ms = 0.f;
-    FEKF_CHECK_CUDA(cudaEventElapsedTime(&ms, ev[k], ev[k + 1]));
-    tot += ms;
-  }
-  if (total_ms) *total_ms = tot;
-  if (launches) *launches = (int64_t)(ev_used / 2);
-  if (rw_launches) {
-    int64_t n = 0;
-    for (char c : ev_rw) n += c;
-    *rw_launches = n;
+    FEKF_CHECK_CUDA(cudaEventElapsedTime(&ms, pairs[k].a, pairs[k].b));
+    t_ms += ms;
+    t_n += 1;
+    t_rw += pairs[k].rw;
   }
   return FEKF_OK;
 }
 
+fekf_status Kf::harvest_graph(GraphTiming* g) {
+  if (!g->pending) return FEKF_OK;
+  g->pending = false;
+  pend_graphs.erase(std::remove(pend_graphs.begin(), pend_graphs.end(), g), pend_graphs.end());
+  return harvest(g->ev, g->ev.size());
+}
+
+fekf_status Kf::timing_ctl(int mode, double* total_ms, int64_t* launches, int64_t* rw_launches) {
+  if (mode == 1) {
+    timing = true;
+    ev_used = 0;
+    for (GraphTiming* g : pend_graphs) g->pending = false;
+    pend_graphs.clear();
+    t_ms = 0.0;
+    t_n = t_rw = 0;
+    return FEKF_OK;
+  }
+  FEKF_TRY(harvest(ev_pool, ev_used));
+  ev_used = 0;
+  while (!pend_graphs.empty()) FEKF_TRY(harvest_graph(pend_graphs.back()));
+  timing = false;
+  if (total_ms) *total_ms = t_ms;
+  if (launches) *launches = t_n;
+  if (rw_launches) *rw_launches = t_rw;
+  return FEKF_OK;
+}
+
 Kf::~Kf() {
-  for (cudaEvent_t e : ev) cudaEventDestroy(e);
+  for (EvPair& e : ev_pool) { cudaEventDestroy(e.a); cudaEventDestroy(e.b); }
   for (DBuf* b : {&P, &items_d, &ws, &gpad, &ub, &ulist, &dotp, &csr_ptr, &csr_idx, &tc_blk, &tc_c, &off_d, &n_d,
                   &state, &counter, &tcoff_d, &dblk, &cub})
     dfree(*b);
@@ -648,29 +694,37 @@ fekf_status Kf::pass(const double* g, bool rw, cudaStream_t s) {
   if (!p.items.empty()) {
     FEKF_CHECK_CUDA(cudaMemsetAsync(counter.p, 0, sizeof(int), s));
     const int grid = std::min<int>((int)p.items.size(), num_sms());
-    if (timing) {
-      while (ev.size() < ev_used + 2) {
-        cudaEvent_t e;
-        FEKF_CHECK_CUDA(cudaEventCreate(&e));
-        ev.push_back(e);
+    EvPair* tp = nullptr;
+    if (timing || capturing) {
+      if (capturing) {
+        rec->emplace_back();
+        tp = &rec->back();
+      } else {
+        if (ev_pool.size() <= ev_used) ev_pool.emplace_back();
+        tp = &ev_pool[ev_used++];
       }
-      FEKF_CHECK_CUDA(cudaEventRecord(ev[ev_used], s));
+      if (!tp->a) {
+        FEKF_CHECK_CUDA(cudaEventCreate(&tp->a));
+        FEKF_CHECK_CUDA(cudaEventCreate(&tp->b));
+      }
+      tp->rw = rw ? 1 : 0;
+      FEKF_CHECK_CUDA(cudaEventRecordWithFlags(tp->a, s, capturing ? cudaEventRecordExternal : cudaEventRecordDefault));
     }
     const int K = rw ? npend : 0;
-    const int stage_elems = TILE_ELEMS + 2 * K * KT;
-    const int nst = (int)std::min<size_t>(MAX_STAGES, (PASS_SMEM - PASS_HDR) / (stage_elems * sizeof(double)));
-    kf_pass_kernel<<<grid, PASS_THREADS, PASS_SMEM, s>>>(P.as<double>(), items_d.as<ItemD>(), (int)p.items.size(),
-                                                          counter.as<int>(), gpad.as<double>(), ulist.as<double>(),
-                                                          p.Npad, rw ? 1 : 0, K, nst, stage_elems,
-                                                          state.as<KfState>(), ws.as<double>());
+    const int stage_bytes = (int)(TILE_ELEMS * elem() + (1 + 2 * K) * KT * sizeof(double));
+    const int nst = (int)std::min<size_t>(MAX_STAGES, (PASS_SMEM - PASS_HDR) / stage_bytes);
+    if (p32)
+      kf_pass_kernel<float><<<grid, PASS_THREADS, PASS_SMEM, s>>>(
+          P.as<float>(), items_d.as<ItemD>(), (int)p.items.size(), counter.as<int>(), gpad.as<double>(),
+          ulist.as<double>(), p.Npad, rw ? 1 : 0, K, nst, stage_bytes, state.as<KfState>(), ws.as<double>());
+    else
+      kf_pass_kernel<double><<<grid, PASS_THREADS, PASS_SMEM, s>>>(
+          P.as<double>(), items_d.as<ItemD>(), (int)p.items.size(), counter.as<int>(), gpad.as<double>(),
+          ulist.as<double>(), p.Npad, rw ? 1 : 0, K, nst, stage_bytes, state.as<KfState>(), ws.as<double>());
     FEKF_LAUNCH_CHECK();
     count_launch();
     if (rw) ++rw_passes; else ++r_passes;
-    if (timing) {
-      FEKF_CHECK_CUDA(cudaEventRecord(ev[ev_used + 1], s));
-      ev_used += 2;
-      ev_rw.push_back(rw ? 1 : 0);
-    }
+    if (tp) FEKF_CHECK_CUDA(cudaEventRecordWithFlags(tp->b, s, capturing ? cudaEventRecordExternal : cudaEventRecordDefault));
   }
   kf_reduce_u_kernel<<<cdiv(p.n_tc, 4), 256, 0, s>>>(ws.as<double>(), csr_ptr.as<long long>(),
                                                       csr_idx.as<long long>(), p.n_tc, ub.as<double>());
@@ -707,9 +761,14 @@ fekf_status Kf::update(const double* g, const double* abe, double sqrt_bs, doubl
 
 fekf_status Kf::flush(cudaStream_t s) {
   if (!plan.items.empty() && npend > 0) {
-    kf_apply_pending_kernel<<<(unsigned)plan.items.size(), 256, 0, s>>>(P.as<double>(), items_d.as<ItemD>(),
-                                                                         ulist.as<double>(), plan.Npad,
-                                                                         state.as<KfState>());
+    if (p32)
+      kf_apply_pending_kernel<<<(unsigned)plan.items.size(), 256, 0, s>>>(P.as<float>(), items_d.as<ItemD>(),
+                                                                           ulist.as<double>(), plan.Npad,
+                                                                           state.as<KfState>());
+    else
+      kf_apply_pending_kernel<<<(unsigned)plan.items.size(), 256, 0, s>>>(P.as<double>(), items_d.as<ItemD>(),
+                                                                           ulist.as<double>(), plan.Npad,
+                                                                           state.as<KfState>());
     FEKF_LAUNCH_CHECK();
   }
   kf_clear_pending_kernel<<<1, 1, 0, s>>>(state.as<KfState>());
@@ -721,9 +780,13 @@ fekf_status Kf::flush(cudaStream_t s) {
 fekf_status Kf::get_block(int b, double* dst, cudaStream_t s) {
   if (b < 0 || b >= plan.L) { set_error("get_block: bad block"); return FEKF_EINVAL; }
   if (plan.items.empty()) return FEKF_OK;
-  kf_get_block_kernel<<<(unsigned)plan.items.size(), 256, 0, s>>>(P.as<double>(), items_d.as<ItemD>(), b, plan.n[b],
-                                                                   ulist.as<double>(), plan.Npad, state.as<KfState>(),
-                                                                   dst);
+  const unsigned nit = (unsigned)plan.items.size();
+  if (p32)
+    kf_get_block_kernel<<<nit, 256, 0, s>>>(P.as<float>(), items_d.as<ItemD>(), b, plan.n[b], ulist.as<double>(),
+                                            plan.Npad, state.as<KfState>(), dst);
+  else
+    kf_get_block_kernel<<<nit, 256, 0, s>>>(P.as<double>(), items_d.as<ItemD>(), b, plan.n[b], ulist.as<double>(),
+                                            plan.Npad, state.as<KfState>(), dst);
   FEKF_LAUNCH_CHECK();
   return FEKF_OK;
 }
@@ -732,8 +795,9 @@ fekf_status Kf::set_block(int b, const double* src, cudaStream_t s) {
   if (b < 0 || b >= plan.L) { set_error("set_block: bad block"); return FEKF_EINVAL; }
   FEKF_TRY(flush(s));
   if (plan.items.empty()) return FEKF_OK;
-  kf_set_block_kernel<<<(unsigned)plan.items.size(), 256, 0, s>>>(P.as<double>(), items_d.as<ItemD>(), b, plan.n[b],
-                                                                   src);
+  const unsigned nit = (unsigned)plan.items.size();
+  if (p32) kf_set_block_kernel<<<nit, 256, 0, s>>>(P.as<float>(), items_d.as<ItemD>(), b, plan.n[b], src);
+  else kf_set_block_kernel<<<nit, 256, 0, s>>>(P.as<double>(), items_d.as<ItemD>(), b, plan.n[b], src);
   FEKF_LAUNCH_CHECK();
   return FEKF_OK;
 }

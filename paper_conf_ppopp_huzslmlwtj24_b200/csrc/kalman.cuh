@@ -50,20 +50,43 @@ int comm_world(fekf_comm* c);
 int comm_rank(fekf_comm* c);
 fekf_status comm_allreduce(fekf_comm* c, double* buf, long long n, cudaStream_t s);
 
+struct EvPair {
+  cudaEvent_t a = nullptr, b = nullptr;
+  char rw = 0;
+};
+
+// Event pairs recorded inside one captured step graph; harvested before the graph is replayed again
+// (by then its previous replay has finished) and when timing stops.
+struct GraphTiming {
+  std::vector<EvPair> ev;
+  bool pending = false;
+};
+
 struct Kf {
   fekf_opt_cfg opt{};
   fekf_comm* comm = nullptr;
   KfPlan plan;
   int defer = 1;                 // corrections deferred before P is rewritten (1 = rewrite every update)
   int npend = 0;                 // host mirror of the device npend
+  bool p32 = false;              // P stored fp32 (opt.precision == 32, reading Z22)
+  size_t elem() const { return p32 ? sizeof(float) : sizeof(double); }
   DBuf P, items_d, ws, gpad, ub, ulist, dotp, csr_ptr, csr_idx, tc_blk, tc_c, off_d, n_d, state, counter;
   DBuf tcoff_d, dblk, cub;       // block -> tile-column offsets, per-block dots, per-block coefficients
+  // Live timing of the P pass: a [start, stop] event pair recorded on the launching stream around every
+  // pass launch.  Eager launches draw pairs from `ev_pool`; while a step graph is being captured the pairs
+  // go to that graph's own list (`rec`, external event-record nodes) and are harvested after each replay.
   bool timing = false;
-  std::vector<cudaEvent_t> ev;   // [start, stop] per timed pass launch
+  bool capturing = false;
+  std::vector<EvPair> ev_pool;
   size_t ev_used = 0;
-  std::vector<char> ev_rw;       // 1 = read-write pass
+  std::vector<EvPair>* rec = nullptr;   // non-null while capturing with timing on
+  double t_ms = 0.0;
+  int64_t t_n = 0, t_rw = 0;
   long long rw_passes = 0, r_passes = 0;
   fekf_status timing_ctl(int mode, double* total_ms, int64_t* launches, int64_t* rw_launches);
+  std::vector<GraphTiming*> pend_graphs;  // replayed graphs whose pairs are not harvested yet
+  fekf_status harvest(std::vector<EvPair>& pairs, size_t n);   // add the elapsed times of n recorded pairs
+  fekf_status harvest_graph(GraphTiming* g);
   fekf_status create(const std::vector<int>& blocks, const fekf_opt_cfg& o, fekf_comm* c);
   ~Kf();
   fekf_status pass(const double* g, bool rw, cudaStream_t s);

@@ -1,6 +1,7 @@
 // DeePMD se_a model context: parameter layout, work buffers and the kernel launchers of the
 // forward / backward / Jacobian passes.  See nets.cu for the math and citations.
 #pragma once
+#include <map>
 #include <memory>
 #include <vector>
 
@@ -37,6 +38,17 @@ struct FitNet {        // fitting net of type t
   DBuf eout, ebar;     // [2F]
 };
 
+// One captured minibatch step (a10: "one CUDA graph").  The launch sequence of a step depends on the
+// host state only through the number of pending Kalman corrections at entry (which passes rewrite P),
+// so graphs are cached by that count and a step-parity bit (two graphs alternate, so the P-pass event
+// pairs of a graph's previous replay can be read back for live timing without stalling the stream).
+struct StepGraph {
+  cudaGraphExec_t exec = nullptr;
+  int npend_after = 0;
+  int64_t launches = 0;
+  GraphTiming tm;
+};
+
 struct Ctx {
   fekf_model_cfg m{};
   fekf_opt_cfg o{};
@@ -64,6 +76,14 @@ struct Ctx {
   DBuf abe, metrics_tmp, abs_sum;
   size_t splitk_elems = 0, colsum_elems = 0;
   int64_t last_launches = 0;
+  // step graphs: inputs are staged into ctx-owned buffers so the captured pointers stay fixed
+  bool use_graph = true;
+  std::map<int, StepGraph> graphs;
+  cudaStream_t gstream = nullptr;
+  cudaEvent_t gev_in = nullptr, gev_out = nullptr;
+  DBuf st_coord, st_box, st_e, st_f, st_fidx, st_met;
+  int64_t nsteps = 0;
+  void drop_graphs();
 
   fekf_status init(const fekf_model_cfg& m, const fekf_opt_cfg& o, int natoms, const int32_t* types_host, int B,
                    int Bg, fekf_comm* comm);

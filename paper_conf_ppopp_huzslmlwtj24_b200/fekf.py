@@ -36,7 +36,7 @@ class ModelCfg(C.Structure):
 class OptCfg(C.Structure):
     _fields_ = [("lambda0", C.c_double), ("nu", C.c_double), ("block_size", C.c_int), ("noise_mode", C.c_int),
                 ("grad_reduce", C.c_int), ("force_groups", C.c_int), ("atoms_per_group", C.c_int),
-                ("p_defer", C.c_int)]
+                ("p_defer", C.c_int), ("precision", C.c_int)]
 
 
 _lib = None
@@ -76,6 +76,7 @@ def lib():
         "fekf_kalman_update": ([vp, vp, vp, i32, i32, vp], i32),
         "fekf_train_step": ([vp, vp, vp, vp, vp, vp, vp, vp], i32),
         "fekf_last_launch_count": ([vp, C.POINTER(i64)], i32),
+        "fekf_set_graph_mode": ([vp, i32], i32),
     }
     for name, (args, res) in sigs.items():
         f = getattr(L, name)
@@ -92,7 +93,7 @@ EXPORTED = [
     "fekf_kf_info", "fekf_kf_pass", "fekf_kf_timing", "fekf_create", "fekf_destroy", "fekf_param_count", "fekf_get_kf",
     "fekf_set_params", "fekf_get_params", "fekf_build_nlist", "fekf_env_mat", "fekf_forward",
     "fekf_energy_jacobian", "fekf_force_jacobian", "fekf_kalman_update", "fekf_train_step",
-    "fekf_last_launch_count",
+    "fekf_last_launch_count", "fekf_set_graph_mode",
 ]
 
 
@@ -156,6 +157,9 @@ def opt_cfg(o=None) -> OptCfg:
     c.force_groups = int(_get(o, "force_groups", 4)) if o is not None else 4
     c.atoms_per_group = int(_get(o, "atoms_per_group", 6)) if o is not None else 6
     c.p_defer = int(_get(o, "p_defer", 15)) if o is not None else 15
+    c.precision = int(_get(o, "precision", 64)) if o is not None else 64
+    if c.precision not in (32, 64):
+        raise ValueError("precision must be 32 or 64")
     return c
 
 
@@ -285,7 +289,7 @@ class Context:
     """Model + optimizer context (fekf_create).  All tensors are CUDA, contiguous; float64 / int32."""
 
     def __init__(self, model, opt=None, natoms=None, types=None, local_batch=1, global_batch=None,
-                 comm: Comm | None = None):
+                 comm: Comm | None = None, graph: bool = True):
         L = lib()
         self.mc = model_cfg(model)
         self.oc = opt_cfg(opt)
@@ -306,6 +310,12 @@ class Context:
         _, blocks = plan_layout(model, self.oc.block_size)
         self.kf = KalmanFilter(blocks, _handle=kh, _owner=self)
         self.comm = comm
+        if not graph:
+            self.set_graph_mode(False)
+
+    def set_graph_mode(self, enable: bool):
+        """a10: replay each minibatch step as one captured CUDA graph (default) or launch eagerly."""
+        _check(lib().fekf_set_graph_mode(self.h, 1 if enable else 0))
 
     # ---- parameters ----
     def set_params(self, w, stream=None):
@@ -377,6 +387,12 @@ class Context:
     def train_step(self, coord, box, e_label, f_label, force_idx, metrics=None, stream=None):
         if metrics is None:
             metrics = torch.empty(8, dtype=torch.float64, device="cuda")
+        na = self.natoms
+        for t, n, name in ((coord, self.B * na * 3, "coord"), (box, self.B * 9, "box"), (e_label, self.B, "e_label"),
+                           (f_label, self.B * na * 3, "f_label"), (metrics, 8, "metrics"),
+                           (force_idx, self.oc.force_groups * self.oc.atoms_per_group, "force_idx")):
+            if t.numel() != n:
+                raise FekfError(1, f"train_step: {name} has {t.numel()} elements, expected {n} (local_batch={self.B})")
         _check(lib().fekf_train_step(self.h, _ptr(coord, torch.float64, "coord"), _ptr(box, torch.float64, "box"),
                                      _ptr(e_label, torch.float64, "e_label"), _ptr(f_label, torch.float64, "f_label"),
                                      _ptr(force_idx, torch.int32, "force_idx"), _ptr(metrics, torch.float64, "metrics"),

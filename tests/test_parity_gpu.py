@@ -148,14 +148,46 @@ def test_kalman_updates(blocks, noise_mode, p_defer):
         assert rel(kf.get_block(b).cpu(), st.P[b]) < 1e-12
 
 
-def test_kalman_full_size_sampled_blocks():
+@pytest.mark.parametrize("blocks", [[5, 70, 130], [1, 200, 127, 65]])
+@pytest.mark.parametrize("p_defer", [1, 5, 16])
+def test_kalman_updates_fp32(blocks, p_defer):
+    """fp32 variant (P stored fp32, reading Z22) against the fp64 oracle: rel 1e-4 (north_star)."""
+    rng = np.random.default_rng(11)
+    opt = dict(lambda0=0.98, nu=0.9987, block_size=1024, noise_mode=0, p_defer=p_defer, precision=32)
+    kf = fk.KalmanFilter(blocks, opt)
+    assert kf.info()["p_bytes_local"] == 4 * 64 * 64 * sum((x + 1) * x // 2 for x in [(n + 63) // 64 for n in blocks])
+    N = sum(blocks)
+    st = O.FEKF(np.zeros(N), blocks, lam=0.98, nu=0.9987, noise_mode=0)
+    st.P = [_rand_spd(rng, n) for n in blocks]
+    for b, P in enumerate(st.P):
+        kf.set_block(b, cu(P))
+    w = torch.zeros(N, dtype=torch.float64, device="cuda")
+    for it in range(max(10, p_defer + 4)):
+        g = rng.standard_normal(N)
+        abe = float(rng.uniform(0.01, 1.0))
+        kf.update(cu(g), cu([abe]), 3.0, w)
+        st.update(g, abe, 9)
+    torch.cuda.synchronize()
+    assert rel(w.cpu(), st.w) < 1e-4
+    for b in range(len(blocks)):
+        assert rel(kf.get_block(b).cpu(), st.P[b]) < 1e-4
+    kf.flush()
+    for b in range(len(blocks)):
+        Pb = kf.get_block(b).cpu().numpy()
+        assert rel(Pb, st.P[b]) < 1e-4
+        assert np.array_equal(Pb, Pb.T)
+
+
+@pytest.mark.parametrize("precision", [64, 32])
+def test_kalman_full_size_sampled_blocks(precision):
     """Bench-size Kalman filter (water-64: 110 blocks, 39 GiB packed P, default p_defer): one update
     checked on sampled blocks against the update recomputed in numpy from the GPU's previous P
     (P_new = (P - A u u^T)/lambda with u = P g per block; w increment sqrt(bs) ABE A u)."""
     wl = get_config("c2_water64")
     _, blocks = fk.plan_layout(wl.model, wl.opt.block_size)
     assert len(blocks) == 110
-    kf = fk.KalmanFilter(blocks, dict(block_size=wl.opt.block_size))
+    kf = fk.KalmanFilter(blocks, dict(block_size=wl.opt.block_size, precision=precision))
+    tol = 1e-11 if precision == 64 else 1e-6   # fp32: the stored P_new is rounded to fp32 (rel 2^-24)
     N = sum(blocks)
     off = np.concatenate([[0], np.cumsum(blocks)])
     gen = torch.Generator(device="cuda").manual_seed(3)
@@ -176,14 +208,18 @@ def test_kalman_full_size_sampled_blocks():
         sl = slice(off[b], off[b + 1])
         u = before[b] @ gn[sl]
         ref = (before[b] - A * np.outer(u, u)) / lam
-        assert rel(kf.get_block(b).cpu(), ref) < 1e-11
-        assert rel(w1[sl] - w0[sl], 4.0 * 0.05 * A * u) < 1e-11
+        assert rel(kf.get_block(b).cpu(), ref) < tol
+        assert rel(w1[sl] - w0[sl], 4.0 * 0.05 * A * u) < tol
 
 
-@pytest.mark.parametrize("name,steps", [("c1_cu32", 10), ("t2_tiny", 4)])
-def test_train_steps(name, steps):
+@pytest.mark.parametrize("name,steps,precision", [("c1_cu32", 10, 64), ("t2_tiny", 4, 64), ("c1_cu32", 10, 32)])
+def test_train_steps(name, steps, precision):
+    """10 minibatch steps (50 KF updates, reading Z20): w and P within rel 1e-9 of the fp64 oracle; the
+    fp32 variant (P stored fp32, reading Z22) within rel 1e-4 (north_star)."""
     wl = get_config(name)
     m, opt = wl.model, wl.opt
+    opt = type(opt)(**{**opt.__dict__, "precision": precision})
+    tol = 1e-9 if precision == 64 else 1e-4
     ds = make_dataset(name, wl.batch * 2)
     na = len(ds["types"])
     w0 = init_weights(m, 3, float(ds["energy"].mean() / na))
@@ -199,10 +235,47 @@ def test_train_steps(name, steps):
         ref = O.train_step(st, ds["coord"][sl], ds["box"][sl], ds["types"], ds["energy"][sl], ds["force"][sl],
                            groups, m, opt)
         mt = met.cpu().numpy()
-        assert abs(mt[0] - ref["abe_e"]) <= 1e-9 * abs(ref["abe_e"])
-        np.testing.assert_allclose(mt[1:5], ref["abe_f"], rtol=1e-9)
+        assert abs(mt[0] - ref["abe_e"]) <= tol * abs(ref["abe_e"])
+        np.testing.assert_allclose(mt[1:5], ref["abe_f"], rtol=tol)
         assert abs(mt[6] - ref["lambda"]) < 1e-14
         assert mt[7] == 0
-    assert rel(ctx.get_params().cpu(), st.w) < 1e-9
+    assert rel(ctx.get_params().cpu(), st.w) < tol
     for b, n in enumerate(st.blocks):
-        assert rel(ctx.kf.get_block(b).cpu(), st.P[b]) < 1e-9
+        assert rel(ctx.kf.get_block(b).cpu(), st.P[b]) < tol
+
+
+def test_step_graph_matches_eager():
+    """a10: the captured step graph (default) and eager launches give bit-identical weights, P and
+    metrics across graph variants (p_defer 2: read-write passes at different updates of a step), and
+    the live P-pass timing sees every pass inside replayed graphs."""
+    wl = get_config("t2_tiny")
+    m = wl.model
+    opt = type(wl.opt)(**{**wl.opt.__dict__, "p_defer": 2})
+    B = wl.batch
+    ds = make_dataset("t2_tiny", B)
+    na = len(ds["types"])
+    w0 = init_weights(m, 3, float(ds["energy"].mean() / na))
+    out = []
+    for graph in (True, False):
+        ctx = fk.Context(m, opt, types=ds["types"], local_batch=B, global_batch=B, graph=graph)
+        ctx.set_params(cu(w0))
+        ctx.kf.timing(True)
+        mets = []
+        for step in range(5):
+            groups = force_groups(na, step, 17, opt.force_groups, opt.atoms_per_group)
+            mets.append(ctx.train_step(cu(ds["coord"]), cu(ds["box"]), cu(ds["energy"]), cu(ds["force"]),
+                                       cu(groups, torch.int32)).clone())
+        ms, n, n_rw = ctx.kf.timing(False)
+        npend, rw_expect = 0, 0
+        for _ in range(25):                              # host mirror of the deferral rule
+            rw = npend >= opt.p_defer
+            rw_expect += rw
+            npend = 1 if rw else npend + 1
+        assert n == 25 and n_rw == rw_expect == 12 and ms > 0
+        assert ctx.last_launch_count() > 50
+        out.append((ctx.get_params().cpu(), [ctx.kf.get_block(b).cpu() for b in range(len(ctx.kf.blocks))],
+                    torch.stack(mets).cpu()))
+        ctx.close()
+    assert torch.equal(out[0][0], out[1][0])
+    assert all(torch.equal(a, b) for a, b in zip(out[0][1], out[1][1]))
+    assert torch.equal(out[0][2], out[1][2])
