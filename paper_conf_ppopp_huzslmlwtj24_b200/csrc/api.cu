@@ -375,7 +375,8 @@ static fekf_status force_grad_pass(Ctx& c, int nb, const double* f_label, const 
                                    double* abs_sum, cudaStream_t s) {
   FEKF_TRY(model_forward(c, nb, false, s));
   FEKF_TRY(seed_force(c, nb, s));
-  FEKF_TRY(model_backward(c, nb, MODE_FORCE, nullptr, s));
+  FEKF_TRY(mark_selected(c, nb, atom_idx, n_sel, s));   // rows touching S_k (tangent-active rows)
+  FEKF_TRY(model_backward(c, nb, MODE_FORCE_SEL, nullptr, s));
   FEKF_TRY(force_error(c, nb, f_label, atom_idx, n_sel, abs_sum, s));
   FEKF_TRY(tangent_env(c, nb, s));
   FEKF_TRY(model_forward(c, nb, true, s));

@@ -291,6 +291,7 @@ struct EmbBwdIO {
   const int* row_idx;
   const int* tidx;                    // tangent rows: tangent row -> primal row (nullptr: primal rows)
   const int* tpos;                    // primal rows, dual: primal row -> tangent row or -1 (nullptr: none)
+  const int* rmap;                    // MODE_FORCE_SEL: row -> primal row (active rows only; nullptr: all)
   int Nm;
   const double* Gbar;                 // primal rows: Gbar (desc_bwd_seed_kernel)
   const double* dR;                   // forces: per-row R~ adjoint less sbar e_0 [R][4]
@@ -401,7 +402,7 @@ __device__ __forceinline__ void bwd_layer(double (&acc)[W::MAXB][2][2][2], doubl
         const int r = warp + NW * i, c = lane + 32 * j;
         y[i][j] = yt[i][j] = hbt[i][j] = 0.0;
         if (c < d && s_slot[r] >= 0) {
-          y[i][j] = tan ? io.Yp[L][(size_t)s_prow[r] * d + c] : ys[r * ldy + c];
+          y[i][j] = (tan || io.rmap) ? io.Yp[L][(size_t)s_prow[r] * d + c] : ys[r * ldy + c];
           const int tp = s_tpos[r];
           if (tp >= 0) {
             yt[i][j] = io.Yt[L][(size_t)tp * d + c];
@@ -451,6 +452,7 @@ __device__ __forceinline__ void bwd_layer(double (&acc)[W::MAXB][2][2][2], doubl
     const int t = threadIdx.x;
     if (t < T * 4) {
       const int r = t >> 2, part = t & 3;
+      // (sbar is written per primal row)
       const double* w0 = sm + W::bW(0);
       double sb = 0.0;
 #pragma unroll
@@ -458,7 +460,7 @@ __device__ __forceinline__ void bwd_layer(double (&acc)[W::MAXB][2][2][2], doubl
       sb += __shfl_xor_sync(0xffffffffu, sb, 1);
       sb += __shfl_xor_sync(0xffffffffu, sb, 2);
       const int row = r0 + r;
-      if (part == 0 && row < R) io.sbar[row] = sb;
+      if (part == 0 && row < R) io.sbar[s_prow[r]] = sb;
       if (io.dR && part < 3) {
         const int be = part, slot = s_slot[r];
         double f = 0.0;
@@ -569,7 +571,7 @@ __device__ __forceinline__ void seed_rows(double* sm, const EmbBwdIO& io, int r0
       const int r = warp + NW * i, c = lane + 32 * j;
       v[i][j] = y[i][j] = yt[i][j] = hbt[i][j] = 0.0;
       if (c < M && r0 + r < R) {
-        v[i][j] = src[(size_t)(r0 + r) * M + c];
+        v[i][j] = src[(size_t)(tan ? r0 + r : s_prow[r]) * M + c];
         y[i][j] = io.Yp[NL - 1][(size_t)s_prow[r] * M + c];
         const int tp = s_tpos[r];
         if (tp >= 0) {
@@ -591,7 +593,7 @@ __device__ __forceinline__ void seed_rows(double* sm, const EmbBwdIO& io, int r0
     }
   if (io.dR && threadIdx.x < T * 4) {
     const int r = threadIdx.x >> 2;
-    s_dr[threadIdx.x] = r0 + r < R ? io.dR[(size_t)r0 * 4 + threadIdx.x] : 0.0;
+    s_dr[threadIdx.x] = r0 + r < R ? io.dR[(size_t)s_prow[r] * 4 + (threadIdx.x & 3)] : 0.0;
   }
 }
 
@@ -631,7 +633,7 @@ __global__ void __launch_bounds__(EMB_BWD_WARPS * 32, 1) emb_bwd_kernel(const do
       const int row = r0 + tid;
       int slot = -1, atom = 0, pr = 0, tp = -1;
       if (row < R) {
-        pr = tan ? io.tidx[row] : row;
+        pr = tan ? io.tidx[row] : (io.rmap ? io.rmap[row] : row);
         slot = io.row_idx[pr];
         atom = slot / io.Nm;
         if (io.tpos) tp = io.tpos[row];
@@ -643,7 +645,7 @@ __global__ void __launch_bounds__(EMB_BWD_WARPS * 32, 1) emb_bwd_kernel(const do
     }
     __syncthreads();
     // the next tile's stored activations (contiguous rows) on their way to L2 while this one computes
-    if (tid == 0) {
+    if (tid == 0 && !io.rmap) {
       const int rn = r0 + gridDim.x * T;
       if (rn + T <= io.Rmax) {
 #pragma unroll
@@ -653,14 +655,16 @@ __global__ void __launch_bounds__(EMB_BWD_WARPS * 32, 1) emb_bwd_kernel(const do
       }
     }
     // ---- [h_{l-1} | 1] for every layer (h recomputed from the stored y) and the middle layers' y
-    if (tid < T * 8) {
+    if (wantw && tid < T * 8) {
       const int r = tid >> 3, cc = tid & 7;
       const int row = r0 + r;
       double v = 0.0;
       if (row < R) v = cc == 0 ? io.hin[row] : (cc == 1 ? one : 0.0);
       sm[W::bAug(0) + r * W::augld(0) + cc] = v;
     }
-    if constexpr (NL >= 2) build_aug<W, 1>(sm, io, r0, R, one);
+    // (rmap rows take no weight gradient and gather their y from the primal rows)
+    if constexpr (NL >= 2)
+      if (!io.rmap) build_aug<W, 1>(sm, io, r0, R, one);
     // ---- seed: hbar_{L-1} = Gbar, zbar_{L-1} (and, for forces, the per-row R~ adjoint)
     seed_rows<W>(sm, io, r0, R, tan, s_dr, s_prow, s_tpos);
     __syncthreads();
@@ -709,7 +713,8 @@ static fekf_status launch_bwd(const double* wp, const EmbBwdIO& io, long long Rm
 template <class W>
 static fekf_status emb_backward_t(Ctx& c, int p, long long Rmax, int mode, double* g, cudaStream_t s) {
   PairNet& P = c.pairs[p];
-  const bool dual = mode == MODE_FORCE_JAC, wantw = mode != MODE_FORCE;
+  const bool sel = mode == MODE_FORCE_SEL;
+  const bool dual = mode == MODE_FORCE_JAC, wantw = mode != MODE_FORCE && !sel;
   const double* wp = c.w.as<double>() + P.L[0].W;
   EmbBwdIO io{};
   io.Rmax = (int)Rmax;
@@ -735,12 +740,13 @@ static fekf_status emb_backward_t(Ctx& c, int p, long long Rmax, int mode, doubl
     FEKF_TRY(launch_bwd<W>(wp, t, Rmax, cap, &gt, s));
     nsets += gt;
   }
-  io.Rdev = c.rowcnt.as<int>() + p;
+  io.Rdev = c.rowcnt.as<int>() + (sel ? c.pairs.size() + p : p);
+  io.rmap = sel ? P.tidx.as<int>() : nullptr;
   io.tpos = dual ? P.tpos.as<int>() : nullptr;
   io.hin = P.hin.as<double>();
   for (int l = 0; l < W::NL; ++l) io.Y[l] = P.Y[l].as<double>();
-  io.sbar = mode == MODE_FORCE ? P.sbar.as<double>() : nullptr;
-  if (mode == MODE_FORCE) {
+  io.sbar = (mode == MODE_FORCE || sel) ? P.sbar.as<double>() : nullptr;
+  if (mode == MODE_FORCE || sel) {
     io.dR = P.Zb[0].template as<double>();
     io.jac = c.jac.as<double>();
     io.rij = c.rij.as<double>();

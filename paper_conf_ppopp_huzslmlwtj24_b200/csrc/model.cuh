@@ -78,6 +78,7 @@ struct Ctx {
   int64_t last_launches = 0;
   // step graphs: inputs are staged into ctx-owned buffers so the captured pointers stay fixed
   bool use_graph = true;
+  bool trows_ready = false;                       // tangent-active rows already built for this force update
   std::map<int, StepGraph> graphs;
   cudaStream_t gstream = nullptr;
   cudaEvent_t gev_in = nullptr, gev_out = nullptr;
@@ -97,8 +98,12 @@ fekf_status launch_envmat(Ctx& c, const double* coord, const double* box, const 
                           double* em, double* jac, double* rij, cudaStream_t s);
 
 // nets.cu
-enum Mode { MODE_ENERGY_GRAD = 0, MODE_FORCE = 1, MODE_FORCE_JAC = 2 };
+// MODE_FORCE_SEL: forces on the selected atoms only (a force update needs F_pred on S_k):
+// the embedding reverse runs over the rows that touch S_k (the tangent-active rows, built beforehand by
+// mark_selected) instead of every row; forces of other atoms are left partial.
+enum Mode { MODE_ENERGY_GRAD = 0, MODE_FORCE = 1, MODE_FORCE_JAC = 2, MODE_FORCE_SEL = 3 };
 fekf_status model_forward(Ctx& c, int nb, bool tangent, cudaStream_t s);
+fekf_status mark_selected(Ctx& c, int nb, const int* atom_idx, int n_sel, cudaStream_t s);
 fekf_status model_backward(Ctx& c, int nb, Mode mode, double* g, cudaStream_t s);
 fekf_status energy_outputs(Ctx& c, int nb, cudaStream_t s);
 fekf_status energy_error(Ctx& c, int nb, const double* e_label, double* abs_sum, cudaStream_t s);

@@ -591,7 +591,7 @@ struct SeedOut {
 __global__ void __launch_bounds__(256)
 desc_bwd_seed_kernel(Geo g, FitPtrs fp, PairPtrs pp, SeedOut so, const double* __restrict__ X,
                      const double* __restrict__ Xd, const double* __restrict__ em, const double* __restrict__ rdot,
-                     int dual, int force, double* __restrict__ Xb, double* __restrict__ Xdb) {
+                     int dual, int force, int sel, double* __restrict__ Xb, double* __restrict__ Xdb) {
   extern __shared__ double sm[];
   const int M = g.M, M2 = g.M2, Nm = g.Nm;
   double* xs = sm;               // [4][M]
@@ -650,6 +650,7 @@ desc_bwd_seed_kernel(Geo g, FitPtrs fp, PairPtrs pp, SeedOut so, const double* _
     const int* tpos = pp.tpos[p];
     for (int s = warp; s < nr; s += blockDim.x >> 5) {
       const int r = r0 + s;
+      if (sel && tpos[r] < 0) continue;   // MODE_FORCE_SEL: rows not touching the selected atoms
       const double* q = rs + (g.sec[tj] + s) * 4;
       const int t = dual ? tpos[r] : -1;
       double pk0 = 0.0, pk1 = 0.0, pk2 = 0.0, pk3 = 0.0;
@@ -1067,10 +1068,31 @@ static fekf_status layer_fwd(const Layer& L, const double* w, long long Rmax, co
   return gemm<false, false>(Rmax, L.dout, L.din, A, L.din, w + L.W, L.dout, e, s, Rdev);
 }
 
+// v = 1 on the selected atoms of every image (0 elsewhere) and the active-row sets of every pair.
+// force_error later sets v = +-1 on the same atoms, so the tangent forward reuses these row sets.
+__global__ void mark_sel_kernel(int nb, int Na, const int* __restrict__ atom_idx, int n_sel, double* __restrict__ v) {
+  for (int e = threadIdx.x; e < nb * Na * 3; e += blockDim.x) v[e] = 0.0;
+  __syncthreads();
+  for (int e = threadIdx.x; e < nb * n_sel * 3; e += blockDim.x) {
+    const int b = e / (n_sel * 3), q = (e / 3) % n_sel, al = e % 3;
+    v[((size_t)b * Na + atom_idx[q]) * 3 + al] = 1.0;
+  }
+}
+
+fekf_status mark_selected(Ctx& c, int nb, const int* atom_idx, int n_sel, cudaStream_t s) {
+  mark_sel_kernel<<<1, 1024, 0, s>>>(nb, c.Na, atom_idx, n_sel, c.vdir.as<double>());
+  FEKF_LAUNCH_CHECK();
+  count_launch();
+  FEKF_TRY(build_trows(c, nb, s));
+  c.trows_ready = true;
+  return FEKF_OK;
+}
+
 fekf_status model_forward(Ctx& c, int nb, bool tangent, cudaStream_t s) {
   const double* w = c.w.as<double>();
   Geo g = make_geo(c, nb);
-  if (tangent) FEKF_TRY(build_trows(c, nb, s));
+  if (tangent && !c.trows_ready) FEKF_TRY(build_trows(c, nb, s));
+  if (tangent) c.trows_ready = false;
   // embedding nets (compacted rows)
   const bool fused = emb_fused_ok(c);
   for (size_t p = 0; p < c.pairs.size(); ++p) {
@@ -1222,7 +1244,9 @@ fekf_status tangent_env(Ctx& c, int nb, cudaStream_t s) {
 fekf_status model_backward(Ctx& c, int nb, Mode mode, double* gout, cudaStream_t s) {
   const double* w = c.w.as<double>();
   const bool dual = mode == MODE_FORCE_JAC;
-  const bool want_w = mode != MODE_FORCE;
+  if (mode == MODE_FORCE_SEL && !emb_fused_ok(c)) mode = MODE_FORCE;   // per-layer path: every row
+  const bool force = mode == MODE_FORCE || mode == MODE_FORCE_SEL;
+  const bool want_w = !force;
   Geo g = make_geo(c, nb);
   PairPtrs pp = make_pp(c);
   FitPtrs fp = make_fp(c, nb);
@@ -1295,7 +1319,8 @@ fekf_status model_backward(Ctx& c, int nb, Mode mode, double* gout, cudaStream_t
     }
     desc_bwd_seed_kernel<<<nb * c.Na, 256, smem, s>>>(g, fp, pp, so, c.X.as<double>(), c.X.as<double>() + Xoff,
                                                       c.em.as<double>(), c.rdot.as<double>(), dual ? 1 : 0,
-                                                      mode == MODE_FORCE ? 1 : 0, c.Xb.as<double>(),
+                                                      force ? 1 : 0, mode == MODE_FORCE_SEL ? 1 : 0,
+                                                      c.Xb.as<double>(),
                                                       c.Xb.as<double>() + Xoff);
   } else {
     const size_t smem = (8 * c.M + 2 * c.M * (c.M2 + 1)) * sizeof(double);
@@ -1306,7 +1331,7 @@ fekf_status model_backward(Ctx& c, int nb, Mode mode, double* gout, cudaStream_t
   count_launch();
   // ---- embedding nets (compacted rows; tangent rows separately) ----
   if (emb_fused_ok(c)) {
-    if (mode == MODE_FORCE) {  // forces / per-atom virials accumulate inside the fused backward
+    if (force) {  // forces / per-atom virials accumulate inside the fused backward
       FEKF_CHECK_CUDA(cudaMemsetAsync(c.force.p, 0, sizeof(double) * nb * c.Na * 3, s));
       FEKF_CHECK_CUDA(cudaMemsetAsync(c.vatom.p, 0, sizeof(double) * nb * c.Na * 9, s));
     }
@@ -1368,7 +1393,7 @@ fekf_status model_backward(Ctx& c, int nb, Mode mode, double* gout, cudaStream_t
     }
   }
   }
-  if (mode == MODE_FORCE) {
+  if (force) {
     if (!emb_fused_ok(c)) {
       FEKF_CHECK_CUDA(cudaMemsetAsync(c.force.p, 0, sizeof(double) * nb * c.Na * 3, s));
       prod_force_kernel<<<nb * c.Na, 128, 0, s>>>(g, pp, c.Xb.as<double>(), c.jac.as<double>(), c.rij.as<double>(),
