@@ -510,6 +510,34 @@ fekf_status fekf_kf_create(const int32_t* block_sizes_host, int nblocks, const f
   *out = k;
   return FEKF_OK;
 }
+fekf_status fekf_kf_create_shard(const int32_t* block_sizes_host, int nblocks, const fekf_opt_cfg* opt, int world,
+                                 int rank, fekf_kf** out) {
+  if (!block_sizes_host || nblocks < 1 || !opt || !out || world < 1 || rank < 0 || rank >= world) {
+    set_error("kf_create_shard: bad args");
+    return FEKF_EINVAL;
+  }
+  for (int i = 0; i < nblocks; ++i)
+    if (block_sizes_host[i] < 1) { set_error("kf_create_shard: block size < 1"); return FEKF_EINVAL; }
+  fekf_kf* k = new fekf_kf();
+  fekf_status st = k->kf.create(std::vector<int>(block_sizes_host, block_sizes_host + nblocks), *opt, nullptr, world, rank);
+  if (st != FEKF_OK) { delete k; return st; }
+  *out = k;
+  return FEKF_OK;
+}
+fekf_status fekf_kf_update_begin(fekf_kf* k, const double* g, cudaStream_t s) {
+  if (!k || !g) { set_error("kf_update_begin: null"); return FEKF_EINVAL; }
+  return k->kf.update_begin(g, s);
+}
+fekf_status fekf_kf_partial_u(fekf_kf* k, double** u, int64_t* n) {
+  if (!k || !u || !n) { set_error("kf_partial_u: null"); return FEKF_EINVAL; }
+  *u = k->kf.ub.as<double>();
+  *n = k->kf.plan.Npad;
+  return FEKF_OK;
+}
+fekf_status fekf_kf_update_end(fekf_kf* k, const double* abe, double sqrt_bs, double* w, cudaStream_t s) {
+  if (!k || !abe || !w) { set_error("kf_update_end: null"); return FEKF_EINVAL; }
+  return k->kf.update_end(abe, sqrt_bs, w, s);
+}
 fekf_status fekf_kf_destroy(fekf_kf* k) { delete k; return FEKF_OK; }
 fekf_status fekf_kf_update(fekf_kf* k, const double* g, const double* abe, double sqrt_bs, double* w, cudaStream_t s) {
   if (!k || !g || !abe || !w) { set_error("kf_update: null"); return FEKF_EINVAL; }

@@ -578,7 +578,7 @@ static int num_sms() {
   return sms;
 }
 
-fekf_status Kf::create(const std::vector<int>& blocks, const fekf_opt_cfg& o, fekf_comm* c) {
+fekf_status Kf::create(const std::vector<int>& blocks, const fekf_opt_cfg& o, fekf_comm* c, int world_o, int rank_o) {
   opt = o;
   comm = c;
   defer = std::max(1, std::min(KMAX, o.p_defer > 0 ? o.p_defer : 1));
@@ -589,6 +589,7 @@ fekf_status Kf::create(const std::vector<int>& blocks, const fekf_opt_cfg& o, fe
   p32 = o.precision == 32;
   int world = 1, rank = 0;
   if (comm) { world = comm_world(comm); rank = comm_rank(comm); }
+  else if (world_o > 0) { world = world_o; rank = rank_o; }
   plan.build(blocks, world, rank, SEG_TILES);
   const KfPlan& p = plan;
   FEKF_TRY(dalloc(P, (size_t)p.tiles_local * TILE_ELEMS * elem() + 16));
@@ -736,10 +737,24 @@ fekf_status Kf::pass(const double* g, bool rw, cudaStream_t s) {
 // One update (Alg. 1 lines 8-13).  The stored P is rewritten only when `defer` corrections are
 // pending; otherwise the pass is read-only and the corrections are applied to u in vector form.
 fekf_status Kf::update(const double* g, const double* abe, double sqrt_bs, double* w, cudaStream_t s) {
+  FEKF_TRY(update_begin(g, s));
+  if (comm && comm_world(comm) > 1) FEKF_TRY(comm_allreduce(comm, ub.as<double>(), plan.Npad, s));
+  return update_end(abe, sqrt_bs, w, s);
+}
+
+fekf_status Kf::update_begin(const double* g, cudaStream_t s) {
+  if (in_update) { set_error("kf update_begin: previous update not ended"); return FEKF_ESTATE; }
+  cur_rw = npend >= defer;
+  FEKF_TRY(pass(g, cur_rw, s));
+  in_update = true;
+  return FEKF_OK;
+}
+
+fekf_status Kf::update_end(const double* abe, double sqrt_bs, double* w, cudaStream_t s) {
+  if (!in_update) { set_error("kf update_end: no update begun"); return FEKF_ESTATE; }
+  in_update = false;
   const KfPlan& p = plan;
-  const bool rw = npend >= defer;
-  FEKF_TRY(pass(g, rw, s));
-  if (comm && comm_world(comm) > 1) FEKF_TRY(comm_allreduce(comm, ub.as<double>(), p.Npad, s));
+  const bool rw = cur_rw;
   const int K = rw ? 0 : npend;
   kf_dot_kernel<<<cdiv(p.n_tc, 8), 256, 0, s>>>(gpad.as<double>(), ub.as<double>(), ulist.as<double>(), p.Npad, K,
                                                 p.n_tc, dotp.as<double>());

@@ -87,10 +87,15 @@ struct Kf {
   std::vector<GraphTiming*> pend_graphs;  // replayed graphs whose pairs are not harvested yet
   fekf_status harvest(std::vector<EvPair>& pairs, size_t n);   // add the elapsed times of n recorded pairs
   fekf_status harvest_graph(GraphTiming* g);
-  fekf_status create(const std::vector<int>& blocks, const fekf_opt_cfg& o, fekf_comm* c);
+  // world/rank > 0 without a communicator: shard plan of that rank, exchange of u left to the caller
+  fekf_status create(const std::vector<int>& blocks, const fekf_opt_cfg& o, fekf_comm* c, int world = 0, int rank = 0);
   ~Kf();
   fekf_status pass(const double* g, bool rw, cudaStream_t s);
   fekf_status update(const double* g, const double* abe, double sqrt_bs, double* w, cudaStream_t s);
+  // update = begin (P pass: this rank's partial u) + all-reduce of u over ranks + end (A, K, w, lambda)
+  bool in_update = false, cur_rw = false;
+  fekf_status update_begin(const double* g, cudaStream_t s);
+  fekf_status update_end(const double* abe, double sqrt_bs, double* w, cudaStream_t s);
   fekf_status flush(cudaStream_t s);
   fekf_status get_block(int b, double* dst, cudaStream_t s);
   fekf_status set_block(int b, const double* src, cudaStream_t s);

@@ -265,86 +265,8 @@ static const int* rcount(Ctx& c, int p) { return c.rowcnt.as<int>() + p; }
 static const int* tcount(Ctx& c, int p) { return c.rowcnt.as<int>() + c.pairs.size() + p; }
 
 // ---------------------------------------------------------------------------------------------
-// compaction (one CTA per pair; fixed-order scans -> deterministic row order)
+// compaction (fixed-order scans -> deterministic row order); primal rows: build_rows below
 // ---------------------------------------------------------------------------------------------
-// One CTA (32 warps) per pair: per-atom valid-slot counts by warp ballots (the sorted section is a
-// valid prefix), an exclusive scan in fixed order, then the compacted row -> slot map.
-__global__ void __launch_bounds__(1024)
-rows_kernel(Geo g, int ti, int tj, const int* __restrict__ nl_j, int* __restrict__ row_start,
-            int* __restrict__ row_idx, int* __restrict__ cnt) {
-  __shared__ int wsum[32];
-  const int E = g.nb * g.ncnt[ti];
-  const int sel = g.sel[tj];
-  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  auto base_of = [&](int e) {
-    const int b = e / g.ncnt[ti], k = e % g.ncnt[ti];
-    const int i = g.atoms[g.atoms_off[ti] + k];
-    return ((size_t)b * g.Na + i) * g.Nm + g.sec[tj];
-  };
-  // counts -> row_start[e] (temporarily)
-  for (int e0 = warp; e0 < E; e0 += 32 * 4) {
-    int c4[4];
-#pragma unroll
-    for (int u = 0; u < 4; ++u) {
-      const int e = e0 + 32 * u;
-      int c = 0;
-      if (e < E) {
-        const size_t base = base_of(e);
-        for (int s0 = 0; s0 < sel; s0 += 32) {
-          const bool v = s0 + lane < sel && nl_j[base + s0 + lane] >= 0;
-          c += __popc(__ballot_sync(0xffffffffu, v));
-        }
-      }
-      c4[u] = c;
-    }
-    if (lane == 0)
-#pragma unroll
-      for (int u = 0; u < 4; ++u)
-        if (e0 + 32 * u < E) row_start[e0 + 32 * u] = c4[u];
-  }
-  __syncthreads();
-  // exclusive scan: contiguous chunk per thread, then a block scan of the chunk sums
-  const int per = (E + 1023) / 1024;
-  const int a0 = min(E, (int)threadIdx.x * per), a1 = min(E, a0 + per);
-  int local = 0;
-  for (int e = a0; e < a1; ++e) local += row_start[e];
-  int x = local;
-#pragma unroll
-  for (int o = 1; o < 32; o <<= 1) {
-    const int y = __shfl_up_sync(0xffffffffu, x, o);
-    if (lane >= o) x += y;
-  }
-  if (lane == 31) wsum[warp] = x;
-  __syncthreads();
-  if (warp == 0) {
-    int w = wsum[lane];
-#pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-      const int y = __shfl_up_sync(0xffffffffu, w, o);
-      if (lane >= o) w += y;
-    }
-    wsum[lane] = w;
-  }
-  __syncthreads();
-  int run = x - local + (warp > 0 ? wsum[warp - 1] : 0);
-  for (int e = a0; e < a1; ++e) {
-    const int c = row_start[e];
-    row_start[e] = run;
-    run += c;
-  }
-  if (threadIdx.x == 1023) {
-    row_start[E] = wsum[31];
-    *cnt = wsum[31];
-  }
-  __syncthreads();
-  // row -> slot map
-  for (int e = warp; e < E; e += 32) {
-    const int r0 = row_start[e], n = row_start[e + 1] - r0;
-    const size_t base = base_of(e);
-    for (int s0 = lane; s0 < n; s0 += 32) row_idx[r0 + s0] = (int)(base + s0);
-  }
-}
-
 // active tangent rows: v_i != 0 or v_j != 0 (R~-dot = J (v_j - v_i) vanishes otherwise).
 // Three passes (chunk counts, chunk scan, scatter), chunks of 1024 rows, order = primal order.
 constexpr int TCHUNK = 1024;
@@ -1016,15 +938,100 @@ static FitPtrs make_fp(Ctx& c, int nb) {
   return fp;
 }
 
+// Row compaction for all pairs at once, three launches (blockIdx.y = pair): per-atom valid-slot
+// counts (a warp per centre atom, ballots over its sorted section), one CTA per pair scanning the counts
+// into row_start (fixed order: deterministic row order), then the row -> slot scatter (a warp per atom).
+struct RowsArgs {
+  int ti[NP], tj[NP];
+  int* row_start[NP];
+  int* row_idx[NP];
+  int* cnt;
+};
+__device__ __forceinline__ size_t rows_base(const Geo& g, int ti, int tj, int e) {
+  const int b = e / g.ncnt[ti], k = e % g.ncnt[ti];
+  const int i = g.atoms[g.atoms_off[ti] + k];
+  return ((size_t)b * g.Na + i) * g.Nm + g.sec[tj];
+}
+__global__ void __launch_bounds__(256) rows_count_kernel(Geo g, RowsArgs ra, const int* __restrict__ nl_j) {
+  const int p = blockIdx.y, ti = ra.ti[p], tj = ra.tj[p];
+  const int e = blockIdx.x * 8 + (threadIdx.x >> 5), lane = threadIdx.x & 31;
+  if (e >= g.nb * g.ncnt[ti]) return;
+  const size_t base = rows_base(g, ti, tj, e);
+  const int sel = g.sel[tj];
+  int c = 0;
+  for (int s0 = 0; s0 < sel; s0 += 32) c += __popc(__ballot_sync(0xffffffffu, s0 + lane < sel && nl_j[base + s0 + lane] >= 0));
+  if (lane == 0) ra.row_start[p][e] = c;
+}
+__global__ void __launch_bounds__(1024) rows_scan_kernel(Geo g, RowsArgs ra) {
+  __shared__ int wsum[32];
+  const int p = blockIdx.x, E = g.nb * g.ncnt[ra.ti[p]];
+  int* rs = ra.row_start[p];
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int per = (E + 1023) / 1024;
+  const int a0 = min(E, (int)threadIdx.x * per), a1 = min(E, a0 + per);
+  int local = 0;
+  for (int e = a0; e < a1; ++e) local += rs[e];
+  int x = local;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const int y = __shfl_up_sync(0xffffffffu, x, o);
+    if (lane >= o) x += y;
+  }
+  if (lane == 31) wsum[warp] = x;
+  __syncthreads();
+  if (warp == 0) {
+    int w = wsum[lane];
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const int y = __shfl_up_sync(0xffffffffu, w, o);
+      if (lane >= o) w += y;
+    }
+    wsum[lane] = w;
+  }
+  __syncthreads();
+  int run = x - local + (warp > 0 ? wsum[warp - 1] : 0);
+  for (int e = a0; e < a1; ++e) {
+    const int c = rs[e];
+    rs[e] = run;
+    run += c;
+  }
+  if (threadIdx.x == 1023) {
+    rs[E] = wsum[31];
+    ra.cnt[p] = wsum[31];
+  }
+}
+__global__ void __launch_bounds__(256) rows_scatter_kernel(Geo g, RowsArgs ra) {
+  const int p = blockIdx.y, ti = ra.ti[p], tj = ra.tj[p];
+  const int e = blockIdx.x * 8 + (threadIdx.x >> 5), lane = threadIdx.x & 31;
+  if (e >= g.nb * g.ncnt[ti]) return;
+  const int r0 = ra.row_start[p][e], n = ra.row_start[p][e + 1] - r0;
+  const size_t base = rows_base(g, ti, tj, e);
+  for (int s0 = lane; s0 < n; s0 += 32) ra.row_idx[p][r0 + s0] = (int)(base + s0);
+}
+
 fekf_status build_rows(Ctx& c, int nb, cudaStream_t s) {
   Geo g = make_geo(c, nb);
-  for (size_t p = 0; p < c.pairs.size(); ++p) {
+  RowsArgs ra{};
+  int emax = 0;
+  const int np = (int)c.pairs.size();
+  for (int p = 0; p < np; ++p) {
     PairNet& P = c.pairs[p];
-    rows_kernel<<<1, 1024, 0, s>>>(g, P.ti, P.tj, c.nl_j.as<int>(), P.row_start.as<int>(), P.row_idx.as<int>(),
-                                   c.rowcnt.as<int>() + p);
-    FEKF_LAUNCH_CHECK();
-    count_launch();
+    ra.ti[p] = P.ti;
+    ra.tj[p] = P.tj;
+    ra.row_start[p] = P.row_start.as<int>();
+    ra.row_idx[p] = P.row_idx.as<int>();
+    emax = std::max(emax, nb * (int)c.atoms_of[P.ti].size());
   }
+  ra.cnt = c.rowcnt.as<int>();
+  if (emax == 0) return FEKF_OK;
+  const dim3 grid(cdiv(emax, 8), np);
+  rows_count_kernel<<<grid, 256, 0, s>>>(g, ra, c.nl_j.as<int>());
+  FEKF_LAUNCH_CHECK();
+  rows_scan_kernel<<<np, 1024, 0, s>>>(g, ra);
+  FEKF_LAUNCH_CHECK();
+  rows_scatter_kernel<<<grid, 256, 0, s>>>(g, ra);
+  FEKF_LAUNCH_CHECK();
+  count_launch(3);
   return FEKF_OK;
 }
 

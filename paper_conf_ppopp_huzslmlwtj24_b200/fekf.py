@@ -59,6 +59,9 @@ def lib():
         "fekf_comm_destroy": ([vp], i32), "fekf_comm_allreduce_sum": ([vp, vp, i64, vp], i32),
         "fekf_kf_create": ([vp, i32, C.POINTER(OptCfg), vp, C.POINTER(vp)], i32), "fekf_kf_destroy": ([vp], i32),
         "fekf_kf_update": ([vp, vp, vp, dbl, vp, vp], i32), "fekf_kf_flush": ([vp, vp], i32),
+        "fekf_kf_create_shard": ([vp, i32, C.POINTER(OptCfg), i32, i32, C.POINTER(vp)], i32),
+        "fekf_kf_update_begin": ([vp, vp, vp], i32), "fekf_kf_update_end": ([vp, vp, dbl, vp, vp], i32),
+        "fekf_kf_partial_u": ([vp, C.POINTER(vp), C.POINTER(i64)], i32),
         "fekf_kf_get_block": ([vp, i32, vp, vp], i32), "fekf_kf_set_block": ([vp, i32, vp, vp], i32),
         "fekf_kf_get_state": ([vp, C.POINTER(dbl), C.POINTER(dbl), C.POINTER(i32)], i32),
         "fekf_kf_info": ([vp, C.POINTER(i64), C.POINTER(i64), C.POINTER(i64), C.POINTER(i64)], i32),
@@ -90,6 +93,7 @@ EXPORTED = [
     "fekf_last_error", "fekf_version", "fekf_plan_layout", "fekf_plan_shard", "fekf_get_unique_id",
     "fekf_comm_init", "fekf_comm_destroy", "fekf_comm_allreduce_sum", "fekf_kf_create", "fekf_kf_destroy",
     "fekf_kf_update", "fekf_kf_flush", "fekf_kf_get_block", "fekf_kf_set_block", "fekf_kf_get_state",
+    "fekf_kf_create_shard", "fekf_kf_update_begin", "fekf_kf_partial_u", "fekf_kf_update_end",
     "fekf_kf_info", "fekf_kf_pass", "fekf_kf_timing", "fekf_create", "fekf_destroy", "fekf_param_count", "fekf_get_kf",
     "fekf_set_params", "fekf_get_params", "fekf_build_nlist", "fekf_env_mat", "fekf_forward",
     "fekf_energy_jacobian", "fekf_force_jacobian", "fekf_kalman_update", "fekf_train_step",
@@ -223,7 +227,9 @@ class Comm:
 class KalmanFilter:
     """Blocked FEKF Kalman filter over packed-symmetric P (fekf_kf_*)."""
 
-    def __init__(self, blocks, opt=None, comm: Comm | None = None, _handle=None, _owner=None):
+    def __init__(self, blocks, opt=None, comm: Comm | None = None, _handle=None, _owner=None, shard=None):
+        """shard=(world, rank): this rank's P tiles with no communicator; the caller exchanges u
+        (update_begin / partial_u / update_end)."""
         self.blocks = list(blocks)
         self._owner = _owner
         if _handle is not None:
@@ -233,12 +239,34 @@ class KalmanFilter:
             self.h = C.c_void_p()
             oc = opt_cfg(opt)
             arr = (C.c_int32 * len(self.blocks))(*self.blocks)
-            _check(lib().fekf_kf_create(arr, len(self.blocks), C.byref(oc), comm.h if comm else None, C.byref(self.h)))
+            if shard is not None:
+                _check(lib().fekf_kf_create_shard(arr, len(self.blocks), C.byref(oc), int(shard[0]), int(shard[1]),
+                                                  C.byref(self.h)))
+            else:
+                _check(lib().fekf_kf_create(arr, len(self.blocks), C.byref(oc), comm.h if comm else None,
+                                            C.byref(self.h)))
             self._own = True
 
     def update(self, g, abe, sqrt_bs, w, stream=None):
         _check(lib().fekf_kf_update(self.h, _ptr(g, torch.float64, "g"), _ptr(abe, torch.float64, "abe"),
                                     float(sqrt_bs), _ptr(w, torch.float64, "w"), _stream(stream)))
+
+    def update_begin(self, g, stream=None):
+        _check(lib().fekf_kf_update_begin(self.h, _ptr(g, torch.float64, "g"), _stream(stream)))
+
+    def partial_u(self):
+        """Zero-copy view of this rank's partial u (padded layout) between update_begin and update_end."""
+        p, n = C.c_void_p(), C.c_int64()
+        _check(lib().fekf_kf_partial_u(self.h, C.byref(p), C.byref(n)))
+
+        class _View:
+            __cuda_array_interface__ = {"shape": (n.value,), "typestr": "<f8", "data": (p.value, False),
+                                        "version": 2, "strides": None}
+        return torch.as_tensor(_View(), device="cuda")
+
+    def update_end(self, abe, sqrt_bs, w, stream=None):
+        _check(lib().fekf_kf_update_end(self.h, _ptr(abe, torch.float64, "abe"), float(sqrt_bs),
+                                        _ptr(w, torch.float64, "w"), _stream(stream)))
 
     def pass_only(self, g, stream=None):
         _check(lib().fekf_kf_pass(self.h, _ptr(g, torch.float64, "g"), _stream(stream)))

@@ -279,3 +279,64 @@ def test_step_graph_matches_eager():
     assert torch.equal(out[0][0], out[1][0])
     assert all(torch.equal(a, b) for a, b in zip(out[0][1], out[1][1]))
     assert torch.equal(out[0][2], out[1][2])
+
+
+def test_rmse_trajectory_and_time_to_target():
+    """Metric (iii), minutes to target RMSE: the GPU's test-set RMSE trajectory follows the
+    oracle's stored one (tests/golden/rmse_c1_cu32.json, written by tools/make_rmse_target.py from the
+    oracle alone) within rel 1e-6 and reaches the oracle's S_o target by step S_o."""
+    import json
+    import os
+    import sys
+    sys.path.insert(0, os.path.join(os.path.dirname(os.path.dirname(__file__)), "tools"))
+    import time_to_rmse
+    gold = json.load(open(os.path.join(os.path.dirname(__file__), "golden", "rmse_c1_cu32.json")))
+    out = time_to_rmse.run("c1_cu32", gold["S_o"], gold["every"], stop_at_target=False)
+    assert out["flags"] == 0
+    assert [s for s, _, _ in out["trajectory"]] == [s for s, _, _ in gold["trajectory"]]
+    assert out["max_rel_dev_vs_oracle"] < 1e-6
+    assert out["reached"] is not None and out["reached"]["step"] == gold["target_step"]
+
+
+@pytest.mark.parametrize("world", [2, 3])
+@pytest.mark.parametrize("precision", [64, 32])
+def test_kalman_sharded_ranks(world, precision):
+    """P sharded over `world` ranks (north_star; fekf_plan_shard tile-row segments) run in one process:
+    each rank's filter streams only its own tiles, the partial u's are summed (the all-reduce the NCCL
+    path does), and the weights and every block of P match the fp64 oracle after updates that cross
+    read-write passes (rel 1e-12; fp32 P storage rel 1e-4)."""
+    rng = np.random.default_rng(5)
+    blocks = [5, 70, 130, 200, 64]
+    opt = dict(lambda0=0.98, nu=0.9987, block_size=1024, noise_mode=0, p_defer=3, precision=precision)
+    kfs = [fk.KalmanFilter(blocks, opt, shard=(world, r)) for r in range(world)]
+    tiles = [kf.info()["tiles_local"] for kf in kfs]
+    assert sum(tiles) == sum((x + 1) * x // 2 for x in [(n + 63) // 64 for n in blocks]) and min(tiles) > 0
+    N = sum(blocks)
+    st = O.FEKF(np.zeros(N), blocks, lam=0.98, nu=0.9987, noise_mode=0)
+    st.P = [_rand_spd(rng, n) for n in blocks]
+    for kf in kfs:
+        for b, P in enumerate(st.P):
+            kf.set_block(b, cu(P))
+    ws = [torch.zeros(N, dtype=torch.float64, device="cuda") for _ in range(world)]
+    for it in range(9):
+        g = rng.standard_normal(N)
+        abe = float(rng.uniform(0.01, 1.0))
+        gd, ad = cu(g), cu([abe])
+        for kf in kfs:
+            kf.update_begin(gd)
+        us = [kf.partial_u() for kf in kfs]
+        tot = torch.stack(us).sum(0)
+        for u in us:
+            u.copy_(tot)
+        for kf, w in zip(kfs, ws):
+            kf.update_end(ad, 3.0, w)
+        st.update(g, abe, 9)
+    torch.cuda.synchronize()
+    tol = 1e-12 if precision == 64 else 1e-4
+    for w in ws:
+        assert rel(w.cpu(), st.w) < tol
+    for b, n in enumerate(blocks):
+        full = torch.zeros(n, n, dtype=torch.float64, device="cuda")
+        for kf in kfs:
+            kf.get_block(b, out=full)           # each rank fills its own tiles (both triangles)
+        assert rel(full.cpu(), st.P[b]) < tol

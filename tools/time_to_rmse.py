@@ -1,0 +1,128 @@
+#!/usr/bin/env python
+"""Minutes to target RMSE (BASELINE.json metric (iii)): FEKF training on the GPU through the
+C ABI until the test-set RMSE (E_rmse per atom + F_rmse per component) reaches the target.
+
+  python tools/time_to_rmse.py [--config c1_cu32] [--max-steps 200] [--every 8] [--target X]
+
+The target defaults to tests/golden/rmse_<config>.json (written by tools/make_rmse_target.py from the
+fp64 CPU oracle alone): the best RMSE the oracle reached within S_o steps from the same initial weights
+on the same minibatch / force-atom schedule.  Training time is measured on the device (CUDA events around the train
+steps only); evaluation (forward on the test split every `--every` steps) is timed separately.  Without a
+golden file (e.g. water-64, whose oracle P does not fit a host), `--target` or the GPU's own trajectory
+is reported, unpinned.  Prints one JSON line.
+"""
+import argparse
+import json
+import math
+import os
+import sys
+import time
+
+import numpy as np
+import torch
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+import paper_conf_ppopp_huzslmlwtj24_b200 as fk  # noqa: E402
+from fixtures import get_config, make_dataset, init_weights, batch_schedule, force_groups  # noqa: E402
+
+
+def run(config, max_steps, every, target=None, precision=64, stop_at_target=True):
+    wl = get_config(config)
+    m = wl.model
+    opt = type(wl.opt)(**{**wl.opt.__dict__, "precision": precision})
+    gold_path = os.path.join(ROOT, "tests", "golden", f"rmse_{config}.json")
+    gold = json.load(open(gold_path)) if os.path.exists(gold_path) else None
+    if target is None and gold is not None:
+        target = gold["target"]
+    tr = make_dataset(config, split="train")
+    te = make_dataset(config, split="test")
+    na = len(tr["types"])
+    B = wl.batch
+    w0 = init_weights(m, 3, float(tr["energy"].mean() / na))
+    dev = lambda x, dt=torch.float64: torch.as_tensor(np.ascontiguousarray(x)).to(dt).cuda()
+    ctx = fk.Context(m, opt, types=tr["types"], local_batch=B, global_batch=B)
+    ctx.set_params(dev(w0))
+    # the whole training and test sets resident in HBM; minibatches gathered by index on the device
+    X, BX, E, F = dev(tr["coord"]), dev(tr["box"]), dev(tr["energy"]), dev(tr["force"])
+    tX, tB = dev(te["coord"]), dev(te["box"])
+    tE, tF = dev(te["energy"]), dev(te["force"])
+    nte = len(te["energy"])
+    metrics = torch.zeros(8, dtype=torch.float64, device="cuda")
+
+    def evaluate():
+        es, fs = [], []
+        for a in range(0, nte, B):
+            n = min(B, nte - a)
+            _, e, f, _ = ctx.forward(tX[a:a + n], tB[a:a + n])
+            es.append(e[:n])
+            fs.append(f[:n])
+        e = torch.cat(es)
+        f = torch.cat(fs)
+        er = math.sqrt(float((((e - tE) / na) ** 2).mean()))
+        fr = math.sqrt(float(((f - tF) ** 2).mean()))
+        return er, fr
+
+    traj = [[0, *evaluate()]]
+    train_ms = 0.0
+    eval_s = 0.0
+    reached = None
+    step = 0
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    while step < max_steps:
+        n = min(every, max_steps - step)
+        idx = [torch.as_tensor(batch_schedule(wl.n_train, B, step + k, wl.seed)).cuda() for k in range(n)]
+        grp = [dev(force_groups(na, step + k, wl.seed, opt.force_groups, opt.atoms_per_group), torch.int32)
+               for k in range(n)]
+        bat = [(X[i].contiguous(), BX[i].contiguous(), E[i].contiguous(), F[i].contiguous()) for i in idx]
+        torch.cuda.synchronize()
+        e0.record()
+        for k in range(n):
+            ctx.train_step(*bat[k], grp[k], metrics)
+        e1.record()
+        torch.cuda.synchronize()
+        train_ms += e0.elapsed_time(e1)
+        step += n
+        t1 = time.perf_counter()
+        er, fr = evaluate()
+        eval_s += time.perf_counter() - t1
+        traj.append([step, er, fr])
+        # reached: at or below the target, which matches the oracle only up to rounding (rel 1e-6)
+        if target is not None and reached is None and er + fr <= target * (1.0 + 1e-6):
+            reached = {"step": step, "train_s": train_ms / 1000.0}
+            if stop_at_target:
+                break
+    flags = int(metrics[7].item())
+    ctx.close()
+    out = {"metric": "minutes to target RMSE", "config": config, "precision": precision, "target": target,
+           "target_source": ("oracle S_o=%d (tests/golden/rmse_%s.json)" % (gold["S_o"], config)) if gold and
+           target == gold["target"] else ("given" if target is not None else None),
+           "reached": reached, "minutes_to_target": reached["train_s"] / 60.0 if reached else None,
+           "steps_run": step, "train_s": train_ms / 1000.0, "ms_per_step": train_ms / max(step, 1),
+           "eval_s": eval_s, "final_rmse": traj[-1][1] + traj[-1][2], "trajectory": traj, "flags": flags}
+    if gold is not None:
+        g = {s: (e, f) for s, e, f in gold["trajectory"]}
+        common = [(s, e, f) for s, e, f in traj if s in g]
+        out["max_rel_dev_vs_oracle"] = max(
+            (max(abs(e - g[s][0]) / g[s][0], abs(f - g[s][1]) / g[s][1]) for s, e, f in common), default=None)
+        out["oracle_train_s_for_S_o"] = gold.get("oracle_train_seconds")
+        # the oracle's own time to the same target (its per-step time on the host that wrote the file)
+        out["oracle_minutes_to_target"] = gold["oracle_train_seconds"] * gold["target_step"] / gold["S_o"] / 60.0
+        out["oracle_threads"] = gold.get("oracle_threads")
+    return out
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--config", default="c1_cu32")
+    ap.add_argument("--max-steps", type=int, default=200)
+    ap.add_argument("--every", type=int, default=8)
+    ap.add_argument("--target", type=float, default=None)
+    ap.add_argument("--precision", type=int, default=64, choices=[64, 32])
+    ap.add_argument("--full", action="store_true", help="keep training after the target (trajectory)")
+    a = ap.parse_args()
+    print(json.dumps(run(a.config, a.max_steps, a.every, a.target, a.precision, not a.full)), flush=True)
+
+
+if __name__ == "__main__":
+    main()
