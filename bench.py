@@ -289,11 +289,12 @@ def run_fekf(args, rank, world, local):
         try:
             with open(prof) as f:
                 pj = json.load(f)
-            if pj.get("workload") == args.config and world == 1 and pj.get("precision", 64) == args.precision:
-                # DRAM bytes per launch from one ncu --set full capture, blended over the read-only and
-                # read-write launches of this run (a read-write pass moves twice the read-only bytes)
-                ro = pj["ro_dram_bytes_per_launch"] / pj["ro_alg_bytes_per_launch"]
-                rwr = pj["rw_traffic_over_alg"]
+            pp = pj.get("by_precision", {}).get(str(args.precision))
+            if pj.get("workload") == args.config and world == 1 and pp:
+                # DRAM bytes per launch from ncu captures, scaled to this run's algorithmic bytes and blended
+                # over its read-only / read-write launches
+                ro = pp["ro_dram_bytes_per_launch"] / pp["ro_alg_bytes_per_launch"]
+                rwr = pp["rw_dram_bytes_per_launch"] / pp["rw_alg_bytes_per_launch"]
                 traffic = (stream * ro * (pass_n - pass_rw) + 2 * stream * rwr * pass_rw) / pass_n
         except Exception:
             pass

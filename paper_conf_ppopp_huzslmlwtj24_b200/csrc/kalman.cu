@@ -27,7 +27,8 @@ namespace fekf {
 // ------------------------------------------------------------------------------------------------
 // host planner
 // ------------------------------------------------------------------------------------------------
-void KfPlan::build(const std::vector<int>& blocks, int world_, int rank_, int seg_tiles) {
+void KfPlan::build(const std::vector<int>& blocks, int world_, int rank_, int seg_tiles, int row_slots) {
+  rps = row_slots;
   n = blocks;
   L = (int)n.size();
   world = world_;
@@ -86,10 +87,10 @@ void KfPlan::build(const std::vector<int>& blocks, int world_, int rank_, int se
   tiles_local = tile_off;
   const int64_t n_items = (int64_t)items.size();
   for (int64_t k = 0; k < n_items; ++k) {
-    items[k].row_slot = (int)k;
-    items[k].col_slot0 = (long long)(n_items + items[k].tile_off);
+    items[k].row_slot = (int)k;   // slots row_slot*rps .. +rps-1
+    items[k].col_slot0 = (long long)(rps * n_items + items[k].tile_off);
   }
-  ws_slots = n_items + tiles_local;
+  ws_slots = rps * n_items + tiles_local;
   // per-tile owner in canonical packed order (for fekf_plan_shard)
   tile_owner.clear();
   tile_owner.reserve(total_tiles);
@@ -100,7 +101,7 @@ void KfPlan::build(const std::vector<int>& blocks, int world_, int rank_, int se
   std::vector<std::vector<std::pair<long long, long long>>> rows(n_tc), cols(n_tc);
   for (int64_t k = 0; k < n_items; ++k) {
     const ItemD& d = items[k];
-    rows[tc_off[d.blk] + d.I].push_back({d.J0, d.row_slot});
+    for (int g = 0; g < rps; ++g) rows[tc_off[d.blk] + d.I].push_back({(long long)d.J0 * rps + g, (long long)d.row_slot * rps + g});
     for (int t = 0; t < d.nJ; ++t) {
       int J = d.J0 + t;
       if (J == d.I) continue;
@@ -177,6 +178,7 @@ __device__ __forceinline__ void consumer_bar() { asm volatile("bar.sync 1, 256;"
 // ------------------------------------------------------------------------------------------------
 constexpr int MAX_STAGES = 12;
 constexpr int TILE_ELEMS = KT * KT;
+constexpr int VS = KT + 8;   // SMEM stride of the correction vectors: DMMA fragment loads at the 2-wavefront minimum
 
 // Storage element of P: fp64 (default) or fp32 (the fp32 variant, reading Z22).  A lane handles two
 // adjacent columns of a tile row; values are widened to fp64 for every product and correction.
@@ -196,18 +198,68 @@ constexpr size_t PASS_SMEM = 227 * 1024 - 256;  // + 128 B of static shared memo
 // columns J) it needs.
 constexpr size_t PASS_HDR = 2 * MAX_STAGES * sizeof(uint64_t) + MAX_STAGES * sizeof(int4) + 2 * 8 * KT * sizeof(double);
 
+// Deferred corrections of one tile on the FP64 tensor path: C = (beta o U_I) U_J^T, a [64 x K] x [K x 64]
+// product (K <= 16, zero-padded to a multiple of 4) done as m8n8k4 DMMAs, each warp owning 8-row strips;
+// then B <- sigma (B - C) in place in the stage.  A scalar k-loop issued ~10 shared loads per 16 FMAs and
+// made a read-write pass with 15 pending corrections compute-bound (18 ms fp64 / 27 ms fp32 for
+// water-64's 41 / 21 GB instead of the 12.3 / 6.3 ms of its traffic).
+__device__ __forceinline__ void dmma884k(double& d0, double& d1, double a, double b) {
+  asm volatile("mma.sync.aligned.m8n8k4.row.col.f64.f64.f64.f64 {%0,%1}, {%2}, {%3}, {%0,%1};"
+               : "+d"(d0), "+d"(d1)
+               : "d"(a), "d"(b));
+}
+template <typename PT, int NSTRIP>
+__device__ __forceinline__ void apply_corrections(PT* t, const double* vI, const double* vJ, const double* s_beta,
+                                                  int K, double sig, int strip0, int lane) {
+  const int fr = lane >> 2, fk = lane & 3;
+#pragma unroll
+  for (int sp = 0; sp < NSTRIP; ++sp) {
+    const int m0 = 8 * (strip0 + sp);
+    double c[8][2];
+#pragma unroll
+    for (int j = 0; j < 8; ++j) c[j][0] = c[j][1] = 0.0;
+    for (int k0 = 0; k0 < K; k0 += 4) {
+      const int k = k0 + fk;
+      const bool kv = k < K;
+      const double a = kv ? s_beta[k] * vI[k * VS + m0 + fr] : 0.0;
+      double b[8];
+#pragma unroll
+      for (int j = 0; j < 8; ++j) b[j] = kv ? vJ[k * VS + 8 * j + fr] : 0.0;
+#pragma unroll
+      for (int j = 0; j < 8; ++j) dmma884k(c[j][0], c[j][1], a, b[j]);
+    }
+    PT* row = t + (m0 + fr) * KT + 2 * fk;
+#pragma unroll
+    for (int j = 0; j < 8; ++j) {
+      double2 v = ld2(row + 8 * j);
+      v.x = sig * (v.x - c[j][0]);
+      v.y = sig * (v.y - c[j][1]);
+      st2(row + 8 * j, v);
+    }
+  }
+}
+
 // rw = 0: read-only pass, u_B = B g.  rw = 1: B <- sigma (B - sum_{k<K} beta_k u_k u_k^T) written back,
 // then u_B = B_new g.  Tile-row segments are pulled from an atomic counter by a producer warp that
-// streams each 32 KiB tile (and, for rw, the 2K 512-byte vector segments it needs) with TMA bulk copies
-// into a ring of `nst` stages (fp64: 6 for read-only passes, fewer when corrections ride along; fp32
-// tiles are 16 KiB, so twice as many).  `stage_bytes` = tile bytes + (1 + 2K)*T*8: the tile, its g_J
-// segment and the 2K correction segments.
-template <typename PT>
+// streams each tile (and its g_J segment, and for rw the 2K 512-byte vector segments it needs) with TMA
+// bulk copies into a ring of `nst` stages (fp64: 6 for read-only passes, fewer when corrections ride
+// along; fp32 tiles are 16 KiB, so twice as many).  `stage_bytes` = tile bytes + (T + 2K*VS)*8.
+//
+// The 8 consumer warps form NG independent groups of 8/NG warps (named barrier 1 + group); group g
+// takes the stages s = g (mod NG), so NG tiles are in flight in the consumers at once.  fp64 uses one
+// group (a 32 KiB tile leaves enough time per tile); fp32 uses two: with a 16 KiB tile the per-tile
+// latency chain (stage wait, loads, conversions, FMA chains, barrier, column reduction) of a single group
+// no longer fits in the tile's HBM time.  Row partials: NG slots per item (a group flushes its share at
+// its last tile of the item; an item shorter than NG tiles zeroes the slots of the groups it skips).
+template <typename PT, int NG>
 __global__ void __launch_bounds__(PASS_THREADS, 1)
 kf_pass_kernel(PT* __restrict__ P, const ItemD* __restrict__ items, int n_items, int* counter,
                const double* __restrict__ gpad, const double* __restrict__ ulist, long long npad, int rw, int K,
                int nst, int stage_bytes, const KfState* st, double* __restrict__ ws) {
   constexpr uint32_t TILE_BYTES = TILE_ELEMS * sizeof(PT);
+  constexpr int NGW = 8 / NG;            // warps per group
+  constexpr int RPW = KT / NGW;          // rows per warp and tile
+  constexpr int GT = NGW * 32;           // threads per group
   extern __shared__ __align__(128) unsigned char smem[];
   uint64_t* full = reinterpret_cast<uint64_t*>(smem);
   uint64_t* empty = full + MAX_STAGES;
@@ -231,14 +283,15 @@ kf_pass_kernel(PT* __restrict__ P, const ItemD* __restrict__ items, int n_items,
     if (lane == 0) {
       int s = 0;
       uint32_t ph = 0;
-      const uint32_t bytes = TILE_BYTES + (1u + 2u * (uint32_t)K) * KT * sizeof(double);
+      const uint32_t bytes = TILE_BYTES + (1u + 2u * (uint32_t)K) * KT * sizeof(double);   // bytes landed
       while (true) {
         const int itx = atomicAdd(counter, 1);
         if (itx >= n_items) break;
         const ItemD it = items[itx];
         for (int t = 0; t < it.nJ; ++t) {
           mbar_wait(&empty[s], ph ^ 1);
-          meta[s] = make_int4(itx, it.J0 + t, (t == 0 ? 1 : 0) | (t == it.nJ - 1 ? 2 : 0), 0);
+          // flags: 1 first tile of the item for its group, 2 last one, 4 item shorter than NG tiles
+          meta[s] = make_int4(itx, it.J0 + t, (t < NG ? 1 : 0) | (t >= it.nJ - NG ? 2 : 0) | (it.nJ < NG ? 4 : 0), 0);
           unsigned char* st_s = stages + (size_t)s * stage_bytes;
           double* st_g = reinterpret_cast<double*>(st_s + TILE_BYTES);
           double* st_v = st_g + KT;
@@ -248,15 +301,18 @@ kf_pass_kernel(PT* __restrict__ P, const ItemD* __restrict__ items, int n_items,
           tma_load_1d(st_g, gpad + it.vbase + (size_t)(it.J0 + t) * KT, KT * sizeof(double), &full[s]);
           for (int k = 0; k < K; ++k) {
             const double* uk = ulist + (size_t)k * npad + it.vbase;
-            tma_load_1d(st_v + k * KT, uk + (size_t)it.I * KT, KT * sizeof(double), &full[s]);
-            tma_load_1d(st_v + (K + k) * KT, uk + (size_t)(it.J0 + t) * KT, KT * sizeof(double), &full[s]);
+            tma_load_1d(st_v + k * VS, uk + (size_t)it.I * KT, KT * sizeof(double), &full[s]);
+            tma_load_1d(st_v + (K + k) * VS, uk + (size_t)(it.J0 + t) * KT, KT * sizeof(double), &full[s]);
           }
           if (++s == nst) { s = 0; ph ^= 1; }
         }
       }
-      mbar_wait(&empty[s], ph ^ 1);
-      meta[s] = make_int4(-1, 0, 0, 0);
-      mbar_arrive(&full[s]);
+      for (int g = 0; g < NG; ++g) {  // one end marker per consumer group
+        mbar_wait(&empty[s], ph ^ 1);
+        meta[s] = make_int4(-1, 0, 0, 0);
+        mbar_arrive(&full[s]);
+        if (++s == nst) { s = 0; ph ^= 1; }
+      }
     }
     return;
   }
@@ -265,14 +321,16 @@ kf_pass_kernel(PT* __restrict__ P, const ItemD* __restrict__ items, int n_items,
   __shared__ double s_beta[KMAX];
   if (tid < KMAX) s_beta[tid] = tid < K ? st->beta[tid] : 0.0;
   asm volatile("bar.sync 1, 256;" ::: "memory");  // consumer warps only
+  const int gi = warp / NGW, wg = warp % NGW, tg = tid - gi * GT;
   const double sig = st->sigma;
   const int c0 = 2 * lane;
-  double gI[8], racc[8];
+  double gI[RPW], racc[RPW];
 #pragma unroll
-  for (int k = 0; k < 8; ++k) { gI[k] = 0.0; racc[k] = 0.0; }
-  int s = 0, prev_s = -1;
+  for (int k = 0; k < RPW; ++k) { gI[k] = 0.0; racc[k] = 0.0; }
+  int s = gi, prev_s = -1;
   uint32_t ph = 0;
   uint32_t tcount = 0;
+  double* colg = colred + gi * (2 * NGW * KT);
   while (true) {
     mbar_wait(&full[s], ph);
     const int4 mt = meta[s];
@@ -282,8 +340,8 @@ kf_pass_kernel(PT* __restrict__ P, const ItemD* __restrict__ items, int n_items,
     const bool first = mt.z & 1, last = mt.z & 2, diag = (J == it.I);
     if (first) {
 #pragma unroll
-      for (int k = 0; k < 8; ++k) {
-        gI[k] = __ldg(gpad + it.vbase + (long long)it.I * KT + warp + 8 * k);
+      for (int k = 0; k < RPW; ++k) {
+        gI[k] = __ldg(gpad + it.vbase + (long long)it.I * KT + wg + NGW * k);
         racc[k] = 0.0;
       }
     }
@@ -291,47 +349,33 @@ kf_pass_kernel(PT* __restrict__ P, const ItemD* __restrict__ items, int n_items,
     const double* vg = reinterpret_cast<const double*>(t + TILE_ELEMS);
     const double2 gJ = *reinterpret_cast<const double2*>(vg + c0);
     const double* vI = vg + KT;
-    const double* vJ = vI + K * KT;
+    const double* vJ = vI + K * VS;
     double ca0 = 0.0, ca1 = 0.0;
-    double2 v[8];
-#pragma unroll
-    for (int q = 0; q < 8; ++q) v[q] = ld2(t + (warp + 8 * q) * KT + c0);
     if (rw) {
-      // sum_k beta_k u_k[r] u_k[c] for this lane's rows r and columns c, k outermost (u_k[c] loaded once)
-      double2 cc[8];
+      // B <- sigma (B - C) on the tensor path, 8-row strips per warp; then the group re-reads the
+      // rewritten tile (u_B = B_new g with B_new as stored) in its own element layout
+      apply_corrections<PT, RPW / 8>(t, vI, vJ, s_beta, K, sig, wg * (RPW / 8), lane);
+      asm volatile("bar.sync %0, %1;" ::"r"(1 + gi), "r"(GT) : "memory");
+    }
 #pragma unroll
-      for (int q = 0; q < 8; ++q) cc[q] = make_double2(0.0, 0.0);
-      for (int k = 0; k < K; ++k) {
-        const double2 uj = *reinterpret_cast<const double2*>(vJ + k * KT + c0);
-        const double bk = s_beta[k];
+    for (int h = 0; h < RPW / 8; ++h) {
+      double2 v[8];
 #pragma unroll
-        for (int q = 0; q < 8; ++q) {
-          const double bu = bk * vI[k * KT + warp + 8 * q];
-          cc[q].x = fma(bu, uj.x, cc[q].x);
-          cc[q].y = fma(bu, uj.y, cc[q].y);
-        }
-      }
+      for (int q = 0; q < 8; ++q) v[q] = ld2(t + (wg + NGW * (8 * h + q)) * KT + c0);
 #pragma unroll
       for (int q = 0; q < 8; ++q) {
-        v[q].x = sig * (v[q].x - cc[q].x);
-        v[q].y = sig * (v[q].y - cc[q].y);
-        st2(t + (warp + 8 * q) * KT + c0, v[q]);
-        if constexpr (sizeof(PT) == 4) v[q] = ld2(t + (warp + 8 * q) * KT + c0);  // u_B = B_new g, B_new as stored
+        racc[8 * h + q] = fma(v[q].x, gJ.x, fma(v[q].y, gJ.y, racc[8 * h + q]));
+        ca0 = fma(v[q].x, gI[8 * h + q], ca0);
+        ca1 = fma(v[q].y, gI[8 * h + q], ca1);
       }
     }
-#pragma unroll
-    for (int q = 0; q < 8; ++q) {
-      racc[q] = fma(v[q].x, gJ.x, fma(v[q].y, gJ.y, racc[q]));
-      ca0 = fma(v[q].x, gI[q], ca0);
-      ca1 = fma(v[q].y, gI[q], ca1);
-    }
-    double* cr = colred + (tcount & 1) * (8 * KT);
+    double* cr = colg + (tcount & 1) * (NGW * KT);
     if (!diag) {
-      cr[warp * KT + c0] = ca0;
-      cr[warp * KT + c0 + 1] = ca1;
+      cr[wg * KT + c0] = ca0;
+      cr[wg * KT + c0 + 1] = ca1;
     }
-    consumer_bar();
-    if (tid == 0) {
+    asm volatile("bar.sync %0, %1;" ::"r"(1 + gi), "r"(GT) : "memory");
+    if (tg == 0) {
       if (rw) {
         fence_proxy_async();
         tma_store_1d(P + (size_t)(it.tile_off + (J - it.J0)) * TILE_ELEMS, t, TILE_BYTES);
@@ -342,28 +386,34 @@ kf_pass_kernel(PT* __restrict__ P, const ItemD* __restrict__ items, int n_items,
         }
         prev_s = s;
       } else {
-        mbar_arrive(&empty[s]);  // read-only: the stage is free once every consumer passed the barrier
+        mbar_arrive(&empty[s]);  // read-only: the stage is free once every consumer of the group passed
       }
     }
-    if (!diag && tid < KT) {
+    if (!diag && tg < KT) {
       double a = 0.0;
 #pragma unroll
-      for (int w = 0; w < 8; ++w) a += cr[w * KT + tid];
-      ws[(size_t)(it.col_slot0 + (J - it.J0)) * KT + tid] = a;
+      for (int w = 0; w < NGW; ++w) a += cr[w * KT + tg];
+      ws[(size_t)(it.col_slot0 + (J - it.J0)) * KT + tg] = a;
     }
     if (last) {
+      double* rs = ws + ((size_t)it.row_slot * NG + gi) * KT;
 #pragma unroll
-      for (int q = 0; q < 8; ++q) {
+      for (int q = 0; q < RPW; ++q) {
         double v = racc[q];
 #pragma unroll
         for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
-        if (lane == 0) ws[(size_t)it.row_slot * KT + warp + 8 * q] = v;
+        if (lane == 0) rs[wg + NGW * q] = v;
+      }
+      if (NG > 1 && (mt.z & 4) && tg < KT) {   // the other groups never see this item
+        for (int g = 0; g < NG; ++g)
+          if (g != gi) ws[((size_t)it.row_slot * NG + g) * KT + tg] = 0.0;
       }
     }
-    if (++s == nst) { s = 0; ph ^= 1; }
+    s += NG;
+    if (s >= nst) { s -= nst; ph ^= 1; }
     ++tcount;
   }
-  if (tid == 0) {
+  if (tg == 0) {
     if (prev_s >= 0) {
       bulk_wait_read<0>();
       mbar_arrive(&empty[prev_s]);
@@ -590,7 +640,8 @@ fekf_status Kf::create(const std::vector<int>& blocks, const fekf_opt_cfg& o, fe
   int world = 1, rank = 0;
   if (comm) { world = comm_world(comm); rank = comm_rank(comm); }
   else if (world_o > 0) { world = world_o; rank = rank_o; }
-  plan.build(blocks, world, rank, SEG_TILES);
+  ng = p32 ? 2 : 1;   // fp64: one group (measured: a second group slows the read-write pass)
+  plan.build(blocks, world, rank, SEG_TILES, ng);
   const KfPlan& p = plan;
   FEKF_TRY(dalloc(P, (size_t)p.tiles_local * TILE_ELEMS * elem() + 16));
   FEKF_TRY(dalloc(items_d, std::max<size_t>(1, p.items.size()) * sizeof(ItemD)));
@@ -627,8 +678,8 @@ fekf_status Kf::create(const std::vector<int>& blocks, const fekf_opt_cfg& o, fe
   s.c_mult = o.noise_mode == 0 ? (double)p.L : 1.0;
   FEKF_CHECK_CUDA(cudaMemcpy(state.p, &s, sizeof(KfState), cudaMemcpyHostToDevice));
   FEKF_CHECK_CUDA(cudaMemset(ulist.p, 0, (size_t)KMAX * p.Npad * sizeof(double)));
-  FEKF_CHECK_CUDA(cudaFuncSetAttribute(kf_pass_kernel<double>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)PASS_SMEM));
-  FEKF_CHECK_CUDA(cudaFuncSetAttribute(kf_pass_kernel<float>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)PASS_SMEM));
+  FEKF_CHECK_CUDA(cudaFuncSetAttribute(kf_pass_kernel<double, 1>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)PASS_SMEM));
+  FEKF_CHECK_CUDA(cudaFuncSetAttribute(kf_pass_kernel<float, 2>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)PASS_SMEM));
   if (!p.items.empty()) {
     if (p32) kf_init_kernel<<<(unsigned)p.items.size(), 256>>>(P.as<float>(), items_d.as<ItemD>(), n_d.as<int>());
     else kf_init_kernel<<<(unsigned)p.items.size(), 256>>>(P.as<double>(), items_d.as<ItemD>(), n_d.as<int>());
@@ -712,14 +763,15 @@ fekf_status Kf::pass(const double* g, bool rw, cudaStream_t s) {
       FEKF_CHECK_CUDA(cudaEventRecordWithFlags(tp->a, s, capturing ? cudaEventRecordExternal : cudaEventRecordDefault));
     }
     const int K = rw ? npend : 0;
-    const int stage_bytes = (int)(TILE_ELEMS * elem() + (1 + 2 * K) * KT * sizeof(double));
-    const int nst = (int)std::min<size_t>(MAX_STAGES, (PASS_SMEM - PASS_HDR) / stage_bytes);
+    const int stage_bytes = (int)(TILE_ELEMS * elem() + (KT + 2 * K * VS) * sizeof(double));
+    int nst = (int)std::min<size_t>(MAX_STAGES, (PASS_SMEM - PASS_HDR) / stage_bytes);
+    if (ng == 2) nst &= ~1;   // two consumer groups alternate stages
     if (p32)
-      kf_pass_kernel<float><<<grid, PASS_THREADS, PASS_SMEM, s>>>(
+      kf_pass_kernel<float, 2><<<grid, PASS_THREADS, PASS_SMEM, s>>>(
           P.as<float>(), items_d.as<ItemD>(), (int)p.items.size(), counter.as<int>(), gpad.as<double>(),
           ulist.as<double>(), p.Npad, rw ? 1 : 0, K, nst, stage_bytes, state.as<KfState>(), ws.as<double>());
     else
-      kf_pass_kernel<double><<<grid, PASS_THREADS, PASS_SMEM, s>>>(
+      kf_pass_kernel<double, 1><<<grid, PASS_THREADS, PASS_SMEM, s>>>(
           P.as<double>(), items_d.as<ItemD>(), (int)p.items.size(), counter.as<int>(), gpad.as<double>(),
           ulist.as<double>(), p.Npad, rw ? 1 : 0, K, nst, stage_bytes, state.as<KfState>(), ws.as<double>());
     FEKF_LAUNCH_CHECK();

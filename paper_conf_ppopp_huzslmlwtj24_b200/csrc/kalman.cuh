@@ -42,7 +42,8 @@ struct KfPlan {
   std::vector<int> owner;             // owner rank of every canonical item
   std::vector<int> tile_owner;        // owner rank of every tile, canonical packed order
   std::vector<long long> csr_ptr, csr_idx;
-  void build(const std::vector<int>& blocks, int world, int rank, int seg_tiles);
+  int rps = 1;                        // row-partial slots per item (consumer groups of the P pass)
+  void build(const std::vector<int>& blocks, int world, int rank, int seg_tiles, int row_slots = 1);
 };
 
 // communicator helpers (comm.cu)
@@ -69,6 +70,7 @@ struct Kf {
   int defer = 1;                 // corrections deferred before P is rewritten (1 = rewrite every update)
   int npend = 0;                 // host mirror of the device npend
   bool p32 = false;              // P stored fp32 (opt.precision == 32, reading Z22)
+  int ng = 1;                    // consumer groups of the P pass
   size_t elem() const { return p32 ? sizeof(float) : sizeof(double); }
   DBuf P, items_d, ws, gpad, ub, ulist, dotp, csr_ptr, csr_idx, tc_blk, tc_c, off_d, n_d, state, counter;
   DBuf tcoff_d, dblk, cub;       // block -> tile-column offsets, per-block dots, per-block coefficients

@@ -245,8 +245,8 @@ def test_train_steps(name, steps, precision):
 
 
 def test_step_graph_matches_eager():
-    """a10: the captured step graph (default) and eager launches give bit-identical weights, P and
-    metrics across graph variants (p_defer 2: read-write passes at different updates of a step), and
+    """a10: the captured step graph (default) and eager launches give the same weights, P and metrics
+    (up to the order of the force-scatter atomics) across graph variants (p_defer 2: read-write passes at different updates of a step), and
     the live P-pass timing sees every pass inside replayed graphs."""
     wl = get_config("t2_tiny")
     m = wl.model
@@ -276,9 +276,11 @@ def test_step_graph_matches_eager():
         out.append((ctx.get_params().cpu(), [ctx.kf.get_block(b).cpu() for b in range(len(ctx.kf.blocks))],
                     torch.stack(mets).cpu()))
         ctx.close()
-    assert torch.equal(out[0][0], out[1][0])
-    assert all(torch.equal(a, b) for a, b in zip(out[0][1], out[1][1]))
-    assert torch.equal(out[0][2], out[1][2])
+    # same kernels in the same order; the only run-to-run freedom is the order of the fp64 atomics of the
+    # force scatter (F_i += f, F_j -= f), which can move a force, hence an ABE_F, by an ulp
+    assert rel(out[0][0], out[1][0]) < 1e-13
+    assert all(rel(a, b) < 1e-13 for a, b in zip(out[0][1], out[1][1]))
+    assert rel(out[0][2], out[1][2]) < 1e-13
 
 
 def test_rmse_trajectory_and_time_to_target():
