@@ -17,7 +17,7 @@ int comm_world(fekf_comm* c) { return c ? c->world : 1; }
 int comm_rank(fekf_comm* c) { return c ? c->rank : 0; }
 
 fekf_status comm_allreduce(fekf_comm* c, double* buf, long long n, cudaStream_t s) {
-  if (!c || c->world <= 1) return FEKF_OK;
+  if (!c || !c->nc) return FEKF_OK;
   ncclResult_t r = ncclAllReduce(buf, buf, (size_t)n, ncclDouble, ncclSum, c->nc, s);
   if (r != ncclSuccess) {
     set_error(std::string("ncclAllReduce: ") + ncclGetErrorString(r));
@@ -46,7 +46,7 @@ fekf_status fekf_comm_init(int rank, int world, const unsigned char id_host[128]
   fekf_comm* c = new fekf_comm();
   c->rank = rank;
   c->world = world;
-  if (world > 1) {
+  {  // a single-rank communicator is a real NCCL communicator too (exercises the same path on one GPU)
     ncclUniqueId id;
     std::memcpy(&id, id_host, 128);
     ncclResult_t r = ncclCommInitRank(&c->nc, world, id, rank);

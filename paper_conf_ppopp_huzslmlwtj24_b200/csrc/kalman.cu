@@ -790,7 +790,7 @@ fekf_status Kf::pass(const double* g, bool rw, cudaStream_t s) {
 // pending; otherwise the pass is read-only and the corrections are applied to u in vector form.
 fekf_status Kf::update(const double* g, const double* abe, double sqrt_bs, double* w, cudaStream_t s) {
   FEKF_TRY(update_begin(g, s));
-  if (comm && comm_world(comm) > 1) FEKF_TRY(comm_allreduce(comm, ub.as<double>(), plan.Npad, s));
+  if (comm) FEKF_TRY(comm_allreduce(comm, ub.as<double>(), plan.Npad, s));
   return update_end(abe, sqrt_bs, w, s);
 }
 

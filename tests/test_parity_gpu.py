@@ -342,3 +342,56 @@ def test_kalman_sharded_ranks(world, precision):
         for kf in kfs:
             kf.get_block(b, out=full)           # each rank fills its own tiles (both triangles)
         assert rel(full.cpu(), st.P[b]) < tol
+
+
+def test_nccl_single_rank_step():
+    """a8 through NCCL on one GPU: a context built on a single-rank NCCL communicator (both all-reduces,
+    [g || error sum] and the partial u, captured in the step graph) trains exactly like one without."""
+    wl = get_config("t2_tiny")
+    m, opt = wl.model, wl.opt
+    B = wl.batch
+    ds = make_dataset("t2_tiny", B)
+    na = len(ds["types"])
+    w0 = init_weights(m, 3, float(ds["energy"].mean() / na))
+    comm = fk.Comm(0, 1, fk.Comm.unique_id())
+    buf = torch.arange(5, dtype=torch.float64, device="cuda")
+    comm.allreduce_sum(buf)
+    torch.cuda.synchronize()
+    assert torch.equal(buf.cpu(), torch.arange(5, dtype=torch.float64))
+    outs = []
+    for c in (comm, None):
+        ctx = fk.Context(m, opt, types=ds["types"], local_batch=B, global_batch=B, comm=c)
+        ctx.set_params(cu(w0))
+        for step in range(3):
+            groups = force_groups(na, step, 17, opt.force_groups, opt.atoms_per_group)
+            met = ctx.train_step(cu(ds["coord"]), cu(ds["box"]), cu(ds["energy"]), cu(ds["force"]),
+                                 cu(groups, torch.int32))
+        assert met.cpu()[7] == 0
+        outs.append(ctx.get_params().cpu())
+        ctx.close()
+    comm.close()
+    assert rel(outs[0], outs[1]) < 1e-13
+
+
+def test_rlekf_instance_by_instance():
+    """batch size 1 (the RLEKF instance-by-instance schedule) on the same kernels:
+    10 single-image minibatches (50 KF updates) against the oracle, rel 1e-9."""
+    wl = get_config("c1_cu32")
+    m, opt = wl.model, wl.opt
+    ds = make_dataset("c1_cu32", 10)
+    na = len(ds["types"])
+    w0 = init_weights(m, 3, float(ds["energy"].mean() / na))
+    ctx = fk.Context(m, opt, types=ds["types"], local_batch=1, global_batch=1)
+    ctx.set_params(cu(w0))
+    st = O.FEKF.create(w0, m, opt)
+    for step in range(10):
+        sl = slice(step, step + 1)
+        groups = force_groups(na, step, 17, opt.force_groups, opt.atoms_per_group)
+        met = ctx.train_step(cu(ds["coord"][sl]), cu(ds["box"][sl]), cu(ds["energy"][sl]), cu(ds["force"][sl]),
+                             cu(groups, torch.int32))
+        ref = O.train_step(st, ds["coord"][sl], ds["box"][sl], ds["types"], ds["energy"][sl], ds["force"][sl],
+                           groups, m, opt)
+        assert abs(met.cpu().numpy()[0] - ref["abe_e"]) <= 1e-9 * abs(ref["abe_e"])
+    assert rel(ctx.get_params().cpu(), st.w) < 1e-9
+    assert rel(ctx.kf.get_block(0).cpu(), st.P[0]) < 1e-9
+    ctx.close()
