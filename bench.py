@@ -306,7 +306,7 @@ def run_fekf(args, rank, world, local):
     out = {"metric": METRIC, "value": value, "unit": "images/s", "n_gpus": world, "steps": args.steps,
            "warmup": args.warmup, "ms_per_step": ms / args.steps, "higher_is_better": True, "scaling": "weak",
            "vs_baseline": None, "dtype": "f64" if args.precision == 64 else "f64 nets / f32 P",
-           "data": "synthetic (seeded perturbed water-64 lattices, LJ labels)",
+           "data": "synthetic (seeded perturbed %s snapshots, LJ labels)" % wl.system.name,
            "config": {"workload": args.config, "images_per_gpu": B, "global_batch": Bg, "n_atoms": na,
                       "n_params": ctx.n_params, "p_blocks": len(blocks), "p_bytes_per_gpu": info["p_bytes_local"],
                       "parallelism": f"dp{world}" + (" + P sharded" if world > 1 else ""),

@@ -395,3 +395,36 @@ def test_rlekf_instance_by_instance():
     assert rel(ctx.get_params().cpu(), st.w) < 1e-9
     assert rel(ctx.kf.get_block(0).cpu(), st.P[0]) < 1e-9
     ctx.close()
+
+
+def test_full_batch_water64_bench_config():
+    """The bench's launch configuration (water-64, local_batch 32, 1 027 082 parameters, 41 GB of P)
+    against the oracle: the energy and force Jacobians over all 32 images (rel 1e-11), the forward on
+    sampled images (rel 1e-12), and the forces of the selected atoms a force update uses."""
+    wl = get_config("c2_water64")
+    m = wl.model
+    B = wl.batch
+    ds = make_dataset("c2_water64", B)
+    na = len(ds["types"])
+    w = init_weights(m, 3, float(ds["energy"].mean() / na))
+    ctx = fk.Context(m, wl.opt, types=ds["types"], local_batch=B, global_batch=B)
+    ctx.set_params(cu(w))
+    X, BX = cu(ds["coord"]), cu(ds["box"])
+    rj, rs, _ = O.build_nlist(ds["coord"], ds["box"], ds["types"], m.rcut, m.sel)
+    g, s = ctx.energy_jacobian(X, BX, cu(ds["energy"]))
+    gr, sr, _ = O.energy_grad(w, ds["coord"], ds["box"], ds["types"], rj, rs, ds["energy"], m)
+    assert rel(g.cpu(), gr) < 1e-11
+    assert abs(float(s.cpu()[0]) - sr) <= 1e-13 * max(1.0, abs(sr))
+    atoms = force_groups(na, 3, wl.seed)[1]
+    g, s = ctx.force_jacobian(X, BX, cu(ds["force"]), cu(atoms, torch.int32))
+    gr, sr, _ = O.force_grad(w, ds["coord"], ds["box"], ds["types"], rj, rs, ds["force"], atoms, m)
+    assert rel(g.cpu(), gr) < 1e-11
+    assert abs(float(s.cpu()[0]) - sr) <= 1e-12 * max(1.0, abs(sr))
+    ea, e, f, v = ctx.forward(X, BX)
+    for b in (0, 17, 31):
+        sl = slice(b, b + 1)
+        Ea, E, F, V = O.energy_force_virial(w, ds["coord"][sl], ds["box"][sl], ds["types"], rj[sl], rs[sl], m)
+        assert rel(e[sl].cpu(), E) < 1e-12
+        assert rel(f[sl].cpu(), F) < 1e-12
+        assert rel(v[sl].cpu().reshape(-1, 3, 3), V) < 1e-12
+    ctx.close()
