@@ -107,18 +107,19 @@ struct EmbFwdIO {
 // Forward layer L >= 1 on the current tile: h_L = skip(h_{L-1}) + y_L, y_L = tanh(h_{L-1} W_L + b_L)
 // (primal) or (1 - y_L^2)(hdot_{L-1} W_L) (tangent rows, y_L of the primal row).
 template <class W, int L>
-__device__ __forceinline__ void fwd_layer(double* sm, const EmbFwdIO& io, int r0, int R, bool tan, const int* s_prow) {
+__device__ __forceinline__ void fwd_layer(double* sm, const double* __restrict__ wimg, const EmbFwdIO& io, int r0, int R,
+                                          bool tan, const int* s_prow) {
   constexpr int T = W::T, NW = EMB_FWD_WARPS;
   constexpr int din = W::din(L), d = W::d(L), skip = W::skip(L);
   constexpr int LDI = W::fALD((L - 1) & 1), LDO = W::fALD(L & 1);
-  const double* in = sm + W::fA((L - 1) & 1);
-  double* out = sm + W::fA(L & 1);
-  const double* bs = sm + W::fB(L);
+  const double* in = sm + W::sA((L - 1) & 1);
+  double* out = sm + W::sA(L & 1);
+  const double* bs = sm + W::sB(L);
   double* Yl = io.Y[L];
   double* Hl = io.H[L];
   const double* Ypl = io.Yp[L];
   cta_mma<false, T / 8, pad8(d) / 8, pad4(din), LDI, sld(d), NW>(
-      in, sm + W::fW(L), [&](int r, int c, double z0, double z1) {
+      in, wimg + W::fW(L), [&](int r, int c, double z0, double z1) {
         const int row = r0 + r;
         const bool live = row < R;
         double h[2];
@@ -146,8 +147,24 @@ __device__ __forceinline__ void fwd_layer(double* sm, const EmbFwdIO& io, int r0
   __syncthreads();
 }
 
+// zero-padded global image of the W_l ([pad4(din)][sld(d)], the forward's layout) for the L1 path
 template <class W>
-__global__ void __launch_bounds__(EMB_FWD_WARPS * 32) emb_fwd_kernel(const double* __restrict__ wp, EmbFwdIO io) {
+__global__ void emb_pack_kernel(const double* __restrict__ wp, double* __restrict__ wimg) {
+  const int tid = blockIdx.x * blockDim.x + threadIdx.x, nth = gridDim.x * blockDim.x;
+  for (int c = tid; c < pad8(W::d(0)); c += nth) wimg[W::fW(0) + c] = c < W::d(0) ? wp[W::goff(0) + c] : 0.0;
+#pragma unroll
+  for (int l = 1; l < W::NL; ++l) {
+    const int din = W::din(l), d = W::d(l), ld = sld(d), n = pad4(din) * ld;
+    for (int e = tid; e < n; e += nth) {
+      const int k = e / ld, j = e % ld;
+      wimg[W::fW(l) + e] = (k < din && j < d) ? wp[W::goff(l) + k * d + j] : 0.0;
+    }
+  }
+}
+
+template <class W>
+__global__ void __launch_bounds__(EMB_FWD_WARPS * 32) emb_fwd_kernel(const double* __restrict__ wp,
+                                                                     const double* __restrict__ wimg, EmbFwdIO io) {
   extern __shared__ __align__(16) double sm[];
   constexpr int T = W::T, NW = EMB_FWD_WARPS, NL = W::NL, RPW = T / NW;
   __shared__ double s_in[2][T];
@@ -155,22 +172,11 @@ __global__ void __launch_bounds__(EMB_FWD_WARPS * 32) emb_fwd_kernel(const doubl
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   const bool tan = io.tidx != nullptr;
   const int R = min(io.Rmax, *io.Rdev);
-  // ---- stage W_l (zero-padded to [pad4(din)][sld(d)]) and b_l
-  for (int c = tid; c < pad8(W::d(0)); c += blockDim.x) sm[W::fW(0) + c] = c < W::d(0) ? wp[W::goff(0) + c] : 0.0;
-#pragma unroll
-  for (int l = 1; l < NL; ++l) {
-    constexpr int dummy = 0;
-    (void)dummy;
-    const int din = W::din(l), d = W::d(l), ld = sld(d), n = pad4(din) * ld;
-    for (int e = tid; e < n; e += blockDim.x) {
-      const int k = e / ld, j = e % ld;
-      sm[W::fW(l) + e] = (k < din && j < d) ? wp[W::goff(l) + k * d + j] : 0.0;
-    }
-  }
+  // ---- stage b_l (W_l is read through L1 from wimg)
 #pragma unroll
   for (int l = 0; l < NL; ++l)
     for (int c = tid; c < pad8(W::d(l)); c += blockDim.x)
-      sm[W::fB(l) + c] = c < W::d(l) ? wp[W::goff(l) + W::din(l) * W::d(l) + c] : 0.0;
+      sm[W::sB(l) + c] = c < W::d(l) ? wp[W::goff(l) + W::din(l) * W::d(l) + c] : 0.0;
 
   // The next tile's input (row -> primal row -> slot -> s) is fetched by warp 0 in three dependent
   // steps spread over the current tile's layers, so its latency hides behind the compute.
@@ -206,9 +212,9 @@ __global__ void __launch_bounds__(EMB_FWD_WARPS * 32) emb_fwd_kernel(const doubl
     // ---- layer 0 (input width 1): elementwise
     {
       constexpr int d = W::d(0), w8 = pad8(d), CJ = (w8 + 31) / 32, ld = W::fALD(0);
-      double* out = sm + W::fA(0);
-      const double* w0 = sm + W::fW(0);
-      const double* b0 = sm + W::fB(0);
+      double* out = sm + W::sA(0);
+      const double* w0 = wimg + W::fW(0);
+      const double* b0 = sm + W::sB(0);
       double yp[RPW][CJ];
 #pragma unroll
       for (int i = 0; i < RPW; ++i)
@@ -242,10 +248,10 @@ __global__ void __launch_bounds__(EMB_FWD_WARPS * 32) emb_fwd_kernel(const doubl
     __syncthreads();
     fetch_b();
     // ---- layers 1..NL-1: DMMA with the bias / tanh / skip epilogue in the accumulators
-    if constexpr (NL >= 2) fwd_layer<W, 1>(sm, io, r0, R, tan, s_prowb);
+    if constexpr (NL >= 2) fwd_layer<W, 1>(sm, wimg, io, r0, R, tan, s_prowb);
     fetch_c();
-    if constexpr (NL >= 3) fwd_layer<W, 2>(sm, io, r0, R, tan, s_prowb);
-    if constexpr (NL >= 4) fwd_layer<W, 3>(sm, io, r0, R, tan, s_prowb);
+    if constexpr (NL >= 3) fwd_layer<W, 2>(sm, wimg, io, r0, R, tan, s_prowb);
+    if constexpr (NL >= 4) fwd_layer<W, 3>(sm, wimg, io, r0, R, tan, s_prowb);
     fetch_d(rn, buf ^ 1);
     buf ^= 1;
   }
@@ -267,18 +273,23 @@ static fekf_status emb_forward_t(Ctx& c, int p, long long Rmax, bool tangent, cu
     io.H[l] = l + 1 < W::NL ? nullptr : (tangent ? P.Ht[l].as<double>() : P.H[l].as<double>());
     io.Yp[l] = P.Y[l].as<double>();
   }
-  constexpr size_t smem = sizeof(double) * W::F_SMEM;
+  constexpr size_t smem = sizeof(double) * W::F_SMEM_ACT;
+  static_assert(W::F_W <= EMB_WIMG, "W image buffer");
   static int occ = 0;
   if (!occ) {
     FEKF_CHECK_CUDA(cudaFuncSetAttribute(emb_fwd_kernel<W>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
     FEKF_CHECK_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, emb_fwd_kernel<W>, EMB_FWD_WARPS * 32, smem));
     if (occ < 1) { set_error("emb_fwd_kernel: does not fit on an SM"); return FEKF_EINVAL; }
   }
+  const double* wp = c.w.as<double>() + P.L[0].W;
+  double* wimg = P.wimg.as<double>();
+  emb_pack_kernel<W><<<8, 256, 0, s>>>(wp, wimg);
+  FEKF_LAUNCH_CHECK();
   const long long tiles = (Rmax + EMB_T - 1) / EMB_T;
   const int grid = (int)std::max<long long>(1, std::min<long long>(tiles, (long long)num_sms() * occ));
-  emb_fwd_kernel<W><<<grid, EMB_FWD_WARPS * 32, smem, s>>>(c.w.as<double>() + P.L[0].W, io);
+  emb_fwd_kernel<W><<<grid, EMB_FWD_WARPS * 32, smem, s>>>(wp, wimg, io);
   FEKF_LAUNCH_CHECK();
-  count_launch();
+  count_launch(2);
   return FEKF_OK;
 }
 

@@ -17,6 +17,7 @@ namespace fekf {
 constexpr int EMB_T = 32;       // rows per CTA tile
 constexpr int EMB_FWD_WARPS = 8;
 constexpr int EMB_BWD_WARPS = 16;
+constexpr int EMB_WIMG = 1 << 14;   // doubles per pair for the padded global W image (forward, L1 path)
 
 __host__ __device__ constexpr int pad4(int x) { return (x + 3) & ~3; }
 __host__ __device__ constexpr int pad8(int x) { return (x + 7) & ~7; }
@@ -54,6 +55,13 @@ struct EmbW {
   __host__ __device__ static constexpr int fALD(int q) { return sld(maxw(q)); }
   __host__ __device__ static constexpr int fA(int q) { return fB(NL) + (q ? T * fALD(0) : 0); }
   static constexpr int F_SMEM = fA(1) + T * fALD(1);
+  // The forward kernel reads W through L1 from a zero-padded global image with the [0, F_W) part of the
+  // layout above (written once per launch by emb_pack_kernel); its SMEM holds only biases + activations,
+  // so more CTAs fit on an SM (the weights are shared by every CTA through L1).
+  static constexpr int F_W = fW(NL);
+  __host__ __device__ static constexpr int sB(int l) { return fB(l) - F_W; }
+  __host__ __device__ static constexpr int sA(int q) { return fA(q) - F_W; }
+  static constexpr int F_SMEM_ACT = F_SMEM - F_W;
   // ---- backward: W_0 | W_l [pad8(din)][sld(d)] | aug_l [T][sld(din+1)] | 3 x buf [T][BLD] | rr [T][8]
   __host__ __device__ static constexpr int bW(int l) {
     int o = pad8(D0);

@@ -204,7 +204,7 @@ constexpr size_t PASS_HDR = 2 * MAX_STAGES * sizeof(uint64_t) + MAX_STAGES * siz
 // made a read-write pass with 15 pending corrections compute-bound (18 ms fp64 / 27 ms fp32 for
 // water-64's 41 / 21 GB instead of the 12.3 / 6.3 ms of its traffic).
 __device__ __forceinline__ void dmma884k(double& d0, double& d1, double a, double b) {
-  asm volatile("mma.sync.aligned.m8n8k4.row.col.f64.f64.f64.f64 {%0,%1}, {%2}, {%3}, {%0,%1};"
+  asm("mma.sync.aligned.m8n8k4.row.col.f64.f64.f64.f64 {%0,%1}, {%2}, {%3}, {%0,%1};"
                : "+d"(d0), "+d"(d1)
                : "d"(a), "d"(b));
 }
