@@ -2,5 +2,5 @@
 
 The compute path is libfekf.so (csrc/, C ABI in include/fekf.h); `fekf` is its ctypes binding.
 """
-from .fekf import (Comm, Context, FekfError, KalmanFilter, lib, model_cfg, opt_cfg, plan_layout,  # noqa: F401
+from .fekf import (Comm, Context, FekfError, KalmanFilter, lib, model_cfg, opt_cfg, opt_defaults, plan_layout,  # noqa: F401
                    plan_shard, EXPORTED, LIB_PATH)

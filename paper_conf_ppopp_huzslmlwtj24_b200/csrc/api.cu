@@ -488,6 +488,22 @@ fekf_status fekf_plan_layout(const fekf_model_cfg* m, int block_size, int64_t* n
   return FEKF_OK;
 }
 
+fekf_status fekf_opt_defaults(int global_batch, fekf_opt_cfg* o) {
+  if (!o || global_batch < 1) { set_error("opt_defaults: bad args"); return FEKF_EINVAL; }
+  *o = fekf_opt_cfg{};
+  const bool large = global_batch > 1024;
+  o->lambda0 = large ? 0.90 : 0.98;
+  o->nu = large ? 0.996 : 0.9987;
+  o->block_size = 10240;
+  o->noise_mode = 0;
+  o->grad_reduce = 0;
+  o->force_groups = 4;
+  o->atoms_per_group = 6;
+  o->p_defer = 15;
+  o->precision = 64;
+  return FEKF_OK;
+}
+
 fekf_status fekf_plan_shard(const int32_t* blocks_host, int nblocks, int world, int rank, int64_t* tiles_local,
                             int64_t* bytes_local, int32_t* tile_owner_host) {
   if (!blocks_host || nblocks < 1 || world < 1 || rank < 0 || rank >= world) { set_error("plan_shard: bad args"); return FEKF_EINVAL; }

@@ -59,6 +59,7 @@ def lib():
         "fekf_comm_destroy": ([vp], i32), "fekf_comm_allreduce_sum": ([vp, vp, i64, vp], i32),
         "fekf_kf_create": ([vp, i32, C.POINTER(OptCfg), vp, C.POINTER(vp)], i32), "fekf_kf_destroy": ([vp], i32),
         "fekf_kf_update": ([vp, vp, vp, dbl, vp, vp], i32), "fekf_kf_flush": ([vp, vp], i32),
+        "fekf_opt_defaults": ([i32, C.POINTER(OptCfg)], i32),
         "fekf_kf_create_shard": ([vp, i32, C.POINTER(OptCfg), i32, i32, C.POINTER(vp)], i32),
         "fekf_kf_update_begin": ([vp, vp, vp], i32), "fekf_kf_update_end": ([vp, vp, dbl, vp, vp], i32),
         "fekf_kf_partial_u": ([vp, C.POINTER(vp), C.POINTER(i64)], i32),
@@ -93,7 +94,7 @@ EXPORTED = [
     "fekf_last_error", "fekf_version", "fekf_plan_layout", "fekf_plan_shard", "fekf_get_unique_id",
     "fekf_comm_init", "fekf_comm_destroy", "fekf_comm_allreduce_sum", "fekf_kf_create", "fekf_kf_destroy",
     "fekf_kf_update", "fekf_kf_flush", "fekf_kf_get_block", "fekf_kf_set_block", "fekf_kf_get_state",
-    "fekf_kf_create_shard", "fekf_kf_update_begin", "fekf_kf_partial_u", "fekf_kf_update_end",
+    "fekf_opt_defaults", "fekf_kf_create_shard", "fekf_kf_update_begin", "fekf_kf_partial_u", "fekf_kf_update_end",
     "fekf_kf_info", "fekf_kf_pass", "fekf_kf_timing", "fekf_create", "fekf_destroy", "fekf_param_count", "fekf_get_kf",
     "fekf_set_params", "fekf_get_params", "fekf_build_nlist", "fekf_env_mat", "fekf_forward",
     "fekf_energy_jacobian", "fekf_force_jacobian", "fekf_kalman_update", "fekf_train_step",
@@ -165,6 +166,14 @@ def opt_cfg(o=None) -> OptCfg:
     if c.precision not in (32, 64):
         raise ValueError("precision must be 32 or 64")
     return c
+
+
+def opt_defaults(global_batch):
+    """The paper's optimizer defaults for a global minibatch (lambda/nu 0.98/0.9987, 0.90/0.996
+    above 1024 images; N_b 10240, 4 force updates) as a dict for Context / KalmanFilter."""
+    c = OptCfg()
+    _check(lib().fekf_opt_defaults(int(global_batch), C.byref(c)))
+    return {k: getattr(c, k) for k, _ in OptCfg._fields_}
 
 
 def plan_layout(m, block_size=10240):

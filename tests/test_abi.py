@@ -69,3 +69,18 @@ def test_bad_config_rejected():
     m = dict(ntypes=1, rcut=4.0, rcut_smth=5.0, sel=[10], emb=[4], m2=2, fit=[8])
     with pytest.raises(fk.FekfError):
         fk.plan_layout(m, 100)
+
+
+def test_opt_defaults_follow_the_paper():
+    """P:L221 (lambda, nu; the bs > 1024 preset) and P:L293 (N_b, 4 force updates) from the golden file."""
+    import json
+    gold = json.load(open(os.path.join(ROOT, "tests", "golden", "paper_model.json")))
+    lam = gold["lambda"]
+    d = fk.opt_defaults(64)
+    assert d["lambda0"] == lam["lambda0"] and d["nu"] == lam["nu"]
+    assert d["block_size"] == gold["block_size"]["value"] and d["force_groups"] == 4
+    assert fk.opt_defaults(1024)["lambda0"] == lam["lambda0"]
+    big = fk.opt_defaults(4096)
+    assert big["lambda0"] == lam["lambda0_large"] and big["nu"] == lam["nu_large"]
+    with pytest.raises(fk.FekfError):
+        fk.opt_defaults(0)
