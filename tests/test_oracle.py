@@ -358,6 +358,89 @@ def test_fekf_bs1_is_rlekf():
         np.testing.assert_allclose(st.P[i], Pn[i], rtol=1e-12, atol=1e-14)
 
 
+# Naive-EKF (fusiform; readings N1-N4)
+def test_naive_one_sample_is_rlekf():
+    """bs = 1: E(K . ABE) = K . ABE, the single-sample EKF (RLEKF) written out independently."""
+    rng = np.random.default_rng(21)
+    blocks = [4, 6]
+    P0 = [_rand_spd(rng, n) for n in blocks]
+    st = O.NaiveEKF(np.zeros(10), blocks, lam=0.98, nu=0.9987)
+    st.P = [p.copy() for p in P0]
+    H = rng.standard_normal(10)
+    eps = 0.41
+    st.update_naive([H], [eps])
+    lam, L = 0.98, len(blocks)
+    Hs = [H[:4], H[4:]]
+    a = sum(h @ p @ h for h, p in zip(Hs, P0)) / lam + L
+    K = [p @ h / lam / a for h, p in zip(Hs, P0)]
+    Pn = [(np.eye(len(h)) - np.outer(k, h)) @ p / lam for h, p, k in zip(Hs, P0, K)]
+    np.testing.assert_allclose(st.w, np.concatenate(K) * eps, rtol=1e-13)
+    for i in range(2):
+        np.testing.assert_allclose(st.P[i], Pn[i], rtol=1e-12, atol=1e-14)
+
+
+def test_naive_scalar_closed_form():
+    """1 x 1 P: A_i = 1/(lam + g_i^2 p), P' = (p / lam) mean_i(lam / (lam + g_i^2 p)),
+    w' = w + mean_i(ABE_i A_i p g_i) — the averaged scalar Kalman filter by hand."""
+    p, lam = 1.7, 0.95
+    g = np.array([0.3, -1.1, 2.0, 0.05])
+    abe = np.array([0.2, 0.7, 0.01, 1.3])
+    st = O.NaiveEKF(np.array([0.5]), [1], lam=lam, nu=0.99)
+    st.P = [np.array([[p]])]
+    st.update_naive([np.array([x]) for x in g], abe)
+    A = 1.0 / (lam + g * g * p)
+    assert st.P[0][0, 0] == pytest.approx(p / lam * np.mean(lam * A), rel=1e-14)
+    assert st.w[0] == pytest.approx(0.5 + np.mean(abe * A * p * g), rel=1e-14)
+    assert st.lam == pytest.approx(lam * 0.99 + 0.01, abs=4e-16)
+
+
+def test_naive_identical_samples_and_permutation():
+    """n copies of one sample = that sample alone; the update is invariant under sample order;
+    P stays symmetric positive definite; the per-sample P_i obey Sherman-Morrison (1 block: c = lam)."""
+    rng = np.random.default_rng(5)
+    blocks = [7]
+    P0 = _rand_spd(rng, 7)
+    g = rng.standard_normal(7)
+    one = O.NaiveEKF(np.zeros(7), blocks, lam=0.97, nu=0.99)
+    one.P = [P0.copy()]
+    one.update_naive([g], [0.3])
+    many = O.NaiveEKF(np.zeros(7), blocks, lam=0.97, nu=0.99)
+    many.P = [P0.copy()]
+    many.update_naive([g] * 5, [0.3] * 5)
+    np.testing.assert_allclose(many.P[0], one.P[0], rtol=1e-13, atol=1e-15)
+    np.testing.assert_allclose(many.w, one.w, rtol=1e-13, atol=1e-16)
+    # Sherman-Morrison: P_1 = (P0^-1 + g g^T / lam)^-1 / lam
+    np.testing.assert_allclose(one.P[0], np.linalg.inv(np.linalg.inv(P0) + np.outer(g, g) / 0.97) / 0.97,
+                               rtol=1e-11, atol=1e-13)
+    G = [rng.standard_normal(7) for _ in range(6)]
+    ab = list(rng.uniform(0.1, 1.0, 6))
+    a = O.NaiveEKF(np.zeros(7), blocks, lam=0.97, nu=0.99)
+    a.P = [P0.copy()]
+    a.update_naive(G, ab)
+    perm = [3, 0, 5, 1, 4, 2]
+    b = O.NaiveEKF(np.zeros(7), blocks, lam=0.97, nu=0.99)
+    b.P = [P0.copy()]
+    b.update_naive([G[i] for i in perm], [ab[i] for i in perm])
+    np.testing.assert_allclose(a.P[0], b.P[0], rtol=1e-13, atol=1e-15)
+    np.testing.assert_allclose(a.w, b.w, rtol=1e-13, atol=1e-16)
+    assert np.array_equal(a.P[0], a.P[0].T)
+    np.linalg.cholesky(a.P[0])
+    # the mean of per-sample SPD matrices, each (P0^-1 + g_i g_i^T / lam)^-1 / lam
+    ref = sum(np.linalg.inv(np.linalg.inv(P0) + np.outer(x, x) / 0.97) / 0.97 for x in G) / 6
+    np.testing.assert_allclose(a.P[0], ref, rtol=1e-10, atol=1e-12)
+
+
+def test_naive_train_step_runs():
+    wl, m, ds, w = _setup("t2_tiny", n=2)
+    st = O.NaiveEKF.create(w, m, wl.opt)
+    out = O.naive_train_step(st, ds["coord"], ds["box"], ds["types"], ds["energy"], ds["force"],
+                             force_groups(len(ds["types"]), 0, 9), m)
+    assert len(out["abe_f"]) == 4 and len(out["A_e"]) == 2
+    assert np.all(np.isfinite(st.w)) and st.t == 5
+    for P in st.P:
+        np.linalg.cholesky(P)
+
+
 def test_lambda_closed_form(gold):
     lam0, nu = gold["lambda"]["lambda0"], gold["lambda"]["nu"]
     st = O.FEKF(np.zeros(2), [2], lam=lam0, nu=nu)
