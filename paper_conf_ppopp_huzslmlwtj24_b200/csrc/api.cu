@@ -323,7 +323,7 @@ Ctx::~Ctx() {
   if (gstream) cudaStreamDestroy(gstream);
   if (gev_in) cudaEventDestroy(gev_in);
   if (gev_out) cudaEventDestroy(gev_out);
-  for (DBuf* b : {&st_coord, &st_box, &st_e, &st_f, &st_fidx, &st_met}) dfree(*b);
+  for (DBuf* b : {&st_coord, &st_box, &st_e, &st_f, &st_fidx, &st_met, &naive_G, &naive_es, &naive_abe}) dfree(*b);
   kfo.reset();
   kf = nullptr;
   for (DBuf* b : {&types_d, &tindex_d, &atoms_d, &atoms_off_d, &sel_d, &sec_d, &err_d, &w, &gbuf, &nl_j, &nl_s,
@@ -413,6 +413,59 @@ static fekf_status step_body(Ctx& c, const double* coord, const double* box, con
     count_launch();
     FEKF_TRY(c.kf->update(g, c.abe.as<double>(), sqrt_bs, c.w.as<double>(), s));
   }
+  metrics_kernel<<<1, 1, 0, s>>>(c.kf->state.as<KfState>(), c.err_d.as<int>(), c.overflow.as<int>(), nb, metrics);
+  FEKF_LAUNCH_CHECK();
+  count_launch();
+  return FEKF_OK;
+}
+
+// Naive-EKF minibatch: per-image gradients and errors into the rank-n update (naive.cu).
+__global__ void naive_abe_kernel(const double* esum, int n, double scale, double* abe, double* metric) {
+  double m = 0.0;
+  for (int b = 0; b < n; ++b) {
+    abe[b] = esum[b] * scale;
+    m += abe[b];
+  }
+  if (metric) *metric = m / n;
+}
+
+static fekf_status naive_step_body(Ctx& c, const double* coord, const double* box, const double* e_label,
+                                   const double* f_label, const int32_t* force_idx, double* metrics, cudaStream_t s) {
+  const int nb = c.B;
+  const size_t na3 = (size_t)c.Na * 3;
+  if (!c.naive_G.p) {
+    FEKF_TRY(dalloc(c.naive_G, sizeof(double) * (size_t)nb * c.Np));
+    FEKF_TRY(dalloc(c.naive_es, sizeof(double) * nb));
+    FEKF_TRY(dalloc(c.naive_abe, sizeof(double) * nb));
+  }
+  double* G = c.naive_G.as<double>();
+  double* es = c.naive_es.as<double>();
+  double* ab = c.naive_abe.as<double>();
+  FEKF_CHECK_CUDA(cudaMemsetAsync(metrics, 0, sizeof(double) * 8, s));
+  // energy update: g_b, |e_b| / N_a of image b alone
+  for (int b = 0; b < nb; ++b) {
+    FEKF_TRY(geometry(c, coord + b * na3, box + (size_t)b * 9, 1, s));
+    FEKF_TRY(energy_grad_pass(c, 1, e_label + b, G + (size_t)b * c.Np, es + b, s));
+  }
+  naive_abe_kernel<<<1, 1, 0, s>>>(es, nb, 1.0, ab, metrics + 0);
+  FEKF_LAUNCH_CHECK();
+  count_launch();
+  FEKF_TRY(c.kf->update_naive(G, c.Np, ab, nb, c.w.as<double>(), nullptr, s));
+  // force updates
+  const int apg = c.o.atoms_per_group;
+  for (int k = 0; k < c.o.force_groups; ++k) {
+    for (int b = 0; b < nb; ++b) {
+      FEKF_TRY(geometry(c, coord + b * na3, box + (size_t)b * 9, 1, s));
+      FEKF_TRY(force_grad_pass(c, 1, f_label + b * na3, force_idx + (size_t)k * apg, apg, G + (size_t)b * c.Np,
+                               es + b, s));
+    }
+    naive_abe_kernel<<<1, 1, 0, s>>>(es, nb, 1.0 / ((double)apg * 3) / c.Na, ab, k < 4 ? metrics + 1 + k : nullptr);
+    FEKF_LAUNCH_CHECK();
+    count_launch();
+    FEKF_TRY(c.kf->update_naive(G, c.Np, ab, nb, c.w.as<double>(), nullptr, s));
+  }
+  // neighbour-list overflow of every image (the per-image passes above reuse slot 0)
+  FEKF_TRY(launch_nlist(c, coord, box, nb, c.nl_j.as<int>(), c.nl_s.as<int>(), c.overflow.as<int>(), s));
   metrics_kernel<<<1, 1, 0, s>>>(c.kf->state.as<KfState>(), c.err_d.as<int>(), c.overflow.as<int>(), nb, metrics);
   FEKF_LAUNCH_CHECK();
   count_launch();
@@ -737,6 +790,31 @@ fekf_status fekf_train_step(fekf_ctx* ctx, const double* coord, const double* bo
   c.last_launches = G->launches;
   ++c.nsteps;
   return FEKF_OK;
+}
+
+fekf_status fekf_naive_train_step(fekf_ctx* ctx, const double* coord, const double* box, const double* e_label,
+                                  const double* f_label, const int32_t* force_idx, double* metrics, cudaStream_t s) {
+  if (!ctx || !coord || !box || !e_label || !f_label || !metrics || (!force_idx && ctx->c.o.force_groups > 0)) {
+    set_error("naive_train_step: null");
+    return FEKF_EINVAL;
+  }
+  Ctx& c = ctx->c;
+  if (c.B != c.Bg || c.B > NAIVE_NMAX || c.comm) {
+    set_error("naive_train_step: single rank with local_batch <= 32 only");
+    return FEKF_EINVAL;
+  }
+  if (c.gstream) FEKF_CHECK_CUDA(cudaStreamSynchronize(c.gstream));   // earlier graph replays
+  const int64_t l0 = g_launches;
+  FEKF_TRY(naive_step_body(c, coord, box, e_label, f_label, force_idx, metrics, s));
+  c.last_launches = g_launches - l0;
+  ++c.nsteps;
+  return FEKF_OK;
+}
+
+fekf_status fekf_kf_update_naive(fekf_kf* k, const double* G, int64_t ldg, const double* abe, int n, double* w,
+                                 double* A_out, cudaStream_t s) {
+  if (!k || !G || !abe || !w) { set_error("kf_update_naive: null"); return FEKF_EINVAL; }
+  return k->kf.update_naive(G, ldg, abe, n, w, A_out, s);
 }
 
 fekf_status fekf_set_graph_mode(fekf_ctx* ctx, int enable) {

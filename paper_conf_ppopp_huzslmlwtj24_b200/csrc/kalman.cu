@@ -732,7 +732,7 @@ fekf_status Kf::timing_ctl(int mode, double* total_ms, int64_t* launches, int64_
 Kf::~Kf() {
   for (EvPair& e : ev_pool) { cudaEventDestroy(e.a); cudaEventDestroy(e.b); }
   for (DBuf* b : {&P, &items_d, &ws, &gpad, &ub, &ulist, &dotp, &csr_ptr, &csr_idx, &tc_blk, &tc_c, &off_d, &n_d,
-                  &state, &counter, &tcoff_d, &dblk, &cub})
+                  &state, &counter, &tcoff_d, &dblk, &cub, &nG, &nU, &nws, &ndot, &ncoef})
     dfree(*b);
 }
 

@@ -9,6 +9,7 @@ namespace fekf {
 constexpr int KT = FEKF_TILE;    // tile edge (64 fp64 = 32 KiB per tile)
 constexpr int SEG_TILES = 32;    // max tiles per work item (tile-row segment)
 constexpr int KMAX = 16;         // max deferred rank-1 corrections held before P is rewritten
+constexpr int NAIVE_NMAX = 32;   // max samples of one Naive-EKF update (naive.cu)
 
 // One P-pass work item: tiles (I, J0..J0+nJ-1) of block `blk`, stored contiguously at tile_off.
 struct ItemD {
@@ -102,6 +103,11 @@ struct Kf {
   fekf_status get_block(int b, double* dst, cudaStream_t s);
   fekf_status set_block(int b, const double* src, cudaStream_t s);
   fekf_status get_state(double* lambda, double* A_last, int* flags);
+  // Naive-EKF (naive.cu): n per-sample gradients G [n][ldg], per-sample ABE [n]; rank-n update of P
+  DBuf nG, nU, nws, ndot, ncoef;
+  int naive_np = 0;
+  fekf_status update_naive(const double* G, long long ldg, const double* abe, int n, double* w, double* A_out,
+                           cudaStream_t s);
 };
 
 }  // namespace fekf

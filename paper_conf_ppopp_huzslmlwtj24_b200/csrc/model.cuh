@@ -75,6 +75,7 @@ struct Ctx {
   DBuf chunks;                                    // [npairs * max_chunks] tangent-row scan workspace
   int max_chunks = 1;
   DBuf abe, metrics_tmp, abs_sum;
+  DBuf naive_G, naive_es, naive_abe;              // Naive-EKF step: [B][Np] per-image g, [B] error sums, [B] ABE
   size_t splitk_elems = 0, colsum_elems = 0;
   int64_t last_launches = 0;
   // step graphs: inputs are staged into ctx-owned buffers so the captured pointers stay fixed

@@ -81,6 +81,8 @@ def lib():
         "fekf_train_step": ([vp, vp, vp, vp, vp, vp, vp, vp], i32),
         "fekf_last_launch_count": ([vp, C.POINTER(i64)], i32),
         "fekf_set_graph_mode": ([vp, i32], i32),
+        "fekf_kf_update_naive": ([vp, vp, i64, vp, i32, vp, vp, vp], i32),
+        "fekf_naive_train_step": ([vp, vp, vp, vp, vp, vp, vp, vp], i32),
     }
     for name, (args, res) in sigs.items():
         f = getattr(L, name)
@@ -98,7 +100,7 @@ EXPORTED = [
     "fekf_kf_info", "fekf_kf_pass", "fekf_kf_timing", "fekf_create", "fekf_destroy", "fekf_param_count", "fekf_get_kf",
     "fekf_set_params", "fekf_get_params", "fekf_build_nlist", "fekf_env_mat", "fekf_forward",
     "fekf_energy_jacobian", "fekf_force_jacobian", "fekf_kalman_update", "fekf_train_step",
-    "fekf_last_launch_count", "fekf_set_graph_mode",
+    "fekf_last_launch_count", "fekf_set_graph_mode", "fekf_kf_update_naive", "fekf_naive_train_step",
 ]
 
 
@@ -259,6 +261,15 @@ class KalmanFilter:
     def update(self, g, abe, sqrt_bs, w, stream=None):
         _check(lib().fekf_kf_update(self.h, _ptr(g, torch.float64, "g"), _ptr(abe, torch.float64, "abe"),
                                     float(sqrt_bs), _ptr(w, torch.float64, "w"), _stream(stream)))
+
+    def update_naive(self, G, abe, w, A_out=None, stream=None):
+        """Naive-EKF update (fekf_kf_update_naive): G [n, ldg] per-sample gradients, abe [n]."""
+        if G.dim() != 2 or abe.numel() != G.shape[0]:
+            raise FekfError(1, "update_naive: G must be [n, ldg] and abe [n]")
+        _check(lib().fekf_kf_update_naive(self.h, _ptr(G, torch.float64, "G"), int(G.stride(0)),
+                                          _ptr(abe, torch.float64, "abe"), int(G.shape[0]), _ptr(w, torch.float64, "w"),
+                                          _ptr(A_out, torch.float64, "A_out") if A_out is not None else None,
+                                          _stream(stream)))
 
     def update_begin(self, g, stream=None):
         _check(lib().fekf_kf_update_begin(self.h, _ptr(g, torch.float64, "g"), _stream(stream)))
@@ -434,6 +445,23 @@ class Context:
                                      _ptr(e_label, torch.float64, "e_label"), _ptr(f_label, torch.float64, "f_label"),
                                      _ptr(force_idx, torch.int32, "force_idx"), _ptr(metrics, torch.float64, "metrics"),
                                      _stream(stream)))
+        return metrics
+
+    def naive_train_step(self, coord, box, e_label, f_label, force_idx, metrics=None, stream=None):
+        """Naive-EKF minibatch (fekf_naive_train_step): per-image gradients, rank-B Kalman updates."""
+        if metrics is None:
+            metrics = torch.empty(8, dtype=torch.float64, device="cuda")
+        na = self.natoms
+        for t, n, name in ((coord, self.B * na * 3, "coord"), (box, self.B * 9, "box"), (e_label, self.B, "e_label"),
+                           (f_label, self.B * na * 3, "f_label"), (metrics, 8, "metrics"),
+                           (force_idx, self.oc.force_groups * self.oc.atoms_per_group, "force_idx")):
+            if t.numel() != n:
+                raise FekfError(1, f"naive_train_step: {name} has {t.numel()} elements, expected {n}")
+        _check(lib().fekf_naive_train_step(self.h, _ptr(coord, torch.float64, "coord"), _ptr(box, torch.float64, "box"),
+                                           _ptr(e_label, torch.float64, "e_label"),
+                                           _ptr(f_label, torch.float64, "f_label"),
+                                           _ptr(force_idx, torch.int32, "force_idx"),
+                                           _ptr(metrics, torch.float64, "metrics"), _stream(stream)))
         return metrics
 
     def last_launch_count(self):

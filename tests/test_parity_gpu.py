@@ -428,3 +428,101 @@ def test_full_batch_water64_bench_config():
         assert rel(f[sl].cpu(), F) < 1e-12
         assert rel(v[sl].cpu().reshape(-1, 3, 3), V) < 1e-12
     ctx.close()
+
+
+# ------------------------------------------------------------------------------------------
+# Naive-EKF (Fig. 5; readings N1-N4): fekf_kf_update_naive and
+# fekf_naive_train_step against oracle.NaiveEKF
+# ------------------------------------------------------------------------------------------
+@pytest.mark.parametrize("blocks", [[5, 70, 130], [64], [1, 200, 127, 65]])
+@pytest.mark.parametrize("n", [1, 3, 8, 13, 32])
+def test_naive_kalman_updates(blocks, n):
+    """Rank-n updates over ragged blocks (tile tails, 1-element block, several tile rows), with FEKF
+    updates in between so pending deferred corrections are flushed first: w, P, A_i rel 1e-12."""
+    rng = np.random.default_rng(100 + n)
+    opt = dict(lambda0=0.98, nu=0.9987, block_size=1024, noise_mode=0, p_defer=5)
+    kf = fk.KalmanFilter(blocks, opt)
+    N = sum(blocks)
+    st = O.NaiveEKF(np.zeros(N), blocks, lam=0.98, nu=0.9987)
+    st.P = [_rand_spd(rng, k) for k in blocks]
+    for b, P in enumerate(st.P):
+        kf.set_block(b, cu(P))
+    w = torch.zeros(N, dtype=torch.float64, device="cuda")
+    A_gpu = torch.zeros(n, dtype=torch.float64, device="cuda")
+    for it in range(4):
+        if it == 2:   # two FEKF updates: deferred corrections pending at the next naive update
+            for _ in range(2):
+                g = rng.standard_normal(N)
+                kf.update(cu(g), cu([0.2]), 2.0, w)
+                st.update(g, 0.2, 4)
+        G = rng.standard_normal((n, N))
+        abe = rng.uniform(0.01, 1.0, n)
+        kf.update_naive(cu(G), cu(abe), w, A_gpu)
+        A_ref = st.update_naive(list(G), list(abe))
+        torch.cuda.synchronize()
+        assert rel(A_gpu.cpu(), A_ref) < 1e-12
+    assert rel(w.cpu(), st.w) < 1e-12
+    for b in range(len(blocks)):
+        assert rel(kf.get_block(b).cpu(), st.P[b]) < 1e-12
+    assert abs(kf.state()["lambda"] - st.lam) < 1e-15
+
+
+def test_naive_full_size_sampled_blocks():
+    """Bench-size filter (water-64: 110 blocks, 39 GiB packed P), n = 32 samples: one naive update
+    checked on sampled blocks against numpy from the GPU's previous P: u_i = P g_i per block,
+    P_new = (P - sum_i (A_i/n) u_i u_i^T)/lambda, w += sum_i (ABE_i A_i / n) u_i."""
+    wl = get_config("c2_water64")
+    _, blocks = fk.plan_layout(wl.model, wl.opt.block_size)
+    kf = fk.KalmanFilter(blocks, dict(block_size=wl.opt.block_size))
+    N = sum(blocks)
+    n = 32
+    off = np.concatenate([[0], np.cumsum(blocks)])
+    gen = torch.Generator(device="cuda").manual_seed(5)
+    w = torch.zeros(N, dtype=torch.float64, device="cuda")
+    abe = torch.rand(n, dtype=torch.float64, device="cuda", generator=gen) * 0.1
+    A = torch.zeros(n, dtype=torch.float64, device="cuda")
+    kf.update_naive(torch.randn(n, N, dtype=torch.float64, device="cuda", generator=gen) * 1e-2, abe, w, A)
+    sample = [0, 55, 109]
+    before = {b: kf.get_block(b).cpu().numpy() for b in sample}
+    lam = kf.state()["lambda"]
+    w0 = w.cpu().numpy()
+    G = torch.randn(n, N, dtype=torch.float64, device="cuda", generator=gen) * 1e-2
+    kf.update_naive(G, abe, w, A)
+    Gn, An, ab, w1 = G.cpu().numpy(), A.cpu().numpy(), abe.cpu().numpy(), w.cpu().numpy()
+    assert np.all(np.isfinite(An)) and np.all(An > 0)
+    for b in sample:
+        sl = slice(off[b], off[b + 1])
+        U = before[b] @ Gn[:, sl].T                  # [n_b, n]
+        ref = (before[b] - (U * (An / n)) @ U.T) / lam
+        assert rel(kf.get_block(b).cpu(), ref) < 1e-11
+        assert rel(w1[sl] - w0[sl], U @ (ab * An / n)) < 1e-11
+
+
+@pytest.mark.parametrize("name,nb,steps", [("t2_tiny", 3, 2), ("c1_cu32", 4, 3)])
+def test_naive_train_steps(name, nb, steps):
+    """Naive-EKF minibatches through the C ABI (per-image Jacobians, rank-B updates) against
+    oracle.naive_train_step: per-update ABE means, lambda, w and P."""
+    wl = get_config(name)
+    m, opt = wl.model, wl.opt
+    ds = make_dataset(name, nb * 2)
+    na = len(ds["types"])
+    w0 = init_weights(m, 3, float(ds["energy"].mean() / na))
+    ctx = fk.Context(m, opt, types=ds["types"], local_batch=nb, global_batch=nb)
+    ctx.set_params(cu(w0))
+    st = O.NaiveEKF.create(w0, m, opt)
+    for step in range(steps):
+        sl = slice((step % 2) * nb, (step % 2) * nb + nb)
+        groups = force_groups(na, step, 17, opt.force_groups, opt.atoms_per_group)
+        met = ctx.naive_train_step(cu(ds["coord"][sl]), cu(ds["box"][sl]), cu(ds["energy"][sl]),
+                                   cu(ds["force"][sl]), cu(groups, torch.int32))
+        ref = O.naive_train_step(st, ds["coord"][sl], ds["box"][sl], ds["types"], ds["energy"][sl],
+                                 ds["force"][sl], groups, m)
+        mt = met.cpu().numpy()
+        assert abs(mt[0] - ref["abe_e"]) <= 1e-10 * abs(ref["abe_e"])
+        np.testing.assert_allclose(mt[1:5], ref["abe_f"], rtol=1e-10)
+        assert abs(mt[5] - ref["A_last"][-1]) <= 1e-10 * abs(ref["A_last"][-1])
+        assert abs(mt[6] - ref["lambda"]) < 1e-14
+        assert mt[7] == 0
+    assert rel(ctx.get_params().cpu(), st.w) < 1e-9
+    for b in range(len(st.blocks)):
+        assert rel(ctx.kf.get_block(b).cpu(), st.P[b]) < 1e-9
