@@ -30,6 +30,7 @@ namespace fekf {
 namespace {
 
 constexpr int NKF_THREADS = 256;         // 8 warps, each an 8-row strip of the 64-row tile
+constexpr int MV_THREADS = 512;          // pass 1: warps 0-7 the row product, warps 8-15 the column product
 constexpr int LDP = KT + 4;              // SMEM row stride of a P tile: conflict-free A-fragment loads both ways
 constexpr int TILE_E = KT * KT;
 
@@ -47,16 +48,17 @@ template <int N>
 __device__ __forceinline__ void cp_wait() { asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory"); }
 
 // 64 rows x NP doubles of a [Npad][NP] vector set -> SMEM rows of stride NP + 4
-template <int NP>
+template <int NP, int NTH = NKF_THREADS>
 __device__ __forceinline__ void stage_vec(double* dst, const double* src, int tid) {
   constexpr int C = NP / 2;  // 16-byte chunks per row
-  for (int e = tid; e < KT * C; e += NKF_THREADS) {
+  for (int e = tid; e < KT * C; e += NTH) {
     const int r = e / C, q = e % C;
     cp16(dst + r * (NP + 4) + 2 * q, src + (size_t)r * NP + 2 * q);
   }
 }
+template <int NTH>
 __device__ __forceinline__ void stage_tile(double* dst, const double* src, int tid) {
-  for (int e = tid; e < KT * (KT / 2); e += NKF_THREADS) {
+  for (int e = tid; e < KT * (KT / 2); e += NTH) {
     const int r = e / (KT / 2), q = e % (KT / 2);
     cp16(dst + r * LDP + 2 * q, src + (size_t)r * KT + 2 * q);
   }
@@ -83,7 +85,7 @@ __global__ void nkf_pad_kernel(const double* __restrict__ G, long long ldg, int 
 // Pass 1: partial U = P G over this rank's items.  One CTA per SM pulls items (largest first) from a
 // counter; each tile of an item and the G_J segment it needs are double-buffered in SMEM by cp.async.
 template <int NP>
-__global__ void __launch_bounds__(NKF_THREADS, 1)
+__global__ void __launch_bounds__(MV_THREADS, 1)
 nkf_mv_kernel(const double* __restrict__ P, const ItemD* __restrict__ items, int n_items, int* counter,
               const double* __restrict__ gN, double* __restrict__ ws) {
   constexpr int LDG = NP + 4, NT = NP / 8;
@@ -93,7 +95,8 @@ nkf_mv_kernel(const double* __restrict__ P, const ItemD* __restrict__ items, int
   double* const sGI = sm + 2 * KT * LDP + 2 * KT * LDG;
   __shared__ int s_item;
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31, fr = lane >> 2, fk = lane & 3;
-  const int m0 = 8 * warp;
+  const bool colw = warp >= 8;                       // column-product warp (warp-uniform role)
+  const int m0 = 8 * (warp & 7);
   for (;;) {
     if (tid == 0) s_item = atomicAdd(counter, 1);
     __syncthreads();
@@ -102,9 +105,9 @@ nkf_mv_kernel(const double* __restrict__ P, const ItemD* __restrict__ items, int
     const ItemD it = items[k];
     const double* Pt = P + (size_t)it.tile_off * TILE_E;
     const double* gI = gN + (size_t)(it.vbase + (long long)it.I * KT) * NP;
-    stage_vec<NP>(sGI, gI, tid);
-    stage_tile(sP, Pt, tid);
-    stage_vec<NP>(sGJ, gN + (size_t)(it.vbase + (long long)it.J0 * KT) * NP, tid);
+    stage_vec<NP, MV_THREADS>(sGI, gI, tid);
+    stage_tile<MV_THREADS>(sP, Pt, tid);
+    stage_vec<NP, MV_THREADS>(sGJ, gN + (size_t)(it.vbase + (long long)it.J0 * KT) * NP, tid);
     cp_commit();
     double acc[NT][2];
 #pragma unroll
@@ -112,8 +115,9 @@ nkf_mv_kernel(const double* __restrict__ P, const ItemD* __restrict__ items, int
     for (int t = 0; t < it.nJ; ++t) {
       const int b = t & 1;
       if (t + 1 < it.nJ) {
-        stage_tile(sP + (b ^ 1) * KT * LDP, Pt + (size_t)(t + 1) * TILE_E, tid);
-        stage_vec<NP>(sGJ + (b ^ 1) * KT * LDG, gN + (size_t)(it.vbase + (long long)(it.J0 + t + 1) * KT) * NP, tid);
+        stage_tile<MV_THREADS>(sP + (b ^ 1) * KT * LDP, Pt + (size_t)(t + 1) * TILE_E, tid);
+        stage_vec<NP, MV_THREADS>(sGJ + (b ^ 1) * KT * LDG,
+                                  gN + (size_t)(it.vbase + (long long)(it.J0 + t + 1) * KT) * NP, tid);
         cp_commit();
         cp_wait<1>();
       } else {
@@ -121,15 +125,16 @@ nkf_mv_kernel(const double* __restrict__ P, const ItemD* __restrict__ items, int
       }
       __syncthreads();
       const double* p = sP + b * KT * LDP;
-      const double* gj = sGJ + b * KT * LDG;
-      // U_I[m0..m0+7][:] += P[m0..m0+7][:] G_J
+      if (!colw) {
+        // U_I[m0..m0+7][:] += P[m0..m0+7][:] G_J
+        const double* gj = sGJ + b * KT * LDG;
 #pragma unroll 4
-      for (int ks = 0; ks < KT / 4; ++ks) {
-        const double a = p[(m0 + fr) * LDP + 4 * ks + fk];
+        for (int ks = 0; ks < KT / 4; ++ks) {
+          const double a = p[(m0 + fr) * LDP + 4 * ks + fk];
 #pragma unroll
-        for (int j = 0; j < NT; ++j) dmma(acc[j][0], acc[j][1], a, gj[(4 * ks + fk) * LDG + 8 * j + fr]);
-      }
-      if (it.J0 + t != it.I) {
+          for (int j = 0; j < NT; ++j) dmma(acc[j][0], acc[j][1], a, gj[(4 * ks + fk) * LDG + 8 * j + fr]);
+        }
+      } else if (it.J0 + t != it.I) {
         // U_J[m0..m0+7][:] = P[:][m0..m0+7]^T G_I -> the tile's column-partial slot
         double z[NT][2];
 #pragma unroll
@@ -146,9 +151,11 @@ nkf_mv_kernel(const double* __restrict__ P, const ItemD* __restrict__ items, int
       }
       __syncthreads();   // buffer b is refilled at t + 2
     }
-    double* dst = ws + (size_t)it.row_slot * KT * NP + (m0 + fr) * NP + 2 * fk;
+    if (!colw) {
+      double* dst = ws + (size_t)it.row_slot * KT * NP + (m0 + fr) * NP + 2 * fk;
 #pragma unroll
-    for (int j = 0; j < NT; ++j) *reinterpret_cast<double2*>(dst + 8 * j) = make_double2(acc[j][0], acc[j][1]);
+      for (int j = 0; j < NT; ++j) *reinterpret_cast<double2*>(dst + 8 * j) = make_double2(acc[j][0], acc[j][1]);
+    }
   }
 }
 
@@ -242,8 +249,9 @@ __global__ void __launch_bounds__(NKF_THREADS)
 nkf_correct_kernel(double* __restrict__ P, const ItemD* __restrict__ items, const double* __restrict__ U,
                    const double* __restrict__ coef, int n) {
   constexpr int LDG = NP + 4;
-  __shared__ __align__(16) double sUI[KT * LDG];
-  __shared__ __align__(16) double sUJ[KT * LDG];
+  extern __shared__ __align__(16) double smc[];
+  double* const sUI = smc;                              // [KT * LDG]
+  double (*sUJ)[KT * LDG] = reinterpret_cast<double (*)[KT * LDG]>(smc + KT * LDG);   // [2][KT * LDG]
   __shared__ double sc[NP];
   const ItemD it = items[blockIdx.x];
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31, fr = lane >> 2, fk = lane & 3;
@@ -251,10 +259,22 @@ nkf_correct_kernel(double* __restrict__ P, const ItemD* __restrict__ items, cons
   if (tid < NP) sc[tid] = tid < n ? coef[tid] : 0.0;
   const double inv_lam = coef[96];
   stage_vec<NP>(sUI, U + (size_t)(it.vbase + (long long)it.I * KT) * NP, tid);
+  stage_vec<NP>(sUJ[0], U + (size_t)(it.vbase + (long long)it.J0 * KT) * NP, tid);
+  cp_commit();
   for (int t = 0; t < it.nJ; ++t) {
-    stage_vec<NP>(sUJ, U + (size_t)(it.vbase + (long long)(it.J0 + t) * KT) * NP, tid);
-    cp_commit();
-    cp_wait<0>();
+    const int b = t & 1;
+    // this thread's 16 elements of the tile, in flight while U_J arrives and the correction is formed
+    double* row = P + (size_t)(it.tile_off + t) * TILE_E + (m0 + fr) * KT + 2 * fk;
+    double2 v[8];
+#pragma unroll
+    for (int q = 0; q < 8; ++q) v[q] = *reinterpret_cast<const double2*>(row + 8 * q);
+    if (t + 1 < it.nJ) {
+      stage_vec<NP>(sUJ[b ^ 1], U + (size_t)(it.vbase + (long long)(it.J0 + t + 1) * KT) * NP, tid);
+      cp_commit();
+      cp_wait<1>();
+    } else {
+      cp_wait<0>();
+    }
     __syncthreads();
     double c[8][2];
 #pragma unroll
@@ -264,17 +284,15 @@ nkf_correct_kernel(double* __restrict__ P, const ItemD* __restrict__ items, cons
       const int kk = 4 * ks + fk;
       const double a = sc[kk] * sUI[(m0 + fr) * LDG + kk];
 #pragma unroll
-      for (int q = 0; q < 8; ++q) dmma(c[q][0], c[q][1], a, sUJ[(8 * q + fr) * LDG + kk]);
+      for (int q = 0; q < 8; ++q) dmma(c[q][0], c[q][1], a, sUJ[b][(8 * q + fr) * LDG + kk]);
     }
-    double* row = P + (size_t)(it.tile_off + t) * TILE_E + (m0 + fr) * KT + 2 * fk;
 #pragma unroll
     for (int q = 0; q < 8; ++q) {
-      double2 v = *reinterpret_cast<const double2*>(row + 8 * q);
-      v.x = (v.x - c[q][0]) * inv_lam;
-      v.y = (v.y - c[q][1]) * inv_lam;
-      *reinterpret_cast<double2*>(row + 8 * q) = v;
+      v[q].x = (v[q].x - c[q][0]) * inv_lam;
+      v[q].y = (v[q].y - c[q][1]) * inv_lam;
+      *reinterpret_cast<double2*>(row + 8 * q) = v[q];
     }
-    __syncthreads();   // sUJ is restaged for the next tile
+    __syncthreads();   // sUJ[b] is restaged at t + 2
   }
 }
 
@@ -304,7 +322,7 @@ static fekf_status naive_launch(Kf& k, const double* G, long long ldg, const dou
     const size_t smem = mv_smem(NP);
     FEKF_CHECK_CUDA(cudaFuncSetAttribute(nkf_mv_kernel<NP>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
     const int grid = std::min<int>((int)p.items.size(), sms);
-    nkf_mv_kernel<NP><<<grid, NKF_THREADS, smem, s>>>(k.P.as<double>(), k.items_d.as<ItemD>(), (int)p.items.size(),
+    nkf_mv_kernel<NP><<<grid, MV_THREADS, smem, s>>>(k.P.as<double>(), k.items_d.as<ItemD>(), (int)p.items.size(),
                                                       k.counter.as<int>(), k.nG.as<double>(), k.nws.as<double>());
     FEKF_LAUNCH_CHECK();
     count_launch();
@@ -328,7 +346,9 @@ static fekf_status naive_launch(Kf& k, const double* G, long long ldg, const dou
   FEKF_LAUNCH_CHECK();
   count_launch(4);
   if (!p.items.empty()) {
-    nkf_correct_kernel<NP><<<(unsigned)p.items.size(), NKF_THREADS, 0, s>>>(
+    const size_t csm = (size_t)3 * KT * (NP + 4) * sizeof(double);
+    FEKF_CHECK_CUDA(cudaFuncSetAttribute(nkf_correct_kernel<NP>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)csm));
+    nkf_correct_kernel<NP><<<(unsigned)p.items.size(), NKF_THREADS, csm, s>>>(
         k.P.as<double>(), k.items_d.as<ItemD>(), k.nU.as<double>(), k.ncoef.as<double>(), n);
     FEKF_LAUNCH_CHECK();
     count_launch();
