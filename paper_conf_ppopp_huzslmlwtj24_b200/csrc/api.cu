@@ -6,6 +6,7 @@
 // blocked Kalman update (lines 8-13).
 #include <algorithm>
 #include <cmath>
+#include <cstdlib>
 #include <cstring>
 #include <string>
 
@@ -284,7 +285,18 @@ fekf_status Ctx::init(const fekf_model_cfg& mm, const fekf_opt_cfg& oo, int nato
   }
   kfo.reset(new fekf_kf());
   kf = &kfo->kf;
+  {
+    // blocks holding any embedding parameter (they come first in the layout) get their gradient last
+    long long acc = 0;
+    int late = 0;
+    const long long emb_end = fits.empty() ? Np : fits[0].L[0].W;
+    while (late < (int)blocks.size() && acc < emb_end) acc += blocks[late++];
+    kf->late_blocks = late;
+    const char* e = getenv("FEKF_SPLIT_SMS");
+    kf->split_sms = comm ? 0 : (e ? atoi(e) : 96);
+  }
   FEKF_TRY(kf->create(blocks, o, comm));
+  if (kf->split_sms > 0) FEKF_CHECK_CUDA(cudaEventCreateWithFlags(&ev_fit, cudaEventDisableTiming));
   int dev = 0;
   FEKF_CHECK_CUDA(cudaGetDevice(&dev));
   int maxsm = 0;
@@ -323,6 +335,7 @@ Ctx::~Ctx() {
   if (gstream) cudaStreamDestroy(gstream);
   if (gev_in) cudaEventDestroy(gev_in);
   if (gev_out) cudaEventDestroy(gev_out);
+  if (ev_fit) cudaEventDestroy(ev_fit);
   for (DBuf* b : {&st_coord, &st_box, &st_e, &st_f, &st_fidx, &st_met, &naive_G, &naive_es, &naive_abe}) dfree(*b);
   kfo.reset();
   kf = nullptr;
@@ -395,13 +408,16 @@ static fekf_status step_body(Ctx& c, const double* coord, const double* box, con
   double* esum = g + c.Np;
   FEKF_CHECK_CUDA(cudaMemsetAsync(metrics, 0, sizeof(double) * 8, s));
   FEKF_TRY(geometry(c, coord, box, nb, s));
-  // energy update (1 per minibatch)
+  // energy update (1 per minibatch); with one GPU the P pass of the fitting blocks overlaps the tail of
+  // the reverse pass (split pass, Kf::pass)
+  const bool split = c.ev_fit && !c.comm;
+  c.split_armed = split;
   FEKF_TRY(energy_grad_pass(c, nb, e_label, g, esum, s));
   FEKF_TRY(comm_allreduce(c.comm, g, c.Np + 1, s));
   abe_kernel<<<1, 1, 0, s>>>(esum, 1.0 / c.Bg, c.abe.as<double>(), metrics + 0);
   FEKF_LAUNCH_CHECK();
   count_launch();
-  FEKF_TRY(c.kf->update(g, c.abe.as<double>(), sqrt_bs, c.w.as<double>(), s));
+  FEKF_TRY(c.kf->update(g, c.abe.as<double>(), sqrt_bs, c.w.as<double>(), s, split ? c.ev_fit : nullptr));
   // force updates
   const int apg = c.o.atoms_per_group;
   for (int k = 0; k < c.o.force_groups; ++k) {
@@ -411,8 +427,9 @@ static fekf_status step_body(Ctx& c, const double* coord, const double* box, con
                                k < 4 ? metrics + 1 + k : nullptr);
     FEKF_LAUNCH_CHECK();
     count_launch();
-    FEKF_TRY(c.kf->update(g, c.abe.as<double>(), sqrt_bs, c.w.as<double>(), s));
+    FEKF_TRY(c.kf->update(g, c.abe.as<double>(), sqrt_bs, c.w.as<double>(), s, split ? c.ev_fit : nullptr));
   }
+  c.split_armed = false;
   metrics_kernel<<<1, 1, 0, s>>>(c.kf->state.as<KfState>(), c.err_d.as<int>(), c.overflow.as<int>(), nb, metrics);
   FEKF_LAUNCH_CHECK();
   count_launch();

@@ -703,8 +703,8 @@ __global__ void emb_wgrad_reduce_kernel(const double* __restrict__ ws, int nsets
 }
 
 template <class W>
-static fekf_status launch_bwd(const double* wp, const EmbBwdIO& io, long long Rmax, int max_grid, int* grid_out,
-                              cudaStream_t s) {
+static fekf_status launch_bwd(const double* wp, const EmbBwdIO& io, long long Rmax, int max_grid, int sms,
+                              int* grid_out, cudaStream_t s) {
   constexpr size_t smem = sizeof(double) * W::B_SMEM;
   static int occ = 0;
   if (!occ) {
@@ -713,7 +713,7 @@ static fekf_status launch_bwd(const double* wp, const EmbBwdIO& io, long long Rm
     if (occ < 1) { set_error("emb_bwd_kernel: does not fit on an SM"); return FEKF_EINVAL; }
   }
   const long long tiles = (Rmax + EMB_T - 1) / EMB_T;
-  const int grid = (int)std::max<long long>(1, std::min<long long>({tiles, (long long)num_sms() * occ, (long long)max_grid}));
+  const int grid = (int)std::max<long long>(1, std::min<long long>({tiles, (long long)sms * occ, (long long)max_grid}));
   emb_bwd_kernel<W><<<grid, EMB_BWD_WARPS * 32, smem, s>>>(wp, io);
   FEKF_LAUNCH_CHECK();
   count_launch();
@@ -738,6 +738,7 @@ static fekf_status emb_backward_t(Ctx& c, int p, long long Rmax, int mode, doubl
     io.Hbt[l] = P.Hbt[l].as<double>();
   }
   const int cap = (int)std::min<size_t>(1 << 20, c.splitk_elems / (2 * (size_t)W::GS));
+  const int sms = c.emb_sms > 0 ? c.emb_sms : num_sms();   // split P pass: the SMs it leaves free
   double* ws = c.splitk_ws.as<double>();
   int nsets = 0;
   if (dual) {
@@ -748,7 +749,7 @@ static fekf_status emb_backward_t(Ctx& c, int p, long long Rmax, int mode, doubl
     for (int l = 0; l < W::NL; ++l) t.Y[l] = P.Yt[l].as<double>();
     t.ws = ws;
     int gt = 0;
-    FEKF_TRY(launch_bwd<W>(wp, t, Rmax, cap, &gt, s));
+    FEKF_TRY(launch_bwd<W>(wp, t, Rmax, cap, sms, &gt, s));
     nsets += gt;
   }
   io.Rdev = c.rowcnt.as<int>() + (sel ? c.pairs.size() + p : p);
@@ -768,7 +769,7 @@ static fekf_status emb_backward_t(Ctx& c, int p, long long Rmax, int mode, doubl
   }
   io.ws = wantw ? ws + (size_t)nsets * W::GS : nullptr;
   int gp = 0;
-  FEKF_TRY(launch_bwd<W>(wp, io, Rmax, cap, &gp, s));
+  FEKF_TRY(launch_bwd<W>(wp, io, Rmax, cap, sms, &gp, s));
   if (wantw) {
     nsets += gp;
     emb_wgrad_reduce_kernel<<<cdiv(W::GS, 256), 256, 0, s>>>(ws, nsets, W::GS, g + P.L[0].W);

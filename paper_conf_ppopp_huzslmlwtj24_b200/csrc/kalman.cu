@@ -17,6 +17,7 @@
 // Partial u's go to a workspace slot per (item row) / (tile column) and are summed in a fixed order
 // (kf_reduce_u) — no floating-point atomics, bit-reproducible.
 #include <algorithm>
+#include <cstdlib>
 #include <cmath>
 #include <numeric>
 
@@ -27,8 +28,9 @@ namespace fekf {
 // ------------------------------------------------------------------------------------------------
 // host planner
 // ------------------------------------------------------------------------------------------------
-void KfPlan::build(const std::vector<int>& blocks, int world_, int rank_, int seg_tiles, int row_slots) {
+void KfPlan::build(const std::vector<int>& blocks, int world_, int rank_, int seg_tiles, int row_slots, int late) {
   rps = row_slots;
+  late_blocks = late;
   n = blocks;
   L = (int)n.size();
   world = world_;
@@ -72,11 +74,15 @@ void KfPlan::build(const std::vector<int>& blocks, int world_, int rank_, int se
     owner[k] = r;
     load[r] += all[k].nJ;
   }
-  // this rank's items, largest first (dynamic scheduling on the device picks them in this order)
+  // this rank's items, largest first (dynamic scheduling on the device picks them in this order); the
+  // early blocks' items ahead of the late blocks' items
+  std::stable_partition(order.begin(), order.end(), [&](int k) { return all[k].blk >= late_blocks; });
   items.clear();
+  n_early = 0;
   int64_t tile_off = 0;
   for (int k : order) {
     if (owner[k] != rank) continue;
+    if (all[k].blk >= late_blocks) ++n_early;
     ItemD d;
     d.blk = all[k].blk; d.I = all[k].I; d.J0 = all[k].J0; d.nJ = all[k].nJ;
     d.tile_off = tile_off;
@@ -427,8 +433,8 @@ kf_pass_kernel(PT* __restrict__ P, const ItemD* __restrict__ items, int n_items,
 // ------------------------------------------------------------------------------------------------
 // g (flat, n_i per block) -> padded vector (n_t*T per block, zero pad)
 __global__ void kf_pad_kernel(const double* __restrict__ g, double* __restrict__ gpad, const int* tc_blk,
-                              const int* tc_c, const long long* off, const int* nblk, long long npad) {
-  long long p = (long long)blockIdx.x * blockDim.x + threadIdx.x;
+                              const int* tc_c, const long long* off, const int* nblk, long long p0, long long npad) {
+  long long p = p0 + (long long)blockIdx.x * blockDim.x + threadIdx.x;
   if (p >= npad) return;
   const long long tc = p / KT;
   const int b = tc_blk[tc];
@@ -641,7 +647,8 @@ fekf_status Kf::create(const std::vector<int>& blocks, const fekf_opt_cfg& o, fe
   if (comm) { world = comm_world(comm); rank = comm_rank(comm); }
   else if (world_o > 0) { world = world_o; rank = rank_o; }
   ng = p32 ? 2 : 1;   // fp64: one group (measured: a second group slows the read-write pass)
-  plan.build(blocks, world, rank, SEG_TILES, ng);
+  if (const char* e = getenv("FEKF_FP64_NG")) if (!p32 && atoi(e) == 2) ng = 2;   // experiments
+  plan.build(blocks, world, rank, SEG_TILES, ng, world == 1 ? std::min<int>(late_blocks, (int)blocks.size()) : 0);
   const KfPlan& p = plan;
   FEKF_TRY(dalloc(P, (size_t)p.tiles_local * TILE_ELEMS * elem() + 16));
   FEKF_TRY(dalloc(items_d, std::max<size_t>(1, p.items.size()) * sizeof(ItemD)));
@@ -658,6 +665,7 @@ fekf_status Kf::create(const std::vector<int>& blocks, const fekf_opt_cfg& o, fe
   FEKF_TRY(dalloc(n_d, p.L * sizeof(int)));
   FEKF_TRY(dalloc(state, sizeof(KfState)));
   FEKF_TRY(dalloc(counter, sizeof(int)));
+  FEKF_TRY(dalloc(counter2, sizeof(int)));
   FEKF_TRY(dalloc(tcoff_d, (p.L + 1) * sizeof(long long)));
   FEKF_TRY(dalloc(dblk, (size_t)(1 + KMAX) * p.L * sizeof(double)));
   FEKF_TRY(dalloc(cub, (size_t)KMAX * p.L * sizeof(double)));
@@ -680,10 +688,20 @@ fekf_status Kf::create(const std::vector<int>& blocks, const fekf_opt_cfg& o, fe
   FEKF_CHECK_CUDA(cudaMemset(ulist.p, 0, (size_t)KMAX * p.Npad * sizeof(double)));
   FEKF_CHECK_CUDA(cudaFuncSetAttribute(kf_pass_kernel<double, 1>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)PASS_SMEM));
   FEKF_CHECK_CUDA(cudaFuncSetAttribute(kf_pass_kernel<float, 2>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)PASS_SMEM));
+  FEKF_CHECK_CUDA(cudaFuncSetAttribute(kf_pass_kernel<double, 2>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)PASS_SMEM));
   if (!p.items.empty()) {
     if (p32) kf_init_kernel<<<(unsigned)p.items.size(), 256>>>(P.as<float>(), items_d.as<ItemD>(), n_d.as<int>());
     else kf_init_kernel<<<(unsigned)p.items.size(), 256>>>(P.as<double>(), items_d.as<ItemD>(), n_d.as<int>());
     FEKF_LAUNCH_CHECK();
+  }
+  if (split_sms > 0 && plan.n_early > 0 && !comm && world == 1) {
+    // highest priority: the early pass's CTAs take SMs ahead of the reverse pass's queued CTAs
+    int lo = 0, hi = 0;
+    FEKF_CHECK_CUDA(cudaDeviceGetStreamPriorityRange(&lo, &hi));
+    FEKF_CHECK_CUDA(cudaStreamCreateWithPriority(&side, cudaStreamNonBlocking, hi));
+    FEKF_CHECK_CUDA(cudaEventCreateWithFlags(&ev_early, cudaEventDisableTiming));
+  } else {
+    split_sms = 0;
   }
   FEKF_CHECK_CUDA(cudaDeviceSynchronize());
   npend = 0;
@@ -696,8 +714,10 @@ fekf_status Kf::harvest(std::vector<EvPair>& pairs, size_t n) {
     float ms = 0.f;
     FEKF_CHECK_CUDA(cudaEventElapsedTime(&ms, pairs[k].a, pairs[k].b));
     t_ms += ms;
-    t_n += 1;
-    t_rw += pairs[k].rw;
+    if (!pairs[k].part) {
+      t_n += 1;
+      t_rw += pairs[k].rw;
+    }
   }
   return FEKF_OK;
 }
@@ -730,54 +750,96 @@ fekf_status Kf::timing_ctl(int mode, double* total_ms, int64_t* launches, int64_
 }
 
 Kf::~Kf() {
+  if (side) { cudaStreamSynchronize(side); cudaStreamDestroy(side); }
+  if (ev_early) cudaEventDestroy(ev_early);
   for (EvPair& e : ev_pool) { cudaEventDestroy(e.a); cudaEventDestroy(e.b); }
   for (DBuf* b : {&P, &items_d, &ws, &gpad, &ub, &ulist, &dotp, &csr_ptr, &csr_idx, &tc_blk, &tc_c, &off_d, &n_d,
-                  &state, &counter, &tcoff_d, &dblk, &cub, &nG, &nU, &nws, &ndot, &ncoef})
+                  &state, &counter, &counter2, &tcoff_d, &dblk, &cub, &nG, &nU, &nws, &ndot, &ncoef})
     dfree(*b);
 }
 
-fekf_status Kf::pass(const double* g, bool rw, cudaStream_t s) {
+// One launch of the P pass over items [i0, i0 + n) with its own work counter, bracketed by a timing
+// event pair when timing or capturing.
+fekf_status Kf::pass_launch(bool rw, int i0, int n, int* ctr, int grid, cudaStream_t s, int part) {
   const KfPlan& p = plan;
-  const int tb = 256;
-  kf_pad_kernel<<<cdiv(p.Npad, tb), tb, 0, s>>>(g, gpad.as<double>(), tc_blk.as<int>(), tc_c.as<int>(),
-                                                 off_d.as<long long>(), n_d.as<int>(), p.Npad);
+  FEKF_CHECK_CUDA(cudaMemsetAsync(ctr, 0, sizeof(int), s));
+  EvPair* tp = nullptr;
+  if (timing || capturing) {
+    if (capturing) {
+      rec->emplace_back();
+      tp = &rec->back();
+    } else {
+      if (ev_pool.size() <= ev_used) ev_pool.emplace_back();
+      tp = &ev_pool[ev_used++];
+    }
+    if (!tp->a) {
+      FEKF_CHECK_CUDA(cudaEventCreate(&tp->a));
+      FEKF_CHECK_CUDA(cudaEventCreate(&tp->b));
+    }
+    tp->rw = rw ? 1 : 0;
+    tp->part = (char)part;
+    FEKF_CHECK_CUDA(cudaEventRecordWithFlags(tp->a, s, capturing ? cudaEventRecordExternal : cudaEventRecordDefault));
+  }
+  const int K = rw ? npend : 0;
+  const int stage_bytes = (int)(TILE_ELEMS * elem() + (KT + 2 * K * VS) * sizeof(double));
+  int nst = (int)std::min<size_t>(MAX_STAGES, (PASS_SMEM - PASS_HDR) / stage_bytes);
+  if (ng == 2) nst &= ~1;   // two consumer groups alternate stages
+  const ItemD* it = items_d.as<ItemD>() + i0;
+  if (p32)
+    kf_pass_kernel<float, 2><<<grid, PASS_THREADS, PASS_SMEM, s>>>(
+        P.as<float>(), it, n, ctr, gpad.as<double>(), ulist.as<double>(), p.Npad, rw ? 1 : 0, K, nst, stage_bytes,
+        state.as<KfState>(), ws.as<double>());
+  else if (ng == 2)
+    kf_pass_kernel<double, 2><<<grid, PASS_THREADS, PASS_SMEM, s>>>(
+        P.as<double>(), it, n, ctr, gpad.as<double>(), ulist.as<double>(), p.Npad, rw ? 1 : 0, K, nst, stage_bytes,
+        state.as<KfState>(), ws.as<double>());
+  else
+    kf_pass_kernel<double, 1><<<grid, PASS_THREADS, PASS_SMEM, s>>>(
+        P.as<double>(), it, n, ctr, gpad.as<double>(), ulist.as<double>(), p.Npad, rw ? 1 : 0, K, nst, stage_bytes,
+        state.as<KfState>(), ws.as<double>());
   FEKF_LAUNCH_CHECK();
   count_launch();
-  if (!p.items.empty()) {
-    FEKF_CHECK_CUDA(cudaMemsetAsync(counter.p, 0, sizeof(int), s));
-    const int grid = std::min<int>((int)p.items.size(), num_sms());
-    EvPair* tp = nullptr;
-    if (timing || capturing) {
-      if (capturing) {
-        rec->emplace_back();
-        tp = &rec->back();
-      } else {
-        if (ev_pool.size() <= ev_used) ev_pool.emplace_back();
-        tp = &ev_pool[ev_used++];
-      }
-      if (!tp->a) {
-        FEKF_CHECK_CUDA(cudaEventCreate(&tp->a));
-        FEKF_CHECK_CUDA(cudaEventCreate(&tp->b));
-      }
-      tp->rw = rw ? 1 : 0;
-      FEKF_CHECK_CUDA(cudaEventRecordWithFlags(tp->a, s, capturing ? cudaEventRecordExternal : cudaEventRecordDefault));
-    }
-    const int K = rw ? npend : 0;
-    const int stage_bytes = (int)(TILE_ELEMS * elem() + (KT + 2 * K * VS) * sizeof(double));
-    int nst = (int)std::min<size_t>(MAX_STAGES, (PASS_SMEM - PASS_HDR) / stage_bytes);
-    if (ng == 2) nst &= ~1;   // two consumer groups alternate stages
-    if (p32)
-      kf_pass_kernel<float, 2><<<grid, PASS_THREADS, PASS_SMEM, s>>>(
-          P.as<float>(), items_d.as<ItemD>(), (int)p.items.size(), counter.as<int>(), gpad.as<double>(),
-          ulist.as<double>(), p.Npad, rw ? 1 : 0, K, nst, stage_bytes, state.as<KfState>(), ws.as<double>());
-    else
-      kf_pass_kernel<double, 1><<<grid, PASS_THREADS, PASS_SMEM, s>>>(
-          P.as<double>(), items_d.as<ItemD>(), (int)p.items.size(), counter.as<int>(), gpad.as<double>(),
-          ulist.as<double>(), p.Npad, rw ? 1 : 0, K, nst, stage_bytes, state.as<KfState>(), ws.as<double>());
+  if (tp) FEKF_CHECK_CUDA(cudaEventRecordWithFlags(tp->b, s, capturing ? cudaEventRecordExternal : cudaEventRecordDefault));
+  return FEKF_OK;
+}
+
+fekf_status Kf::pass(const double* g, bool rw, cudaStream_t s, cudaEvent_t ready) {
+  const KfPlan& p = plan;
+  const int tb = 256;
+  const int n_items = (int)p.items.size();
+  const bool split = ready && side && split_sms > 0 && p.n_early > 0;
+  if (split) {
+    // early blocks: pad + pass on the side stream as soon as their gradient is final
+    const long long p0 = p.tc_off[p.late_blocks] * KT;
+    FEKF_CHECK_CUDA(cudaStreamWaitEvent(side, ready, 0));
+    kf_pad_kernel<<<cdiv(p.Npad - p0, tb), tb, 0, side>>>(g, gpad.as<double>(), tc_blk.as<int>(), tc_c.as<int>(),
+                                                           off_d.as<long long>(), n_d.as<int>(), p0, p.Npad);
     FEKF_LAUNCH_CHECK();
     count_launch();
+    FEKF_TRY(pass_launch(rw, 0, p.n_early, counter2.as<int>(), std::min(p.n_early, split_sms), side));
+    FEKF_CHECK_CUDA(cudaEventRecord(ev_early, side));
+    // late blocks on the producing stream
+    if (p0 > 0) {
+      kf_pad_kernel<<<cdiv(p0, tb), tb, 0, s>>>(g, gpad.as<double>(), tc_blk.as<int>(), tc_c.as<int>(),
+                                                off_d.as<long long>(), n_d.as<int>(), 0, p0);
+      FEKF_LAUNCH_CHECK();
+      count_launch();
+    }
+    if (n_items > p.n_early)
+      FEKF_TRY(pass_launch(rw, p.n_early, n_items - p.n_early, counter.as<int>(),
+                           std::min(n_items - p.n_early, num_sms()), s, 1));
+    FEKF_CHECK_CUDA(cudaStreamWaitEvent(s, ev_early, 0));
+  } else {
+    kf_pad_kernel<<<cdiv(p.Npad, tb), tb, 0, s>>>(g, gpad.as<double>(), tc_blk.as<int>(), tc_c.as<int>(),
+                                                   off_d.as<long long>(), n_d.as<int>(), 0, p.Npad);
+    FEKF_LAUNCH_CHECK();
+    count_launch();
+    static const int cap = [] { const char* e = getenv("FEKF_PASS_SMS"); return e ? atoi(e) : 0; }();   // experiments
+    if (n_items > 0)
+      FEKF_TRY(pass_launch(rw, 0, n_items, counter.as<int>(), std::min(n_items, cap > 0 ? cap : num_sms()), s));
+  }
+  if (n_items > 0) {
     if (rw) ++rw_passes; else ++r_passes;
-    if (tp) FEKF_CHECK_CUDA(cudaEventRecordWithFlags(tp->b, s, capturing ? cudaEventRecordExternal : cudaEventRecordDefault));
   }
   kf_reduce_u_kernel<<<cdiv(p.n_tc, 4), 256, 0, s>>>(ws.as<double>(), csr_ptr.as<long long>(),
                                                       csr_idx.as<long long>(), p.n_tc, ub.as<double>());
@@ -788,16 +850,17 @@ fekf_status Kf::pass(const double* g, bool rw, cudaStream_t s) {
 
 // One update (Alg. 1 lines 8-13).  The stored P is rewritten only when `defer` corrections are
 // pending; otherwise the pass is read-only and the corrections are applied to u in vector form.
-fekf_status Kf::update(const double* g, const double* abe, double sqrt_bs, double* w, cudaStream_t s) {
-  FEKF_TRY(update_begin(g, s));
+fekf_status Kf::update(const double* g, const double* abe, double sqrt_bs, double* w, cudaStream_t s,
+                       cudaEvent_t ready) {
+  FEKF_TRY(update_begin(g, s, ready));
   if (comm) FEKF_TRY(comm_allreduce(comm, ub.as<double>(), plan.Npad, s));
   return update_end(abe, sqrt_bs, w, s);
 }
 
-fekf_status Kf::update_begin(const double* g, cudaStream_t s) {
+fekf_status Kf::update_begin(const double* g, cudaStream_t s, cudaEvent_t ready) {
   if (in_update) { set_error("kf update_begin: previous update not ended"); return FEKF_ESTATE; }
   cur_rw = npend >= defer;
-  FEKF_TRY(pass(g, cur_rw, s));
+  FEKF_TRY(pass(g, cur_rw, s, ready));
   in_update = true;
   return FEKF_OK;
 }

@@ -44,7 +44,10 @@ struct KfPlan {
   std::vector<int> tile_owner;        // owner rank of every tile, canonical packed order
   std::vector<long long> csr_ptr, csr_idx;
   int rps = 1;                        // row-partial slots per item (consumer groups of the P pass)
-  void build(const std::vector<int>& blocks, int world, int rank, int seg_tiles, int row_slots = 1);
+  // blocks [0, late_blocks) are "late" (their gradient is the last one the reverse pass finishes): this
+  // rank's items of the other ("early") blocks come first, n_early of them, so a pass can be split in two
+  int late_blocks = 0, n_early = 0;
+  void build(const std::vector<int>& blocks, int world, int rank, int seg_tiles, int row_slots = 1, int late = 0);
 };
 
 // communicator helpers (comm.cu)
@@ -55,6 +58,7 @@ fekf_status comm_allreduce(fekf_comm* c, double* buf, long long n, cudaStream_t 
 struct EvPair {
   cudaEvent_t a = nullptr, b = nullptr;
   char rw = 0;
+  char part = 0;   // 1: second launch of a split pass (its time adds to the pass; not counted as a pass)
 };
 
 // Event pairs recorded inside one captured step graph; harvested before the graph is replayed again
@@ -93,11 +97,20 @@ struct Kf {
   // world/rank > 0 without a communicator: shard plan of that rank, exchange of u left to the caller
   fekf_status create(const std::vector<int>& blocks, const fekf_opt_cfg& o, fekf_comm* c, int world = 0, int rank = 0);
   ~Kf();
-  fekf_status pass(const double* g, bool rw, cudaStream_t s);
-  fekf_status update(const double* g, const double* abe, double sqrt_bs, double* w, cudaStream_t s);
+  // Split pass (single process): with `ready` (an event recorded on the producing stream once the early
+  // blocks' gradient is final) the early items stream on `split_sms` SMs from a side stream while the
+  // producer finishes the late blocks' gradient; the late items follow on `s`.
+  int late_blocks = 0, split_sms = 0;
+  cudaStream_t side = nullptr;
+  cudaEvent_t ev_early = nullptr;
+  DBuf counter2;
+  fekf_status pass(const double* g, bool rw, cudaStream_t s, cudaEvent_t ready = nullptr);
+  fekf_status pass_launch(bool rw, int i0, int n, int* ctr, int grid, cudaStream_t s, int part = 0);
+  fekf_status update(const double* g, const double* abe, double sqrt_bs, double* w, cudaStream_t s,
+                     cudaEvent_t ready = nullptr);
   // update = begin (P pass: this rank's partial u) + all-reduce of u over ranks + end (A, K, w, lambda)
   bool in_update = false, cur_rw = false;
-  fekf_status update_begin(const double* g, cudaStream_t s);
+  fekf_status update_begin(const double* g, cudaStream_t s, cudaEvent_t ready = nullptr);
   fekf_status update_end(const double* abe, double sqrt_bs, double* w, cudaStream_t s);
   fekf_status flush(cudaStream_t s);
   fekf_status get_block(int b, double* dst, cudaStream_t s);

@@ -83,6 +83,12 @@ struct Ctx {
   bool trows_ready = false;                       // tangent-active rows already built for this force update
   std::map<int, StepGraph> graphs;
   cudaStream_t gstream = nullptr;
+  // Split P pass (kalman.cu Kf::pass): model_backward records ev_fit once the fitting nets' weight
+  // gradients are final (split_armed, set by the step around a gradient pass that feeds an update) and
+  // caps the embedding backward at emb_sms SMs while the early P pass streams on the others.
+  cudaEvent_t ev_fit = nullptr;
+  bool split_armed = false;
+  int emb_sms = 0;
   cudaEvent_t gev_in = nullptr, gev_out = nullptr;
   DBuf st_coord, st_box, st_e, st_f, st_fidx, st_met;
   int64_t nsteps = 0;

@@ -87,7 +87,7 @@ __global__ void nkf_pad_kernel(const double* __restrict__ G, long long ldg, int 
 template <int NP>
 __global__ void __launch_bounds__(MV_THREADS, 1)
 nkf_mv_kernel(const double* __restrict__ P, const ItemD* __restrict__ items, int n_items, int* counter,
-              const double* __restrict__ gN, double* __restrict__ ws) {
+              const double* __restrict__ gN, double* __restrict__ ws, int rps) {
   constexpr int LDG = NP + 4, NT = NP / 8;
   extern __shared__ __align__(16) double sm[];
   double* const sP = sm;                             // [2][KT * LDP]
@@ -152,9 +152,14 @@ nkf_mv_kernel(const double* __restrict__ P, const ItemD* __restrict__ items, int
       __syncthreads();   // buffer b is refilled at t + 2
     }
     if (!colw) {
-      double* dst = ws + (size_t)it.row_slot * KT * NP + (m0 + fr) * NP + 2 * fk;
+      // the plan's rps row slots per item: the sum goes to the first, the others are zeroed
+      double* dst = ws + (size_t)it.row_slot * rps * KT * NP + (m0 + fr) * NP + 2 * fk;
 #pragma unroll
       for (int j = 0; j < NT; ++j) *reinterpret_cast<double2*>(dst + 8 * j) = make_double2(acc[j][0], acc[j][1]);
+      for (int g = 1; g < rps; ++g)
+#pragma unroll
+        for (int j = 0; j < NT; ++j)
+          *reinterpret_cast<double2*>(dst + (size_t)g * KT * NP + 8 * j) = make_double2(0.0, 0.0);
     }
   }
 }
@@ -323,7 +328,7 @@ static fekf_status naive_launch(Kf& k, const double* G, long long ldg, const dou
     FEKF_CHECK_CUDA(cudaFuncSetAttribute(nkf_mv_kernel<NP>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
     const int grid = std::min<int>((int)p.items.size(), sms);
     nkf_mv_kernel<NP><<<grid, MV_THREADS, smem, s>>>(k.P.as<double>(), k.items_d.as<ItemD>(), (int)p.items.size(),
-                                                      k.counter.as<int>(), k.nG.as<double>(), k.nws.as<double>());
+                                                      k.counter.as<int>(), k.nG.as<double>(), k.nws.as<double>(), p.rps);
     FEKF_LAUNCH_CHECK();
     count_launch();
   }

@@ -1248,6 +1248,17 @@ fekf_status tangent_env(Ctx& c, int nb, cudaStream_t s) {
 // Reverse pass from the fitting-output seeds (ebar).  MODE_ENERGY_GRAD: weight gradients of the
 // primal graph.  MODE_FORCE: adjoints down to s and R~, then forces/virials.  MODE_FORCE_JAC: weight
 // gradients of the dual (primal+tangent) graph.
+static int sm_count() {
+  static int n = 0;
+  if (!n) {
+    int dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev);
+    if (n <= 0) n = 148;
+  }
+  return n;
+}
+
 fekf_status model_backward(Ctx& c, int nb, Mode mode, double* gout, cudaStream_t s) {
   const double* w = c.w.as<double>();
   const bool dual = mode == MODE_FORCE_JAC;
@@ -1306,6 +1317,12 @@ fekf_status model_backward(Ctx& c, int nb, Mode mode, double* gout, cudaStream_t
                                     L.dout, -1, 0, 0, 1, e};
     }
     if (nj) FEKF_TRY(wgrad_group(c, jobs, nj, s));
+    if (l == 0 && want_w && c.split_armed) {
+      // the fitting blocks' gradient is final: the early P pass may start (Kf::pass); the rest of this
+      // reverse pass leaves it split_sms SMs
+      FEKF_CHECK_CUDA(cudaEventRecord(c.ev_fit, s));
+      c.emb_sms = std::max(1, sm_count() - c.kf->split_sms);
+    }
     FEKF_TRY(gemm_group<false, true>(dg, nd, s));
   }
   // ---- descriptor (Eq. 4) ----
@@ -1412,6 +1429,7 @@ fekf_status model_backward(Ctx& c, int nb, Mode mode, double* gout, cudaStream_t
     FEKF_LAUNCH_CHECK();
     count_launch();
   }
+  c.emb_sms = 0;
   return FEKF_OK;
 }
 
