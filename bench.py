@@ -218,6 +218,7 @@ def run_fekf(args, rank, world, local):
     torch.cuda.synchronize()
     barrier()
     pass_ms, pass_n, pass_rw = ctx.kf.timing(False)
+    parts = ctx.kf.timing_parts()
     clk = clocks.stop()
     ms = e0.elapsed_time(e1)
     launches = ctx.last_launch_count() * args.steps
@@ -320,7 +321,9 @@ def run_fekf(args, rank, world, local):
             "frac": (achieved / peak) if achieved else None, "traffic": traffic,
             "peak_source": peak_kind, "alg_bytes_per_launch": alg_bytes, "avg_launch_ms": avg_pass_s * 1000.0,
             "launches_timed": pass_n, "rw_launches": pass_rw, "share_of_step": (pass_ms / max(ms, 1e-9)),
-            "split_pass_early_sms": split_sms, "standalone": standalone}
+            "split_pass_early_sms": split_sms, "standalone": standalone,
+            "split_ms_per_pass": dict(zip(["early", "late", "early_start_to_reverse_done"],
+                                          [x / max(pass_n, 1) for x in parts]))}
 
     out = {"metric": METRIC, "value": value, "unit": "images/s", "n_gpus": world, "steps": args.steps,
            "warmup": args.warmup, "ms_per_step": ms / args.steps, "higher_is_better": True, "scaling": "weak",

@@ -713,6 +713,8 @@ fekf_status Kf::harvest(std::vector<EvPair>& pairs, size_t n) {
     FEKF_CHECK_CUDA(cudaEventSynchronize(pairs[k].b));
     float ms = 0.f;
     FEKF_CHECK_CUDA(cudaEventElapsedTime(&ms, pairs[k].a, pairs[k].b));
+    t_part[(int)pairs[k].part] += ms;
+    if (pairs[k].part == 2) continue;
     t_ms += ms;
     if (!pairs[k].part) {
       t_n += 1;
@@ -736,6 +738,7 @@ fekf_status Kf::timing_ctl(int mode, double* total_ms, int64_t* launches, int64_
     for (GraphTiming* g : pend_graphs) g->pending = false;
     pend_graphs.clear();
     t_ms = 0.0;
+    t_part[0] = t_part[1] = t_part[2] = 0.0;
     t_n = t_rw = 0;
     return FEKF_OK;
   }
@@ -812,12 +815,35 @@ fekf_status Kf::pass(const double* g, bool rw, cudaStream_t s, cudaEvent_t ready
     // early blocks: pad + pass on the side stream as soon as their gradient is final
     const long long p0 = p.tc_off[p.late_blocks] * KT;
     FEKF_CHECK_CUDA(cudaStreamWaitEvent(side, ready, 0));
+    // diagnostic pair (timing only): early pass start on the side stream -> the producing stream is done
+    // with the reverse pass (index, not pointer: the pair lists grow below)
+    std::vector<EvPair>* dl = nullptr;
+    size_t di = 0;
+    if (timing || capturing) {
+      dl = capturing ? rec : &ev_pool;
+      if (capturing) {
+        rec->emplace_back();
+        di = rec->size() - 1;
+      } else {
+        if (ev_pool.size() <= ev_used) ev_pool.emplace_back();
+        di = ev_used++;
+      }
+      EvPair& d = (*dl)[di];
+      if (!d.a) {
+        FEKF_CHECK_CUDA(cudaEventCreate(&d.a));
+        FEKF_CHECK_CUDA(cudaEventCreate(&d.b));
+      }
+      d.part = 2;
+      FEKF_CHECK_CUDA(cudaEventRecordWithFlags(d.a, side, capturing ? cudaEventRecordExternal : cudaEventRecordDefault));
+    }
     kf_pad_kernel<<<cdiv(p.Npad - p0, tb), tb, 0, side>>>(g, gpad.as<double>(), tc_blk.as<int>(), tc_c.as<int>(),
                                                            off_d.as<long long>(), n_d.as<int>(), p0, p.Npad);
     FEKF_LAUNCH_CHECK();
     count_launch();
     FEKF_TRY(pass_launch(rw, 0, p.n_early, counter2.as<int>(), std::min(p.n_early, split_sms), side));
     FEKF_CHECK_CUDA(cudaEventRecord(ev_early, side));
+    if (dl)
+      FEKF_CHECK_CUDA(cudaEventRecordWithFlags((*dl)[di].b, s, capturing ? cudaEventRecordExternal : cudaEventRecordDefault));
     // late blocks on the producing stream
     if (p0 > 0) {
       kf_pad_kernel<<<cdiv(p0, tb), tb, 0, s>>>(g, gpad.as<double>(), tc_blk.as<int>(), tc_c.as<int>(),

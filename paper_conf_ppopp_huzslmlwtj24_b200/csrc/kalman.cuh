@@ -58,7 +58,8 @@ fekf_status comm_allreduce(fekf_comm* c, double* buf, long long n, cudaStream_t 
 struct EvPair {
   cudaEvent_t a = nullptr, b = nullptr;
   char rw = 0;
-  char part = 0;   // 1: second launch of a split pass (its time adds to the pass; not counted as a pass)
+  char part = 0;   // 1: second launch of a split pass (its time adds to the pass; not counted as a pass);
+                   // 2: diagnostic pair (early pass start -> producer stream done with the reverse pass)
 };
 
 // Event pairs recorded inside one captured step graph; harvested before the graph is replayed again
@@ -88,6 +89,7 @@ struct Kf {
   size_t ev_used = 0;
   std::vector<EvPair>* rec = nullptr;   // non-null while capturing with timing on
   double t_ms = 0.0;
+  double t_part[3] = {0.0, 0.0, 0.0};   // split passes: early launch, late launch, early start -> tail done
   int64_t t_n = 0, t_rw = 0;
   long long rw_passes = 0, r_passes = 0;
   fekf_status timing_ctl(int mode, double* total_ms, int64_t* launches, int64_t* rw_launches);

@@ -82,6 +82,7 @@ def lib():
         "fekf_last_launch_count": ([vp, C.POINTER(i64)], i32),
         "fekf_set_graph_mode": ([vp, i32], i32),
         "fekf_kf_update_naive": ([vp, vp, i64, vp, i32, vp, vp, vp], i32),
+        "fekf_kf_timing_parts": ([vp, vp], i32),
         "fekf_naive_train_step": ([vp, vp, vp, vp, vp, vp, vp, vp], i32),
     }
     for name, (args, res) in sigs.items():
@@ -101,6 +102,7 @@ EXPORTED = [
     "fekf_set_params", "fekf_get_params", "fekf_build_nlist", "fekf_env_mat", "fekf_forward",
     "fekf_energy_jacobian", "fekf_force_jacobian", "fekf_kalman_update", "fekf_train_step",
     "fekf_last_launch_count", "fekf_set_graph_mode", "fekf_kf_update_naive", "fekf_naive_train_step",
+    "fekf_kf_timing_parts",
 ]
 
 
@@ -287,6 +289,12 @@ class KalmanFilter:
     def update_end(self, abe, sqrt_bs, w, stream=None):
         _check(lib().fekf_kf_update_end(self.h, _ptr(abe, torch.float64, "abe"), float(sqrt_bs),
                                         _ptr(w, torch.float64, "w"), _stream(stream)))
+
+    def timing_parts(self):
+        """[early, late, early start -> reverse pass done] summed ms of the last timing window (split pass)."""
+        a = (C.c_double * 3)()
+        _check(lib().fekf_kf_timing_parts(self.h, a))
+        return list(a)
 
     def pass_only(self, g, stream=None):
         _check(lib().fekf_kf_pass(self.h, _ptr(g, torch.float64, "g"), _stream(stream)))
