@@ -42,6 +42,8 @@ def parse():
     ap.add_argument("--precision", type=int, default=64, choices=[64, 32],
                     help="storage precision of P (32 = the fp32 variant, reading Z22; nets stay fp64)")
     ap.add_argument("--p-defer", type=int, default=None, help="override the deferred-correction depth")
+    ap.add_argument("--p-mode", type=int, default=0, choices=[0, 1],
+                    help="N > 1: 0 = P sharded over ranks (partial u all-reduced), 1 = replicated (the paper, P:L229)")
     return ap.parse_args()
 
 
@@ -171,7 +173,7 @@ def run_fekf(args, rank, world, local):
     torch.cuda.set_device(local)
     wl = get_config(args.config)
     m, opt = wl.model, wl.opt
-    over = {"precision": args.precision}
+    over = {"precision": args.precision, "p_mode": args.p_mode}
     if args.p_defer is not None:
         over["p_defer"] = args.p_defer
     opt = type(opt)(**{**opt.__dict__, **over})
@@ -331,7 +333,7 @@ def run_fekf(args, rank, world, local):
            "data": "synthetic (seeded perturbed %s snapshots, LJ labels)" % wl.system.name,
            "config": {"workload": args.config, "images_per_gpu": B, "global_batch": Bg, "n_atoms": na,
                       "n_params": ctx.n_params, "p_blocks": len(blocks), "p_bytes_per_gpu": info["p_bytes_local"],
-                      "parallelism": f"dp{world}" + (" + P sharded" if world > 1 else ""),
+                      "parallelism": f"dp{world}" + ((" + P replicated" if args.p_mode else " + P sharded") if world > 1 else ""),
                       "p_precision": args.precision, "p_defer": opt.p_defer,
                       "l2": "inputs larger than L2: P (%.1f GiB packed) is streamed 5x per step"
                             % (info["p_bytes_local"] / 2**30)},

@@ -63,6 +63,7 @@ class OptConfig:
     atoms_per_group: int = 6
     p_defer: int = 15        # CUDA path only: deferred rank-1 corrections of P (same P up to rounding)
     precision: int = 64      # CUDA path only: storage precision of P (32 = the fp32 variant, reading Z22)
+    p_mode: int = 0          # CUDA path only, world > 1: 0 = P sharded over ranks, 1 = replicated
 
 
 @dataclass

@@ -644,8 +644,15 @@ fekf_status Kf::create(const std::vector<int>& blocks, const fekf_opt_cfg& o, fe
   }
   p32 = o.precision == 32;
   int world = 1, rank = 0;
-  if (comm) { world = comm_world(comm); rank = comm_rank(comm); }
-  else if (world_o > 0) { world = world_o; rank = rank_o; }
+  if (o.p_mode != 0 && o.p_mode != 1) {
+    set_error("kf_create: p_mode must be 0 (sharded) or 1 (replicated)");
+    return FEKF_EINVAL;
+  }
+  replicated = o.p_mode == 1;
+  if (!replicated) {
+    if (comm) { world = comm_world(comm); rank = comm_rank(comm); }
+    else if (world_o > 0) { world = world_o; rank = rank_o; }
+  }
   ng = p32 ? 2 : 1;   // fp64: one group (measured: a second group slows the read-write pass)
   if (const char* e = getenv("FEKF_FP64_NG")) if (!p32 && atoi(e) == 2) ng = 2;   // experiments
   plan.build(blocks, world, rank, SEG_TILES, ng, world == 1 ? std::min<int>(late_blocks, (int)blocks.size()) : 0);
@@ -879,7 +886,7 @@ fekf_status Kf::pass(const double* g, bool rw, cudaStream_t s, cudaEvent_t ready
 fekf_status Kf::update(const double* g, const double* abe, double sqrt_bs, double* w, cudaStream_t s,
                        cudaEvent_t ready) {
   FEKF_TRY(update_begin(g, s, ready));
-  if (comm) FEKF_TRY(comm_allreduce(comm, ub.as<double>(), plan.Npad, s));
+  if (comm && !replicated) FEKF_TRY(comm_allreduce(comm, ub.as<double>(), plan.Npad, s));
   return update_end(abe, sqrt_bs, w, s);
 }
 

@@ -76,6 +76,7 @@ struct Kf {
   int defer = 1;                 // corrections deferred before P is rewritten (1 = rewrite every update)
   int npend = 0;                 // host mirror of the device npend
   bool p32 = false;              // P stored fp32 (opt.precision == 32, reading Z22)
+  bool replicated = false;       // opt.p_mode == 1: every rank holds all of P, no u exchange
   int ng = 1;                    // consumer groups of the P pass
   size_t elem() const { return p32 ? sizeof(float) : sizeof(double); }
   DBuf P, items_d, ws, gpad, ub, ulist, dotp, csr_ptr, csr_idx, tc_blk, tc_c, off_d, n_d, state, counter;

@@ -336,7 +336,7 @@ static fekf_status naive_launch(Kf& k, const double* G, long long ldg, const dou
       k.nws.as<double>(), k.csr_ptr.as<long long>(), k.csr_idx.as<long long>(), k.nU.as<double>());
   FEKF_LAUNCH_CHECK();
   count_launch();
-  if (k.comm) FEKF_TRY(comm_allreduce(k.comm, k.nU.as<double>(), p.Npad * NP, s));
+  if (k.comm && !k.replicated) FEKF_TRY(comm_allreduce(k.comm, k.nU.as<double>(), p.Npad * NP, s));
   nkf_dot_kernel<NP><<<(unsigned)p.n_tc, 8 * NP, 0, s>>>(k.nG.as<double>(), k.nU.as<double>(), p.n_tc,
                                                          k.ndot.as<double>());
   FEKF_LAUNCH_CHECK();

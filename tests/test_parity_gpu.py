@@ -344,11 +344,14 @@ def test_kalman_sharded_ranks(world, precision):
         assert rel(full.cpu(), st.P[b]) < tol
 
 
-def test_nccl_single_rank_step():
+@pytest.mark.parametrize("p_mode", [0, 1])
+def test_nccl_single_rank_step(p_mode):
     """a8 through NCCL on one GPU: a context built on a single-rank NCCL communicator (both all-reduces,
-    [g || error sum] and the partial u, captured in the step graph) trains exactly like one without."""
+    [g || error sum] and the partial u, captured in the step graph; p_mode 1 = replicated P, no u
+    exchange) trains exactly like one without."""
     wl = get_config("t2_tiny")
     m, opt = wl.model, wl.opt
+    opt = type(opt)(**{**opt.__dict__, "p_mode": p_mode})
     B = wl.batch
     ds = make_dataset("t2_tiny", B)
     na = len(ds["types"])
