@@ -327,6 +327,7 @@ void Ctx::drop_graphs() {
     for (EvPair& e : kv.second.tm.ev) { cudaEventDestroy(e.a); cudaEventDestroy(e.b); }
   }
   graphs.clear();
+  graphs_ready = false;
 }
 
 Ctx::~Ctx() {
@@ -795,6 +796,28 @@ fekf_status fekf_train_step(fekf_ctx* ctx, const double* coord, const double* bo
     FEKF_CHECK_CUDA(cudaMemcpyAsync(c.st_fidx.p, force_idx, sizeof(int32_t) * c.o.force_groups * c.o.atoms_per_group,
                                     cudaMemcpyDeviceToDevice, s));
   StepGraph* G = nullptr;
+  if (!c.graphs_ready) {
+    // Capture every variant the step can take (pending-correction count at entry 0..p_defer, step parity)
+    // once, here, instead of the first time each count comes round: a capture + instantiate of the ~540
+    // nodes costs a few ms, and the count cycles through all p_defer + 1 values only every 16 steps.
+    Kf& k = *c.kf;
+    const int np0 = k.npend;
+    const int64_t ns0 = c.nsteps;
+    for (int np = 0; np <= k.defer; ++np)
+      for (int par = 0; par < 2; ++par) {
+        k.npend = np;
+        c.nsteps = par;
+        fekf_status st = step_graph(c, &G);
+        if (st != FEKF_OK) {
+          k.npend = np0;
+          c.nsteps = ns0;
+          return st;
+        }
+      }
+    k.npend = np0;
+    c.nsteps = ns0;
+    c.graphs_ready = true;
+  }
   FEKF_TRY(step_graph(c, &G));
   if (G->tm.pending) FEKF_TRY(c.kf->harvest_graph(&G->tm));
   FEKF_CHECK_CUDA(cudaEventRecord(c.gev_in, s));

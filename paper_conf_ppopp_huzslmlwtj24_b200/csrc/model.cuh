@@ -80,6 +80,7 @@ struct Ctx {
   int64_t last_launches = 0;
   // step graphs: inputs are staged into ctx-owned buffers so the captured pointers stay fixed
   bool use_graph = true;
+  bool graphs_ready = false;   // every (pending-correction count, parity) variant captured
   bool trows_ready = false;                       // tangent-active rows already built for this force update
   std::map<int, StepGraph> graphs;
   cudaStream_t gstream = nullptr;
