@@ -856,6 +856,21 @@ fekf_status fekf_naive_train_step(fekf_ctx* ctx, const double* coord, const doub
   return FEKF_OK;
 }
 
+fekf_status fekf_kf_update_naive_begin(fekf_kf* k, const double* G, int64_t ldg, int n, cudaStream_t s) {
+  if (!k || !G) { set_error("kf_update_naive_begin: null"); return FEKF_EINVAL; }
+  return k->kf.update_naive_begin(G, ldg, n, s);
+}
+fekf_status fekf_kf_naive_partial_u(fekf_kf* k, double** U, int64_t* len) {
+  if (!k || !U || !len) { set_error("kf_naive_partial_u: null"); return FEKF_EINVAL; }
+  if (k->kf.naive_n <= 0) { set_error("kf_naive_partial_u: no naive update begun"); return FEKF_ESTATE; }
+  *U = k->kf.nU.as<double>();
+  *len = k->kf.naive_u_len();
+  return FEKF_OK;
+}
+fekf_status fekf_kf_update_naive_end(fekf_kf* k, const double* abe, double* w, double* A_out, cudaStream_t s) {
+  if (!k || !abe || !w) { set_error("kf_update_naive_end: null"); return FEKF_EINVAL; }
+  return k->kf.update_naive_end(abe, w, A_out, s);
+}
 fekf_status fekf_kf_update_naive(fekf_kf* k, const double* G, int64_t ldg, const double* abe, int n, double* w,
                                  double* A_out, cudaStream_t s) {
   if (!k || !G || !abe || !w) { set_error("kf_update_naive: null"); return FEKF_EINVAL; }

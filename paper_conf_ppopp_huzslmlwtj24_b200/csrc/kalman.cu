@@ -891,7 +891,7 @@ fekf_status Kf::update(const double* g, const double* abe, double sqrt_bs, doubl
 }
 
 fekf_status Kf::update_begin(const double* g, cudaStream_t s, cudaEvent_t ready) {
-  if (in_update) { set_error("kf update_begin: previous update not ended"); return FEKF_ESTATE; }
+  if (in_update || naive_n > 0) { set_error("kf update_begin: previous update not ended"); return FEKF_ESTATE; }
   cur_rw = npend >= defer;
   FEKF_TRY(pass(g, cur_rw, s, ready));
   in_update = true;

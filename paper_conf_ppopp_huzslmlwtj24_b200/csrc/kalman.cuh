@@ -122,8 +122,12 @@ struct Kf {
   // Naive-EKF (naive.cu): n per-sample gradients G [n][ldg], per-sample ABE [n]; rank-n update of P
   DBuf nG, nU, nws, ndot, ncoef;
   int naive_np = 0;
+  int naive_n = 0;               // > 0 between update_naive_begin and update_naive_end
   fekf_status update_naive(const double* G, long long ldg, const double* abe, int n, double* w, double* A_out,
                            cudaStream_t s);
+  fekf_status update_naive_begin(const double* G, long long ldg, int n, cudaStream_t s);
+  fekf_status update_naive_end(const double* abe, double* w, double* A_out, cudaStream_t s);
+  long long naive_u_len() const;
 };
 
 }  // namespace fekf

@@ -305,9 +305,9 @@ static int np_for(int n) { return n <= 8 ? 8 : n <= 16 ? 16 : 32; }
 
 static size_t mv_smem(int NP) { return (size_t)(2 * KT * LDP + 3 * KT * (NP + 4)) * sizeof(double); }
 
+// begin: pad G, pass 1 over this rank's tiles and the per-tile-column reduction -> this rank's partial U
 template <int NP>
-static fekf_status naive_launch(Kf& k, const double* G, long long ldg, const double* abe, int n, double* w,
-                                double* A_out, cudaStream_t s) {
+static fekf_status naive_begin_t(Kf& k, const double* G, long long ldg, int n, cudaStream_t s) {
   const KfPlan& p = k.plan;
   const int tb = 256;
   nkf_pad_kernel<NP><<<cdiv(p.Npad * NP, tb), tb, 0, s>>>(G, ldg, n, k.nG.as<double>(), k.tc_blk.as<int>(),
@@ -328,7 +328,7 @@ static fekf_status naive_launch(Kf& k, const double* G, long long ldg, const dou
     FEKF_CHECK_CUDA(cudaFuncSetAttribute(nkf_mv_kernel<NP>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
     const int grid = std::min<int>((int)p.items.size(), sms);
     nkf_mv_kernel<NP><<<grid, MV_THREADS, smem, s>>>(k.P.as<double>(), k.items_d.as<ItemD>(), (int)p.items.size(),
-                                                      k.counter.as<int>(), k.nG.as<double>(), k.nws.as<double>(), p.rps);
+                                                     k.counter.as<int>(), k.nG.as<double>(), k.nws.as<double>(), p.rps);
     FEKF_LAUNCH_CHECK();
     count_launch();
   }
@@ -336,7 +336,13 @@ static fekf_status naive_launch(Kf& k, const double* G, long long ldg, const dou
       k.nws.as<double>(), k.csr_ptr.as<long long>(), k.csr_idx.as<long long>(), k.nU.as<double>());
   FEKF_LAUNCH_CHECK();
   count_launch();
-  if (k.comm && !k.replicated) FEKF_TRY(comm_allreduce(k.comm, k.nU.as<double>(), p.Npad * NP, s));
+  return FEKF_OK;
+}
+
+// end: A_i, w, lambda from the (summed) U, then the rank-n correction of this rank's tiles
+template <int NP>
+static fekf_status naive_end_t(Kf& k, const double* abe, int n, double* w, double* A_out, cudaStream_t s) {
+  const KfPlan& p = k.plan;
   nkf_dot_kernel<NP><<<(unsigned)p.n_tc, 8 * NP, 0, s>>>(k.nG.as<double>(), k.nU.as<double>(), p.n_tc,
                                                          k.ndot.as<double>());
   FEKF_LAUNCH_CHECK();
@@ -361,12 +367,11 @@ static fekf_status naive_launch(Kf& k, const double* G, long long ldg, const dou
   return FEKF_OK;
 }
 
-fekf_status Kf::update_naive(const double* G, long long ldg, const double* abe, int n, double* w, double* A_out,
-                             cudaStream_t s) {
+fekf_status Kf::update_naive_begin(const double* G, long long ldg, int n, cudaStream_t s) {
   if (p32) { set_error("kf_update_naive: fp64 P only"); return FEKF_EINVAL; }
   if (n < 1 || n > NAIVE_NMAX) { set_error("kf_update_naive: n must be in [1, 32]"); return FEKF_EINVAL; }
   if (ldg < plan.N) { set_error("kf_update_naive: ldg < N"); return FEKF_EINVAL; }
-  if (in_update) { set_error("kf_update_naive: an FEKF update is in progress"); return FEKF_ESTATE; }
+  if (in_update || naive_n > 0) { set_error("kf_update_naive: an update is in progress"); return FEKF_ESTATE; }
   const int NP = np_for(n);
   if (naive_np < NP) {   // workspace for the widest vector set seen so far
     for (DBuf* b : {&nG, &nU, &nws, &ndot, &ncoef}) dfree(*b);
@@ -378,9 +383,30 @@ fekf_status Kf::update_naive(const double* G, long long ldg, const double* abe, 
     naive_np = NP;
   }
   if (npend > 0) FEKF_TRY(flush(s));   // P_t is now the stored P (sigma = 1, no deferred terms)
-  if (NP == 8) return naive_launch<8>(*this, G, ldg, abe, n, w, A_out, s);
-  if (NP == 16) return naive_launch<16>(*this, G, ldg, abe, n, w, A_out, s);
-  return naive_launch<32>(*this, G, ldg, abe, n, w, A_out, s);
+  naive_n = n;
+  if (NP == 8) return naive_begin_t<8>(*this, G, ldg, n, s);
+  if (NP == 16) return naive_begin_t<16>(*this, G, ldg, n, s);
+  return naive_begin_t<32>(*this, G, ldg, n, s);
+}
+
+fekf_status Kf::update_naive_end(const double* abe, double* w, double* A_out, cudaStream_t s) {
+  if (naive_n <= 0) { set_error("kf_update_naive_end: no naive update begun"); return FEKF_ESTATE; }
+  const int n = naive_n;
+  naive_n = 0;
+  const int NP = np_for(n);
+  if (NP == 8) return naive_end_t<8>(*this, abe, n, w, A_out, s);
+  if (NP == 16) return naive_end_t<16>(*this, abe, n, w, A_out, s);
+  return naive_end_t<32>(*this, abe, n, w, A_out, s);
+}
+
+// The U layout of the partial / summed vector set: [N_pad][roundup8(n)] (position-major)
+long long Kf::naive_u_len() const { return naive_n > 0 ? plan.Npad * np_for(naive_n) : 0; }
+
+fekf_status Kf::update_naive(const double* G, long long ldg, const double* abe, int n, double* w, double* A_out,
+                             cudaStream_t s) {
+  FEKF_TRY(update_naive_begin(G, ldg, n, s));
+  if (comm && !replicated) FEKF_TRY(comm_allreduce(comm, nU.as<double>(), naive_u_len(), s));
+  return update_naive_end(abe, w, A_out, s);
 }
 
 }  // namespace fekf

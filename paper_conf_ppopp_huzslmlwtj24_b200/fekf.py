@@ -83,6 +83,9 @@ def lib():
         "fekf_set_graph_mode": ([vp, i32], i32),
         "fekf_kf_update_naive": ([vp, vp, i64, vp, i32, vp, vp, vp], i32),
         "fekf_kf_timing_parts": ([vp, vp], i32),
+        "fekf_kf_update_naive_begin": ([vp, vp, i64, i32, vp], i32),
+        "fekf_kf_naive_partial_u": ([vp, C.POINTER(vp), C.POINTER(i64)], i32),
+        "fekf_kf_update_naive_end": ([vp, vp, vp, vp, vp], i32),
         "fekf_naive_train_step": ([vp, vp, vp, vp, vp, vp, vp, vp], i32),
     }
     for name, (args, res) in sigs.items():
@@ -102,7 +105,7 @@ EXPORTED = [
     "fekf_set_params", "fekf_get_params", "fekf_build_nlist", "fekf_env_mat", "fekf_forward",
     "fekf_energy_jacobian", "fekf_force_jacobian", "fekf_kalman_update", "fekf_train_step",
     "fekf_last_launch_count", "fekf_set_graph_mode", "fekf_kf_update_naive", "fekf_naive_train_step",
-    "fekf_kf_timing_parts",
+    "fekf_kf_timing_parts", "fekf_kf_update_naive_begin", "fekf_kf_naive_partial_u", "fekf_kf_update_naive_end",
 ]
 
 
@@ -275,6 +278,27 @@ class KalmanFilter:
                                           _ptr(abe, torch.float64, "abe"), int(G.shape[0]), _ptr(w, torch.float64, "w"),
                                           _ptr(A_out, torch.float64, "A_out") if A_out is not None else None,
                                           _stream(stream)))
+
+    def update_naive_begin(self, G, stream=None):
+        if G.dim() != 2:
+            raise FekfError(1, "update_naive_begin: G must be [n, ldg]")
+        _check(lib().fekf_kf_update_naive_begin(self.h, _ptr(G, torch.float64, "G"), int(G.stride(0)), int(G.shape[0]),
+                                                _stream(stream)))
+
+    def naive_partial_u(self):
+        """Zero-copy view of this rank's partial U ([N_pad * roundup8(n)]) between naive begin and end."""
+        p, n = C.c_void_p(), C.c_int64()
+        _check(lib().fekf_kf_naive_partial_u(self.h, C.byref(p), C.byref(n)))
+
+        class _View:
+            __cuda_array_interface__ = {"shape": (n.value,), "typestr": "<f8", "data": (p.value, False),
+                                        "version": 2, "strides": None}
+        return torch.as_tensor(_View(), device="cuda")
+
+    def update_naive_end(self, abe, w, A_out=None, stream=None):
+        _check(lib().fekf_kf_update_naive_end(self.h, _ptr(abe, torch.float64, "abe"), _ptr(w, torch.float64, "w"),
+                                              _ptr(A_out, torch.float64, "A_out") if A_out is not None else None,
+                                              _stream(stream)))
 
     def update_begin(self, g, stream=None):
         _check(lib().fekf_kf_update_begin(self.h, _ptr(g, torch.float64, "g"), _stream(stream)))

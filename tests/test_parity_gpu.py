@@ -529,3 +529,44 @@ def test_naive_train_steps(name, nb, steps):
     assert rel(ctx.get_params().cpu(), st.w) < 1e-9
     for b in range(len(st.blocks)):
         assert rel(ctx.kf.get_block(b).cpu(), st.P[b]) < 1e-9
+
+
+@pytest.mark.parametrize("world", [2, 3])
+def test_naive_sharded_ranks(world):
+    """Naive-EKF with P sharded over `world` ranks in one process (the multi-GPU layout): every rank gets
+    all samples' G, streams only its tiles, the partial U's are summed (the all-reduce of U that replaces
+    the paper's P all-reduce, Fig. 5c), and w and every block of P match oracle.NaiveEKF (rel 1e-12)."""
+    rng = np.random.default_rng(8)
+    blocks = [5, 70, 130, 200, 64]
+    opt = dict(lambda0=0.98, nu=0.9987, block_size=1024, noise_mode=0, p_defer=3)
+    kfs = [fk.KalmanFilter(blocks, opt, shard=(world, r)) for r in range(world)]
+    N = sum(blocks)
+    st = O.NaiveEKF(np.zeros(N), blocks, lam=0.98, nu=0.9987)
+    st.P = [_rand_spd(rng, n) for n in blocks]
+    for kf in kfs:
+        for b, P in enumerate(st.P):
+            kf.set_block(b, cu(P))
+    ws = [torch.zeros(N, dtype=torch.float64, device="cuda") for _ in range(world)]
+    for it, n in enumerate([5, 12, 32]):
+        G = rng.standard_normal((n, N))
+        abe = rng.uniform(0.01, 1.0, n)
+        Gd, ad = cu(G), cu(abe)
+        for kf in kfs:
+            kf.update_naive_begin(Gd)
+        us = [kf.naive_partial_u() for kf in kfs]
+        tot = torch.stack(us).sum(0)
+        for u in us:
+            u.copy_(tot)
+        for kf, w in zip(kfs, ws):
+            kf.update_naive_end(ad, w)
+        st.update_naive(list(G), list(abe))
+    torch.cuda.synchronize()
+    for w in ws:
+        assert rel(w.cpu(), st.w) < 1e-12
+    for b, n in enumerate(blocks):
+        full = torch.zeros(n, n, dtype=torch.float64, device="cuda")
+        for kf in kfs:
+            kf.get_block(b, out=full)
+        assert rel(full.cpu(), st.P[b]) < 1e-12
+    with pytest.raises(fk.FekfError):
+        kfs[0].update_naive_end(ad, ws[0])        # end without begin
