@@ -108,6 +108,11 @@ __device__ __forceinline__ void cp_async8(double* dst, const double* src, bool v
   const int n = valid ? 8 : 0;  // src-size 0: zero-fill
   asm volatile("cp.async.ca.shared.global [%0], [%1], 8, %2;" ::"r"(d), "l"(src), "r"(n) : "memory");
 }
+__device__ __forceinline__ void cp_async16z(double* dst, const double* src, bool valid) {
+  const unsigned d = (unsigned)__cvta_generic_to_shared(dst);
+  const int n = valid ? 16 : 0;  // src-size 0: zero-fill
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(d), "l"(src), "r"(n) : "memory");
+}
 __device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
 template <int N>
 __device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory"); }
@@ -210,7 +215,21 @@ dgemm_kernel(const __grid_constant__ GemmGroup<Epi> G) {
   for (int i = 0; i < TI; ++i)
 #pragma unroll
     for (int j = 0; j < TJ; ++j) acc[i][j][0] = acc[i][j][1] = 0.0;
+  // 16-byte copies (two doubles along the contiguous dimension) when the problem's strides, bases and
+  // extents keep every pair inside one row and aligned; per problem, so warp-uniform
+  const bool a16 = !TA && aug_m < 0 && !(lda & 1) && !(reinterpret_cast<size_t>(A) & 15) && !(K & 1) && !(kps & 1);
+  const bool b16 = !(ldb & 1) && !(reinterpret_cast<size_t>(B) & 15) && (TB ? (!(K & 1) && !(kps & 1)) : !(N & 1));
   auto issue = [&](int buf, int k0) {
+    if (a16) {
+#pragma unroll
+      for (int q = 0; q < AE / 2; ++q) {
+        const int idx = tid + 256 * q;
+        const int r = idx / (GB_K / 2), kk = 2 * (idx % (GB_K / 2));
+        const int m = m0 + r, k = k0 + kk;
+        const bool ok = m < M && k < kend;
+        cp_async16z(&a_at(buf, r, kk), ok ? A + (size_t)m * lda + k : A, ok);
+      }
+    } else {
 #pragma unroll
     for (int q = 0; q < AE; ++q) {
       const int idx = tid + 256 * q;
@@ -225,6 +244,19 @@ dgemm_kernel(const __grid_constant__ GemmGroup<Epi> G) {
         const double* src = ok ? (TA ? A + (size_t)k * lda + m : A + (size_t)m * lda + k) : A;
         cp_async8(dst, src, ok);
       }
+    }
+    }
+    if (b16) {
+#pragma unroll
+      for (int q = 0; q < BE / 2; ++q) {
+        const int idx = tid + 256 * q;
+        int c, kk;
+        if (!TB) { kk = idx / (BN / 2); c = 2 * (idx % (BN / 2)); } else { c = idx / (GB_K / 2); kk = 2 * (idx % (GB_K / 2)); }
+        const int n = n0 + c, k = k0 + kk;
+        const bool ok = n < N && k < kend;
+        cp_async16z(&b_at(buf, c, kk), ok ? (TB ? B + (size_t)n * ldb + k : B + (size_t)k * ldb + n) : B, ok);
+      }
+      return;
     }
 #pragma unroll
     for (int q = 0; q < BE; ++q) {
