@@ -323,7 +323,8 @@ def run_fekf(args, rank, world, local):
             "frac": (achieved / peak) if achieved else None, "traffic": traffic,
             "peak_source": peak_kind, "alg_bytes_per_launch": alg_bytes, "avg_launch_ms": avg_pass_s * 1000.0,
             "launches_timed": pass_n, "rw_launches": pass_rw, "share_of_step": (pass_ms / max(ms, 1e-9)),
-            "split_pass_early_sms": split_sms, "standalone": standalone,
+            "split_pass_early_sms": split_sms, "split_updates": "force updates (the energy update's pass is unsplit)",
+            "standalone": standalone,
             "split_ms_per_pass": dict(zip(["early", "late", "early_start_to_reverse_done"],
                                           [x / max(pass_n, 1) for x in parts]))}
 

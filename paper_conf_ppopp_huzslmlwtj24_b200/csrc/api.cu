@@ -412,13 +412,15 @@ static fekf_status step_body(Ctx& c, const double* coord, const double* box, con
   // energy update (1 per minibatch); with one GPU the P pass of the fitting blocks overlaps the tail of
   // the reverse pass (split pass, Kf::pass)
   const bool split = c.ev_fit && !c.comm;
-  c.split_armed = split;
+  static const int split_e = [] { const char* e = getenv("FEKF_SPLIT_E"); return e ? atoi(e) : 0; }();  // measured: 0
+  c.split_armed = split && split_e;
   FEKF_TRY(energy_grad_pass(c, nb, e_label, g, esum, s));
   FEKF_TRY(comm_allreduce(c.comm, g, c.Np + 1, s));
   abe_kernel<<<1, 1, 0, s>>>(esum, 1.0 / c.Bg, c.abe.as<double>(), metrics + 0);
   FEKF_LAUNCH_CHECK();
   count_launch();
-  FEKF_TRY(c.kf->update(g, c.abe.as<double>(), sqrt_bs, c.w.as<double>(), s, split ? c.ev_fit : nullptr));
+  FEKF_TRY(c.kf->update(g, c.abe.as<double>(), sqrt_bs, c.w.as<double>(), s, c.split_armed ? c.ev_fit : nullptr));
+  c.split_armed = split;
   // force updates
   const int apg = c.o.atoms_per_group;
   for (int k = 0; k < c.o.force_groups; ++k) {
