@@ -261,7 +261,8 @@ template <typename PT, int NG>
 __global__ void __launch_bounds__(PASS_THREADS, 1)
 kf_pass_kernel(PT* __restrict__ P, const ItemD* __restrict__ items, int n_items, int* counter,
                const double* __restrict__ gpad, const double* __restrict__ ulist, long long npad, int rw, int K,
-               int nst, int stage_bytes, const KfState* st, double* __restrict__ ws) {
+               int nst, int stage_bytes, const KfState* st, double* __restrict__ ws, const ItemD* __restrict__ items2,
+               int n_items2, int* counter2) {
   constexpr uint32_t TILE_BYTES = TILE_ELEMS * sizeof(PT);
   constexpr int NGW = 8 / NG;            // warps per group
   constexpr int RPW = KT / NGW;          // rows per warp and tile
@@ -289,15 +290,25 @@ kf_pass_kernel(PT* __restrict__ P, const ItemD* __restrict__ items, int n_items,
     if (lane == 0) {
       int s = 0;
       uint32_t ph = 0;
+      bool own = true;
       const uint32_t bytes = TILE_BYTES + (1u + 2u * (uint32_t)K) * KT * sizeof(double);   // bytes landed
       while (true) {
-        const int itx = atomicAdd(counter, 1);
-        if (itx >= n_items) break;
-        const ItemD it = items[itx];
+        // own list first, then (split pass, late launch) the early launch's unclaimed items
+        int itx = -1, lst = 0;
+        if (own) {
+          itx = atomicAdd(counter, 1);
+          if (itx >= n_items) own = false;
+        }
+        if (!own) {
+          itx = n_items2 > 0 ? atomicAdd(counter2, 1) : n_items2;
+          if (itx >= n_items2) break;
+          lst = 1;
+        }
+        const ItemD it = (lst ? items2 : items)[itx];
         for (int t = 0; t < it.nJ; ++t) {
           mbar_wait(&empty[s], ph ^ 1);
           // flags: 1 first tile of the item for its group, 2 last one, 4 item shorter than NG tiles
-          meta[s] = make_int4(itx, it.J0 + t, (t < NG ? 1 : 0) | (t >= it.nJ - NG ? 2 : 0) | (it.nJ < NG ? 4 : 0), 0);
+          meta[s] = make_int4(itx, it.J0 + t, (t < NG ? 1 : 0) | (t >= it.nJ - NG ? 2 : 0) | (it.nJ < NG ? 4 : 0), lst);
           unsigned char* st_s = stages + (size_t)s * stage_bytes;
           double* st_g = reinterpret_cast<double*>(st_s + TILE_BYTES);
           double* st_v = st_g + KT;
@@ -341,7 +352,7 @@ kf_pass_kernel(PT* __restrict__ P, const ItemD* __restrict__ items, int n_items,
     mbar_wait(&full[s], ph);
     const int4 mt = meta[s];
     if (mt.x < 0) break;
-    const ItemD it = items[mt.x];
+    const ItemD it = (mt.w ? items2 : items)[mt.x];
     const int J = mt.y;
     const bool first = mt.z & 1, last = mt.z & 2, diag = (J == it.I);
     if (first) {
@@ -707,6 +718,7 @@ fekf_status Kf::create(const std::vector<int>& blocks, const fekf_opt_cfg& o, fe
     FEKF_CHECK_CUDA(cudaDeviceGetStreamPriorityRange(&lo, &hi));
     FEKF_CHECK_CUDA(cudaStreamCreateWithPriority(&side, cudaStreamNonBlocking, hi));
     FEKF_CHECK_CUDA(cudaEventCreateWithFlags(&ev_early, cudaEventDisableTiming));
+    FEKF_CHECK_CUDA(cudaEventCreateWithFlags(&ev_ctr, cudaEventDisableTiming));
   } else {
     split_sms = 0;
   }
@@ -762,6 +774,7 @@ fekf_status Kf::timing_ctl(int mode, double* total_ms, int64_t* launches, int64_
 Kf::~Kf() {
   if (side) { cudaStreamSynchronize(side); cudaStreamDestroy(side); }
   if (ev_early) cudaEventDestroy(ev_early);
+  if (ev_ctr) cudaEventDestroy(ev_ctr);
   for (EvPair& e : ev_pool) { cudaEventDestroy(e.a); cudaEventDestroy(e.b); }
   for (DBuf* b : {&P, &items_d, &ws, &gpad, &ub, &ulist, &dotp, &csr_ptr, &csr_idx, &tc_blk, &tc_c, &off_d, &n_d,
                   &state, &counter, &counter2, &tcoff_d, &dblk, &cub, &nG, &nU, &nws, &ndot, &ncoef})
@@ -770,9 +783,10 @@ Kf::~Kf() {
 
 // One launch of the P pass over items [i0, i0 + n) with its own work counter, bracketed by a timing
 // event pair when timing or capturing.
-fekf_status Kf::pass_launch(bool rw, int i0, int n, int* ctr, int grid, cudaStream_t s, int part) {
+fekf_status Kf::pass_launch(bool rw, int i0, int n, int* ctr, int grid, cudaStream_t s, int part, int i2, int n2,
+                            int* ctr2, bool zero_ctr) {
   const KfPlan& p = plan;
-  FEKF_CHECK_CUDA(cudaMemsetAsync(ctr, 0, sizeof(int), s));
+  if (zero_ctr) FEKF_CHECK_CUDA(cudaMemsetAsync(ctr, 0, sizeof(int), s));
   EvPair* tp = nullptr;
   if (timing || capturing) {
     if (capturing) {
@@ -795,18 +809,19 @@ fekf_status Kf::pass_launch(bool rw, int i0, int n, int* ctr, int grid, cudaStre
   int nst = (int)std::min<size_t>(MAX_STAGES, (PASS_SMEM - PASS_HDR) / stage_bytes);
   if (ng == 2) nst &= ~1;   // two consumer groups alternate stages
   const ItemD* it = items_d.as<ItemD>() + i0;
+  const ItemD* it2 = items_d.as<ItemD>() + i2;
   if (p32)
     kf_pass_kernel<float, 2><<<grid, PASS_THREADS, PASS_SMEM, s>>>(
         P.as<float>(), it, n, ctr, gpad.as<double>(), ulist.as<double>(), p.Npad, rw ? 1 : 0, K, nst, stage_bytes,
-        state.as<KfState>(), ws.as<double>());
+        state.as<KfState>(), ws.as<double>(), it2, n2, ctr2);
   else if (ng == 2)
     kf_pass_kernel<double, 2><<<grid, PASS_THREADS, PASS_SMEM, s>>>(
         P.as<double>(), it, n, ctr, gpad.as<double>(), ulist.as<double>(), p.Npad, rw ? 1 : 0, K, nst, stage_bytes,
-        state.as<KfState>(), ws.as<double>());
+        state.as<KfState>(), ws.as<double>(), it2, n2, ctr2);
   else
     kf_pass_kernel<double, 1><<<grid, PASS_THREADS, PASS_SMEM, s>>>(
         P.as<double>(), it, n, ctr, gpad.as<double>(), ulist.as<double>(), p.Npad, rw ? 1 : 0, K, nst, stage_bytes,
-        state.as<KfState>(), ws.as<double>());
+        state.as<KfState>(), ws.as<double>(), it2, n2, ctr2);
   FEKF_LAUNCH_CHECK();
   count_launch();
   if (tp) FEKF_CHECK_CUDA(cudaEventRecordWithFlags(tp->b, s, capturing ? cudaEventRecordExternal : cudaEventRecordDefault));
@@ -847,7 +862,10 @@ fekf_status Kf::pass(const double* g, bool rw, cudaStream_t s, cudaEvent_t ready
                                                            off_d.as<long long>(), n_d.as<int>(), p0, p.Npad);
     FEKF_LAUNCH_CHECK();
     count_launch();
-    FEKF_TRY(pass_launch(rw, 0, p.n_early, counter2.as<int>(), std::min(p.n_early, split_sms), side));
+    FEKF_CHECK_CUDA(cudaMemsetAsync(counter2.p, 0, sizeof(int), side));
+    FEKF_CHECK_CUDA(cudaEventRecord(ev_ctr, side));   // the late launch below shares counter2
+    FEKF_TRY(pass_launch(rw, 0, p.n_early, counter2.as<int>(), std::min(p.n_early, split_sms), side, 0, 0, 0, nullptr,
+                         false));
     FEKF_CHECK_CUDA(cudaEventRecord(ev_early, side));
     if (dl)
       FEKF_CHECK_CUDA(cudaEventRecordWithFlags((*dl)[di].b, s, capturing ? cudaEventRecordExternal : cudaEventRecordDefault));
@@ -858,9 +876,11 @@ fekf_status Kf::pass(const double* g, bool rw, cudaStream_t s, cudaEvent_t ready
       FEKF_LAUNCH_CHECK();
       count_launch();
     }
-    if (n_items > p.n_early)
-      FEKF_TRY(pass_launch(rw, p.n_early, n_items - p.n_early, counter.as<int>(),
-                           std::min(n_items - p.n_early, num_sms()), s, 1));
+    FEKF_CHECK_CUDA(cudaStreamWaitEvent(s, ev_ctr, 0));
+    // the late launch takes the late items, then helps finish the early launch's unclaimed items on the
+    // SMs the reverse pass has released (shared counter; every item's partials go to its fixed slots)
+    FEKF_TRY(pass_launch(rw, p.n_early, n_items - p.n_early, counter.as<int>(), num_sms(), s, 1, 0, p.n_early,
+                         counter2.as<int>()));
     FEKF_CHECK_CUDA(cudaStreamWaitEvent(s, ev_early, 0));
   } else {
     kf_pad_kernel<<<cdiv(p.Npad, tb), tb, 0, s>>>(g, gpad.as<double>(), tc_blk.as<int>(), tc_c.as<int>(),

@@ -105,10 +105,11 @@ struct Kf {
   // producer finishes the late blocks' gradient; the late items follow on `s`.
   int late_blocks = 0, split_sms = 0;
   cudaStream_t side = nullptr;
-  cudaEvent_t ev_early = nullptr;
+  cudaEvent_t ev_early = nullptr, ev_ctr = nullptr;
   DBuf counter2;
   fekf_status pass(const double* g, bool rw, cudaStream_t s, cudaEvent_t ready = nullptr);
-  fekf_status pass_launch(bool rw, int i0, int n, int* ctr, int grid, cudaStream_t s, int part = 0);
+  fekf_status pass_launch(bool rw, int i0, int n, int* ctr, int grid, cudaStream_t s, int part = 0, int i2 = 0,
+                          int n2 = 0, int* ctr2 = nullptr, bool zero_ctr = true);
   fekf_status update(const double* g, const double* abe, double sqrt_bs, double* w, cudaStream_t s,
                      cudaEvent_t ready = nullptr);
   // update = begin (P pass: this rank's partial u) + all-reduce of u over ranks + end (A, K, w, lambda)

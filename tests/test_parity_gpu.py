@@ -244,6 +244,41 @@ def test_train_steps(name, steps, precision):
         assert rel(ctx.kf.get_block(b).cpu(), st.P[b]) < tol
 
 
+def test_train_steps_split_pass():
+    """The split P pass (one GPU: the force updates' fitting-block pass overlaps the reverse pass on a side
+    stream; the late launch takes the embedding blocks, then steals the early launch's unclaimed items):
+    c1_cu32 with N_b = 1024 has the embedding parameters in block 0 and fitting-only blocks after it, so
+    the split is active.  8 minibatch steps in graph mode (crossing read-write passes, p_defer 3) match
+    the oracle at rel 1e-9 (w, every block of P)."""
+    wl = get_config("c1_cu32")
+    m = wl.model
+    opt = type(wl.opt)(**{**wl.opt.__dict__, "block_size": 1024, "p_defer": 3})
+    ds = make_dataset("c1_cu32", wl.batch * 2)
+    na = len(ds["types"])
+    w0 = init_weights(m, 3, float(ds["energy"].mean() / na))
+    B = wl.batch
+    _, blocks = fk.plan_layout(m, 1024)
+    assert len(blocks) > 2
+    ctx = fk.Context(m, opt, types=ds["types"], local_batch=B, global_batch=B)
+    ctx.set_params(cu(w0))
+    st = O.FEKF.create(w0, m, opt)
+    ctx.kf.timing(True)
+    for step in range(8):
+        sl = slice((step % 2) * B, (step % 2) * B + B)
+        groups = force_groups(na, step, 17, opt.force_groups, opt.atoms_per_group)
+        ctx.train_step(cu(ds["coord"][sl]), cu(ds["box"][sl]), cu(ds["energy"][sl]), cu(ds["force"][sl]),
+                       cu(groups, torch.int32))
+        O.train_step(st, ds["coord"][sl], ds["box"][sl], ds["types"], ds["energy"][sl], ds["force"][sl],
+                     groups, m, opt)
+    torch.cuda.synchronize()
+    ctx.kf.timing(False)
+    parts = ctx.kf.timing_parts()
+    assert parts[1] > 0.0            # late launches ran: the split was active
+    assert rel(ctx.get_params().cpu(), st.w) < 1e-9
+    for b in range(len(st.blocks)):
+        assert rel(ctx.kf.get_block(b).cpu(), st.P[b]) < 1e-9
+
+
 def test_step_graph_matches_eager():
     """a10: the captured step graph (default) and eager launches give the same weights, P and metrics
     (up to the order of the force-scatter atomics) across graph variants (p_defer 2: read-write passes at different updates of a step), and
