@@ -64,7 +64,9 @@ def load_peaks():
 # clocks sampled during the timed region (B200_PROFILING.md clocks line)
 # ---------------------------------------------------------------------------------------------
 class Clocks:
-    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,clocks_event_reasons.hw_slowdown,"
+    # started before the warm-up (nvidia-smi's own start-up touches the driver for a few hundred ms and
+    # must not overlap the timed region); only the samples stamped inside [mark(), stop()) are kept
+    Q = ("timestamp,index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,clocks_event_reasons.hw_slowdown,"
          "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
          "clocks_event_reasons.sw_power_cap")
 
@@ -77,7 +79,13 @@ class Clocks:
         except Exception:
             self.p = None
 
+    def mark(self):
+        import datetime
+        self.t0 = datetime.datetime.now()
+
     def stop(self):
+        import datetime
+        t1 = datetime.datetime.now()
         if self.p is None:
             return None
         self.p.terminate()
@@ -90,8 +98,13 @@ class Clocks:
         with open(self.f.name) as f:
             for line in f:
                 parts = [x.strip() for x in line.split(",")]
-                if len(parts) >= 9:
-                    rows.append(parts)
+                if len(parts) >= 10:
+                    try:
+                        ts = datetime.datetime.strptime(parts[0], "%Y/%m/%d %H:%M:%S.%f")
+                    except ValueError:
+                        continue
+                    if getattr(self, "t0", None) is None or self.t0 <= ts <= t1:
+                        rows.append(parts[1:])
         os.unlink(self.f.name)
         if not rows:
             return None
@@ -203,11 +216,13 @@ def run_fekf(args, rank, world, local):
         h = s % 2
         ctx.train_step(coord[h], box[h], elab[h], flab[h], fidx[s], metrics)
 
+    clocks = Clocks(local)
     for s in range(args.warmup):
         step(s)
     torch.cuda.synchronize()
     barrier()
-    clocks = Clocks(local)
+    time.sleep(0.4)   # sampler running at its 200 ms period
+    clocks.mark()
     ctx.kf.timing(True)
     stream = torch.cuda.current_stream()
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
