@@ -530,6 +530,8 @@ static fekf_status step_graph(Ctx& c, StepGraph** out) {
       c.graphs.erase(key);
       FEKF_CHECK_CUDA(e);
     }
+    // upload now (setup), not at the graph's first launch inside the step loop
+    FEKF_CHECK_CUDA(cudaGraphUpload(G.exec, c.gstream));
   }
   *out = &G;
   return FEKF_OK;
