@@ -605,3 +605,43 @@ def test_naive_sharded_ranks(world):
         assert rel(full.cpu(), st.P[b]) < 1e-12
     with pytest.raises(fk.FekfError):
         kfs[0].update_naive_end(ad, ws[0])        # end without begin
+
+
+@pytest.mark.parametrize("rcut", [0.5, 1.2])
+def test_degenerate_neighbourhoods(rcut):
+    """Edge cases of the method's input: r_c = 0.5 A leaves every atom without neighbours (no embedding
+    rows at all: D = 0, E_i = F(0), F = 0, the embedding-net gradients are 0); r_c = 1.2 A keeps only the
+    O-H bonds (H atoms: one neighbour, no same-type neighbour, ragged per-type sections).  Forward, both
+    Jacobians and one training step match the oracle."""
+    wl = get_config("t2_tiny")
+    m = type(wl.model)(**{**wl.model.__dict__, "rcut": rcut, "rcut_smth": rcut / 2})
+    ds = make_dataset("t2_tiny", 2)
+    w = init_weights(m, 3, float(ds["energy"].mean() / len(ds["types"])))
+    ctx = fk.Context(m, wl.opt, types=ds["types"], local_batch=2, global_batch=2)
+    ctx.set_params(cu(w))
+    rj, rs, _ = O.build_nlist(ds["coord"], ds["box"], ds["types"], m.rcut, m.sel)
+    nv = int((rj >= 0).sum())
+    assert (nv == 0) if rcut < 0.9 else (0 < nv < rj.size // 4)
+    ea, e, f, v = ctx.forward(cu(ds["coord"]), cu(ds["box"]))
+    Ea, E, F, V = O.energy_force_virial(w, ds["coord"], ds["box"], ds["types"], rj, rs, m)
+    assert rel(e.cpu(), E) < 1e-12 and rel(ea.cpu(), Ea) < 1e-12
+    if nv == 0:
+        assert float(f.abs().max()) == 0.0 and float(v.abs().max()) == 0.0
+    else:
+        assert rel(f.cpu(), F) < 1e-12 and rel(v.cpu().reshape(-1, 3, 3), V) < 1e-12
+    g, s = ctx.energy_jacobian(cu(ds["coord"]), cu(ds["box"]), cu(ds["energy"]))
+    gr, sr, _ = O.energy_grad(w, ds["coord"], ds["box"], ds["types"], rj, rs, ds["energy"], m)
+    assert rel(g.cpu(), gr) < 1e-11
+    atoms = force_groups(len(ds["types"]), 0, 5)[0]
+    g, s = ctx.force_jacobian(cu(ds["coord"]), cu(ds["box"]), cu(ds["force"]), cu(atoms, torch.int32))
+    gr, sr, _ = O.force_grad(w, ds["coord"], ds["box"], ds["types"], rj, rs, ds["force"], atoms, m)
+    if nv == 0:
+        assert float(g.abs().max()) == 0.0 and float(np.abs(gr).max()) == 0.0
+    else:
+        assert rel(g.cpu(), gr) < 1e-11
+    st = O.FEKF.create(w, m, wl.opt)
+    groups = force_groups(len(ds["types"]), 0, 17, wl.opt.force_groups, wl.opt.atoms_per_group)
+    met = ctx.train_step(cu(ds["coord"]), cu(ds["box"]), cu(ds["energy"]), cu(ds["force"]), cu(groups, torch.int32))
+    O.train_step(st, ds["coord"], ds["box"], ds["types"], ds["energy"], ds["force"], groups, m, wl.opt)
+    assert np.all(np.isfinite(met.cpu().numpy()))
+    assert rel(ctx.get_params().cpu(), st.w) < 1e-9
