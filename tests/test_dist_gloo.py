@@ -4,7 +4,9 @@
   * the early reduction: per-rank gradient/error sums all-reduced over ranks equal the
     single-process sums over the whole minibatch (oracle, fp64);
   * sharded P: per-rank partial u from the rank's own packed tiles (row + transposed contributions),
-    all-reduced, equals P g — the exchange the CUDA path does with ncclAllReduce.
+    all-reduced, equals P g — the exchange the CUDA path does with ncclAllReduce;
+  * Naive-EKF over ranks: all-gathered per-sample gradients, all-reduced partial U, per-rank rank-n
+    correction of the owned tiles == oracle.NaiveEKF on the global samples.
 """
 import os
 import socket
@@ -109,6 +111,57 @@ def _worker(rank, port, q):
         ref = np.concatenate([Ps[b] @ gv[off[b]:off[b + 1]] for b in range(len(blocks))])
         res["sharded_u"] = float(np.abs(ut.numpy() - ref).max() / np.abs(ref).max())
         res["mine"] = mine
+
+        # 4. Naive-EKF over ranks (readings N1-N4): each rank's local samples' gradients and
+        #    errors are all-gathered, the partial U = P G of the rank's tiles is all-reduced (instead of
+        #    the paper's P all-reduce), then every rank applies the same w step and the rank-n correction
+        #    to its own tiles; equals oracle.NaiveEKF over the global samples
+        lam, L = 0.98, len(blocks)
+        Gl = rng.standard_normal((2, sum(blocks))) + rank      # this rank's 2 samples (differ per rank)
+        al = np.abs(rng.standard_normal(2)) + 0.1 * rank
+        Gt = [torch.zeros(2, sum(blocks), dtype=torch.float64) for _ in range(WORLD)]
+        At = [torch.zeros(2, dtype=torch.float64) for _ in range(WORLD)]
+        dist.all_gather(Gt, torch.tensor(Gl))
+        dist.all_gather(At, torch.tensor(al))
+        G = torch.cat(Gt).numpy()
+        ab = torch.cat(At).numpy()
+        nS = len(G)
+        U = np.zeros((sum(blocks), nS))
+        for (b, I, J), ow in zip(_tiles(blocks), owner):
+            if ow != rank:
+                continue
+            n = blocks[b]
+            r0, r1 = I * TILE, min(n, (I + 1) * TILE)
+            c0, c1 = J * TILE, min(n, (J + 1) * TILE)
+            if r0 >= n or c0 >= n:
+                continue
+            Pt = Ps[b][r0:r1, c0:c1]
+            U[off[b] + r0:off[b] + r1] += Pt @ G[:, off[b] + c0:off[b] + c1].T
+            if I != J:
+                U[off[b] + c0:off[b] + c1] += Pt.T @ G[:, off[b] + r0:off[b] + r1].T
+        Ut = torch.tensor(U)
+        dist.all_reduce(Ut)
+        U = Ut.numpy()
+        A = 1.0 / (L * lam + np.einsum("pi,ip->i", U, G))
+        dw = U @ (ab * A) / nS
+        st = O.NaiveEKF(np.zeros(sum(blocks)), blocks, lam=lam, nu=0.9987)
+        st.P = [P.copy() for P in Ps]
+        A_ref = st.update_naive(list(G), list(ab))
+        res["naive_A"] = float(np.abs(A - np.array(A_ref)).max() / np.abs(A_ref).max())
+        res["naive_w"] = float(np.abs(dw - st.w).max() / np.abs(st.w).max())
+        err = 0.0
+        for (b, I, J), ow in zip(_tiles(blocks), owner):
+            if ow != rank:
+                continue
+            n = blocks[b]
+            r0, r1 = I * TILE, min(n, (I + 1) * TILE)
+            c0, c1 = J * TILE, min(n, (J + 1) * TILE)
+            if r0 >= n or c0 >= n:
+                continue
+            Ub = U[off[b]:off[b + 1]]
+            Pn = (Ps[b][r0:r1, c0:c1] - (Ub[r0:r1] * (A / nS)) @ Ub[c0:c1].T) / lam
+            err = max(err, float(np.abs(Pn - st.P[b][r0:r1, c0:c1]).max() / np.abs(st.P[b]).max()))
+        res["naive_P"] = err
         q.put((rank, res))
         dist.destroy_process_group()
     except Exception as e:  # pragma: no cover
@@ -133,3 +186,4 @@ def test_gloo_world2():
         assert res["err_sum"] < 1e-13
         assert res["sharded_u"] < 1e-12
         assert res["mine"] > 0
+        assert res["naive_A"] < 1e-12 and res["naive_w"] < 1e-12 and res["naive_P"] < 1e-12
