@@ -64,28 +64,69 @@ def load_peaks():
 # clocks sampled during the timed region (B200_PROFILING.md clocks line)
 # ---------------------------------------------------------------------------------------------
 class Clocks:
-    # started before the warm-up (nvidia-smi's own start-up touches the driver for a few hundred ms and
-    # must not overlap the timed region); only the samples stamped inside [mark(), stop()) are kept
-    Q = ("timestamp,index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,clocks_event_reasons.hw_slowdown,"
-         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
-         "clocks_event_reasons.sw_power_cap")
+    """SM clock and clock-event reasons sampled every 20 ms by an NVML thread (nvidia_ml_py) between mark()
+    and stop() — the timed region; initialised before the warm-up so NVML's start-up never overlaps it.
+    Falls back to an `nvidia-smi -lms 100` subprocess when NVML is unavailable."""
+    REASONS = (("hw_slowdown", 0x8), ("hw_thermal_slowdown", 0x40), ("sw_thermal_slowdown", 0x20),
+               ("sw_power_cap", 0x4))
 
     def __init__(self, index):
+        import threading
         self.index = index
-        self.f = tempfile.NamedTemporaryFile("w+", suffix=".csv", delete=False)
+        self.rows = []
+        self.on = False
+        self.stop_ev = threading.Event()
+        self.nv = None
+        self.p = None
         try:
-            self.p = subprocess.Popen(["nvidia-smi", "-i", str(index), f"--query-gpu={self.Q}", "--format=csv,noheader,nounits",
-                                       "-lms", "200"], stdout=self.f, stderr=subprocess.DEVNULL)
+            import pynvml
+            pynvml.nvmlInit()
+            self.nv = pynvml
+            self.h = pynvml.nvmlDeviceGetHandleByIndex(index)
+            self.max_mhz = float(pynvml.nvmlDeviceGetMaxClockInfo(self.h, pynvml.NVML_CLOCK_SM))
+            self.t = threading.Thread(target=self._run, daemon=True)
+            self.t.start()
         except Exception:
-            self.p = None
+            self.nv = None
+            self.f = tempfile.NamedTemporaryFile("w+", suffix=".csv", delete=False)
+            q = ("timestamp,clocks.sm,clocks.max.sm,clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+                 "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+            try:
+                self.p = subprocess.Popen(["nvidia-smi", "-i", str(index), f"--query-gpu={q}",
+                                           "--format=csv,noheader,nounits", "-lms", "100"],
+                                          stdout=self.f, stderr=subprocess.DEVNULL)
+            except Exception:
+                self.p = None
+
+    def _run(self):
+        while not self.stop_ev.is_set():
+            if self.on:
+                try:
+                    sm = float(self.nv.nvmlDeviceGetClockInfo(self.h, self.nv.NVML_CLOCK_SM))
+                    rs = int(self.nv.nvmlDeviceGetCurrentClocksEventReasons(self.h))
+                    self.rows.append((sm, rs))
+                except Exception:
+                    pass
+            self.stop_ev.wait(0.02)
 
     def mark(self):
         import datetime
         self.t0 = datetime.datetime.now()
+        self.on = True
 
     def stop(self):
         import datetime
         t1 = datetime.datetime.now()
+        self.on = False
+        if self.nv is not None:
+            self.stop_ev.set()
+            self.t.join(1.0)
+            if not self.rows:
+                return None
+            sm = [r[0] for r in self.rows]
+            reasons = sorted({n for _, m in self.rows for n, bit in self.REASONS if m & bit})
+            return {"sm_mhz": statistics.median(sm), "sm_max_mhz": self.max_mhz, "reasons": reasons,
+                    "samples": len(self.rows), "source": "nvml, 20 ms"}
         if self.p is None:
             return None
         self.p.terminate()
@@ -98,7 +139,7 @@ class Clocks:
         with open(self.f.name) as f:
             for line in f:
                 parts = [x.strip() for x in line.split(",")]
-                if len(parts) >= 10:
+                if len(parts) >= 7:
                     try:
                         ts = datetime.datetime.strptime(parts[0], "%Y/%m/%d %H:%M:%S.%f")
                     except ValueError:
@@ -108,12 +149,12 @@ class Clocks:
         os.unlink(self.f.name)
         if not rows:
             return None
-        sm = [float(r[1]) for r in rows if r[1].replace(".", "").isdigit()]
-        mx = [float(r[2]) for r in rows if r[2].replace(".", "").isdigit()]
-        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
-        reasons = sorted({names[k] for r in rows for k in range(4) if r[5 + k].lower().startswith("active")})
+        sm = [float(r[0]) for r in rows if r[0].replace(".", "").isdigit()]
+        mx = [float(r[1]) for r in rows if r[1].replace(".", "").isdigit()]
+        names = [n for n, _ in self.REASONS]
+        reasons = sorted({names[k] for r in rows for k in range(4) if r[2 + k].lower().startswith("active")})
         return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
-                "reasons": reasons, "samples": len(rows)}
+                "reasons": reasons, "samples": len(rows), "source": "nvidia-smi, 100 ms"}
 
 
 # ---------------------------------------------------------------------------------------------
@@ -221,7 +262,6 @@ def run_fekf(args, rank, world, local):
         step(s)
     torch.cuda.synchronize()
     barrier()
-    time.sleep(0.4)   # sampler running at its 200 ms period
     clocks.mark()
     ctx.kf.timing(True)
     stream = torch.cuda.current_stream()
