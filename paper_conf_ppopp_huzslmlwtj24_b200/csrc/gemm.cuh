@@ -218,9 +218,35 @@ dgemm_kernel(const __grid_constant__ GemmGroup<Epi> G) {
   // 16-byte copies (two doubles along the contiguous dimension) when the problem's strides, bases and
   // extents keep every pair inside one row and aligned; per problem, so warp-uniform
   const bool a16 = !TA && aug_m < 0 && !(lda & 1) && !(reinterpret_cast<size_t>(A) & 15) && !(K & 1) && !(kps & 1);
+  // TA (A stored [K x M], m-contiguous): pairs (m, m+1) of real columns go as one 16-byte copy; the pair
+  // holding the last real column / the "ones" row is done element by element
+  const bool a16t = TA && !(lda & 1) && !(reinterpret_cast<size_t>(A) & 15);
+  const int mreal = aug_m >= 0 ? min(M, aug_m) : M;
   const bool b16 = !(ldb & 1) && !(reinterpret_cast<size_t>(B) & 15) && (TB ? (!(K & 1) && !(kps & 1)) : !(N & 1));
   auto issue = [&](int buf, int k0) {
-    if (a16) {
+    if (a16t) {
+#pragma unroll
+      for (int q = 0; q < AE / 2; ++q) {
+        const int idx = tid + 256 * q;
+        const int kk = idx / (BM / 2), r = 2 * (idx % (BM / 2));
+        const int m = m0 + r, k = k0 + kk;
+        const bool kin = k < kend;
+        if (m + 1 < mreal) {
+          cp_async16z(&a_at(buf, r, kk), kin ? A + (size_t)k * lda + m : A, kin);
+        } else {
+#pragma unroll
+          for (int h = 0; h < 2; ++h) {
+            double* dst = &a_at(buf, r + h, kk);
+            if (m + h == aug_m) {
+              *dst = (k < aug_k) ? 1.0 : 0.0;
+            } else {
+              const bool ok = m + h < M && kin;
+              cp_async8(dst, ok ? A + (size_t)k * lda + m + h : A, ok);
+            }
+          }
+        }
+      }
+    } else if (a16) {
 #pragma unroll
       for (int q = 0; q < AE / 2; ++q) {
         const int idx = tid + 256 * q;
