@@ -841,6 +841,42 @@ fekf_status fekf_train_step(fekf_ctx* ctx, const double* coord, const double* bo
   return FEKF_OK;
 }
 
+// One captured graph of the Naive-EKF minibatch per pending-FEKF-correction count at entry (after the
+// first naive update the count is 0, so one graph serves every later step).
+static fekf_status naive_graph(Ctx& c, StepGraph** out) {
+  Kf& k = *c.kf;
+  const int key = (1 << 20) | k.npend;
+  StepGraph& G = c.graphs[key];
+  if (!G.exec) {
+    const int npend0 = k.npend;
+    const int64_t l0 = g_launches;
+    FEKF_CHECK_CUDA(cudaStreamBeginCapture(c.gstream, cudaStreamCaptureModeRelaxed));
+    fekf_status st = naive_step_body(c, c.st_coord.as<double>(), c.st_box.as<double>(), c.st_e.as<double>(),
+                                     c.st_f.as<double>(), c.st_fidx.as<int32_t>(), c.st_met.as<double>(), c.gstream);
+    cudaGraph_t graph = nullptr;
+    cudaError_t e = cudaStreamEndCapture(c.gstream, &graph);
+    G.npend_after = k.npend;
+    G.launches = g_launches - l0;
+    k.npend = npend0;
+    g_launches = l0;
+    if (st != FEKF_OK || e != cudaSuccess) {
+      if (graph) cudaGraphDestroy(graph);
+      c.graphs.erase(key);
+      if (st != FEKF_OK) return st;
+      FEKF_CHECK_CUDA(e);
+    }
+    e = cudaGraphInstantiate(&G.exec, graph, 0);
+    cudaGraphDestroy(graph);
+    if (e != cudaSuccess) {
+      c.graphs.erase(key);
+      FEKF_CHECK_CUDA(e);
+    }
+    FEKF_CHECK_CUDA(cudaGraphUpload(G.exec, c.gstream));
+  }
+  *out = &G;
+  return FEKF_OK;
+}
+
 fekf_status fekf_naive_train_step(fekf_ctx* ctx, const double* coord, const double* box, const double* e_label,
                                   const double* f_label, const int32_t* force_idx, double* metrics, cudaStream_t s) {
   if (!ctx || !coord || !box || !e_label || !f_label || !metrics || (!force_idx && ctx->c.o.force_groups > 0)) {
@@ -852,10 +888,36 @@ fekf_status fekf_naive_train_step(fekf_ctx* ctx, const double* coord, const doub
     set_error("naive_train_step: single rank with local_batch <= 32 only");
     return FEKF_EINVAL;
   }
-  if (c.gstream) FEKF_CHECK_CUDA(cudaStreamSynchronize(c.gstream));   // earlier graph replays
-  const int64_t l0 = g_launches;
-  FEKF_TRY(naive_step_body(c, coord, box, e_label, f_label, force_idx, metrics, s));
-  c.last_launches = g_launches - l0;
+  // eager on the first call (it allocates the per-image gradient and Naive-EKF workspaces), then one
+  // captured graph per step like fekf_train_step
+  const int np_needed = c.B <= 8 ? 8 : (c.B <= 16 ? 16 : 32);   // naive.cu's vector-set width for B samples
+  if (!c.use_graph || !c.gstream || !c.naive_G.p || c.kf->naive_np < np_needed) {
+    if (c.gstream) FEKF_CHECK_CUDA(cudaStreamSynchronize(c.gstream));   // earlier graph replays
+    const int64_t l0 = g_launches;
+    FEKF_TRY(naive_step_body(c, coord, box, e_label, f_label, force_idx, metrics, s));
+    c.last_launches = g_launches - l0;
+    ++c.nsteps;
+    return FEKF_OK;
+  }
+  const size_t na3 = sizeof(double) * (size_t)c.B * c.Na * 3;
+  FEKF_CHECK_CUDA(cudaMemcpyAsync(c.st_coord.p, coord, na3, cudaMemcpyDeviceToDevice, s));
+  FEKF_CHECK_CUDA(cudaMemcpyAsync(c.st_box.p, box, sizeof(double) * c.B * 9, cudaMemcpyDeviceToDevice, s));
+  FEKF_CHECK_CUDA(cudaMemcpyAsync(c.st_e.p, e_label, sizeof(double) * c.B, cudaMemcpyDeviceToDevice, s));
+  FEKF_CHECK_CUDA(cudaMemcpyAsync(c.st_f.p, f_label, na3, cudaMemcpyDeviceToDevice, s));
+  if (c.o.force_groups > 0)
+    FEKF_CHECK_CUDA(cudaMemcpyAsync(c.st_fidx.p, force_idx, sizeof(int32_t) * c.o.force_groups * c.o.atoms_per_group,
+                                    cudaMemcpyDeviceToDevice, s));
+  StepGraph* G = nullptr;
+  FEKF_TRY(naive_graph(c, &G));
+  FEKF_CHECK_CUDA(cudaEventRecord(c.gev_in, s));
+  FEKF_CHECK_CUDA(cudaStreamWaitEvent(c.gstream, c.gev_in, 0));
+  FEKF_CHECK_CUDA(cudaGraphLaunch(G->exec, c.gstream));
+  FEKF_CHECK_CUDA(cudaEventRecord(c.gev_out, c.gstream));
+  FEKF_CHECK_CUDA(cudaStreamWaitEvent(s, c.gev_out, 0));
+  FEKF_CHECK_CUDA(cudaMemcpyAsync(metrics, c.st_met.p, sizeof(double) * 8, cudaMemcpyDeviceToDevice, s));
+  c.kf->npend = G->npend_after;
+  g_launches += G->launches;
+  c.last_launches = G->launches;
   ++c.nsteps;
   return FEKF_OK;
 }
