@@ -373,7 +373,7 @@ def run_fekf(args, rank, world, local):
         standalone = {"achieved": sa, "frac": sa / peak, "avg_launch_ms": sa_ms / sa_n, "launches": sa_n,
                       "pass": "read-only, all SMs"}
         del gs
-    split_sms = int(os.environ.get("FEKF_SPLIT_SMS", "96" if args.precision == 64 else "0")) if world == 1 else 0
+    split_sms = int(os.environ.get("FEKF_SPLIT_SMS", "96" if args.precision == 64 else "80")) if world == 1 else 0
     roof = {"kernel": "kf_pass_kernel", "bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
             "frac": (achieved / peak) if achieved else None, "traffic": traffic,
             "peak_source": peak_kind, "alg_bytes_per_launch": alg_bytes, "avg_launch_ms": avg_pass_s * 1000.0,

@@ -293,7 +293,7 @@ fekf_status Ctx::init(const fekf_model_cfg& mm, const fekf_opt_cfg& oo, int nato
     while (late < (int)blocks.size() && acc < emb_end) acc += blocks[late++];
     kf->late_blocks = late;
     const char* e = getenv("FEKF_SPLIT_SMS");
-    kf->split_sms = comm ? 0 : (e ? atoi(e) : (o.precision == 32 ? 0 : 96));   // measured defaults
+    kf->split_sms = comm ? 0 : (e ? atoi(e) : (o.precision == 32 ? 80 : 96));   // measured defaults
   }
   FEKF_TRY(kf->create(blocks, o, comm));
   if (kf->split_sms > 0) FEKF_CHECK_CUDA(cudaEventCreateWithFlags(&ev_fit, cudaEventDisableTiming));

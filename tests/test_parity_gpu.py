@@ -244,7 +244,8 @@ def test_train_steps(name, steps, precision):
         assert rel(ctx.kf.get_block(b).cpu(), st.P[b]) < tol
 
 
-def test_train_steps_split_pass():
+@pytest.mark.parametrize("precision", [64, 32])
+def test_train_steps_split_pass(precision):
     """The split P pass (one GPU: the force updates' fitting-block pass overlaps the reverse pass on a side
     stream; the late launch takes the embedding blocks, then steals the early launch's unclaimed items):
     c1_cu32 with N_b = 1024 has the embedding parameters in block 0 and fitting-only blocks after it, so
@@ -252,7 +253,8 @@ def test_train_steps_split_pass():
     the oracle at rel 1e-9 (w, every block of P)."""
     wl = get_config("c1_cu32")
     m = wl.model
-    opt = type(wl.opt)(**{**wl.opt.__dict__, "block_size": 1024, "p_defer": 3})
+    opt = type(wl.opt)(**{**wl.opt.__dict__, "block_size": 1024, "p_defer": 3, "precision": precision})
+    tol = 1e-9 if precision == 64 else 1e-4
     ds = make_dataset("c1_cu32", wl.batch * 2)
     na = len(ds["types"])
     w0 = init_weights(m, 3, float(ds["energy"].mean() / na))
@@ -274,9 +276,9 @@ def test_train_steps_split_pass():
     ctx.kf.timing(False)
     parts = ctx.kf.timing_parts()
     assert parts[1] > 0.0            # late launches ran: the split was active
-    assert rel(ctx.get_params().cpu(), st.w) < 1e-9
+    assert rel(ctx.get_params().cpu(), st.w) < tol
     for b in range(len(st.blocks)):
-        assert rel(ctx.kf.get_block(b).cpu(), st.P[b]) < 1e-9
+        assert rel(ctx.kf.get_block(b).cpu(), st.P[b]) < tol
 
 
 def test_step_graph_matches_eager():
