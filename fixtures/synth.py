@@ -41,6 +41,10 @@ class ModelConfig:
     m2: int              # M^< (16)
     fit: list            # fitting hidden widths h_1..h_F
     fit_resnet_dt: int = 1   # SURVEY §8c Z14, pinned by the 26 651 count
+    switch_kind: int = 0     # Z8: 0 = C2 quintic sw(u), 1 = cosine 0.5 cos(pi u) + 0.5
+    type_one_side: int = 0   # Z15: 0 = embedding net per (t_i, t_j), 1 = per neighbour type t_j only
+    env_avg: list = None     # Z11: per centre type [ntypes][4] shift of the R~ rows (None = 0)
+    env_std: list = None     # Z11: per centre type [ntypes][4] scale of the R~ rows (None = 1)
 
     @property
     def nm(self):
@@ -171,9 +175,12 @@ def _molecules(kind, n_side, L, rng):
 
 
 def _alloy(a, cells, ntypes, rng):
+    """Random substitutional fcc alloy: every site draws a type; atoms are then listed sorted by type
+    (stable), so the types stay spatially random while the layout convention holds."""
     pts, box, _ = _fcc(a, cells)
-    types = np.sort(rng.integers(0, ntypes, size=len(pts))).astype(np.int32)
-    return pts, box, types
+    t = rng.integers(0, ntypes, size=len(pts))
+    order = np.argsort(t, kind="stable")
+    return pts[order], box, t[order].astype(np.int32)
 
 
 def build_lattice(spec: SystemSpec, rng):
@@ -340,15 +347,17 @@ def make_dataset(name, n_images=None, seed=None, split="train", labels=True):
 # parameters (flat vector in the layout order of SURVEY §8c step 1; random init Z17)
 # ----------------------------------------------------------------------------------------------
 def tensor_shapes(m: ModelConfig):
-    """[(name, shape)] in storage order: embedding nets (ti,tj) lexicographic, then fitting nets."""
+    """[(name, shape)] in storage order: embedding nets (ti,tj) lexicographic (or per tj with
+    type_one_side), then fitting nets."""
     out = []
-    for ti in range(m.ntypes):
-        for tj in range(m.ntypes):
-            prev = 1
-            for l, d in enumerate(m.emb):
-                out.append((f"emb{ti}{tj}.W{l}", (prev, d)))
-                out.append((f"emb{ti}{tj}.b{l}", (d,)))
-                prev = d
+    nets = [f"{tj}" for tj in range(m.ntypes)] if getattr(m, "type_one_side", 0) else \
+        [f"{ti}{tj}" for ti in range(m.ntypes) for tj in range(m.ntypes)]
+    for nm in nets:
+        prev = 1
+        for l, d in enumerate(m.emb):
+            out.append((f"emb{nm}.W{l}", (prev, d)))
+            out.append((f"emb{nm}.b{l}", (d,)))
+            prev = d
     for ti in range(m.ntypes):
         prev = m.M * m.m2
         for l, h in enumerate(m.fit):

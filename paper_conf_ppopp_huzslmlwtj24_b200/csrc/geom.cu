@@ -51,6 +51,15 @@ nlist_kernel(const double* __restrict__ coord, const double* __restrict__ box, c
   }
   __syncthreads();
   const int ma = s_m[0], mb = s_m[1], mc = s_m[2];
+  if (ma > SHIFT_OFF || mb > SHIFT_OFF || mc > SHIFT_OFF) {
+    // periodic images beyond the shift-id encoding (|n| <= 7; r_c more than 7 face spacings): the list is
+    // left empty and the fault flag raised (metrics[7] bit 2) instead of mis-decoded shifts
+    if (tid == 0) atomicOr(err_flag, 2);
+    int* oj = nl_j + ((size_t)b * Na + i) * Nm;
+    int* os = nl_s + ((size_t)b * Na + i) * Nm;
+    for (int p = tid; p < Nm; p += NL_THREADS) { oj[p] = -1; os[p] = -1; }
+    return;
+  }
   const int na_ = 2 * ma + 1, nb_ = 2 * mb + 1, nc_ = 2 * mc + 1;
   const long long nshift = (long long)na_ * nb_ * nc_;
   const double* xi = coord + ((size_t)b * Na + i) * 3;

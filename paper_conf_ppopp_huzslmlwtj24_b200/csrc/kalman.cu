@@ -523,16 +523,20 @@ __global__ void kf_finish_kernel(const double* __restrict__ dblk, int L, int K, 
     const double A = 1.0 / (st->c_mult * lam + gtu);
     const double e = abe ? *abe : 0.0;
     const int slot = rw ? 0 : st->npend;
+    // a non-finite A or ABE (a bad batch) makes the update a no-op apart from the latched flag: the
+    // deferred slot holds a zero correction (kf_vec_kernel stores u = 0 there), w, sigma and lambda stay
+    const bool bad = !isfinite(A) || !isfinite(e);
+    st->skip = bad ? 1 : 0;
     st->sig_cur = sig;
     st->A_last = A;
-    st->coef_w = sqrt_bs * e * A;
+    st->coef_w = bad ? 0.0 : sqrt_bs * e * A;
     st->slot = slot;
-    st->beta[slot] = A / sig;
+    st->beta[slot] = bad ? 0.0 : A / sig;
     st->npend = slot + 1;
-    st->sigma = sig / lam;
-    st->lambda = lam * st->nu + 1.0 - st->nu;
+    st->sigma = bad ? sig : sig / lam;
+    if (!bad) st->lambda = lam * st->nu + 1.0 - st->nu;
     st->t += 1;
-    if (!isfinite(A) || !isfinite(e)) st->flags |= 2;
+    if (bad) st->flags |= 2;
   }
 }
 
@@ -544,6 +548,10 @@ __global__ void kf_vec_kernel(const double* __restrict__ ub, double* __restrict_
   if (p >= npad) return;
   const long long tc = p / KT;
   const int b = tc_blk[tc];
+  if (st->skip) {   // non-finite update: zero correction, w untouched
+    ulist[(size_t)st->slot * npad + p] = 0.0;
+    return;
+  }
   double v = ub[p];
   for (int k = 0; k < K; ++k) v -= cub[(size_t)k * L + b] * ulist[(size_t)k * npad + p];
   v *= st->sig_cur;
@@ -829,6 +837,7 @@ fekf_status Kf::pass_launch(bool rw, int i0, int n, int* ctr, int grid, cudaStre
 }
 
 fekf_status Kf::pass(const double* g, bool rw, cudaStream_t s, cudaEvent_t ready) {
+  FEKF_TRY(idle_check("kf_pass"));
   const KfPlan& p = plan;
   const int tb = 256;
   const int n_items = (int)p.items.size();
@@ -942,7 +951,16 @@ fekf_status Kf::update_end(const double* abe, double sqrt_bs, double* w, cudaStr
   return FEKF_OK;
 }
 
+fekf_status Kf::idle_check(const char* what) const {
+  if (in_update || naive_n > 0) {
+    set_error(std::string(what) + ": not allowed between an update's begin and end");
+    return FEKF_ESTATE;
+  }
+  return FEKF_OK;
+}
+
 fekf_status Kf::flush(cudaStream_t s) {
+  FEKF_TRY(idle_check("kf_flush"));
   if (!plan.items.empty() && npend > 0) {
     if (p32)
       kf_apply_pending_kernel<<<(unsigned)plan.items.size(), 256, 0, s>>>(P.as<float>(), items_d.as<ItemD>(),
@@ -962,6 +980,7 @@ fekf_status Kf::flush(cudaStream_t s) {
 
 fekf_status Kf::get_block(int b, double* dst, cudaStream_t s) {
   if (b < 0 || b >= plan.L) { set_error("get_block: bad block"); return FEKF_EINVAL; }
+  FEKF_TRY(idle_check("kf_get_block"));
   if (plan.items.empty()) return FEKF_OK;
   const unsigned nit = (unsigned)plan.items.size();
   if (p32)

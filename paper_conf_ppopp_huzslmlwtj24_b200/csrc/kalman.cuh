@@ -29,7 +29,7 @@ struct KfState {
   double sig_cur;              // sigma used to form the current u
   double beta[KMAX];           // deferred coefficients
   long long t;
-  int npend, flags, slot, pad_;
+  int npend, flags, slot, skip;   // skip: the last update saw a non-finite A / ABE (no-op)
 };
 
 struct KfPlan {
@@ -117,6 +117,7 @@ struct Kf {
   fekf_status update_begin(const double* g, cudaStream_t s, cudaEvent_t ready = nullptr);
   fekf_status update_end(const double* abe, double sqrt_bs, double* w, cudaStream_t s);
   fekf_status flush(cudaStream_t s);
+  fekf_status idle_check(const char* what) const;   // FEKF_ESTATE between an update's begin and end
   fekf_status get_block(int b, double* dst, cudaStream_t s);
   fekf_status set_block(int b, const double* src, cudaStream_t s);
   fekf_status get_state(double* lambda, double* A_last, int* flags);

@@ -225,8 +225,9 @@ __global__ void nkf_state_kernel(KfState* st, double* __restrict__ coef, int n) 
   for (int j = 0; j < n; ++j) ok = ok && isfinite(coef[64 + j]) && isfinite(coef[32 + j]);
   const double lam = st->lambda;
   coef[96] = 1.0 / lam;
+  coef[97] = ok ? 0.0 : 1.0;   // a non-finite A_i / ABE_i: the update is a no-op (w, P, lambda kept)
   st->A_last = coef[64 + n - 1];
-  st->lambda = lam * st->nu + 1.0 - st->nu;
+  if (ok) st->lambda = lam * st->nu + 1.0 - st->nu;
   st->t += 1;
   if (!ok) st->flags |= 2;
 }
@@ -241,7 +242,7 @@ __global__ void nkf_vec_kernel(const double* __restrict__ U, const double* __res
   const long long tc = p / KT;
   const int b = tc_blk[tc];
   const int loc = tc_c[tc] * KT + (int)(p % KT);
-  if (loc >= nblk[b]) return;
+  if (loc >= nblk[b] || coef[97] != 0.0) return;
   double v = 0.0;
   for (int j = 0; j < n; ++j) v = fma(coef[32 + j], U[(size_t)p * NP + j], v);
   w[off[b] + loc] += v;
@@ -258,6 +259,7 @@ nkf_correct_kernel(double* __restrict__ P, const ItemD* __restrict__ items, cons
   double* const sUI = smc;                              // [KT * LDG]
   double (*sUJ)[KT * LDG] = reinterpret_cast<double (*)[KT * LDG]>(smc + KT * LDG);   // [2][KT * LDG]
   __shared__ double sc[NP];
+  if (coef[97] != 0.0) return;   // non-finite update (nkf_state_kernel): P untouched
   const ItemD it = items[blockIdx.x];
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31, fr = lane >> 2, fk = lane & 3;
   const int m0 = 8 * warp;

@@ -833,22 +833,20 @@ __global__ void energy_scatter_kernel(Geo g, FitPtrs fp, double* __restrict__ ea
 }
 
 // energy update errors (Alg. 1 lines 3-6): e_b = (Y_b - E_b)/N_a, flip when E_b >= Y_b; seeds s_b/N_a
+// (any local batch: the seed of row r is formed from its image's energy directly, no per-image staging)
 __global__ void energy_error_kernel(Geo g, FitPtrs fp, const double* __restrict__ etot, const double* __restrict__ label,
                                     double seed_scale, double* __restrict__ abs_sum) {
-  __shared__ double sb[1024];
   if (threadIdx.x == 0) {
     double a = 0.0;
-    for (int b = 0; b < g.nb; ++b) {
-      const double E = etot[b], Y = label[b];
-      a += fabs((Y - E) / g.Na);
-      sb[b] = (E >= Y ? -1.0 : 1.0) * seed_scale / g.Na;
-    }
+    for (int b = 0; b < g.nb; ++b) a += fabs((label[b] - etot[b]) / g.Na);
     *abs_sum = a;
   }
-  __syncthreads();
   for (int t = 0; t < g.nt; ++t) {
     const long long F = (long long)g.nb * g.ncnt[t];
-    for (long long r = threadIdx.x; r < F; r += blockDim.x) fp.ebar[t][r] = sb[r / g.ncnt[t]];
+    for (long long r = threadIdx.x; r < F; r += blockDim.x) {
+      const long long b = r / g.ncnt[t];
+      fp.ebar[t][r] = (etot[b] >= label[b] ? -1.0 : 1.0) * seed_scale / g.Na;
+    }
   }
 }
 

@@ -13,7 +13,7 @@ test split every `--every` steps.  The target is the best (lowest) RMSE the orac
 S_o steps (reading R1 of DESIGN.md: the EKF trajectory is not monotone, so "the oracle's RMSE after S_o
 steps" is taken as the best one it attained), with the step it first reached it.
 
-  python tools/make_rmse_target.py [--config c1_cu32] [--steps 64] [--every 8]
+  python tools/make_rmse_target.py [--config c1_cu32] [--steps 200] [--every 8] [--threads N] [--out PATH]
 """
 import argparse
 import json
@@ -35,8 +35,10 @@ def main():
     ap.add_argument("--config", default="c1_cu32")
     ap.add_argument("--steps", type=int, default=64)
     ap.add_argument("--every", type=int, default=8)
+    ap.add_argument("--threads", type=int, default=0)
+    ap.add_argument("--out", default="")
     args = ap.parse_args()
-    torch.set_num_threads(os.cpu_count() or 1)
+    torch.set_num_threads(args.threads or os.cpu_count() or 1)
     wl = get_config(args.config)
     m, opt = wl.model, wl.opt
     tr = make_dataset(args.config, split="train")
@@ -73,7 +75,7 @@ def main():
         "target_step": min(traj, key=lambda x: x[1] + x[2])[0], "final": traj[-1][1] + traj[-1][2],
         "oracle_train_seconds": train_s, "oracle_threads": torch.get_num_threads(),
     }
-    path = os.path.join(ROOT, "tests", "golden", f"rmse_{args.config}.json")
+    path = args.out or os.path.join(ROOT, "tests", "golden", f"rmse_{args.config}.json")
     with open(path, "w") as f:
         json.dump(out, f, indent=1)
     print("wrote", path, "target", out["target"])
