@@ -149,8 +149,10 @@ def random_rotation(rng):
 
 
 def _molecules(kind, n_side, L, rng):
-    """Molecules on an n_side^3 grid with random orientations. Heavy atoms first (type 0)."""
-    sp = L / n_side
+    """Molecules on an n_side^3 grid (or an (nx, ny, nz) grid of spacing L / n_side[0]) with random
+    orientations. Heavy atoms first (type 0)."""
+    grid = tuple(n_side) if isinstance(n_side, (tuple, list)) else (n_side, n_side, n_side)
+    sp = L / grid[0]
     heavy, light = [], []
     if kind == "water":
         roh, ang = 0.9572, math.radians(104.52)
@@ -161,9 +163,9 @@ def _molecules(kind, n_side, L, rng):
         local = rch * t / math.sqrt(3.0)
     else:
         raise ValueError(kind)
-    for i in range(n_side):
-        for j in range(n_side):
-            for k in range(n_side):
+    for i in range(grid[0]):
+        for j in range(grid[1]):
+            for k in range(grid[2]):
                 c = (np.array([i, j, k], dtype=np.float64) + 0.5) * sp
                 rot = random_rotation(rng)
                 heavy.append(c)
@@ -171,7 +173,7 @@ def _molecules(kind, n_side, L, rng):
                     light.append(c + rot @ v)
     pts = np.concatenate([np.array(heavy), np.array(light)], axis=0)
     types = np.concatenate([np.zeros(len(heavy)), np.ones(len(light))]).astype(np.int32)
-    return pts, np.diag([L, L, L]).astype(np.float64), types
+    return pts, np.diag([sp * g for g in grid]).astype(np.float64), types
 
 
 def _alloy(a, cells, ntypes, rng):
@@ -260,6 +262,19 @@ def lj_energy_forces(coord, box, types, lj, rc):
 _CU_LJ = {(0, 0): (0.4093, 2.338)}
 _WATER_LJ = {(0, 0): (0.0067, 3.166), (0, 1): (0.2, 0.855), (1, 1): (0.05, 1.35)}
 _CH4_LJ = {(0, 0): (0.0045, 3.4), (0, 1): (0.2, 0.971), (1, 1): (0.01, 1.6)}
+_AL_LJ = {(0, 0): (0.392, 2.551)}                  # minimum at 2^(1/6) sigma = 2.864 A = a/sqrt(2)
+_SI_LJ = {(0, 0): (0.30, 2.094)}                   # minimum at the Si-Si bond, 2.351 A
+_MG_LJ = {(0, 0): (0.20, 2.860)}                   # minimum at a = 3.21 A
+_NACL_LJ = {(0, 0): (0.0115, 2.58), (0, 1): (0.10, 2.512), (1, 1): (0.0128, 4.40)}   # Na-Cl min at a/2
+
+
+def _lorentz_berthelot(eps, sig):
+    """Pair (eps_ij, sigma_ij) = (sqrt(eps_i eps_j), (sigma_i + sigma_j)/2) for every type pair."""
+    n = len(eps)
+    return {(i, j): (math.sqrt(eps[i] * eps[j]), 0.5 * (sig[i] + sig[j])) for i in range(n) for j in range(i, n)}
+
+
+_ALLOY_LJ = _lorentz_berthelot([0.40, 0.30, 0.35, 0.45], [2.30, 2.40, 2.45, 2.55])
 
 
 def _workloads():
@@ -296,6 +311,40 @@ def _workloads():
         SystemSpec("H2O-8", "water", {"n_side": 2, "L": 6.21}, sigma=0.05, lj=_WATER_LJ, lj_cut=4.0),
         ModelConfig(2, 4.0, 1.0, [12, 24], [4, 8, 16], 3, [16, 16]),
         batch=3, n_train=12, n_test=4, seed=SEED_BASE + 6)
+    # ---- C4: the 8-system sweep shaped like the paper's Table 3: atom counts of
+    # the paper's datasets, perturbed lattices with LJ (Lorentz-Berthelot) labels, C2's nets
+    c2_emb, c2_fit = [25, 50, 100], [240, 240, 240]
+    w["c4_al32"] = Workload(
+        "c4_al32", SystemSpec("Al32", "fcc", {"a": 4.05, "cells": (2, 2, 2)}, sigma=0.10, lj=_AL_LJ, lj_cut=6.0),
+        ModelConfig(1, 6.0, 0.5, [64], c2_emb, 16, c2_fit), batch=32, n_train=4096, n_test=512, seed=SEED_BASE + 11)
+    w["c4_si72"] = Workload(     # 3x3x1 diamond cells: orthorhombic, c = 5.43 A < 2 r_c (two image shells)
+        "c4_si72", SystemSpec("Si72", "diamond", {"a": 5.43, "cells": (3, 3, 1)}, sigma=0.08, lj=_SI_LJ, lj_cut=6.0),
+        ModelConfig(1, 6.0, 0.5, [56], c2_emb, 16, c2_fit), batch=32, n_train=4096, n_test=512, seed=SEED_BASE + 12)
+    w["c4_nacl64"] = Workload(
+        "c4_nacl64", SystemSpec("NaCl64", "rocksalt", {"a": 5.64, "cells": (2, 2, 2)}, sigma=0.08, lj=_NACL_LJ,
+                                lj_cut=6.0),
+        ModelConfig(2, 6.0, 0.5, [24, 24], c2_emb, 16, c2_fit), batch=32, n_train=4096, n_test=512,
+        seed=SEED_BASE + 13)
+    w["c4_mg36"] = Workload(     # hcp 3x3x2: a triclinic (hexagonal) cell
+        "c4_mg36", SystemSpec("Mg36", "hcp", {"a": 3.21, "c": 5.21, "cells": (3, 3, 2)}, sigma=0.08, lj=_MG_LJ,
+                              lj_cut=6.0),
+        ModelConfig(1, 6.0, 0.5, [56], c2_emb, 16, c2_fit), batch=32, n_train=4096, n_test=512, seed=SEED_BASE + 14)
+    w["c4_h2o48"] = Workload(    # 16 molecules on a 4x2x2 grid at 1 g/cm^3
+        "c4_h2o48", SystemSpec("H2O-48", "water", {"n_side": (4, 2, 2), "L": 12.42}, sigma=0.05, lj=_WATER_LJ,
+                               lj_cut=6.0),
+        ModelConfig(2, 6.0, 0.5, [46, 92], c2_emb, 16, c2_fit), batch=32, n_train=4096, n_test=512,
+        seed=SEED_BASE + 15)
+    w["c4_alloy108"] = Workload(  # random 4-type fcc alloy (FEKF_MAX_TYPES types)
+        "c4_alloy108", SystemSpec("Alloy108", "alloy", {"a": 3.615, "cells": (3, 3, 3), "ntypes": 4}, sigma=0.10,
+                                  lj=_ALLOY_LJ, lj_cut=6.0),
+        ModelConfig(4, 6.0, 0.5, [40, 40, 40, 40], c2_emb, 16, c2_fit), batch=32, n_train=4096, n_test=512,
+        seed=SEED_BASE + 16)
+    # perfect lattice (sigma = 0, no strain): exact r^2 ties in every shell (tie-break tests); sel 16 cuts
+    # the second fcc shell (6 atoms at r = a) in the middle
+    w["t_cu32_perfect"] = Workload(
+        "t_cu32_perfect", SystemSpec("Cu32", "fcc", {"a": 3.615, "cells": (2, 2, 2)}, sigma=0.0, lj=_CU_LJ,
+                                     lj_cut=4.0),
+        ModelConfig(1, 4.0, 3.0, [48], [8, 16, 32], 4, [32, 32]), batch=2, n_train=4, n_test=2, seed=SEED_BASE + 17)
     return w
 
 

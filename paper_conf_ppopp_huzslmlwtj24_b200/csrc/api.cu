@@ -62,6 +62,8 @@ static fekf_status check_model(const fekf_model_cfg& m) {
   }
   if (nm < 1) { set_error("sum(sel) must be positive"); return FEKF_EINVAL; }
   if (!(m.rcut > 0) || !(m.rcut_smth >= 0) || !(m.rcut_smth < m.rcut)) { set_error("need 0 <= rcut_smth < rcut"); return FEKF_EINVAL; }
+  if (m.switch_kind != 0 && m.switch_kind != 1) { set_error("switch_kind must be 0 (quintic) or 1 (cosine)"); return FEKF_EINVAL; }
+  if (m.type_one_side != 0 && m.type_one_side != 1) { set_error("type_one_side must be 0 or 1"); return FEKF_EINVAL; }
   return FEKF_OK;
 }
 
@@ -80,6 +82,10 @@ static long long build_layout(const fekf_model_cfg& m, std::vector<long long>* s
   };
   for (int ti = 0; ti < m.ntypes; ++ti)
     for (int tj = 0; tj < m.ntypes; ++tj) {
+      if (m.type_one_side && ti > 0) {   // one net per neighbour type t_j (reading Z15 flag): shared
+        if (emb) emb->push_back((*emb)[tj]);
+        continue;
+      }
       std::vector<Layer> Ls;
       int din = 1;
       for (int l = 0; l < m.n_emb; ++l) {
@@ -192,6 +198,12 @@ fekf_status Ctx::init(const fekf_model_cfg& mm, const fekf_opt_cfg& oo, int nato
   FEKF_TRY(dalloc(sel_d, sizeof(int) * FEKF_MAX_TYPES));
   FEKF_TRY(dalloc(sec_d, sizeof(int) * (FEKF_MAX_TYPES + 1)));
   FEKF_TRY(dalloc(err_d, sizeof(int) * 4));
+  FEKF_TRY(dalloc(env_stats, sizeof(double) * 2 * nt * 4));
+  {
+    std::vector<double> st(2 * nt * 4, 0.0);
+    for (int q = nt * 4; q < 2 * nt * 4; ++q) st[q] = 1.0;   // avg 0, std 1: no normalisation
+    FEKF_CHECK_CUDA(cudaMemcpy(env_stats.p, st.data(), sizeof(double) * st.size(), cudaMemcpyHostToDevice));
+  }
   FEKF_CHECK_CUDA(cudaMemcpy(types_d.p, types.data(), sizeof(int) * Na, cudaMemcpyHostToDevice));
   FEKF_CHECK_CUDA(cudaMemcpy(tindex_d.p, tindex.data(), sizeof(int) * Na, cudaMemcpyHostToDevice));
   FEKF_CHECK_CUDA(cudaMemcpy(atoms_d.p, atoms_cat.data(), sizeof(int) * Na, cudaMemcpyHostToDevice));
@@ -340,7 +352,7 @@ Ctx::~Ctx() {
   for (DBuf* b : {&st_coord, &st_box, &st_e, &st_f, &st_fidx, &st_met, &naive_G, &naive_es, &naive_abe}) dfree(*b);
   kfo.reset();
   kf = nullptr;
-  for (DBuf* b : {&types_d, &tindex_d, &atoms_d, &atoms_off_d, &sel_d, &sec_d, &err_d, &w, &gbuf, &nl_j, &nl_s,
+  for (DBuf* b : {&types_d, &tindex_d, &atoms_d, &atoms_off_d, &sel_d, &sec_d, &err_d, &env_stats, &w, &gbuf, &nl_j, &nl_s,
                   &overflow, &em, &jac, &rij, &rdot, &vdir, &X, &Xb, &eatom, &etot, &force, &virial, &vatom, &splitk_ws,
                   &colsum_ws, &abe, &metrics_tmp, &abs_sum, &rowcnt, &chunks})
     dfree(*b);
@@ -545,7 +557,7 @@ using namespace fekf;
 extern "C" {
 
 const char* fekf_last_error(void) { return g_err.c_str(); }
-int fekf_version(void) { return 1; }
+int fekf_version(void) { return 2; }
 
 fekf_status fekf_plan_layout(const fekf_model_cfg* m, int block_size, int64_t* n_params, int32_t* blocks_host, int cap,
                              int* nblocks) {
@@ -703,6 +715,24 @@ fekf_status fekf_get_params(const fekf_ctx* c, double* w, cudaStream_t s) {
   return FEKF_OK;
 }
 
+fekf_status fekf_set_env_stats(fekf_ctx* ctx, const double* avg, const double* sd) {
+  if (!ctx) { set_error("set_env_stats: null"); return FEKF_EINVAL; }
+  Ctx& c = ctx->c;
+  std::vector<double> st(2 * c.nt * 4);
+  for (int q = 0; q < c.nt * 4; ++q) {
+    st[q] = avg ? avg[q] : 0.0;
+    st[c.nt * 4 + q] = sd ? sd[q] : 1.0;
+    if (!std::isfinite(st[q]) || !std::isfinite(st[c.nt * 4 + q]) || !(st[c.nt * 4 + q] > 0)) {
+      set_error("set_env_stats: avg must be finite, std finite and > 0");
+      return FEKF_EINVAL;
+    }
+  }
+  if (c.gstream) FEKF_CHECK_CUDA(cudaStreamSynchronize(c.gstream));   // replays in flight read the table
+  FEKF_CHECK_CUDA(cudaDeviceSynchronize());
+  FEKF_CHECK_CUDA(cudaMemcpy(c.env_stats.p, st.data(), sizeof(double) * st.size(), cudaMemcpyHostToDevice));
+  return FEKF_OK;
+}
+
 static fekf_status check_nb(const Ctx& c, int nb) {
   if (nb < 1 || nb > c.B) { set_error("nb must be in [1, local_batch]"); return FEKF_EINVAL; }
   return FEKF_OK;
@@ -783,7 +813,7 @@ fekf_status fekf_train_step(fekf_ctx* ctx, const double* coord, const double* bo
     return FEKF_EINVAL;
   }
   Ctx& c = ctx->c;
-  if (!c.use_graph) {
+  if (!c.use_graph || comm_is_loopback(c.comm)) {   // loopback collectives are host barriers: eager only
     const int64_t l0 = g_launches;
     FEKF_TRY(step_body(c, coord, box, e_label, f_label, force_idx, metrics, s));
     c.last_launches = g_launches - l0;

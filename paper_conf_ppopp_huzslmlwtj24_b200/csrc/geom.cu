@@ -1,4 +1,6 @@
 // (a1) neighbour list and (a2) smooth environment matrix — P:L83 (§2.1 item 1).
+#include <math_constants.h>
+
 #include "model.cuh"
 
 namespace fekf {
@@ -132,10 +134,13 @@ nlist_kernel(const double* __restrict__ coord, const double* __restrict__ box, c
 
 // R~ row s(r)(1, d/r), J = dR~/dd (4x3) and d for every slot; zeros for padding.
 // s(r) = sw(u)/r, u = (r - r_cs)/(r_c - r_cs), sw = 1 (r < r_cs), u^3(-6u^2+15u-10)+1 (reading Z8).
+// switch_kind 1: sw = 0.5 cos(pi u) + 0.5.  stats [2][ntypes][4] (avg | std, reading Z11): valid rows of
+// a centre atom of type t become (row - avg[t]) / std[t], J rows / std[t].
 __global__ void envmat_kernel(const double* __restrict__ coord, const double* __restrict__ box,
                               const int* __restrict__ nl_j, const int* __restrict__ nl_s, int Na, int Nm,
-                              long long nslots, double rcut, double rcs, double* __restrict__ em,
-                              double* __restrict__ jac, double* __restrict__ rij) {
+                              long long nslots, double rcut, double rcs, int switch_kind,
+                              const int* __restrict__ types, const double* __restrict__ stats, int ntypes,
+                              double* __restrict__ em, double* __restrict__ jac, double* __restrict__ rij) {
   const long long idx = (long long)blockIdx.x * blockDim.x + threadIdx.x;
   if (idx >= nslots) return;
   const int j = nl_j[idx];
@@ -176,8 +181,15 @@ __global__ void envmat_kernel(const double* __restrict__ coord, const double* __
   } else if (r < rcut) {
     const double h = rcut - rcs;
     const double u = (r - rcs) / h;
-    sw = u * u * u * (-6.0 * u * u + 15.0 * u - 10.0) + 1.0;
-    dsw = (-30.0 * u * u * u * u + 60.0 * u * u * u - 30.0 * u * u) / h;
+    if (switch_kind == 1) {
+      double sp, cp;
+      sincospi(u, &sp, &cp);
+      sw = 0.5 * cp + 0.5;
+      dsw = -0.5 * CUDART_PI * sp / h;
+    } else {
+      sw = u * u * u * (-6.0 * u * u + 15.0 * u - 10.0) + 1.0;
+      dsw = (-30.0 * u * u * u * u + 60.0 * u * u * u - 30.0 * u * u) / h;
+    }
   } else {
     sw = 0.0;
     dsw = 0.0;
@@ -186,17 +198,19 @@ __global__ void envmat_kernel(const double* __restrict__ coord, const double* __
   const double ds = dsw / r - sw / r2;   // d s / d r
   const double ir = 1.0 / r;
   const double e[3] = {d[0] * ir, d[1] * ir, d[2] * ir};
-  o_em[0] = s;
-  o_em[1] = s * d[0] / r;
-  o_em[2] = s * d[1] / r;
-  o_em[3] = s * d[2] / r;
+  const double* avg = stats + types[bi % Na] * 4;
+  const double* sd = stats + (ntypes + types[bi % Na]) * 4;
+  o_em[0] = (s - avg[0]) / sd[0];
+  o_em[1] = (s * d[0] / r - avg[1]) / sd[1];
+  o_em[2] = (s * d[1] / r - avg[2]) / sd[2];
+  o_em[3] = (s * d[2] / r - avg[3]) / sd[3];
 #pragma unroll
-  for (int be = 0; be < 3; ++be) o_j[be] = ds * e[be];
+  for (int be = 0; be < 3; ++be) o_j[be] = ds * e[be] / sd[0];
 #pragma unroll
   for (int a = 0; a < 3; ++a)
 #pragma unroll
     for (int be = 0; be < 3; ++be)
-      o_j[3 * (a + 1) + be] = ds * e[be] * e[a] + s * ((a == be ? ir : 0.0) - e[a] * e[be] * ir);
+      o_j[3 * (a + 1) + be] = (ds * e[be] * e[a] + s * ((a == be ? ir : 0.0) - e[a] * e[be] * ir)) / sd[a + 1];
 #pragma unroll
   for (int k = 0; k < 3; ++k) o_d[k] = d[k];
 }
@@ -216,8 +230,9 @@ fekf_status launch_nlist(Ctx& c, const double* coord, const double* box, int nb,
 fekf_status launch_envmat(Ctx& c, const double* coord, const double* box, const int* nl_j, const int* nl_s, int nb,
                           double* em, double* jac, double* rij, cudaStream_t s) {
   const long long n = (long long)nb * c.Na * c.Nm;
-  envmat_kernel<<<cdiv(n, 128), 128, 0, s>>>(coord, box, nl_j, nl_s, c.Na, c.Nm, n, c.m.rcut, c.m.rcut_smth, em, jac,
-                                              rij);
+  envmat_kernel<<<cdiv(n, 128), 128, 0, s>>>(coord, box, nl_j, nl_s, c.Na, c.Nm, n, c.m.rcut, c.m.rcut_smth,
+                                              c.m.switch_kind, c.types_d.as<int>(), c.env_stats.as<double>(), c.nt,
+                                              em, jac, rij);
   FEKF_LAUNCH_CHECK();
   count_launch();
   return FEKF_OK;

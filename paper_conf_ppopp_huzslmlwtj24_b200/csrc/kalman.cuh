@@ -53,6 +53,7 @@ struct KfPlan {
 // communicator helpers (comm.cu)
 int comm_world(fekf_comm* c);
 int comm_rank(fekf_comm* c);
+bool comm_is_loopback(fekf_comm* c);
 fekf_status comm_allreduce(fekf_comm* c, double* buf, long long n, cudaStream_t s);
 
 struct EvPair {

@@ -66,6 +66,7 @@ struct Ctx {
   Kf* kf = nullptr;
   // device
   DBuf types_d, tindex_d, atoms_d, atoms_off_d, sel_d, sec_d, err_d;
+  DBuf env_stats;                                 // [2][nt][4]: avg | std of the R~ rows (reading Z11)
   DBuf w, gbuf;                                   // [Np], [Np + 1] (g || error sum, the allreduce payload)
   DBuf nl_j, nl_s, overflow, em, jac, rij, rdot, vdir;
   DBuf X, Xb;                                     // [2 * B*Na*4*M] (primal | tangent)

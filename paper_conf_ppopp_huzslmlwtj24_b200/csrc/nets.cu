@@ -31,7 +31,7 @@ namespace fekf {
 // wrote).  32 outputs x 8 split-lanes per CTA, fixed 8-way combine -> deterministic.
 __global__ void splitk_reduce_kernel(const double* __restrict__ ws, int S0max, int S1max, int kps,
                                      const int* __restrict__ K0dev, const int* __restrict__ K1dev, int M, int N,
-                                     double* __restrict__ out) {
+                                     double* __restrict__ out, int accum) {
   __shared__ double red[8][32];
   const int lane = threadIdx.x & 31, zl = threadIdx.x >> 5;
   const long long i = (long long)blockIdx.x * 32 + lane;
@@ -50,7 +50,7 @@ __global__ void splitk_reduce_kernel(const double* __restrict__ ws, int S0max, i
     double t = red[0][lane];
 #pragma unroll
     for (int q = 1; q < 8; ++q) t += red[q][lane];
-    out[i] = t;
+    out[i] = accum ? out[i] + t : t;
   }
 }
 
@@ -58,7 +58,8 @@ struct Seg {
   const double* H; const double* Zb; long long kmax; const int* kdev; int ones;
 };
 
-static fekf_status wgrad(Ctx& c, int din, int dout, Seg s0, Seg s1, double* gout, cudaStream_t s) {
+// accum: add into gout (embedding nets shared by several type pairs, type_one_side) instead of writing
+static fekf_status wgrad(Ctx& c, int din, int dout, Seg s0, Seg s1, double* gout, cudaStream_t s, bool accum = false) {
   const int M = din + 1, N = dout;
   const long long tiles = (long long)cdiv(M, 64) * cdiv(N, 64);
   const long long kmax = std::max(s0.kmax, s1.kmax);
@@ -69,7 +70,7 @@ static fekf_status wgrad(Ctx& c, int din, int dout, Seg s0, Seg s1, double* gout
   while (nsplit(s0) + nsplit(s1) > budget) kps *= 2;
   const long long S0 = nsplit(s0), S1 = nsplit(s1);
   if (S0 + S1 == 0) return FEKF_OK;
-  if (S0 == 1 && S1 == 0)
+  if (S0 == 1 && S1 == 0 && !accum)
     return gemm<true, false>(M, N, (int)s0.kmax, s0.H, din, s0.Zb, dout, EpiStore{gout, dout}, s, nullptr, s0.kdev,
                              din, s0.ones ? (int)s0.kmax : 0);
   double* ws = c.splitk_ws.as<double>();
@@ -78,7 +79,7 @@ static fekf_status wgrad(Ctx& c, int din, int dout, Seg s0, Seg s1, double* gout
   if (S1) FEKF_TRY(gemm<true, false>(M, N, (int)s1.kmax, s1.H, din, s1.Zb, dout, EpiPartial{ws, M, N, (int)S0}, s,
                                      nullptr, s1.kdev, din, s1.ones ? (int)s1.kmax : 0, (int)S1, kps));
   splitk_reduce_kernel<<<cdiv((long long)M * N, 32), 256, 0, s>>>(ws, (int)S0, (int)S1, kps, s0.kdev, s1.kdev, M, N,
-                                                                  gout);
+                                                                  gout, accum ? 1 : 0);
   FEKF_LAUNCH_CHECK();
   count_launch();
   return FEKF_OK;
@@ -129,7 +130,7 @@ static fekf_status wgrad_group(Ctx& c, WgradJob* jobs, int n, cudaStream_t s) {
     if (S0[q] + S1[q] == 0) continue;
     splitk_reduce_kernel<<<cdiv((long long)M * N, 32), 256, 0, s>>>(c.splitk_ws.as<double>() + off[q], (int)S0[q],
                                                                     (int)S1[q], (int)kps_[q], J.s0.kdev, J.s1.kdev, M,
-                                                                    N, J.gout);
+                                                                    N, J.gout, 0);
     FEKF_LAUNCH_CHECK();
     count_launch();
   }
@@ -1395,7 +1396,7 @@ fekf_status model_backward(Ctx& c, int nb, Mode mode, double* gout, cudaStream_t
         const double* Hpt = l == 0 ? P.hin_t.as<double>() : P.Ht[l - 1].as<double>();
         FEKF_TRY(wgrad(c, L.din, L.dout, Seg{Hp, P.Zb[l].as<double>(), Rmax, rc, 1},
                        Seg{dual ? Hpt : nullptr, dual ? P.Zbt[l].as<double>() : nullptr, dual ? Rmax : 0, tc, 0},
-                       gout + L.W, s));
+                       gout + L.W, s, true));
       }
       if (l > 0) {
         if (dual) {

@@ -30,7 +30,8 @@ class FekfError(RuntimeError):
 class ModelCfg(C.Structure):
     _fields_ = [("ntypes", C.c_int), ("rcut", C.c_double), ("rcut_smth", C.c_double), ("sel", C.c_int * MAX_TYPES),
                 ("n_emb", C.c_int), ("emb", C.c_int * MAX_LAYERS), ("m2", C.c_int), ("n_fit", C.c_int),
-                ("fit", C.c_int * MAX_LAYERS), ("fit_resnet_dt", C.c_int)]
+                ("fit", C.c_int * MAX_LAYERS), ("fit_resnet_dt", C.c_int), ("switch_kind", C.c_int),
+                ("type_one_side", C.c_int)]
 
 
 class OptCfg(C.Structure):
@@ -87,6 +88,8 @@ def lib():
         "fekf_kf_naive_partial_u": ([vp, C.POINTER(vp), C.POINTER(i64)], i32),
         "fekf_kf_update_naive_end": ([vp, vp, vp, vp, vp], i32),
         "fekf_naive_train_step": ([vp, vp, vp, vp, vp, vp, vp, vp], i32),
+        "fekf_set_env_stats": ([vp, vp, vp], i32),
+        "fekf_comm_init_loopback": ([i32, vp], i32),
     }
     for name, (args, res) in sigs.items():
         f = getattr(L, name)
@@ -106,6 +109,7 @@ EXPORTED = [
     "fekf_energy_jacobian", "fekf_force_jacobian", "fekf_kalman_update", "fekf_train_step",
     "fekf_last_launch_count", "fekf_set_graph_mode", "fekf_kf_update_naive", "fekf_naive_train_step",
     "fekf_kf_timing_parts", "fekf_kf_update_naive_begin", "fekf_kf_naive_partial_u", "fekf_kf_update_naive_end",
+    "fekf_set_env_stats", "fekf_comm_init_loopback",
 ]
 
 
@@ -156,6 +160,8 @@ def model_cfg(m) -> ModelCfg:
     for i, v in enumerate(fit):
         c.fit[i] = int(v)
     c.fit_resnet_dt = int(_get(m, "fit_resnet_dt", 1))
+    c.switch_kind = int(_get(m, "switch_kind", 0) or 0)
+    c.type_one_side = int(_get(m, "type_one_side", 0) or 0)
     return c
 
 
@@ -216,6 +222,20 @@ class Comm:
         buf = (C.c_ubyte * 128).from_buffer_copy(uid)
         _check(lib().fekf_comm_init(rank, world, buf, C.byref(self.h)))
         self.rank, self.world = rank, world
+
+    @classmethod
+    def loopback(cls, world):
+        """fekf_comm_init_loopback: `world` rank handles of one in-process group (one GPU, one host thread
+        per rank)."""
+        arr = (C.c_void_p * world)()
+        _check(lib().fekf_comm_init_loopback(world, arr))
+        out = []
+        for r in range(world):
+            c = cls.__new__(cls)
+            c.h = C.c_void_p(arr[r])
+            c.rank, c.world = r, world
+            out.append(c)
+        return out
 
     @staticmethod
     def unique_id() -> bytes:
@@ -395,6 +415,21 @@ class Context:
         self.comm = comm
         if not graph:
             self.set_graph_mode(False)
+        if _get(model, "env_avg", None) is not None or _get(model, "env_std", None) is not None:
+            self.set_env_stats(_get(model, "env_avg", None), _get(model, "env_std", None))
+
+    def set_env_stats(self, avg=None, std=None):
+        """Descriptor statistics per centre type [ntypes][4] (fekf_set_env_stats, reading Z11)."""
+        nt = self.mc.ntypes
+
+        def host(a):
+            if a is None:
+                return None
+            flat = [float(v) for row in a for v in row]
+            if len(flat) != nt * 4:
+                raise FekfError(1, f"env stats must be [{nt}][4]")
+            return (C.c_double * len(flat))(*flat)
+        _check(lib().fekf_set_env_stats(self.h, host(avg), host(std)))
 
     def set_graph_mode(self, enable: bool):
         """a10: replay each minibatch step as one captured CUDA graph (default) or launch eagerly."""

@@ -26,7 +26,7 @@ def test_library_exports_every_declared_symbol():
     for name in decl:
         assert hasattr(L, name), name
     assert set(decl) == set(fk.EXPORTED)
-    assert L.fekf_version() == 1
+    assert L.fekf_version() == 2
 
 
 @pytest.mark.parametrize("name", sorted(CONFIGS))
