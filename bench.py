@@ -195,6 +195,58 @@ def oracle_sample(name, n_img=1, kf_blocks=1, seed=99):
                       f"5 updates over all blocks"}
 
 
+FP64_PEAK_TFLOPS = 37.1   # measured DMMA rate (tools/fp64_peak.cu on this pool's B200, round 1); guide-derived
+                          # 148 SMs x 64 DFMA/clk x 2 x 1.965 GHz = 37.2
+
+
+def nets_work(m, nl_j, types, groups):
+    """Executed FLOPs of the nets in one minibatch step (1 energy + len(groups) force updates), counted
+    from the step's own neighbour list: GEMM work as 2 flops per multiply-add over the VALID rows only
+    (n_v per type pair), the force updates' tangent / restricted rows over the ACTIVE rows only (rows
+    whose centre or neighbour is a selected atom).  Elementwise work (tanh, adjoint products) is counted
+    separately as tanh evaluations.  nl_j [B][Na][N_m] (int), types [Na]."""
+    nl_j = np.asarray(nl_j)
+    types = np.asarray(types)
+    B, na, _ = nl_j.shape
+    sec = np.concatenate([[0], np.cumsum(m.sel)]).astype(int)
+    d = list(m.emb)
+    din = [1] + d[:-1]
+    fwd_row = 2 * sum(a * b for a, b in zip(din, d))
+    dg_row = 2 * sum(a * b for a, b in zip(din[1:], d[1:]))
+    wg_row = 2 * sum((a + 1) * b for a, b in zip(din, d))
+    M, M2 = m.emb[-1], m.m2
+    desc_row = 2 * 4 * M                 # X += R~^T G (per row), reverse: Gbar and dR~ (x2)
+    desc_atom = 2 * 4 * M * M2           # D = X^T X^<, reverse Eq. 4 (x2)
+    h = [M * M2] + list(m.fit)
+    fit_fwd = 2 * (sum(a * b for a, b in zip(h[:-1], h[1:])) + h[-1])
+    fit_dg = fit_fwd
+    fit_wg = 2 * (sum((a + 1) * b for a, b in zip(h[:-1], h[1:])) + h[-1] + 1)
+    valid = nl_j >= 0
+    N = int(valid.sum())                  # valid embedding rows (all pairs)
+    F = B * na                            # fitting rows
+    fl = 0.0
+    # energy update: forward, full reverse with weight gradients
+    fl += N * (fwd_row + desc_row) + F * (desc_atom + fit_fwd)
+    fl += F * (fit_dg + fit_wg + 2 * desc_atom) + N * (dg_row + wg_row + 2 * desc_row)
+    T_all = []
+    for g in groups:
+        sel = np.zeros(na, bool)
+        sel[np.asarray(g)] = True
+        j = np.where(valid, nl_j, 0)
+        act = valid & (sel[None, :, None] | sel[j])
+        T = int(act.sum())
+        T_all.append(T)
+        fl += N * (fwd_row + desc_row) + F * (desc_atom + fit_fwd)                  # primal forward
+        fl += F * (fit_dg + 2 * desc_atom) + T * (dg_row + 2 * desc_row)          # forces on S_k (restricted)
+        fl += T * (fwd_row + 2 * desc_row) + F * (2 * desc_atom + fit_fwd)        # tangent forward
+        fl += 2 * F * (fit_dg + fit_wg) + F * 4 * desc_atom                       # dual reverse, fitting
+        fl += (N + T) * (dg_row + wg_row) + (N + T) * 2 * desc_row                 # dual reverse, embedding
+    ng = len(groups)
+    tanh = (N * sum(d) + F * sum(m.fit)) * (1 + ng)      # primal forwards only (tangent rows reuse y)
+    return {"flops_per_step": fl, "valid_rows": N, "padded_slots": int(nl_j.size), "fitting_rows": F,
+            "active_rows_per_force_update": (sum(T_all) / max(ng, 1)), "tanh_per_step": int(tanh)}
+
+
 def run_reference(args, rank, world):
     if rank != 0:
         return
@@ -373,6 +425,32 @@ def run_fekf(args, rank, world, local):
         standalone = {"achieved": sa, "frac": sa / peak, "avg_launch_ms": sa_ms / sa_n, "launches": sa_n,
                       "pass": "read-only, all SMs"}
         del gs
+    # ---- nets roofline: the step's nets work (E Jacobian + force_groups force Jacobians, the same kernels
+    # the step runs, on all SMs, eager launches on this stream) against the fp64 DMMA peak
+    nets = None
+    try:
+        nj, _, _ = ctx.build_nlist(coord[0], box[0])
+        s0 = nsteps - 1
+        work = nets_work(m, nj.cpu().numpy(), ds["types"], gidx[s0])
+        torch.cuda.synchronize()
+        reps = 3
+        n0, n1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        for r in range(reps + 1):
+            if r == 1:
+                n0.record(stream)
+            ctx.energy_jacobian(coord[0], box[0], elab[0])
+            for k in range(opt.force_groups):
+                ctx.force_jacobian(coord[0], box[0], flab[0], fidx[s0][k])
+        n1.record(stream)
+        torch.cuda.synchronize()
+        nets_ms = n0.elapsed_time(n1) / reps
+        tf = work["flops_per_step"] / (nets_ms / 1000.0) / 1e12
+        nets = {"kernels": "emb_fwd/emb_bwd/dgemm/desc_* (E + %d F Jacobians)" % opt.force_groups, "bound": "fp64",
+                "achieved": tf, "peak": FP64_PEAK_TFLOPS, "unit": "TFLOP/s", "frac": tf / FP64_PEAK_TFLOPS,
+                "peak_source": "measured DMMA (tools/fp64_peak.cu)", "ms_per_step_alone": nets_ms,
+                "share_of_step_if_serial": nets_ms / (ms / args.steps), **work}
+    except Exception as e:   # instrumentation only: never lose the bench line over it
+        nets = {"error": str(e)[:200]}
     split_sms = int(os.environ.get("FEKF_SPLIT_SMS", "96" if args.precision == 64 else "80")) if world == 1 else 0
     roof = {"kernel": "kf_pass_kernel", "bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
             "frac": (achieved / peak) if achieved else None, "traffic": traffic,
@@ -393,7 +471,7 @@ def run_fekf(args, rank, world, local):
                       "p_precision": args.precision, "p_defer": opt.p_defer,
                       "l2": "inputs larger than L2: P (%.1f GiB packed) is streamed 5x per step"
                             % (info["p_bytes_local"] / 2**30)},
-           "roofline": roof, "e2e": e2e, "gpu_launches": int(launches), "clocks": clk,
+           "roofline": roof, "roofline_nets": nets, "e2e": e2e, "gpu_launches": int(launches), "clocks": clk,
            "last_metrics": {"abe_e": met[0], "abe_f": list(met[1:5]), "A_last": met[5], "lambda": met[6],
                             "flags": met[7]}}
     if rank == 0 and world == 1 and not args.no_cpu_baseline:

@@ -339,6 +339,15 @@ def _workloads():
                                   lj=_ALLOY_LJ, lj_cut=6.0),
         ModelConfig(4, 6.0, 0.5, [40, 40, 40, 40], c2_emb, 16, c2_fit), batch=32, n_train=4096, n_test=512,
         seed=SEED_BASE + 16)
+    # C4 time-to-target variants: the same systems with C1-sized nets and minibatch 4, so the fp64 CPU
+    # oracle (dense P blocks) can produce the target trajectory (metric (iii)) in minutes
+    for key in ["c4_al32", "c4_si72", "c4_nacl64", "c4_mg36", "c4_h2o48", "c4_alloy108"]:
+        base = w[key]
+        bm = base.model
+        name = key.replace("c4_", "c4s_")
+        w[name] = Workload(name, base.system, ModelConfig(bm.ntypes, bm.rcut, bm.rcut_smth, list(bm.sel), [8, 16, 32],
+                                                          4, [32, 32]),
+                           batch=4, n_train=64, n_test=16, seed=base.seed)
     # perfect lattice (sigma = 0, no strain): exact r^2 ties in every shell (tie-break tests); sel 16 cuts
     # the second fcc shell (6 atoms at r = a) in the middle
     w["t_cu32_perfect"] = Workload(

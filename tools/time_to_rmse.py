@@ -103,8 +103,9 @@ def run(config, max_steps, every, target=None, precision=64, stop_at_target=True
     if gold is not None:
         g = {s: (e, f) for s, e, f in gold["trajectory"]}
         common = [(s, e, f) for s, e, f in traj if s in g]
-        out["max_rel_dev_vs_oracle"] = max(
-            (max(abs(e - g[s][0]) / g[s][0], abs(f - g[s][1]) / g[s][1]) for s, e, f in common), default=None)
+        devs = [[s, max(abs(e - g[s][0]) / g[s][0], abs(f - g[s][1]) / g[s][1])] for s, e, f in common]
+        out["dev_vs_oracle"] = devs
+        out["max_rel_dev_vs_oracle"] = max((d for _, d in devs), default=None)
         out["oracle_train_s_for_S_o"] = gold.get("oracle_train_seconds")
         # the oracle's own time to the same target (its per-step time on the host that wrote the file)
         out["oracle_minutes_to_target"] = gold["oracle_train_seconds"] * gold["target_step"] / gold["S_o"] / 60.0
