@@ -435,13 +435,14 @@ def run_fekf(args, rank, world, local):
         torch.cuda.synchronize()
         reps = 3
         n0, n1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        cs = torch.cuda.current_stream()
         for r in range(reps + 1):
             if r == 1:
-                n0.record(stream)
+                n0.record(cs)
             ctx.energy_jacobian(coord[0], box[0], elab[0])
             for k in range(opt.force_groups):
                 ctx.force_jacobian(coord[0], box[0], flab[0], fidx[s0][k])
-        n1.record(stream)
+        n1.record(cs)
         torch.cuda.synchronize()
         nets_ms = n0.elapsed_time(n1) / reps
         tf = work["flops_per_step"] / (nets_ms / 1000.0) / 1e12

@@ -265,7 +265,6 @@ fekf_status Ctx::init(const fekf_model_cfg& mm, const fekf_opt_cfg& oo, int nato
     FEKF_TRY(dalloc(P.hin, sizeof(double) * R1));
     FEKF_TRY(dalloc(P.hin_t, sizeof(double) * R1));
     FEKF_TRY(dalloc(P.sbar, sizeof(double) * R1));
-    FEKF_TRY(dalloc(P.wimg, sizeof(double) * (1 << 14)));
     const size_t nl = P.L.size();
     for (auto* v : {&P.Y, &P.H, &P.Hb, &P.Zb, &P.Yt, &P.Ht, &P.Hbt, &P.Zbt}) v->resize(nl);
     for (size_t l = 0; l < nl; ++l) {
@@ -357,7 +356,7 @@ Ctx::~Ctx() {
                   &colsum_ws, &abe, &metrics_tmp, &abs_sum, &rowcnt, &chunks})
     dfree(*b);
   for (auto& P : pairs) {
-    for (DBuf* b : {&P.row_idx, &P.row_start, &P.tidx, &P.tpos, &P.hin, &P.hin_t, &P.sbar, &P.wimg}) dfree(*b);
+    for (DBuf* b : {&P.row_idx, &P.row_start, &P.tidx, &P.tpos, &P.hin, &P.hin_t, &P.sbar}) dfree(*b);
     for (auto* v : {&P.Y, &P.H, &P.Hb, &P.Zb, &P.Yt, &P.Ht, &P.Hbt, &P.Zbt}) for (auto& b : *v) dfree(b);
   }
   for (auto& F : fits) {

@@ -78,6 +78,31 @@ __device__ __forceinline__ void l2_prefetch(const void* p, unsigned bytes) {
   asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(p), "r"(bytes) : "memory");
 }
 
+// dense W [din][d] -> zero-padded SMEM image [ROWS][sld(d)], every global load of a thread issued before its
+// first store (a plain strided loop serialises one L2 round trip per element)
+template <int din, int d, int ROWS, int NTH>
+__device__ __forceinline__ void stage_mat(double* __restrict__ dst, const double* __restrict__ src, int tid) {
+  constexpr int ld = sld(d), n = ROWS * ld, IT = (n + NTH - 1) / NTH;
+  double v[IT];
+#pragma unroll
+  for (int i = 0; i < IT; ++i) {
+    const int e = tid + i * NTH, k = e / ld, j = e % ld;
+    v[i] = (e < n && k < din && j < d) ? __ldg(src + k * d + j) : 0.0;
+  }
+#pragma unroll
+  for (int i = 0; i < IT; ++i) {
+    const int e = tid + i * NTH;
+    if (e < n) dst[e] = v[i];
+  }
+}
+template <class W, int L, int NTH>
+__device__ __forceinline__ void stage_fwd_w(double* sm, const double* __restrict__ wp, int tid) {
+  if constexpr (L < W::NL) {
+    stage_mat<W::din(L), W::d(L), pad4(W::din(L)), NTH>(sm + W::fW(L), wp + W::goff(L), tid);
+    stage_fwd_w<W, L + 1, NTH>(sm, wp, tid);
+  }
+}
+
 static int g_num_sms = 0;
 static int num_sms() {
   if (!g_num_sms) {
@@ -104,156 +129,155 @@ struct EmbFwdIO {
   const double* Yp[FEKF_MAX_LAYERS];  // tangent: primal y_l, indexed by primal row
 };
 
-// Forward layer L >= 1 on the current tile: h_L = skip(h_{L-1}) + y_L, y_L = tanh(h_{L-1} W_L + b_L)
-// (primal) or (1 - y_L^2)(hdot_{L-1} W_L) (tangent rows, y_L of the primal row).
+// Forward, warp-tiled: every warp runs all layers of its own RT-row tiles (RT / 8 DMMA strips of 8 rows)
+// with no CTA-wide barrier; W_l and b_l are staged once per (persistent, one per SM) CTA in SMEM, a
+// layer's accumulators live in registers and its epilogue (bias, tanh, skip, the y / h stores) works on
+// them directly, the next layer's A operand goes through the warp's own SMEM buffer (__syncwarp only).
+// The next tile's inputs (row -> primal row -> slot -> s) are fetched in three dependent steps spread over
+// the current tile's layers.  Tangent rows: ydot = (1 - y^2) zdot with y of the primal row, no bias.
 template <class W, int L>
-__device__ __forceinline__ void fwd_layer(double* sm, const double* __restrict__ wimg, const EmbFwdIO& io, int r0, int R,
-                                          bool tan, const int* s_prow) {
-  constexpr int T = W::T, NW = EMB_FWD_WARPS;
-  constexpr int din = W::din(L), d = W::d(L), skip = W::skip(L);
-  constexpr int LDI = W::fALD((L - 1) & 1), LDO = W::fALD(L & 1);
-  const double* in = sm + W::sA((L - 1) & 1);
-  double* out = sm + W::sA(L & 1);
-  const double* bs = sm + W::sB(L);
+__device__ __forceinline__ void wfwd_layer(const double* __restrict__ sm, double* __restrict__ wb,
+                                           const EmbFwdIO& io, int r0, int R, bool tan, const int (&prs)[W::RT / 8]) {
+  constexpr int MS = W::RT / 8;   // 8-row DMMA strips per warp tile
+  constexpr int din = W::din(L), d = W::d(L), K4 = pad4(din), NT = pad8(d) / 8, skip = W::skip(L);
+  constexpr bool last = L + 1 == W::NL;
+  constexpr int LDI = W::wALD((L - 1) & 1), LDO = W::wALD(L & 1), LDB = sld(d);
+  const int lane = threadIdx.x & 31, fr = lane >> 2, fk = lane & 3;
+  const double* in = wb + ((L - 1) & 1) * W::RT * W::wALD(0);
+  double* out = wb + (L & 1) * W::RT * W::wALD(0);
+  const double* Bw = sm + W::fW(L);
+  const double* bs = sm + W::fB(L);
+  double acc[MS][NT][2];
+#pragma unroll
+  for (int i = 0; i < MS; ++i)
+#pragma unroll
+    for (int j = 0; j < NT; ++j) acc[i][j][0] = acc[i][j][1] = 0.0;
+#pragma unroll
+  for (int k = 0; k < K4; k += 4) {
+    double a[MS];
+#pragma unroll
+    for (int i = 0; i < MS; ++i) a[i] = in[(8 * i + fr) * LDI + k + fk];
+#pragma unroll
+    for (int j = 0; j < NT; ++j) {
+      const double b = Bw[(k + fk) * LDB + 8 * j + fr];
+#pragma unroll
+      for (int i = 0; i < MS; ++i) dmma884(acc[i][j][0], acc[i][j][1], a[i], b);
+    }
+  }
   double* Yl = io.Y[L];
   double* Hl = io.H[L];
   const double* Ypl = io.Yp[L];
-  cta_mma<false, T / 8, pad8(d) / 8, pad4(din), LDI, sld(d), NW>(
-      in, wimg + W::fW(L), [&](int r, int c, double z0, double z1) {
-        const int row = r0 + r;
-        const bool live = row < R;
-        double h[2];
-        const double z[2] = {z0, z1};
 #pragma unroll
-        for (int q = 0; q < 2; ++q) {
-          const int cc = c + q;
-          double y;
-          if (tan) {
-            const int pr = s_prow[r];
-            const double yp = (cc < d && pr >= 0) ? Ypl[(size_t)pr * d + cc] : 0.0;
-            y = (1.0 - yp * yp) * z[q];
-          } else {
-            y = tanh_fp64(z[q] + bs[cc]);
-          }
-          const double sk = skip == 1 ? in[r * LDI + cc] : (skip == 2 ? in[r * LDI + (cc % din)] : 0.0);
-          h[q] = cc < d ? sk + y : 0.0;
-          if (live && cc < d) {
-            Yl[(size_t)row * d + cc] = y;
-            if (Hl) Hl[(size_t)row * d + cc] = h[q];
-          }
+  for (int i = 0; i < MS; ++i) {
+    const int r = 8 * i + fr, row = r0 + r;
+    const bool live = row < R;
+    const int pr = prs[i];
+#pragma unroll
+    for (int j = 0; j < NT; ++j) {
+      const int c = 8 * j + 2 * fk;
+      double y[2], h[2];
+#pragma unroll
+      for (int q = 0; q < 2; ++q) {
+        const int cc = c + q;
+        if (tan) {
+          const double yp = (cc < d && pr >= 0) ? Ypl[(size_t)pr * d + cc] : 0.0;
+          y[q] = (1.0 - yp * yp) * acc[i][j][q];
+        } else {
+          y[q] = tanh_fp64(acc[i][j][q] + bs[cc]);
         }
-        *reinterpret_cast<double2*>(out + r * LDO + c) = make_double2(h[0], h[1]);
-      });
-  __syncthreads();
-}
-
-// zero-padded global image of the W_l ([pad4(din)][sld(d)], the forward's layout) for the L1 path
-template <class W>
-__global__ void emb_pack_kernel(const double* __restrict__ wp, double* __restrict__ wimg) {
-  const int tid = blockIdx.x * blockDim.x + threadIdx.x, nth = gridDim.x * blockDim.x;
-  for (int c = tid; c < pad8(W::d(0)); c += nth) wimg[W::fW(0) + c] = c < W::d(0) ? wp[W::goff(0) + c] : 0.0;
+        const double sk = skip == 1 ? in[r * LDI + cc] : (skip == 2 ? in[r * LDI + (cc % din)] : 0.0);
+        h[q] = cc < d ? sk + y[q] : 0.0;
+      }
+      if (live) {
+        if ((d & 1) == 0 && c < d) {
+          *reinterpret_cast<double2*>(Yl + (size_t)row * d + c) = make_double2(y[0], y[1]);
+          if (last) *reinterpret_cast<double2*>(Hl + (size_t)row * d + c) = make_double2(h[0], h[1]);
+        } else {
 #pragma unroll
-  for (int l = 1; l < W::NL; ++l) {
-    const int din = W::din(l), d = W::d(l), ld = sld(d), n = pad4(din) * ld;
-    for (int e = tid; e < n; e += nth) {
-      const int k = e / ld, j = e % ld;
-      wimg[W::fW(l) + e] = (k < din && j < d) ? wp[W::goff(l) + k * d + j] : 0.0;
+          for (int q = 0; q < 2; ++q)
+            if (c + q < d) {
+              Yl[(size_t)row * d + c + q] = y[q];
+              if (last) Hl[(size_t)row * d + c + q] = h[q];
+            }
+        }
+      }
+      if (!last) *reinterpret_cast<double2*>(out + r * LDO + c) = make_double2(h[0], h[1]);
     }
   }
+  __syncwarp();
 }
 
 template <class W>
-__global__ void __launch_bounds__(EMB_FWD_WARPS * 32) emb_fwd_kernel(const double* __restrict__ wp,
-                                                                     const double* __restrict__ wimg, EmbFwdIO io) {
+__global__ void __launch_bounds__(W::WNW * 32, 1) emb_fwd_kernel(const double* __restrict__ wp, EmbFwdIO io) {
   extern __shared__ __align__(16) double sm[];
-  constexpr int T = W::T, NW = EMB_FWD_WARPS, NL = W::NL, RPW = T / NW;
-  __shared__ double s_in[2][T];
-  __shared__ int s_prow[2][T];
-  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+  constexpr int NL = W::NL, RT = W::RT, NW = W::WNW, d0 = W::d(0), d0p = pad8(d0), LD0 = W::wALD(0);
+  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31, fr = lane >> 2;
   const bool tan = io.tidx != nullptr;
   const int R = min(io.Rmax, *io.Rdev);
-  // ---- stage b_l (W_l is read through L1 from wimg)
+  // ---- stage W_l [pad4(din)][sld(d)] (zero padded) and b_l once per CTA
+  for (int c = tid; c < d0p; c += NW * 32) sm[W::fW(0) + c] = c < d0 ? __ldg(wp + W::goff(0) + c) : 0.0;
+  if constexpr (NL >= 2) stage_fwd_w<W, 1, NW * 32>(sm, wp, tid);
 #pragma unroll
   for (int l = 0; l < NL; ++l)
-    for (int c = tid; c < pad8(W::d(l)); c += blockDim.x)
-      sm[W::sB(l) + c] = c < W::d(l) ? wp[W::goff(l) + W::din(l) * W::d(l) + c] : 0.0;
-
-  // The next tile's input (row -> primal row -> slot -> s) is fetched by warp 0 in three dependent
-  // steps spread over the current tile's layers, so its latency hides behind the compute.
+    for (int c = tid; c < pad8(W::d(l)); c += NW * 32)
+      sm[W::fB(l) + c] = c < W::d(l) ? __ldg(wp + W::goff(l) + W::din(l) * W::d(l) + c) : 0.0;
+  double* wb = sm + W::WS + warp * W::WRP;
+  __syncthreads();
+  const int ntiles = (R + RT - 1) / RT;
+  const int gw = blockIdx.x * NW + warp, nwt = gridDim.x * NW;
+  // lanes 0..15 carry row lane of the tile: primal row, slot, input s (current and next tile)
   int nx_pr = -1, nx_slot = -1;
   double nx_v = 0.0;
-  auto fetch_a = [&](int rn) {
-    nx_pr = -1;
-    if (tid < T && rn + tid < R) nx_pr = tan ? io.tidx[rn + tid] : rn + tid;
-  };
-  auto fetch_b = [&]() { nx_slot = (tid < T && nx_pr >= 0) ? io.row_idx[nx_pr] : -1; };
+  auto fetch_a = [&](int rn) { nx_pr = (lane < RT && rn + lane < R) ? (tan ? io.tidx[rn + lane] : rn + lane) : -1; };
+  static_assert(RT == 8 || RT == 16, "warp tile rows");
+  auto fetch_b = [&]() { nx_slot = nx_pr >= 0 ? io.row_idx[nx_pr] : -1; };
   auto fetch_c = [&]() { nx_v = nx_slot >= 0 ? io.src[(size_t)nx_slot * 4] : 0.0; };
-  auto fetch_d = [&](int rn, int b) {
-    if (tid < T) {
-      s_in[b][tid] = nx_v;
-      s_prow[b][tid] = nx_pr;
-      if (rn + tid < R) io.hin[rn + tid] = nx_v;
-    }
-  };
-  const int ntiles = (R + T - 1) / T;
-  int buf = 0;
-  if ((int)blockIdx.x < ntiles) {
-    fetch_a(blockIdx.x * T);
+  if (gw < ntiles) {
+    fetch_a(gw * RT);
     fetch_b();
     fetch_c();
-    fetch_d(blockIdx.x * T, 0);
   }
-  for (int tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
-    const int r0 = tile * T, rn = r0 + gridDim.x * T;
-    __syncthreads();  // weights staged / this tile's inputs in s_in[buf] / previous tile's buffers consumed
+  for (int tile = gw; tile < ntiles; tile += nwt) {
+    const int r0 = tile * RT, rn = r0 + nwt * RT;
+    const double s_in = nx_v;
+    const int cur_pr = nx_pr;
+    if (lane < RT && r0 + lane < R) io.hin[r0 + lane] = s_in;
     fetch_a(rn);
-    const double* s_inb = s_in[buf];
-    const int* s_prowb = s_prow[buf];
-    // ---- layer 0 (input width 1): elementwise
+    int prs[RT / 8];
+#pragma unroll
+    for (int i = 0; i < RT / 8; ++i) prs[i] = __shfl_sync(0xffffffffu, cur_pr, 8 * i + fr);
+    // ---- layer 0 (input width 1): elementwise into buffer 0
     {
-      constexpr int d = W::d(0), w8 = pad8(d), CJ = (w8 + 31) / 32, ld = W::fALD(0);
-      double* out = sm + W::sA(0);
-      const double* w0 = wimg + W::fW(0);
-      const double* b0 = sm + W::sB(0);
-      double yp[RPW][CJ];
-#pragma unroll
-      for (int i = 0; i < RPW; ++i)
-#pragma unroll
-        for (int j = 0; j < CJ; ++j) {
-          const int r = warp + NW * i, c = lane + 32 * j;
-          const int pr = s_prowb[r];
-          yp[i][j] = (tan && c < d && pr >= 0) ? io.Yp[0][(size_t)pr * d + c] : 0.0;
-        }
-#pragma unroll
-      for (int i = 0; i < RPW; ++i)
-#pragma unroll
-        for (int j = 0; j < CJ; ++j) {
-          const int r = warp + NW * i, c = lane + 32 * j;
-          if (c < w8) {
-            const int row = r0 + r;
-            double h = 0.0;
-            if (c < d) {
-              const double z = s_inb[r] * w0[c];
-              h = tan ? (1.0 - yp[i][j] * yp[i][j]) * z : tanh_fp64(z + b0[c]);
-              if (row < R) {
-                const size_t o = (size_t)row * d + c;
-                io.Y[0][o] = h;
-                if (io.H[0]) io.H[0][o] = h;
-              }
-            }
-            out[r * ld + c] = h;
+      const double* w0 = sm + W::fW(0);
+      const double* b0 = sm + W::fB(0);
+#pragma unroll 2
+      for (int e = lane; e < RT * d0p; e += 32) {
+        const int r = e / d0p, c = e % d0p;
+        const double sv = __shfl_sync(0xffffffffu, s_in, r);
+        const int pr = __shfl_sync(0xffffffffu, cur_pr, r);
+        double h = 0.0;
+        if (c < d0) {
+          const double z = sv * w0[c];
+          if (tan) {
+            const double yp = pr >= 0 ? io.Yp[0][(size_t)pr * d0 + c] : 0.0;
+            h = (1.0 - yp * yp) * z;
+          } else {
+            h = tanh_fp64(z + b0[c]);
+          }
+          if (r0 + r < R) {
+            io.Y[0][(size_t)(r0 + r) * d0 + c] = h;
+            if (NL == 1) io.H[0][(size_t)(r0 + r) * d0 + c] = h;
           }
         }
+        if (NL > 1) wb[r * LD0 + c] = h;
+      }
+      __syncwarp();
     }
-    __syncthreads();
+    if constexpr (NL >= 2) wfwd_layer<W, 1>(sm, wb, io, r0, R, tan, prs);
     fetch_b();
-    // ---- layers 1..NL-1: DMMA with the bias / tanh / skip epilogue in the accumulators
-    if constexpr (NL >= 2) fwd_layer<W, 1>(sm, wimg, io, r0, R, tan, s_prowb);
+    if constexpr (NL >= 3) wfwd_layer<W, 2>(sm, wb, io, r0, R, tan, prs);
+    if constexpr (NL >= 4) wfwd_layer<W, 3>(sm, wb, io, r0, R, tan, prs);
     fetch_c();
-    if constexpr (NL >= 3) fwd_layer<W, 2>(sm, wimg, io, r0, R, tan, s_prowb);
-    if constexpr (NL >= 4) fwd_layer<W, 3>(sm, wimg, io, r0, R, tan, s_prowb);
-    fetch_d(rn, buf ^ 1);
-    buf ^= 1;
   }
 }
 
@@ -273,23 +297,19 @@ static fekf_status emb_forward_t(Ctx& c, int p, long long Rmax, bool tangent, cu
     io.H[l] = l + 1 < W::NL ? nullptr : (tangent ? P.Ht[l].as<double>() : P.H[l].as<double>());
     io.Yp[l] = P.Y[l].as<double>();
   }
-  constexpr size_t smem = sizeof(double) * W::F_SMEM_ACT;
-  static_assert(W::F_W <= EMB_WIMG, "W image buffer");
-  static int occ = 0;
-  if (!occ) {
+  constexpr size_t smem = sizeof(double) * W::W_SMEM;
+  static_assert(W::WNW >= 4, "emb_fwd_kernel: too few warps fit");
+  static bool attr = false;
+  if (!attr) {
     FEKF_CHECK_CUDA(cudaFuncSetAttribute(emb_fwd_kernel<W>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-    FEKF_CHECK_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, emb_fwd_kernel<W>, EMB_FWD_WARPS * 32, smem));
-    if (occ < 1) { set_error("emb_fwd_kernel: does not fit on an SM"); return FEKF_EINVAL; }
+    attr = true;
   }
   const double* wp = c.w.as<double>() + P.L[0].W;
-  double* wimg = P.wimg.as<double>();
-  emb_pack_kernel<W><<<8, 256, 0, s>>>(wp, wimg);
+  const long long wtiles = (Rmax + W::RT - 1) / W::RT;
+  const int grid = (int)std::max<long long>(1, std::min<long long>((wtiles + W::WNW - 1) / W::WNW, (long long)num_sms()));
+  emb_fwd_kernel<W><<<grid, W::WNW * 32, smem, s>>>(wp, io);
   FEKF_LAUNCH_CHECK();
-  const long long tiles = (Rmax + EMB_T - 1) / EMB_T;
-  const int grid = (int)std::max<long long>(1, std::min<long long>(tiles, (long long)num_sms() * occ));
-  emb_fwd_kernel<W><<<grid, EMB_FWD_WARPS * 32, smem, s>>>(wp, wimg, io);
-  FEKF_LAUNCH_CHECK();
-  count_launch(2);
+  count_launch(1);
   return FEKF_OK;
 }
 

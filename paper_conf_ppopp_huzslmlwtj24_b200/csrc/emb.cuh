@@ -1,7 +1,8 @@
-// Fused embedding-net kernels (sm_100a, fp64 DMMA m8n8k4): one CTA runs every layer of the
-// embedding net G = E_{L-1} o ... o E_0(s) (skip rule: reading Z12) on a tile of rows with
-// the activations resident in shared memory, instead of one GEMM launch per layer with the
-// activations round-tripping through HBM.  The kernels are compiled for the embedding widths of the
+// Fused embedding-net kernels (sm_100a, fp64 DMMA m8n8k4): every layer of the embedding net
+// G = E_{L-1} o ... o E_0(s) (skip rule: reading Z12) runs in one kernel with the activations
+// on chip, instead of one GEMM launch per layer with the activations round-tripping through HBM: the
+// forward per warp on 16-row tiles (no CTA barrier), the backward per CTA on 32-row tiles (its weight
+// gradients are split over the warps).  The kernels are compiled for the embedding widths of the
 // configured models (all index math constant-folded); other widths take the per-layer GEMM path.
 //
 // Shared-memory layout (doubles).  Every matrix uses a leading dimension ld = 16*ceil(w8/16) + 4
@@ -14,10 +15,8 @@
 
 namespace fekf {
 
-constexpr int EMB_T = 32;       // rows per CTA tile
-constexpr int EMB_FWD_WARPS = 8;
+constexpr int EMB_T = 32;       // rows per CTA tile of the backward
 constexpr int EMB_BWD_WARPS = 16;
-constexpr int EMB_WIMG = 1 << 14;   // doubles per pair for the padded global W image (forward, L1 path)
 
 __host__ __device__ constexpr int pad4(int x) { return (x + 3) & ~3; }
 __host__ __device__ constexpr int pad8(int x) { return (x + 7) & ~7; }
@@ -41,7 +40,7 @@ struct EmbW {
       if (parity < 0 || (l & 1) == parity) m = d(l) > m ? d(l) : m;
     return m;
   }
-  // ---- forward: W_0 [pad8(d0)] | W_l [pad4(din)][sld(d)] | b_l [pad8(d)] | act0 [T][ald0] | act1 [T][ald1]
+  // ---- forward: W_0 [pad8(d0)] | W_l [pad4(din)][sld(d)] | b_l [pad8(d)] | per-warp activations
   __host__ __device__ static constexpr int fW(int l) {
     int o = pad8(D0);
     for (int k = 1; k < l; ++k) o += pad4(din(k)) * sld(d(k));
@@ -52,16 +51,21 @@ struct EmbW {
     for (int k = 0; k < l; ++k) o += pad8(d(k));
     return o;
   }
-  __host__ __device__ static constexpr int fALD(int q) { return sld(maxw(q)); }
-  __host__ __device__ static constexpr int fA(int q) { return fB(NL) + (q ? T * fALD(0) : 0); }
-  static constexpr int F_SMEM = fA(1) + T * fALD(1);
-  // The forward kernel reads W through L1 from a zero-padded global image with the [0, F_W) part of the
-  // layout above (written once per launch by emb_pack_kernel); its SMEM holds only biases + activations,
-  // so more CTAs fit on an SM (the weights are shared by every CTA through L1).
-  static constexpr int F_W = fW(NL);
-  __host__ __device__ static constexpr int sB(int l) { return fB(l) - F_W; }
-  __host__ __device__ static constexpr int sA(int q) { return fA(q) - F_W; }
-  static constexpr int F_SMEM_ACT = F_SMEM - F_W;
+  // ---- warp-tiled forward (emb_fwd_kernel): W_l and b_l as above ([0, fB(NL)) of the layout), then per
+  // warp two activation buffers of RT rows (layer l's h in buffer l & 1, the last layer's never staged)
+  static constexpr int RT = 8;                                    // rows per warp tile (one DMMA strip)
+  __host__ __device__ static constexpr int wmaxw(int parity) {
+    int m = 1;
+    for (int l = 0; l + 1 < NL; ++l)
+      if ((l & 1) == parity) m = d(l) > m ? d(l) : m;
+    return m;
+  }
+  __host__ __device__ static constexpr int wALD(int q) { return sld(wmaxw(q)); }
+  static constexpr int WS = fB(NL);                              // weights + biases (doubles)
+  static constexpr int WRP = RT * (wALD(0) + wALD(1));           // per-warp activations (doubles)
+  static constexpr int WNW_FIT = (227 * 1024 / 8 - 32 - WS) / WRP;
+  static constexpr int WNW = WNW_FIT > 24 ? 24 : WNW_FIT;        // warps per CTA (one CTA per SM)
+  static constexpr int W_SMEM = WS + WNW * WRP;
   // ---- backward: W_0 | W_l [pad8(din)][sld(d)] | aug_l [T][sld(din+1)] | 3 x buf [T][BLD] | rr [T][8]
   __host__ __device__ static constexpr int bW(int l) {
     int o = pad8(D0);

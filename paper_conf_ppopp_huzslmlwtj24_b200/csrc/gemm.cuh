@@ -226,8 +226,9 @@ dgemm_kernel(const __grid_constant__ GemmGroup<Epi> G) {
   auto issue = [&](int buf, int k0) {
     if (a16t) {
 #pragma unroll
-      for (int q = 0; q < AE / 2; ++q) {
+      for (int q = 0; q < (AE + 1) / 2; ++q) {
         const int idx = tid + 256 * q;
+        if (AE & 1 && idx >= BM * GB_K / 2) break;
         const int kk = idx / (BM / 2), r = 2 * (idx % (BM / 2));
         const int m = m0 + r, k = k0 + kk;
         const bool kin = k < kend;
@@ -248,8 +249,9 @@ dgemm_kernel(const __grid_constant__ GemmGroup<Epi> G) {
       }
     } else if (a16) {
 #pragma unroll
-      for (int q = 0; q < AE / 2; ++q) {
+      for (int q = 0; q < (AE + 1) / 2; ++q) {
         const int idx = tid + 256 * q;
+        if (AE & 1 && idx >= BM * GB_K / 2) break;
         const int r = idx / (GB_K / 2), kk = 2 * (idx % (GB_K / 2));
         const int m = m0 + r, k = k0 + kk;
         const bool ok = m < M && k < kend;
@@ -274,8 +276,9 @@ dgemm_kernel(const __grid_constant__ GemmGroup<Epi> G) {
     }
     if (b16) {
 #pragma unroll
-      for (int q = 0; q < BE / 2; ++q) {
+      for (int q = 0; q < (BE + 1) / 2; ++q) {
         const int idx = tid + 256 * q;
+        if (BE & 1 && idx >= BN * GB_K / 2) break;
         int c, kk;
         if (!TB) { kk = idx / (BN / 2); c = 2 * (idx % (BN / 2)); } else { c = idx / (GB_K / 2); kk = 2 * (idx % (GB_K / 2)); }
         const int n = n0 + c, k = k0 + kk;
@@ -360,7 +363,8 @@ static fekf_status gemm_launch(GemmGroup<Epi>& G, cudaStream_t s) {
 }
 
 // One launch for every problem of the group.  Tile from the group's shape: N <= 32 -> 128x32
-// (embedding widths); otherwise 64x64 (warps 32x16) unless the group has many rows -> 128x64.
+// (embedding widths); N a multiple of 80 up to 320 (the fitting widths) -> 128x80; otherwise 64x64
+// (warps 32x16) unless the group has many rows -> 128x64.
 template <bool TA, bool TB, class Epi>
 static fekf_status gemm_group(GemmProb<Epi>* probs, int n, cudaStream_t s) {
   GemmGroup<Epi> G{};
@@ -376,6 +380,9 @@ static fekf_status gemm_group(GemmProb<Epi>* probs, int n, cudaStream_t s) {
   }
   if (G.n == 0) return FEKF_OK;
   if (nmax <= 32) return gemm_launch<128, 32, 32, 16, TA, TB>(G, s);
+  // the fitting widths (240): 128 x 80 tiles (warps 32 x 40) put N in 3 tiles and 6144 rows in 48, one
+  // wave of 144 CTAs on 148 SMs (64 x 64 tiles: 384 CTAs, 2.6 waves), with 0.45 fragment loads per DMMA
+  if (!TA && nmax % 80 == 0 && nmax <= 320 && rows >= 2048) return gemm_launch<128, 80, 32, 40, TA, TB>(G, s);
   if (rows < 65536) return gemm_launch<64, 64, 32, 16, TA, TB>(G, s);
   return gemm_launch<128, 64, 32, 32, TA, TB>(G, s);
 }

@@ -234,12 +234,24 @@ __device__ __forceinline__ void apply_corrections(PT* t, const double* vI, const
 #pragma unroll
       for (int j = 0; j < 8; ++j) dmma884k(c[j][0], c[j][1], a, b[j]);
     }
+    // The fragment puts 4 lanes on each of 8 rows (lane = 4 fr + fk, columns 8j + 2fk, +1).  Rows are
+    // 64 elements apart, so visiting the column chunks j in the same order on every row would land the
+    // lanes of one shared-memory phase (8 lanes for 16-byte fp64 pairs, 16 for 8-byte fp32 pairs) on the
+    // same banks.  Row fr visits chunk q ^ (fr & X) at step q instead (X = 1 fp64, 3 fp32): the rows of a
+    // phase then cover disjoint banks.  The accumulator is picked with compile-time indices (selects).
+    constexpr int X = sizeof(PT) == 8 ? 1 : 3;
+    const int rx = fr & X;
     PT* row = t + (m0 + fr) * KT + 2 * fk;
 #pragma unroll
-    for (int j = 0; j < 8; ++j) {
+    for (int q = 0; q < 8; ++q) {
+      double a0 = c[q][0], a1 = c[q][1];
+#pragma unroll
+      for (int x = 1; x <= X; ++x)
+        if (rx == x) { a0 = c[q ^ x][0]; a1 = c[q ^ x][1]; }
+      const int j = q ^ rx;
       double2 v = ld2(row + 8 * j);
-      v.x = sig * (v.x - c[j][0]);
-      v.y = sig * (v.y - c[j][1]);
+      v.x = sig * (v.x - a0);
+      v.y = sig * (v.y - a1);
       st2(row + 8 * j, v);
     }
   }
@@ -387,10 +399,7 @@ kf_pass_kernel(PT* __restrict__ P, const ItemD* __restrict__ items, int n_items,
       }
     }
     double* cr = colg + (tcount & 1) * (NGW * KT);
-    if (!diag) {
-      cr[wg * KT + c0] = ca0;
-      cr[wg * KT + c0 + 1] = ca1;
-    }
+    if (!diag) *reinterpret_cast<double2*>(cr + wg * KT + c0) = make_double2(ca0, ca1);
     asm volatile("bar.sync %0, %1;" ::"r"(1 + gi), "r"(GT) : "memory");
     if (tg == 0) {
       if (rw) {

@@ -26,7 +26,6 @@ struct PairNet {       // embedding net of the type pair (ti, tj)
   std::vector<DBuf> Y, H, Hb, Zb;       // primal   [R x d_l]
   std::vector<DBuf> Yt, Ht, Hbt, Zbt;   // tangent  [R x d_l] (only the first T rows are live)
   DBuf sbar;           // [R] adjoint of s (forces)
-  DBuf wimg;           // zero-padded W image for the fused forward (emb.cuh EMB_WIMG)
 };
 
 struct FitNet {        // fitting net of type t

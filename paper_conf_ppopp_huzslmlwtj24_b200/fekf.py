@@ -271,8 +271,10 @@ class KalmanFilter:
         (update_begin / partial_u / update_end)."""
         self.blocks = list(blocks)
         self._owner = _owner
+        self._h = C.c_void_p()
         if _handle is not None:
-            self.h = _handle
+            if _owner is None:
+                self._h = _handle
             self._own = False
         else:
             self.h = C.c_void_p()
@@ -285,6 +287,15 @@ class KalmanFilter:
                 _check(lib().fekf_kf_create(arr, len(self.blocks), C.byref(oc), comm.h if comm else None,
                                             C.byref(self.h)))
             self._own = True
+
+    @property
+    def h(self):
+        # a context's filter follows the context's handle (null once the context is closed)
+        return self._owner._kh if self._owner is not None else self._h
+
+    @h.setter
+    def h(self, v):
+        self._h = v
 
     def update(self, g, abe, sqrt_bs, w, stream=None):
         _check(lib().fekf_kf_update(self.h, _ptr(g, torch.float64, "g"), _ptr(abe, torch.float64, "abe"),
@@ -411,7 +422,7 @@ class Context:
         kh = C.c_void_p()
         _check(L.fekf_get_kf(self.h, C.byref(kh)))
         _, blocks = plan_layout(model, self.oc.block_size)
-        self.kf = KalmanFilter(blocks, _handle=kh, _owner=self)
+        self._kh, self._blocks = kh, blocks
         self.comm = comm
         if not graph:
             self.set_graph_mode(False)
@@ -430,6 +441,12 @@ class Context:
                 raise FekfError(1, f"env stats must be [{nt}][4]")
             return (C.c_double * len(flat))(*flat)
         _check(lib().fekf_set_env_stats(self.h, host(avg), host(std)))
+
+    @property
+    def kf(self):
+        """The context's filter (fekf_get_kf).  A fresh wrapper per access that keeps the context alive,
+        so the context itself holds no reference cycle and is freed as soon as the caller drops it."""
+        return KalmanFilter(self._blocks, _handle=self._kh, _owner=self)
 
     def set_graph_mode(self, enable: bool):
         """a10: replay each minibatch step as one captured CUDA graph (default) or launch eagerly."""
@@ -541,7 +558,7 @@ class Context:
 
     def close(self):
         if self.h:
-            self.kf.h = C.c_void_p()
+            self._kh = C.c_void_p()
             lib().fekf_destroy(self.h)
             self.h = C.c_void_p()
 
