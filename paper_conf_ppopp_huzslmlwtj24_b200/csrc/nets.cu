@@ -357,90 +357,131 @@ __global__ void emb_l0_kernel(int Rmax, const int* __restrict__ Rdev, int d, con
 }
 
 // X = R~^T G / N_m (4 x M) per atom and D = X^T X^< (Fig. 6); tangent: Xdot = (Rdot^T G + R~^T Gdot)/N_m,
-// Ddot = Xdot^T X^< + X^T Xdot^<.  One CTA per atom; fixed summation order over (tj, slot).
-__global__ void desc_fwd_kernel(Geo g, PairPtrs pp, FitPtrs fp, const double* __restrict__ em,
-                                const double* __restrict__ rdot, int tangent, double* __restrict__ X,
-                                double* __restrict__ Xd) {
+// Ddot = Xdot^T X^< + X^T Xdot^<.  One CTA (8 warps) per atom: warp w takes the atom's rows w, w + 8, ... of
+// every pair (lane l holds columns l, l + 32, l + 64, l + 96 of a row: one coalesced 8-byte load each); the
+// tangent pass skips the rows with no tangent row (tpos < 0) in the same loop.  The 8 warps' partial sums
+// are combined in a fixed order (deterministic).
+constexpr int DESC_THREADS = 256, DESC_MC = 4;   // columns per lane: M <= 128
+__global__ void __launch_bounds__(DESC_THREADS, 4)
+desc_fwd_kernel(const __grid_constant__ Geo g, const __grid_constant__ PairPtrs pp, const __grid_constant__ FitPtrs fp,
+                const double* __restrict__ em, const double* __restrict__ rdot, int tangent, double* __restrict__ X,
+                double* __restrict__ Xd) {
   extern __shared__ double sm[];
   const int M = g.M, M2 = g.M2, Nm = g.Nm;
   double* xs = sm;            // [4][M]
   double* xds = sm + 4 * M;   // [4][M]
   double* rs = xds + 4 * M;   // [Nm][4] R~ rows of the atom (contiguous in em)
   double* rds = rs + 4 * Nm;  // [Nm][4] R~dot rows
-  int* act = reinterpret_cast<int*>(rds + 4 * Nm);  // tangent: (slot, primal row, tangent row) of active rows
-  __shared__ int s_nact;
+  double* red = rds + 4 * Nm; // [8][4][128] per-warp partial sums of one column chunk
   const int atom = blockIdx.x;
   const int b = atom / g.Na, i = atom % g.Na;
   const int ti = g.types[i], k = g.tindex[i];
   const int e = b * g.ncnt[ti] + k;
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   for (int q = threadIdx.x; q < 4 * Nm; q += blockDim.x) {
-    rs[q] = em[(size_t)atom * Nm * 4 + q];
-    if (tangent) rds[q] = rdot[(size_t)atom * Nm * 4 + q];
+    cp_async8(rs + q, em + (size_t)atom * Nm * 4 + q, true);
+    if (tangent) cp_async8(rds + q, rdot + (size_t)atom * Nm * 4 + q, true);
   }
-  if (tangent && threadIdx.x == 0) {  // active rows of this atom, in (tj, slot) order
-    int n = 0;
+  cp_async_commit();
+  cp_async_wait<0>();
+  __syncthreads();
+  const double inv = 1.0 / g.Nm;
+  double* xw = tangent ? xds : xs;
+  double* xo = (tangent ? Xd : X) + (size_t)atom * 4 * M;
+  for (int m0 = 0; m0 < M; m0 += 32 * DESC_MC) {   // column chunks of 128 (one pass for M <= 128)
+    double acc[DESC_MC][4];
+#pragma unroll
+    for (int c = 0; c < DESC_MC; ++c) acc[c][0] = acc[c][1] = acc[c][2] = acc[c][3] = 0.0;
     for (int tj = 0; tj < g.nt; ++tj) {
       const int p = ti * g.nt + tj;
       const int r0 = pp.row_start[p][e], r1 = pp.row_start[p][e + 1];
-      for (int r = r0; r < r1; ++r) {
-        const int t = pp.tpos[p][r];
-        if (t >= 0) { act[3 * n] = (p << 16) | (g.sec[tj] + r - r0); act[3 * n + 1] = r; act[3 * n + 2] = t; ++n; }
-      }
-    }
-    s_nact = n;
-  }
-  __syncthreads();
-  for (int m = threadIdx.x; m < M; m += blockDim.x) {
-    double a0 = 0, a1 = 0, a2 = 0, a3 = 0;
-    if (!tangent) {
-      for (int tj = 0; tj < g.nt; ++tj) {
-        const int p = ti * g.nt + tj;
-        const int r0 = pp.row_start[p][e], r1 = pp.row_start[p][e + 1];
-        const double* G = pp.G[p] + m;
-        const double* er = rs + 4 * g.sec[tj];
-        int r = r0;
-        for (; r + 4 <= r1; r += 4) {  // four rows' loads in flight
-          double gv[4];
+      const double* er = rs + 4 * g.sec[tj];
+      const double* ed = rds + 4 * g.sec[tj];
+      constexpr int RS = DESC_THREADS / 32;
+      if (!tangent) {   // two rows per iteration: 8 loads in flight per lane
+        const double* Gp = pp.G[p];
+        int r = r0 + warp;
+        for (; r + RS < r1; r += 2 * RS) {
+          double gv[2][DESC_MC];
 #pragma unroll
-          for (int u = 0; u < 4; ++u) gv[u] = G[(size_t)(r + u) * M];
+          for (int u = 0; u < 2; ++u)
 #pragma unroll
-          for (int u = 0; u < 4; ++u) {
-            const double* q = er + 4 * (r + u - r0);
-            a0 = fma(q[0], gv[u], a0); a1 = fma(q[1], gv[u], a1); a2 = fma(q[2], gv[u], a2); a3 = fma(q[3], gv[u], a3);
+            for (int c = 0; c < DESC_MC; ++c) {
+              const int m = m0 + lane + 32 * c;
+              gv[u][c] = m < M ? Gp[(size_t)(r + u * RS) * M + m] : 0.0;
+            }
+#pragma unroll
+          for (int u = 0; u < 2; ++u) {
+            const double* q = er + 4 * (r + u * RS - r0);
+#pragma unroll
+            for (int c = 0; c < DESC_MC; ++c)
+#pragma unroll
+              for (int a = 0; a < 4; ++a) acc[c][a] = fma(q[a], gv[u][c], acc[c][a]);
           }
         }
-        for (; r < r1; ++r) {
-          const double gv = G[(size_t)r * M];
+        if (r < r1) {
           const double* q = er + 4 * (r - r0);
-          a0 = fma(q[0], gv, a0); a1 = fma(q[1], gv, a1); a2 = fma(q[2], gv, a2); a3 = fma(q[3], gv, a3);
+          double gv[DESC_MC];
+#pragma unroll
+          for (int c = 0; c < DESC_MC; ++c) {
+            const int m = m0 + lane + 32 * c;
+            gv[c] = m < M ? Gp[(size_t)r * M + m] : 0.0;
+          }
+#pragma unroll
+          for (int c = 0; c < DESC_MC; ++c)
+#pragma unroll
+            for (int a = 0; a < 4; ++a) acc[c][a] = fma(q[a], gv[c], acc[c][a]);
+        }
+        continue;
+      }
+      // tangent: the warp's rows r0 + warp + RS*l (l = lane) are tested 32 at a time (one tpos load each, in
+      // flight together); only the rows with a tangent row (R~dot, Gdot != 0) are visited
+      for (int base = r0 + warp; base < r1; base += 32 * RS) {
+        const int rl = base + RS * lane;
+        const int tl = rl < r1 ? pp.tpos[p][rl] : -1;
+        unsigned act = __ballot_sync(0xffffffffu, tl >= 0);
+        while (act) {
+          const int j = __ffs(act) - 1;
+          act &= act - 1;
+          const int r = base + RS * j;
+          const int t = __shfl_sync(0xffffffffu, tl, j);
+          const double* q = er + 4 * (r - r0);
+          const double* qd = ed + 4 * (r - r0);
+          double gv[DESC_MC], gd[DESC_MC];
+#pragma unroll
+          for (int c = 0; c < DESC_MC; ++c) {
+            const int m = m0 + lane + 32 * c;
+            gv[c] = m < M ? pp.G[p][(size_t)r * M + m] : 0.0;
+            gd[c] = m < M ? pp.Gt[p][(size_t)t * M + m] : 0.0;
+          }
+#pragma unroll
+          for (int c = 0; c < DESC_MC; ++c)
+#pragma unroll
+            for (int a = 0; a < 4; ++a) acc[c][a] = fma(qd[a], gv[c], fma(q[a], gd[c], acc[c][a]));
         }
       }
-    } else {
-      const int n = s_nact;
-      for (int a = 0; a < n; ++a) {
-        const int p = act[3 * a] >> 16, sl = act[3 * a] & 0xffff, r = act[3 * a + 1], t = act[3 * a + 2];
-        const double gv = pp.G[p][(size_t)r * M + m];
-        const double gd = pp.Gt[p][(size_t)t * M + m];
-        const double* er = rs + 4 * sl;
-        const double* ed = rds + 4 * sl;
-        a0 = fma(ed[0], gv, fma(er[0], gd, a0));
-        a1 = fma(ed[1], gv, fma(er[1], gd, a1));
-        a2 = fma(ed[2], gv, fma(er[2], gd, a2));
-        a3 = fma(ed[3], gv, fma(er[3], gd, a3));
-      }
     }
-    const double inv = 1.0 / g.Nm;
-    double* xw = tangent ? xds : xs;
-    double* xo = (tangent ? Xd : X) + (size_t)atom * 4 * M;
-    xw[m] = a0 * inv; xw[M + m] = a1 * inv; xw[2 * M + m] = a2 * inv; xw[3 * M + m] = a3 * inv;
-    xo[m] = xw[m]; xo[M + m] = xw[M + m]; xo[2 * M + m] = xw[2 * M + m]; xo[3 * M + m] = xw[3 * M + m];
-  }
-  __syncthreads();
-  if (tangent) {
-    const double* xo = X + (size_t)atom * 4 * M;
-    for (int q = threadIdx.x; q < 4 * M; q += blockDim.x) xs[q] = xo[q];
+#pragma unroll
+    for (int c = 0; c < DESC_MC; ++c)
+#pragma unroll
+      for (int a = 0; a < 4; ++a) red[(warp * 4 + a) * (32 * DESC_MC) + lane + 32 * c] = acc[c][a];
+    __syncthreads();
+    for (int q = threadIdx.x; q < 4 * 32 * DESC_MC; q += blockDim.x) {
+      const int a = q / (32 * DESC_MC), m = m0 + q % (32 * DESC_MC);
+      if (m >= M) continue;
+      double v = 0.0;
+#pragma unroll
+      for (int w = 0; w < DESC_THREADS / 32; ++w) v += red[(w * 4 + a) * (32 * DESC_MC) + q % (32 * DESC_MC)];
+      xw[a * M + m] = v * inv;
+      xo[a * M + m] = v * inv;
+    }
     __syncthreads();
   }
+  if (tangent) {
+    const double* xp = X + (size_t)atom * 4 * M;
+    for (int q = threadIdx.x; q < 4 * M; q += blockDim.x) xs[q] = xp[q];
+  }
+  __syncthreads();
   const long long row = (long long)b * g.ncnt[ti] + k;
   double* D = fp.D[ti] + (size_t)(tangent ? fp.F[ti] + row : row) * M * M2;
   for (int q = threadIdx.x; q < M * M2; q += blockDim.x) {
@@ -511,10 +552,12 @@ struct SeedOut {
   double* hbt[NP];
   double* dr[NP];
 };
-__global__ void __launch_bounds__(256)
-desc_bwd_seed_kernel(Geo g, FitPtrs fp, PairPtrs pp, SeedOut so, const double* __restrict__ X,
-                     const double* __restrict__ Xd, const double* __restrict__ em, const double* __restrict__ rdot,
-                     int dual, int force, int sel, double* __restrict__ Xb, double* __restrict__ Xdb) {
+template <bool dual, bool force, bool sel>
+__global__ void __launch_bounds__(256, dual ? 2 : 4)
+desc_bwd_seed_kernel(const __grid_constant__ Geo g, const __grid_constant__ FitPtrs fp,
+                     const __grid_constant__ PairPtrs pp, const __grid_constant__ SeedOut so,
+                     const double* __restrict__ X, const double* __restrict__ Xd, const double* __restrict__ em,
+                     const double* __restrict__ rdot, double* __restrict__ Xb, double* __restrict__ Xdb) {
   extern __shared__ double sm[];
   const int M = g.M, M2 = g.M2, Nm = g.Nm;
   double* xs = sm;               // [4][M]
@@ -532,87 +575,155 @@ desc_bwd_seed_kernel(Geo g, FitPtrs fp, PairPtrs pp, SeedOut so, const double* _
   const long long row = (long long)b * g.ncnt[ti] + k;
   const double* Dbp = fp.Db[ti] + (size_t)row * M * M2;
   const double* Ddbp = fp.Db[ti] + (size_t)(fp.F[ti] + row) * M * M2;
+  // staging with cp.async: every copy of the CTA in flight at once (no per-element load -> store latency)
   for (int e = tid; e < 4 * M; e += blockDim.x) {
-    xs[e] = X[(size_t)atom * 4 * M + e];
-    if (dual) xds[e] = Xd[(size_t)atom * 4 * M + e];
+    cp_async8(xs + e, X + (size_t)atom * 4 * M + e, true);
+    if (dual) cp_async8(xds + e, Xd + (size_t)atom * 4 * M + e, true);
   }
   for (int e = tid; e < M * M2; e += blockDim.x) {
     const int ep = (e / M2) * (M2 + 1) + e % M2;  // row stride M2 + 1: conflict-free in both loops below
-    db[ep] = Dbp[e];
-    if (dual) ddb[ep] = Ddbp[e];
+    cp_async8(db + ep, Dbp + e, true);
+    if (dual) cp_async8(ddb + ep, Ddbp + e, true);
   }
   for (int e = tid; e < 4 * Nm; e += blockDim.x) {
-    rs[e] = em[(size_t)atom * Nm * 4 + e];
-    if (dual) rds[e] = rdot[(size_t)atom * Nm * 4 + e];
+    cp_async8(rs + e, em + (size_t)atom * Nm * 4 + e, true);
+    if (dual) cp_async8(rds + e, rdot + (size_t)atom * Nm * 4 + e, true);
+  }
+  cp_async_commit();
+  cp_async_wait<0>();
+  __syncthreads();
+  // Eq. 4 in two phases so no thread runs a long serial chain: (A) the M-term sums of the first M^<
+  // columns, T[kk][p] = sum_m Dbar[m][p] x[kk][m] (p < M^<), by 4 threads each (M/4 terms, combined by
+  // shuffles in a fixed order); (B) the M^<-term sums of every (kk, p) plus T.  ta/td hold T in xbs/xdbs.
+  {
+    const int no = 4 * M2, part = tid & 3, no8 = (no + 7) & ~7;   // whole warps run the shuffles
+    for (int o = tid >> 2; o < no8; o += blockDim.x >> 2) {
+      const bool valid = o < no;
+      const int kk = valid ? o / M2 : 0, p = valid ? o % M2 : 0;
+      const double* x = xs + kk * M;
+      const double* xd = xds + kk * M;
+      double a = 0.0, ad = 0.0;
+      for (int m = part; valid && m < M; m += 4) {
+        a = fma(db[m * (M2 + 1) + p], x[m], a);
+        if (dual) {
+          a = fma(ddb[m * (M2 + 1) + p], xd[m], a);
+          ad = fma(ddb[m * (M2 + 1) + p], x[m], ad);
+        }
+      }
+      a += __shfl_xor_sync(0xffffffffu, a, 1);
+      a += __shfl_xor_sync(0xffffffffu, a, 2);
+      ad += __shfl_xor_sync(0xffffffffu, ad, 1);
+      ad += __shfl_xor_sync(0xffffffffu, ad, 2);
+      if (part == 0 && valid) {
+        xbs[kk * M + p] = a;
+        if (dual) xdbs[kk * M + p] = ad;
+      }
+    }
   }
   __syncthreads();
   for (int e = tid; e < 4 * M; e += blockDim.x) {
     const int kk = e / M, p = e % M;
     const double* x = xs + kk * M;
-    double a = 0.0, ad = 0.0;
+    double a = p < M2 ? xbs[e] : 0.0, ad = (dual && p < M2) ? xdbs[e] : 0.0;
     for (int n = 0; n < M2; ++n) a = fma(db[p * (M2 + 1) + n], x[n], a);
-    if (p < M2)
-      for (int m = 0; m < M; ++m) a = fma(db[m * (M2 + 1) + p], x[m], a);
     if (dual) {
       const double* xd = xds + kk * M;
       for (int n = 0; n < M2; ++n) { a = fma(ddb[p * (M2 + 1) + n], xd[n], a); ad = fma(ddb[p * (M2 + 1) + n], x[n], ad); }
-      if (p < M2)
-        for (int m = 0; m < M; ++m) { a = fma(ddb[m * (M2 + 1) + p], xd[m], a); ad = fma(ddb[m * (M2 + 1) + p], x[m], ad); }
-      xdbs[e] = ad;
-      Xdb[(size_t)atom * 4 * M + e] = ad;
     }
-    xbs[e] = a;
     Xb[(size_t)atom * 4 * M + e] = a;
+    if (dual) Xdb[(size_t)atom * 4 * M + e] = ad;
+  }
+  __syncthreads();   // every T read before the final values overwrite xbs / xdbs
+  for (int e = tid; e < 4 * M; e += blockDim.x) {
+    xbs[e] = Xb[(size_t)atom * 4 * M + e];
+    if (dual) xdbs[e] = Xdb[(size_t)atom * 4 * M + e];
   }
   __syncthreads();
   const double inv = 1.0 / Nm;
   const int e0 = b * g.ncnt[ti] + k;
-  for (int tj = 0; tj < g.nt; ++tj) {
-    const int p = ti * g.nt + tj;
-    const int r0 = pp.row_start[p][e0], nr = pp.row_start[p][e0 + 1] - r0;
-    const int* tpos = pp.tpos[p];
-    for (int s = warp; s < nr; s += blockDim.x >> 5) {
-      const int r = r0 + s;
-      if (sel && tpos[r] < 0) continue;   // MODE_FORCE_SEL: rows not touching the selected atoms
-      const double* q = rs + (g.sec[tj] + s) * 4;
-      const int t = dual ? tpos[r] : -1;
-      double pk0 = 0.0, pk1 = 0.0, pk2 = 0.0, pk3 = 0.0;
-      const double* Gr = force ? pp.G[p] + (size_t)r * M : nullptr;
-      for (int m0 = 0; m0 < M; m0 += 128) {
+  // per row: Gbar = (R~ Xbar [+ R~dot Xdotbar]) / N_m, [Hdotbar = R~ Xdotbar / N_m on tangent rows],
+  // [dR = G Xbar^T / N_m]; the lane's Xbar (Xdotbar) columns m = m0 + lane + 32 u stay in registers
+  for (int m0 = 0; m0 < M; m0 += 128) {
+    double xb[4][4], xdb[4][4];
+#pragma unroll
+    for (int u = 0; u < 4; ++u) {
+      const int m = m0 + lane + 32 * u;
+#pragma unroll
+      for (int a = 0; a < 4; ++a) {
+        xb[u][a] = m < M ? xbs[a * M + m] : 0.0;
+        xdb[u][a] = (dual && m < M) ? xdbs[a * M + m] : 0.0;
+      }
+    }
+    for (int tj = 0; tj < g.nt; ++tj) {
+      const int p = ti * g.nt + tj;
+      const int r0 = pp.row_start[p][e0], nr = pp.row_start[p][e0 + 1] - r0;
+      const int* __restrict__ tpos = pp.tpos[p];
+      double* __restrict__ gbar = so.gbar[p];
+      double* __restrict__ hbt = so.hbt[p];
+      double* __restrict__ dr = so.dr[p];
+      const double* __restrict__ Gp = pp.G[p];
+      const double* rsj = rs + g.sec[tj] * 4;
+      const double* rdsj = rds + g.sec[tj] * 4;
+      auto row_body = [&](int s_, int t) {
+        const int r = r0 + s_;
+        const double* q = rsj + s_ * 4;
+        const double q0 = q[0], q1 = q[1], q2 = q[2], q3 = q[3];
+        double d0 = 0.0, d1 = 0.0, d2 = 0.0, d3 = 0.0;
+        if (dual && t >= 0) { const double* qd = rdsj + s_ * 4; d0 = qd[0]; d1 = qd[1]; d2 = qd[2]; d3 = qd[3]; }
         double gv[4];
 #pragma unroll
-        for (int u = 0; u < 4; ++u) {  // this row's G loads all in flight before their use
+        for (int u = 0; u < 4; ++u) {
           const int m = m0 + lane + 32 * u;
-          gv[u] = (force && m < M) ? Gr[m] : 0.0;
+          gv[u] = (force && m < M) ? Gp[(size_t)r * M + m] : 0.0;
         }
+        double pk0 = 0.0, pk1 = 0.0, pk2 = 0.0, pk3 = 0.0;
 #pragma unroll
         for (int u = 0; u < 4; ++u) {
           const int m = m0 + lane + 32 * u;
           if (m >= M) continue;
-          double v = q[0] * xbs[m] + q[1] * xbs[M + m] + q[2] * xbs[2 * M + m] + q[3] * xbs[3 * M + m];
-          if (t >= 0) {
-            const double* qd = rds + (g.sec[tj] + s) * 4;
-            v += qd[0] * xdbs[m] + qd[1] * xdbs[M + m] + qd[2] * xdbs[2 * M + m] + qd[3] * xdbs[3 * M + m];
-            so.hbt[p][(size_t)t * M + m] =
-                (q[0] * xdbs[m] + q[1] * xdbs[M + m] + q[2] * xdbs[2 * M + m] + q[3] * xdbs[3 * M + m]) * inv;
+          double v = q0 * xb[u][0] + q1 * xb[u][1] + q2 * xb[u][2] + q3 * xb[u][3];
+          if (dual && t >= 0) {
+            v += d0 * xdb[u][0] + d1 * xdb[u][1] + d2 * xdb[u][2] + d3 * xdb[u][3];
+            hbt[(size_t)t * M + m] = (q0 * xdb[u][0] + q1 * xdb[u][1] + q2 * xdb[u][2] + q3 * xdb[u][3]) * inv;
           }
-          so.gbar[p][(size_t)r * M + m] = v * inv;
+          gbar[(size_t)r * M + m] = v * inv;
           if (force) {
-            pk0 = fma(gv[u], xbs[m], pk0);
-            pk1 = fma(gv[u], xbs[M + m], pk1);
-            pk2 = fma(gv[u], xbs[2 * M + m], pk2);
-            pk3 = fma(gv[u], xbs[3 * M + m], pk3);
+            pk0 = fma(gv[u], xb[u][0], pk0);
+            pk1 = fma(gv[u], xb[u][1], pk1);
+            pk2 = fma(gv[u], xb[u][2], pk2);
+            pk3 = fma(gv[u], xb[u][3], pk3);
           }
         }
-      }
-      if (force) {
-        for (int o = 16; o > 0; o >>= 1) {
-          pk0 += __shfl_xor_sync(0xffffffffu, pk0, o);
-          pk1 += __shfl_xor_sync(0xffffffffu, pk1, o);
-          pk2 += __shfl_xor_sync(0xffffffffu, pk2, o);
-          pk3 += __shfl_xor_sync(0xffffffffu, pk3, o);
+        if (force) {
+          for (int o = 16; o > 0; o >>= 1) {
+            pk0 += __shfl_xor_sync(0xffffffffu, pk0, o);
+            pk1 += __shfl_xor_sync(0xffffffffu, pk1, o);
+            pk2 += __shfl_xor_sync(0xffffffffu, pk2, o);
+            pk3 += __shfl_xor_sync(0xffffffffu, pk3, o);
+          }
+          if (lane < 4) {
+            const double pv = lane == 0 ? pk0 : lane == 1 ? pk1 : lane == 2 ? pk2 : pk3;
+            if (m0 == 0) dr[(size_t)r * 4 + lane] = pv * inv;
+            else dr[(size_t)r * 4 + lane] += pv * inv;
+          }
         }
-        if (lane < 4) so.dr[p][(size_t)r * 4 + lane] = (lane == 0 ? pk0 : lane == 1 ? pk1 : lane == 2 ? pk2 : pk3) * inv;
+      };
+      constexpr int RS = 8;   // warps
+      if (sel || dual) {
+        // rows tested 32 at a time per warp (tpos loads in flight together); MODE_FORCE_SEL visits only the
+        // rows touching the selected atoms, the dual pass every row with its tangent row (or -1)
+        for (int base = warp; base < nr; base += 32 * RS) {
+          const int sl = base + RS * lane;
+          const int tl = sl < nr ? tpos[r0 + sl] : -1;
+          unsigned act = __ballot_sync(0xffffffffu, sel ? tl >= 0 : sl < nr);
+          while (act) {
+            const int j = __ffs(act) - 1;
+            act &= act - 1;
+            row_body(base + RS * j, __shfl_sync(0xffffffffu, tl, j));
+          }
+        }
+      } else {
+        for (int s_ = warp; s_ < nr; s_ += RS) row_body(s_, -1);
       }
     }
   }
@@ -1141,10 +1252,15 @@ fekf_status model_forward(Ctx& c, int nb, bool tangent, cudaStream_t s) {
   // descriptor
   PairPtrs pp = make_pp(c);
   FitPtrs fp = make_fp(c, nb);
-  const size_t smem = (8 * (size_t)c.M + 8 * (size_t)c.Nm) * sizeof(double) + 3 * sizeof(int) * c.Nm;
+  const size_t smem = (8 * (size_t)c.M + 8 * (size_t)c.Nm + 4 * 32 * DESC_MC * (DESC_THREADS / 32)) * sizeof(double);
   const size_t Xoff = (size_t)c.B * c.Na * 4 * c.M;
-  desc_fwd_kernel<<<nb * c.Na, 128, smem, s>>>(g, pp, fp, c.em.as<double>(), c.rdot.as<double>(), tangent ? 1 : 0,
-                                               c.X.as<double>(), c.X.as<double>() + Xoff);
+  static size_t dattr = 0;
+  if (smem > dattr) {
+    FEKF_CHECK_CUDA(cudaFuncSetAttribute(desc_fwd_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    dattr = smem;
+  }
+  desc_fwd_kernel<<<nb * c.Na, DESC_THREADS, smem, s>>>(g, pp, fp, c.em.as<double>(), c.rdot.as<double>(),
+                                                        tangent ? 1 : 0, c.X.as<double>(), c.X.as<double>() + Xoff);
   FEKF_LAUNCH_CHECK();
   count_launch();
   // fitting nets (stacked rows: the tangent half starts at row F); one grouped GEMM per layer over types
@@ -1335,16 +1451,16 @@ fekf_status model_backward(Ctx& c, int nb, Mode mode, double* gout, cudaStream_t
       so.dr[p] = P.Zb[0].as<double>();
     }
     const size_t smem = (16 * (size_t)c.M + 2 * (size_t)c.M * (c.M2 + 1) + 8 * (size_t)c.Nm) * sizeof(double);
-    static size_t attr = 0;
-    if (smem > attr) {
-      FEKF_CHECK_CUDA(cudaFuncSetAttribute(desc_bwd_seed_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-      attr = smem;
-    }
-    desc_bwd_seed_kernel<<<nb * c.Na, 256, smem, s>>>(g, fp, pp, so, c.X.as<double>(), c.X.as<double>() + Xoff,
-                                                      c.em.as<double>(), c.rdot.as<double>(), dual ? 1 : 0,
-                                                      force ? 1 : 0, mode == MODE_FORCE_SEL ? 1 : 0,
-                                                      c.Xb.as<double>(),
-                                                      c.Xb.as<double>() + Xoff);
+    auto launch = [&](auto kern) -> fekf_status {
+      FEKF_CHECK_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+      kern<<<nb * c.Na, 256, smem, s>>>(g, fp, pp, so, c.X.as<double>(), c.X.as<double>() + Xoff, c.em.as<double>(),
+                                        c.rdot.as<double>(), c.Xb.as<double>(), c.Xb.as<double>() + Xoff);
+      return FEKF_OK;
+    };
+    if (dual) FEKF_TRY(launch(desc_bwd_seed_kernel<true, false, false>));
+    else if (mode == MODE_FORCE_SEL) FEKF_TRY(launch(desc_bwd_seed_kernel<false, true, true>));
+    else if (force) FEKF_TRY(launch(desc_bwd_seed_kernel<false, true, false>));
+    else FEKF_TRY(launch(desc_bwd_seed_kernel<false, false, false>));
   } else {
     const size_t smem = (8 * c.M + 2 * c.M * (c.M2 + 1)) * sizeof(double);
     desc_bwd_kernel<<<nb * c.Na, 128, smem, s>>>(g, fp, c.X.as<double>(), c.X.as<double>() + Xoff, dual ? 1 : 0,
