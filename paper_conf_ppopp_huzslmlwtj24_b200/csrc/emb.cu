@@ -135,9 +135,9 @@ struct EmbFwdIO {
 // them directly, the next layer's A operand goes through the warp's own SMEM buffer (__syncwarp only).
 // The next tile's inputs (row -> primal row -> slot -> s) are fetched in three dependent steps spread over
 // the current tile's layers.  Tangent rows: ydot = (1 - y^2) zdot with y of the primal row, no bias.
-template <class W, int L>
+template <class W, int L, bool tan>
 __device__ __forceinline__ void wfwd_layer(const double* __restrict__ sm, double* __restrict__ wb,
-                                           const EmbFwdIO& io, int r0, int R, bool tan, const int (&prs)[W::RT / 8]) {
+                                           const EmbFwdIO& io, int r0, int R, const int (&prs)[W::RT / 8]) {
   constexpr int MS = W::RT / 8;   // 8-row DMMA strips per warp tile
   constexpr int din = W::din(L), d = W::d(L), K4 = pad4(din), NT = pad8(d) / 8, skip = W::skip(L);
   constexpr bool last = L + 1 == W::NL;
@@ -172,6 +172,17 @@ __device__ __forceinline__ void wfwd_layer(const double* __restrict__ sm, double
     const int r = 8 * i + fr, row = r0 + r;
     const bool live = row < R;
     const int pr = prs[i];
+    // tangent rows: the primal row's y of every output of this strip, all gathers in flight at once
+    double ypv[tan ? NT : 1][2];
+    if constexpr (tan) {
+#pragma unroll
+      for (int j = 0; j < NT; ++j)
+#pragma unroll
+        for (int q = 0; q < 2; ++q) {
+          const int cc = 8 * j + 2 * fk + q;
+          ypv[j][q] = (cc < d && pr >= 0) ? Ypl[(size_t)pr * d + cc] : 0.0;
+        }
+    }
 #pragma unroll
     for (int j = 0; j < NT; ++j) {
       const int c = 8 * j + 2 * fk;
@@ -179,8 +190,8 @@ __device__ __forceinline__ void wfwd_layer(const double* __restrict__ sm, double
 #pragma unroll
       for (int q = 0; q < 2; ++q) {
         const int cc = c + q;
-        if (tan) {
-          const double yp = (cc < d && pr >= 0) ? Ypl[(size_t)pr * d + cc] : 0.0;
+        if constexpr (tan) {
+          const double yp = ypv[j][q];
           y[q] = (1.0 - yp * yp) * acc[i][j][q];
         } else {
           y[q] = tanh_fp64(acc[i][j][q] + bs[cc]);
@@ -207,12 +218,16 @@ __device__ __forceinline__ void wfwd_layer(const double* __restrict__ sm, double
   __syncwarp();
 }
 
-template <class W>
-__global__ void __launch_bounds__(W::WNW * 32, 1) emb_fwd_kernel(const double* __restrict__ wp, EmbFwdIO io) {
+// warps per CTA: the primal forward fills the SM; the tangent forward (a few % of the rows, no tanh,
+// gathers of the primal y) runs 12 warps with the register room to keep a strip's gathers in flight
+template <class W, bool tan>
+__host__ __device__ constexpr int fwd_warps() { return tan ? (W::WNW < 12 ? W::WNW : 12) : W::WNW; }
+
+template <class W, bool tan>
+__global__ void __launch_bounds__(fwd_warps<W, tan>() * 32, 1) emb_fwd_kernel(const double* __restrict__ wp, EmbFwdIO io) {
   extern __shared__ __align__(16) double sm[];
-  constexpr int NL = W::NL, RT = W::RT, NW = W::WNW, d0 = W::d(0), d0p = pad8(d0), LD0 = W::wALD(0);
+  constexpr int NL = W::NL, RT = W::RT, NW = fwd_warps<W, tan>(), d0 = W::d(0), d0p = pad8(d0), LD0 = W::wALD(0);
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31, fr = lane >> 2;
-  const bool tan = io.tidx != nullptr;
   const int R = min(io.Rmax, *io.Rdev);
   // ---- stage W_l [pad4(din)][sld(d)] (zero padded) and b_l once per CTA
   for (int c = tid; c < d0p; c += NW * 32) sm[W::fW(0) + c] = c < d0 ? __ldg(wp + W::goff(0) + c) : 0.0;
@@ -250,17 +265,27 @@ __global__ void __launch_bounds__(W::WNW * 32, 1) emb_fwd_kernel(const double* _
     {
       const double* w0 = sm + W::fW(0);
       const double* b0 = sm + W::fB(0);
-#pragma unroll 2
-      for (int e = lane; e < RT * d0p; e += 32) {
+      constexpr int E0 = (RT * d0p + 31) / 32;
+      double yp0[tan ? E0 : 1];
+      if constexpr (tan) {   // the primal y_0 of every element first (gathers in flight together)
+#pragma unroll
+        for (int u = 0; u < E0; ++u) {
+          const int e = lane + 32 * u, r = e / d0p, c = e % d0p;
+          const int pr = __shfl_sync(0xffffffffu, cur_pr, r & (RT - 1));
+          yp0[u] = (e < RT * d0p && c < d0 && pr >= 0) ? io.Yp[0][(size_t)pr * d0 + c] : 0.0;
+        }
+      }
+#pragma unroll
+      for (int u = 0; u < E0; ++u) {
+        const int e = lane + 32 * u;
+        if (e >= RT * d0p) break;
         const int r = e / d0p, c = e % d0p;
         const double sv = __shfl_sync(0xffffffffu, s_in, r);
-        const int pr = __shfl_sync(0xffffffffu, cur_pr, r);
         double h = 0.0;
         if (c < d0) {
           const double z = sv * w0[c];
-          if (tan) {
-            const double yp = pr >= 0 ? io.Yp[0][(size_t)pr * d0 + c] : 0.0;
-            h = (1.0 - yp * yp) * z;
+          if constexpr (tan) {
+            h = (1.0 - yp0[u] * yp0[u]) * z;
           } else {
             h = tanh_fp64(z + b0[c]);
           }
@@ -273,10 +298,10 @@ __global__ void __launch_bounds__(W::WNW * 32, 1) emb_fwd_kernel(const double* _
       }
       __syncwarp();
     }
-    if constexpr (NL >= 2) wfwd_layer<W, 1>(sm, wb, io, r0, R, tan, prs);
+    if constexpr (NL >= 2) wfwd_layer<W, 1, tan>(sm, wb, io, r0, R, prs);
     fetch_b();
-    if constexpr (NL >= 3) wfwd_layer<W, 2>(sm, wb, io, r0, R, tan, prs);
-    if constexpr (NL >= 4) wfwd_layer<W, 3>(sm, wb, io, r0, R, tan, prs);
+    if constexpr (NL >= 3) wfwd_layer<W, 2, tan>(sm, wb, io, r0, R, prs);
+    if constexpr (NL >= 4) wfwd_layer<W, 3, tan>(sm, wb, io, r0, R, prs);
     fetch_c();
   }
 }
@@ -297,17 +322,18 @@ static fekf_status emb_forward_t(Ctx& c, int p, long long Rmax, bool tangent, cu
     io.H[l] = l + 1 < W::NL ? nullptr : (tangent ? P.Ht[l].as<double>() : P.H[l].as<double>());
     io.Yp[l] = P.Y[l].as<double>();
   }
-  constexpr size_t smem = sizeof(double) * W::W_SMEM;
   static_assert(W::WNW >= 4, "emb_fwd_kernel: too few warps fit");
-  static bool attr = false;
-  if (!attr) {
-    FEKF_CHECK_CUDA(cudaFuncSetAttribute(emb_fwd_kernel<W>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-    attr = true;
-  }
   const double* wp = c.w.as<double>() + P.L[0].W;
   const long long wtiles = (Rmax + W::RT - 1) / W::RT;
-  const int grid = (int)std::max<long long>(1, std::min<long long>((wtiles + W::WNW - 1) / W::WNW, (long long)num_sms()));
-  emb_fwd_kernel<W><<<grid, W::WNW * 32, smem, s>>>(wp, io);
+  auto launch = [&](auto kern, int nw) -> fekf_status {
+    const size_t smem = sizeof(double) * (W::WS + (size_t)nw * W::WRP);
+    FEKF_CHECK_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    const int grid = (int)std::max<long long>(1, std::min<long long>((wtiles + nw - 1) / nw, (long long)num_sms()));
+    kern<<<grid, nw * 32, smem, s>>>(wp, io);
+    return FEKF_OK;
+  };
+  if (tangent) FEKF_TRY(launch(emb_fwd_kernel<W, true>, fwd_warps<W, true>()));
+  else FEKF_TRY(launch(emb_fwd_kernel<W, false>, fwd_warps<W, false>()));
   FEKF_LAUNCH_CHECK();
   count_launch(1);
   return FEKF_OK;
