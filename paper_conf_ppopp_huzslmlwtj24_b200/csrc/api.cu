@@ -304,7 +304,7 @@ fekf_status Ctx::init(const fekf_model_cfg& mm, const fekf_opt_cfg& oo, int nato
     while (late < (int)blocks.size() && acc < emb_end) acc += blocks[late++];
     kf->late_blocks = late;
     const char* e = getenv("FEKF_SPLIT_SMS");
-    kf->split_sms = comm ? 0 : (e ? atoi(e) : (o.precision == 32 ? 80 : 96));   // measured defaults
+    kf->split_sms = e ? atoi(e) : (o.precision == 32 ? 80 : 96);   // measured defaults
   }
   FEKF_TRY(kf->create(blocks, o, comm));
   if (kf->split_sms > 0) FEKF_CHECK_CUDA(cudaEventCreateWithFlags(&ev_fit, cudaEventDisableTiming));
@@ -422,7 +422,7 @@ static fekf_status step_body(Ctx& c, const double* coord, const double* box, con
   FEKF_TRY(geometry(c, coord, box, nb, s));
   // energy update (1 per minibatch); with one GPU the P pass of the fitting blocks overlaps the tail of
   // the reverse pass (split pass, Kf::pass)
-  const bool split = c.ev_fit && !c.comm;
+  const bool split = c.ev_fit != nullptr;
   static const int split_e = [] { const char* e = getenv("FEKF_SPLIT_E"); return e ? atoi(e) : 0; }();  // measured: 0
   c.split_armed = split && split_e;
   FEKF_TRY(energy_grad_pass(c, nb, e_label, g, esum, s));
@@ -436,9 +436,21 @@ static fekf_status step_body(Ctx& c, const double* coord, const double* box, con
   const int apg = c.o.atoms_per_group;
   for (int k = 0; k < c.o.force_groups; ++k) {
     FEKF_TRY(force_grad_pass(c, nb, f_label, force_idx + (size_t)k * apg, apg, g, esum, s));
+    const double scale = 1.0 / ((double)c.Bg * apg * 3) / c.Na;
+    if (split && c.comm) {
+      // N > 1 with the split pass: the early reduction of [g || error sum] is done by the pass in two
+      // segments (fitting blocks + error sum on the side stream as soon as they are final, embedding blocks
+      // after the reverse pass), so the Kalman stream still overlaps the reverse pass
+      FEKF_TRY(c.kf->update_begin(g, s, c.ev_fit, g));
+      abe_kernel<<<1, 1, 0, s>>>(esum, scale, c.abe.as<double>(), k < 4 ? metrics + 1 + k : nullptr);
+      FEKF_LAUNCH_CHECK();
+      count_launch();
+      if (!c.kf->replicated) FEKF_TRY(comm_allreduce(c.comm, c.kf->ub.as<double>(), c.kf->plan.Npad, s));
+      FEKF_TRY(c.kf->update_end(c.abe.as<double>(), sqrt_bs, c.w.as<double>(), s));
+      continue;
+    }
     FEKF_TRY(comm_allreduce(c.comm, g, c.Np + 1, s));
-    abe_kernel<<<1, 1, 0, s>>>(esum, 1.0 / ((double)c.Bg * apg * 3) / c.Na, c.abe.as<double>(),
-                               k < 4 ? metrics + 1 + k : nullptr);
+    abe_kernel<<<1, 1, 0, s>>>(esum, scale, c.abe.as<double>(), k < 4 ? metrics + 1 + k : nullptr);
     FEKF_LAUNCH_CHECK();
     count_launch();
     FEKF_TRY(c.kf->update(g, c.abe.as<double>(), sqrt_bs, c.w.as<double>(), s, split ? c.ev_fit : nullptr));

@@ -683,7 +683,7 @@ fekf_status Kf::create(const std::vector<int>& blocks, const fekf_opt_cfg& o, fe
   }
   ng = p32 ? 2 : 1;   // fp64: one group (measured: a second group slows the read-write pass)
   if (const char* e = getenv("FEKF_FP64_NG")) if (!p32 && atoi(e) == 2) ng = 2;   // experiments
-  plan.build(blocks, world, rank, SEG_TILES, ng, world == 1 ? std::min<int>(late_blocks, (int)blocks.size()) : 0);
+  plan.build(blocks, world, rank, SEG_TILES, ng, std::min<int>(late_blocks, (int)blocks.size()));
   const KfPlan& p = plan;
   FEKF_TRY(dalloc(P, (size_t)p.tiles_local * TILE_ELEMS * elem() + 16));
   FEKF_TRY(dalloc(items_d, std::max<size_t>(1, p.items.size()) * sizeof(ItemD)));
@@ -729,7 +729,7 @@ fekf_status Kf::create(const std::vector<int>& blocks, const fekf_opt_cfg& o, fe
     else kf_init_kernel<<<(unsigned)p.items.size(), 256>>>(P.as<double>(), items_d.as<ItemD>(), n_d.as<int>());
     FEKF_LAUNCH_CHECK();
   }
-  if (split_sms > 0 && plan.n_early > 0 && !comm && world == 1) {
+  if (split_sms > 0 && plan.n_early > 0) {
     // highest priority: the early pass's CTAs take SMs ahead of the reverse pass's queued CTAs
     int lo = 0, hi = 0;
     FEKF_CHECK_CUDA(cudaDeviceGetStreamPriorityRange(&lo, &hi));
@@ -845,9 +845,10 @@ fekf_status Kf::pass_launch(bool rw, int i0, int n, int* ctr, int grid, cudaStre
   return FEKF_OK;
 }
 
-fekf_status Kf::pass(const double* g, bool rw, cudaStream_t s, cudaEvent_t ready) {
+fekf_status Kf::pass(const double* g, bool rw, cudaStream_t s, cudaEvent_t ready, double* ar_g) {
   FEKF_TRY(idle_check("kf_pass"));
   const KfPlan& p = plan;
+  if (ar_g && !comm) ar_g = nullptr;
   const int tb = 256;
   const int n_items = (int)p.items.size();
   const bool split = ready && side && split_sms > 0 && p.n_early > 0;
@@ -855,6 +856,8 @@ fekf_status Kf::pass(const double* g, bool rw, cudaStream_t s, cudaEvent_t ready
     // early blocks: pad + pass on the side stream as soon as their gradient is final
     const long long p0 = p.tc_off[p.late_blocks] * KT;
     FEKF_CHECK_CUDA(cudaStreamWaitEvent(side, ready, 0));
+    // the early blocks' gradient segment and the error sum g[N] are final: their all-reduce goes first
+    if (ar_g) FEKF_TRY(comm_allreduce(comm, ar_g + p.off[p.late_blocks], p.N + 1 - p.off[p.late_blocks], side));
     // diagnostic pair (timing only): early pass start on the side stream -> the producing stream is done
     // with the reverse pass (index, not pointer: the pair lists grow below)
     std::vector<EvPair>* dl = nullptr;
@@ -888,6 +891,7 @@ fekf_status Kf::pass(const double* g, bool rw, cudaStream_t s, cudaEvent_t ready
     if (dl)
       FEKF_CHECK_CUDA(cudaEventRecordWithFlags((*dl)[di].b, s, capturing ? cudaEventRecordExternal : cudaEventRecordDefault));
     // late blocks on the producing stream
+    if (ar_g && p.off[p.late_blocks] > 0) FEKF_TRY(comm_allreduce(comm, ar_g, p.off[p.late_blocks], s));
     if (p0 > 0) {
       kf_pad_kernel<<<cdiv(p0, tb), tb, 0, s>>>(g, gpad.as<double>(), tc_blk.as<int>(), tc_c.as<int>(),
                                                 off_d.as<long long>(), n_d.as<int>(), 0, p0);
@@ -901,6 +905,7 @@ fekf_status Kf::pass(const double* g, bool rw, cudaStream_t s, cudaEvent_t ready
                          counter2.as<int>()));
     FEKF_CHECK_CUDA(cudaStreamWaitEvent(s, ev_early, 0));
   } else {
+    if (ar_g) FEKF_TRY(comm_allreduce(comm, ar_g, p.N + 1, s));
     kf_pad_kernel<<<cdiv(p.Npad, tb), tb, 0, s>>>(g, gpad.as<double>(), tc_blk.as<int>(), tc_c.as<int>(),
                                                    off_d.as<long long>(), n_d.as<int>(), 0, p.Npad);
     FEKF_LAUNCH_CHECK();
@@ -928,10 +933,10 @@ fekf_status Kf::update(const double* g, const double* abe, double sqrt_bs, doubl
   return update_end(abe, sqrt_bs, w, s);
 }
 
-fekf_status Kf::update_begin(const double* g, cudaStream_t s, cudaEvent_t ready) {
+fekf_status Kf::update_begin(const double* g, cudaStream_t s, cudaEvent_t ready, double* ar_g) {
   if (in_update || naive_n > 0) { set_error("kf update_begin: previous update not ended"); return FEKF_ESTATE; }
   cur_rw = npend >= defer;
-  FEKF_TRY(pass(g, cur_rw, s, ready));
+  FEKF_TRY(pass(g, cur_rw, s, ready, ar_g));
   in_update = true;
   return FEKF_OK;
 }

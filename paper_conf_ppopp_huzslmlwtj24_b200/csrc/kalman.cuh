@@ -101,21 +101,26 @@ struct Kf {
   // world/rank > 0 without a communicator: shard plan of that rank, exchange of u left to the caller
   fekf_status create(const std::vector<int>& blocks, const fekf_opt_cfg& o, fekf_comm* c, int world = 0, int rank = 0);
   ~Kf();
-  // Split pass (single process): with `ready` (an event recorded on the producing stream once the early
-  // blocks' gradient is final) the early items stream on `split_sms` SMs from a side stream while the
-  // producer finishes the late blocks' gradient; the late items follow on `s`.
+  // Split pass: with `ready` (an event recorded on the producing stream once the early blocks' gradient is
+  // final) the early items stream on `split_sms` SMs from a side stream while the producer finishes the late
+  // blocks' gradient; the late items follow on `s`.  With a communicator the gradient's all-reduce is split
+  // the same way (pass(ar_g)), so the overlap survives at N > 1.
   int late_blocks = 0, split_sms = 0;
   cudaStream_t side = nullptr;
   cudaEvent_t ev_early = nullptr, ev_ctr = nullptr;
   DBuf counter2;
-  fekf_status pass(const double* g, bool rw, cudaStream_t s, cudaEvent_t ready = nullptr);
+  // ar_g (with a communicator): g is not yet all-reduced over the ranks; the pass all-reduces it in place, in
+  // two segments with the split (the early blocks' segment and the error sum at g[N] on the side stream as
+  // soon as `ready` fires, the late blocks' segment on `s`), else in one piece on `s` (the early reduction,
+  // P:L170)
+  fekf_status pass(const double* g, bool rw, cudaStream_t s, cudaEvent_t ready = nullptr, double* ar_g = nullptr);
   fekf_status pass_launch(bool rw, int i0, int n, int* ctr, int grid, cudaStream_t s, int part = 0, int i2 = 0,
                           int n2 = 0, int* ctr2 = nullptr, bool zero_ctr = true);
   fekf_status update(const double* g, const double* abe, double sqrt_bs, double* w, cudaStream_t s,
                      cudaEvent_t ready = nullptr);
   // update = begin (P pass: this rank's partial u) + all-reduce of u over ranks + end (A, K, w, lambda)
   bool in_update = false, cur_rw = false;
-  fekf_status update_begin(const double* g, cudaStream_t s, cudaEvent_t ready = nullptr);
+  fekf_status update_begin(const double* g, cudaStream_t s, cudaEvent_t ready = nullptr, double* ar_g = nullptr);
   fekf_status update_end(const double* abe, double sqrt_bs, double* w, cudaStream_t s);
   fekf_status flush(cudaStream_t s);
   fekf_status idle_check(const char* what) const;   // FEKF_ESTATE between an update's begin and end

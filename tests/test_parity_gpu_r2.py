@@ -300,7 +300,8 @@ def test_loopback_ranks_train_step(world, p_mode):
     """B_g = 8 images over `world` contexts on one GPU (local batch 8/world), P sharded by tile-row
     segments (p_mode 0: partial u all-reduced) or replicated (p_mode 1), [g || sum|e|] all-reduced
     (the early reduction), sqrt(B_g) and ABE / B_g (readings Z2-Z4): 3 minibatch steps with
-    N_b = 1024 (several blocks, read-write passes at p_defer 2) equal oracle.train_step on the global batch."""
+    N_b = 1024 (several blocks, read-write passes at p_defer 2) equal oracle.train_step on the global batch.
+    The force updates keep the split P pass at N > 1 (gradient all-reduced in two segments)."""
     wl = get_config("c1_cu32")
     m = wl.model
     opt = OptConfig(block_size=1024, p_defer=2, p_mode=p_mode)
@@ -314,6 +315,7 @@ def test_loopback_ranks_train_step(world, p_mode):
     for c in ctxs:
         c.set_params(cu(w0))
     torch.cuda.synchronize()
+    ctxs[0].kf.timing(True)
     steps = 3
     groups = [force_groups(na, s, 17, opt.force_groups, opt.atoms_per_group) for s in range(steps)]
 
@@ -327,6 +329,10 @@ def test_loopback_ranks_train_step(world, p_mode):
         return mets, ctxs[r].get_params().cpu().numpy()
 
     outs = _run_ranks(world, fn)
+    ctxs[0].kf.timing(False)
+    # the split pass stays on with a communicator: the all-reduce of g runs in two segments (the fitting
+    # blocks' on the side stream ahead of the early pass), the late launch ran
+    assert ctxs[0].kf.timing_parts()[1] > 0.0
     st = O.FEKF.create(w0, m, opt)
     refs = [O.train_step(st, ds["coord"], ds["box"], ds["types"], ds["energy"], ds["force"], groups[s], m, opt)
             for s in range(steps)]
@@ -416,3 +422,23 @@ def test_bench_config_step_closed_form():
         dP = P2 - np.eye(n) / lam1     # the rank-2 part, held element-wise
         assert elem_rel(Pg - np.eye(n) / lam1, dP, 1e-4) < 1e-6
     ctx.close()
+
+
+# ------------------------------------------------------------------------------------------
+# the large-batch preset (B_g > 1024: lambda0 0.90, nu 0.996)
+# ------------------------------------------------------------------------------------------
+def test_large_batch_preset_train_steps():
+    """A global minibatch of 1100 images (> 1024, so fekf_opt_defaults gives the paper's large-batch
+    setting lambda0 = 0.90, nu = 0.996) in one context (local batch 1100: the energy seeds of
+    more than 1024 images per launch) against the oracle, 2 minibatch steps, rel 1e-9."""
+    wl = get_config("t2_tiny")
+    m = wl.model
+    d = fk.opt_defaults(1100)
+    assert d["lambda0"] == 0.90 and d["nu"] == 0.996
+    opt = OptConfig(**{k: d[k] for k in ("lambda0", "nu", "block_size", "noise_mode", "grad_reduce", "force_groups",
+                                         "atoms_per_group", "p_defer")})
+    B = 1100
+    ds = make_dataset("t2_tiny", B)
+    na = len(ds["types"])
+    w0 = init_weights(m, 3, float(ds["energy"].mean() / na))
+    _train_compare(m, opt, ds, w0, B=B, steps=2, tol=1e-9)
