@@ -420,40 +420,38 @@ static fekf_status step_body(Ctx& c, const double* coord, const double* box, con
   double* esum = g + c.Np;
   FEKF_CHECK_CUDA(cudaMemsetAsync(metrics, 0, sizeof(double) * 8, s));
   FEKF_TRY(geometry(c, coord, box, nb, s));
-  // energy update (1 per minibatch); with one GPU the P pass of the fitting blocks overlaps the tail of
-  // the reverse pass (split pass, Kf::pass)
+  // Every update's P pass starts on the fitting blocks as soon as their gradient is final and overlaps
+  // the tail of the reverse pass (split pass, Kf::pass); with a communicator the early reduction of
+  // [g || error sum] is split the same way (Kf::pass ar_g), so the overlap holds at N > 1 too.
   const bool split = c.ev_fit != nullptr;
-  static const int split_e = [] { const char* e = getenv("FEKF_SPLIT_E"); return e ? atoi(e) : 0; }();  // measured: 0
+  // measured: round 1 kept the energy update unsplit (its reverse-pass tail was too short
+  // to cover the slower 96-SM pass); with round 2's nets 1 wins (593 / 591 vs 586 / 585 images/s)
+  static const int split_e = [] { const char* e = getenv("FEKF_SPLIT_E"); return e ? atoi(e) : 1; }();
+  auto kalman = [&](double scale, double* metric) -> fekf_status {
+    if (c.split_armed && c.comm) {
+      FEKF_TRY(c.kf->update_begin(g, s, c.ev_fit, g));
+      abe_kernel<<<1, 1, 0, s>>>(esum, scale, c.abe.as<double>(), metric);
+      FEKF_LAUNCH_CHECK();
+      count_launch();
+      if (!c.kf->replicated) FEKF_TRY(comm_allreduce(c.comm, c.kf->ub.as<double>(), c.kf->plan.Npad, s));
+      return c.kf->update_end(c.abe.as<double>(), sqrt_bs, c.w.as<double>(), s);
+    }
+    FEKF_TRY(comm_allreduce(c.comm, g, c.Np + 1, s));
+    abe_kernel<<<1, 1, 0, s>>>(esum, scale, c.abe.as<double>(), metric);
+    FEKF_LAUNCH_CHECK();
+    count_launch();
+    return c.kf->update(g, c.abe.as<double>(), sqrt_bs, c.w.as<double>(), s, c.split_armed ? c.ev_fit : nullptr);
+  };
+  // energy update (1 per minibatch)
   c.split_armed = split && split_e;
   FEKF_TRY(energy_grad_pass(c, nb, e_label, g, esum, s));
-  FEKF_TRY(comm_allreduce(c.comm, g, c.Np + 1, s));
-  abe_kernel<<<1, 1, 0, s>>>(esum, 1.0 / c.Bg, c.abe.as<double>(), metrics + 0);
-  FEKF_LAUNCH_CHECK();
-  count_launch();
-  FEKF_TRY(c.kf->update(g, c.abe.as<double>(), sqrt_bs, c.w.as<double>(), s, c.split_armed ? c.ev_fit : nullptr));
+  FEKF_TRY(kalman(1.0 / c.Bg, metrics + 0));
   c.split_armed = split;
   // force updates
   const int apg = c.o.atoms_per_group;
   for (int k = 0; k < c.o.force_groups; ++k) {
     FEKF_TRY(force_grad_pass(c, nb, f_label, force_idx + (size_t)k * apg, apg, g, esum, s));
-    const double scale = 1.0 / ((double)c.Bg * apg * 3) / c.Na;
-    if (split && c.comm) {
-      // N > 1 with the split pass: the early reduction of [g || error sum] is done by the pass in two
-      // segments (fitting blocks + error sum on the side stream as soon as they are final, embedding blocks
-      // after the reverse pass), so the Kalman stream still overlaps the reverse pass
-      FEKF_TRY(c.kf->update_begin(g, s, c.ev_fit, g));
-      abe_kernel<<<1, 1, 0, s>>>(esum, scale, c.abe.as<double>(), k < 4 ? metrics + 1 + k : nullptr);
-      FEKF_LAUNCH_CHECK();
-      count_launch();
-      if (!c.kf->replicated) FEKF_TRY(comm_allreduce(c.comm, c.kf->ub.as<double>(), c.kf->plan.Npad, s));
-      FEKF_TRY(c.kf->update_end(c.abe.as<double>(), sqrt_bs, c.w.as<double>(), s));
-      continue;
-    }
-    FEKF_TRY(comm_allreduce(c.comm, g, c.Np + 1, s));
-    abe_kernel<<<1, 1, 0, s>>>(esum, scale, c.abe.as<double>(), k < 4 ? metrics + 1 + k : nullptr);
-    FEKF_LAUNCH_CHECK();
-    count_launch();
-    FEKF_TRY(c.kf->update(g, c.abe.as<double>(), sqrt_bs, c.w.as<double>(), s, split ? c.ev_fit : nullptr));
+    FEKF_TRY(kalman(1.0 / ((double)c.Bg * apg * 3) / c.Na, k < 4 ? metrics + 1 + k : nullptr));
   }
   c.split_armed = false;
   metrics_kernel<<<1, 1, 0, s>>>(c.kf->state.as<KfState>(), c.err_d.as<int>(), c.overflow.as<int>(), nb, metrics);

@@ -215,8 +215,8 @@ __device__ __forceinline__ void dmma884k(double& d0, double& d1, double a, doubl
                : "d"(a), "d"(b));
 }
 template <typename PT, int NSTRIP>
-__device__ __forceinline__ void apply_corrections(PT* t, const double* vI, const double* vJ, const double* s_beta,
-                                                  int K, double sig, int strip0, int lane) {
+__device__ __forceinline__ void apply_corrections(PT* t, const double (&ai)[NSTRIP][KMAX / 4], const double* vJ, int K,
+                                                  double sig, int strip0, int lane) {
   const int fr = lane >> 2, fk = lane & 3;
 #pragma unroll
   for (int sp = 0; sp < NSTRIP; ++sp) {
@@ -224,10 +224,13 @@ __device__ __forceinline__ void apply_corrections(PT* t, const double* vI, const
     double c[8][2];
 #pragma unroll
     for (int j = 0; j < 8; ++j) c[j][0] = c[j][1] = 0.0;
-    for (int k0 = 0; k0 < K; k0 += 4) {
+#pragma unroll
+    for (int ks = 0; ks < KMAX / 4; ++ks) {
+      const int k0 = 4 * ks;
+      if (k0 >= K) break;
       const int k = k0 + fk;
       const bool kv = k < K;
-      const double a = kv ? s_beta[k] * vI[k * VS + m0 + fr] : 0.0;
+      const double a = ai[sp][ks];   // beta_k u_k[row m0 + fr] of this item (registers, loaded at item start)
       double b[8];
 #pragma unroll
       for (int j = 0; j < 8; ++j) b[j] = kv ? vJ[k * VS + 8 * j + fr] : 0.0;
@@ -261,7 +264,9 @@ __device__ __forceinline__ void apply_corrections(PT* t, const double* vI, const
 // then u_B = B_new g.  Tile-row segments are pulled from an atomic counter by a producer warp that
 // streams each tile (and its g_J segment, and for rw the 2K 512-byte vector segments it needs) with TMA
 // bulk copies into a ring of `nst` stages (fp64: 6 for read-only passes, fewer when corrections ride
-// along; fp32 tiles are 16 KiB, so twice as many).  `stage_bytes` = tile bytes + (T + 2K*VS)*8.
+// along; fp32 tiles are 16 KiB, so twice as many).  `stage_bytes` = tile bytes + (T + K*VS)*8: a stage carries
+// the tile's column segments u_k[J]; the row segments u_k[I] are the same for every tile of an item and are
+// loaded once per item into the consumers' registers (round 1 staged both per tile: 4 stages, now 5).
 //
 // The 8 consumer warps form NG independent groups of 8/NG warps (named barrier 1 + group); group g
 // takes the stages s = g (mod NG), so NG tiles are in flight in the consumers at once.  fp64 uses one
@@ -303,7 +308,7 @@ kf_pass_kernel(PT* __restrict__ P, const ItemD* __restrict__ items, int n_items,
       int s = 0;
       uint32_t ph = 0;
       bool own = true;
-      const uint32_t bytes = TILE_BYTES + (1u + 2u * (uint32_t)K) * KT * sizeof(double);   // bytes landed
+      const uint32_t bytes = TILE_BYTES + (1u + (uint32_t)K) * KT * sizeof(double);   // bytes landed
       while (true) {
         // own list first, then (split pass, late launch) the early launch's unclaimed items
         int itx = -1, lst = 0;
@@ -328,10 +333,10 @@ kf_pass_kernel(PT* __restrict__ P, const ItemD* __restrict__ items, int n_items,
           tma_load_1d(st_s, P + (size_t)(it.tile_off + t) * TILE_ELEMS, TILE_BYTES, &full[s]);
           // g_J rides with its tile: no dependent global load on the consumers' per-tile path
           tma_load_1d(st_g, gpad + it.vbase + (size_t)(it.J0 + t) * KT, KT * sizeof(double), &full[s]);
-          for (int k = 0; k < K; ++k) {
+          for (int k = 0; k < K; ++k) {   // the column segments u_k[J] (the row segments u_k[I] of an item
+                                            // sit in the consumers' registers)
             const double* uk = ulist + (size_t)k * npad + it.vbase;
-            tma_load_1d(st_v + k * VS, uk + (size_t)it.I * KT, KT * sizeof(double), &full[s]);
-            tma_load_1d(st_v + (K + k) * VS, uk + (size_t)(it.J0 + t) * KT, KT * sizeof(double), &full[s]);
+            tma_load_1d(st_v + k * VS, uk + (size_t)(it.J0 + t) * KT, KT * sizeof(double), &full[s]);
           }
           if (++s == nst) { s = 0; ph ^= 1; }
         }
@@ -354,6 +359,7 @@ kf_pass_kernel(PT* __restrict__ P, const ItemD* __restrict__ items, int n_items,
   const double sig = st->sigma;
   const int c0 = 2 * lane;
   double gI[RPW], racc[RPW];
+  double ai[RPW / 8][KMAX / 4];
 #pragma unroll
   for (int k = 0; k < RPW; ++k) { gI[k] = 0.0; racc[k] = 0.0; }
   int s = gi, prev_s = -1;
@@ -373,17 +379,27 @@ kf_pass_kernel(PT* __restrict__ P, const ItemD* __restrict__ items, int n_items,
         gI[k] = __ldg(gpad + it.vbase + (long long)it.I * KT + wg + NGW * k);
         racc[k] = 0.0;
       }
+      if (rw) {   // beta_k u_k[row] of this warp's correction strips, fixed for the whole item
+        const int fr = lane >> 2, fk = lane & 3;
+#pragma unroll
+        for (int sp = 0; sp < RPW / 8; ++sp)
+#pragma unroll
+          for (int ks = 0; ks < KMAX / 4; ++ks) {
+            const int k = 4 * ks + fk;
+            const int row = 8 * (wg * (RPW / 8) + sp) + fr;
+            ai[sp][ks] = k < K ? s_beta[k] * __ldg(ulist + (size_t)k * npad + it.vbase + (long long)it.I * KT + row) : 0.0;
+          }
+      }
     }
     PT* t = reinterpret_cast<PT*>(stages + (size_t)s * stage_bytes);
     const double* vg = reinterpret_cast<const double*>(t + TILE_ELEMS);
     const double2 gJ = *reinterpret_cast<const double2*>(vg + c0);
-    const double* vI = vg + KT;
-    const double* vJ = vI + K * VS;
+    const double* vJ = vg + KT;
     double ca0 = 0.0, ca1 = 0.0;
     if (rw) {
       // B <- sigma (B - C) on the tensor path, 8-row strips per warp; then the group re-reads the
       // rewritten tile (u_B = B_new g with B_new as stored) in its own element layout
-      apply_corrections<PT, RPW / 8>(t, vI, vJ, s_beta, K, sig, wg * (RPW / 8), lane);
+      apply_corrections<PT, RPW / 8>(t, ai, vJ, K, sig, wg * (RPW / 8), lane);
       asm volatile("bar.sync %0, %1;" ::"r"(1 + gi), "r"(GT) : "memory");
     }
 #pragma unroll
@@ -822,7 +838,7 @@ fekf_status Kf::pass_launch(bool rw, int i0, int n, int* ctr, int grid, cudaStre
     FEKF_CHECK_CUDA(cudaEventRecordWithFlags(tp->a, s, capturing ? cudaEventRecordExternal : cudaEventRecordDefault));
   }
   const int K = rw ? npend : 0;
-  const int stage_bytes = (int)(TILE_ELEMS * elem() + (KT + 2 * K * VS) * sizeof(double));
+  const int stage_bytes = (int)(TILE_ELEMS * elem() + (KT + K * VS) * sizeof(double));
   int nst = (int)std::min<size_t>(MAX_STAGES, (PASS_SMEM - PASS_HDR) / stage_bytes);
   if (ng == 2) nst &= ~1;   // two consumer groups alternate stages
   const ItemD* it = items_d.as<ItemD>() + i0;

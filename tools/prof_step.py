@@ -76,9 +76,9 @@ def main():
         if short(e.name) == "kf_vec_kernel":
             ups.append(cur)
             cur = []
-    u = ups[1]
+    u = ups[int(os.environ.get("PROF_UPDATE", "1"))]
     b0 = u[0].time_range.start
-    print("\ntimeline of update 2 (force): start offset, duration (us), kernel")
+    print("\ntimeline of update %d: start offset, duration (us), kernel" % (ups.index(u) + 1))
     for e in u:
         print("%9.1f %8.1f  %s" % (e.time_range.start - b0, e.time_range.elapsed_us(), short(e.name)))
     ctx.close()
