@@ -328,6 +328,7 @@ def run_fekf(args, rank, world, local):
     barrier()
     pass_ms, pass_n, pass_rw = ctx.kf.timing(False)
     parts = ctx.kf.timing_parts()
+    span_ms = ctx.kf.timing_span()
     clk = clocks.stop()
     ms = e0.elapsed_time(e1)
     launches = ctx.last_launch_count() * args.steps
@@ -390,9 +391,13 @@ def run_fekf(args, rank, world, local):
     stream = esize / 2 * sum(n * (n + 1) for n in blocks) * info["tiles_local"] / total_tiles
     alg_total = stream * (2 * pass_rw + (pass_n - pass_rw))
     alg_bytes = alg_total / max(pass_n, 1)
-    avg_pass_s = (pass_ms / max(pass_n, 1)) / 1000.0
+    # a split pass is two overlapping launches (early on the side stream, late on the producing one); the
+    # pass's duration is its wall span (early start -> later end), the launch-duration sum double-counts
+    # the overlap and is reported beside it
+    avg_pass_s = (span_ms / max(pass_n, 1)) / 1000.0
     peak, peak_kind = load_peaks()
-    achieved = alg_total / (pass_ms / 1000.0) / 1e9 if pass_ms > 0 else None
+    achieved = alg_total / (span_ms / 1000.0) / 1e9 if span_ms > 0 else None
+    achieved_sum = alg_total / (pass_ms / 1000.0) / 1e9 if pass_ms > 0 else None
     traffic = None
     prof = os.path.join(ROOT, "profiles", "kf_pass_traffic.json")
     if os.path.exists(prof) and pass_n > 0:
@@ -456,7 +461,9 @@ def run_fekf(args, rank, world, local):
     roof = {"kernel": "kf_pass_kernel", "bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
             "frac": (achieved / peak) if achieved else None, "traffic": traffic,
             "peak_source": peak_kind, "alg_bytes_per_launch": alg_bytes, "avg_launch_ms": avg_pass_s * 1000.0,
-            "launches_timed": pass_n, "rw_launches": pass_rw, "share_of_step": (pass_ms / max(ms, 1e-9)),
+            "duration": "wall span per pass (split pass: early launch start -> later launch end), CUDA events",
+            "achieved_launch_sum": achieved_sum, "frac_launch_sum": (achieved_sum / peak) if achieved_sum else None,
+            "launches_timed": pass_n, "rw_launches": pass_rw, "share_of_step": (span_ms / max(ms, 1e-9)),
             "split_pass_early_sms": split_sms, "split_updates": "force updates (the energy update's pass is unsplit)",
             "standalone": standalone,
             "split_ms_per_pass": dict(zip(["early", "late", "early_start_to_reverse_done"],

@@ -687,6 +687,11 @@ fekf_status fekf_kf_timing_parts(const fekf_kf* k, double* ms3) {
   for (int i = 0; i < 3; ++i) ms3[i] = k->kf.t_part[i];
   return FEKF_OK;
 }
+fekf_status fekf_kf_timing_span(const fekf_kf* k, double* span_ms) {
+  if (!k || !span_ms) { set_error("kf_timing_span: null"); return FEKF_EINVAL; }
+  *span_ms = k->kf.t_span;
+  return FEKF_OK;
+}
 fekf_status fekf_kf_timing(fekf_kf* k, int mode, double* total_ms, int64_t* launches, int64_t* rw_launches) {
   if (!k || (mode != 0 && mode != 1)) { set_error("kf_timing: bad args"); return FEKF_EINVAL; }
   return k->kf.timing_ctl(mode, total_ms, launches, rw_launches);

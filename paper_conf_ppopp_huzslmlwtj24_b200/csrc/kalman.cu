@@ -761,6 +761,10 @@ fekf_status Kf::create(const std::vector<int>& blocks, const fekf_opt_cfg& o, fe
 }
 
 fekf_status Kf::harvest(std::vector<EvPair>& pairs, size_t n) {
+  // wall span of each pass: an unsplit pass's launch; a split pass from its early launch's start to the
+  // later of the two launches' ends (the pairs of one pass are recorded consecutively: early, then late)
+  long long pend = -1;
+  float pend_ms = 0.f;
   for (size_t k = 0; k < n; ++k) {
     FEKF_CHECK_CUDA(cudaEventSynchronize(pairs[k].b));
     float ms = 0.f;
@@ -771,8 +775,17 @@ fekf_status Kf::harvest(std::vector<EvPair>& pairs, size_t n) {
     if (!pairs[k].part) {
       t_n += 1;
       t_rw += pairs[k].rw;
+      if (pend >= 0) t_span += pend_ms;
+      pend = (long long)k;
+      pend_ms = ms;
+    } else if (pend >= 0) {
+      float to_late = 0.f;
+      FEKF_CHECK_CUDA(cudaEventElapsedTime(&to_late, pairs[pend].a, pairs[k].b));
+      t_span += std::max(pend_ms, to_late);
+      pend = -1;
     }
   }
+  if (pend >= 0) t_span += pend_ms;
   return FEKF_OK;
 }
 
@@ -791,6 +804,7 @@ fekf_status Kf::timing_ctl(int mode, double* total_ms, int64_t* launches, int64_
     pend_graphs.clear();
     t_ms = 0.0;
     t_part[0] = t_part[1] = t_part[2] = 0.0;
+    t_span = 0.0;
     t_n = t_rw = 0;
     return FEKF_OK;
   }

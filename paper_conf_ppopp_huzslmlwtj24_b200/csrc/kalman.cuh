@@ -92,6 +92,7 @@ struct Kf {
   std::vector<EvPair>* rec = nullptr;   // non-null while capturing with timing on
   double t_ms = 0.0;
   double t_part[3] = {0.0, 0.0, 0.0};   // split passes: early launch, late launch, early start -> tail done
+  double t_span = 0.0;                  // summed wall span of the timed passes (split: early start -> last end)
   int64_t t_n = 0, t_rw = 0;
   long long rw_passes = 0, r_passes = 0;
   fekf_status timing_ctl(int mode, double* total_ms, int64_t* launches, int64_t* rw_launches);

@@ -90,6 +90,7 @@ def lib():
         "fekf_naive_train_step": ([vp, vp, vp, vp, vp, vp, vp, vp], i32),
         "fekf_set_env_stats": ([vp, vp, vp], i32),
         "fekf_comm_init_loopback": ([i32, vp], i32),
+        "fekf_kf_timing_span": ([vp, C.POINTER(dbl)], i32),
     }
     for name, (args, res) in sigs.items():
         f = getattr(L, name)
@@ -109,7 +110,7 @@ EXPORTED = [
     "fekf_energy_jacobian", "fekf_force_jacobian", "fekf_kalman_update", "fekf_train_step",
     "fekf_last_launch_count", "fekf_set_graph_mode", "fekf_kf_update_naive", "fekf_naive_train_step",
     "fekf_kf_timing_parts", "fekf_kf_update_naive_begin", "fekf_kf_naive_partial_u", "fekf_kf_update_naive_end",
-    "fekf_set_env_stats", "fekf_comm_init_loopback",
+    "fekf_set_env_stats", "fekf_comm_init_loopback", "fekf_kf_timing_span",
 ]
 
 
@@ -347,6 +348,12 @@ class KalmanFilter:
     def update_end(self, abe, sqrt_bs, w, stream=None):
         _check(lib().fekf_kf_update_end(self.h, _ptr(abe, torch.float64, "abe"), float(sqrt_bs),
                                         _ptr(w, torch.float64, "w"), _stream(stream)))
+
+    def timing_span(self):
+        """Summed wall ms of the passes of the last timing window (split passes: early start -> last end)."""
+        v = C.c_double()
+        _check(lib().fekf_kf_timing_span(self.h, C.byref(v)))
+        return v.value
 
     def timing_parts(self):
         """[early, late, early start -> reverse pass done] summed ms of the last timing window (split pass)."""
