@@ -737,6 +737,11 @@ fekf_status Kf::create(const std::vector<int>& blocks, const fekf_opt_cfg& o, fe
   s.c_mult = o.noise_mode == 0 ? (double)p.L : 1.0;
   FEKF_CHECK_CUDA(cudaMemcpy(state.p, &s, sizeof(KfState), cudaMemcpyHostToDevice));
   FEKF_CHECK_CUDA(cudaMemset(ulist.p, 0, (size_t)KMAX * p.Npad * sizeof(double)));
+  // the work counters are zeroed before every launch (stream-ordered memset, a graph node when captured);
+  // zeroing them once here too keeps compute-sanitizer's initcheck, which does not see graph memset nodes,
+  // free of false reports
+  FEKF_CHECK_CUDA(cudaMemset(counter.p, 0, sizeof(int)));
+  FEKF_CHECK_CUDA(cudaMemset(counter2.p, 0, sizeof(int)));
   FEKF_CHECK_CUDA(cudaFuncSetAttribute(kf_pass_kernel<double, 1>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)PASS_SMEM));
   FEKF_CHECK_CUDA(cudaFuncSetAttribute(kf_pass_kernel<float, 2>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)PASS_SMEM));
   FEKF_CHECK_CUDA(cudaFuncSetAttribute(kf_pass_kernel<double, 2>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)PASS_SMEM));

@@ -442,3 +442,41 @@ def test_large_batch_preset_train_steps():
     na = len(ds["types"])
     w0 = init_weights(m, 3, float(ds["energy"].mean() / na))
     _train_compare(m, opt, ds, w0, B=B, steps=2, tol=1e-9)
+
+
+# ------------------------------------------------------------------------------------------
+# fault handling: a non-finite update is dropped (flag latched, optimizer state kept)
+# ------------------------------------------------------------------------------------------
+def test_nonfinite_update_is_skipped():
+    """A NaN energy label makes the energy update's ABE non-finite: that update is a no-op (w, P and lambda
+    keep their values) with bit 1 of the fault flags set, and the step's 4 force updates proceed, so the
+    weights equal those of a step whose energy update was skipped (lambda advanced 4 times, not 5)."""
+    wl = get_config("t2_tiny")
+    m, opt = wl.model, OptConfig(p_defer=2)
+    B = wl.batch
+    ds = make_dataset("t2_tiny", B)
+    na = len(ds["types"])
+    w0 = init_weights(m, 3, float(ds["energy"].mean() / na))
+    groups = force_groups(na, 0, 17, opt.force_groups, opt.atoms_per_group)
+    e_bad = ds["energy"].copy()
+    e_bad[1] = np.nan
+    ctx = fk.Context(m, opt, types=ds["types"], local_batch=B, global_batch=B)
+    ctx.set_params(cu(w0))
+    met = ctx.train_step(cu(ds["coord"]), cu(ds["box"]), cu(e_bad), cu(ds["force"]), cu(groups, torch.int32))
+    mt = met.cpu().numpy()
+    assert int(mt[7]) & 2
+    lam = 1.0 - (1.0 - opt.lambda0) * opt.nu ** 4
+    assert abs(mt[6] - lam) < 1e-14
+    # reference: the oracle's step without its energy update (the 4 force updates from the same w, P = I)
+    st = O.FEKF.create(w0, m, opt)
+    nl = O.build_nlist(ds["coord"], ds["box"], ds["types"], m.rcut, m.sel)
+    for atoms in groups:
+        g, s, _ = O.force_grad(st.w, ds["coord"], ds["box"], ds["types"], nl[0], nl[1], ds["force"], atoms, m)
+        st.update(g, s / (B * len(atoms) * 3) / na, B)
+    wg = ctx.get_params().cpu().numpy()
+    assert np.all(np.isfinite(wg))
+    assert rel(wg, st.w) < 1e-9
+    for b in range(len(st.blocks)):
+        Pb = ctx.kf.get_block(b).cpu().numpy()
+        assert np.all(np.isfinite(Pb)) and rel(Pb, st.P[b]) < 1e-9
+    ctx.close()
