@@ -223,6 +223,11 @@ fekf_status Ctx::init(const fekf_model_cfg& mm, const fekf_opt_cfg& oo, int nato
   FEKF_TRY(dalloc(rij, sizeof(double) * nslots * 3));
   FEKF_TRY(dalloc(rdot, sizeof(double) * nslots * 4));
   FEKF_TRY(dalloc(vdir, sizeof(double) * B * Na * 3));
+  FEKF_TRY(dalloc(frow, sizeof(double) * nslots * 3));
+  FEKF_TRY(dalloc(rev_cnt, sizeof(int) * (size_t)B * Na * Na));
+  FEKF_TRY(dalloc(rev_off, sizeof(int) * ((size_t)B * Na + 1)));
+  FEKF_TRY(dalloc(rev_idx, sizeof(int) * nslots));
+  FEKF_CHECK_CUDA(cudaMemset(frow.p, 0, sizeof(double) * nslots * 3));
   FEKF_TRY(dalloc(X, sizeof(double) * 2 * B * Na * 4 * M));
   FEKF_TRY(dalloc(Xb, sizeof(double) * 2 * B * Na * 4 * M));
   FEKF_TRY(dalloc(eatom, sizeof(double) * B * Na));
@@ -352,7 +357,7 @@ Ctx::~Ctx() {
   kfo.reset();
   kf = nullptr;
   for (DBuf* b : {&types_d, &tindex_d, &atoms_d, &atoms_off_d, &sel_d, &sec_d, &err_d, &env_stats, &w, &gbuf, &nl_j, &nl_s,
-                  &overflow, &em, &jac, &rij, &rdot, &vdir, &X, &Xb, &eatom, &etot, &force, &virial, &vatom, &splitk_ws,
+                  &overflow, &em, &jac, &rij, &rdot, &vdir, &frow, &rev_cnt, &rev_off, &rev_idx, &X, &Xb, &eatom, &etot, &force, &virial, &vatom, &splitk_ws,
                   &colsum_ws, &abe, &metrics_tmp, &abs_sum, &rowcnt, &chunks})
     dfree(*b);
   for (auto& P : pairs) {
@@ -385,6 +390,7 @@ static fekf_status geometry(Ctx& c, const double* coord, const double* box, int 
   FEKF_TRY(launch_envmat(c, coord, box, c.nl_j.as<int>(), c.nl_s.as<int>(), nb, c.em.as<double>(), c.jac.as<double>(),
                          c.rij.as<double>(), s));
   FEKF_TRY(build_rows(c, nb, s));
+  FEKF_TRY(build_reverse(c, nb, s));
   return FEKF_OK;
 }
 

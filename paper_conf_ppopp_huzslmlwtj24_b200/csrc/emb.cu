@@ -349,7 +349,6 @@ struct EmbBwdIO {
   const int* tidx;                    // tangent rows: tangent row -> primal row (nullptr: primal rows)
   const int* tpos;                    // primal rows, dual: primal row -> tangent row or -1 (nullptr: none)
   const int* rmap;                    // MODE_FORCE_SEL: row -> primal row (active rows only; nullptr: all)
-  int Nm;
   const double* Gbar;                 // primal rows: Gbar (desc_bwd_seed_kernel)
   const double* dR;                   // forces: per-row R~ adjoint less sbar e_0 [R][4]
   const double* hin;                  // s / s-dot per row
@@ -359,14 +358,9 @@ struct EmbBwdIO {
   double* Hbt[FEKF_MAX_LAYERS];       // hdotbar_l: written by tangent rows, read by dual primal rows
   double* sbar;                       // forces: s-bar per primal row
   double* ws;                         // weight-gradient partials [gridDim.x][GS] (nullptr: none)
-  // forces (prod_force fused, MODE_FORCE): dE/dR~_row = dR + sbar e_0 ; f = (dE/dR~) J ;
-  // F_i += f, F_j -= f (F = -dE/dx) ; W_i -= d (x) f
+  // forces (MODE_FORCE / MODE_FORCE_SEL): dE/dR~_row = dR + sbar e_0 ; f = dE/dd = (dE/dR~) J per slot
   const double* jac;
-  const double* rij;
-  const int* nl_j;
-  int Na;
-  double* force;
-  double* vatom;
+  double* frow;
 };
 
 // weight-gradient blocks of layer L: [Wbar_L ; bbar_L] += [h_{L-1} | 1]^T zbar_L over the tile's rows
@@ -425,20 +419,11 @@ __device__ __forceinline__ void write_partials(const double (&acc)[W::MAXB][2][2
   }
 }
 
-// a [T][12] scratch area for the force epilogue: the adjoint buffer the layer-0 step does not use
-template <class W>
-__device__ __forceinline__ double* hn_scratch(double* sm) {
-  constexpr int step = W::NL - 1;
-  constexpr int bx = (3 - step % 3) % 3, bn = (bx + 2) % 3;
-  static_assert(W::BLD >= 12, "scratch");
-  return sm + W::bBuf(bn);
-}
-
 // One layer L of the reverse chain on the current tile (buffers rotate with the step from the top).
 template <class W, int L>
 __device__ __forceinline__ void bwd_layer(double (&acc)[W::MAXB][2][2][2], double* sm, const EmbBwdIO& io, int r0, int R,
                                           bool tan, bool wantw, const int* s_slot, const int* s_prow,
-                                          const int* s_tpos, const int* s_atom, const double* s_dr) {
+                                          const int* s_tpos, const double* s_dr) {
   constexpr int T = W::T, NW = EMB_BWD_WARPS, RPW = T / NW, BLD = W::BLD;
   constexpr int step = W::NL - 1 - L;
   constexpr int bx = (3 - step % 3) % 3, bz = (bx + 1) % 3, bn = (bx + 2) % 3;
@@ -504,8 +489,8 @@ __device__ __forceinline__ void bwd_layer(double (&acc)[W::MAXB][2][2][2], doubl
     });
     __syncthreads();
   } else if (io.sbar) {
-    // sbar = zbar_0 . W_0 (4 threads per row), then the row's dE/dd and the force / virial scatter
-    double* sf = hn_scratch<W>(sm);  // [T][12]: f (3) | -d (x) f (9), in a buffer the chain is done with
+    // sbar = zbar_0 . W_0 (4 threads per row), then the row's dE/dd = (dR + sbar e_0) J, stored per slot;
+    // the forces and virials are gathered from these in a fixed order (force_gather_kernel, nets.cu)
     const int t = threadIdx.x;
     if (t < T * 4) {
       const int r = t >> 2, part = t & 3;
@@ -518,38 +503,11 @@ __device__ __forceinline__ void bwd_layer(double (&acc)[W::MAXB][2][2][2], doubl
       sb += __shfl_xor_sync(0xffffffffu, sb, 2);
       const int row = r0 + r;
       if (part == 0 && row < R) io.sbar[s_prow[r]] = sb;
-      if (io.dR && part < 3) {
+      if (io.dR && part < 3 && row < R) {
         const int be = part, slot = s_slot[r];
-        double f = 0.0;
-        if (row < R) {
-          const double* J = io.jac + (size_t)slot * 12;
-          f = (s_dr[r * 4] + sb) * J[be] + s_dr[r * 4 + 1] * J[3 + be] + s_dr[r * 4 + 2] * J[6 + be] +
-              s_dr[r * 4 + 3] * J[9 + be];
-          const int atom = s_atom[r], j = io.nl_j[slot];
-          atomicAdd(io.force + ((size_t)(atom / io.Na) * io.Na + j) * 3 + be, -f);
-        }
-        sf[r * 12 + be] = f;
-      }
-    }
-    if (io.dR) {
-      __syncthreads();
-      if (t < T * 9) {
-        const int r = t / 9, q = t % 9, a = q / 3, be = q % 3;
-        double v = 0.0;
-        if (r0 + r < R) v = -io.rij[(size_t)s_slot[r] * 3 + a] * sf[r * 12 + be];
-        sf[r * 12 + 3 + q] = v;
-      }
-      __syncthreads();
-      // rows of one centre atom are consecutive: one atomic per (segment, component)
-      if (t < T * 12) {
-        const int r = t / 12, q = t % 12;
-        const int atom = s_atom[r];
-        if (r0 + r < R && (r == 0 || s_atom[r - 1] != atom)) {
-          double sum = 0.0;
-          for (int k = r; k < T && r0 + k < R && s_atom[k] == atom; ++k) sum += sf[k * 12 + q];
-          if (q < 3) atomicAdd(io.force + (size_t)atom * 3 + q, sum);
-          else atomicAdd(io.vatom + (size_t)atom * 9 + q - 3, sum);
-        }
+        const double* J = io.jac + (size_t)slot * 12;
+        io.frow[(size_t)slot * 3 + be] = (s_dr[r * 4] + sb) * J[be] + s_dr[r * 4 + 1] * J[3 + be] +
+                                         s_dr[r * 4 + 2] * J[6 + be] + s_dr[r * 4 + 3] * J[9 + be];
       }
     }
   }
@@ -658,7 +616,7 @@ template <class W>
 __global__ void __launch_bounds__(EMB_BWD_WARPS * 32, 1) emb_bwd_kernel(const double* __restrict__ wp, EmbBwdIO io) {
   extern __shared__ __align__(16) double sm[];
   constexpr int T = W::T, NW = EMB_BWD_WARPS, NL = W::NL, RPW = T / NW;
-  __shared__ int s_slot[T], s_atom[T], s_prow[T], s_tpos[T];
+  __shared__ int s_slot[T], s_prow[T], s_tpos[T];
   __shared__ double s_dr[T * 4];
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   const bool tan = io.tidx != nullptr;
@@ -688,15 +646,13 @@ __global__ void __launch_bounds__(EMB_BWD_WARPS * 32, 1) emb_bwd_kernel(const do
     __syncthreads();
     if (tid < T) {
       const int row = r0 + tid;
-      int slot = -1, atom = 0, pr = 0, tp = -1;
+      int slot = -1, pr = 0, tp = -1;
       if (row < R) {
         pr = tan ? io.tidx[row] : (io.rmap ? io.rmap[row] : row);
         slot = io.row_idx[pr];
-        atom = slot / io.Nm;
         if (io.tpos) tp = io.tpos[row];
       }
       s_slot[tid] = slot;
-      s_atom[tid] = atom;
       s_prow[tid] = pr;
       s_tpos[tid] = tp;
     }
@@ -725,10 +681,10 @@ __global__ void __launch_bounds__(EMB_BWD_WARPS * 32, 1) emb_bwd_kernel(const do
     // ---- seed: hbar_{L-1} = Gbar, zbar_{L-1} (and, for forces, the per-row R~ adjoint)
     seed_rows<W>(sm, io, r0, R, tan, s_dr, s_prow, s_tpos);
     __syncthreads();
-    if constexpr (NL >= 4) bwd_layer<W, 3>(acc, sm, io, r0, R, tan, wantw, s_slot, s_prow, s_tpos, s_atom, s_dr);
-    if constexpr (NL >= 3) bwd_layer<W, 2>(acc, sm, io, r0, R, tan, wantw, s_slot, s_prow, s_tpos, s_atom, s_dr);
-    if constexpr (NL >= 2) bwd_layer<W, 1>(acc, sm, io, r0, R, tan, wantw, s_slot, s_prow, s_tpos, s_atom, s_dr);
-    bwd_layer<W, 0>(acc, sm, io, r0, R, tan, wantw, s_slot, s_prow, s_tpos, s_atom, s_dr);
+    if constexpr (NL >= 4) bwd_layer<W, 3>(acc, sm, io, r0, R, tan, wantw, s_slot, s_prow, s_tpos, s_dr);
+    if constexpr (NL >= 3) bwd_layer<W, 2>(acc, sm, io, r0, R, tan, wantw, s_slot, s_prow, s_tpos, s_dr);
+    if constexpr (NL >= 2) bwd_layer<W, 1>(acc, sm, io, r0, R, tan, wantw, s_slot, s_prow, s_tpos, s_dr);
+    bwd_layer<W, 0>(acc, sm, io, r0, R, tan, wantw, s_slot, s_prow, s_tpos, s_dr);
   }
   if (wantw) {
     double* out = io.ws + (size_t)blockIdx.x * W::GS;
@@ -776,7 +732,6 @@ static fekf_status emb_backward_t(Ctx& c, int p, long long Rmax, int mode, doubl
   EmbBwdIO io{};
   io.Rmax = (int)Rmax;
   io.row_idx = P.row_idx.as<int>();
-  io.Nm = c.Nm;
   io.Gbar = P.Hb[W::NL - 1].template as<double>();
   for (int l = 0; l < W::NL; ++l) {
     io.Yp[l] = P.Y[l].as<double>();
@@ -807,11 +762,7 @@ static fekf_status emb_backward_t(Ctx& c, int p, long long Rmax, int mode, doubl
   if (mode == MODE_FORCE || sel) {
     io.dR = P.Zb[0].template as<double>();
     io.jac = c.jac.as<double>();
-    io.rij = c.rij.as<double>();
-    io.nl_j = c.nl_j.as<int>();
-    io.Na = c.Na;
-    io.force = c.force.as<double>();
-    io.vatom = c.vatom.as<double>();
+    io.frow = c.frow.as<double>();
   }
   io.ws = wantw ? ws + (size_t)nsets * W::GS : nullptr;
   int gp = 0;

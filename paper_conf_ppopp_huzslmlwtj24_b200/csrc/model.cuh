@@ -68,6 +68,12 @@ struct Ctx {
   DBuf env_stats;                                 // [2][nt][4]: avg | std of the R~ rows (reading Z11)
   DBuf w, gbuf;                                   // [Np], [Np + 1] (g || error sum, the allreduce payload)
   DBuf nl_j, nl_s, overflow, em, jac, rij, rdot, vdir;
+  // atomics-free force scatter (reverse neighbour map, built once per geometry): frow [slot][3] = dE/dd of
+  // every valid slot, rev_off [B*Na + 1] / rev_idx [slots] = for every atom j the slots whose neighbour is
+  // j, in slot order; rev_cnt [B][Na][Na] scratch of the deterministic fill
+  DBuf frow, rev_cnt, rev_off, rev_idx;
+  const int* sel_atoms = nullptr;                 // MODE_FORCE_SEL: the force group's atoms (mark_selected)
+  int n_sel_atoms = 0;
   DBuf X, Xb;                                     // [2 * B*Na*4*M] (primal | tangent)
   DBuf eatom, etot, force, virial, vatom;
   DBuf splitk_ws, colsum_ws;
@@ -120,6 +126,7 @@ fekf_status force_error(Ctx& c, int nb, const double* f_label, const int* atom_i
                         cudaStream_t s);
 fekf_status tangent_env(Ctx& c, int nb, cudaStream_t s);
 fekf_status build_rows(Ctx& c, int nb, cudaStream_t s);
+fekf_status build_reverse(Ctx& c, int nb, cudaStream_t s);
 fekf_status seed_force(Ctx& c, int nb, cudaStream_t s);
 
 }  // namespace fekf

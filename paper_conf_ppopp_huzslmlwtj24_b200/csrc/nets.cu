@@ -832,14 +832,11 @@ emb_seed_atom_kernel(Geo g, PairPtrs pp, SeedPtrs sp, const double* __restrict__
   }
 }
 
-// prod_force / prod_virial: dE/dR~_row = G Xbar^T / N_m + sbar e_0 ; f = dE/dd = (dE/dR~) J ;
-// F_i += f, F_j -= f (F = -dE/dx), W -= d (x) f.  One CTA (4 warps) per centre atom: the
-// atom's own force and virial are reduced in the CTA (fixed order), only F_j needs atomics.
+// prod_force (per-layer embedding path): dE/dR~_row = G Xbar^T / N_m + sbar e_0 ; f = dE/dd = (dE/dR~) J per
+// slot into frow (the forces / virials are gathered by force_gather_kernel).  One CTA (4 warps) per atom.
 __global__ void __launch_bounds__(128)
 prod_force_kernel(Geo g, PairPtrs pp, const double* __restrict__ Xb, const double* __restrict__ jac,
-                  const double* __restrict__ rij, const int* __restrict__ nl_j, double* __restrict__ force,
-                  double* __restrict__ vatom) {
-  __shared__ double red[4][12];
+                  const int* __restrict__ nl_j, double* __restrict__ frow) {
   const int atom = blockIdx.x;
   const int b = atom / g.Na, i = atom % g.Na;
   const int ti = g.types[i], k = g.tindex[i];
@@ -848,11 +845,9 @@ prod_force_kernel(Geo g, PairPtrs pp, const double* __restrict__ Xb, const doubl
   const int M = g.M;
   const double* xb = Xb + (size_t)atom * 4 * M;
   const double inv = 1.0 / g.Nm;
-  double fi[3] = {0, 0, 0}, vir[9] = {0, 0, 0, 0, 0, 0, 0, 0, 0};
   for (int slot = warp; slot < g.Nm; slot += 4) {
     const size_t idx = (size_t)atom * g.Nm + slot;
-    const int j = nl_j[idx];
-    if (j < 0) continue;
+    if (nl_j[idx] < 0) continue;
     int tj = 0;
     while (slot >= g.sec[tj + 1]) ++tj;
     const int p = ti * g.nt + tj;
@@ -869,38 +864,168 @@ prod_force_kernel(Geo g, PairPtrs pp, const double* __restrict__ Xb, const doubl
       a2 += __shfl_xor_sync(0xffffffffu, a2, o);
       a3 += __shfl_xor_sync(0xffffffffu, a3, o);
     }
-    if (lane == 0) {
-      const double rb[4] = {a0 * inv + pp.sbar[p][r], a1 * inv, a2 * inv, a3 * inv};
+    if (lane < 3) {
+      const double rb0 = a0 * inv + pp.sbar[p][r], rb1 = a1 * inv, rb2 = a2 * inv, rb3 = a3 * inv;
       const double* J = jac + idx * 12;
-      const double* d = rij + idx * 3;
-      double f[3];
-#pragma unroll
-      for (int be = 0; be < 3; ++be) f[be] = rb[0] * J[be] + rb[1] * J[3 + be] + rb[2] * J[6 + be] + rb[3] * J[9 + be];
-      double* Fj = force + ((size_t)b * g.Na + j) * 3;
-#pragma unroll
-      for (int be = 0; be < 3; ++be) {
-        fi[be] += f[be];
-        atomicAdd(Fj + be, -f[be]);
-      }
-#pragma unroll
-      for (int a = 0; a < 3; ++a)
-#pragma unroll
-        for (int be = 0; be < 3; ++be) vir[3 * a + be] -= d[a] * f[be];
+      frow[idx * 3 + lane] = rb0 * J[lane] + rb1 * J[3 + lane] + rb2 * J[6 + lane] + rb3 * J[9 + lane];
     }
   }
-  if (lane == 0) {
-#pragma unroll
-    for (int q = 0; q < 3; ++q) red[warp][q] = fi[q];
-#pragma unroll
-    for (int q = 0; q < 9; ++q) red[warp][3 + q] = vir[q];
-  }
-  __syncthreads();
-  if (threadIdx.x < 12) {
-    const double v = red[0][threadIdx.x] + red[1][threadIdx.x] + red[2][threadIdx.x] + red[3][threadIdx.x];
-    if (threadIdx.x < 3) atomicAdd(force + (size_t)atom * 3 + threadIdx.x, v);
-    else vatom[(size_t)atom * 9 + threadIdx.x - 3] = v;
+}
+
+// ---------------------------------------------------------------------------------------------
+// Atomics-free force / virial scatter.  Per slot (atom i, neighbour j, d = x_j + S - x_i) the reverse pass
+// stores f = dE/dd; F = -dE/dx gives F_i += f and F_j -= f, W_i -= d (x) f.  The reverse
+// neighbour map lists, for every atom j of an image, the slots whose neighbour is j in slot order, so every
+// force is a fixed-order sum (bit-reproducible run to run, graph or eager).
+// ---------------------------------------------------------------------------------------------
+// rev_cnt[b][i][j] = number of slots of atom i with neighbour j (order-free integer counts)
+__global__ void __launch_bounds__(256) rev_count_kernel(int nb, int Na, int Nm, const int* __restrict__ nl_j,
+                                                        int* __restrict__ cnt) {
+  const int a = blockIdx.x * 8 + (threadIdx.x >> 5), lane = threadIdx.x & 31;
+  if (a >= nb * Na) return;
+  int* row = cnt + (size_t)a * Na;
+  for (int s0 = lane; s0 < Nm; s0 += 32) {
+    const int j = nl_j[(size_t)a * Nm + s0];
+    if (j >= 0) atomicAdd(row + j, 1);
   }
 }
+// per (image, j): exclusive prefix over the centre atoms i in place (cnt -> first position of atom i's
+// entries inside bucket j) and the bucket size
+__global__ void rev_prefix_kernel(int nb, int Na, int* __restrict__ cnt, int* __restrict__ tot) {
+  const int q = blockIdx.x * blockDim.x + threadIdx.x;
+  if (q >= nb * Na) return;
+  const int b = q / Na, j = q % Na;
+  int run = 0;
+  for (int i = 0; i < Na; ++i) {
+    int* c = cnt + ((size_t)b * Na + i) * Na + j;
+    const int v = *c;
+    *c = run;
+    run += v;
+  }
+  tot[q] = run;
+}
+// exclusive scan of the bucket sizes (one CTA, fixed order) -> rev_off[0 .. nb*Na]
+__global__ void __launch_bounds__(1024) rev_scan_kernel(int n, int* __restrict__ off) {
+  __shared__ int wsum[32];
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int per = (n + 1023) / 1024;
+  const int a0 = min(n, (int)threadIdx.x * per), a1 = min(n, a0 + per);
+  int local = 0;
+  for (int e = a0; e < a1; ++e) local += off[e];
+  int x = local;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const int y = __shfl_up_sync(0xffffffffu, x, o);
+    if (lane >= o) x += y;
+  }
+  if (lane == 31) wsum[warp] = x;
+  __syncthreads();
+  if (warp == 0) {
+    int w = wsum[lane];
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const int y = __shfl_up_sync(0xffffffffu, w, o);
+      if (lane >= o) w += y;
+    }
+    wsum[lane] = w;
+  }
+  __syncthreads();
+  int run = x - local + (warp > 0 ? wsum[warp - 1] : 0);
+  for (int e = a0; e < a1; ++e) {
+    const int c = off[e];
+    off[e] = run;
+    run += c;
+  }
+  if (threadIdx.x == 1023) off[n] = wsum[31];
+}
+// fill: one warp per centre atom walks its slots in order; lanes with the same neighbour j inside a chunk
+// are ranked by lane (match_any), and the atom's own cursor row of rev_cnt (touched by this warp only)
+// carries the count across chunks -> every bucket in (i, slot) order, deterministic
+__global__ void __launch_bounds__(256) rev_fill_kernel(int nb, int Na, int Nm, const int* __restrict__ nl_j,
+                                                       int* __restrict__ cnt, const int* __restrict__ off,
+                                                       int* __restrict__ idx) {
+  const int a = blockIdx.x * 8 + (threadIdx.x >> 5), lane = threadIdx.x & 31;
+  if (a >= nb * Na) return;
+  const int b = a / Na;
+  int* cur = cnt + (size_t)a * Na;
+  for (int s0 = 0; s0 < Nm; s0 += 32) {
+    const int sl = s0 + lane;
+    const int j = sl < Nm ? nl_j[(size_t)a * Nm + sl] : -1;
+    const unsigned grp = __match_any_sync(0xffffffffu, j);
+    const int rk = __popc(grp & ((1u << lane) - 1u));
+    int base = 0;
+    if (j >= 0) base = off[(size_t)b * Na + j] + cur[j];
+    __syncwarp();
+    if (j >= 0) {
+      idx[base + rk] = (int)((size_t)a * Nm + sl);
+      if (rk == 0) cur[j] += __popc(grp);
+    }
+    __syncwarp();
+  }
+}
+
+fekf_status build_reverse(Ctx& c, int nb, cudaStream_t s) {
+  const int na = c.Na, n = nb * na;
+  int* cnt = c.rev_cnt.as<int>();
+  int* off = c.rev_off.as<int>();
+  FEKF_CHECK_CUDA(cudaMemsetAsync(cnt, 0, sizeof(int) * (size_t)n * na, s));
+  rev_count_kernel<<<cdiv(n, 8), 256, 0, s>>>(nb, na, c.Nm, c.nl_j.as<int>(), cnt);
+  FEKF_LAUNCH_CHECK();
+  rev_prefix_kernel<<<cdiv(n, 128), 128, 0, s>>>(nb, na, cnt, off);
+  FEKF_LAUNCH_CHECK();
+  rev_scan_kernel<<<1, 1024, 0, s>>>(n, off);
+  FEKF_LAUNCH_CHECK();
+  rev_fill_kernel<<<cdiv(n, 8), 256, 0, s>>>(nb, na, c.Nm, c.nl_j.as<int>(), cnt, off, c.rev_idx.as<int>());
+  FEKF_LAUNCH_CHECK();
+  count_launch(4);
+  return FEKF_OK;
+}
+
+// F_i = sum_{own slots} f - sum_{slots with neighbour i} f ;  W_i = - sum_{own slots} d (x) f.
+// One warp per atom (all atoms, or the listed ones of every image); lane-strided sums combined by a fixed
+// butterfly: deterministic.
+__global__ void __launch_bounds__(256) force_gather_kernel(int nb, int Na, int Nm, const int* __restrict__ sel,
+                                                           int n_sel, const int* __restrict__ nl_j,
+                                                           const double* __restrict__ rij,
+                                                           const double* __restrict__ frow,
+                                                           const int* __restrict__ off, const int* __restrict__ idx,
+                                                           double* __restrict__ force, double* __restrict__ vatom) {
+  const int w = blockIdx.x * 8 + (threadIdx.x >> 5), lane = threadIdx.x & 31;
+  const int nw = sel ? nb * n_sel : nb * Na;
+  if (w >= nw) return;
+  const int a = sel ? (w / n_sel) * Na + sel[w % n_sel] : w;
+  double v[12];
+#pragma unroll
+  for (int q = 0; q < 12; ++q) v[q] = 0.0;
+  for (int sl = lane; sl < Nm; sl += 32) {
+    const size_t e = (size_t)a * Nm + sl;
+    if (nl_j[e] < 0) continue;
+    const double f0 = frow[e * 3], f1 = frow[e * 3 + 1], f2 = frow[e * 3 + 2];
+    const double d0 = rij[e * 3], d1 = rij[e * 3 + 1], d2 = rij[e * 3 + 2];
+    v[0] += f0; v[1] += f1; v[2] += f2;
+    v[3] -= d0 * f0; v[4] -= d0 * f1; v[5] -= d0 * f2;
+    v[6] -= d1 * f0; v[7] -= d1 * f1; v[8] -= d1 * f2;
+    v[9] -= d2 * f0; v[10] -= d2 * f1; v[11] -= d2 * f2;
+  }
+  for (int q = off[a] + lane; q < off[a + 1]; q += 32) {
+    const size_t e = (size_t)idx[q];
+    v[0] -= frow[e * 3];
+    v[1] -= frow[e * 3 + 1];
+    v[2] -= frow[e * 3 + 2];
+  }
+#pragma unroll
+  for (int q = 0; q < 12; ++q)
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) v[q] += __shfl_xor_sync(0xffffffffu, v[q], o);
+  if (lane < 3) force[(size_t)a * 3 + lane] = lane == 0 ? v[0] : (lane == 1 ? v[1] : v[2]);
+  else if (lane < 12) {
+    double x = 0.0;
+#pragma unroll
+    for (int q = 3; q < 12; ++q) if (lane == q) x = v[q];
+    vatom[(size_t)a * 9 + lane - 3] = x;
+  }
+}
+
 // per-image virial = sum of the atoms' contributions in atom order (deterministic)
 __global__ void virial_reduce_kernel(const double* __restrict__ vatom, int Na, double* __restrict__ virial) {
   const int b = blockIdx.x, q = threadIdx.x;
@@ -1197,6 +1322,8 @@ __global__ void mark_sel_kernel(int nb, int Na, const int* __restrict__ atom_idx
 }
 
 fekf_status mark_selected(Ctx& c, int nb, const int* atom_idx, int n_sel, cudaStream_t s) {
+  c.sel_atoms = atom_idx;
+  c.n_sel_atoms = n_sel;
   mark_sel_kernel<<<1, 1024, 0, s>>>(nb, c.Na, atom_idx, n_sel, c.vdir.as<double>());
   FEKF_LAUNCH_CHECK();
   count_launch();
@@ -1470,10 +1597,6 @@ fekf_status model_backward(Ctx& c, int nb, Mode mode, double* gout, cudaStream_t
   count_launch();
   // ---- embedding nets (compacted rows; tangent rows separately) ----
   if (emb_fused_ok(c)) {
-    if (force) {  // forces / per-atom virials accumulate inside the fused backward
-      FEKF_CHECK_CUDA(cudaMemsetAsync(c.force.p, 0, sizeof(double) * nb * c.Na * 3, s));
-      FEKF_CHECK_CUDA(cudaMemsetAsync(c.vatom.p, 0, sizeof(double) * nb * c.Na * 9, s));
-    }
     for (size_t p = 0; p < c.pairs.size(); ++p) {
       const long long Rmax = pair_rows(c, (int)p, nb);
       if (Rmax == 0) continue;
@@ -1534,12 +1657,20 @@ fekf_status model_backward(Ctx& c, int nb, Mode mode, double* gout, cudaStream_t
   }
   if (force) {
     if (!emb_fused_ok(c)) {
-      FEKF_CHECK_CUDA(cudaMemsetAsync(c.force.p, 0, sizeof(double) * nb * c.Na * 3, s));
-      prod_force_kernel<<<nb * c.Na, 128, 0, s>>>(g, pp, c.Xb.as<double>(), c.jac.as<double>(), c.rij.as<double>(),
-                                                  c.nl_j.as<int>(), c.force.as<double>(), c.vatom.as<double>());
+      prod_force_kernel<<<nb * c.Na, 128, 0, s>>>(g, pp, c.Xb.as<double>(), c.jac.as<double>(), c.nl_j.as<int>(),
+                                                  c.frow.as<double>());
       FEKF_LAUNCH_CHECK();
       count_launch();
     }
+    // MODE_FORCE_SEL: only the selected atoms' forces are formed (their slots are exactly the active rows)
+    const bool sel = mode == MODE_FORCE_SEL && c.sel_atoms;
+    const int nw = sel ? nb * c.n_sel_atoms : nb * c.Na;
+    force_gather_kernel<<<cdiv(nw, 8), 256, 0, s>>>(nb, c.Na, c.Nm, sel ? c.sel_atoms : nullptr, c.n_sel_atoms,
+                                                    c.nl_j.as<int>(), c.rij.as<double>(), c.frow.as<double>(),
+                                                    c.rev_off.as<int>(), c.rev_idx.as<int>(), c.force.as<double>(),
+                                                    c.vatom.as<double>());
+    FEKF_LAUNCH_CHECK();
+    count_launch();
     virial_reduce_kernel<<<nb, 32, 0, s>>>(c.vatom.as<double>(), c.Na, c.virial.as<double>());
     FEKF_LAUNCH_CHECK();
     count_launch();
