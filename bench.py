@@ -464,7 +464,7 @@ def run_fekf(args, rank, world, local):
             "duration": "wall span per pass (split pass: early launch start -> later launch end), CUDA events",
             "achieved_launch_sum": achieved_sum, "frac_launch_sum": (achieved_sum / peak) if achieved_sum else None,
             "launches_timed": pass_n, "rw_launches": pass_rw, "share_of_step": (span_ms / max(ms, 1e-9)),
-            "split_pass_early_sms": split_sms, "split_updates": "force updates (the energy update's pass is unsplit)",
+            "split_pass_early_sms": split_sms, "split_updates": "energy and force updates" if os.environ.get("FEKF_SPLIT_E", "1") != "0" else "force updates",
             "standalone": standalone,
             "split_ms_per_pass": dict(zip(["early", "late", "early_start_to_reverse_done"],
                                           [x / max(pass_n, 1) for x in parts]))}

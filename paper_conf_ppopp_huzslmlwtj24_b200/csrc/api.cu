@@ -244,7 +244,7 @@ fekf_status Ctx::init(const fekf_model_cfg& mm, const fekf_opt_cfg& oo, int nato
   FEKF_TRY(dalloc(splitk_ws, sizeof(double) * splitk_elems));
   int maxh = 1;
   for (int l = 0; l < m.n_fit; ++l) maxh = std::max(maxh, m.fit[l]);
-  colsum_elems = (size_t)(cdiv(2LL * B * Na, 64) + 2) * maxh;
+  colsum_elems = (size_t)(2 * 148 + 2) * maxh;   // act_bwd_dt: at most 2 x 148 row chunks
   FEKF_TRY(dalloc(colsum_ws, sizeof(double) * colsum_elems));
 
   pairs.clear();

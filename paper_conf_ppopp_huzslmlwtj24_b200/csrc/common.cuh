@@ -36,7 +36,7 @@ void set_error(const std::string& msg);
     if (s__ != FEKF_OK) return s__;    \
   } while (0)
 
-inline int cdiv(int64_t a, int64_t b) { return (int)((a + b - 1) / b); }
+__host__ __device__ inline int cdiv(int64_t a, int64_t b) { return (int)((a + b - 1) / b); }
 
 // Device buffer owned by the library (cudaMalloc; freed in the owner's destructor).
 struct DBuf {

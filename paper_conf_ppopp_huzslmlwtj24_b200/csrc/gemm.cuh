@@ -157,13 +157,14 @@ __device__ __forceinline__ GemmProb<Epi> pick(const GemmGroup<Epi>& G, int q) {
 
 // Mainloop: GB_STAGES-deep cp.async ring (global -> SMEM without register staging), one
 // __syncthreads per BK slice, warp tiles of (WM/8) x (WN/8) DMMA 8x8 tiles.
-template <int BM, int BN, int WM, int WN, bool TA, bool TB, class Epi>
-__global__ void __launch_bounds__(256)
+template <int BM, int BN, int WM, int WN, bool TA, bool TB, class Epi, int NW = 8>
+__global__ void __launch_bounds__(32 * NW)
 dgemm_kernel(const __grid_constant__ GemmGroup<Epi> G) {
+  constexpr int NT = 32 * NW;
   constexpr int NWN = BN / WN;
-  static_assert((BM / WM) * NWN == 8, "8 warps");
+  static_assert((BM / WM) * NWN == NW, "warp grid");
   constexpr int TI = WM / 8, TJ = WN / 8;
-  constexpr int AE = BM * GB_K / 256, BE = BN * GB_K / 256;
+  constexpr int AE = (BM * GB_K + NT - 1) / NT, BE = (BN * GB_K + NT - 1) / NT;
   // SMEM layout follows the operand's global layout so consecutive threads copy consecutive
   // addresses: k-contiguous [mn][GB_LDS] (A row-major / B given as [N x K]) or mn-contiguous
   // [k][MN + 4] (A given as [K x M] / B row-major [K x N]).  Both strides make the 8x4 DMMA fragment
@@ -227,8 +228,8 @@ dgemm_kernel(const __grid_constant__ GemmGroup<Epi> G) {
     if (a16t) {
 #pragma unroll
       for (int q = 0; q < (AE + 1) / 2; ++q) {
-        const int idx = tid + 256 * q;
-        if (AE & 1 && idx >= BM * GB_K / 2) break;
+        const int idx = tid + NT * q;
+        if (idx >= BM * GB_K / 2) break;
         const int kk = idx / (BM / 2), r = 2 * (idx % (BM / 2));
         const int m = m0 + r, k = k0 + kk;
         const bool kin = k < kend;
@@ -250,8 +251,8 @@ dgemm_kernel(const __grid_constant__ GemmGroup<Epi> G) {
     } else if (a16) {
 #pragma unroll
       for (int q = 0; q < (AE + 1) / 2; ++q) {
-        const int idx = tid + 256 * q;
-        if (AE & 1 && idx >= BM * GB_K / 2) break;
+        const int idx = tid + NT * q;
+        if (idx >= BM * GB_K / 2) break;
         const int r = idx / (GB_K / 2), kk = 2 * (idx % (GB_K / 2));
         const int m = m0 + r, k = k0 + kk;
         const bool ok = m < M && k < kend;
@@ -260,7 +261,8 @@ dgemm_kernel(const __grid_constant__ GemmGroup<Epi> G) {
     } else {
 #pragma unroll
     for (int q = 0; q < AE; ++q) {
-      const int idx = tid + 256 * q;
+      const int idx = tid + NT * q;
+      if (BM * GB_K % NT && idx >= BM * GB_K) break;
       int r, kk;
       if (!TA) { r = idx / GB_K; kk = idx % GB_K; } else { kk = idx / BM; r = idx % BM; }
       const int m = m0 + r, k = k0 + kk;
@@ -277,8 +279,8 @@ dgemm_kernel(const __grid_constant__ GemmGroup<Epi> G) {
     if (b16) {
 #pragma unroll
       for (int q = 0; q < (BE + 1) / 2; ++q) {
-        const int idx = tid + 256 * q;
-        if (BE & 1 && idx >= BN * GB_K / 2) break;
+        const int idx = tid + NT * q;
+        if (idx >= BN * GB_K / 2) break;
         int c, kk;
         if (!TB) { kk = idx / (BN / 2); c = 2 * (idx % (BN / 2)); } else { c = idx / (GB_K / 2); kk = 2 * (idx % (GB_K / 2)); }
         const int n = n0 + c, k = k0 + kk;
@@ -289,7 +291,8 @@ dgemm_kernel(const __grid_constant__ GemmGroup<Epi> G) {
     }
 #pragma unroll
     for (int q = 0; q < BE; ++q) {
-      const int idx = tid + 256 * q;
+      const int idx = tid + NT * q;
+      if (BN * GB_K % NT && idx >= BN * GB_K) break;
       int c, kk;
       if (!TB) { kk = idx / BN; c = idx % BN; } else { c = idx / GB_K; kk = idx % GB_K; }
       const int n = n0 + c, k = k0 + kk;
@@ -336,14 +339,14 @@ dgemm_kernel(const __grid_constant__ GemmGroup<Epi> G) {
       }
 }
 
-template <int BM, int BN, int WM, int WN, bool TA, bool TB, class Epi>
+template <int BM, int BN, int WM, int WN, bool TA, bool TB, class Epi, int NW = 8>
 static fekf_status gemm_launch(GemmGroup<Epi>& G, cudaStream_t s) {
   constexpr size_t asz = TA ? GB_K * (BM + 4) : BM * GB_LDS;
   constexpr size_t bsz = TB ? BN * GB_LDS : GB_K * (BN + 4);
   constexpr size_t smem = sizeof(double) * GB_STAGES * (asz + bsz);
   static bool attr = false;
   if (!attr) {
-    FEKF_CHECK_CUDA(cudaFuncSetAttribute(dgemm_kernel<BM, BN, WM, WN, TA, TB, Epi>,
+    FEKF_CHECK_CUDA(cudaFuncSetAttribute(dgemm_kernel<BM, BN, WM, WN, TA, TB, Epi, NW>,
                                          cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
     attr = true;
   }
@@ -356,7 +359,7 @@ static fekf_status gemm_launch(GemmGroup<Epi>& G, cudaStream_t s) {
   }
   for (int q = G.n; q <= GG_MAX; ++q) G.start[q] = tot;
   if (tot == 0) return FEKF_OK;
-  dgemm_kernel<BM, BN, WM, WN, TA, TB, Epi><<<tot, 256, smem, s>>>(G);
+  dgemm_kernel<BM, BN, WM, WN, TA, TB, Epi, NW><<<tot, 32 * NW, smem, s>>>(G);
   FEKF_LAUNCH_CHECK();
   count_launch();
   return FEKF_OK;
@@ -381,12 +384,14 @@ static fekf_status gemm_group(GemmProb<Epi>* probs, int n, cudaStream_t s) {
   }
   if (G.n == 0) return FEKF_OK;
   if (nmax <= 32) return gemm_launch<128, 32, 32, 16, TA, TB>(G, s);
-  // the fitting widths (240) over a long K (the first fitting layer, K = M M^< = 1600): 128 x 80 tiles (warps
-  // 32 x 40) put N in 3 tiles and 6144 rows in 48, one wave of 144 CTAs on 148 SMs (64 x 64 tiles: 384 CTAs,
-  // 2.6 waves), with 0.45 fragment loads per DMMA; measured 220 -> 203 us (ncu).  With K = 240 the 64 x 64
-  // tiles win (several CTAs per SM hide the short main loop's prologue / epilogue: 49 vs 62 us)
+  // the fitting widths (240) over a long K (the first fitting layer, K = M M^< = 1600): 128 x 80 tiles put N
+  // in 3 tiles and 6144 rows in 48, one wave of 144 CTAs on 148 SMs (64 x 64 tiles: 384 CTAs,
+  // 2.6 waves): measured 220 -> 203 us (ncu); then 16 warps of 16 x 40 instead of 8 of 32 x 40 (4 warps per
+  // SMSP instead of 2, at 0.7 instead of 0.45 fragment loads per DMMA): 196 -> 181 us live.  With K = 240 the
+  // 64 x 64 tiles win (several CTAs per SM hide the short main loop's prologue / epilogue: 49 vs 62 us); 128 x
+  // 64 tiles with 16 warps measured slower there
   if (!TA && nmax % 80 == 0 && nmax <= 320 && rows >= 2048 && kmin >= 512)
-    return gemm_launch<128, 80, 32, 40, TA, TB>(G, s);
+    return gemm_launch<128, 80, 16, 40, TA, TB, Epi, 16>(G, s);
   if (rows < 65536) return gemm_launch<64, 64, 32, 16, TA, TB>(G, s);
   return gemm_launch<128, 64, 32, 32, TA, TB>(G, s);
 }

@@ -28,10 +28,47 @@ namespace fekf {
 // =================================================================================================
 // Sum the live split-K partials in a fixed order: splits [0, S0eff) of segment 0 and
 // [S0max, S0max + S1eff) of segment 1, where S*eff follow the device row counts (empty splits never
-// wrote).  32 outputs x 8 split-lanes per CTA, fixed 8-way combine -> deterministic.
-__global__ void splitk_reduce_kernel(const double* __restrict__ ws, int S0max, int S1max, int kps,
-                                     const int* __restrict__ K0dev, const int* __restrict__ K1dev, int M, int N,
-                                     double* __restrict__ out, int accum) {
+// wrote).  Two outputs per thread (16-byte loads when the workspace rows allow), the splits summed in
+// index order -> deterministic.  All split loads of one thread are independent (unrolled by 4), so the
+// kernel streams the (L2-resident) workspace instead of waiting on one load per split.
+template <bool V2>
+__global__ void __launch_bounds__(256) splitk_reduce_kernel(const double* __restrict__ ws, int S0max, int S1max,
+                                                            int kps, const int* __restrict__ K0dev,
+                                                            const int* __restrict__ K1dev, int M, int N,
+                                                            double* __restrict__ out, int accum) {
+  const long long MN = (long long)M * N;
+  const long long i = 2 * ((long long)blockIdx.x * blockDim.x + threadIdx.x);
+  if (i >= MN) return;
+  int S0 = S0max, S1 = S1max;
+  if (K0dev) S0 = min(S0max, max(1, (*K0dev + kps - 1) / kps));
+  if (K1dev && S1max > 0) S1 = min(S1max, max(1, (*K1dev + kps - 1) / kps));
+  const bool two = i + 1 < MN;
+  double a0 = 0.0, a1 = 0.0;
+  auto seg = [&](const double* base, int S) {
+#pragma unroll 4
+    for (int z = 0; z < S; ++z) {
+      const double* p = base + (size_t)z * MN + i;
+      if (V2) {
+        const double2 v = *reinterpret_cast<const double2*>(p);
+        a0 += v.x;
+        a1 += v.y;
+      } else {
+        a0 += p[0];
+        if (two) a1 += p[1];
+      }
+    }
+  };
+  seg(ws, S0);
+  seg(ws + (size_t)S0max * MN, S1);
+  out[i] = accum ? out[i] + a0 : a0;
+  if (two) out[i + 1] = accum ? out[i + 1] + a1 : a1;
+}
+// Few outputs over many splits (the fitting output layer: 241 x 1 over 2 x 64 splits): 32 outputs x 8
+// split-lanes per CTA, fixed 8-way combine.
+__global__ void __launch_bounds__(256) splitk_reduce_lanes_kernel(const double* __restrict__ ws, int S0max, int S1max,
+                                                                  int kps, const int* __restrict__ K0dev,
+                                                                  const int* __restrict__ K1dev, int M, int N,
+                                                                  double* __restrict__ out, int accum) {
   __shared__ double red[8][32];
   const int lane = threadIdx.x & 31, zl = threadIdx.x >> 5;
   const long long i = (long long)blockIdx.x * 32 + lane;
@@ -41,7 +78,9 @@ __global__ void splitk_reduce_kernel(const double* __restrict__ ws, int S0max, i
   if (K1dev && S1max > 0) S1 = min(S1max, max(1, (*K1dev + kps - 1) / kps));
   double a = 0.0;
   if (i < MN) {
+#pragma unroll 4
     for (int z = zl; z < S0; z += 8) a += ws[(size_t)z * MN + i];
+#pragma unroll 4
     for (int z = zl; z < S1; z += 8) a += ws[(size_t)(S0max + z) * MN + i];
   }
   red[zl][lane] = a;
@@ -52,6 +91,19 @@ __global__ void splitk_reduce_kernel(const double* __restrict__ ws, int S0max, i
     for (int q = 1; q < 8; ++q) t += red[q][lane];
     out[i] = accum ? out[i] + t : t;
   }
+}
+static void splitk_reduce(const double* ws, int S0, int S1, int kps, const int* k0, const int* k1, int M, int N,
+                          double* out, bool accum, cudaStream_t s) {
+  const long long MN = (long long)M * N;
+  if (S0 + S1 > 16) {
+    splitk_reduce_lanes_kernel<<<cdiv(MN, 32), 256, 0, s>>>(ws, S0, S1, kps, k0, k1, M, N, out, accum ? 1 : 0);
+    return;
+  }
+  const unsigned blocks = (unsigned)cdiv(cdiv(MN, 2), 256);
+  if (!(MN & 1) && !(reinterpret_cast<size_t>(ws) & 15))
+    splitk_reduce_kernel<true><<<blocks, 256, 0, s>>>(ws, S0, S1, kps, k0, k1, M, N, out, accum ? 1 : 0);
+  else
+    splitk_reduce_kernel<false><<<blocks, 256, 0, s>>>(ws, S0, S1, kps, k0, k1, M, N, out, accum ? 1 : 0);
 }
 
 struct Seg {
@@ -78,8 +130,7 @@ static fekf_status wgrad(Ctx& c, int din, int dout, Seg s0, Seg s1, double* gout
                                      s0.kdev, din, s0.ones ? (int)s0.kmax : 0, (int)S0, kps));
   if (S1) FEKF_TRY(gemm<true, false>(M, N, (int)s1.kmax, s1.H, din, s1.Zb, dout, EpiPartial{ws, M, N, (int)S0}, s,
                                      nullptr, s1.kdev, din, s1.ones ? (int)s1.kmax : 0, (int)S1, kps));
-  splitk_reduce_kernel<<<cdiv((long long)M * N, 32), 256, 0, s>>>(ws, (int)S0, (int)S1, kps, s0.kdev, s1.kdev, M, N,
-                                                                  gout, accum ? 1 : 0);
+  splitk_reduce(ws, (int)S0, (int)S1, kps, s0.kdev, s1.kdev, M, N, gout, accum, s);
   FEKF_LAUNCH_CHECK();
   count_launch();
   return FEKF_OK;
@@ -128,9 +179,8 @@ static fekf_status wgrad_group(Ctx& c, WgradJob* jobs, int n, cudaStream_t s) {
     const WgradJob& J = jobs[q];
     const int M = J.din + 1, N = J.dout;
     if (S0[q] + S1[q] == 0) continue;
-    splitk_reduce_kernel<<<cdiv((long long)M * N, 32), 256, 0, s>>>(c.splitk_ws.as<double>() + off[q], (int)S0[q],
-                                                                    (int)S1[q], (int)kps_[q], J.s0.kdev, J.s1.kdev, M,
-                                                                    N, J.gout, 0);
+    splitk_reduce(c.splitk_ws.as<double>() + off[q], (int)S0[q], (int)S1[q], (int)kps_[q], J.s0.kdev, J.s1.kdev, M,
+                  N, J.gout, false, s);
     FEKF_LAUNCH_CHECK();
     count_launch();
   }
@@ -188,32 +238,66 @@ __global__ void emb_act_bwd_kernel(int Rmax, const int* __restrict__ Rdev, int d
   Zb[i] = z;
 }
 
-// dt-grad: out[c] = sum_r A[r][c] B[r][c] (two fixed-order stages)
-__global__ void colsum_prod_kernel(const double* __restrict__ A, const double* __restrict__ B, long long rows, int d,
-                                   int chunk, double* __restrict__ ws) {
+// act_bwd fused with the timestep gradient of the layer (two fixed-order stages):
+//   dt[c] = sum_r y[r][c] hbar[r][c] + sum_r ydot[r][c] hdotbar[r][c]   (h = skip + dt * y)
+// block b: rows [b chunk, (b+1) chunk) of the primal half (and the same rows of the tangent half), one
+// thread per column (coalesced rows); the per-block sums go to ws[b][c] and colsum_reduce adds them.
+__global__ void act_bwd_dt_kernel(long long R, int d, const double* __restrict__ Y, const double* __restrict__ Hb,
+                                  const double* __restrict__ dt, int dual, double* __restrict__ Zb, int chunk,
+                                  double* __restrict__ ws) {
   const long long r0 = (long long)blockIdx.x * chunk;
-  const long long r1 = min(rows, r0 + chunk);
+  const long long r1 = min(R, r0 + chunk);
   for (int c = threadIdx.x; c < d; c += blockDim.x) {
-    double a = 0.0;
-    for (long long r = r0; r < r1; ++r) a += A[(size_t)r * d + c] * B[(size_t)r * d + c];
-    ws[(size_t)blockIdx.x * d + c] = a;
+    const double dtc = dt[c];
+    double acc = 0.0;
+#pragma unroll 4
+    for (long long r = r0; r < r1; ++r) {
+      const size_t i = (size_t)r * d + c;
+      const double y = Y[i], hb = Hb[i];
+      const double t = 1.0 - y * y;
+      acc += y * hb;
+      if (dual) {
+        const size_t j = (size_t)R * d + i;
+        const double yd = Y[j], hdb = Hb[j];
+        const double ydb = hdb * dtc;
+        Zb[i] = t * (hb * dtc) - 2.0 * y * yd * ydb;
+        Zb[j] = t * ydb;
+        acc += yd * hdb;
+      } else {
+        Zb[i] = t * (hb * dtc);
+      }
+    }
+    ws[(size_t)blockIdx.x * d + c] = acc;
   }
 }
+// out[c] = sum_k ws[k][c]: 32 columns x 8 chunk-lanes per CTA, fixed 8-way combine
 __global__ void colsum_reduce_kernel(const double* __restrict__ ws, int nchunk, int d, double* __restrict__ out) {
-  const int c = blockIdx.x * blockDim.x + threadIdx.x;
-  if (c >= d) return;
+  __shared__ double red[8][33];
+  const int cl = threadIdx.x & 31, z = threadIdx.x >> 5;
+  const int c = blockIdx.x * 32 + cl;
   double a = 0.0;
-  for (int k = 0; k < nchunk; ++k) a += ws[(size_t)k * d + c];
-  out[c] = a;
+  if (c < d) {
+#pragma unroll 4
+    for (int k = z; k < nchunk; k += 8) a += ws[(size_t)k * d + c];
+  }
+  red[z][cl] = a;
+  __syncthreads();
+  if (z == 0 && c < d) {
+    double t = red[0][cl];
+#pragma unroll
+    for (int q = 1; q < 8; ++q) t += red[q][cl];
+    out[c] = t;
+  }
 }
-static fekf_status colsum_prod(Ctx& c, const double* A, const double* B, long long rows, int d, double* out,
-                               cudaStream_t s) {
-  const int chunk = 64;
-  int nchunk = cdiv(rows, chunk);
+static fekf_status act_bwd_dt(Ctx& c, long long R, int d, const double* Y, const double* Hb, const double* dt,
+                              bool dual, double* Zb, double* gdt, cudaStream_t s) {
+  const int chunk = (int)std::max<long long>(4, cdiv(R, 2 * 148));
+  const int nchunk = (int)cdiv(R, chunk);
   if ((size_t)nchunk * d > c.colsum_elems) { set_error("colsum workspace too small"); return FEKF_EINVAL; }
-  colsum_prod_kernel<<<nchunk, 256, 0, s>>>(A, B, rows, d, chunk, c.colsum_ws.as<double>());
+  act_bwd_dt_kernel<<<nchunk, std::min(256, (d + 31) / 32 * 32), 0, s>>>(R, d, Y, Hb, dt, dual ? 1 : 0, Zb, chunk,
+                                                                         c.colsum_ws.as<double>());
   FEKF_LAUNCH_CHECK();
-  colsum_reduce_kernel<<<cdiv(d, 256), 256, 0, s>>>(c.colsum_ws.as<double>(), nchunk, d, out);
+  colsum_reduce_kernel<<<cdiv(d, 32), 256, 0, s>>>(c.colsum_ws.as<double>(), nchunk, d, gdt);
   FEKF_LAUNCH_CHECK();
   count_launch(2);
   return FEKF_OK;
@@ -281,31 +365,68 @@ __device__ __forceinline__ bool row_active(int r, int Na, int Nm, const int* __r
   const double* vj = v + ((size_t)b * Na + j) * 3;
   return vi[0] != 0.0 || vi[1] != 0.0 || vi[2] != 0.0 || vj[0] != 0.0 || vj[1] != 0.0 || vj[2] != 0.0;
 }
-__global__ void __launch_bounds__(TCHUNK)
-tcount_kernel(int Na, int Nm, int Rmax, const int* __restrict__ Rdev, const int* __restrict__ row_idx,
-              const int* __restrict__ nl_j, const double* __restrict__ v, int* __restrict__ chunk_cnt) {
-  const int R = min(Rmax, *Rdev);
+// every pair in one launch per pass (blockIdx.y = pair; chunks past a pair's extent exit)
+struct TrowArgs {
+  int Na, Nm;
+  const int* nl_j; const double* v;
+  int Rmax[NP];
+  const int* Rdev[NP];
+  const int* row_idx[NP];
+  int* ck[NP];
+  int* cnt[NP];
+  int* tidx[NP];
+  int* tpos[NP];
+};
+__global__ void __launch_bounds__(TCHUNK) tcount_kernel(const __grid_constant__ TrowArgs A) {
+  const int p = blockIdx.y;
+  if ((int)blockIdx.x >= cdiv(A.Rmax[p], TCHUNK)) return;
+  const int R = min(A.Rmax[p], *A.Rdev[p]);
   const int r = blockIdx.x * TCHUNK + threadIdx.x;
-  const bool a = r < R && row_active(r, Na, Nm, row_idx, nl_j, v);
+  const bool a = r < R && row_active(r, A.Na, A.Nm, A.row_idx[p], A.nl_j, A.v);
   const int n = __syncthreads_count(a);
-  if (threadIdx.x == 0) chunk_cnt[blockIdx.x] = n;
+  if (threadIdx.x == 0) A.ck[p][blockIdx.x] = n;
 }
-__global__ void tscan_kernel(int* __restrict__ chunk_cnt, int nchunk, int* __restrict__ cnt) {
-  if (threadIdx.x == 0) {
-    int run = 0;
-    for (int k = 0; k < nchunk; ++k) { const int x = chunk_cnt[k]; chunk_cnt[k] = run; run += x; }
-    *cnt = run;
+// exclusive scan of one pair's chunk counts (block p): each thread owns a run of consecutive chunks
+__global__ void __launch_bounds__(1024) tscan_kernel(const __grid_constant__ TrowArgs A) {
+  __shared__ int wsum[32];
+  const int p = blockIdx.x;
+  const int nchunk = cdiv(A.Rmax[p], TCHUNK);
+  int* ck = A.ck[p];
+  const int per = cdiv(nchunk, 1024);
+  const int k0 = min(nchunk, (int)threadIdx.x * per), k1 = min(nchunk, k0 + per);
+  int mine = 0;
+  for (int k = k0; k < k1; ++k) mine += ck[k];
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  int incl = mine;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const int y = __shfl_up_sync(0xffffffffu, incl, o);
+    if (lane >= o) incl += y;
   }
+  if (lane == 31) wsum[warp] = incl;
+  __syncthreads();
+  if (warp == 0) {
+    int x = wsum[lane], xi = x;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const int y = __shfl_up_sync(0xffffffffu, xi, o);
+      if (lane >= o) xi += y;
+    }
+    wsum[lane] = xi - x;
+    if (lane == 31) *A.cnt[p] = xi;
+  }
+  __syncthreads();
+  int run = wsum[warp] + incl - mine;
+  for (int k = k0; k < k1; ++k) { const int x = ck[k]; ck[k] = run; run += x; }
 }
-__global__ void __launch_bounds__(TCHUNK)
-tscatter_kernel(int Na, int Nm, int Rmax, const int* __restrict__ Rdev, const int* __restrict__ row_idx,
-                const int* __restrict__ nl_j, const double* __restrict__ v, const int* __restrict__ chunk_off,
-                int* __restrict__ tidx, int* __restrict__ tpos) {
+__global__ void __launch_bounds__(TCHUNK) tscatter_kernel(const __grid_constant__ TrowArgs A) {
   __shared__ int wsum[TCHUNK / 32];
-  const int R = min(Rmax, *Rdev);
+  const int p = blockIdx.y;
+  if ((int)blockIdx.x >= cdiv(A.Rmax[p], TCHUNK)) return;
+  const int R = min(A.Rmax[p], *A.Rdev[p]);
   const int r = blockIdx.x * TCHUNK + threadIdx.x;
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-  const bool a = r < R && row_active(r, Na, Nm, row_idx, nl_j, v);
+  const bool a = r < R && row_active(r, A.Na, A.Nm, A.row_idx[p], A.nl_j, A.v);
   const unsigned bal = __ballot_sync(0xffffffffu, a);
   if (lane == 0) wsum[warp] = __popc(bal);
   __syncthreads();
@@ -316,11 +437,11 @@ tscatter_kernel(int Na, int Nm, int Rmax, const int* __restrict__ Rdev, const in
   __syncthreads();
   if (r < R) {
     if (a) {
-      const int t = chunk_off[blockIdx.x] + wsum[warp] + __popc(bal & ((1u << lane) - 1u));
-      tidx[t] = r;
-      tpos[r] = t;
+      const int t = A.ck[p][blockIdx.x] + wsum[warp] + __popc(bal & ((1u << lane) - 1u));
+      A.tidx[p][t] = r;
+      A.tpos[p][r] = t;
     } else {
-      tpos[r] = -1;
+      A.tpos[p][r] = -1;
     }
   }
 }
@@ -1271,23 +1392,34 @@ fekf_status build_rows(Ctx& c, int nb, cudaStream_t s) {
 }
 
 static fekf_status build_trows(Ctx& c, int nb, cudaStream_t s) {
+  TrowArgs A{};
+  A.Na = c.Na;
+  A.Nm = c.Nm;
+  A.nl_j = c.nl_j.as<int>();
+  A.v = c.vdir.as<double>();
+  int np = 0, cmax = 0;
   for (size_t p = 0; p < c.pairs.size(); ++p) {
     PairNet& P = c.pairs[p];
     const long long Rmax = pair_rows(c, (int)p, nb);
     if (Rmax == 0) continue;
-    const int nchunk = cdiv(Rmax, TCHUNK);
-    int* ck = c.chunks.as<int>() + p * c.max_chunks;
-    tcount_kernel<<<nchunk, TCHUNK, 0, s>>>(c.Na, c.Nm, (int)Rmax, rcount(c, (int)p), P.row_idx.as<int>(),
-                                            c.nl_j.as<int>(), c.vdir.as<double>(), ck);
-    FEKF_LAUNCH_CHECK();
-    tscan_kernel<<<1, 32, 0, s>>>(ck, nchunk, c.rowcnt.as<int>() + c.pairs.size() + p);
-    FEKF_LAUNCH_CHECK();
-    tscatter_kernel<<<nchunk, TCHUNK, 0, s>>>(c.Na, c.Nm, (int)Rmax, rcount(c, (int)p), P.row_idx.as<int>(),
-                                              c.nl_j.as<int>(), c.vdir.as<double>(), ck, P.tidx.as<int>(),
-                                              P.tpos.as<int>());
-    FEKF_LAUNCH_CHECK();
-    count_launch(3);
+    A.Rmax[np] = (int)Rmax;
+    A.Rdev[np] = rcount(c, (int)p);
+    A.row_idx[np] = P.row_idx.as<int>();
+    A.ck[np] = c.chunks.as<int>() + p * c.max_chunks;
+    A.cnt[np] = c.rowcnt.as<int>() + c.pairs.size() + p;
+    A.tidx[np] = P.tidx.as<int>();
+    A.tpos[np] = P.tpos.as<int>();
+    cmax = std::max(cmax, cdiv(Rmax, TCHUNK));
+    ++np;
   }
+  if (np == 0) return FEKF_OK;
+  tcount_kernel<<<dim3(cmax, np), TCHUNK, 0, s>>>(A);
+  FEKF_LAUNCH_CHECK();
+  tscan_kernel<<<np, 1024, 0, s>>>(A);
+  FEKF_LAUNCH_CHECK();
+  tscatter_kernel<<<dim3(cmax, np), TCHUNK, 0, s>>>(A);
+  FEKF_LAUNCH_CHECK();
+  count_launch(3);
   return FEKF_OK;
 }
 
@@ -1540,10 +1672,15 @@ fekf_status model_backward(Ctx& c, int nb, Mode mode, double* gout, cudaStream_t
       const long long nF = dual ? 2 * F : F;
       const Layer& L = Fn.L[l];
       const double* dt = L.dt >= 0 ? w + L.dt : nullptr;
-      act_bwd_kernel<<<cdiv(F * L.dout, 256), 256, 0, s>>>(F, L.dout, Fn.Y[l].as<double>(), Fn.Hb[l].as<double>(), dt,
-                                                            dual ? 1 : 0, Fn.Zb[l].as<double>());
-      FEKF_LAUNCH_CHECK();
-      count_launch();
+      if (want_w && dt) {
+        FEKF_TRY(act_bwd_dt(c, F, L.dout, Fn.Y[l].as<double>(), Fn.Hb[l].as<double>(), dt, dual,
+                            Fn.Zb[l].as<double>(), gout + L.dt, s));
+      } else {
+        act_bwd_kernel<<<cdiv(F * L.dout, 256), 256, 0, s>>>(F, L.dout, Fn.Y[l].as<double>(), Fn.Hb[l].as<double>(),
+                                                              dt, dual ? 1 : 0, Fn.Zb[l].as<double>());
+        FEKF_LAUNCH_CHECK();
+        count_launch();
+      }
       const double* Hprev = l == 0 ? Fn.D.as<double>() : Fn.H[l - 1].as<double>();
       if (want_w) {
         // stacked rows; the ones column covers the primal half only (bias not in the tangent)
@@ -1551,7 +1688,6 @@ fekf_status model_backward(Ctx& c, int nb, Mode mode, double* gout, cudaStream_t
                               Seg{dual ? Hprev + (size_t)F * L.din : nullptr,
                                   dual ? Fn.Zb[l].as<double>() + (size_t)F * L.dout : nullptr, dual ? F : 0, nullptr, 0},
                               gout + L.W};
-        if (L.dt >= 0) FEKF_TRY(colsum_prod(c, Fn.Y[l].as<double>(), Fn.Hb[l].as<double>(), nF, L.dout, gout + L.dt, s));
       }
       double* out = l == 0 ? Fn.Db.as<double>() : Fn.Hb[l - 1].as<double>();
       EpiDgrad e{out, L.din, Fn.Hb[l].as<double>(), L.dout, l == 0 ? 0 : L.skip, L.din};
