@@ -388,9 +388,10 @@ _C4_GOLD = sorted(f[5:-5] for f in os.listdir(os.path.join(os.path.dirname(__fil
 @pytest.mark.parametrize("config", _C4_GOLD)
 def test_c4_time_to_target(config):
     """Metric (iii) on the Table-3 systems (C4 small-batch variants, tests/golden/rmse_c4s_*.json: the
-    oracle alone, S_o = 300 steps, every 20).  The GPU trajectory equals the oracle's at rel 1e-9 through
-    step 120 (before the learning onset; the chaotic growth of rounding differences afterwards is the same
-    as in the c1 test) and reaches the oracle's S_o-step RMSE within 1.5 S_o steps."""
+    oracle alone, S_o = 300 steps, every 20).  The GPU trajectory equals the oracle's at rel 1e-9 on the
+    plateau before the learning onset (the oracle's RMSE still above 0.9 x its step-20 value; the chaotic
+    growth of rounding differences afterwards is the same as in the c1 test) and reaches the oracle's
+    S_o-step RMSE within 1.5 S_o steps."""
     import json
     import sys
     sys.path.insert(0, os.path.join(os.path.dirname(os.path.dirname(__file__)), "tools"))
@@ -398,8 +399,11 @@ def test_c4_time_to_target(config):
     gold = json.load(open(os.path.join(os.path.dirname(__file__), "golden", f"rmse_{config}.json")))
     out = time_to_rmse.run(config, int(1.5 * gold["S_o"]), gold["every"], stop_at_target=True)
     assert out["flags"] == 0
-    early = [d for s, d in out["dev_vs_oracle"] if s <= 120]
-    assert len(early) == 7 and max(early) < 1e-9
+    tr = gold["trajectory"]
+    plateau = 0.9 * (tr[1][1] + tr[1][2])
+    onset = next(s for s, e, f in tr[1:] if e + f < plateau)
+    early = [d for s, d in out["dev_vs_oracle"] if s < onset]
+    assert len(early) >= 4 and max(early) < 1e-9
     assert out["reached"] is not None and out["reached"]["step"] <= int(1.5 * gold["S_o"])
 
 

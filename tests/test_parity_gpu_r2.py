@@ -106,6 +106,19 @@ def test_c4_system_model_parity(name):
     _check_model_pieces(m, ds, w, 2)
 
 
+def test_alloy4_wide_fitting_tiles_ragged():
+    """The first fitting layer's 128 x 80 / 16-warp GEMM (taken from 2048 fitting rows, K = 1600) with per-type
+    row counts that are not multiples of the tile (B = 24 images of the random 4-type alloy: 888 / 648 / 552 /
+    504 rows): forward, both Jacobians (primal and tangent rows) against the oracle."""
+    name = "c4_alloy108"
+    wl = get_config(name)
+    ds = make_dataset(name, 24)
+    w = init_weights(wl.model, 3, float(ds["energy"].mean() / len(ds["types"])))
+    rows = [24 * int((ds["types"] == t).sum()) for t in range(4)]
+    assert sum(rows) >= 2048 and any(r % 128 for r in rows)
+    _check_model_pieces(wl.model, ds, w, 24)
+
+
 def test_alloy4_train_steps():
     """A 4-type system (FEKF_MAX_TYPES; 16 embedding nets) through whole minibatch steps, small nets."""
     wl = get_config("c4_alloy108")
