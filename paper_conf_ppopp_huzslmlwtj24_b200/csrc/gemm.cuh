@@ -372,7 +372,7 @@ template <bool TA, bool TB, class Epi>
 static fekf_status gemm_group(GemmProb<Epi>* probs, int n, cudaStream_t s) {
   GemmGroup<Epi> G{};
   long long rows = 0;
-  int nmax = 0, kmin = 1 << 30;
+  int nmax = 0;
   for (int q = 0; q < n; ++q) {
     if (probs[q].M <= 0 || probs[q].N <= 0) continue;
     if (probs[q].kps <= 0) probs[q].kps = probs[q].K;
@@ -380,17 +380,16 @@ static fekf_status gemm_group(GemmProb<Epi>* probs, int n, cudaStream_t s) {
     G.p[G.n++] = probs[q];
     rows += probs[q].M;
     nmax = std::max(nmax, probs[q].N);
-    kmin = std::min(kmin, probs[q].kps);
   }
   if (G.n == 0) return FEKF_OK;
   if (nmax <= 32) return gemm_launch<128, 32, 32, 16, TA, TB>(G, s);
   // the fitting widths (240) over a long K (the first fitting layer, K = M M^< = 1600): 128 x 80 tiles put N
   // in 3 tiles and 6144 rows in 48, one wave of 144 CTAs on 148 SMs (64 x 64 tiles: 384 CTAs,
   // 2.6 waves): measured 220 -> 203 us (ncu); then 16 warps of 16 x 40 instead of 8 of 32 x 40 (4 warps per
-  // SMSP instead of 2, at 0.7 instead of 0.45 fragment loads per DMMA): 196 -> 181 us live.  With K = 240 the
-  // 64 x 64 tiles win (several CTAs per SM hide the short main loop's prologue / epilogue: 49 vs 62 us); 128 x
-  // 64 tiles with 16 warps measured slower there
-  if (!TA && nmax % 80 == 0 && nmax <= 320 && rows >= 2048 && kmin >= 512)
+  // SMSP instead of 2, at 0.7 instead of 0.45 fragment loads per DMMA): 196 -> 181 us live.  The 16-warp tile
+  // also wins for the K = 240 layers (forward 47 -> 42.5 us, data gradient 36.4 -> 33.2 us; the 8-warp 128 x 80
+  // tile lost to 64 x 64 there, 62 vs 49 us); 128 x 64 tiles with 16 warps measured slower on the generic path
+  if (!TA && nmax % 80 == 0 && nmax <= 320 && rows >= 2048)
     return gemm_launch<128, 80, 16, 40, TA, TB, Epi, 16>(G, s);
   if (rows < 65536) return gemm_launch<64, 64, 32, 16, TA, TB>(G, s);
   return gemm_launch<128, 64, 32, 32, TA, TB>(G, s);

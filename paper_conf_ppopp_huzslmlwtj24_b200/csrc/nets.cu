@@ -1807,9 +1807,11 @@ fekf_status model_backward(Ctx& c, int nb, Mode mode, double* gout, cudaStream_t
                                                     c.vatom.as<double>());
     FEKF_LAUNCH_CHECK();
     count_launch();
-    virial_reduce_kernel<<<nb, 32, 0, s>>>(c.vatom.as<double>(), c.Na, c.virial.as<double>());
-    FEKF_LAUNCH_CHECK();
-    count_launch();
+    if (!sel) {   // the force updates use the selected atoms' forces only: no virial there
+      virial_reduce_kernel<<<nb, 32, 0, s>>>(c.vatom.as<double>(), c.Na, c.virial.as<double>());
+      FEKF_LAUNCH_CHECK();
+      count_launch();
+    }
   }
   c.emb_sms = 0;
   return FEKF_OK;
