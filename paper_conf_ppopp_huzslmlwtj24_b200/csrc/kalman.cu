@@ -214,48 +214,63 @@ __device__ __forceinline__ void dmma884k(double& d0, double& d1, double a, doubl
                : "+d"(d0), "+d"(d1)
                : "d"(a), "d"(b));
 }
-template <typename PT, int NSTRIP>
+// Warp tile of the correction: NSTRIP 8-row strips x NJ 8-column chunks.  fp64 (one group of 8 warps): 2 strips
+// x 4 chunks (warp w: strips 2 (w >> 1) + {0, 1}, columns 32 (w & 1) + [0, 32)), so each u_k[J] fragment load
+// feeds 2 DMMAs (8-row strips x all 8 chunks per warp loaded every fragment for a single DMMA; the pass is
+// shared-memory bound there).  fp32 (groups of 4 warps): 2 strips x 8 chunks.
+template <typename PT, int NSTRIP, int NJ>
 __device__ __forceinline__ void apply_corrections(PT* t, const double (&ai)[NSTRIP][KMAX / 4], const double* vJ, int K,
-                                                  double sig, int strip0, int lane) {
+                                                  double sig, int strip0, int j0, int lane) {
   const int fr = lane >> 2, fk = lane & 3;
+  // strips sharing each fragment load: all of them while their accumulators fit (fp64: 2 x 4 chunks), else
+  // one at a time (fp32: 8 chunks per strip)
+  constexpr int SG = NSTRIP * NJ <= 8 ? NSTRIP : 1;
+  constexpr int X = sizeof(PT) == 8 ? 1 : 3;
+  static_assert(NJ > X, "rotation stays inside the warp's chunks");
+  const int rx = fr & X;
 #pragma unroll
-  for (int sp = 0; sp < NSTRIP; ++sp) {
-    const int m0 = 8 * (strip0 + sp);
-    double c[8][2];
+  for (int s0 = 0; s0 < NSTRIP; s0 += SG) {
+    double c[SG][NJ][2];
 #pragma unroll
-    for (int j = 0; j < 8; ++j) c[j][0] = c[j][1] = 0.0;
+    for (int sp = 0; sp < SG; ++sp)
+#pragma unroll
+      for (int j = 0; j < NJ; ++j) c[sp][j][0] = c[sp][j][1] = 0.0;
 #pragma unroll
     for (int ks = 0; ks < KMAX / 4; ++ks) {
       const int k0 = 4 * ks;
       if (k0 >= K) break;
       const int k = k0 + fk;
       const bool kv = k < K;
-      const double a = ai[sp][ks];   // beta_k u_k[row m0 + fr] of this item (registers, loaded at item start)
-      double b[8];
+      double b[NJ];
 #pragma unroll
-      for (int j = 0; j < 8; ++j) b[j] = kv ? vJ[k * VS + 8 * j + fr] : 0.0;
+      for (int j = 0; j < NJ; ++j) b[j] = kv ? vJ[k * VS + 8 * (j0 + j) + fr] : 0.0;
 #pragma unroll
-      for (int j = 0; j < 8; ++j) dmma884k(c[j][0], c[j][1], a, b[j]);
+      for (int sp = 0; sp < SG; ++sp) {
+        const double a = ai[s0 + sp][ks];   // beta_k u_k[row] of this item (registers, loaded at item start)
+#pragma unroll
+        for (int j = 0; j < NJ; ++j) dmma884k(c[sp][j][0], c[sp][j][1], a, b[j]);
+      }
     }
     // The fragment puts 4 lanes on each of 8 rows (lane = 4 fr + fk, columns 8j + 2fk, +1).  Rows are
     // 64 elements apart, so visiting the column chunks j in the same order on every row would land the
     // lanes of one shared-memory phase (8 lanes for 16-byte fp64 pairs, 16 for 8-byte fp32 pairs) on the
     // same banks.  Row fr visits chunk q ^ (fr & X) at step q instead (X = 1 fp64, 3 fp32): the rows of a
     // phase then cover disjoint banks.  The accumulator is picked with compile-time indices (selects).
-    constexpr int X = sizeof(PT) == 8 ? 1 : 3;
-    const int rx = fr & X;
-    PT* row = t + (m0 + fr) * KT + 2 * fk;
 #pragma unroll
-    for (int q = 0; q < 8; ++q) {
-      double a0 = c[q][0], a1 = c[q][1];
+    for (int sp = 0; sp < SG; ++sp) {
+      PT* row = t + (8 * (strip0 + s0 + sp) + fr) * KT + 2 * fk + 8 * j0;
 #pragma unroll
-      for (int x = 1; x <= X; ++x)
-        if (rx == x) { a0 = c[q ^ x][0]; a1 = c[q ^ x][1]; }
-      const int j = q ^ rx;
-      double2 v = ld2(row + 8 * j);
-      v.x = sig * (v.x - a0);
-      v.y = sig * (v.y - a1);
-      st2(row + 8 * j, v);
+      for (int q = 0; q < NJ; ++q) {
+        double a0 = c[sp][q][0], a1 = c[sp][q][1];
+#pragma unroll
+        for (int x = 1; x <= X; ++x)
+          if (rx == x) { a0 = c[sp][q ^ x][0]; a1 = c[sp][q ^ x][1]; }
+        const int j = q ^ rx;
+        double2 v = ld2(row + 8 * j);
+        v.x = sig * (v.x - a0);
+        v.y = sig * (v.y - a1);
+        st2(row + 8 * j, v);
+      }
     }
   }
 }
@@ -359,7 +374,11 @@ kf_pass_kernel(PT* __restrict__ P, const ItemD* __restrict__ items, int n_items,
   const double sig = st->sigma;
   const int c0 = 2 * lane;
   double gI[RPW], racc[RPW];
-  double ai[RPW / 8][KMAX / 4];
+  // correction warp tile (apply_corrections): 2 strips x NJC chunks; fp64 (8 warps): column half wg & 1
+  constexpr int NJC = NGW == 8 ? 4 : 8;
+  const int cstrip0 = NGW == 8 ? 2 * (wg >> 1) : 2 * wg, cj0 = NGW == 8 ? 4 * (wg & 1) : 0;
+  static_assert(NGW * 2 * NJC == 64, "correction tiles cover the 8 x 8 chunks of a tile");
+  double ai[2][KMAX / 4];
 #pragma unroll
   for (int k = 0; k < RPW; ++k) { gI[k] = 0.0; racc[k] = 0.0; }
   int s = gi, prev_s = -1;
@@ -382,11 +401,11 @@ kf_pass_kernel(PT* __restrict__ P, const ItemD* __restrict__ items, int n_items,
       if (rw) {   // beta_k u_k[row] of this warp's correction strips, fixed for the whole item
         const int fr = lane >> 2, fk = lane & 3;
 #pragma unroll
-        for (int sp = 0; sp < RPW / 8; ++sp)
+        for (int sp = 0; sp < 2; ++sp)
 #pragma unroll
           for (int ks = 0; ks < KMAX / 4; ++ks) {
             const int k = 4 * ks + fk;
-            const int row = 8 * (wg * (RPW / 8) + sp) + fr;
+            const int row = 8 * (cstrip0 + sp) + fr;
             ai[sp][ks] = k < K ? s_beta[k] * __ldg(ulist + (size_t)k * npad + it.vbase + (long long)it.I * KT + row) : 0.0;
           }
       }
@@ -397,9 +416,9 @@ kf_pass_kernel(PT* __restrict__ P, const ItemD* __restrict__ items, int n_items,
     const double* vJ = vg + KT;
     double ca0 = 0.0, ca1 = 0.0;
     if (rw) {
-      // B <- sigma (B - C) on the tensor path, 8-row strips per warp; then the group re-reads the
-      // rewritten tile (u_B = B_new g with B_new as stored) in its own element layout
-      apply_corrections<PT, RPW / 8>(t, ai, vJ, K, sig, wg * (RPW / 8), lane);
+      // B <- sigma (B - C) on the tensor path, a 16 x 32 (fp64) or 16 x 64 (fp32) warp tile; then the group
+      // re-reads the rewritten tile (u_B = B_new g with B_new as stored) in its own element layout
+      apply_corrections<PT, 2, NJC>(t, ai, vJ, K, sig, cstrip0, cj0, lane);
       asm volatile("bar.sync %0, %1;" ::"r"(1 + gi), "r"(GT) : "memory");
     }
 #pragma unroll
