@@ -216,8 +216,11 @@ __device__ __forceinline__ void dmma884k(double& d0, double& d1, double a, doubl
 }
 // Warp tile of the correction: NSTRIP 8-row strips x NJ 8-column chunks.  fp64 (one group of 8 warps): 2 strips
 // x 4 chunks (warp w: strips 2 (w >> 1) + {0, 1}, columns 32 (w & 1) + [0, 32)), so each u_k[J] fragment load
-// feeds 2 DMMAs (8-row strips x all 8 chunks per warp loaded every fragment for a single DMMA; the pass is
-// shared-memory bound there).  fp32 (groups of 4 warps): 2 strips x 8 chunks.
+// feeds 2 DMMAs (8-row strips x all 8 chunks per warp loaded every fragment for a single DMMA: 14.99 -> 14.36 ms
+// per read-write pass in the step; 4 strips x 2 chunks measured 14.46).  fp32 (groups of 4 warps): 2 strips x 8.
+#ifndef CORR_STRIPS
+#define CORR_STRIPS 2
+#endif
 template <typename PT, int NSTRIP, int NJ>
 __device__ __forceinline__ void apply_corrections(PT* t, const double (&ai)[NSTRIP][KMAX / 4], const double* vJ, int K,
                                                   double sig, int strip0, int j0, int lane) {
@@ -374,11 +377,12 @@ kf_pass_kernel(PT* __restrict__ P, const ItemD* __restrict__ items, int n_items,
   const double sig = st->sigma;
   const int c0 = 2 * lane;
   double gI[RPW], racc[RPW];
-  // correction warp tile (apply_corrections): 2 strips x NJC chunks; fp64 (8 warps): column half wg & 1
-  constexpr int NJC = NGW == 8 ? 4 : 8;
-  const int cstrip0 = NGW == 8 ? 2 * (wg >> 1) : 2 * wg, cj0 = NGW == 8 ? 4 * (wg & 1) : 0;
-  static_assert(NGW * 2 * NJC == 64, "correction tiles cover the 8 x 8 chunks of a tile");
-  double ai[2][KMAX / 4];
+  // correction warp tile (apply_corrections): NSC strips x NJC chunks; fp64 (8 warps): 4 strips x 2 chunks
+  // (column quarter wg & 3), fp32 (4 warps per group): 2 strips x 8 chunks
+  constexpr int NSC = NGW == 8 ? CORR_STRIPS : 2, NJC = 64 / (NGW * NSC);
+  const int cstrip0 = NSC * (wg / (8 / NJC)), cj0 = NJC * (wg % (8 / NJC));
+  static_assert(NGW * NSC * NJC == 64, "correction tiles cover the 8 x 8 chunks of a tile");
+  double ai[NSC][KMAX / 4];
 #pragma unroll
   for (int k = 0; k < RPW; ++k) { gI[k] = 0.0; racc[k] = 0.0; }
   int s = gi, prev_s = -1;
@@ -401,7 +405,7 @@ kf_pass_kernel(PT* __restrict__ P, const ItemD* __restrict__ items, int n_items,
       if (rw) {   // beta_k u_k[row] of this warp's correction strips, fixed for the whole item
         const int fr = lane >> 2, fk = lane & 3;
 #pragma unroll
-        for (int sp = 0; sp < 2; ++sp)
+        for (int sp = 0; sp < NSC; ++sp)
 #pragma unroll
           for (int ks = 0; ks < KMAX / 4; ++ks) {
             const int k = 4 * ks + fk;
@@ -418,7 +422,7 @@ kf_pass_kernel(PT* __restrict__ P, const ItemD* __restrict__ items, int n_items,
     if (rw) {
       // B <- sigma (B - C) on the tensor path, a 16 x 32 (fp64) or 16 x 64 (fp32) warp tile; then the group
       // re-reads the rewritten tile (u_B = B_new g with B_new as stored) in its own element layout
-      apply_corrections<PT, 2, NJC>(t, ai, vJ, K, sig, cstrip0, cj0, lane);
+      apply_corrections<PT, NSC, NJC>(t, ai, vJ, K, sig, cstrip0, cj0, lane);
       asm volatile("bar.sync %0, %1;" ::"r"(1 + gi), "r"(GT) : "memory");
     }
 #pragma unroll
