@@ -40,7 +40,9 @@ def parse():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--precision", type=int, default=64, choices=[64, 32],
-                    help="storage precision of P (32 = the fp32 variant, reading Z22; nets stay fp64)")
+                    help="64, or 32 = the fp32 variant (P stored fp32 and fp32 nets, reading Z22)")
+    ap.add_argument("--net-precision", type=int, default=0, choices=[0, 32, 64],
+                    help="nets' arithmetic: 0 = follow --precision, 32 or 64")
     ap.add_argument("--p-defer", type=int, default=None, help="override the deferred-correction depth")
     ap.add_argument("--p-mode", type=int, default=0, choices=[0, 1],
                     help="N > 1: 0 = P sharded over ranks (partial u all-reduced), 1 = replicated (the paper, P:L229)")
@@ -197,6 +199,13 @@ def oracle_sample(name, n_img=1, kf_blocks=1, seed=99):
 
 FP64_PEAK_TFLOPS = 37.1   # measured DMMA rate (tools/fp64_peak.cu on this pool's B200, round 1); guide-derived
                           # 148 SMs x 64 DFMA/clk x 2 x 1.965 GHz = 37.2
+# fp32 nets: the rate of their contraction primitive, the fp32-accurate 8x8x4 product from two
+# mma.sync.m16n8k4 tf32 (real.cuh), measured by tools/fp32_peak.cu on this pool's B200
+# (mma.sync.m16n8k4 tf32 measured at 138.5 TFLOP/s; an fp32-accurate 8x8x4 product takes two of them = the
+# four hi/lo products: 138.5 / 4 = 34.6; the microbench's loop, which re-splits its operands every product,
+# reaches 24.5).  FP32 FFMA measured 71.5 TFLOP/s.
+FP32_SPLIT_PEAK_TFLOPS = 34.6
+FP32_PEAK_SOURCE = "measured mma.sync tf32 rate / 4 split products (tools/fp32_peak.cu)"
 
 
 def nets_work(m, nl_j, types, groups):
@@ -279,12 +288,13 @@ def run_fekf(args, rank, world, local):
     torch.cuda.set_device(local)
     wl = get_config(args.config)
     m, opt = wl.model, wl.opt
-    over = {"precision": args.precision, "p_mode": args.p_mode}
+    over = {"precision": args.precision, "p_mode": args.p_mode, "net_precision": args.net_precision}
     if args.p_defer is not None:
         over["p_defer"] = args.p_defer
     opt = type(opt)(**{**opt.__dict__, **over})
     B = wl.batch
     Bg = B * world
+    net_prec = args.net_precision or args.precision
     ds = make_dataset(args.config, 2 * B, seed=wl.seed + 1000 * rank)
     na = len(ds["types"])
     w0 = init_weights(m, 3, float(make_dataset(args.config, 4, seed=wl.seed)["energy"].mean() / na))
@@ -451,9 +461,13 @@ def run_fekf(args, rank, world, local):
         torch.cuda.synchronize()
         nets_ms = n0.elapsed_time(n1) / reps
         tf = work["flops_per_step"] / (nets_ms / 1000.0) / 1e12
-        nets = {"kernels": "emb_fwd/emb_bwd/dgemm/desc_* (E + %d F Jacobians)" % opt.force_groups, "bound": "fp64",
-                "achieved": tf, "peak": FP64_PEAK_TFLOPS, "unit": "TFLOP/s", "frac": tf / FP64_PEAK_TFLOPS,
-                "peak_source": "measured DMMA (tools/fp64_peak.cu)", "ms_per_step_alone": nets_ms,
+        if net_prec == 32:
+            npk, nsrc, nbound = FP32_SPLIT_PEAK_TFLOPS, FP32_PEAK_SOURCE, "fp32 (split-tf32 tensor products)"
+        else:
+            npk, nsrc, nbound = FP64_PEAK_TFLOPS, "measured DMMA (tools/fp64_peak.cu)", "fp64"
+        nets = {"kernels": "emb_fwd/emb_bwd/dgemm/desc_* (E + %d F Jacobians)" % opt.force_groups, "bound": nbound,
+                "achieved": tf, "peak": npk, "unit": "TFLOP/s", "frac": tf / npk,
+                "peak_source": nsrc, "ms_per_step_alone": nets_ms,
                 "share_of_step_if_serial": nets_ms / (ms / args.steps), **work}
     except Exception as e:   # instrumentation only: never lose the bench line over it
         nets = {"error": str(e)[:200]}
@@ -471,12 +485,13 @@ def run_fekf(args, rank, world, local):
 
     out = {"metric": METRIC, "value": value, "unit": "images/s", "n_gpus": world, "steps": args.steps,
            "warmup": args.warmup, "ms_per_step": ms / args.steps, "higher_is_better": True, "scaling": "weak",
-           "vs_baseline": None, "dtype": "f64" if args.precision == 64 else "f64 nets / f32 P",
+           "vs_baseline": None, "dtype": {(64, 64): "f64", (32, 32): "f32", (32, 64): "f64 nets / f32 P",
+                                           (64, 32): "f32 nets / f64 P"}[(args.precision, net_prec)],
            "data": "synthetic (seeded perturbed %s snapshots, LJ labels)" % wl.system.name,
            "config": {"workload": args.config, "images_per_gpu": B, "global_batch": Bg, "n_atoms": na,
                       "n_params": ctx.n_params, "p_blocks": len(blocks), "p_bytes_per_gpu": info["p_bytes_local"],
                       "parallelism": f"dp{world}" + ((" + P replicated" if args.p_mode else " + P sharded") if world > 1 else ""),
-                      "p_precision": args.precision, "p_defer": opt.p_defer,
+                      "p_precision": args.precision, "net_precision": net_prec, "p_defer": opt.p_defer,
                       "l2": "inputs larger than L2: P (%.1f GiB packed) is streamed 5x per step"
                             % (info["p_bytes_local"] / 2**30)},
            "roofline": roof, "roofline_nets": nets, "e2e": e2e, "gpu_launches": int(launches), "clocks": clk,

@@ -66,7 +66,8 @@ class OptConfig:
     force_groups: int = 4
     atoms_per_group: int = 6
     p_defer: int = 15        # CUDA path only: deferred rank-1 corrections of P (same P up to rounding)
-    precision: int = 64      # CUDA path only: storage precision of P (32 = the fp32 variant, reading Z22)
+    precision: int = 64      # CUDA path only: 32 = the fp32 variant (P stored fp32 and fp32 nets, reading Z22)
+    net_precision: int = 0   # CUDA path only: nets' arithmetic, 0 = follow precision, 32 / 64
     p_mode: int = 0          # CUDA path only, world > 1: 0 = P sharded over ranks, 1 = replicated
 
 

@@ -162,6 +162,11 @@ fekf_status Ctx::init(const fekf_model_cfg& mm, const fekf_opt_cfg& oo, int nato
   }
   m = mm;
   o = oo;
+  if (o.net_precision != 0 && o.net_precision != 32 && o.net_precision != 64) {
+    set_error("create: net_precision must be 0 (follow precision), 32 or 64");
+    return FEKF_EINVAL;
+  }
+  net_prec = o.net_precision ? o.net_precision : (o.precision == 32 ? 32 : 64);
   Na = natoms;
   B = Bl;
   Bg = Bglob;
@@ -222,6 +227,12 @@ fekf_status Ctx::init(const fekf_model_cfg& mm, const fekf_opt_cfg& oo, int nato
   FEKF_TRY(dalloc(jac, sizeof(double) * nslots * 12));
   FEKF_TRY(dalloc(rij, sizeof(double) * nslots * 3));
   FEKF_TRY(dalloc(rdot, sizeof(double) * nslots * 4));
+  if (net_prec == 32) {   // the fp32 nets' copies of the fp64 geometry and weights (nets.cu)
+    FEKF_TRY(dalloc(em32, sizeof(float) * nslots * 4));
+    FEKF_TRY(dalloc(jac32, sizeof(float) * nslots * 12));
+    FEKF_TRY(dalloc(rij32, sizeof(float) * nslots * 3));
+    FEKF_TRY(dalloc(w32, sizeof(float) * Np));
+  }
   FEKF_TRY(dalloc(vdir, sizeof(double) * B * Na * 3));
   FEKF_TRY(dalloc(frow, sizeof(double) * nslots * 3));
   FEKF_TRY(dalloc(rev_cnt, sizeof(int) * (size_t)B * Na * Na));
@@ -357,7 +368,7 @@ Ctx::~Ctx() {
   kfo.reset();
   kf = nullptr;
   for (DBuf* b : {&types_d, &tindex_d, &atoms_d, &atoms_off_d, &sel_d, &sec_d, &err_d, &env_stats, &w, &gbuf, &nl_j, &nl_s,
-                  &overflow, &em, &jac, &rij, &rdot, &vdir, &frow, &rev_cnt, &rev_off, &rev_idx, &X, &Xb, &eatom, &etot, &force, &virial, &vatom, &splitk_ws,
+                  &overflow, &em, &jac, &rij, &rdot, &em32, &jac32, &rij32, &w32, &vdir, &frow, &rev_cnt, &rev_off, &rev_idx, &X, &Xb, &eatom, &etot, &force, &virial, &vatom, &splitk_ws,
                   &colsum_ws, &abe, &metrics_tmp, &abs_sum, &rowcnt, &chunks})
     dfree(*b);
   for (auto& P : pairs) {
@@ -389,6 +400,7 @@ static fekf_status geometry(Ctx& c, const double* coord, const double* box, int 
   FEKF_TRY(launch_nlist(c, coord, box, nb, c.nl_j.as<int>(), c.nl_s.as<int>(), c.overflow.as<int>(), s));
   FEKF_TRY(launch_envmat(c, coord, box, c.nl_j.as<int>(), c.nl_s.as<int>(), nb, c.em.as<double>(), c.jac.as<double>(),
                          c.rij.as<double>(), s));
+  FEKF_TRY(prepare_geometry(c, nb, s));   // fp32 nets: fp32 copies of R~, J, d
   FEKF_TRY(build_rows(c, nb, s));
   FEKF_TRY(build_reverse(c, nb, s));
   return FEKF_OK;
@@ -603,6 +615,7 @@ fekf_status fekf_opt_defaults(int global_batch, fekf_opt_cfg* o) {
   o->atoms_per_group = 6;
   o->p_defer = 15;
   o->precision = 64;
+  o->net_precision = 0;
   return FEKF_OK;
 }
 

@@ -1,19 +1,21 @@
-// Fused embedding-net kernels (sm_100a, fp64 DMMA m8n8k4): every layer of the embedding net
+// Fused embedding-net kernels (sm_100a; fp64 DMMA m8n8k4, fp32 the split-tf32 pair of real.cuh): every layer of the embedding net
 // G = E_{L-1} o ... o E_0(s) (skip rule: reading Z12) runs in one kernel with the activations
 // on chip, instead of one GEMM launch per layer with the activations round-tripping through HBM: the
 // forward per warp on 16-row tiles (no CTA barrier), the backward per CTA on 32-row tiles (its weight
 // gradients are split over the warps).  The kernels are compiled for the embedding widths of the
 // configured models (all index math constant-folded); other widths take the per-layer GEMM path.
 //
-// Shared-memory layout (doubles).  Every matrix uses a leading dimension ld = 16*ceil(w8/16) + 4
+// Shared-memory layout (elements of the nets' type, real.cuh).  Every matrix uses a leading dimension ld = 16*ceil(w8/16) + 4
 // (w8 = width rounded up to 8): ld = 4 (mod 16) makes both DMMA fragment patterns conflict-free,
 //   row pattern        (m = lane/4, k = lane%4) at m*ld + k     (A of a forward / data-gradient GEMM)
 //   transposed pattern (k = lane%4, n = lane/4) at k*ld + n     (B of a forward GEMM, A/B of a W-grad)
 // because each half-warp then touches 16 distinct 8-byte bank pairs.
 #pragma once
 #include "model.cuh"
+#include "real.cuh"
 
 namespace fekf {
+namespace FEKF_NETNS {
 
 constexpr int EMB_T = 32;       // rows per CTA tile of the backward
 constexpr int EMB_BWD_WARPS = 16;
@@ -61,9 +63,9 @@ struct EmbW {
     return m;
   }
   __host__ __device__ static constexpr int wALD(int q) { return sld(wmaxw(q)); }
-  static constexpr int WS = fB(NL);                              // weights + biases (doubles)
-  static constexpr int WRP = RT * (wALD(0) + wALD(1));           // per-warp activations (doubles)
-  static constexpr int WNW_FIT = (227 * 1024 / 8 - 32 - WS) / WRP;
+  static constexpr int WS = fB(NL);                              // weights + biases (elements)
+  static constexpr int WRP = RT * (wALD(0) + wALD(1));           // per-warp activations (elements)
+  static constexpr int WNW_FIT = ((int)(227 * 1024 / sizeof(real)) - 32 - WS) / WRP;
   static constexpr int WNW = WNW_FIT > 24 ? 24 : WNW_FIT;        // warps per CTA (one CTA per SM)
   static constexpr int W_SMEM = WS + WNW * WRP;
   // ---- backward: W_0 | W_l [pad8(din)][sld(d)] | aug_l [T][sld(din+1)] | 3 x buf [T][BLD] | rr [T][8]
@@ -105,10 +107,25 @@ struct EmbW {
   static constexpr int MAXB = (NBLK + EMB_BWD_WARPS - 1) / EMB_BWD_WARPS;
 };
 
+// the nets' views of the context's fp64 inputs: fp32 copies for the fp32 nets (nets.cu prepare_geometry,
+// model_forward), the fp64 buffers themselves otherwise
+#ifdef FEKF_NETS32
+inline real* em_of(const Ctx& c) { return c.em32.as<real>(); }
+inline real* jac_of(const Ctx& c) { return c.jac32.as<real>(); }
+inline real* rij_of(const Ctx& c) { return c.rij32.as<real>(); }
+inline real* w_of(const Ctx& c) { return c.w32.as<real>(); }
+#else
+inline real* em_of(const Ctx& c) { return c.em.as<real>(); }
+inline real* jac_of(const Ctx& c) { return c.jac.as<real>(); }
+inline real* rij_of(const Ctx& c) { return c.rij.as<real>(); }
+inline real* w_of(const Ctx& c) { return c.w.as<real>(); }
+#endif
+
 bool emb_fused_ok(const Ctx& c);
 fekf_status emb_forward(Ctx& c, int p, long long Rmax, bool tangent, cudaStream_t s);
 // Reverse pass of one pair's embedding net from the atoms' X-bar (mode: nets.cu Mode).  Adds the
 // weight gradients (ENERGY_GRAD, FORCE_JAC) into g, or writes s-bar per row (FORCE).
 fekf_status emb_backward(Ctx& c, int p, long long Rmax, int mode, double* g, cudaStream_t s);
 
+}  // namespace FEKF_NETNS
 }  // namespace fekf

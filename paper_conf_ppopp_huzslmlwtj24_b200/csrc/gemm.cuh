@@ -1,55 +1,59 @@
-// fp64 GEMM for the embedding / fitting layers on the sm_100a FP64 tensor path (DMMA,
-// mma.sync.m8n8k4.f64; measured on B200 at the same 37 TFLOP/s as FP64 FFMA but with ~5x less
-// shared-memory traffic per FMA).  tcgen05 has no fp64 kind, and TF32 would break the fp64 parity.
+// GEMM for the embedding / fitting layers in the nets' type (real.cuh).  fp64: the sm_100a FP64 tensor path
+// (DMMA, mma.sync.m8n8k4.f64; measured on B200 at the same 37 TFLOP/s as FP64 FFMA but with ~5x less
+// shared-memory traffic per FMA); tcgen05 has no fp64 kind, and TF32 would break the fp64 parity.
+// fp32: the same fragments through real.cuh's split-tf32 pair of mma.sync.m16n8k4 (fp32-accurate).
 // C = op(A) op(B) with a fused epilogue:
 //   TA: A stored [K x M] (weight gradients, K = rows); TB: B stored [N x K] (data gradients, W^T).
 //   Optional "ones" row aug_m of op(A): (k < aug_k ? 1 : 0), so [W-grad ; b-grad] = [H | 1]^T Zbar.
 //   Mdev / Kdev: device-resident row counts (compacted rows); CTAs past them exit.
 // CTA tile BM x BN x 16, 8 warps each WM x WN (WM/8 x WN/8 DMMA tiles), operands staged in SMEM
-// k-contiguous with a 20-double row stride (conflict-free fragment loads), 3-stage cp.async ring.
+// k-contiguous with a 20-element row stride (conflict-free fragment loads), 3-stage cp.async ring.
 #pragma once
 #include <algorithm>
 
 #include "model.cuh"
 #include "mathx.cuh"
+#include "real.cuh"
 
 namespace fekf {
+namespace FEKF_NETNS {
 
 constexpr int GB_K = 16;
 constexpr int GB_LDS = GB_K + 4;
 
 // Every epilogue gets split(z) (the CTA's split-K index) before its first use.
-struct EpiStore {
-  double* C; int ldc;
+template <class O>
+struct EpiStore {   // O = double: a weight gradient straight into g (fp64 whatever the nets' precision)
+  O* C; int ldc;
   __device__ void split(int) {}
-  __device__ void operator()(int r, int c, double v) const { C[(size_t)r * ldc + c] = v; }
+  __device__ void operator()(int r, int c, real v) const { C[(size_t)r * ldc + c] = (O)v; }
 };
 struct EpiPartial {
-  double* ws; int M, N; int zoff;
+  real* ws; int M, N; int zoff;
   __device__ void split(int z) { zoff += z; }
-  __device__ void operator()(int r, int c, double v) const {
+  __device__ void operator()(int r, int c, real v) const {
     ws[((size_t)zoff * M + r) * N + c] = v;
   }
 };
 // forward layer: y = tanh(z + b) (primal) or ydot = (1 - y^2) zdot (tangent); h = skip(h_prev) + dt*y
 struct EpiFwd {
   __device__ void split(int) {}
-  double* Y; double* H; int ld;
-  const double* bias; const double* dt;
-  const double* Hp; int ldp; int skip; int dprev;
-  const double* Yprim;    // non-null: tangent rows; primal y of row rowmap[r] (or r)
+  real* Y; real* H; int ld;
+  const real* bias; const real* dt;
+  const real* Hp; int ldp; int skip; int dprev;
+  const real* Yprim;    // non-null: tangent rows; primal y of row rowmap[r] (or r)
   const int* rowmap;
-  __device__ void operator()(int r, int c, double v) const {
-    double sk = 0.0;
+  __device__ void operator()(int r, int c, real v) const {
+    real sk = 0.0;
     if (skip == 1) sk = Hp[(size_t)r * ldp + c];
     else if (skip == 2) sk = Hp[(size_t)r * ldp + (c % dprev)];
-    double y;
+    real y;
     if (Yprim == nullptr) {
-      y = tanh_fp64(v + bias[c]);
+      y = tanh_r(v + bias[c]);
     } else {
       const int rp = rowmap ? rowmap[r] : r;
-      const double yp = Yprim[(size_t)rp * ld + c];
-      y = (1.0 - yp * yp) * v;
+      const real yp = Yprim[(size_t)rp * ld + c];
+      y = (real(1) - yp * yp) * v;
     }
     Y[(size_t)r * ld + c] = y;
     H[(size_t)r * ld + c] = sk + (dt ? dt[c] * y : y);
@@ -58,9 +62,9 @@ struct EpiFwd {
 // data gradient: hbar_prev = Zbar W^T + skip^T(hbar)
 struct EpiDgrad {
   __device__ void split(int) {}
-  double* out; int ldo; const double* Hb; int ld; int skip; int dprev;
-  __device__ void operator()(int r, int c, double v) const {
-    double s = 0.0;
+  real* out; int ldo; const real* Hb; int ld; int skip; int dprev;
+  __device__ void operator()(int r, int c, real v) const {
+    real s = 0.0;
     if (skip == 1) s = Hb[(size_t)r * ld + c];
     else if (skip == 2) s = Hb[(size_t)r * ld + c] + Hb[(size_t)r * ld + c + dprev];
     out[(size_t)r * ldo + c] = v + s;
@@ -73,49 +77,29 @@ struct EpiDgrad {
 // tangent launch: y of the primal row rowmap[r].
 struct EpiDgradAct {
   __device__ void split(int) {}
-  double* out; int ldo; const double* Hb; int ld; int skip; int dprev;
-  const double* Y; double* Zb;
-  const int* tpos; const double* Yt; const double* Hbt;
+  real* out; int ldo; const real* Hb; int ld; int skip; int dprev;
+  const real* Y; real* Zb;
+  const int* tpos; const real* Yt; const real* Hbt;
   const int* rowmap;
-  __device__ void operator()(int r, int c, double v) const {
-    double s = 0.0;
+  __device__ void operator()(int r, int c, real v) const {
+    real s = 0.0;
     if (skip == 1) s = Hb[(size_t)r * ld + c];
     else if (skip == 2) s = Hb[(size_t)r * ld + c] + Hb[(size_t)r * ld + c + dprev];
-    const double hb = v + s;
+    const real hb = v + s;
     const size_t o = (size_t)r * ldo + c;
     out[o] = hb;
-    const double y = Y[(rowmap ? (size_t)rowmap[r] : (size_t)r) * ldo + c];
-    double z = (1.0 - y * y) * hb;
+    const real y = Y[(rowmap ? (size_t)rowmap[r] : (size_t)r) * ldo + c];
+    real z = (real(1) - y * y) * hb;
     if (tpos) {
       const int tr = tpos[r];
       if (tr >= 0) {
         const size_t ot = (size_t)tr * ldo + c;
-        z -= 2.0 * y * Yt[ot] * Hbt[ot];
+        z -= real(2) * y * Yt[ot] * Hbt[ot];
       }
     }
     Zb[o] = z;
   }
 };
-
-__device__ __forceinline__ void dmma884(double& d0, double& d1, double a, double b) {
-  asm("mma.sync.aligned.m8n8k4.row.col.f64.f64.f64.f64 {%0,%1}, {%2}, {%3}, {%0,%1};"
-               : "+d"(d0), "+d"(d1)
-               : "d"(a), "d"(b));
-}
-
-__device__ __forceinline__ void cp_async8(double* dst, const double* src, bool valid) {
-  const unsigned d = (unsigned)__cvta_generic_to_shared(dst);
-  const int n = valid ? 8 : 0;  // src-size 0: zero-fill
-  asm volatile("cp.async.ca.shared.global [%0], [%1], 8, %2;" ::"r"(d), "l"(src), "r"(n) : "memory");
-}
-__device__ __forceinline__ void cp_async16z(double* dst, const double* src, bool valid) {
-  const unsigned d = (unsigned)__cvta_generic_to_shared(dst);
-  const int n = valid ? 16 : 0;  // src-size 0: zero-fill
-  asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(d), "l"(src), "r"(n) : "memory");
-}
-__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
-template <int N>
-__device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory"); }
 
 constexpr int GB_STAGES = 3;
 
@@ -127,8 +111,8 @@ struct GemmProb {
   int M, N, K;
   const int* Mdev;   // device row count (compacted rows) or nullptr
   const int* Kdev;   // device K (split-K over rows) or nullptr
-  const double* A; int lda;
-  const double* B; int ldb;
+  const real* A; int lda;
+  const real* B; int ldb;
   int aug_m, aug_k;  // "ones" row of op(A) (bias gradient), -1: none
   int kps, splits;   // K per split, number of splits
   Epi epi;
@@ -171,13 +155,13 @@ dgemm_kernel(const __grid_constant__ GemmGroup<Epi> G) {
   // loads bank-conflict free.
   constexpr int ASZ = TA ? GB_K * (BM + 4) : BM * GB_LDS;
   constexpr int BSZ = TB ? BN * GB_LDS : GB_K * (BN + 4);
-  extern __shared__ __align__(16) double gsm[];
-  double* As0 = gsm;
-  double* Bs0 = gsm + GB_STAGES * ASZ;
-  auto a_at = [&](int buf, int m, int k) -> double& {
+  extern __shared__ __align__(16) real gsm[];
+  real* As0 = gsm;
+  real* Bs0 = gsm + GB_STAGES * ASZ;
+  auto a_at = [&](int buf, int m, int k) -> real& {
     return TA ? As0[buf * ASZ + k * (BM + 4) + m] : As0[buf * ASZ + m * GB_LDS + k];
   };
-  auto b_at = [&](int buf, int n, int k) -> double& {
+  auto b_at = [&](int buf, int n, int k) -> real& {
     return TB ? Bs0[buf * BSZ + n * GB_LDS + k] : Bs0[buf * BSZ + k * (BN + 4) + n];
   };
   int q = 0;
@@ -193,8 +177,8 @@ dgemm_kernel(const __grid_constant__ GemmGroup<Epi> G) {
   const int bm = local % mtq, bn = (local / mtq) % ntq, bz = local / (mtq * ntq);
   int M = P.M, K = P.K, aug_k = P.aug_k;
   const int N = P.N, lda = P.lda, ldb = P.ldb, aug_m = P.aug_m, kps = P.kps;
-  const double* __restrict__ A = P.A;
-  const double* __restrict__ B = P.B;
+  const real* __restrict__ A = P.A;
+  const real* __restrict__ B = P.B;
   Epi epi = P.epi;
   epi.split(bz);
   if (P.Mdev) M = min(M, *P.Mdev);
@@ -211,19 +195,19 @@ dgemm_kernel(const __grid_constant__ GemmGroup<Epi> G) {
   const int warp = tid >> 5, lane = tid & 31;
   const int wm = warp / NWN, wn = warp % NWN;
   const int fr = lane >> 2, fk = lane & 3;
-  double acc[TI][TJ][2];
+  real acc[TI][TJ][2];
 #pragma unroll
   for (int i = 0; i < TI; ++i)
 #pragma unroll
     for (int j = 0; j < TJ; ++j) acc[i][j][0] = acc[i][j][1] = 0.0;
-  // 16-byte copies (two doubles along the contiguous dimension) when the problem's strides, bases and
+  // two-element copies (16 bytes fp64, 8 bytes fp32, along the contiguous dimension) when the problem's strides, bases and
   // extents keep every pair inside one row and aligned; per problem, so warp-uniform
-  const bool a16 = !TA && aug_m < 0 && !(lda & 1) && !(reinterpret_cast<size_t>(A) & 15) && !(K & 1) && !(kps & 1);
-  // TA (A stored [K x M], m-contiguous): pairs (m, m+1) of real columns go as one 16-byte copy; the pair
+  const bool a16 = !TA && aug_m < 0 && !(lda & 1) && !(reinterpret_cast<size_t>(A) & PAIR_MASK) && !(K & 1) && !(kps & 1);
+  // TA (A stored [K x M], m-contiguous): pairs (m, m+1) of real columns go as one two-element copy; the pair
   // holding the last real column / the "ones" row is done element by element
-  const bool a16t = TA && !(lda & 1) && !(reinterpret_cast<size_t>(A) & 15);
+  const bool a16t = TA && !(lda & 1) && !(reinterpret_cast<size_t>(A) & PAIR_MASK);
   const int mreal = aug_m >= 0 ? min(M, aug_m) : M;
-  const bool b16 = !(ldb & 1) && !(reinterpret_cast<size_t>(B) & 15) && (TB ? (!(K & 1) && !(kps & 1)) : !(N & 1));
+  const bool b16 = !(ldb & 1) && !(reinterpret_cast<size_t>(B) & PAIR_MASK) && (TB ? (!(K & 1) && !(kps & 1)) : !(N & 1));
   auto issue = [&](int buf, int k0) {
     if (a16t) {
 #pragma unroll
@@ -234,16 +218,16 @@ dgemm_kernel(const __grid_constant__ GemmGroup<Epi> G) {
         const int m = m0 + r, k = k0 + kk;
         const bool kin = k < kend;
         if (m + 1 < mreal) {
-          cp_async16z(&a_at(buf, r, kk), kin ? A + (size_t)k * lda + m : A, kin);
+          cp_async2(&a_at(buf, r, kk), kin ? A + (size_t)k * lda + m : A, kin);
         } else {
 #pragma unroll
           for (int h = 0; h < 2; ++h) {
-            double* dst = &a_at(buf, r + h, kk);
+            real* dst = &a_at(buf, r + h, kk);
             if (m + h == aug_m) {
-              *dst = (k < aug_k) ? 1.0 : 0.0;
+              *dst = (k < aug_k) ? real(1) : real(0);
             } else {
               const bool ok = m + h < M && kin;
-              cp_async8(dst, ok ? A + (size_t)k * lda + m + h : A, ok);
+              cp_async1(dst, ok ? A + (size_t)k * lda + m + h : A, ok);
             }
           }
         }
@@ -256,7 +240,7 @@ dgemm_kernel(const __grid_constant__ GemmGroup<Epi> G) {
         const int r = idx / (GB_K / 2), kk = 2 * (idx % (GB_K / 2));
         const int m = m0 + r, k = k0 + kk;
         const bool ok = m < M && k < kend;
-        cp_async16z(&a_at(buf, r, kk), ok ? A + (size_t)m * lda + k : A, ok);
+        cp_async2(&a_at(buf, r, kk), ok ? A + (size_t)m * lda + k : A, ok);
       }
     } else {
 #pragma unroll
@@ -266,13 +250,13 @@ dgemm_kernel(const __grid_constant__ GemmGroup<Epi> G) {
       int r, kk;
       if (!TA) { r = idx / GB_K; kk = idx % GB_K; } else { kk = idx / BM; r = idx % BM; }
       const int m = m0 + r, k = k0 + kk;
-      double* dst = &a_at(buf, r, kk);
+      real* dst = &a_at(buf, r, kk);
       if (m == aug_m) {
-        *dst = (k < aug_k) ? 1.0 : 0.0;
+        *dst = (k < aug_k) ? real(1) : real(0);
       } else {
         const bool ok = m < M && k < kend;
-        const double* src = ok ? (TA ? A + (size_t)k * lda + m : A + (size_t)m * lda + k) : A;
-        cp_async8(dst, src, ok);
+        const real* src = ok ? (TA ? A + (size_t)k * lda + m : A + (size_t)m * lda + k) : A;
+        cp_async1(dst, src, ok);
       }
     }
     }
@@ -285,7 +269,7 @@ dgemm_kernel(const __grid_constant__ GemmGroup<Epi> G) {
         if (!TB) { kk = idx / (BN / 2); c = 2 * (idx % (BN / 2)); } else { c = idx / (GB_K / 2); kk = 2 * (idx % (GB_K / 2)); }
         const int n = n0 + c, k = k0 + kk;
         const bool ok = n < N && k < kend;
-        cp_async16z(&b_at(buf, c, kk), ok ? (TB ? B + (size_t)n * ldb + k : B + (size_t)k * ldb + n) : B, ok);
+        cp_async2(&b_at(buf, c, kk), ok ? (TB ? B + (size_t)n * ldb + k : B + (size_t)k * ldb + n) : B, ok);
       }
       return;
     }
@@ -297,8 +281,8 @@ dgemm_kernel(const __grid_constant__ GemmGroup<Epi> G) {
       if (!TB) { kk = idx / BN; c = idx % BN; } else { c = idx / GB_K; kk = idx % GB_K; }
       const int n = n0 + c, k = k0 + kk;
       const bool ok = n < N && k < kend;
-      const double* src = ok ? (TB ? B + (size_t)n * ldb + k : B + (size_t)k * ldb + n) : B;
-      cp_async8(&b_at(buf, c, kk), src, ok);
+      const real* src = ok ? (TB ? B + (size_t)n * ldb + k : B + (size_t)k * ldb + n) : B;
+      cp_async1(&b_at(buf, c, kk), src, ok);
     }
   };
   const int nk = kend > kbeg ? (kend - kbeg + GB_K - 1) / GB_K : 0;
@@ -316,11 +300,11 @@ dgemm_kernel(const __grid_constant__ GemmGroup<Epi> G) {
     const int buf = t % GB_STAGES;
 #pragma unroll
     for (int ks = 0; ks < GB_K; ks += 4) {
-      double a[TI], b[TJ];
+      frag_t a[TI], b[TJ];
 #pragma unroll
-      for (int i = 0; i < TI; ++i) a[i] = a_at(buf, wm * WM + i * 8 + fr, ks + fk);
+      for (int i = 0; i < TI; ++i) a[i] = frag(a_at(buf, wm * WM + i * 8 + fr, ks + fk));
 #pragma unroll
-      for (int j = 0; j < TJ; ++j) b[j] = b_at(buf, wn * WN + j * 8 + fr, ks + fk);
+      for (int j = 0; j < TJ; ++j) b[j] = frag(b_at(buf, wn * WN + j * 8 + fr, ks + fk));
 #pragma unroll
       for (int i = 0; i < TI; ++i)
 #pragma unroll
@@ -343,7 +327,7 @@ template <int BM, int BN, int WM, int WN, bool TA, bool TB, class Epi, int NW = 
 static fekf_status gemm_launch(GemmGroup<Epi>& G, cudaStream_t s) {
   constexpr size_t asz = TA ? GB_K * (BM + 4) : BM * GB_LDS;
   constexpr size_t bsz = TB ? BN * GB_LDS : GB_K * (BN + 4);
-  constexpr size_t smem = sizeof(double) * GB_STAGES * (asz + bsz);
+  constexpr size_t smem = sizeof(real) * GB_STAGES * (asz + bsz);
   static bool attr = false;
   if (!attr) {
     FEKF_CHECK_CUDA(cudaFuncSetAttribute(dgemm_kernel<BM, BN, WM, WN, TA, TB, Epi, NW>,
@@ -396,11 +380,12 @@ static fekf_status gemm_group(GemmProb<Epi>* probs, int n, cudaStream_t s) {
 }
 
 template <bool TA, bool TB, class Epi>
-static fekf_status gemm(long long M, int N, int K, const double* A, int lda, const double* B, int ldb, Epi epi,
+static fekf_status gemm(long long M, int N, int K, const real* A, int lda, const real* B, int ldb, Epi epi,
                         cudaStream_t s, const int* Mdev = nullptr, const int* Kdev = nullptr, int aug_m = -1,
                         int aug_k = 0, int splits = 1, int kps = 0) {
   GemmProb<Epi> p{(int)M, N, K, Mdev, Kdev, A, lda, B, ldb, aug_m, aug_k, kps, splits, epi};
   return gemm_group<TA, TB>(&p, 1, s);
 }
 
+}  // namespace FEKF_NETNS
 }  // namespace fekf

@@ -111,4 +111,9 @@ __device__ __forceinline__ double tanh_fp64(double x) {
   return copysign(qq, x);
 }
 
+// the nets' activation in their own precision (real.cuh): fp64 above, fp32 the CUDA math library's tanhf
+// (max 2 ulp)
+__device__ __forceinline__ double tanh_r(double x) { return tanh_fp64(x); }
+__device__ __forceinline__ float tanh_r(float x) { return tanhf(x); }
+
 }  // namespace fekf

@@ -68,6 +68,10 @@ struct Ctx {
   DBuf env_stats;                                 // [2][nt][4]: avg | std of the R~ rows (reading Z11)
   DBuf w, gbuf;                                   // [Np], [Np + 1] (g || error sum, the allreduce payload)
   DBuf nl_j, nl_s, overflow, em, jac, rij, rdot, vdir;
+  // fp32 nets (net_prec 32): fp32 copies of R~, its Jacobian, d and the weights (nets.cu prepare_geometry /
+  // model_forward); every other nets buffer holds elements of the nets' type
+  int net_prec = 64;
+  DBuf em32, jac32, rij32, w32;
   // atomics-free force scatter (reverse neighbour map, built once per geometry): frow [slot][3] = dE/dd of
   // every valid slot, rev_off [B*Na + 1] / rev_idx [slots] = for every atom j the slots whose neighbour is
   // j, in slot order; rev_cnt [B][Na][Na] scratch of the deterministic fill
@@ -112,22 +116,50 @@ fekf_status launch_nlist(Ctx& c, const double* coord, const double* box, int nb,
 fekf_status launch_envmat(Ctx& c, const double* coord, const double* box, const int* nl_j, const int* nl_s, int nb,
                           double* em, double* jac, double* rij, cudaStream_t s);
 
-// nets.cu
+// nets.cu (compiled twice, real.cuh: n64 = fp64 nets, n32 = fp32 nets)
 // MODE_FORCE_SEL: forces on the selected atoms only (a force update needs F_pred on S_k):
 // the embedding reverse runs over the rows that touch S_k (the tangent-active rows, built beforehand by
 // mark_selected) instead of every row; forces of other atoms are left partial.
 enum Mode { MODE_ENERGY_GRAD = 0, MODE_FORCE = 1, MODE_FORCE_JAC = 2, MODE_FORCE_SEL = 3 };
-fekf_status model_forward(Ctx& c, int nb, bool tangent, cudaStream_t s);
-fekf_status mark_selected(Ctx& c, int nb, const int* atom_idx, int n_sel, cudaStream_t s);
-fekf_status model_backward(Ctx& c, int nb, Mode mode, double* g, cudaStream_t s);
-fekf_status energy_outputs(Ctx& c, int nb, cudaStream_t s);
-fekf_status energy_error(Ctx& c, int nb, const double* e_label, double* abs_sum, cudaStream_t s);
-fekf_status force_error(Ctx& c, int nb, const double* f_label, const int* atom_idx, int n_sel, double* abs_sum,
-                        cudaStream_t s);
-fekf_status tangent_env(Ctx& c, int nb, cudaStream_t s);
-fekf_status build_rows(Ctx& c, int nb, cudaStream_t s);
-fekf_status build_reverse(Ctx& c, int nb, cudaStream_t s);
-fekf_status seed_force(Ctx& c, int nb, cudaStream_t s);
+#define FEKF_NETS_API                                                                                       \
+  fekf_status prepare_geometry(Ctx& c, int nb, cudaStream_t s);                                             \
+  fekf_status model_forward(Ctx& c, int nb, bool tangent, cudaStream_t s);                                  \
+  fekf_status mark_selected(Ctx& c, int nb, const int* atom_idx, int n_sel, cudaStream_t s);                \
+  fekf_status model_backward(Ctx& c, int nb, Mode mode, double* g, cudaStream_t s);                         \
+  fekf_status energy_outputs(Ctx& c, int nb, cudaStream_t s);                                               \
+  fekf_status energy_error(Ctx& c, int nb, const double* e_label, double* abs_sum, cudaStream_t s);         \
+  fekf_status force_error(Ctx& c, int nb, const double* f_label, const int* atom_idx, int n_sel,            \
+                          double* abs_sum, cudaStream_t s);                                                 \
+  fekf_status tangent_env(Ctx& c, int nb, cudaStream_t s);                                                  \
+  fekf_status build_rows(Ctx& c, int nb, cudaStream_t s);                                                   \
+  fekf_status build_reverse(Ctx& c, int nb, cudaStream_t s);                                                \
+  fekf_status seed_force(Ctx& c, int nb, cudaStream_t s);
+namespace n64 { FEKF_NETS_API }
+namespace n32 { FEKF_NETS_API }
+#undef FEKF_NETS_API
+// the nets' precision of a context (fekf_opt_cfg::net_precision; 0 follows `precision`)
+inline bool nets32(const Ctx& c) { return c.net_prec == 32; }
+#define FEKF_NETS_CALL(f) return nets32(c) ? n32::f : n64::f
+inline fekf_status prepare_geometry(Ctx& c, int nb, cudaStream_t s) { FEKF_NETS_CALL(prepare_geometry(c, nb, s)); }
+inline fekf_status model_forward(Ctx& c, int nb, bool t, cudaStream_t s) { FEKF_NETS_CALL(model_forward(c, nb, t, s)); }
+inline fekf_status mark_selected(Ctx& c, int nb, const int* a, int n, cudaStream_t s) {
+  FEKF_NETS_CALL(mark_selected(c, nb, a, n, s));
+}
+inline fekf_status model_backward(Ctx& c, int nb, Mode m, double* g, cudaStream_t s) {
+  FEKF_NETS_CALL(model_backward(c, nb, m, g, s));
+}
+inline fekf_status energy_outputs(Ctx& c, int nb, cudaStream_t s) { FEKF_NETS_CALL(energy_outputs(c, nb, s)); }
+inline fekf_status energy_error(Ctx& c, int nb, const double* e, double* a, cudaStream_t s) {
+  FEKF_NETS_CALL(energy_error(c, nb, e, a, s));
+}
+inline fekf_status force_error(Ctx& c, int nb, const double* f, const int* idx, int n, double* a, cudaStream_t s) {
+  FEKF_NETS_CALL(force_error(c, nb, f, idx, n, a, s));
+}
+inline fekf_status tangent_env(Ctx& c, int nb, cudaStream_t s) { FEKF_NETS_CALL(tangent_env(c, nb, s)); }
+inline fekf_status build_rows(Ctx& c, int nb, cudaStream_t s) { FEKF_NETS_CALL(build_rows(c, nb, s)); }
+inline fekf_status build_reverse(Ctx& c, int nb, cudaStream_t s) { FEKF_NETS_CALL(build_reverse(c, nb, s)); }
+inline fekf_status seed_force(Ctx& c, int nb, cudaStream_t s) { FEKF_NETS_CALL(seed_force(c, nb, s)); }
+#undef FEKF_NETS_CALL
 
 }  // namespace fekf
 

@@ -1,4 +1,5 @@
-// DeePMD se_a nets on sm_100a, fp64: forward, backward to coordinates, energy- and force-Jacobians.
+// DeePMD se_a nets on sm_100a: forward, backward to coordinates, energy- and force-Jacobians.  Written over
+// the nets' type `real` (real.cuh): compiled as fp64 (this file, namespace n64) and as fp32 (nets32.cu, n32).
 //
 //   embedding  G = E2 o E1 o E0(s)          P:L84-90 (§2.1 item 2), skip rule: reading Z12
 //   descriptor X = R~^T G / N_m, D = X^T X^<   P:L92, P:L233 (Fig. 6), scale 1/N_m: reading Z13
@@ -20,6 +21,7 @@
 #include "emb.cuh"
 
 namespace fekf {
+namespace FEKF_NETNS {
 
 // =================================================================================================
 // weight gradients: [W-grad ; b-grad] (din+1 x dout) = [H | 1]^T Zbar + [Hdot | 0]^T Zdotbar
@@ -32,7 +34,7 @@ namespace fekf {
 // index order -> deterministic.  All split loads of one thread are independent (unrolled by 4), so the
 // kernel streams the (L2-resident) workspace instead of waiting on one load per split.
 template <bool V2>
-__global__ void __launch_bounds__(256) splitk_reduce_kernel(const double* __restrict__ ws, int S0max, int S1max,
+__global__ void __launch_bounds__(256) splitk_reduce_kernel(const real* __restrict__ ws, int S0max, int S1max,
                                                             int kps, const int* __restrict__ K0dev,
                                                             const int* __restrict__ K1dev, int M, int N,
                                                             double* __restrict__ out, int accum) {
@@ -43,13 +45,13 @@ __global__ void __launch_bounds__(256) splitk_reduce_kernel(const double* __rest
   if (K0dev) S0 = min(S0max, max(1, (*K0dev + kps - 1) / kps));
   if (K1dev && S1max > 0) S1 = min(S1max, max(1, (*K1dev + kps - 1) / kps));
   const bool two = i + 1 < MN;
-  double a0 = 0.0, a1 = 0.0;
-  auto seg = [&](const double* base, int S) {
+  real a0 = 0.0, a1 = 0.0;
+  auto seg = [&](const real* base, int S) {
 #pragma unroll 4
     for (int z = 0; z < S; ++z) {
-      const double* p = base + (size_t)z * MN + i;
+      const real* p = base + (size_t)z * MN + i;
       if (V2) {
-        const double2 v = *reinterpret_cast<const double2*>(p);
+        const real2 v = *reinterpret_cast<const real2*>(p);
         a0 += v.x;
         a1 += v.y;
       } else {
@@ -65,18 +67,18 @@ __global__ void __launch_bounds__(256) splitk_reduce_kernel(const double* __rest
 }
 // Few outputs over many splits (the fitting output layer: 241 x 1 over 2 x 64 splits): 32 outputs x 8
 // split-lanes per CTA, fixed 8-way combine.
-__global__ void __launch_bounds__(256) splitk_reduce_lanes_kernel(const double* __restrict__ ws, int S0max, int S1max,
+__global__ void __launch_bounds__(256) splitk_reduce_lanes_kernel(const real* __restrict__ ws, int S0max, int S1max,
                                                                   int kps, const int* __restrict__ K0dev,
                                                                   const int* __restrict__ K1dev, int M, int N,
                                                                   double* __restrict__ out, int accum) {
-  __shared__ double red[8][32];
+  __shared__ real red[8][32];
   const int lane = threadIdx.x & 31, zl = threadIdx.x >> 5;
   const long long i = (long long)blockIdx.x * 32 + lane;
   const long long MN = (long long)M * N;
   int S0 = S0max, S1 = S1max;
   if (K0dev) S0 = min(S0max, max(1, (*K0dev + kps - 1) / kps));
   if (K1dev && S1max > 0) S1 = min(S1max, max(1, (*K1dev + kps - 1) / kps));
-  double a = 0.0;
+  real a = 0.0;
   if (i < MN) {
 #pragma unroll 4
     for (int z = zl; z < S0; z += 8) a += ws[(size_t)z * MN + i];
@@ -86,13 +88,13 @@ __global__ void __launch_bounds__(256) splitk_reduce_lanes_kernel(const double* 
   red[zl][lane] = a;
   __syncthreads();
   if (zl == 0 && i < MN) {
-    double t = red[0][lane];
+    real t = red[0][lane];
 #pragma unroll
     for (int q = 1; q < 8; ++q) t += red[q][lane];
     out[i] = accum ? out[i] + t : t;
   }
 }
-static void splitk_reduce(const double* ws, int S0, int S1, int kps, const int* k0, const int* k1, int M, int N,
+static void splitk_reduce(const real* ws, int S0, int S1, int kps, const int* k0, const int* k1, int M, int N,
                           double* out, bool accum, cudaStream_t s) {
   const long long MN = (long long)M * N;
   if (S0 + S1 > 16) {
@@ -107,7 +109,7 @@ static void splitk_reduce(const double* ws, int S0, int S1, int kps, const int* 
 }
 
 struct Seg {
-  const double* H; const double* Zb; long long kmax; const int* kdev; int ones;
+  const real* H; const real* Zb; long long kmax; const int* kdev; int ones;
 };
 
 // accum: add into gout (embedding nets shared by several type pairs, type_one_side) instead of writing
@@ -123,9 +125,9 @@ static fekf_status wgrad(Ctx& c, int din, int dout, Seg s0, Seg s1, double* gout
   const long long S0 = nsplit(s0), S1 = nsplit(s1);
   if (S0 + S1 == 0) return FEKF_OK;
   if (S0 == 1 && S1 == 0 && !accum)
-    return gemm<true, false>(M, N, (int)s0.kmax, s0.H, din, s0.Zb, dout, EpiStore{gout, dout}, s, nullptr, s0.kdev,
+    return gemm<true, false>(M, N, (int)s0.kmax, s0.H, din, s0.Zb, dout, EpiStore<double>{gout, dout}, s, nullptr, s0.kdev,
                              din, s0.ones ? (int)s0.kmax : 0);
-  double* ws = c.splitk_ws.as<double>();
+  real* ws = c.splitk_ws.as<real>();
   if (S0) FEKF_TRY(gemm<true, false>(M, N, (int)s0.kmax, s0.H, din, s0.Zb, dout, EpiPartial{ws, M, N, 0}, s, nullptr,
                                      s0.kdev, din, s0.ones ? (int)s0.kmax : 0, (int)S0, kps));
   if (S1) FEKF_TRY(gemm<true, false>(M, N, (int)s1.kmax, s1.H, din, s1.Zb, dout, EpiPartial{ws, M, N, (int)S0}, s,
@@ -165,7 +167,7 @@ static fekf_status wgrad_group(Ctx& c, WgradJob* jobs, int n, cudaStream_t s) {
     kps_[q] = kps;
     off[q] = used;
     used += (size_t)(S0[q] + S1[q]) * M * N;
-    double* ws = c.splitk_ws.as<double>() + off[q];
+    real* ws = c.splitk_ws.as<real>() + off[q];
     if (S0[q])
       pr[np++] = GemmProb<EpiPartial>{M, N, (int)J.s0.kmax, nullptr, J.s0.kdev, J.s0.H, J.din, J.s0.Zb, J.dout,
                                       J.din, J.s0.ones ? (int)J.s0.kmax : 0, kps, (int)S0[q], EpiPartial{ws, M, N, 0}};
@@ -179,7 +181,7 @@ static fekf_status wgrad_group(Ctx& c, WgradJob* jobs, int n, cudaStream_t s) {
     const WgradJob& J = jobs[q];
     const int M = J.din + 1, N = J.dout;
     if (S0[q] + S1[q] == 0) continue;
-    splitk_reduce(c.splitk_ws.as<double>() + off[q], (int)S0[q], (int)S1[q], (int)kps_[q], J.s0.kdev, J.s1.kdev, M,
+    splitk_reduce(c.splitk_ws.as<real>() + off[q], (int)S0[q], (int)S1[q], (int)kps_[q], J.s0.kdev, J.s1.kdev, M,
                   N, J.gout, false, s);
     FEKF_LAUNCH_CHECK();
     count_launch();
@@ -192,21 +194,21 @@ static fekf_status wgrad_group(Ctx& c, WgradJob* jobs, int n, cudaStream_t s) {
 // =================================================================================================
 // fitting (stacked rows): zbar = (1 - y^2) ybar - 2 y ydot ydotbar, zdotbar = (1 - y^2) ydotbar;
 // ybar = dt * hbar on residual layers with a timestep vector, else hbar.
-__global__ void act_bwd_kernel(long long R, int d, const double* __restrict__ Y, const double* __restrict__ Hb,
-                               const double* __restrict__ dt, int dual, double* __restrict__ Zb) {
+__global__ void act_bwd_kernel(long long R, int d, const real* __restrict__ Y, const real* __restrict__ Hb,
+                               const real* __restrict__ dt, int dual, real* __restrict__ Zb) {
   const long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x;
   if (i >= R * d) return;
   const int c = (int)(i % d);
-  const double y = Y[i];
-  const double t = 1.0 - y * y;
-  double yb = Hb[i];
+  const real y = Y[i];
+  const real t = real(1) - y * y;
+  real yb = Hb[i];
   if (dt) yb *= dt[c];
   if (dual) {
     const size_t j = (size_t)R * d + i;
-    const double yd = Y[j];
-    double ydb = Hb[j];
+    const real yd = Y[j];
+    real ydb = Hb[j];
     if (dt) ydb *= dt[c];
-    Zb[i] = t * yb - 2.0 * y * yd * ydb;
+    Zb[i] = t * yb - real(2) * y * yd * ydb;
     Zb[j] = t * ydb;
   } else {
     Zb[i] = t * yb;
@@ -214,24 +216,24 @@ __global__ void act_bwd_kernel(long long R, int d, const double* __restrict__ Y,
 }
 
 // embedding (compacted rows; tangent rows via tpos)
-__global__ void emb_act_bwd_kernel(int Rmax, const int* __restrict__ Rdev, int d, const double* __restrict__ Y,
-                                   const double* __restrict__ Hb, const int* __restrict__ tpos,
-                                   const double* __restrict__ Yt, const double* __restrict__ Hbt, int dual,
-                                   double* __restrict__ Zb, double* __restrict__ Zbt) {
+__global__ void emb_act_bwd_kernel(int Rmax, const int* __restrict__ Rdev, int d, const real* __restrict__ Y,
+                                   const real* __restrict__ Hb, const int* __restrict__ tpos,
+                                   const real* __restrict__ Yt, const real* __restrict__ Hbt, int dual,
+                                   real* __restrict__ Zb, real* __restrict__ Zbt) {
   const long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x;
   const long long R = min(Rmax, *Rdev);
   if (i >= R * d) return;
   const long long r = i / d;
   const int c = (int)(i % d);
-  const double y = Y[i];
-  const double t = 1.0 - y * y;
-  double z = t * Hb[i];
+  const real y = Y[i];
+  const real t = real(1) - y * y;
+  real z = t * Hb[i];
   if (dual) {
     const int tr = tpos[r];
     if (tr >= 0) {
       const size_t j = (size_t)tr * d + c;
-      const double ydb = Hbt[j];
-      z -= 2.0 * y * Yt[j] * ydb;
+      const real ydb = Hbt[j];
+      z -= real(2) * y * Yt[j] * ydb;
       Zbt[j] = t * ydb;
     }
   }
@@ -242,25 +244,25 @@ __global__ void emb_act_bwd_kernel(int Rmax, const int* __restrict__ Rdev, int d
 //   dt[c] = sum_r y[r][c] hbar[r][c] + sum_r ydot[r][c] hdotbar[r][c]   (h = skip + dt * y)
 // block b: rows [b chunk, (b+1) chunk) of the primal half (and the same rows of the tangent half), one
 // thread per column (coalesced rows); the per-block sums go to ws[b][c] and colsum_reduce adds them.
-__global__ void act_bwd_dt_kernel(long long R, int d, const double* __restrict__ Y, const double* __restrict__ Hb,
-                                  const double* __restrict__ dt, int dual, double* __restrict__ Zb, int chunk,
-                                  double* __restrict__ ws) {
+__global__ void act_bwd_dt_kernel(long long R, int d, const real* __restrict__ Y, const real* __restrict__ Hb,
+                                  const real* __restrict__ dt, int dual, real* __restrict__ Zb, int chunk,
+                                  real* __restrict__ ws) {
   const long long r0 = (long long)blockIdx.x * chunk;
   const long long r1 = min(R, r0 + chunk);
   for (int c = threadIdx.x; c < d; c += blockDim.x) {
-    const double dtc = dt[c];
-    double acc = 0.0;
+    const real dtc = dt[c];
+    real acc = 0.0;
 #pragma unroll 4
     for (long long r = r0; r < r1; ++r) {
       const size_t i = (size_t)r * d + c;
-      const double y = Y[i], hb = Hb[i];
-      const double t = 1.0 - y * y;
+      const real y = Y[i], hb = Hb[i];
+      const real t = real(1) - y * y;
       acc += y * hb;
       if (dual) {
         const size_t j = (size_t)R * d + i;
-        const double yd = Y[j], hdb = Hb[j];
-        const double ydb = hdb * dtc;
-        Zb[i] = t * (hb * dtc) - 2.0 * y * yd * ydb;
+        const real yd = Y[j], hdb = Hb[j];
+        const real ydb = hdb * dtc;
+        Zb[i] = t * (hb * dtc) - real(2) * y * yd * ydb;
         Zb[j] = t * ydb;
         acc += yd * hdb;
       } else {
@@ -271,11 +273,11 @@ __global__ void act_bwd_dt_kernel(long long R, int d, const double* __restrict__
   }
 }
 // out[c] = sum_k ws[k][c]: 32 columns x 8 chunk-lanes per CTA, fixed 8-way combine
-__global__ void colsum_reduce_kernel(const double* __restrict__ ws, int nchunk, int d, double* __restrict__ out) {
-  __shared__ double red[8][33];
+__global__ void colsum_reduce_kernel(const real* __restrict__ ws, int nchunk, int d, double* __restrict__ out) {
+  __shared__ real red[8][33];
   const int cl = threadIdx.x & 31, z = threadIdx.x >> 5;
   const int c = blockIdx.x * 32 + cl;
-  double a = 0.0;
+  real a = 0.0;
   if (c < d) {
 #pragma unroll 4
     for (int k = z; k < nchunk; k += 8) a += ws[(size_t)k * d + c];
@@ -283,21 +285,21 @@ __global__ void colsum_reduce_kernel(const double* __restrict__ ws, int nchunk, 
   red[z][cl] = a;
   __syncthreads();
   if (z == 0 && c < d) {
-    double t = red[0][cl];
+    real t = red[0][cl];
 #pragma unroll
     for (int q = 1; q < 8; ++q) t += red[q][cl];
     out[c] = t;
   }
 }
-static fekf_status act_bwd_dt(Ctx& c, long long R, int d, const double* Y, const double* Hb, const double* dt,
-                              bool dual, double* Zb, double* gdt, cudaStream_t s) {
+static fekf_status act_bwd_dt(Ctx& c, long long R, int d, const real* Y, const real* Hb, const real* dt,
+                              bool dual, real* Zb, double* gdt, cudaStream_t s) {
   const int chunk = (int)std::max<long long>(4, cdiv(R, 2 * 148));
   const int nchunk = (int)cdiv(R, chunk);
   if ((size_t)nchunk * d > c.colsum_elems) { set_error("colsum workspace too small"); return FEKF_EINVAL; }
   act_bwd_dt_kernel<<<nchunk, std::min(256, (d + 31) / 32 * 32), 0, s>>>(R, d, Y, Hb, dt, dual ? 1 : 0, Zb, chunk,
-                                                                         c.colsum_ws.as<double>());
+                                                                         c.colsum_ws.as<real>());
   FEKF_LAUNCH_CHECK();
-  colsum_reduce_kernel<<<cdiv(d, 32), 256, 0, s>>>(c.colsum_ws.as<double>(), nchunk, d, gdt);
+  colsum_reduce_kernel<<<cdiv(d, 32), 256, 0, s>>>(c.colsum_ws.as<real>(), nchunk, d, gdt);
   FEKF_LAUNCH_CHECK();
   count_launch(2);
   return FEKF_OK;
@@ -316,18 +318,18 @@ struct Geo {
   const int* atoms_off;  // [nt+1]
 };
 struct PairPtrs {
-  const double* G[NP];       // primal H_last (G)
-  const double* Gt[NP];      // tangent H_last (Gdot)
+  const real* G[NP];       // primal H_last (G)
+  const real* Gt[NP];      // tangent H_last (Gdot)
   const int* row_start[NP];
   const int* row_idx[NP];
   const int* tpos[NP];
-  const double* sbar[NP];
+  const real* sbar[NP];
 };
 struct FitPtrs {
-  double* D[FEKF_MAX_TYPES];
-  const double* Db[FEKF_MAX_TYPES];
-  double* eout[FEKF_MAX_TYPES];
-  double* ebar[FEKF_MAX_TYPES];
+  real* D[FEKF_MAX_TYPES];
+  const real* Db[FEKF_MAX_TYPES];
+  real* eout[FEKF_MAX_TYPES];
+  real* ebar[FEKF_MAX_TYPES];
   long long F[FEKF_MAX_TYPES];
 };
 
@@ -356,19 +358,19 @@ static const int* tcount(Ctx& c, int p) { return c.rowcnt.as<int>() + c.pairs.si
 // Three passes (chunk counts, chunk scan, scatter), chunks of 1024 rows, order = primal order.
 constexpr int TCHUNK = 1024;
 __device__ __forceinline__ bool row_active(int r, int Na, int Nm, const int* __restrict__ row_idx,
-                                           const int* __restrict__ nl_j, const double* __restrict__ v) {
+                                           const int* __restrict__ nl_j, const real* __restrict__ v) {
   const int idx = row_idx[r];
   const int atom = idx / Nm;
   const int b = atom / Na;
   const int j = nl_j[idx];
-  const double* vi = v + (size_t)atom * 3;
-  const double* vj = v + ((size_t)b * Na + j) * 3;
+  const real* vi = v + (size_t)atom * 3;
+  const real* vj = v + ((size_t)b * Na + j) * 3;
   return vi[0] != 0.0 || vi[1] != 0.0 || vi[2] != 0.0 || vj[0] != 0.0 || vj[1] != 0.0 || vj[2] != 0.0;
 }
 // every pair in one launch per pass (blockIdx.y = pair; chunks past a pair's extent exit)
 struct TrowArgs {
   int Na, Nm;
-  const int* nl_j; const double* v;
+  const int* nl_j; const real* v;
   int Rmax[NP];
   const int* Rdev[NP];
   const int* row_idx[NP];
@@ -448,7 +450,7 @@ __global__ void __launch_bounds__(TCHUNK) tscatter_kernel(const __grid_constant_
 
 // embedding input s (primal rows) or s-dot (tangent rows) = column 0 of R~ / R~-dot
 __global__ void emb_input_kernel(int Rmax, const int* __restrict__ Rdev, const int* __restrict__ row_idx,
-                                 const int* __restrict__ tidx, const double* __restrict__ src, double* __restrict__ out) {
+                                 const int* __restrict__ tidx, const real* __restrict__ src, real* __restrict__ out) {
   const int r = blockIdx.x * blockDim.x + threadIdx.x;
   if (r >= min(Rmax, *Rdev)) return;
   const int pr = tidx ? tidx[r] : r;
@@ -456,22 +458,22 @@ __global__ void emb_input_kernel(int Rmax, const int* __restrict__ Rdev, const i
 }
 
 // embedding layer 0 (input width 1): y = tanh(s W0 + b0), h = y;  tangent: ydot = (1 - y^2) sdot W0
-__global__ void emb_l0_kernel(int Rmax, const int* __restrict__ Rdev, int d, const double* __restrict__ s,
-                              const double* __restrict__ W, const double* __restrict__ bias,
-                              const double* __restrict__ Yprim, const int* __restrict__ rowmap, double* __restrict__ Y,
-                              double* __restrict__ H) {
+__global__ void emb_l0_kernel(int Rmax, const int* __restrict__ Rdev, int d, const real* __restrict__ s,
+                              const real* __restrict__ W, const real* __restrict__ bias,
+                              const real* __restrict__ Yprim, const int* __restrict__ rowmap, real* __restrict__ Y,
+                              real* __restrict__ H) {
   const long long e = (long long)blockIdx.x * blockDim.x + threadIdx.x;
   const long long R = min(Rmax, *Rdev);
   if (e >= R * d) return;
   const long long r = e / d;
   const int c = (int)(e % d);
-  const double z = s[r] * W[c];
-  double y;
+  const real z = s[r] * W[c];
+  real y;
   if (Yprim == nullptr) {
-    y = tanh_fp64(z + bias[c]);
+    y = tanh_r(z + bias[c]);
   } else {
-    const double yp = Yprim[(size_t)rowmap[r] * d + c];
-    y = (1.0 - yp * yp) * z;
+    const real yp = Yprim[(size_t)rowmap[r] * d + c];
+    y = (real(1) - yp * yp) * z;
   }
   Y[e] = y;
   H[e] = y;
@@ -485,55 +487,55 @@ __global__ void emb_l0_kernel(int Rmax, const int* __restrict__ Rdev, int d, con
 constexpr int DESC_THREADS = 256, DESC_MC = 4;   // columns per lane: M <= 128
 __global__ void __launch_bounds__(DESC_THREADS, 4)
 desc_fwd_kernel(const __grid_constant__ Geo g, const __grid_constant__ PairPtrs pp, const __grid_constant__ FitPtrs fp,
-                const double* __restrict__ em, const double* __restrict__ rdot, int tangent, double* __restrict__ X,
-                double* __restrict__ Xd) {
-  extern __shared__ double sm[];
+                const real* __restrict__ em, const real* __restrict__ rdot, int tangent, real* __restrict__ X,
+                real* __restrict__ Xd) {
+  extern __shared__ real sm[];
   const int M = g.M, M2 = g.M2, Nm = g.Nm;
-  double* xs = sm;            // [4][M]
-  double* xds = sm + 4 * M;   // [4][M]
-  double* rs = xds + 4 * M;   // [Nm][4] R~ rows of the atom (contiguous in em)
-  double* rds = rs + 4 * Nm;  // [Nm][4] R~dot rows
-  double* red = rds + 4 * Nm; // [8][4][128] per-warp partial sums of one column chunk
+  real* xs = sm;            // [4][M]
+  real* xds = sm + 4 * M;   // [4][M]
+  real* rs = xds + 4 * M;   // [Nm][4] R~ rows of the atom (contiguous in em)
+  real* rds = rs + 4 * Nm;  // [Nm][4] R~dot rows
+  real* red = rds + 4 * Nm; // [8][4][128] per-warp partial sums of one column chunk
   const int atom = blockIdx.x;
   const int b = atom / g.Na, i = atom % g.Na;
   const int ti = g.types[i], k = g.tindex[i];
   const int e = b * g.ncnt[ti] + k;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   for (int q = threadIdx.x; q < 4 * Nm; q += blockDim.x) {
-    cp_async8(rs + q, em + (size_t)atom * Nm * 4 + q, true);
-    if (tangent) cp_async8(rds + q, rdot + (size_t)atom * Nm * 4 + q, true);
+    cp_async1(rs + q, em + (size_t)atom * Nm * 4 + q, true);
+    if (tangent) cp_async1(rds + q, rdot + (size_t)atom * Nm * 4 + q, true);
   }
   cp_async_commit();
   cp_async_wait<0>();
   __syncthreads();
-  const double inv = 1.0 / g.Nm;
-  double* xw = tangent ? xds : xs;
-  double* xo = (tangent ? Xd : X) + (size_t)atom * 4 * M;
+  const real inv = real(1) / g.Nm;
+  real* xw = tangent ? xds : xs;
+  real* xo = (tangent ? Xd : X) + (size_t)atom * 4 * M;
   for (int m0 = 0; m0 < M; m0 += 32 * DESC_MC) {   // column chunks of 128 (one pass for M <= 128)
-    double acc[DESC_MC][4];
+    real acc[DESC_MC][4];
 #pragma unroll
     for (int c = 0; c < DESC_MC; ++c) acc[c][0] = acc[c][1] = acc[c][2] = acc[c][3] = 0.0;
     for (int tj = 0; tj < g.nt; ++tj) {
       const int p = ti * g.nt + tj;
       const int r0 = pp.row_start[p][e], r1 = pp.row_start[p][e + 1];
-      const double* er = rs + 4 * g.sec[tj];
-      const double* ed = rds + 4 * g.sec[tj];
+      const real* er = rs + 4 * g.sec[tj];
+      const real* ed = rds + 4 * g.sec[tj];
       constexpr int RS = DESC_THREADS / 32;
       if (!tangent) {   // two rows per iteration: 8 loads in flight per lane
-        const double* Gp = pp.G[p];
+        const real* Gp = pp.G[p];
         int r = r0 + warp;
         for (; r + RS < r1; r += 2 * RS) {
-          double gv[2][DESC_MC];
+          real gv[2][DESC_MC];
 #pragma unroll
           for (int u = 0; u < 2; ++u)
 #pragma unroll
             for (int c = 0; c < DESC_MC; ++c) {
               const int m = m0 + lane + 32 * c;
-              gv[u][c] = m < M ? Gp[(size_t)(r + u * RS) * M + m] : 0.0;
+              gv[u][c] = m < M ? Gp[(size_t)(r + u * RS) * M + m] : real(0);
             }
 #pragma unroll
           for (int u = 0; u < 2; ++u) {
-            const double* q = er + 4 * (r + u * RS - r0);
+            const real* q = er + 4 * (r + u * RS - r0);
 #pragma unroll
             for (int c = 0; c < DESC_MC; ++c)
 #pragma unroll
@@ -541,12 +543,12 @@ desc_fwd_kernel(const __grid_constant__ Geo g, const __grid_constant__ PairPtrs 
           }
         }
         if (r < r1) {
-          const double* q = er + 4 * (r - r0);
-          double gv[DESC_MC];
+          const real* q = er + 4 * (r - r0);
+          real gv[DESC_MC];
 #pragma unroll
           for (int c = 0; c < DESC_MC; ++c) {
             const int m = m0 + lane + 32 * c;
-            gv[c] = m < M ? Gp[(size_t)r * M + m] : 0.0;
+            gv[c] = m < M ? Gp[(size_t)r * M + m] : real(0);
           }
 #pragma unroll
           for (int c = 0; c < DESC_MC; ++c)
@@ -566,14 +568,14 @@ desc_fwd_kernel(const __grid_constant__ Geo g, const __grid_constant__ PairPtrs 
           act &= act - 1;
           const int r = base + RS * j;
           const int t = __shfl_sync(0xffffffffu, tl, j);
-          const double* q = er + 4 * (r - r0);
-          const double* qd = ed + 4 * (r - r0);
-          double gv[DESC_MC], gd[DESC_MC];
+          const real* q = er + 4 * (r - r0);
+          const real* qd = ed + 4 * (r - r0);
+          real gv[DESC_MC], gd[DESC_MC];
 #pragma unroll
           for (int c = 0; c < DESC_MC; ++c) {
             const int m = m0 + lane + 32 * c;
-            gv[c] = m < M ? pp.G[p][(size_t)r * M + m] : 0.0;
-            gd[c] = m < M ? pp.Gt[p][(size_t)t * M + m] : 0.0;
+            gv[c] = m < M ? pp.G[p][(size_t)r * M + m] : real(0);
+            gd[c] = m < M ? pp.Gt[p][(size_t)t * M + m] : real(0);
           }
 #pragma unroll
           for (int c = 0; c < DESC_MC; ++c)
@@ -590,7 +592,7 @@ desc_fwd_kernel(const __grid_constant__ Geo g, const __grid_constant__ PairPtrs 
     for (int q = threadIdx.x; q < 4 * 32 * DESC_MC; q += blockDim.x) {
       const int a = q / (32 * DESC_MC), m = m0 + q % (32 * DESC_MC);
       if (m >= M) continue;
-      double v = 0.0;
+      real v = 0.0;
 #pragma unroll
       for (int w = 0; w < DESC_THREADS / 32; ++w) v += red[(w * 4 + a) * (32 * DESC_MC) + q % (32 * DESC_MC)];
       xw[a * M + m] = v * inv;
@@ -599,15 +601,15 @@ desc_fwd_kernel(const __grid_constant__ Geo g, const __grid_constant__ PairPtrs 
     __syncthreads();
   }
   if (tangent) {
-    const double* xp = X + (size_t)atom * 4 * M;
+    const real* xp = X + (size_t)atom * 4 * M;
     for (int q = threadIdx.x; q < 4 * M; q += blockDim.x) xs[q] = xp[q];
   }
   __syncthreads();
   const long long row = (long long)b * g.ncnt[ti] + k;
-  double* D = fp.D[ti] + (size_t)(tangent ? fp.F[ti] + row : row) * M * M2;
+  real* D = fp.D[ti] + (size_t)(tangent ? fp.F[ti] + row : row) * M * M2;
   for (int q = threadIdx.x; q < M * M2; q += blockDim.x) {
     const int m = q / M2, n = q % M2;
-    double v;
+    real v;
     if (!tangent) {
       v = xs[m] * xs[n] + xs[M + m] * xs[M + n] + xs[2 * M + m] * xs[2 * M + n] + xs[3 * M + m] * xs[3 * M + n];
     } else {
@@ -621,20 +623,20 @@ desc_fwd_kernel(const __grid_constant__ Geo g, const __grid_constant__ PairPtrs 
 
 // Eq. 4: dE/dX = X^< Dbar^T + [X Dbar into the first M^< columns].
 //   Xbar = B(X, Dbar) + B(Xdot, Ddotbar) ; Xdotbar = B(X, Ddotbar)   (dual)
-__global__ void desc_bwd_kernel(Geo g, FitPtrs fp, const double* __restrict__ X, const double* __restrict__ Xd, int dual,
-                                double* __restrict__ Xb, double* __restrict__ Xdb) {
-  extern __shared__ double sm[];
+__global__ void desc_bwd_kernel(Geo g, FitPtrs fp, const real* __restrict__ X, const real* __restrict__ Xd, int dual,
+                                real* __restrict__ Xb, real* __restrict__ Xdb) {
+  extern __shared__ real sm[];
   const int M = g.M, M2 = g.M2;
-  double* xs = sm;
-  double* xds = xs + 4 * M;
-  double* db = xds + 4 * M;
-  double* ddb = db + M * (M2 + 1);
+  real* xs = sm;
+  real* xds = xs + 4 * M;
+  real* db = xds + 4 * M;
+  real* ddb = db + M * (M2 + 1);
   const int atom = blockIdx.x;
   const int b = atom / g.Na, i = atom % g.Na;
   const int ti = g.types[i], k = g.tindex[i];
   const long long row = (long long)b * g.ncnt[ti] + k;
-  const double* Dbp = fp.Db[ti] + (size_t)row * M * M2;
-  const double* Ddbp = fp.Db[ti] + (size_t)(fp.F[ti] + row) * M * M2;
+  const real* Dbp = fp.Db[ti] + (size_t)row * M * M2;
+  const real* Ddbp = fp.Db[ti] + (size_t)(fp.F[ti] + row) * M * M2;
   for (int e = threadIdx.x; e < 4 * M; e += blockDim.x) {
     xs[e] = X[(size_t)atom * 4 * M + e];
     if (dual) xds[e] = Xd[(size_t)atom * 4 * M + e];
@@ -647,13 +649,13 @@ __global__ void desc_bwd_kernel(Geo g, FitPtrs fp, const double* __restrict__ X,
   __syncthreads();
   for (int e = threadIdx.x; e < 4 * M; e += blockDim.x) {
     const int kk = e / M, p = e % M;
-    const double* x = xs + kk * M;
-    double a = 0.0, ad = 0.0;
+    const real* x = xs + kk * M;
+    real a = 0.0, ad = 0.0;
     for (int n = 0; n < M2; ++n) a = fma(db[p * (M2 + 1) + n], x[n], a);
     if (p < M2)
       for (int m = 0; m < M; ++m) a = fma(db[m * (M2 + 1) + p], x[m], a);
     if (dual) {
-      const double* xd = xds + kk * M;
+      const real* xd = xds + kk * M;
       for (int n = 0; n < M2; ++n) { a = fma(ddb[p * (M2 + 1) + n], xd[n], a); ad = fma(ddb[p * (M2 + 1) + n], x[n], ad); }
       if (p < M2)
         for (int m = 0; m < M; ++m) { a = fma(ddb[m * (M2 + 1) + p], xd[m], a); ad = fma(ddb[m * (M2 + 1) + p], x[m], ad); }
@@ -669,46 +671,46 @@ __global__ void desc_bwd_kernel(Geo g, FitPtrs fp, const double* __restrict__ X,
 //   dR_r = G_r Xbar^T / N_m                             (forces: the R~ adjoint less sbar e_0)
 // One CTA (8 warps) per centre atom; the atom's R~ (and R~dot) rows are contiguous and staged once.
 struct SeedOut {
-  double* gbar[NP];
-  double* hbt[NP];
-  double* dr[NP];
+  real* gbar[NP];
+  real* hbt[NP];
+  real* dr[NP];
 };
 template <bool dual, bool force, bool sel>
 __global__ void __launch_bounds__(256, dual ? 2 : 4)
 desc_bwd_seed_kernel(const __grid_constant__ Geo g, const __grid_constant__ FitPtrs fp,
                      const __grid_constant__ PairPtrs pp, const __grid_constant__ SeedOut so,
-                     const double* __restrict__ X, const double* __restrict__ Xd, const double* __restrict__ em,
-                     const double* __restrict__ rdot, double* __restrict__ Xb, double* __restrict__ Xdb) {
-  extern __shared__ double sm[];
+                     const real* __restrict__ X, const real* __restrict__ Xd, const real* __restrict__ em,
+                     const real* __restrict__ rdot, real* __restrict__ Xb, real* __restrict__ Xdb) {
+  extern __shared__ real sm[];
   const int M = g.M, M2 = g.M2, Nm = g.Nm;
-  double* xs = sm;               // [4][M]
-  double* xds = xs + 4 * M;      // [4][M]
-  double* db = xds + 4 * M;      // [M][M2 + 1]
-  double* ddb = db + M * (M2 + 1);  // [M][M2 + 1]
-  double* xbs = ddb + M * (M2 + 1);  // [4][M]  Xbar
-  double* xdbs = xbs + 4 * M;    // [4][M]  Xdotbar
-  double* rs = xdbs + 4 * M;     // [Nm][4] R~ rows of the atom
-  double* rds = rs + 4 * Nm;     // [Nm][4] R~dot rows
+  real* xs = sm;               // [4][M]
+  real* xds = xs + 4 * M;      // [4][M]
+  real* db = xds + 4 * M;      // [M][M2 + 1]
+  real* ddb = db + M * (M2 + 1);  // [M][M2 + 1]
+  real* xbs = ddb + M * (M2 + 1);  // [4][M]  Xbar
+  real* xdbs = xbs + 4 * M;    // [4][M]  Xdotbar
+  real* rs = xdbs + 4 * M;     // [Nm][4] R~ rows of the atom
+  real* rds = rs + 4 * Nm;     // [Nm][4] R~dot rows
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   const int atom = blockIdx.x;
   const int b = atom / g.Na, i = atom % g.Na;
   const int ti = g.types[i], k = g.tindex[i];
   const long long row = (long long)b * g.ncnt[ti] + k;
-  const double* Dbp = fp.Db[ti] + (size_t)row * M * M2;
-  const double* Ddbp = fp.Db[ti] + (size_t)(fp.F[ti] + row) * M * M2;
+  const real* Dbp = fp.Db[ti] + (size_t)row * M * M2;
+  const real* Ddbp = fp.Db[ti] + (size_t)(fp.F[ti] + row) * M * M2;
   // staging with cp.async: every copy of the CTA in flight at once (no per-element load -> store latency)
   for (int e = tid; e < 4 * M; e += blockDim.x) {
-    cp_async8(xs + e, X + (size_t)atom * 4 * M + e, true);
-    if (dual) cp_async8(xds + e, Xd + (size_t)atom * 4 * M + e, true);
+    cp_async1(xs + e, X + (size_t)atom * 4 * M + e, true);
+    if (dual) cp_async1(xds + e, Xd + (size_t)atom * 4 * M + e, true);
   }
   for (int e = tid; e < M * M2; e += blockDim.x) {
     const int ep = (e / M2) * (M2 + 1) + e % M2;  // row stride M2 + 1: conflict-free in both loops below
-    cp_async8(db + ep, Dbp + e, true);
-    if (dual) cp_async8(ddb + ep, Ddbp + e, true);
+    cp_async1(db + ep, Dbp + e, true);
+    if (dual) cp_async1(ddb + ep, Ddbp + e, true);
   }
   for (int e = tid; e < 4 * Nm; e += blockDim.x) {
-    cp_async8(rs + e, em + (size_t)atom * Nm * 4 + e, true);
-    if (dual) cp_async8(rds + e, rdot + (size_t)atom * Nm * 4 + e, true);
+    cp_async1(rs + e, em + (size_t)atom * Nm * 4 + e, true);
+    if (dual) cp_async1(rds + e, rdot + (size_t)atom * Nm * 4 + e, true);
   }
   cp_async_commit();
   cp_async_wait<0>();
@@ -721,9 +723,9 @@ desc_bwd_seed_kernel(const __grid_constant__ Geo g, const __grid_constant__ FitP
     for (int o = tid >> 2; o < no8; o += blockDim.x >> 2) {
       const bool valid = o < no;
       const int kk = valid ? o / M2 : 0, p = valid ? o % M2 : 0;
-      const double* x = xs + kk * M;
-      const double* xd = xds + kk * M;
-      double a = 0.0, ad = 0.0;
+      const real* x = xs + kk * M;
+      const real* xd = xds + kk * M;
+      real a = 0.0, ad = 0.0;
       for (int m = part; valid && m < M; m += 4) {
         a = fma(db[m * (M2 + 1) + p], x[m], a);
         if (dual) {
@@ -744,11 +746,11 @@ desc_bwd_seed_kernel(const __grid_constant__ Geo g, const __grid_constant__ FitP
   __syncthreads();
   for (int e = tid; e < 4 * M; e += blockDim.x) {
     const int kk = e / M, p = e % M;
-    const double* x = xs + kk * M;
-    double a = p < M2 ? xbs[e] : 0.0, ad = (dual && p < M2) ? xdbs[e] : 0.0;
+    const real* x = xs + kk * M;
+    real a = p < M2 ? xbs[e] : real(0), ad = (dual && p < M2) ? xdbs[e] : real(0);
     for (int n = 0; n < M2; ++n) a = fma(db[p * (M2 + 1) + n], x[n], a);
     if (dual) {
-      const double* xd = xds + kk * M;
+      const real* xd = xds + kk * M;
       for (int n = 0; n < M2; ++n) { a = fma(ddb[p * (M2 + 1) + n], xd[n], a); ad = fma(ddb[p * (M2 + 1) + n], x[n], ad); }
     }
     Xb[(size_t)atom * 4 * M + e] = a;
@@ -760,49 +762,49 @@ desc_bwd_seed_kernel(const __grid_constant__ Geo g, const __grid_constant__ FitP
     if (dual) xdbs[e] = Xdb[(size_t)atom * 4 * M + e];
   }
   __syncthreads();
-  const double inv = 1.0 / Nm;
+  const real inv = real(1) / Nm;
   const int e0 = b * g.ncnt[ti] + k;
   // per row: Gbar = (R~ Xbar [+ R~dot Xdotbar]) / N_m, [Hdotbar = R~ Xdotbar / N_m on tangent rows],
   // [dR = G Xbar^T / N_m]; the lane's Xbar (Xdotbar) columns m = m0 + lane + 32 u stay in registers
   for (int m0 = 0; m0 < M; m0 += 128) {
-    double xb[4][4], xdb[4][4];
+    real xb[4][4], xdb[4][4];
 #pragma unroll
     for (int u = 0; u < 4; ++u) {
       const int m = m0 + lane + 32 * u;
 #pragma unroll
       for (int a = 0; a < 4; ++a) {
-        xb[u][a] = m < M ? xbs[a * M + m] : 0.0;
-        xdb[u][a] = (dual && m < M) ? xdbs[a * M + m] : 0.0;
+        xb[u][a] = m < M ? xbs[a * M + m] : real(0);
+        xdb[u][a] = (dual && m < M) ? xdbs[a * M + m] : real(0);
       }
     }
     for (int tj = 0; tj < g.nt; ++tj) {
       const int p = ti * g.nt + tj;
       const int r0 = pp.row_start[p][e0], nr = pp.row_start[p][e0 + 1] - r0;
       const int* __restrict__ tpos = pp.tpos[p];
-      double* __restrict__ gbar = so.gbar[p];
-      double* __restrict__ hbt = so.hbt[p];
-      double* __restrict__ dr = so.dr[p];
-      const double* __restrict__ Gp = pp.G[p];
-      const double* rsj = rs + g.sec[tj] * 4;
-      const double* rdsj = rds + g.sec[tj] * 4;
+      real* __restrict__ gbar = so.gbar[p];
+      real* __restrict__ hbt = so.hbt[p];
+      real* __restrict__ dr = so.dr[p];
+      const real* __restrict__ Gp = pp.G[p];
+      const real* rsj = rs + g.sec[tj] * 4;
+      const real* rdsj = rds + g.sec[tj] * 4;
       auto row_body = [&](int s_, int t) {
         const int r = r0 + s_;
-        const double* q = rsj + s_ * 4;
-        const double q0 = q[0], q1 = q[1], q2 = q[2], q3 = q[3];
-        double d0 = 0.0, d1 = 0.0, d2 = 0.0, d3 = 0.0;
-        if (dual && t >= 0) { const double* qd = rdsj + s_ * 4; d0 = qd[0]; d1 = qd[1]; d2 = qd[2]; d3 = qd[3]; }
-        double gv[4];
+        const real* q = rsj + s_ * 4;
+        const real q0 = q[0], q1 = q[1], q2 = q[2], q3 = q[3];
+        real d0 = 0.0, d1 = 0.0, d2 = 0.0, d3 = 0.0;
+        if (dual && t >= 0) { const real* qd = rdsj + s_ * 4; d0 = qd[0]; d1 = qd[1]; d2 = qd[2]; d3 = qd[3]; }
+        real gv[4];
 #pragma unroll
         for (int u = 0; u < 4; ++u) {
           const int m = m0 + lane + 32 * u;
-          gv[u] = (force && m < M) ? Gp[(size_t)r * M + m] : 0.0;
+          gv[u] = (force && m < M) ? Gp[(size_t)r * M + m] : real(0);
         }
-        double pk0 = 0.0, pk1 = 0.0, pk2 = 0.0, pk3 = 0.0;
+        real pk0 = 0.0, pk1 = 0.0, pk2 = 0.0, pk3 = 0.0;
 #pragma unroll
         for (int u = 0; u < 4; ++u) {
           const int m = m0 + lane + 32 * u;
           if (m >= M) continue;
-          double v = q0 * xb[u][0] + q1 * xb[u][1] + q2 * xb[u][2] + q3 * xb[u][3];
+          real v = q0 * xb[u][0] + q1 * xb[u][1] + q2 * xb[u][2] + q3 * xb[u][3];
           if (dual && t >= 0) {
             v += d0 * xdb[u][0] + d1 * xdb[u][1] + d2 * xdb[u][2] + d3 * xdb[u][3];
             hbt[(size_t)t * M + m] = (q0 * xdb[u][0] + q1 * xdb[u][1] + q2 * xdb[u][2] + q3 * xdb[u][3]) * inv;
@@ -823,7 +825,7 @@ desc_bwd_seed_kernel(const __grid_constant__ Geo g, const __grid_constant__ FitP
             pk3 += __shfl_xor_sync(0xffffffffu, pk3, o);
           }
           if (lane < 4) {
-            const double pv = lane == 0 ? pk0 : lane == 1 ? pk1 : lane == 2 ? pk2 : pk3;
+            const real pv = lane == 0 ? pk0 : lane == 1 ? pk1 : lane == 2 ? pk2 : pk3;
             if (m0 == 0) dr[(size_t)r * 4 + lane] = pv * inv;
             else dr[(size_t)r * 4 + lane] += pv * inv;
           }
@@ -856,10 +858,10 @@ desc_bwd_seed_kernel(const __grid_constant__ Geo g, const __grid_constant__ FitP
 //   zbar = (1 - y^2) Gbar - 2 y ydot Gdotbar ; zdotbar = (1 - y^2) Gdotbar
 __global__ void emb_seed_kernel(int Rmax, const int* __restrict__ Rdev, int M, int Nm,
                                 const int* __restrict__ row_idx, const int* __restrict__ tpos,
-                                const double* __restrict__ em, const double* __restrict__ rdot,
-                                const double* __restrict__ Xb, const double* __restrict__ Xdb, int dual,
-                                const double* __restrict__ Y, const double* __restrict__ Yt, double* __restrict__ Hb,
-                                double* __restrict__ Zb, double* __restrict__ Hbt, double* __restrict__ Zbt) {
+                                const real* __restrict__ em, const real* __restrict__ rdot,
+                                const real* __restrict__ Xb, const real* __restrict__ Xdb, int dual,
+                                const real* __restrict__ Y, const real* __restrict__ Yt, real* __restrict__ Hb,
+                                real* __restrict__ Zb, real* __restrict__ Hbt, real* __restrict__ Zbt) {
   const long long e = (long long)blockIdx.x * blockDim.x + threadIdx.x;
   const long long R = min(Rmax, *Rdev);
   if (e >= R * M) return;
@@ -867,25 +869,25 @@ __global__ void emb_seed_kernel(int Rmax, const int* __restrict__ Rdev, int M, i
   const int m = (int)(e % M);
   const size_t idx = (size_t)row_idx[r];
   const size_t atom = idx / Nm;
-  const double* xb = Xb + atom * 4 * M;
-  const double* rr = em + idx * 4;
-  double a = rr[0] * xb[m] + rr[1] * xb[M + m] + rr[2] * xb[2 * M + m] + rr[3] * xb[3 * M + m];
-  const double inv = 1.0 / Nm;
+  const real* xb = Xb + atom * 4 * M;
+  const real* rr = em + idx * 4;
+  real a = rr[0] * xb[m] + rr[1] * xb[M + m] + rr[2] * xb[2 * M + m] + rr[3] * xb[3 * M + m];
+  const real inv = real(1) / Nm;
   const size_t o = (size_t)r * M + m;
-  const double y = Y[o];
-  const double t = 1.0 - y * y;
+  const real y = Y[o];
+  const real t = real(1) - y * y;
   const int tr = dual ? tpos[r] : -1;
   if (tr >= 0) {
-    const double* xdb = Xdb + atom * 4 * M;
-    const double* rd = rdot + idx * 4;
+    const real* xdb = Xdb + atom * 4 * M;
+    const real* rd = rdot + idx * 4;
     a += rd[0] * xdb[m] + rd[1] * xdb[M + m] + rd[2] * xdb[2 * M + m] + rd[3] * xdb[3 * M + m];
-    const double ad = (rr[0] * xdb[m] + rr[1] * xdb[M + m] + rr[2] * xdb[2 * M + m] + rr[3] * xdb[3 * M + m]) * inv;
+    const real ad = (rr[0] * xdb[m] + rr[1] * xdb[M + m] + rr[2] * xdb[2 * M + m] + rr[3] * xdb[3 * M + m]) * inv;
     const size_t od = (size_t)tr * M + m;
     Hbt[od] = ad;
     Zbt[od] = t * ad;
     a *= inv;
     Hb[o] = a;
-    Zb[o] = t * a - 2.0 * y * Yt[od] * ad;
+    Zb[o] = t * a - real(2) * y * Yt[od] * ad;
   } else {
     a *= inv;
     Hb[o] = a;
@@ -896,20 +898,20 @@ __global__ void emb_seed_kernel(int Rmax, const int* __restrict__ Rdev, int M, i
 // Same as emb_seed_kernel, one CTA per centre atom for all its rows of every pair: the atom's Xbar
 // (and Xdotbar) are staged once in SMEM instead of being re-read for every (row, m).
 struct SeedPtrs {
-  const double* Y[NP];
-  const double* Yt[NP];
-  double* Hb[NP];
-  double* Zb[NP];
-  double* Hbt[NP];
-  double* Zbt[NP];
+  const real* Y[NP];
+  const real* Yt[NP];
+  real* Hb[NP];
+  real* Zb[NP];
+  real* Hbt[NP];
+  real* Zbt[NP];
 };
 __global__ void __launch_bounds__(128)
-emb_seed_atom_kernel(Geo g, PairPtrs pp, SeedPtrs sp, const double* __restrict__ em, const double* __restrict__ rdot,
-                     const double* __restrict__ Xb, const double* __restrict__ Xdb, int dual) {
-  extern __shared__ double sm[];
+emb_seed_atom_kernel(Geo g, PairPtrs pp, SeedPtrs sp, const real* __restrict__ em, const real* __restrict__ rdot,
+                     const real* __restrict__ Xb, const real* __restrict__ Xdb, int dual) {
+  extern __shared__ real sm[];
   const int M = g.M;
-  double* xb = sm;
-  double* xdb = sm + 4 * M;
+  real* xb = sm;
+  real* xdb = sm + 4 * M;
   const int atom = blockIdx.x;
   const int b = atom / g.Na, i = atom % g.Na;
   const int ti = g.types[i], k = g.tindex[i];
@@ -919,7 +921,7 @@ emb_seed_atom_kernel(Geo g, PairPtrs pp, SeedPtrs sp, const double* __restrict__
     if (dual) xdb[q] = Xdb[(size_t)atom * 4 * M + q];
   }
   __syncthreads();
-  const double inv = 1.0 / g.Nm;
+  const real inv = real(1) / g.Nm;
   for (int tj = 0; tj < g.nt; ++tj) {
     const int p = ti * g.nt + tj;
     const int r0 = pp.row_start[p][e], r1 = pp.row_start[p][e + 1];
@@ -928,22 +930,22 @@ emb_seed_atom_kernel(Geo g, PairPtrs pp, SeedPtrs sp, const double* __restrict__
       const int s = q / M, m = q % M;
       const int r = r0 + s;
       const size_t idx = (size_t)atom * g.Nm + g.sec[tj] + s;
-      const double* rr = em + idx * 4;
-      double a = rr[0] * xb[m] + rr[1] * xb[M + m] + rr[2] * xb[2 * M + m] + rr[3] * xb[3 * M + m];
+      const real* rr = em + idx * 4;
+      real a = rr[0] * xb[m] + rr[1] * xb[M + m] + rr[2] * xb[2 * M + m] + rr[3] * xb[3 * M + m];
       const size_t o = (size_t)r * M + m;
-      const double y = sp.Y[p][o];
-      const double t = 1.0 - y * y;
+      const real y = sp.Y[p][o];
+      const real t = real(1) - y * y;
       const int tr = dual ? pp.tpos[p][r] : -1;
       if (tr >= 0) {
-        const double* rd = rdot + idx * 4;
+        const real* rd = rdot + idx * 4;
         a += rd[0] * xdb[m] + rd[1] * xdb[M + m] + rd[2] * xdb[2 * M + m] + rd[3] * xdb[3 * M + m];
-        const double ad = (rr[0] * xdb[m] + rr[1] * xdb[M + m] + rr[2] * xdb[2 * M + m] + rr[3] * xdb[3 * M + m]) * inv;
+        const real ad = (rr[0] * xdb[m] + rr[1] * xdb[M + m] + rr[2] * xdb[2 * M + m] + rr[3] * xdb[3 * M + m]) * inv;
         const size_t od = (size_t)tr * M + m;
         sp.Hbt[p][od] = ad;
         sp.Zbt[p][od] = t * ad;
         a *= inv;
         sp.Hb[p][o] = a;
-        sp.Zb[p][o] = t * a - 2.0 * y * sp.Yt[p][od] * ad;
+        sp.Zb[p][o] = t * a - real(2) * y * sp.Yt[p][od] * ad;
       } else {
         a *= inv;
         sp.Hb[p][o] = a;
@@ -956,16 +958,16 @@ emb_seed_atom_kernel(Geo g, PairPtrs pp, SeedPtrs sp, const double* __restrict__
 // prod_force (per-layer embedding path): dE/dR~_row = G Xbar^T / N_m + sbar e_0 ; f = dE/dd = (dE/dR~) J per
 // slot into frow (the forces / virials are gathered by force_gather_kernel).  One CTA (4 warps) per atom.
 __global__ void __launch_bounds__(128)
-prod_force_kernel(Geo g, PairPtrs pp, const double* __restrict__ Xb, const double* __restrict__ jac,
-                  const int* __restrict__ nl_j, double* __restrict__ frow) {
+prod_force_kernel(Geo g, PairPtrs pp, const real* __restrict__ Xb, const real* __restrict__ jac,
+                  const int* __restrict__ nl_j, real* __restrict__ frow) {
   const int atom = blockIdx.x;
   const int b = atom / g.Na, i = atom % g.Na;
   const int ti = g.types[i], k = g.tindex[i];
   const int e = b * g.ncnt[ti] + k;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int M = g.M;
-  const double* xb = Xb + (size_t)atom * 4 * M;
-  const double inv = 1.0 / g.Nm;
+  const real* xb = Xb + (size_t)atom * 4 * M;
+  const real inv = real(1) / g.Nm;
   for (int slot = warp; slot < g.Nm; slot += 4) {
     const size_t idx = (size_t)atom * g.Nm + slot;
     if (nl_j[idx] < 0) continue;
@@ -973,10 +975,10 @@ prod_force_kernel(Geo g, PairPtrs pp, const double* __restrict__ Xb, const doubl
     while (slot >= g.sec[tj + 1]) ++tj;
     const int p = ti * g.nt + tj;
     const long long r = pp.row_start[p][e] + (slot - g.sec[tj]);
-    const double* gr = pp.G[p] + (size_t)r * M;
-    double a0 = 0, a1 = 0, a2 = 0, a3 = 0;
+    const real* gr = pp.G[p] + (size_t)r * M;
+    real a0 = 0, a1 = 0, a2 = 0, a3 = 0;
     for (int m = lane; m < M; m += 32) {
-      const double gv = gr[m];
+      const real gv = gr[m];
       a0 = fma(gv, xb[m], a0); a1 = fma(gv, xb[M + m], a1); a2 = fma(gv, xb[2 * M + m], a2); a3 = fma(gv, xb[3 * M + m], a3);
     }
     for (int o = 16; o > 0; o >>= 1) {
@@ -986,8 +988,8 @@ prod_force_kernel(Geo g, PairPtrs pp, const double* __restrict__ Xb, const doubl
       a3 += __shfl_xor_sync(0xffffffffu, a3, o);
     }
     if (lane < 3) {
-      const double rb0 = a0 * inv + pp.sbar[p][r], rb1 = a1 * inv, rb2 = a2 * inv, rb3 = a3 * inv;
-      const double* J = jac + idx * 12;
+      const real rb0 = a0 * inv + pp.sbar[p][r], rb1 = a1 * inv, rb2 = a2 * inv, rb3 = a3 * inv;
+      const real* J = jac + idx * 12;
       frow[idx * 3 + lane] = rb0 * J[lane] + rb1 * J[3 + lane] + rb2 * J[6 + lane] + rb3 * J[9 + lane];
     }
   }
@@ -1107,22 +1109,22 @@ fekf_status build_reverse(Ctx& c, int nb, cudaStream_t s) {
 // butterfly: deterministic.
 __global__ void __launch_bounds__(256) force_gather_kernel(int nb, int Na, int Nm, const int* __restrict__ sel,
                                                            int n_sel, const int* __restrict__ nl_j,
-                                                           const double* __restrict__ rij,
-                                                           const double* __restrict__ frow,
+                                                           const real* __restrict__ rij,
+                                                           const real* __restrict__ frow,
                                                            const int* __restrict__ off, const int* __restrict__ idx,
                                                            double* __restrict__ force, double* __restrict__ vatom) {
   const int w = blockIdx.x * 8 + (threadIdx.x >> 5), lane = threadIdx.x & 31;
   const int nw = sel ? nb * n_sel : nb * Na;
   if (w >= nw) return;
   const int a = sel ? (w / n_sel) * Na + sel[w % n_sel] : w;
-  double v[12];
+  real v[12];
 #pragma unroll
   for (int q = 0; q < 12; ++q) v[q] = 0.0;
   for (int sl = lane; sl < Nm; sl += 32) {
     const size_t e = (size_t)a * Nm + sl;
     if (nl_j[e] < 0) continue;
-    const double f0 = frow[e * 3], f1 = frow[e * 3 + 1], f2 = frow[e * 3 + 2];
-    const double d0 = rij[e * 3], d1 = rij[e * 3 + 1], d2 = rij[e * 3 + 2];
+    const real f0 = frow[e * 3], f1 = frow[e * 3 + 1], f2 = frow[e * 3 + 2];
+    const real d0 = rij[e * 3], d1 = rij[e * 3 + 1], d2 = rij[e * 3 + 2];
     v[0] += f0; v[1] += f1; v[2] += f2;
     v[3] -= d0 * f0; v[4] -= d0 * f1; v[5] -= d0 * f2;
     v[6] -= d1 * f0; v[7] -= d1 * f1; v[8] -= d1 * f2;
@@ -1140,7 +1142,7 @@ __global__ void __launch_bounds__(256) force_gather_kernel(int nb, int Na, int N
     for (int o = 16; o > 0; o >>= 1) v[q] += __shfl_xor_sync(0xffffffffu, v[q], o);
   if (lane < 3) force[(size_t)a * 3 + lane] = lane == 0 ? v[0] : (lane == 1 ? v[1] : v[2]);
   else if (lane < 12) {
-    double x = 0.0;
+    real x = 0.0;
 #pragma unroll
     for (int q = 3; q < 12; ++q) if (lane == q) x = v[q];
     vatom[(size_t)a * 9 + lane - 3] = x;
@@ -1157,19 +1159,19 @@ __global__ void virial_reduce_kernel(const double* __restrict__ vatom, int Na, d
 }
 
 // E_i = h_F W_out + b_out (primal rows), Edot_i = hdot_F W_out (tangent rows); one warp per row
-__global__ void fit_out_kernel(long long rows, long long F, int h, const double* __restrict__ H,
-                               const double* __restrict__ W, const double* __restrict__ bout, double* __restrict__ out) {
+__global__ void fit_out_kernel(long long rows, long long F, int h, const real* __restrict__ H,
+                               const real* __restrict__ W, const real* __restrict__ bout, real* __restrict__ out) {
   const long long r = ((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const int lane = threadIdx.x & 31;
   if (r >= rows) return;
-  double a = 0.0;
+  real a = 0.0;
   for (int c = lane; c < h; c += 32) a = fma(H[(size_t)r * h + c], W[c], a);
   for (int o = 16; o > 0; o >>= 1) a += __shfl_xor_sync(0xffffffffu, a, o);
-  if (lane == 0) out[r] = a + (r < F ? bout[0] : 0.0);
+  if (lane == 0) out[r] = a + (r < F ? bout[0] : real(0));
 }
 // adjoint of h_F from the output seeds: Hbar = ebar (x) W_out
-__global__ void fit_out_bwd_kernel(long long rows, int h, const double* __restrict__ ebar, const double* __restrict__ W,
-                                   double* __restrict__ Hb) {
+__global__ void fit_out_bwd_kernel(long long rows, int h, const real* __restrict__ ebar, const real* __restrict__ W,
+                                   real* __restrict__ Hb) {
   const long long e = (long long)blockIdx.x * blockDim.x + threadIdx.x;
   if (e >= rows * h) return;
   Hb[e] = ebar[e / h] * W[e % h];
@@ -1203,7 +1205,7 @@ __global__ void energy_error_kernel(Geo g, FitPtrs fp, const double* __restrict_
     const long long F = (long long)g.nb * g.ncnt[t];
     for (long long r = threadIdx.x; r < F; r += blockDim.x) {
       const long long b = r / g.ncnt[t];
-      fp.ebar[t][r] = (etot[b] >= label[b] ? -1.0 : 1.0) * seed_scale / g.Na;
+      fp.ebar[t][r] = (real)((etot[b] >= label[b] ? -1.0 : 1.0) * seed_scale / g.Na);
     }
   }
 }
@@ -1214,7 +1216,7 @@ __global__ void energy_error_kernel(Geo g, FitPtrs fp, const double* __restrict_
 __global__ void __launch_bounds__(1024) force_error_kernel(Geo g, const double* __restrict__ force,
                                                            const double* __restrict__ label,
                                                            const int* __restrict__ atom_idx, int n_sel, double seed,
-                                                           double* __restrict__ v, FitPtrs fp,
+                                                           real* __restrict__ v, FitPtrs fp,
                                                            double* __restrict__ abs_sum) {
   __shared__ double red[1024];
   for (long long e = threadIdx.x; e < (long long)g.nb * g.Na * 3; e += blockDim.x) v[e] = 0.0;
@@ -1228,7 +1230,7 @@ __global__ void __launch_bounds__(1024) force_error_kernel(Geo g, const double* 
     const size_t o = ((size_t)b * g.Na + atom_idx[q]) * 3 + al;
     const double fpred = force[o], fl = label[o];
     a += fabs(fl - fpred);
-    atomicAdd(v + o, fpred >= fl ? -1.0 : 1.0);
+    atomicAdd(v + o, fpred >= fl ? real(-1) : real(1));
   }
   red[threadIdx.x] = a;
   __syncthreads();
@@ -1239,29 +1241,29 @@ __global__ void __launch_bounds__(1024) force_error_kernel(Geo g, const double* 
   if (threadIdx.x == 0) *abs_sum = red[0];
   for (int t = 0; t < g.nt; ++t) {
     const long long F = (long long)g.nb * g.ncnt[t];
-    for (long long r = threadIdx.x; r < 2 * F; r += blockDim.x) fp.ebar[t][r] = r < F ? 0.0 : seed;
+    for (long long r = threadIdx.x; r < 2 * F; r += blockDim.x) fp.ebar[t][r] = r < F ? real(0) : (real)seed;
   }
 }
 
 // tangent of R~ along v: ddot = v_j - v_i ; Rdot = J ddot
-__global__ void tangent_env_kernel(const double* __restrict__ jac, const int* __restrict__ nl_j, const double* __restrict__ v,
-                                   int Na, int Nm, long long nslots, double* __restrict__ rdot) {
+__global__ void tangent_env_kernel(const real* __restrict__ jac, const int* __restrict__ nl_j, const real* __restrict__ v,
+                                   int Na, int Nm, long long nslots, real* __restrict__ rdot) {
   const long long idx = (long long)blockIdx.x * blockDim.x + threadIdx.x;
   if (idx >= nslots) return;
   const int j = nl_j[idx];
-  double* o = rdot + idx * 4;
+  real* o = rdot + idx * 4;
   if (j < 0) { o[0] = o[1] = o[2] = o[3] = 0.0; return; }
   const long long bi = idx / Nm;
   const int b = (int)(bi / Na);
-  const double* vi = v + bi * 3;
-  const double* vj = v + ((size_t)b * Na + j) * 3;
-  const double dd[3] = {vj[0] - vi[0], vj[1] - vi[1], vj[2] - vi[2]};
-  const double* J = jac + idx * 12;
+  const real* vi = v + bi * 3;
+  const real* vj = v + ((size_t)b * Na + j) * 3;
+  const real dd[3] = {vj[0] - vi[0], vj[1] - vi[1], vj[2] - vi[2]};
+  const real* J = jac + idx * 12;
 #pragma unroll
   for (int k = 0; k < 4; ++k) o[k] = J[3 * k] * dd[0] + J[3 * k + 1] * dd[1] + J[3 * k + 2] * dd[2];
 }
 
-__global__ void fill_kernel(double* p, long long n, double v) {
+__global__ void fill_kernel(real* p, long long n, real v) {
   const long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x;
   if (i < n) p[i] = v;
 }
@@ -1273,22 +1275,22 @@ static PairPtrs make_pp(Ctx& c) {
   PairPtrs pp{};
   for (size_t p = 0; p < c.pairs.size(); ++p) {
     PairNet& P = c.pairs[p];
-    pp.G[p] = P.H.back().as<double>();
-    pp.Gt[p] = P.Ht.back().as<double>();
+    pp.G[p] = P.H.back().as<real>();
+    pp.Gt[p] = P.Ht.back().as<real>();
     pp.row_start[p] = P.row_start.as<int>();
     pp.row_idx[p] = P.row_idx.as<int>();
     pp.tpos[p] = P.tpos.as<int>();
-    pp.sbar[p] = P.sbar.as<double>();
+    pp.sbar[p] = P.sbar.as<real>();
   }
   return pp;
 }
 static FitPtrs make_fp(Ctx& c, int nb) {
   FitPtrs fp{};
   for (int t = 0; t < c.nt; ++t) {
-    fp.D[t] = c.fits[t].D.as<double>();
-    fp.Db[t] = c.fits[t].Db.as<double>();
-    fp.eout[t] = c.fits[t].eout.as<double>();
-    fp.ebar[t] = c.fits[t].ebar.as<double>();
+    fp.D[t] = c.fits[t].D.as<real>();
+    fp.Db[t] = c.fits[t].Db.as<real>();
+    fp.eout[t] = c.fits[t].eout.as<real>();
+    fp.ebar[t] = c.fits[t].ebar.as<real>();
     fp.F[t] = fit_rows(c, t, nb);
   }
   return fp;
@@ -1396,7 +1398,7 @@ static fekf_status build_trows(Ctx& c, int nb, cudaStream_t s) {
   A.Na = c.Na;
   A.Nm = c.Nm;
   A.nl_j = c.nl_j.as<int>();
-  A.v = c.vdir.as<double>();
+  A.v = c.vdir.as<real>();
   int np = 0, cmax = 0;
   for (size_t p = 0; p < c.pairs.size(); ++p) {
     PairNet& P = c.pairs[p];
@@ -1424,8 +1426,8 @@ static fekf_status build_trows(Ctx& c, int nb, cudaStream_t s) {
 }
 
 // one layer of the forward: primal rows (tanh(z + b)) or tangent rows ((1 - y^2) zdot)
-static fekf_status layer_fwd(const Layer& L, const double* w, long long Rmax, const int* Rdev, const double* A,
-                             const double* Hprev, double* Y, double* H, const double* Yprim, const int* rowmap,
+static fekf_status layer_fwd(const Layer& L, const real* w, long long Rmax, const int* Rdev, const real* A,
+                             const real* Hprev, real* Y, real* H, const real* Yprim, const int* rowmap,
                              cudaStream_t s) {
   EpiFwd e;
   e.Y = Y;
@@ -1444,19 +1446,19 @@ static fekf_status layer_fwd(const Layer& L, const double* w, long long Rmax, co
 
 // v = 1 on the selected atoms of every image (0 elsewhere) and the active-row sets of every pair.
 // force_error later sets v = +-1 on the same atoms, so the tangent forward reuses these row sets.
-__global__ void mark_sel_kernel(int nb, int Na, const int* __restrict__ atom_idx, int n_sel, double* __restrict__ v) {
+__global__ void mark_sel_kernel(int nb, int Na, const int* __restrict__ atom_idx, int n_sel, real* __restrict__ v) {
   for (int e = threadIdx.x; e < nb * Na * 3; e += blockDim.x) v[e] = 0.0;
   __syncthreads();
   for (int e = threadIdx.x; e < nb * n_sel * 3; e += blockDim.x) {
     const int b = e / (n_sel * 3), q = (e / 3) % n_sel, al = e % 3;
-    v[((size_t)b * Na + atom_idx[q]) * 3 + al] = 1.0;
+    v[((size_t)b * Na + atom_idx[q]) * 3 + al] = real(1);
   }
 }
 
 fekf_status mark_selected(Ctx& c, int nb, const int* atom_idx, int n_sel, cudaStream_t s) {
   c.sel_atoms = atom_idx;
   c.n_sel_atoms = n_sel;
-  mark_sel_kernel<<<1, 1024, 0, s>>>(nb, c.Na, atom_idx, n_sel, c.vdir.as<double>());
+  mark_sel_kernel<<<1, 1024, 0, s>>>(nb, c.Na, atom_idx, n_sel, c.vdir.as<real>());
   FEKF_LAUNCH_CHECK();
   count_launch();
   FEKF_TRY(build_trows(c, nb, s));
@@ -1464,8 +1466,37 @@ fekf_status mark_selected(Ctx& c, int nb, const int* atom_idx, int n_sel, cudaSt
   return FEKF_OK;
 }
 
+// fp32 nets: fp32 copies of the fp64 inputs (R~, its Jacobian, d: once per geometry; the weights: before
+// every primal forward, i.e. after every Kalman update)
+__global__ void to_real_kernel(const double* __restrict__ src, real* __restrict__ dst, long long n) {
+  const long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i < n) dst[i] = (real)src[i];
+}
+static fekf_status to_real(const DBuf& src, const DBuf& dst, long long n, cudaStream_t s) {
+  if (src.p == dst.p || n <= 0) return FEKF_OK;
+  to_real_kernel<<<cdiv(n, 256), 256, 0, s>>>(src.as<double>(), dst.as<real>(), n);
+  FEKF_LAUNCH_CHECK();
+  count_launch();
+  return FEKF_OK;
+}
+
+fekf_status prepare_geometry(Ctx& c, int nb, cudaStream_t s) {
+#ifdef FEKF_NETS32
+  const long long n = (long long)nb * c.Na * c.Nm;
+  FEKF_TRY(to_real(c.em, c.em32, 4 * n, s));
+  FEKF_TRY(to_real(c.jac, c.jac32, 12 * n, s));
+  FEKF_TRY(to_real(c.rij, c.rij32, 3 * n, s));
+#else
+  (void)c; (void)nb; (void)s;
+#endif
+  return FEKF_OK;
+}
+
 fekf_status model_forward(Ctx& c, int nb, bool tangent, cudaStream_t s) {
-  const double* w = c.w.as<double>();
+#ifdef FEKF_NETS32
+  if (!tangent) FEKF_TRY(to_real(c.w, c.w32, c.Np, s));
+#endif
+  const real* w = w_of(c);
   Geo g = make_geo(c, nb);
   if (tangent && !c.trows_ready) FEKF_TRY(build_trows(c, nb, s));
   if (tangent) c.trows_ready = false;
@@ -1480,46 +1511,46 @@ fekf_status model_forward(Ctx& c, int nb, bool tangent, cudaStream_t s) {
       continue;
     }
     const int* cnt = tangent ? tcount(c, (int)p) : rcount(c, (int)p);
-    double* hin = tangent ? P.hin_t.as<double>() : P.hin.as<double>();
+    real* hin = tangent ? P.hin_t.as<real>() : P.hin.as<real>();
     emb_input_kernel<<<cdiv(Rmax, 256), 256, 0, s>>>((int)Rmax, cnt, P.row_idx.as<int>(),
                                                      tangent ? P.tidx.as<int>() : nullptr,
-                                                     tangent ? c.rdot.as<double>() : c.em.as<double>(), hin);
+                                                     tangent ? c.rdot.as<real>() : em_of(c), hin);
     FEKF_LAUNCH_CHECK();
     count_launch();
     for (size_t l = 0; l < P.L.size(); ++l) {
       if (l == 0 && P.L[0].din == 1) {
         const Layer& L = P.L[0];
         emb_l0_kernel<<<cdiv(Rmax * L.dout, 256), 256, 0, s>>>(
-            (int)Rmax, cnt, L.dout, hin, w + L.W, w + L.b, tangent ? P.Y[0].as<double>() : nullptr,
-            tangent ? P.tidx.as<int>() : nullptr, tangent ? P.Yt[0].as<double>() : P.Y[0].as<double>(),
-            tangent ? P.Ht[0].as<double>() : P.H[0].as<double>());
+            (int)Rmax, cnt, L.dout, hin, w + L.W, w + L.b, tangent ? P.Y[0].as<real>() : nullptr,
+            tangent ? P.tidx.as<int>() : nullptr, tangent ? P.Yt[0].as<real>() : P.Y[0].as<real>(),
+            tangent ? P.Ht[0].as<real>() : P.H[0].as<real>());
         FEKF_LAUNCH_CHECK();
         count_launch();
         continue;
       }
       if (!tangent) {
-        const double* A = l == 0 ? hin : P.H[l - 1].as<double>();
-        FEKF_TRY(layer_fwd(P.L[l], w, Rmax, cnt, A, l == 0 ? nullptr : P.H[l - 1].as<double>(), P.Y[l].as<double>(),
-                           P.H[l].as<double>(), nullptr, nullptr, s));
+        const real* A = l == 0 ? hin : P.H[l - 1].as<real>();
+        FEKF_TRY(layer_fwd(P.L[l], w, Rmax, cnt, A, l == 0 ? nullptr : P.H[l - 1].as<real>(), P.Y[l].as<real>(),
+                           P.H[l].as<real>(), nullptr, nullptr, s));
       } else {
-        const double* A = l == 0 ? hin : P.Ht[l - 1].as<double>();
-        FEKF_TRY(layer_fwd(P.L[l], w, Rmax, cnt, A, l == 0 ? nullptr : P.Ht[l - 1].as<double>(), P.Yt[l].as<double>(),
-                           P.Ht[l].as<double>(), P.Y[l].as<double>(), P.tidx.as<int>(), s));
+        const real* A = l == 0 ? hin : P.Ht[l - 1].as<real>();
+        FEKF_TRY(layer_fwd(P.L[l], w, Rmax, cnt, A, l == 0 ? nullptr : P.Ht[l - 1].as<real>(), P.Yt[l].as<real>(),
+                           P.Ht[l].as<real>(), P.Y[l].as<real>(), P.tidx.as<int>(), s));
       }
     }
   }
   // descriptor
   PairPtrs pp = make_pp(c);
   FitPtrs fp = make_fp(c, nb);
-  const size_t smem = (8 * (size_t)c.M + 8 * (size_t)c.Nm + 4 * 32 * DESC_MC * (DESC_THREADS / 32)) * sizeof(double);
+  const size_t smem = (8 * (size_t)c.M + 8 * (size_t)c.Nm + 4 * 32 * DESC_MC * (DESC_THREADS / 32)) * sizeof(real);
   const size_t Xoff = (size_t)c.B * c.Na * 4 * c.M;
   static size_t dattr = 0;
   if (smem > dattr) {
     FEKF_CHECK_CUDA(cudaFuncSetAttribute(desc_fwd_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
     dattr = smem;
   }
-  desc_fwd_kernel<<<nb * c.Na, DESC_THREADS, smem, s>>>(g, pp, fp, c.em.as<double>(), c.rdot.as<double>(),
-                                                        tangent ? 1 : 0, c.X.as<double>(), c.X.as<double>() + Xoff);
+  desc_fwd_kernel<<<nb * c.Na, DESC_THREADS, smem, s>>>(g, pp, fp, em_of(c), c.rdot.as<real>(),
+                                                        tangent ? 1 : 0, c.X.as<real>(), c.X.as<real>() + Xoff);
   FEKF_LAUNCH_CHECK();
   count_launch();
   // fitting nets (stacked rows: the tangent half starts at row F); one grouped GEMM per layer over types
@@ -1532,12 +1563,12 @@ fekf_status model_forward(Ctx& c, int nb, bool tangent, cudaStream_t s) {
       const long long F = fit_rows(c, t, nb);
       if (F == 0) continue;
       const Layer& L = Fn.L[l];
-      const double* Ain = l == 0 ? Fn.D.as<double>() : Fn.H[l - 1].as<double>();
-      const double* Hprev = l == 0 ? nullptr : Fn.H[l - 1].as<double>();
+      const real* Ain = l == 0 ? Fn.D.as<real>() : Fn.H[l - 1].as<real>();
+      const real* Hprev = l == 0 ? nullptr : Fn.H[l - 1].as<real>();
       const size_t oi = tangent ? (size_t)F * L.din : 0, oo = tangent ? (size_t)F * L.dout : 0;
       EpiFwd e;
-      e.Y = Fn.Y[l].as<double>() + oo;
-      e.H = Fn.H[l].as<double>() + oo;
+      e.Y = Fn.Y[l].as<real>() + oo;
+      e.H = Fn.H[l].as<real>() + oo;
       e.ld = L.dout;
       e.bias = w + L.b;
       e.dt = L.dt >= 0 ? w + L.dt : nullptr;
@@ -1545,7 +1576,7 @@ fekf_status model_forward(Ctx& c, int nb, bool tangent, cudaStream_t s) {
       e.ldp = L.din;
       e.skip = Hprev ? L.skip : 0;
       e.dprev = L.din;
-      e.Yprim = tangent ? Fn.Y[l].as<double>() : nullptr;
+      e.Yprim = tangent ? Fn.Y[l].as<real>() : nullptr;
       e.rowmap = nullptr;
       pr[n++] = GemmProb<EpiFwd>{(int)F, L.dout, L.din, nullptr, nullptr, Ain + oi, L.din, w + L.W, L.dout, -1, 0, 0, 1, e};
     }
@@ -1556,8 +1587,8 @@ fekf_status model_forward(Ctx& c, int nb, bool tangent, cudaStream_t s) {
     const long long F = fit_rows(c, t, nb);
     if (F == 0) continue;
     const int h = Fn.L.back().dout;
-    const double* Hl = Fn.H.back().as<double>();
-    double* eo = Fn.eout.as<double>();
+    const real* Hl = Fn.H.back().as<real>();
+    real* eo = Fn.eout.as<real>();
     fit_out_kernel<<<cdiv(F * 32, 256), 256, 0, s>>>(F, F, h, tangent ? Hl + (size_t)F * h : Hl, w + Fn.Wout, w + Fn.bout,
                                                       tangent ? eo + F : eo);
     FEKF_LAUNCH_CHECK();
@@ -1590,7 +1621,7 @@ fekf_status seed_force(Ctx& c, int nb, cudaStream_t s) {
   for (int t = 0; t < c.nt; ++t) {
     const long long F = fit_rows(c, t, nb);
     if (F == 0) continue;
-    fill_kernel<<<cdiv(F, 256), 256, 0, s>>>(c.fits[t].ebar.as<double>(), F, 1.0);
+    fill_kernel<<<cdiv(F, 256), 256, 0, s>>>(c.fits[t].ebar.as<real>(), F, real(1));
     FEKF_LAUNCH_CHECK();
     count_launch();
   }
@@ -1603,7 +1634,7 @@ fekf_status force_error(Ctx& c, int nb, const double* f_label, const int* atom_i
   FitPtrs fp = make_fp(c, nb);
   double seed = -1.0 / ((double)c.Na * n_sel * 3);
   if (c.o.grad_reduce == 1) seed /= c.Bg;
-  force_error_kernel<<<1, 1024, 0, s>>>(g, c.force.as<double>(), f_label, atom_idx, n_sel, seed, c.vdir.as<double>(), fp,
+  force_error_kernel<<<1, 1024, 0, s>>>(g, c.force.as<double>(), f_label, atom_idx, n_sel, seed, c.vdir.as<real>(), fp,
                                        abs_sum);
   FEKF_LAUNCH_CHECK();
   count_launch();
@@ -1612,8 +1643,8 @@ fekf_status force_error(Ctx& c, int nb, const double* f_label, const int* atom_i
 
 fekf_status tangent_env(Ctx& c, int nb, cudaStream_t s) {
   const long long n = (long long)nb * c.Na * c.Nm;
-  tangent_env_kernel<<<cdiv(n, 256), 256, 0, s>>>(c.jac.as<double>(), c.nl_j.as<int>(), c.vdir.as<double>(), c.Na, c.Nm,
-                                                  n, c.rdot.as<double>());
+  tangent_env_kernel<<<cdiv(n, 256), 256, 0, s>>>(jac_of(c), c.nl_j.as<int>(), c.vdir.as<real>(), c.Na, c.Nm,
+                                                  n, c.rdot.as<real>());
   FEKF_LAUNCH_CHECK();
   count_launch();
   return FEKF_OK;
@@ -1634,7 +1665,7 @@ static int sm_count() {
 }
 
 fekf_status model_backward(Ctx& c, int nb, Mode mode, double* gout, cudaStream_t s) {
-  const double* w = c.w.as<double>();
+  const real* w = w_of(c);
   const bool dual = mode == MODE_FORCE_JAC;
   if (mode == MODE_FORCE_SEL && !emb_fused_ok(c)) mode = MODE_FORCE;   // per-layer path: every row
   const bool force = mode == MODE_FORCE || mode == MODE_FORCE_SEL;
@@ -1650,12 +1681,12 @@ fekf_status model_backward(Ctx& c, int nb, Mode mode, double* gout, cudaStream_t
     if (F == 0) continue;
     const long long nF = dual ? 2 * F : F;
     const int h = Fn.L.back().dout;
-    fit_out_bwd_kernel<<<cdiv(nF * h, 256), 256, 0, s>>>(nF, h, Fn.ebar.as<double>(), w + Fn.Wout, Fn.Hb.back().as<double>());
+    fit_out_bwd_kernel<<<cdiv(nF * h, 256), 256, 0, s>>>(nF, h, Fn.ebar.as<real>(), w + Fn.Wout, Fn.Hb.back().as<real>());
     FEKF_LAUNCH_CHECK();
     count_launch();
     if (want_w) {
-      const double* Hl = Fn.H.back().as<double>();
-      const double* eb = Fn.ebar.as<double>();
+      const real* Hl = Fn.H.back().as<real>();
+      const real* eb = Fn.ebar.as<real>();
       FEKF_TRY(wgrad(c, h, 1, Seg{Hl, eb, F, nullptr, 1},
                      Seg{dual ? Hl + (size_t)F * h : nullptr, dual ? eb + F : nullptr, dual ? F : 0, nullptr, 0},
                      gout + Fn.Wout, s));
@@ -1671,27 +1702,27 @@ fekf_status model_backward(Ctx& c, int nb, Mode mode, double* gout, cudaStream_t
       if (F == 0) continue;
       const long long nF = dual ? 2 * F : F;
       const Layer& L = Fn.L[l];
-      const double* dt = L.dt >= 0 ? w + L.dt : nullptr;
+      const real* dt = L.dt >= 0 ? w + L.dt : nullptr;
       if (want_w && dt) {
-        FEKF_TRY(act_bwd_dt(c, F, L.dout, Fn.Y[l].as<double>(), Fn.Hb[l].as<double>(), dt, dual,
-                            Fn.Zb[l].as<double>(), gout + L.dt, s));
+        FEKF_TRY(act_bwd_dt(c, F, L.dout, Fn.Y[l].as<real>(), Fn.Hb[l].as<real>(), dt, dual,
+                            Fn.Zb[l].as<real>(), gout + L.dt, s));
       } else {
-        act_bwd_kernel<<<cdiv(F * L.dout, 256), 256, 0, s>>>(F, L.dout, Fn.Y[l].as<double>(), Fn.Hb[l].as<double>(),
-                                                              dt, dual ? 1 : 0, Fn.Zb[l].as<double>());
+        act_bwd_kernel<<<cdiv(F * L.dout, 256), 256, 0, s>>>(F, L.dout, Fn.Y[l].as<real>(), Fn.Hb[l].as<real>(),
+                                                              dt, dual ? 1 : 0, Fn.Zb[l].as<real>());
         FEKF_LAUNCH_CHECK();
         count_launch();
       }
-      const double* Hprev = l == 0 ? Fn.D.as<double>() : Fn.H[l - 1].as<double>();
+      const real* Hprev = l == 0 ? Fn.D.as<real>() : Fn.H[l - 1].as<real>();
       if (want_w) {
         // stacked rows; the ones column covers the primal half only (bias not in the tangent)
-        jobs[nj++] = WgradJob{L.din, L.dout, Seg{Hprev, Fn.Zb[l].as<double>(), F, nullptr, 1},
+        jobs[nj++] = WgradJob{L.din, L.dout, Seg{Hprev, Fn.Zb[l].as<real>(), F, nullptr, 1},
                               Seg{dual ? Hprev + (size_t)F * L.din : nullptr,
-                                  dual ? Fn.Zb[l].as<double>() + (size_t)F * L.dout : nullptr, dual ? F : 0, nullptr, 0},
+                                  dual ? Fn.Zb[l].as<real>() + (size_t)F * L.dout : nullptr, dual ? F : 0, nullptr, 0},
                               gout + L.W};
       }
-      double* out = l == 0 ? Fn.Db.as<double>() : Fn.Hb[l - 1].as<double>();
-      EpiDgrad e{out, L.din, Fn.Hb[l].as<double>(), L.dout, l == 0 ? 0 : L.skip, L.din};
-      dg[nd++] = GemmProb<EpiDgrad>{(int)nF, L.din, L.dout, nullptr, nullptr, Fn.Zb[l].as<double>(), L.dout, w + L.W,
+      real* out = l == 0 ? Fn.Db.as<real>() : Fn.Hb[l - 1].as<real>();
+      EpiDgrad e{out, L.din, Fn.Hb[l].as<real>(), L.dout, l == 0 ? 0 : L.skip, L.din};
+      dg[nd++] = GemmProb<EpiDgrad>{(int)nF, L.din, L.dout, nullptr, nullptr, Fn.Zb[l].as<real>(), L.dout, w + L.W,
                                     L.dout, -1, 0, 0, 1, e};
     }
     if (nj) FEKF_TRY(wgrad_group(c, jobs, nj, s));
@@ -1709,15 +1740,15 @@ fekf_status model_backward(Ctx& c, int nb, Mode mode, double* gout, cudaStream_t
     SeedOut so{};
     for (size_t p = 0; p < c.pairs.size(); ++p) {
       PairNet& P = c.pairs[p];
-      so.gbar[p] = P.Hb.back().as<double>();
-      so.hbt[p] = P.Hbt.back().as<double>();
-      so.dr[p] = P.Zb[0].as<double>();
+      so.gbar[p] = P.Hb.back().as<real>();
+      so.hbt[p] = P.Hbt.back().as<real>();
+      so.dr[p] = P.Zb[0].as<real>();
     }
-    const size_t smem = (16 * (size_t)c.M + 2 * (size_t)c.M * (c.M2 + 1) + 8 * (size_t)c.Nm) * sizeof(double);
+    const size_t smem = (16 * (size_t)c.M + 2 * (size_t)c.M * (c.M2 + 1) + 8 * (size_t)c.Nm) * sizeof(real);
     auto launch = [&](auto kern) -> fekf_status {
       FEKF_CHECK_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-      kern<<<nb * c.Na, 256, smem, s>>>(g, fp, pp, so, c.X.as<double>(), c.X.as<double>() + Xoff, c.em.as<double>(),
-                                        c.rdot.as<double>(), c.Xb.as<double>(), c.Xb.as<double>() + Xoff);
+      kern<<<nb * c.Na, 256, smem, s>>>(g, fp, pp, so, c.X.as<real>(), c.X.as<real>() + Xoff, em_of(c),
+                                        c.rdot.as<real>(), c.Xb.as<real>(), c.Xb.as<real>() + Xoff);
       return FEKF_OK;
     };
     if (dual) FEKF_TRY(launch(desc_bwd_seed_kernel<true, false, false>));
@@ -1725,9 +1756,9 @@ fekf_status model_backward(Ctx& c, int nb, Mode mode, double* gout, cudaStream_t
     else if (force) FEKF_TRY(launch(desc_bwd_seed_kernel<false, true, false>));
     else FEKF_TRY(launch(desc_bwd_seed_kernel<false, false, false>));
   } else {
-    const size_t smem = (8 * c.M + 2 * c.M * (c.M2 + 1)) * sizeof(double);
-    desc_bwd_kernel<<<nb * c.Na, 128, smem, s>>>(g, fp, c.X.as<double>(), c.X.as<double>() + Xoff, dual ? 1 : 0,
-                                                 c.Xb.as<double>(), c.Xb.as<double>() + Xoff);
+    const size_t smem = (8 * c.M + 2 * c.M * (c.M2 + 1)) * sizeof(real);
+    desc_bwd_kernel<<<nb * c.Na, 128, smem, s>>>(g, fp, c.X.as<real>(), c.X.as<real>() + Xoff, dual ? 1 : 0,
+                                                 c.Xb.as<real>(), c.Xb.as<real>() + Xoff);
   }
   FEKF_LAUNCH_CHECK();
   count_launch();
@@ -1743,15 +1774,15 @@ fekf_status model_backward(Ctx& c, int nb, Mode mode, double* gout, cudaStream_t
     SeedPtrs sp{};
     for (size_t p = 0; p < c.pairs.size(); ++p) {
       PairNet& P = c.pairs[p];
-      sp.Y[p] = P.Y.back().as<double>();
-      sp.Yt[p] = P.Yt.back().as<double>();
-      sp.Hb[p] = P.Hb.back().as<double>();
-      sp.Zb[p] = P.Zb.back().as<double>();
-      sp.Hbt[p] = P.Hbt.back().as<double>();
-      sp.Zbt[p] = P.Zbt.back().as<double>();
+      sp.Y[p] = P.Y.back().as<real>();
+      sp.Yt[p] = P.Yt.back().as<real>();
+      sp.Hb[p] = P.Hb.back().as<real>();
+      sp.Zb[p] = P.Zb.back().as<real>();
+      sp.Hbt[p] = P.Hbt.back().as<real>();
+      sp.Zbt[p] = P.Zbt.back().as<real>();
     }
-    emb_seed_atom_kernel<<<nb * c.Na, 128, 8 * c.M * sizeof(double), s>>>(
-        g, pp, sp, c.em.as<double>(), c.rdot.as<double>(), c.Xb.as<double>(), c.Xb.as<double>() + Xoff, dual ? 1 : 0);
+    emb_seed_atom_kernel<<<nb * c.Na, 128, 8 * c.M * sizeof(real), s>>>(
+        g, pp, sp, em_of(c), c.rdot.as<real>(), c.Xb.as<real>(), c.Xb.as<real>() + Xoff, dual ? 1 : 0);
     FEKF_LAUNCH_CHECK();
     count_launch();
   }
@@ -1767,34 +1798,34 @@ fekf_status model_backward(Ctx& c, int nb, Mode mode, double* gout, cudaStream_t
     for (int l = nl - 1; l >= 0; --l) {
       const Layer& L = P.L[l];
       if (want_w) {
-        const double* Hp = l == 0 ? P.hin.as<double>() : P.H[l - 1].as<double>();
-        const double* Hpt = l == 0 ? P.hin_t.as<double>() : P.Ht[l - 1].as<double>();
-        FEKF_TRY(wgrad(c, L.din, L.dout, Seg{Hp, P.Zb[l].as<double>(), Rmax, rc, 1},
-                       Seg{dual ? Hpt : nullptr, dual ? P.Zbt[l].as<double>() : nullptr, dual ? Rmax : 0, tc, 0},
+        const real* Hp = l == 0 ? P.hin.as<real>() : P.H[l - 1].as<real>();
+        const real* Hpt = l == 0 ? P.hin_t.as<real>() : P.Ht[l - 1].as<real>();
+        FEKF_TRY(wgrad(c, L.din, L.dout, Seg{Hp, P.Zb[l].as<real>(), Rmax, rc, 1},
+                       Seg{dual ? Hpt : nullptr, dual ? P.Zbt[l].as<real>() : nullptr, dual ? Rmax : 0, tc, 0},
                        gout + L.W, s, true));
       }
       if (l > 0) {
         if (dual) {
-          EpiDgradAct et{P.Hbt[l - 1].as<double>(), L.din, P.Hbt[l].as<double>(), L.dout, L.skip, L.din,
-                         P.Y[l - 1].as<double>(), P.Zbt[l - 1].as<double>(), nullptr, nullptr, nullptr,
+          EpiDgradAct et{P.Hbt[l - 1].as<real>(), L.din, P.Hbt[l].as<real>(), L.dout, L.skip, L.din,
+                         P.Y[l - 1].as<real>(), P.Zbt[l - 1].as<real>(), nullptr, nullptr, nullptr,
                          P.tidx.as<int>()};
-          FEKF_TRY(gemm<false, true>(Rmax, L.din, L.dout, P.Zbt[l].as<double>(), L.dout, w + L.W, L.dout, et, s, tc));
+          FEKF_TRY(gemm<false, true>(Rmax, L.din, L.dout, P.Zbt[l].as<real>(), L.dout, w + L.W, L.dout, et, s, tc));
         }
-        EpiDgradAct e{P.Hb[l - 1].as<double>(), L.din, P.Hb[l].as<double>(), L.dout, L.skip, L.din,
-                      P.Y[l - 1].as<double>(), P.Zb[l - 1].as<double>(), dual ? P.tpos.as<int>() : nullptr,
-                      P.Yt[l - 1].as<double>(), P.Hbt[l - 1].as<double>(), nullptr};
-        FEKF_TRY(gemm<false, true>(Rmax, L.din, L.dout, P.Zb[l].as<double>(), L.dout, w + L.W, L.dout, e, s, rc));
+        EpiDgradAct e{P.Hb[l - 1].as<real>(), L.din, P.Hb[l].as<real>(), L.dout, L.skip, L.din,
+                      P.Y[l - 1].as<real>(), P.Zb[l - 1].as<real>(), dual ? P.tpos.as<int>() : nullptr,
+                      P.Yt[l - 1].as<real>(), P.Hbt[l - 1].as<real>(), nullptr};
+        FEKF_TRY(gemm<false, true>(Rmax, L.din, L.dout, P.Zb[l].as<real>(), L.dout, w + L.W, L.dout, e, s, rc));
       } else if (mode == MODE_FORCE) {
-        FEKF_TRY(gemm<false, true>(Rmax, 1, L.dout, P.Zb[0].as<double>(), L.dout, w + L.W, L.dout,
-                                   EpiStore{P.sbar.as<double>(), 1}, s, rc));
+        FEKF_TRY(gemm<false, true>(Rmax, 1, L.dout, P.Zb[0].as<real>(), L.dout, w + L.W, L.dout,
+                                   EpiStore<real>{P.sbar.as<real>(), 1}, s, rc));
       }
     }
   }
   }
   if (force) {
     if (!emb_fused_ok(c)) {
-      prod_force_kernel<<<nb * c.Na, 128, 0, s>>>(g, pp, c.Xb.as<double>(), c.jac.as<double>(), c.nl_j.as<int>(),
-                                                  c.frow.as<double>());
+      prod_force_kernel<<<nb * c.Na, 128, 0, s>>>(g, pp, c.Xb.as<real>(), jac_of(c), c.nl_j.as<int>(),
+                                                  c.frow.as<real>());
       FEKF_LAUNCH_CHECK();
       count_launch();
     }
@@ -1802,7 +1833,7 @@ fekf_status model_backward(Ctx& c, int nb, Mode mode, double* gout, cudaStream_t
     const bool sel = mode == MODE_FORCE_SEL && c.sel_atoms;
     const int nw = sel ? nb * c.n_sel_atoms : nb * c.Na;
     force_gather_kernel<<<cdiv(nw, 8), 256, 0, s>>>(nb, c.Na, c.Nm, sel ? c.sel_atoms : nullptr, c.n_sel_atoms,
-                                                    c.nl_j.as<int>(), c.rij.as<double>(), c.frow.as<double>(),
+                                                    c.nl_j.as<int>(), rij_of(c), c.frow.as<real>(),
                                                     c.rev_off.as<int>(), c.rev_idx.as<int>(), c.force.as<double>(),
                                                     c.vatom.as<double>());
     FEKF_LAUNCH_CHECK();
@@ -1817,4 +1848,5 @@ fekf_status model_backward(Ctx& c, int nb, Mode mode, double* gout, cudaStream_t
   return FEKF_OK;
 }
 
+}  // namespace FEKF_NETNS
 }  // namespace fekf

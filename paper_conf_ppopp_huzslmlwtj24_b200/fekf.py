@@ -37,7 +37,8 @@ class ModelCfg(C.Structure):
 class OptCfg(C.Structure):
     _fields_ = [("lambda0", C.c_double), ("nu", C.c_double), ("block_size", C.c_int), ("noise_mode", C.c_int),
                 ("grad_reduce", C.c_int), ("force_groups", C.c_int), ("atoms_per_group", C.c_int),
-                ("p_defer", C.c_int), ("precision", C.c_int), ("p_mode", C.c_int)]
+                ("p_defer", C.c_int), ("precision", C.c_int), ("p_mode", C.c_int),
+                ("net_precision", C.c_int)]
 
 
 _lib = None
@@ -178,6 +179,9 @@ def opt_cfg(o=None) -> OptCfg:
     c.p_defer = int(_get(o, "p_defer", 15)) if o is not None else 15
     c.precision = int(_get(o, "precision", 64)) if o is not None else 64
     c.p_mode = int(_get(o, "p_mode", 0)) if o is not None else 0
+    c.net_precision = int(_get(o, "net_precision", 0) or 0) if o is not None else 0
+    if c.net_precision not in (0, 32, 64):
+        raise ValueError("net_precision must be 0 (follow precision), 32 or 64")
     if c.p_mode not in (0, 1):
         raise ValueError("p_mode must be 0 (sharded) or 1 (replicated)")
     if c.precision not in (32, 64):

@@ -22,6 +22,7 @@ from fixtures import get_config, make_dataset, init_weights, force_groups  # noq
 
 
 def short(n):
+    n = n.replace("fekf::n64::", "fekf::").replace("fekf::n32::", "fekf::")
     m = re.search(r"dgemm_kernel<(\d+), (\d+), \d+, \d+, (\w+), (\w+), fekf::(\w+)", n)
     if m:
         return "dgemm<%s,%s,%s>" % (m.group(1), m.group(2), m.group(5))
@@ -34,9 +35,12 @@ def main():
     ap.add_argument("--config", default="c2_water64")
     ap.add_argument("--steps", type=int, default=2)
     ap.add_argument("--eager", action="store_true")
+    ap.add_argument("--precision", type=int, default=64)
+    ap.add_argument("--net-precision", type=int, default=0)
     a = ap.parse_args()
     wl = get_config(a.config)
     m, opt = wl.model, wl.opt
+    opt = type(opt)(**{**opt.__dict__, "precision": a.precision, "net_precision": a.net_precision})
     B = wl.batch
     ds = make_dataset(a.config, B)
     na = len(ds["types"])
