@@ -323,15 +323,191 @@ dgemm_kernel(const __grid_constant__ GemmGroup<Epi> G) {
       }
 }
 
+#ifdef FEKF_NETS32
+// fp32 nets: the same GEMM on the FP32 FFMA pipe (measured 71.5 TFLOP/s on B200, vs 34.6 for an
+// fp32-accurate product on the split-tf32 mma.sync pair; tools/fp32_peak.cu).  256 threads as a 16 x 16
+// grid, each a TM x TN register micro-tile (TM = BM/16 consecutive rows, TN = BN/16 columns strided by 16);
+// both operands staged k-major in SMEM, [k][m] and [k][n] (row stride MN + 4), so a thread's TM rows are
+// TM/4 LDS.128 broadcasts and its columns conflict-free LDS.32 across the 16 column threads.  The
+// operands stored k-contiguous (A row-major, B given as [N x K]) are transposed on the way in by
+// element-wise cp.async (4 bytes each, from coalesced global reads).  Same GemmGroup / split-K / device
+// row-count / "ones" row semantics as dgemm_kernel; the epilogue gets every element of the micro-tile.
+template <int BM, int BN, bool TA, bool TB, class Epi>
+__global__ void __launch_bounds__(256)
+sgemm_kernel(const __grid_constant__ GemmGroup<Epi> G) {
+  constexpr int NT = 256, TM = BM / 16, TN = BN / 16, LA = BM + 4, LB = BN + 4;
+  constexpr int ASZ = GB_K * LA, BSZ = GB_K * LB;
+  static_assert(TM % 4 == 0 && BN % 16 == 0, "sgemm micro-tile");
+  extern __shared__ __align__(16) real gsm[];
+  real* As0 = gsm;
+  real* Bs0 = gsm + GB_STAGES * ASZ;
+  int q = 0;
+#pragma unroll
+  for (int k = 1; k < GG_MAX; ++k)
+    if (k < G.n && (int)blockIdx.x >= G.start[k]) q = k;
+  const GemmProb<Epi> P = pick(G, q);
+  const int local = blockIdx.x - G.start[q];
+  int mtq = G.mt[0], ntq = G.nt[0];
+#pragma unroll
+  for (int k = 1; k < GG_MAX; ++k)
+    if (q == k) { mtq = G.mt[k]; ntq = G.nt[k]; }
+  const int bm = local % mtq, bn = (local / mtq) % ntq, bz = local / (mtq * ntq);
+  int M = P.M, K = P.K, aug_k = P.aug_k;
+  const int N = P.N, lda = P.lda, ldb = P.ldb, aug_m = P.aug_m, kps = P.kps;
+  const real* __restrict__ A = P.A;
+  const real* __restrict__ B = P.B;
+  Epi epi = P.epi;
+  epi.split(bz);
+  if (P.Mdev) M = min(M, *P.Mdev);
+  if (P.Kdev) {
+    const int kd = *P.Kdev;
+    K = min(K, kd);
+    aug_k = min(aug_k, kd);
+  }
+  const int tid = threadIdx.x;
+  const int m0 = bm * BM, n0 = bn * BN;
+  const int kbeg = bz * kps;
+  if (m0 >= M || (bz > 0 && kbeg >= K)) return;  // empty split: the reduction skips it
+  const int kend = min(K, kbeg + kps);
+  const int ty = tid >> 4, tx = tid & 15;
+  real acc[TM][TN];
+#pragma unroll
+  for (int i = 0; i < TM; ++i)
+#pragma unroll
+    for (int j = 0; j < TN; ++j) acc[i][j] = 0.f;
+  // two-element copies along m (TA) / n (!TB) when strides and bases allow
+  const int mreal = aug_m >= 0 ? min(M, aug_m) : M;
+  const bool a2 = TA && !(lda & 1) && !(reinterpret_cast<size_t>(A) & PAIR_MASK);
+  const bool b2 = !TB && !(ldb & 1) && !(reinterpret_cast<size_t>(B) & PAIR_MASK) && !(N & 1);
+  auto issue = [&](int buf, int k0) {
+    real* As = As0 + buf * ASZ;
+    real* Bs = Bs0 + buf * BSZ;
+    if (TA) {   // A stored [K x M]: rows of m, straight
+      if (a2) {
+        for (int idx = tid; idx < GB_K * BM / 2; idx += NT) {
+          const int kk = idx / (BM / 2), r = 2 * (idx % (BM / 2));
+          const int m = m0 + r, k = k0 + kk;
+          const bool kin = k < kend;
+          if (m + 1 < mreal) {
+            cp_async2(As + kk * LA + r, kin ? A + (size_t)k * lda + m : A, kin);
+          } else {
+#pragma unroll
+            for (int h = 0; h < 2; ++h) {
+              real* dst = As + kk * LA + r + h;
+              if (m + h == aug_m) *dst = (k < aug_k) ? real(1) : real(0);
+              else {
+                const bool ok = m + h < M && kin;
+                cp_async1(dst, ok ? A + (size_t)k * lda + m + h : A, ok);
+              }
+            }
+          }
+        }
+      } else {
+        for (int idx = tid; idx < GB_K * BM; idx += NT) {
+          const int kk = idx / BM, r = idx % BM;
+          const int m = m0 + r, k = k0 + kk;
+          real* dst = As + kk * LA + r;
+          if (m == aug_m) *dst = (k < aug_k) ? real(1) : real(0);
+          else {
+            const bool ok = m < M && k < kend;
+            cp_async1(dst, ok ? A + (size_t)k * lda + m : A, ok);
+          }
+        }
+      }
+    } else {   // A row-major [M x K]: coalesced along k, transposed into [k][m]
+      for (int idx = tid; idx < GB_K * BM; idx += NT) {
+        const int r = idx / GB_K, kk = idx % GB_K;
+        const int m = m0 + r, k = k0 + kk;
+        real* dst = As + kk * LA + r;
+        if (m == aug_m) *dst = (k < aug_k) ? real(1) : real(0);
+        else {
+          const bool ok = m < M && k < kend;
+          cp_async1(dst, ok ? A + (size_t)m * lda + k : A, ok);
+        }
+      }
+    }
+    if (!TB) {   // B row-major [K x N]: straight
+      if (b2) {
+        for (int idx = tid; idx < GB_K * BN / 2; idx += NT) {
+          const int kk = idx / (BN / 2), c = 2 * (idx % (BN / 2));
+          const int n = n0 + c, k = k0 + kk;
+          const bool ok = n < N && k < kend;
+          cp_async2(Bs + kk * LB + c, ok ? B + (size_t)k * ldb + n : B, ok);
+        }
+      } else {
+        for (int idx = tid; idx < GB_K * BN; idx += NT) {
+          const int kk = idx / BN, c = idx % BN;
+          const int n = n0 + c, k = k0 + kk;
+          const bool ok = n < N && k < kend;
+          cp_async1(Bs + kk * LB + c, ok ? B + (size_t)k * ldb + n : B, ok);
+        }
+      }
+    } else {   // B given as [N x K]: coalesced along k, transposed into [k][n]
+      for (int idx = tid; idx < GB_K * BN; idx += NT) {
+        const int c = idx / GB_K, kk = idx % GB_K;
+        const int n = n0 + c, k = k0 + kk;
+        const bool ok = n < N && k < kend;
+        cp_async1(Bs + kk * LB + c, ok ? B + (size_t)n * ldb + k : B, ok);
+      }
+    }
+  };
+  const int nk = kend > kbeg ? (kend - kbeg + GB_K - 1) / GB_K : 0;
+#pragma unroll
+  for (int st = 0; st < GB_STAGES - 1; ++st) {
+    if (st < nk) issue(st, kbeg + st * GB_K);
+    cp_async_commit();
+  }
+  for (int t = 0; t < nk; ++t) {
+    cp_async_wait<GB_STAGES - 2>();
+    __syncthreads();  // slice t visible to all; slice t-1's buffer free for reuse
+    const int tn = t + GB_STAGES - 1;
+    if (tn < nk) issue(tn % GB_STAGES, kbeg + tn * GB_K);
+    cp_async_commit();
+    const real* As = As0 + (t % GB_STAGES) * ASZ + ty * TM;
+    const real* Bs = Bs0 + (t % GB_STAGES) * BSZ + tx;
+#pragma unroll
+    for (int kk = 0; kk < GB_K; ++kk) {
+      real a[TM], b[TN];
+#pragma unroll
+      for (int i = 0; i < TM; i += 4) {
+        const float4 v = *reinterpret_cast<const float4*>(As + kk * LA + i);
+        a[i] = v.x; a[i + 1] = v.y; a[i + 2] = v.z; a[i + 3] = v.w;
+      }
+#pragma unroll
+      for (int j = 0; j < TN; ++j) b[j] = Bs[kk * LB + 16 * j];
+#pragma unroll
+      for (int i = 0; i < TM; ++i)
+#pragma unroll
+        for (int j = 0; j < TN; ++j) acc[i][j] = fmaf(a[i], b[j], acc[i][j]);
+    }
+  }
+  cp_async_wait<0>();
+#pragma unroll
+  for (int i = 0; i < TM; ++i)
+#pragma unroll
+    for (int j = 0; j < TN; ++j) {
+      const int r = m0 + ty * TM + i, c = n0 + tx + 16 * j;
+      if (r < M && c < N) epi(r, c, acc[i][j]);
+    }
+}
+#endif
+
 template <int BM, int BN, int WM, int WN, bool TA, bool TB, class Epi, int NW = 8>
 static fekf_status gemm_launch(GemmGroup<Epi>& G, cudaStream_t s) {
+#ifdef FEKF_NETS32
+  constexpr size_t smem = sizeof(real) * GB_STAGES * GB_K * ((BM + 4) + (BN + 4));
+  auto kern = sgemm_kernel<BM, BN, TA, TB, Epi>;
+  constexpr int nthr = 256;
+#else
   constexpr size_t asz = TA ? GB_K * (BM + 4) : BM * GB_LDS;
   constexpr size_t bsz = TB ? BN * GB_LDS : GB_K * (BN + 4);
   constexpr size_t smem = sizeof(real) * GB_STAGES * (asz + bsz);
+  auto kern = dgemm_kernel<BM, BN, WM, WN, TA, TB, Epi, NW>;
+  constexpr int nthr = 32 * NW;
+#endif
   static bool attr = false;
   if (!attr) {
-    FEKF_CHECK_CUDA(cudaFuncSetAttribute(dgemm_kernel<BM, BN, WM, WN, TA, TB, Epi, NW>,
-                                         cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    FEKF_CHECK_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
     attr = true;
   }
   int tot = 0;
@@ -343,7 +519,7 @@ static fekf_status gemm_launch(GemmGroup<Epi>& G, cudaStream_t s) {
   }
   for (int q = G.n; q <= GG_MAX; ++q) G.start[q] = tot;
   if (tot == 0) return FEKF_OK;
-  dgemm_kernel<BM, BN, WM, WN, TA, TB, Epi, NW><<<tot, 32 * NW, smem, s>>>(G);
+  kern<<<tot, nthr, smem, s>>>(G);
   FEKF_LAUNCH_CHECK();
   count_launch();
   return FEKF_OK;
