@@ -66,31 +66,33 @@ nlist_kernel(const double* __restrict__ coord, const double* __restrict__ box, c
   const long long nshift = (long long)na_ * nb_ * nc_;
   const double* xi = coord + ((size_t)b * Na + i) * 3;
   const double xi0 = xi[0], xi1 = xi[1], xi2 = xi[2];
-  const long long ncand = nshift * Na;
-  for (long long q = tid; q < ncand; q += NL_THREADS) {
-    const int j = (int)(q % Na);
-    const long long sidx = q / Na;
+  // shifts outer (uniform over the CTA: no per-candidate integer division), atoms j strided over threads
+  for (long long sidx = 0; sidx < nshift; ++sidx) {
     const int ic = (int)(sidx % nc_) - mc;
     const int ib = (int)((sidx / nc_) % nb_) - mb;
     const int ia = (int)(sidx / ((long long)nc_ * nb_)) - ma;
-    if (j == i && ia == 0 && ib == 0 && ic == 0) continue;
     const double fa = (double)ia, fb = (double)ib, fc = (double)ic;
     double S[3];
 #pragma unroll
     for (int ax = 0; ax < 3; ++ax)
       S[ax] = __dadd_rn(__dadd_rn(__dmul_rn(fa, s_box[ax]), __dmul_rn(fb, s_box[3 + ax])), __dmul_rn(fc, s_box[6 + ax]));
-    const double* xj = coord + ((size_t)b * Na + j) * 3;
-    const double dx = __dadd_rn(__dsub_rn(xj[0], xi0), S[0]);
-    const double dy = __dadd_rn(__dsub_rn(xj[1], xi1), S[1]);
-    const double dz = __dadd_rn(__dsub_rn(xj[2], xi2), S[2]);
-    const double r2 = __dadd_rn(__dadd_rn(__dmul_rn(dx, dx), __dmul_rn(dy, dy)), __dmul_rn(dz, dz));
-    if (r2 < rc2) {
-      const int pos = atomicAdd(&s_cnt, 1);
-      if (pos < NL_CAP) {
-        c_r2[pos] = r2;
-        c_j[pos] = j;
-        c_s[pos] = ((ia + SHIFT_OFF) * SHIFT_BASE + (ib + SHIFT_OFF)) * SHIFT_BASE + (ic + SHIFT_OFF);
-        c_t[pos] = types[j];
+    const int sid = ((ia + SHIFT_OFF) * SHIFT_BASE + (ib + SHIFT_OFF)) * SHIFT_BASE + (ic + SHIFT_OFF);
+    const bool self_shift = ia == 0 && ib == 0 && ic == 0;
+    for (int j = tid; j < Na; j += NL_THREADS) {
+      if (j == i && self_shift) continue;
+      const double* xj = coord + ((size_t)b * Na + j) * 3;
+      const double dx = __dadd_rn(__dsub_rn(xj[0], xi0), S[0]);
+      const double dy = __dadd_rn(__dsub_rn(xj[1], xi1), S[1]);
+      const double dz = __dadd_rn(__dsub_rn(xj[2], xi2), S[2]);
+      const double r2 = __dadd_rn(__dadd_rn(__dmul_rn(dx, dx), __dmul_rn(dy, dy)), __dmul_rn(dz, dz));
+      if (r2 < rc2) {
+        const int pos = atomicAdd(&s_cnt, 1);
+        if (pos < NL_CAP) {
+          c_r2[pos] = r2;
+          c_j[pos] = j;
+          c_s[pos] = sid;
+          c_t[pos] = types[j];
+        }
       }
     }
   }
