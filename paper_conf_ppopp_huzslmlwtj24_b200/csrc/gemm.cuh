@@ -326,17 +326,22 @@ dgemm_kernel(const __grid_constant__ GemmGroup<Epi> G) {
 #ifdef FEKF_NETS32
 // fp32 nets: the same GEMM on the FP32 FFMA pipe (measured 71.5 TFLOP/s on B200, vs 34.6 for an
 // fp32-accurate product on the split-tf32 mma.sync pair; tools/fp32_peak.cu).  256 threads as a 16 x 16
-// grid, each a TM x TN register micro-tile (TM = BM/16 consecutive rows, TN = BN/16 columns strided by 16);
-// both operands staged k-major in SMEM, [k][m] and [k][n] (row stride MN + 4), so a thread's TM rows are
-// TM/4 LDS.128 broadcasts and its columns conflict-free LDS.32 across the 16 column threads.  The
-// operands stored k-contiguous (A row-major, B given as [N x K]) are transposed on the way in by
-// element-wise cp.async (4 bytes each, from coalesced global reads).  Same GemmGroup / split-K / device
-// row-count / "ones" row semantics as dgemm_kernel; the epilogue gets every element of the micro-tile.
+// grid, each a TM x TN register micro-tile (TM = BM/16 rows, TN = BN/16 columns strided by 16), the k loop
+// four at a time.  Operands stay in SMEM in their global orientation: an operand contiguous along k (A
+// row-major, B given as [N x K]) as [row][k] (stride BK + 4, 16-byte cp.async; a thread's rows strided by
+// 16 so the two row groups of a warp hit different banks), one contiguous along m / n as [k][mn] (stride
+// MN + 4; A's TM rows of a thread consecutive and read as float4 along m).  Same GemmGroup / split-K /
+// device row-count / "ones" row semantics as dgemm_kernel; the epilogue gets every element of the tile.
+__device__ __forceinline__ void cp_async16n(float* dst, const float* src, int nbytes) {
+  const unsigned d = (unsigned)__cvta_generic_to_shared(dst);
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(d), "l"(src), "r"(nbytes) : "memory");
+}
 template <int BM, int BN, bool TA, bool TB, class Epi>
 __global__ void __launch_bounds__(256)
 sgemm_kernel(const __grid_constant__ GemmGroup<Epi> G) {
-  constexpr int NT = 256, TM = BM / 16, TN = BN / 16, LA = BM + 4, LB = BN + 4;
-  constexpr int ASZ = GB_K * LA, BSZ = GB_K * LB;
+  constexpr int NT = 256, TM = BM / 16, TN = BN / 16, LK = GB_K + 4, LA = BM + 4, LB = BN + 4;
+  constexpr bool AK = !TA, BK = TB;   // operand contiguous along k
+  constexpr int ASZ = AK ? BM * LK : GB_K * LA, BSZ = BK ? BN * LK : GB_K * LB;
   static_assert(TM % 4 == 0 && BN % 16 == 0, "sgemm micro-tile");
   extern __shared__ __align__(16) real gsm[];
   real* As0 = gsm;
@@ -375,58 +380,73 @@ sgemm_kernel(const __grid_constant__ GemmGroup<Epi> G) {
   for (int i = 0; i < TM; ++i)
 #pragma unroll
     for (int j = 0; j < TN; ++j) acc[i][j] = 0.f;
-  // two-element copies along m (TA) / n (!TB) when strides and bases allow
   const int mreal = aug_m >= 0 ? min(M, aug_m) : M;
-  const bool a2 = TA && !(lda & 1) && !(reinterpret_cast<size_t>(A) & PAIR_MASK);
-  const bool b2 = !TB && !(ldb & 1) && !(reinterpret_cast<size_t>(B) & PAIR_MASK) && !(N & 1);
+  // 16-byte copies along k when the row stride, the base and the split's first k are 16-byte aligned (slices
+  // advance by GB_K); a ragged end of K is zero-filled by the copy's source size
+  const bool a4 = AK && aug_m < 0 && !(lda & 3) && !(reinterpret_cast<size_t>(A) & 15) && !(kbeg & 3);
+  const bool b4 = BK && !(ldb & 3) && !(reinterpret_cast<size_t>(B) & 15) && !(kbeg & 3);
+  const bool a2 = !AK && !(lda & 1) && !(reinterpret_cast<size_t>(A) & PAIR_MASK);
+  const bool b2 = !BK && !(ldb & 1) && !(reinterpret_cast<size_t>(B) & PAIR_MASK) && !(N & 1);
   auto issue = [&](int buf, int k0) {
     real* As = As0 + buf * ASZ;
     real* Bs = Bs0 + buf * BSZ;
-    if (TA) {   // A stored [K x M]: rows of m, straight
-      if (a2) {
-        for (int idx = tid; idx < GB_K * BM / 2; idx += NT) {
-          const int kk = idx / (BM / 2), r = 2 * (idx % (BM / 2));
+    if (AK) {   // A row-major [M x K] -> [m][k]
+      if (a4) {
+        for (int idx = tid; idx < BM * GB_K / 4; idx += NT) {
+          const int r = idx / (GB_K / 4), kk = 4 * (idx % (GB_K / 4));
           const int m = m0 + r, k = k0 + kk;
-          const bool kin = k < kend;
-          if (m + 1 < mreal) {
-            cp_async2(As + kk * LA + r, kin ? A + (size_t)k * lda + m : A, kin);
-          } else {
-#pragma unroll
-            for (int h = 0; h < 2; ++h) {
-              real* dst = As + kk * LA + r + h;
-              if (m + h == aug_m) *dst = (k < aug_k) ? real(1) : real(0);
-              else {
-                const bool ok = m + h < M && kin;
-                cp_async1(dst, ok ? A + (size_t)k * lda + m + h : A, ok);
-              }
-            }
-          }
+          const int nb = (m < M && k < kend) ? 4 * min(4, kend - k) : 0;
+          cp_async16n(As + r * LK + kk, nb ? A + (size_t)m * lda + k : A, nb);
         }
       } else {
-        for (int idx = tid; idx < GB_K * BM; idx += NT) {
-          const int kk = idx / BM, r = idx % BM;
+        for (int idx = tid; idx < BM * GB_K; idx += NT) {
+          const int r = idx / GB_K, kk = idx % GB_K;
           const int m = m0 + r, k = k0 + kk;
-          real* dst = As + kk * LA + r;
+          real* dst = As + r * LK + kk;
           if (m == aug_m) *dst = (k < aug_k) ? real(1) : real(0);
           else {
             const bool ok = m < M && k < kend;
-            cp_async1(dst, ok ? A + (size_t)k * lda + m : A, ok);
+            cp_async1(dst, ok ? A + (size_t)m * lda + k : A, ok);
           }
         }
       }
-    } else {   // A row-major [M x K]: coalesced along k, transposed into [k][m]
-      for (int idx = tid; idx < GB_K * BM; idx += NT) {
-        const int r = idx / GB_K, kk = idx % GB_K;
+    } else {    // A stored [K x M] -> [k][m]
+      for (int idx = tid; idx < GB_K * BM / 2; idx += NT) {
+        const int kk = idx / (BM / 2), r = 2 * (idx % (BM / 2));
         const int m = m0 + r, k = k0 + kk;
-        real* dst = As + kk * LA + r;
-        if (m == aug_m) *dst = (k < aug_k) ? real(1) : real(0);
-        else {
-          const bool ok = m < M && k < kend;
-          cp_async1(dst, ok ? A + (size_t)m * lda + k : A, ok);
+        const bool kin = k < kend;
+        if (a2 && m + 1 < mreal) {
+          cp_async2(As + kk * LA + r, kin ? A + (size_t)k * lda + m : A, kin);
+        } else {
+#pragma unroll
+          for (int h = 0; h < 2; ++h) {
+            real* dst = As + kk * LA + r + h;
+            if (m + h == aug_m) *dst = (k < aug_k) ? real(1) : real(0);
+            else {
+              const bool ok = m + h < M && kin;
+              cp_async1(dst, ok ? A + (size_t)k * lda + m + h : A, ok);
+            }
+          }
         }
       }
     }
-    if (!TB) {   // B row-major [K x N]: straight
+    if (BK) {   // B given as [N x K] -> [n][k]
+      if (b4) {
+        for (int idx = tid; idx < BN * GB_K / 4; idx += NT) {
+          const int c = idx / (GB_K / 4), kk = 4 * (idx % (GB_K / 4));
+          const int n = n0 + c, k = k0 + kk;
+          const int nb = (n < N && k < kend) ? 4 * min(4, kend - k) : 0;
+          cp_async16n(Bs + c * LK + kk, nb ? B + (size_t)n * ldb + k : B, nb);
+        }
+      } else {
+        for (int idx = tid; idx < BN * GB_K; idx += NT) {
+          const int c = idx / GB_K, kk = idx % GB_K;
+          const int n = n0 + c, k = k0 + kk;
+          const bool ok = n < N && k < kend;
+          cp_async1(Bs + c * LK + kk, ok ? B + (size_t)n * ldb + k : B, ok);
+        }
+      }
+    } else {    // B row-major [K x N] -> [k][n]
       if (b2) {
         for (int idx = tid; idx < GB_K * BN / 2; idx += NT) {
           const int kk = idx / (BN / 2), c = 2 * (idx % (BN / 2));
@@ -442,15 +462,10 @@ sgemm_kernel(const __grid_constant__ GemmGroup<Epi> G) {
           cp_async1(Bs + kk * LB + c, ok ? B + (size_t)k * ldb + n : B, ok);
         }
       }
-    } else {   // B given as [N x K]: coalesced along k, transposed into [k][n]
-      for (int idx = tid; idx < GB_K * BN; idx += NT) {
-        const int c = idx / GB_K, kk = idx % GB_K;
-        const int n = n0 + c, k = k0 + kk;
-        const bool ok = n < N && k < kend;
-        cp_async1(Bs + kk * LB + c, ok ? B + (size_t)n * ldb + k : B, ok);
-      }
     }
   };
+  // the thread's rows: AK strided by 16 (conflict-free float4 along k), else TM consecutive (float4 along m)
+  auto row_of = [&](int i) { return AK ? ty + 16 * i : ty * TM + i; };
   const int nk = kend > kbeg ? (kend - kbeg + GB_K - 1) / GB_K : 0;
 #pragma unroll
   for (int st = 0; st < GB_STAGES - 1; ++st) {
@@ -463,22 +478,40 @@ sgemm_kernel(const __grid_constant__ GemmGroup<Epi> G) {
     const int tn = t + GB_STAGES - 1;
     if (tn < nk) issue(tn % GB_STAGES, kbeg + tn * GB_K);
     cp_async_commit();
-    const real* As = As0 + (t % GB_STAGES) * ASZ + ty * TM;
-    const real* Bs = Bs0 + (t % GB_STAGES) * BSZ + tx;
+    const real* As = As0 + (t % GB_STAGES) * ASZ;
+    const real* Bs = Bs0 + (t % GB_STAGES) * BSZ;
 #pragma unroll
-    for (int kk = 0; kk < GB_K; ++kk) {
-      real a[TM], b[TN];
+    for (int k4 = 0; k4 < GB_K; k4 += 4) {
+      real a[TM][4], b[TN][4];
 #pragma unroll
-      for (int i = 0; i < TM; i += 4) {
-        const float4 v = *reinterpret_cast<const float4*>(As + kk * LA + i);
-        a[i] = v.x; a[i + 1] = v.y; a[i + 2] = v.z; a[i + 3] = v.w;
+      for (int i = 0; i < TM; ++i) {
+        if (AK) {
+          const float4 v = *reinterpret_cast<const float4*>(As + row_of(i) * LK + k4);
+          a[i][0] = v.x; a[i][1] = v.y; a[i][2] = v.z; a[i][3] = v.w;
+        } else if (i % 4 == 0) {
+#pragma unroll
+          for (int u = 0; u < 4; ++u) {
+            const float4 v = *reinterpret_cast<const float4*>(As + (k4 + u) * LA + ty * TM + i);
+            a[i][u] = v.x; a[i + 1][u] = v.y; a[i + 2][u] = v.z; a[i + 3][u] = v.w;
+          }
+        }
       }
 #pragma unroll
-      for (int j = 0; j < TN; ++j) b[j] = Bs[kk * LB + 16 * j];
+      for (int j = 0; j < TN; ++j) {
+        if (BK) {
+          const float4 v = *reinterpret_cast<const float4*>(Bs + (tx + 16 * j) * LK + k4);
+          b[j][0] = v.x; b[j][1] = v.y; b[j][2] = v.z; b[j][3] = v.w;
+        } else {
 #pragma unroll
-      for (int i = 0; i < TM; ++i)
+          for (int u = 0; u < 4; ++u) b[j][u] = Bs[(k4 + u) * LB + tx + 16 * j];
+        }
+      }
 #pragma unroll
-        for (int j = 0; j < TN; ++j) acc[i][j] = fmaf(a[i], b[j], acc[i][j]);
+      for (int u = 0; u < 4; ++u)
+#pragma unroll
+        for (int i = 0; i < TM; ++i)
+#pragma unroll
+          for (int j = 0; j < TN; ++j) acc[i][j] = fmaf(a[i][u], b[j][u], acc[i][j]);
     }
   }
   cp_async_wait<0>();
@@ -486,7 +519,7 @@ sgemm_kernel(const __grid_constant__ GemmGroup<Epi> G) {
   for (int i = 0; i < TM; ++i)
 #pragma unroll
     for (int j = 0; j < TN; ++j) {
-      const int r = m0 + ty * TM + i, c = n0 + tx + 16 * j;
+      const int r = m0 + row_of(i), c = n0 + tx + 16 * j;
       if (r < M && c < N) epi(r, c, acc[i][j]);
     }
 }
@@ -495,7 +528,8 @@ sgemm_kernel(const __grid_constant__ GemmGroup<Epi> G) {
 template <int BM, int BN, int WM, int WN, bool TA, bool TB, class Epi, int NW = 8>
 static fekf_status gemm_launch(GemmGroup<Epi>& G, cudaStream_t s) {
 #ifdef FEKF_NETS32
-  constexpr size_t smem = sizeof(real) * GB_STAGES * GB_K * ((BM + 4) + (BN + 4));
+  constexpr size_t smem = sizeof(real) * GB_STAGES * ((TA ? GB_K * (BM + 4) : BM * (GB_K + 4)) +
+                                                      (TB ? BN * (GB_K + 4) : GB_K * (BN + 4)));
   auto kern = sgemm_kernel<BM, BN, TA, TB, Epi>;
   constexpr int nthr = 256;
 #else

@@ -197,7 +197,7 @@ def _train_fp32(m, opt, ds, w0, B, steps):
     ctx.close()
 
 
-@pytest.mark.parametrize("emb", [[6, 12], [5, 10, 20], [8, 8, 8, 8]])
+@pytest.mark.parametrize("emb", [[6, 12], [5, 10, 20], [8, 8, 8, 8], [4, 12, 36]])
 def test_fp32_unfused_embedding_widths(emb):
     """fp32 per-layer embedding path (FFMA GEMMs with the activation-adjoint epilogues, the layer-0 and seed
     kernels, prod_force) and the MODE_FORCE fallback: forward, both Jacobians, 3 steps (fp32 P too)."""
