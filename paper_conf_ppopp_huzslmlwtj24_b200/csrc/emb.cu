@@ -329,7 +329,8 @@ static fekf_status emb_forward_t(Ctx& c, int p, long long Rmax, bool tangent, cu
   auto launch = [&](auto kern, int nw) -> fekf_status {
     const size_t smem = sizeof(real) * (W::WS + (size_t)nw * W::WRP);
     FEKF_CHECK_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-    const int grid = (int)std::max<long long>(1, std::min<long long>((wtiles + nw - 1) / nw, (long long)num_sms()));
+    const int sms = c.emb_grid_cap > 0 ? std::min(c.emb_grid_cap, num_sms()) : num_sms();
+    const int grid = (int)std::max<long long>(1, std::min<long long>((wtiles + nw - 1) / nw, (long long)sms));
     kern<<<grid, nw * 32, smem, s>>>(wp, io);
     return FEKF_OK;
   };
@@ -739,7 +740,8 @@ static fekf_status emb_backward_t(Ctx& c, int p, long long Rmax, int mode, doubl
     io.Yt[l] = P.Yt[l].as<real>();
     io.Hbt[l] = P.Hbt[l].as<real>();
   }
-  const int cap = (int)std::min<size_t>(1 << 20, c.splitk_elems / (2 * (size_t)W::GS));
+  int cap = (int)std::min<size_t>(1 << 20, c.splitk_elems / (2 * (size_t)W::GS));
+  if (c.emb_grid_cap > 0) cap = std::min(cap, c.emb_grid_cap);
   const int sms = c.emb_sms > 0 ? c.emb_sms : num_sms();   // split P pass: the SMs it leaves free
   real* ws = c.splitk_ws.as<real>();
   int nsets = 0;

@@ -100,6 +100,12 @@ struct Ctx {
   cudaEvent_t ev_fit = nullptr;
   bool split_armed = false;
   int emb_sms = 0;
+  // per-pair concurrency of the embedding launches on the step's critical path (primal / tangent forward,
+  // the force-only reverse): one stream per type pair, each launch's persistent grid capped at its share of
+  // the SMs (emb_grid_cap, 0 = no cap) so the pairs run side by side instead of back to back
+  std::vector<cudaStream_t> pstreams;
+  std::vector<cudaEvent_t> pev;      // [0] fork, [1 + p] join of pair p
+  int emb_grid_cap = 0;
   cudaEvent_t gev_in = nullptr, gev_out = nullptr;
   DBuf st_coord, st_box, st_e, st_f, st_fidx, st_met;
   int64_t nsteps = 0;

@@ -1466,6 +1466,48 @@ fekf_status mark_selected(Ctx& c, int nb, const int* atom_idx, int n_sel, cudaSt
   return FEKF_OK;
 }
 
+// The embedding launches of every type pair side by side (one stream per pair, forked from and joined back
+// into s), each persistent grid capped at the pair's share of the SMs by its row bound; serial when the
+// context has no pair streams.  fn(p, stream) issues pair p's launch.
+template <class Fn>
+static fekf_status pairs_concurrent(Ctx& c, int nb, cudaStream_t s, Fn fn) {
+  const int np = (int)c.pairs.size();
+  long long tot = 0;
+  int live = 0;
+  for (int p = 0; p < np; ++p) {
+    const long long r = pair_rows(c, p, nb);
+    tot += r;
+    live += r > 0;
+  }
+  if (c.pstreams.empty() || live < 2) {
+    for (int p = 0; p < np; ++p)
+      if (pair_rows(c, p, nb) > 0) FEKF_TRY(fn(p, s));
+    return FEKF_OK;
+  }
+  static int sms = 0;
+  if (!sms) {
+    int dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    if (sms <= 0) sms = 148;
+  }
+  FEKF_CHECK_CUDA(cudaEventRecord(c.pev[0], s));
+  for (int p = 0; p < np; ++p) {
+    const long long r = pair_rows(c, p, nb);
+    if (r == 0) continue;
+    cudaStream_t ps = c.pstreams[p];
+    FEKF_CHECK_CUDA(cudaStreamWaitEvent(ps, c.pev[0], 0));
+    c.emb_grid_cap = (int)std::max<long long>(1, (long long)sms * r / tot);
+    const fekf_status st = fn(p, ps);
+    c.emb_grid_cap = 0;
+    FEKF_TRY(st);
+    FEKF_CHECK_CUDA(cudaEventRecord(c.pev[1 + p], ps));
+  }
+  for (int p = 0; p < np; ++p)
+    if (pair_rows(c, p, nb) > 0) FEKF_CHECK_CUDA(cudaStreamWaitEvent(s, c.pev[1 + p], 0));
+  return FEKF_OK;
+}
+
 // fp32 nets: fp32 copies of the fp64 inputs (R~, its Jacobian, d: once per geometry; the weights: before
 // every primal forward, i.e. after every Kalman update)
 __global__ void to_real_kernel(const double* __restrict__ src, real* __restrict__ dst, long long n) {
@@ -1502,14 +1544,14 @@ fekf_status model_forward(Ctx& c, int nb, bool tangent, cudaStream_t s) {
   if (tangent) c.trows_ready = false;
   // embedding nets (compacted rows)
   const bool fused = emb_fused_ok(c);
-  for (size_t p = 0; p < c.pairs.size(); ++p) {
+  if (fused)
+    FEKF_TRY(pairs_concurrent(c, nb, s, [&](int p, cudaStream_t ps) {
+      return emb_forward(c, p, pair_rows(c, p, nb), tangent, ps);
+    }));
+  for (size_t p = 0; p < c.pairs.size() && !fused; ++p) {
     PairNet& P = c.pairs[p];
     const long long Rmax = pair_rows(c, (int)p, nb);
     if (Rmax == 0) continue;
-    if (fused) {
-      FEKF_TRY(emb_forward(c, (int)p, Rmax, tangent, s));
-      continue;
-    }
     const int* cnt = tangent ? tcount(c, (int)p) : rcount(c, (int)p);
     real* hin = tangent ? P.hin_t.as<real>() : P.hin.as<real>();
     emb_input_kernel<<<cdiv(Rmax, 256), 256, 0, s>>>((int)Rmax, cnt, P.row_idx.as<int>(),
@@ -1764,10 +1806,16 @@ fekf_status model_backward(Ctx& c, int nb, Mode mode, double* gout, cudaStream_t
   count_launch();
   // ---- embedding nets (compacted rows; tangent rows separately) ----
   if (emb_fused_ok(c)) {
-    for (size_t p = 0; p < c.pairs.size(); ++p) {
-      const long long Rmax = pair_rows(c, (int)p, nb);
-      if (Rmax == 0) continue;
-      FEKF_TRY(emb_backward(c, (int)p, Rmax, (int)mode, gout, s));
+    if (force) {   // force-only reverse (no weight gradients): on the critical path, pairs side by side
+      FEKF_TRY(pairs_concurrent(c, nb, s, [&](int p, cudaStream_t ps) {
+        return emb_backward(c, p, pair_rows(c, p, nb), (int)mode, gout, ps);
+      }));
+    } else {
+      for (size_t p = 0; p < c.pairs.size(); ++p) {
+        const long long Rmax = pair_rows(c, (int)p, nb);
+        if (Rmax == 0) continue;
+        FEKF_TRY(emb_backward(c, (int)p, Rmax, (int)mode, gout, s));
+      }
     }
   } else {
   {
