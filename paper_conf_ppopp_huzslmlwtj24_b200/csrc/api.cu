@@ -256,7 +256,7 @@ fekf_status Ctx::init(const fekf_model_cfg& mm, const fekf_opt_cfg& oo, int nato
   int maxh = 1;
   for (int l = 0; l < m.n_fit; ++l) maxh = std::max(maxh, m.fit[l]);
   colsum_elems = (size_t)(2 * 148 + 2) * maxh;   // act_bwd_dt: at most 2 x 148 row chunks
-  FEKF_TRY(dalloc(colsum_ws, sizeof(double) * colsum_elems));
+  FEKF_TRY(dalloc(colsum_ws, sizeof(double) * colsum_elems * nt));   // one region per atom type
 
   pairs.clear();
   for (int ti = 0; ti < nt; ++ti)

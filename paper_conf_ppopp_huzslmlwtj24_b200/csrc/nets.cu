@@ -193,25 +193,44 @@ static fekf_status wgrad_group(Ctx& c, WgradJob* jobs, int n, cudaStream_t s) {
 // elementwise / small kernels
 // =================================================================================================
 // fitting (stacked rows): zbar = (1 - y^2) ybar - 2 y ydot ydotbar, zdotbar = (1 - y^2) ydotbar;
-// ybar = dt * hbar on residual layers with a timestep vector, else hbar.
-__global__ void act_bwd_kernel(long long R, int d, const real* __restrict__ Y, const real* __restrict__ Hb,
-                               const real* __restrict__ dt, int dual, real* __restrict__ Zb) {
+// ybar = dt * hbar on residual layers with a timestep vector, else hbar.  One launch for every atom type of
+// a layer (blockIdx.y = type; the types' layers have the same widths).
+constexpr int MT = FEKF_MAX_TYPES;
+struct ActArgs {
+  long long R[MT];                  // primal rows per type (the tangent half follows at R)
+  const real* Y[MT];
+  const real* Hb[MT];
+  const real* dt[MT];               // timestep vector or nullptr
+  real* Zb[MT];
+  real* ws[MT];                     // act_bwd_dt: per-type column-partial workspace
+  double* gdt[MT];                  // act_bwd_dt: the timestep gradient (in g)
+  int chunk[MT], nchunk[MT];
+  int d, dual;
+};
+__global__ void act_bwd_kernel(const __grid_constant__ ActArgs A) {
+  const int t = blockIdx.y;
   const long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x;
+  const long long R = A.R[t];
+  const int d = A.d;
   if (i >= R * d) return;
   const int c = (int)(i % d);
+  const real* __restrict__ Y = A.Y[t];
+  const real* __restrict__ Hb = A.Hb[t];
+  const real* __restrict__ dt = A.dt[t];
+  real* __restrict__ Zb = A.Zb[t];
   const real y = Y[i];
-  const real t = real(1) - y * y;
+  const real tt = real(1) - y * y;
   real yb = Hb[i];
   if (dt) yb *= dt[c];
-  if (dual) {
+  if (A.dual) {
     const size_t j = (size_t)R * d + i;
     const real yd = Y[j];
     real ydb = Hb[j];
     if (dt) ydb *= dt[c];
-    Zb[i] = t * yb - real(2) * y * yd * ydb;
-    Zb[j] = t * ydb;
+    Zb[i] = tt * yb - real(2) * y * yd * ydb;
+    Zb[j] = tt * ydb;
   } else {
-    Zb[i] = t * yb;
+    Zb[i] = tt * yb;
   }
 }
 
@@ -242,13 +261,20 @@ __global__ void emb_act_bwd_kernel(int Rmax, const int* __restrict__ Rdev, int d
 
 // act_bwd fused with the timestep gradient of the layer (two fixed-order stages):
 //   dt[c] = sum_r y[r][c] hbar[r][c] + sum_r ydot[r][c] hdotbar[r][c]   (h = skip + dt * y)
-// block b: rows [b chunk, (b+1) chunk) of the primal half (and the same rows of the tangent half), one
-// thread per column (coalesced rows); the per-block sums go to ws[b][c] and colsum_reduce adds them.
-__global__ void act_bwd_dt_kernel(long long R, int d, const real* __restrict__ Y, const real* __restrict__ Hb,
-                                  const real* __restrict__ dt, int dual, real* __restrict__ Zb, int chunk,
-                                  real* __restrict__ ws) {
+// block (b, type): rows [b chunk, (b+1) chunk) of the type's primal half (and the same rows of its tangent
+// half), one thread per column (coalesced rows); the per-block sums go to ws[type][b][c] and colsum_reduce
+// adds them.
+__global__ void act_bwd_dt_kernel(const __grid_constant__ ActArgs A) {
+  const int t = blockIdx.y;
+  if ((int)blockIdx.x >= A.nchunk[t]) return;
+  const long long R = A.R[t];
+  const int d = A.d, chunk = A.chunk[t];
   const long long r0 = (long long)blockIdx.x * chunk;
   const long long r1 = min(R, r0 + chunk);
+  const real* __restrict__ Y = A.Y[t];
+  const real* __restrict__ Hb = A.Hb[t];
+  const real* __restrict__ dt = A.dt[t];
+  real* __restrict__ Zb = A.Zb[t];
   for (int c = threadIdx.x; c < d; c += blockDim.x) {
     const real dtc = dt[c];
     real acc = 0.0;
@@ -256,27 +282,29 @@ __global__ void act_bwd_dt_kernel(long long R, int d, const real* __restrict__ Y
     for (long long r = r0; r < r1; ++r) {
       const size_t i = (size_t)r * d + c;
       const real y = Y[i], hb = Hb[i];
-      const real t = real(1) - y * y;
+      const real tt = real(1) - y * y;
       acc += y * hb;
-      if (dual) {
+      if (A.dual) {
         const size_t j = (size_t)R * d + i;
         const real yd = Y[j], hdb = Hb[j];
         const real ydb = hdb * dtc;
-        Zb[i] = t * (hb * dtc) - real(2) * y * yd * ydb;
-        Zb[j] = t * ydb;
+        Zb[i] = tt * (hb * dtc) - real(2) * y * yd * ydb;
+        Zb[j] = tt * ydb;
         acc += yd * hdb;
       } else {
-        Zb[i] = t * (hb * dtc);
+        Zb[i] = tt * (hb * dtc);
       }
     }
-    ws[(size_t)blockIdx.x * d + c] = acc;
+    A.ws[t][(size_t)blockIdx.x * d + c] = acc;
   }
 }
-// out[c] = sum_k ws[k][c]: 32 columns x 8 chunk-lanes per CTA, fixed 8-way combine
-__global__ void colsum_reduce_kernel(const real* __restrict__ ws, int nchunk, int d, double* __restrict__ out) {
+// out[c] = sum_k ws[k][c]: 32 columns x 8 chunk-lanes per CTA, fixed 8-way combine (blockIdx.y = type)
+__global__ void colsum_reduce_kernel(const __grid_constant__ ActArgs A) {
   __shared__ real red[8][33];
+  const int t = blockIdx.y;
   const int cl = threadIdx.x & 31, z = threadIdx.x >> 5;
-  const int c = blockIdx.x * 32 + cl;
+  const int c = blockIdx.x * 32 + cl, d = A.d, nchunk = A.nchunk[t];
+  const real* __restrict__ ws = A.ws[t];
   real a = 0.0;
   if (c < d) {
 #pragma unroll 4
@@ -285,21 +313,35 @@ __global__ void colsum_reduce_kernel(const real* __restrict__ ws, int nchunk, in
   red[z][cl] = a;
   __syncthreads();
   if (z == 0 && c < d) {
-    real t = red[0][cl];
+    real v = red[0][cl];
 #pragma unroll
-    for (int q = 1; q < 8; ++q) t += red[q][cl];
-    out[c] = t;
+    for (int q = 1; q < 8; ++q) v += red[q][cl];
+    A.gdt[t][c] = v;
   }
 }
-static fekf_status act_bwd_dt(Ctx& c, long long R, int d, const real* Y, const real* Hb, const real* dt,
-                              bool dual, real* Zb, double* gdt, cudaStream_t s) {
-  const int chunk = (int)std::max<long long>(4, cdiv(R, 2 * 148));
-  const int nchunk = (int)cdiv(R, chunk);
-  if ((size_t)nchunk * d > c.colsum_elems) { set_error("colsum workspace too small"); return FEKF_EINVAL; }
-  act_bwd_dt_kernel<<<nchunk, std::min(256, (d + 31) / 32 * 32), 0, s>>>(R, d, Y, Hb, dt, dual ? 1 : 0, Zb, chunk,
-                                                                         c.colsum_ws.as<real>());
+// the activation adjoint of one fitting layer for every type (and, with timestep vectors and weight
+// gradients wanted, the timestep gradients); A's per-type pointers and R filled by the caller
+static fekf_status act_bwd_types(Ctx& c, ActArgs& A, int nt, bool with_dt, cudaStream_t s) {
+  long long Rmax = 0;
+  for (int t = 0; t < nt; ++t) Rmax = std::max(Rmax, A.R[t]);
+  if (Rmax == 0) return FEKF_OK;
+  if (!with_dt) {
+    act_bwd_kernel<<<dim3(cdiv(Rmax * A.d, 256), nt), 256, 0, s>>>(A);
+    FEKF_LAUNCH_CHECK();
+    count_launch();
+    return FEKF_OK;
+  }
+  int cmax = 1;
+  for (int t = 0; t < nt; ++t) {
+    A.chunk[t] = (int)std::max<long long>(4, cdiv(A.R[t], 2 * 148));
+    A.nchunk[t] = A.R[t] > 0 ? (int)cdiv(A.R[t], A.chunk[t]) : 0;
+    if ((size_t)A.nchunk[t] * A.d > c.colsum_elems) { set_error("colsum workspace too small"); return FEKF_EINVAL; }
+    A.ws[t] = c.colsum_ws.as<real>() + (size_t)t * c.colsum_elems;
+    cmax = std::max(cmax, A.nchunk[t]);
+  }
+  act_bwd_dt_kernel<<<dim3(cmax, nt), std::min(256, (A.d + 31) / 32 * 32), 0, s>>>(A);
   FEKF_LAUNCH_CHECK();
-  colsum_reduce_kernel<<<cdiv(d, 32), 256, 0, s>>>(c.colsum_ws.as<real>(), nchunk, d, gdt);
+  colsum_reduce_kernel<<<dim3(cdiv(A.d, 32), nt), 256, 0, s>>>(A);
   FEKF_LAUNCH_CHECK();
   count_launch(2);
   return FEKF_OK;
@@ -1158,23 +1200,37 @@ __global__ void virial_reduce_kernel(const double* __restrict__ vatom, int Na, d
   virial[(size_t)b * 9 + q] = a;
 }
 
-// E_i = h_F W_out + b_out (primal rows), Edot_i = hdot_F W_out (tangent rows); one warp per row
-__global__ void fit_out_kernel(long long rows, long long F, int h, const real* __restrict__ H,
-                               const real* __restrict__ W, const real* __restrict__ bout, real* __restrict__ out) {
+// E_i = h_F W_out + b_out (primal rows), Edot_i = hdot_F W_out (tangent rows); one warp per row; every type
+// in one launch (blockIdx.y = type)
+struct OutArgs {
+  long long rows[MT], F[MT];
+  const real* H[MT];
+  const real* W[MT];
+  const real* b[MT];
+  real* out[MT];
+  const real* ebar[MT];
+  real* Hb[MT];
+  int h;
+};
+__global__ void fit_out_kernel(const __grid_constant__ OutArgs A) {
+  const int t = blockIdx.y;
   const long long r = ((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-  const int lane = threadIdx.x & 31;
-  if (r >= rows) return;
+  const int lane = threadIdx.x & 31, h = A.h;
+  if (r >= A.rows[t]) return;
+  const real* __restrict__ H = A.H[t];
+  const real* __restrict__ W = A.W[t];
   real a = 0.0;
   for (int c = lane; c < h; c += 32) a = fma(H[(size_t)r * h + c], W[c], a);
   for (int o = 16; o > 0; o >>= 1) a += __shfl_xor_sync(0xffffffffu, a, o);
-  if (lane == 0) out[r] = a + (r < F ? bout[0] : real(0));
+  if (lane == 0) A.out[t][r] = a + (r < A.F[t] ? A.b[t][0] : real(0));
 }
 // adjoint of h_F from the output seeds: Hbar = ebar (x) W_out
-__global__ void fit_out_bwd_kernel(long long rows, int h, const real* __restrict__ ebar, const real* __restrict__ W,
-                                   real* __restrict__ Hb) {
+__global__ void fit_out_bwd_kernel(const __grid_constant__ OutArgs A) {
+  const int t = blockIdx.y;
   const long long e = (long long)blockIdx.x * blockDim.x + threadIdx.x;
-  if (e >= rows * h) return;
-  Hb[e] = ebar[e / h] * W[e % h];
+  const int h = A.h;
+  if (e >= A.rows[t] * h) return;
+  A.Hb[t][e] = A.ebar[t][e / h] * A.W[t][e % h];
 }
 
 // per-atom energies back into [nb][Na] and E_b = sum_i E_i, fixed order
@@ -1624,17 +1680,28 @@ fekf_status model_forward(Ctx& c, int nb, bool tangent, cudaStream_t s) {
     }
     FEKF_TRY(gemm_group<false, false>(pr, n, s));
   }
-  for (int t = 0; t < c.nt; ++t) {
-    FitNet& Fn = c.fits[t];
-    const long long F = fit_rows(c, t, nb);
-    if (F == 0) continue;
-    const int h = Fn.L.back().dout;
-    const real* Hl = Fn.H.back().as<real>();
-    real* eo = Fn.eout.as<real>();
-    fit_out_kernel<<<cdiv(F * 32, 256), 256, 0, s>>>(F, F, h, tangent ? Hl + (size_t)F * h : Hl, w + Fn.Wout, w + Fn.bout,
-                                                      tangent ? eo + F : eo);
-    FEKF_LAUNCH_CHECK();
-    count_launch();
+  {
+    OutArgs A{};
+    long long Fmax = 0;
+    A.h = c.fits[0].L.back().dout;
+    for (int t = 0; t < c.nt; ++t) {
+      FitNet& Fn = c.fits[t];
+      const long long F = fit_rows(c, t, nb);
+      const real* Hl = Fn.H.back().as<real>();
+      real* eo = Fn.eout.as<real>();
+      A.rows[t] = F;
+      A.F[t] = F;
+      A.H[t] = tangent ? Hl + (size_t)F * A.h : Hl;
+      A.W[t] = w + Fn.Wout;
+      A.b[t] = w + Fn.bout;
+      A.out[t] = tangent ? eo + F : eo;
+      Fmax = std::max(Fmax, F);
+    }
+    if (Fmax > 0) {
+      fit_out_kernel<<<dim3(cdiv(Fmax * 32, 256), c.nt), 256, 0, s>>>(A);
+      FEKF_LAUNCH_CHECK();
+      count_launch();
+    }
   }
   return FEKF_OK;
 }
@@ -1717,43 +1784,65 @@ fekf_status model_backward(Ctx& c, int nb, Mode mode, double* gout, cudaStream_t
   FitPtrs fp = make_fp(c, nb);
   // ---- fitting nets (stacked rows); weight and data gradients grouped over types per layer ----
   const size_t nfl = c.fits[0].L.size();
-  for (int t = 0; t < c.nt; ++t) {
-    FitNet& Fn = c.fits[t];
-    const long long F = fit_rows(c, t, nb);
-    if (F == 0) continue;
-    const long long nF = dual ? 2 * F : F;
-    const int h = Fn.L.back().dout;
-    fit_out_bwd_kernel<<<cdiv(nF * h, 256), 256, 0, s>>>(nF, h, Fn.ebar.as<real>(), w + Fn.Wout, Fn.Hb.back().as<real>());
-    FEKF_LAUNCH_CHECK();
-    count_launch();
-    if (want_w) {
-      const real* Hl = Fn.H.back().as<real>();
-      const real* eb = Fn.ebar.as<real>();
-      FEKF_TRY(wgrad(c, h, 1, Seg{Hl, eb, F, nullptr, 1},
-                     Seg{dual ? Hl + (size_t)F * h : nullptr, dual ? eb + F : nullptr, dual ? F : 0, nullptr, 0},
-                     gout + Fn.Wout, s));
+  {
+    // output layer of every type: Hbar = ebar (x) W_out in one launch, [W_out ; b_out] gradients grouped
+    OutArgs A{};
+    WgradJob jobs[FEKF_MAX_TYPES];
+    int nj = 0;
+    long long rmax = 0;
+    const int h = c.fits[0].L.back().dout;
+    A.h = h;
+    for (int t = 0; t < c.nt; ++t) {
+      FitNet& Fn = c.fits[t];
+      const long long F = fit_rows(c, t, nb);
+      A.rows[t] = dual ? 2 * F : F;
+      A.ebar[t] = Fn.ebar.as<real>();
+      A.W[t] = w + Fn.Wout;
+      A.Hb[t] = Fn.Hb.back().as<real>();
+      rmax = std::max(rmax, A.rows[t]);
+      if (want_w && F > 0) {
+        const real* Hl = Fn.H.back().as<real>();
+        const real* eb = Fn.ebar.as<real>();
+        jobs[nj++] = WgradJob{h, 1, Seg{Hl, eb, F, nullptr, 1},
+                              Seg{dual ? Hl + (size_t)F * h : nullptr, dual ? eb + F : nullptr, dual ? F : 0, nullptr, 0},
+                              gout + Fn.Wout};
+      }
     }
+    if (rmax > 0) {
+      fit_out_bwd_kernel<<<dim3(cdiv(rmax * h, 256), c.nt), 256, 0, s>>>(A);
+      FEKF_LAUNCH_CHECK();
+      count_launch();
+    }
+    if (nj) FEKF_TRY(wgrad_group(c, jobs, nj, s));
   }
   for (int l = (int)nfl - 1; l >= 0; --l) {
     WgradJob jobs[FEKF_MAX_TYPES];
     GemmProb<EpiDgrad> dg[GG_MAX];
     int nj = 0, nd = 0;
+    {
+      // the layer's activation adjoint (and timestep gradient) for every type in one launch
+      ActArgs A{};
+      A.d = c.fits[0].L[l].dout;
+      A.dual = dual ? 1 : 0;
+      const bool has_dt = c.fits[0].L[l].dt >= 0;
+      for (int t = 0; t < c.nt; ++t) {
+        FitNet& Fn = c.fits[t];
+        const Layer& L = Fn.L[l];
+        A.R[t] = fit_rows(c, t, nb);
+        A.Y[t] = Fn.Y[l].as<real>();
+        A.Hb[t] = Fn.Hb[l].as<real>();
+        A.dt[t] = has_dt ? w + L.dt : nullptr;
+        A.Zb[t] = Fn.Zb[l].as<real>();
+        A.gdt[t] = has_dt ? gout + L.dt : nullptr;
+      }
+      FEKF_TRY(act_bwd_types(c, A, c.nt, want_w && has_dt, s));
+    }
     for (int t = 0; t < c.nt; ++t) {
       FitNet& Fn = c.fits[t];
       const long long F = fit_rows(c, t, nb);
       if (F == 0) continue;
       const long long nF = dual ? 2 * F : F;
       const Layer& L = Fn.L[l];
-      const real* dt = L.dt >= 0 ? w + L.dt : nullptr;
-      if (want_w && dt) {
-        FEKF_TRY(act_bwd_dt(c, F, L.dout, Fn.Y[l].as<real>(), Fn.Hb[l].as<real>(), dt, dual,
-                            Fn.Zb[l].as<real>(), gout + L.dt, s));
-      } else {
-        act_bwd_kernel<<<cdiv(F * L.dout, 256), 256, 0, s>>>(F, L.dout, Fn.Y[l].as<real>(), Fn.Hb[l].as<real>(),
-                                                              dt, dual ? 1 : 0, Fn.Zb[l].as<real>());
-        FEKF_LAUNCH_CHECK();
-        count_launch();
-      }
       const real* Hprev = l == 0 ? Fn.D.as<real>() : Fn.H[l - 1].as<real>();
       if (want_w) {
         // stacked rows; the ones column covers the primal half only (bias not in the tangent)
