@@ -282,9 +282,10 @@ __device__ __forceinline__ void apply_corrections(PT* t, const double (&ai)[NSTR
 // then u_B = B_new g.  Tile-row segments are pulled from an atomic counter by a producer warp that
 // streams each tile (and its g_J segment, and for rw the 2K 512-byte vector segments it needs) with TMA
 // bulk copies into a ring of `nst` stages (fp64: 6 for read-only passes, fewer when corrections ride
-// along; fp32 tiles are 16 KiB, so twice as many).  `stage_bytes` = tile bytes + (T + K*VS)*8: a stage carries
-// the tile's column segments u_k[J]; the row segments u_k[I] are the same for every tile of an item and are
-// loaded once per item into the consumers' registers (round 1 staged both per tile: 4 stages, now 5).
+// along; fp32 tiles are 16 KiB, so twice as many).  `stage_bytes` = tile bytes + (2T + K*VS)*8: a stage carries
+// the tile's column segments u_k[J] and, on a group's first tile of an item, the item's row segment g_I; the
+// row segments u_k[I] are the same for every tile of an item and are loaded once per item into the
+// consumers' registers (round 1 staged both per tile: 4 stages, now 5).
 //
 // The 8 consumer warps form NG independent groups of 8/NG warps (named barrier 1 + group); group g
 // takes the stages s = g (mod NG), so NG tiles are in flight in the consumers at once.  fp64 uses one
@@ -343,14 +344,19 @@ kf_pass_kernel(PT* __restrict__ P, const ItemD* __restrict__ items, int n_items,
         for (int t = 0; t < it.nJ; ++t) {
           mbar_wait(&empty[s], ph ^ 1);
           // flags: 1 first tile of the item for its group, 2 last one, 4 item shorter than NG tiles
-          meta[s] = make_int4(itx, it.J0 + t, (t < NG ? 1 : 0) | (t >= it.nJ - NG ? 2 : 0) | (it.nJ < NG ? 4 : 0), lst);
+          const bool gfirst = t < NG;   // the group's first tile of the item
+          meta[s] = make_int4(itx, it.J0 + t, (gfirst ? 1 : 0) | (t >= it.nJ - NG ? 2 : 0) | (it.nJ < NG ? 4 : 0), lst);
           unsigned char* st_s = stages + (size_t)s * stage_bytes;
           double* st_g = reinterpret_cast<double*>(st_s + TILE_BYTES);
           double* st_v = st_g + KT;
-          mbar_arrive_tx(&full[s], bytes);
+          mbar_arrive_tx(&full[s], bytes + (gfirst ? KT * sizeof(double) : 0u));
           tma_load_1d(st_s, P + (size_t)(it.tile_off + t) * TILE_ELEMS, TILE_BYTES, &full[s]);
           // g_J rides with its tile: no dependent global load on the consumers' per-tile path
           tma_load_1d(st_g, gpad + it.vbase + (size_t)(it.J0 + t) * KT, KT * sizeof(double), &full[s]);
+          // and g_I with the group's first tile of an item (the row segment its row sums and column
+          // partials need for the whole item): the item start no longer waits on global loads
+          if (gfirst)
+            tma_load_1d(st_v + K * VS, gpad + it.vbase + (size_t)it.I * KT, KT * sizeof(double), &full[s]);
           for (int k = 0; k < K; ++k) {   // the column segments u_k[J] (the row segments u_k[I] of an item
                                             // sit in the consumers' registers)
             const double* uk = ulist + (size_t)k * npad + it.vbase;
@@ -397,9 +403,10 @@ kf_pass_kernel(PT* __restrict__ P, const ItemD* __restrict__ items, int n_items,
     const int J = mt.y;
     const bool first = mt.z & 1, last = mt.z & 2, diag = (J == it.I);
     if (first) {
+      const double* vgi = reinterpret_cast<const double*>(stages + (size_t)s * stage_bytes + TILE_BYTES) + KT + K * VS;
 #pragma unroll
       for (int k = 0; k < RPW; ++k) {
-        gI[k] = __ldg(gpad + it.vbase + (long long)it.I * KT + wg + NGW * k);
+        gI[k] = vgi[wg + NGW * k];
         racc[k] = 0.0;
       }
       if (rw) {   // beta_k u_k[row] of this warp's correction strips, fixed for the whole item
@@ -880,7 +887,7 @@ fekf_status Kf::pass_launch(bool rw, int i0, int n, int* ctr, int grid, cudaStre
     FEKF_CHECK_CUDA(cudaEventRecordWithFlags(tp->a, s, capturing ? cudaEventRecordExternal : cudaEventRecordDefault));
   }
   const int K = rw ? npend : 0;
-  const int stage_bytes = (int)(TILE_ELEMS * elem() + (KT + K * VS) * sizeof(double));
+  const int stage_bytes = (int)(TILE_ELEMS * elem() + (2 * KT + K * VS) * sizeof(double));   // + g_J, u_k[J], g_I
   int nst = (int)std::min<size_t>(MAX_STAGES, (PASS_SMEM - PASS_HDR) / stage_bytes);
   if (ng == 2) nst &= ~1;   // two consumer groups alternate stages
   const ItemD* it = items_d.as<ItemD>() + i0;
