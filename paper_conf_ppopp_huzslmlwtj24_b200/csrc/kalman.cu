@@ -425,7 +425,12 @@ kf_pass_kernel(PT* __restrict__ P, const ItemD* __restrict__ items, int n_items,
     const double* vg = reinterpret_cast<const double*>(t + TILE_ELEMS);
     const double2 gJ = *reinterpret_cast<const double2*>(vg + c0);
     const double* vJ = vg + KT;
-    double ca0 = 0.0, ca1 = 0.0;
+    // fp64: the column partials in 2 independent chains of RPW/2 DFMAs (early split launch 6.13 -> 6.08 ms in
+    // ncu); fp32 keeps one chain (4 chains measured 5.39 -> 5.63 ms: its 16-row tiles are register-bound)
+    constexpr int CA = sizeof(PT) == 8 ? 2 : 1;
+    double ca0v[CA], ca1v[CA];
+#pragma unroll
+    for (int q = 0; q < CA; ++q) ca0v[q] = ca1v[q] = 0.0;
     if (rw) {
       // B <- sigma (B - C) on the tensor path, a 16 x 32 (fp64) or 16 x 64 (fp32) warp tile; then the group
       // re-reads the rewritten tile (u_B = B_new g with B_new as stored) in its own element layout
@@ -440,10 +445,13 @@ kf_pass_kernel(PT* __restrict__ P, const ItemD* __restrict__ items, int n_items,
 #pragma unroll
       for (int q = 0; q < 8; ++q) {
         racc[8 * h + q] = fma(v[q].x, gJ.x, fma(v[q].y, gJ.y, racc[8 * h + q]));
-        ca0 = fma(v[q].x, gI[8 * h + q], ca0);
-        ca1 = fma(v[q].y, gI[8 * h + q], ca1);
+        ca0v[q % CA] = fma(v[q].x, gI[8 * h + q], ca0v[q % CA]);
+        ca1v[q % CA] = fma(v[q].y, gI[8 * h + q], ca1v[q % CA]);
       }
     }
+    double ca0 = ca0v[0], ca1 = ca1v[0];
+#pragma unroll
+    for (int q = 1; q < CA; ++q) { ca0 += ca0v[q]; ca1 += ca1v[q]; }
     double* cr = colg + (tcount & 1) * (NGW * KT);
     if (!diag) *reinterpret_cast<double2*>(cr + wg * KT + c0) = make_double2(ca0, ca1);
     asm volatile("bar.sync %0, %1;" ::"r"(1 + gi), "r"(GT) : "memory");
