@@ -187,7 +187,9 @@ constexpr int TILE_ELEMS = KT * KT;
 constexpr int VS = KT + 8;   // SMEM stride of the correction vectors: DMMA fragment loads at the 2-wavefront minimum
 
 // Storage element of P: fp64 (default) or fp32 (the fp32 variant, reading Z22).  A lane handles two
-// adjacent columns of a tile row; values are widened to fp64 for every product and correction.
+// adjacent columns of a tile row; fp64 storage: every product and correction in fp64; fp32 storage: the
+// deferred corrections in fp64 (elements widened, rounded back on store), the u = P g products in fp32 with
+// sums up to one lane's share of an item in fp32 and every sum beyond it in fp64 (kf_pass_kernel).
 __device__ __forceinline__ double2 ld2(const double* p) { return *reinterpret_cast<const double2*>(p); }
 __device__ __forceinline__ double2 ld2(const float* p) {
   const float2 v = *reinterpret_cast<const float2*>(p);
@@ -383,6 +385,7 @@ kf_pass_kernel(PT* __restrict__ P, const ItemD* __restrict__ items, int n_items,
   const double sig = st->sigma;
   const int c0 = 2 * lane;
   double gI[RPW], racc[RPW];
+  float gIf[RPW], raccf[RPW];   // fp32 storage: g_I rounded once per item, the item's row sums in fp32
   // correction warp tile (apply_corrections): NSC strips x NJC chunks; fp64 (8 warps): 4 strips x 2 chunks
   // (column quarter wg & 3), fp32 (4 warps per group): 2 strips x 8 chunks
   constexpr int NSC = NGW == 8 ? CORR_STRIPS : 2, NJC = 64 / (NGW * NSC);
@@ -390,7 +393,7 @@ kf_pass_kernel(PT* __restrict__ P, const ItemD* __restrict__ items, int n_items,
   static_assert(NGW * NSC * NJC == 64, "correction tiles cover the 8 x 8 chunks of a tile");
   double ai[NSC][KMAX / 4];
 #pragma unroll
-  for (int k = 0; k < RPW; ++k) { gI[k] = 0.0; racc[k] = 0.0; }
+  for (int k = 0; k < RPW; ++k) { gI[k] = 0.0; gIf[k] = 0.f; racc[k] = 0.0; raccf[k] = 0.f; }
   int s = gi, prev_s = -1;
   uint32_t ph = 0;
   uint32_t tcount = 0;
@@ -407,7 +410,9 @@ kf_pass_kernel(PT* __restrict__ P, const ItemD* __restrict__ items, int n_items,
 #pragma unroll
       for (int k = 0; k < RPW; ++k) {
         gI[k] = vgi[wg + NGW * k];
+        if constexpr (sizeof(PT) == 4) gIf[k] = __double2float_rn(gI[k]);
         racc[k] = 0.0;
+        raccf[k] = 0.f;
       }
       if (rw) {   // beta_k u_k[row] of this warp's correction strips, fixed for the whole item
         const int fr = lane >> 2, fk = lane & 3;
@@ -437,16 +442,40 @@ kf_pass_kernel(PT* __restrict__ P, const ItemD* __restrict__ items, int n_items,
       apply_corrections<PT, NSC, NJC>(t, ai, vJ, K, sig, cstrip0, cj0, lane);
       asm volatile("bar.sync %0, %1;" ::"r"(1 + gi), "r"(GT) : "memory");
     }
+    if constexpr (sizeof(PT) == 4) {
+      // fp32 storage: the products in fp32 (the stored element is fp32 already; g_I, g_J rounded to fp32); a
+      // lane's row sums over the item's tiles (<= 64 products) and a column's RPW products per tile summed in
+      // fp32, every sum across lanes, warps, items and blocks in fp64.  Widening each element to fp64 first (2 F2F + 2 DFMA per element) made the fp32
+      // pass's consumers the bound of its early split launch (48 GB/s per SM).
+      const float gJx = (float)gJ.x, gJy = (float)gJ.y;
+      float cf0 = 0.f, cf1 = 0.f;
 #pragma unroll
-    for (int h = 0; h < RPW / 8; ++h) {
-      double2 v[8];
+      for (int h = 0; h < RPW / 8; ++h) {
+        float2 v[8];
 #pragma unroll
-      for (int q = 0; q < 8; ++q) v[q] = ld2(t + (wg + NGW * (8 * h + q)) * KT + c0);
+        for (int q = 0; q < 8; ++q)
+          v[q] = *reinterpret_cast<const float2*>(t + (wg + NGW * (8 * h + q)) * KT + c0);
 #pragma unroll
-      for (int q = 0; q < 8; ++q) {
-        racc[8 * h + q] = fma(v[q].x, gJ.x, fma(v[q].y, gJ.y, racc[8 * h + q]));
-        ca0v[q % CA] = fma(v[q].x, gI[8 * h + q], ca0v[q % CA]);
-        ca1v[q % CA] = fma(v[q].y, gI[8 * h + q], ca1v[q % CA]);
+        for (int q = 0; q < 8; ++q) {
+          raccf[8 * h + q] = fmaf(v[q].x, gJx, fmaf(v[q].y, gJy, raccf[8 * h + q]));
+          cf0 = fmaf(v[q].x, gIf[8 * h + q], cf0);
+          cf1 = fmaf(v[q].y, gIf[8 * h + q], cf1);
+        }
+      }
+      ca0v[0] = cf0;
+      ca1v[0] = cf1;
+    } else {
+#pragma unroll
+      for (int h = 0; h < RPW / 8; ++h) {
+        double2 v[8];
+#pragma unroll
+        for (int q = 0; q < 8; ++q) v[q] = ld2(t + (wg + NGW * (8 * h + q)) * KT + c0);
+#pragma unroll
+        for (int q = 0; q < 8; ++q) {
+          racc[8 * h + q] = fma(v[q].x, gJ.x, fma(v[q].y, gJ.y, racc[8 * h + q]));
+          ca0v[q % CA] = fma(v[q].x, gI[8 * h + q], ca0v[q % CA]);
+          ca1v[q % CA] = fma(v[q].y, gI[8 * h + q], ca1v[q % CA]);
+        }
       }
     }
     double ca0 = ca0v[0], ca1 = ca1v[0];
@@ -479,7 +508,7 @@ kf_pass_kernel(PT* __restrict__ P, const ItemD* __restrict__ items, int n_items,
       double* rs = ws + ((size_t)it.row_slot * NG + gi) * KT;
 #pragma unroll
       for (int q = 0; q < RPW; ++q) {
-        double v = racc[q];
+        double v = sizeof(PT) == 4 ? (double)raccf[q] : racc[q];
 #pragma unroll
         for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
         if (lane == 0) rs[wg + NGW * q] = v;
