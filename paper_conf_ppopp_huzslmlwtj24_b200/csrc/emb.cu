@@ -617,10 +617,10 @@ __device__ __forceinline__ void seed_rows(real* sm, const EmbBwdIO& io, int r0, 
 template <class W>
 __global__ void __launch_bounds__(EMB_BWD_WARPS * 32, 1) emb_bwd_kernel(const real* __restrict__ wp, EmbBwdIO io) {
   extern __shared__ __align__(16) real sm[];
-  constexpr int T = W::T, NW = EMB_BWD_WARPS, NL = W::NL, RPW = T / NW;
+  constexpr int T = W::T, NL = W::NL;
   __shared__ int s_slot[T], s_prow[T], s_tpos[T];
   __shared__ real s_dr[T * 4];
-  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+  const int tid = threadIdx.x;
   const bool tan = io.tidx != nullptr;
   const bool wantw = io.ws != nullptr;
   const int R = min(io.Rmax, *io.Rdev);

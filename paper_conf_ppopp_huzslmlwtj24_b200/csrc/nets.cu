@@ -1566,6 +1566,7 @@ static fekf_status pairs_concurrent(Ctx& c, int nb, cudaStream_t s, Fn fn) {
 
 // fp32 nets: fp32 copies of the fp64 inputs (R~, its Jacobian, d: once per geometry; the weights: before
 // every primal forward, i.e. after every Kalman update)
+#ifdef FEKF_NETS32
 __global__ void to_real_kernel(const double* __restrict__ src, real* __restrict__ dst, long long n) {
   const long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x;
   if (i < n) dst[i] = (real)src[i];
@@ -1577,6 +1578,7 @@ static fekf_status to_real(const DBuf& src, const DBuf& dst, long long n, cudaSt
   count_launch();
   return FEKF_OK;
 }
+#endif
 
 fekf_status prepare_geometry(Ctx& c, int nb, cudaStream_t s) {
 #ifdef FEKF_NETS32
