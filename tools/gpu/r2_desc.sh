@@ -1,0 +1,6 @@
+python -m paper_conf_ppopp_huzslmlwtj24_b200.build > /dev/null
+timeout 1500 python -m pytest tests -q -m gpu -x -rf -p no:cacheprovider 2>&1 | tail -4
+timeout 300 python bench.py --steps 10 --warmup 3 --no-e2e --no-cpu-baseline > gpurun_out/bdesc.json 2>/dev/null
+echo "desc stream: $(python tools/bench_brief.py gpurun_out/bdesc.json | head -2 | tr '\n' ' ') $(grep -o '"sm_mhz": [0-9.]*' gpurun_out/bdesc.json)"
+timeout 300 python tools/prof_step.py > gpurun_out/prof_desc.txt 2>/dev/null
+grep "desc_fwd\|wall" gpurun_out/prof_desc.txt
