@@ -84,3 +84,14 @@ def test_opt_defaults_follow_the_paper():
     assert big["lambda0"] == lam["lambda0_large"] and big["nu"] == lam["nu_large"]
     with pytest.raises(fk.FekfError):
         fk.opt_defaults(0)
+
+
+def test_net_precision_knob():
+    """fekf_opt_cfg.net_precision (reading Z22): fekf_opt_defaults sets 0 (follow `precision`); the binding
+    accepts 0 / 32 / 64 and rejects anything else before any C call."""
+    d = fk.opt_defaults(32)
+    assert d["precision"] == 64 and d["net_precision"] == 0
+    for v in (0, 32, 64):
+        assert fk.opt_cfg({**d, "net_precision": v}).net_precision == v
+    with pytest.raises(ValueError):
+        fk.opt_cfg({**d, "net_precision": 16})
