@@ -471,7 +471,13 @@ def run_fekf(args, rank, world, local):
                 "share_of_step_if_serial": nets_ms / (ms / args.steps), **work}
     except Exception as e:   # instrumentation only: never lose the bench line over it
         nets = {"error": str(e)[:200]}
-    split_sms = int(os.environ.get("FEKF_SPLIT_SMS", "96" if args.precision == 64 else "80")) if world == 1 else 0
+    split_sms = int(os.environ.get("FEKF_SPLIT_SMS", "96" if args.precision == 64 else "80"))
+    f_local = info["tiles_local"] / total_tiles
+    if "FEKF_SPLIT_SMS" not in os.environ and f_local < 0.999 and split_sms > 0:
+        # the library's rule for a rank streaming a fraction f of a sharded P (api.cu, Ctx::init)
+        nsm = torch.cuda.get_device_properties(local).multi_processor_count
+        s1 = min(split_sms, nsm - 1)
+        split_sms = max(8, round(nsm * f_local / (f_local + (nsm - s1) / s1)))
     roof = {"kernel": "kf_pass_kernel", "bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
             "frac": (achieved / peak) if achieved else None, "traffic": traffic,
             "peak_source": peak_kind, "alg_bytes_per_launch": alg_bytes, "avg_launch_ms": avg_pass_s * 1000.0,

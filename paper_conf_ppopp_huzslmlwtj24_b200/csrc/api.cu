@@ -323,6 +323,21 @@ fekf_status Ctx::init(const fekf_model_cfg& mm, const fekf_opt_cfg& oo, int nato
     kf->split_sms = e ? atoi(e) : (o.precision == 32 ? 80 : 96);   // measured defaults
   }
   FEKF_TRY(kf->create(blocks, o, comm));
+  if (kf->split_sms > 0 && !getenv("FEKF_SPLIT_SMS") && kf->plan.total_tiles > 0) {
+    // P sharded over the ranks (p_mode 0, world > 1): this rank streams a fraction f of P while its reverse
+    // pass does the work of N = 1 (weak scaling: B images per rank), so the early pass needs fewer SMs.  With
+    // S1 of the Ns SMs balancing the pass against the reverse pass at f = 1 (the measured defaults above),
+    // pass time ~ f / S and reverse time ~ 1 / (Ns - S) balance at S(f) = Ns f / (f + (Ns - S1) / S1):
+    // 96 -> 71 / 46 / 28 early SMs at 2 / 4 / 8 ranks (fp64).  Not measured on real multi-GPU runs.
+    const double f = (double)kf->plan.tiles_local / (double)kf->plan.total_tiles;
+    if (f < 0.999) {
+      int cdev = 0, nsm = 148;
+      FEKF_CHECK_CUDA(cudaGetDevice(&cdev));
+      FEKF_CHECK_CUDA(cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, cdev));
+      const double S1 = std::min<double>(kf->split_sms, nsm - 1), r = (nsm - S1) / S1;
+      kf->split_sms = std::max(8, (int)std::lround(nsm * f / (f + r)));
+    }
+  }
   if (kf->split_sms > 0) FEKF_CHECK_CUDA(cudaEventCreateWithFlags(&ev_fit, cudaEventDisableTiming));
   int dev = 0;
   FEKF_CHECK_CUDA(cudaGetDevice(&dev));
