@@ -10,6 +10,7 @@
 // k-contiguous with a 20-element row stride (conflict-free fragment loads), 3-stage cp.async ring.
 #pragma once
 #include <algorithm>
+#include <cstdlib>
 
 #include "model.cuh"
 #include "mathx.cuh"
@@ -585,7 +586,11 @@ static fekf_status gemm_group(GemmProb<Epi>* probs, int n, cudaStream_t s) {
   // tile lost to 64 x 64 there, 62 vs 49 us); 128 x 64 tiles with 16 warps measured slower on the generic path
   if (!TA && nmax % 80 == 0 && nmax <= 320 && rows >= 2048)
     return gemm_launch<128, 80, 16, 40, TA, TB, Epi, 16>(G, s);
-  if (rows < 65536) return gemm_launch<64, 64, 32, 16, TA, TB>(G, s);
+  static const long long big_rows = [] {   // experiment knob: rows from which the generic path takes 128 x 64
+    const char* v = getenv("FEKF_GEMM_BIG_ROWS");
+    return v ? atoll(v) : 65536LL;
+  }();
+  if (rows < big_rows) return gemm_launch<64, 64, 32, 16, TA, TB>(G, s);
   return gemm_launch<128, 64, 32, 32, TA, TB>(G, s);
 }
 
