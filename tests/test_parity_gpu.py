@@ -336,19 +336,27 @@ def test_step_graph_matches_eager():
     assert torch.equal(out[0][2], out[1][2])
 
 
-def test_step_bit_reproducible():
-    """Two runs of the bench's model class (c1_cu32 with the split pass: N_b 1024) give bit-identical
-    weights, P, forces and metrics: no floating-point atomics anywhere in the step."""
-    wl = get_config("c1_cu32")
+@pytest.mark.parametrize("name,precision", [("c1_cu32", 64), ("t2_tiny", 64), ("t2_tiny", 32)])
+def test_step_bit_reproducible(name, precision):
+    """Two runs of the bench's model class (with the split pass: N_b 1024) give bit-identical weights, P,
+    forces and metrics: no floating-point atomics anywhere in the step.  The second run launches the type
+    pairs' embedding kernels one after another instead of side by side (FEKF_PAIR_STREAMS=0; the 2-type
+    model has 4 pairs): concurrency changes no result either.  Both precisions."""
+    wl = get_config(name)
     m = wl.model
-    opt = type(wl.opt)(**{**wl.opt.__dict__, "block_size": 1024, "p_defer": 3})
+    opt = type(wl.opt)(**{**wl.opt.__dict__, "block_size": 1024, "p_defer": 3, "precision": precision})
     B = wl.batch
-    ds = make_dataset("c1_cu32", B)
+    ds = make_dataset(name, B)
     na = len(ds["types"])
     w0 = init_weights(m, 3, float(ds["energy"].mean() / na))
     out = []
-    for _ in range(2):
-        ctx = fk.Context(m, opt, types=ds["types"], local_batch=B, global_batch=B)
+    for run in range(2):
+        if run == 1:
+            os.environ["FEKF_PAIR_STREAMS"] = "0"
+        try:
+            ctx = fk.Context(m, opt, types=ds["types"], local_batch=B, global_batch=B)
+        finally:
+            os.environ.pop("FEKF_PAIR_STREAMS", None)
         ctx.set_params(cu(w0))
         mets = [ctx.train_step(cu(ds["coord"]), cu(ds["box"]), cu(ds["energy"]), cu(ds["force"]),
                                cu(force_groups(na, s, 17), torch.int32)).clone() for s in range(4)]
