@@ -33,7 +33,7 @@ METRIC = "EKF train images/sec"
 def parse():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--steps", type=int, default=16)   # 16 steps = 80 updates = 5 cycles of the read-write pass (p_defer 15)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--config", default="c2_water64")
     ap.add_argument("--impl", default="fekf", choices=["fekf", "reference"])
